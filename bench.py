@@ -1,0 +1,364 @@
+#!/usr/bin/env python
+"""bench.py -- HPCCG CG hot path on B200 (BASELINE.json metric).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+                    [--workload hpccg128|hpccg20|hpccg256|hpccg512s]
+
+One STEP = one whole HPCCG solve on the synthetic on-device-generated problem:
+init (p = x, Ap = A p, r = b - Ap, r.r) + `iters` CG iterations (SpMV with
+fused p.Ap, fused x/r update + r.r, p update; device-side scalars; CUDA-graph
+replay) + the max|x - 1| verification -- rows a.2-a.9 of DESIGN.md.  The
+problem (a.1) is generated once per run (HPCCG times only the solve); its
+time is reported as config.gen_ms.  x is reset to 0 (x0, A5) before every
+step by our waxpby kernel.
+
+value = CG GFLOP/s of the whole job = sum over ranks of niters (2 nnz + 10 n)
+        / max-over-ranks device time of the K timed steps (exact nnz, A15).
+e2e   = the same metric through the public C-ABI with HOST buffers: every
+        step copies x0 from pinned host memory in and the solution x back out.
+roofline = the SpMV kernel (dominant), algorithmic bytes 12 nnz + 16 n per
+        launch / its CUDA-event launch duration inside the timed region.
+Multi-GPU (torchrun): z-slab weak scaling, one rank per GPU, NCCL halo +
+        allreduce inside the library; torch.distributed only bootstraps.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "HPCCG CG GFLOP/s and SpMV HBM GB/s (fp64) at 1/2/4/8 B200 vs HBM roofline"
+WORKLOADS = {
+    # name: (nx, ny, nz per GPU, CG iterations, BASELINE config index)
+    "hpccg128": (128, 128, 128, 500, 1),
+    "hpccg20": (20, 30, 10, 149, 0),
+    "hpccg256": (256, 256, 256, 200, 2),
+    "hpccg512s": (512, 512, 512, 200, 3),
+}
+FALLBACK_HBM_GBS = 6650.0  # B200_PROFILING.md fallback, used only without MEASURED_PEAKS.json
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    return FALLBACK_HBM_GBS, "fallback (B200_PROFILING.md)"
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled during the timed region."""
+    Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap,utilization.gpu")
+
+    def __init__(self, index: int):
+        self.index, self.proc, self.lines = index, None, []
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index), "--query-gpu=" + self.Q,
+                 "--format=csv,noheader,nounits", "-lms", "100"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def __exit__(self, *a):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        sm, mx, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            f = [x.strip() for x in ln.split(",")]
+            if len(f) < 8:
+                continue
+            try:
+                s, m, util = float(f[0]), float(f[1]), float(f[7])
+            except ValueError:
+                continue
+            mx = m
+            if util > 0:
+                sm.append(s)
+                for nm, v in zip(names, f[3:7]):
+                    if v.lower().startswith("active"):
+                        reasons.add(nm)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": mx,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def cg_flops(niters, nnz, n):
+    return float(niters) * (2.0 * nnz + 10.0 * n)
+
+
+# ------------------------------------------------------------ oracle (CPU)
+
+def oracle_sample(nx, ny, nz, iters_cap, budget_s):
+    """Time the CPU oracle (as it stands) on a bounded sample of the
+    workload: the same generated problem, m CG iterations, all host cores."""
+    import oracle
+    t0 = time.perf_counter()
+    prob = oracle.generate(nx, ny, nz)
+    gen_s = time.perf_counter() - t0
+    r1 = oracle.cg(prob, 2, 0.0)           # calibrate: 1 iteration
+    per_it = max(r1["times"][0], 1e-6)
+    m = int(max(1, min(iters_cap, budget_s / per_it)))
+    r = oracle.cg(prob, m + 1, 0.0)
+    t = r["times"][0]
+    gflops = cg_flops(r["niters"], prob.nnz, prob.n) / t * 1e-9
+    return {"value": gflops, "iters": r["niters"], "seconds": t, "gen_s": gen_s,
+            "cores": oracle.get_threads(), "prob": prob}
+
+
+def run_reference(args, nx, ny, nz, iters, cfg_index):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return 0
+    import oracle
+    oracle.build()
+    prob = oracle.generate(nx, ny, nz)
+    m = max(1, min(iters, args.ref_iters))
+    for _ in range(args.warmup):
+        oracle.cg(prob, m + 1, 0.0)
+    tot, flops = 0.0, 0.0
+    for _ in range(args.steps):
+        r = oracle.cg(prob, m + 1, 0.0)
+        tot += r["times"][0]
+        flops += cg_flops(r["niters"], prob.nnz, prob.n)
+    val = flops / tot * 1e-9
+    sample = (f"oracle CG on the {nx}x{ny}x{nz} problem, {m} iterations per step "
+              f"(bounded sample of the {iters}-iteration workload), OpenMP all host cores")
+    line = {
+        "metric": METRIC, "value": round(val, 4), "unit": "GFLOP/s", "impl": "reference",
+        "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": round(tot / args.steps * 1e3, 3), "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+        "data": "synthetic (HPCCG generation, deterministic)",
+        "config": {"workload": args.workload, "baseline_config": cfg_index, "nx": nx, "ny": ny,
+                   "nz": nz, "iters_per_step": m},
+        "cpu_baseline": {"value": round(val, 4), "unit": "GFLOP/s", "cores": oracle.get_threads(),
+                         "kind": "oracle", "sample": sample},
+        "e2e": {"value": round(val, 4), "unit": "GFLOP/s", "h2d_bytes_per_step": 0,
+                "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+# -------------------------------------------------------------------- ours
+
+def run_ours(args, nx, ny, nz, iters, cfg_index):
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_sc_valero_laragmtv24_b200 import hpccg as H
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world != args.gpus:
+        raise SystemExit(f"--gpus {args.gpus} but WORLD_SIZE={world}")
+    if not torch.cuda.is_available():
+        raise SystemExit("bench.py needs a CUDA device (no CPU fallback)")
+    torch.cuda.set_device(local)
+    uid = None
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        obj = [H.hpccg_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(obj, src=0)
+        uid = obj[0]
+
+    stream = torch.cuda.Stream()
+    ctx = H.Context(local, stream=stream.cuda_stream, rank=rank, nranks=world, unique_id=uid)
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    prob = H.Problem(ctx, nx, ny, nz)
+    e1.record(stream)
+    torch.cuda.synchronize()
+    gen_ms = e0.elapsed_time(e1)
+    n, nnz_local = prob.n, prob.info["nnz_local"]
+    nnz_global = prob.info["nnz_global"]
+    prob.set_option(H.HPCCG_OPT_GRAPH, 1)
+    prob.set_option(H.HPCCG_OPT_TIMING, 1 if args.phase_timing else 0)
+    xptr = prob.vec_ptr(H.HPCCG_VEC_X)
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    def step():
+        ctx.waxpby(n, 0.0, xptr, 0.0, xptr, xptr)        # x0 = 0 (A5)
+        r = prob.solve(iters + 1, 0.0)                     # `iters` iterations (A4)
+        err = prob.maxabsdiff()
+        return r, err
+
+    for _ in range(args.warmup):
+        step()
+    barrier()
+    spmv_ms = spmv_n = 0.0
+    niters_tot = 0
+    l0 = ctx.launch_count
+    with ClockSampler(local) as clk:
+        barrier()
+        t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        t0.record(stream)
+        for _ in range(args.steps):
+            r, err = step()
+            st = prob.stats()
+            spmv_ms += st["spmv_ms"]
+            spmv_n += st["spmv_launches"]
+            niters_tot += r["niters"]
+        t1.record(stream)
+        barrier()
+    launches = ctx.launch_count - l0
+    ms = t0.elapsed_time(t1)
+    tmax = torch.tensor([ms], dtype=torch.float64, device="cuda")
+    flops_local = torch.tensor([cg_flops(niters_tot, nnz_local, n)], dtype=torch.float64,
+                               device="cuda")
+    if world > 1:
+        dist.all_reduce(tmax, op=dist.ReduceOp.MAX)
+        dist.all_reduce(flops_local, op=dist.ReduceOp.SUM)
+    ms_max = float(tmax.item())
+    value = float(flops_local.item()) / (ms_max * 1e-3) * 1e-9
+
+    # ---- e2e: public API with host buffers (pinned) each step
+    h_x0 = torch.zeros(n, dtype=torch.float64).pin_memory()
+    h_x = torch.empty(n, dtype=torch.float64).pin_memory()
+
+    def step_e2e():
+        prob.set_vec_ptr(H.HPCCG_VEC_X, h_x0.data_ptr())   # H2D 8n
+        r = prob.solve(iters + 1, 0.0)
+        prob.get_vec_ptr(H.HPCCG_VEC_X, h_x.data_ptr())    # D2H 8n
+        err = prob.maxabsdiff()                             # D2H 8 B
+        return r, err
+
+    step_e2e()
+    barrier()
+    t0.record(stream)
+    ni_e2e = 0
+    for _ in range(args.steps):
+        r_e, _ = step_e2e()
+        ni_e2e += r_e["niters"]
+    t1.record(stream)
+    barrier()
+    te = torch.tensor([t0.elapsed_time(t1)], dtype=torch.float64, device="cuda")
+    fe = torch.tensor([cg_flops(ni_e2e, nnz_local, n)], dtype=torch.float64, device="cuda")
+    if world > 1:
+        dist.all_reduce(te, op=dist.ReduceOp.MAX)
+        dist.all_reduce(fe, op=dist.ReduceOp.SUM)
+    e2e_value = float(fe.item()) / (float(te.item()) * 1e-3) * 1e-9
+    x_host_err = float(np.max(np.abs(h_x.numpy() - 1.0)))
+
+    if rank == 0:
+        peak, peak_src = peaks()
+        spmv_bytes = 12.0 * nnz_local + 16.0 * n
+        roof = None
+        if spmv_n > 0 and spmv_ms > 0:
+            avg_ms = spmv_ms / spmv_n
+            ach = spmv_bytes / (avg_ms * 1e-3) * 1e-9
+            roof = {"bound": "hbm", "kernel": "spmv27_kernel<true>", "achieved": round(ach, 1),
+                    "peak": peak, "unit": "GB/s", "frac": round(ach / peak, 4),
+                    "frac_of_8TBs_nominal": round(ach / 8000.0, 4),
+                    "traffic": traffic_from_profiles(args.workload),
+                    "algorithmic_bytes_per_launch": spmv_bytes, "avg_launch_us": round(avg_ms * 1e3, 2),
+                    "peak_source": peak_src,
+                    "spmv_share_of_step": round(spmv_ms / ms, 4) if ms > 0 else None}
+        cpu = None
+        if world == 1 and not args.no_cpu_baseline:
+            cs = oracle_sample(nx, ny, nz, iters, args.cpu_budget)
+            cpu = {"value": round(cs["value"], 4), "unit": "GFLOP/s", "cores": cs["cores"],
+                   "kind": "oracle",
+                   "sample": f"oracle CG (C, OpenMP) on the same {nx}x{ny}x{nz} problem, "
+                             f"{cs['iters']} iterations ({cs['seconds']:.1f} s) of the "
+                             f"{iters}-iteration step"}
+        t_iter_us = ms_max * 1e3 / max(niters_tot, 1)
+        line = {
+            "metric": METRIC, "value": round(value, 3), "unit": "GFLOP/s", "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms_max / args.steps, 4),
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+            "data": "synthetic (HPCCG 27-point problem generated on device, b = A.1)",
+            "config": {"workload": args.workload, "baseline_config": cfg_index,
+                       "nx": nx, "ny": ny, "nz_per_gpu": nz, "iters": iters,
+                       "global_rows": n * world, "global_nnz": nnz_global,
+                       "parallelism": f"zslab{world}", "graph": not args.phase_timing,
+                       "phase_timing_events": bool(args.phase_timing),
+                       "l2": "inputs larger than L2 (ELL %.0f MB/GPU > 126 MB)" % (324e-6 * n),
+                       "gen_ms": round(gen_ms, 3)},
+            "t_iter_us": round(t_iter_us, 3),
+            "niters_per_step": niters_tot // args.steps,
+            "max_abs_x_minus_1": err, "normr": r["normr"],
+            "gpu_launches": launches,
+            "clocks": clk.summary(),
+            "e2e": {"value": round(e2e_value, 3), "unit": "GFLOP/s", "h2d_bytes_per_step": 8 * n,
+                    "d2h_bytes_per_step": 8 * n + 8, "max_abs_x_minus_1_host": x_host_err},
+            "roofline": roof,
+            "cpu_baseline": cpu,
+        }
+        print(json.dumps(line), flush=True)
+    prob.free()
+    ctx.close()
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+def traffic_from_profiles(workload):
+    """dram bytes per SpMV launch from the committed ncu --set full summary."""
+    p = os.path.join(ROOT, "profiles", "spmv_traffic.json")
+    if not os.path.exists(p):
+        return None
+    try:
+        return json.load(open(p)).get(workload, {}).get("dram_bytes_per_launch")
+    except Exception:
+        return None
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
+    ap.add_argument("--workload", choices=sorted(WORKLOADS), default="hpccg128")
+    ap.add_argument("--iters", type=int, default=None, help="override CG iterations per step")
+    ap.add_argument("--phase-timing", type=int, default=1,
+                    help="1: CUDA events around every phase (roofline from the timed region)")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-budget", type=float, default=12.0, help="seconds of oracle CG")
+    ap.add_argument("--ref-iters", type=int, default=5, help="oracle iterations per reference step")
+    args = ap.parse_args()
+    if args.warmup < 3:
+        raise SystemExit("--warmup must be >= 3")
+    nx, ny, nz, iters, cfg = WORKLOADS[args.workload]
+    if args.iters:
+        iters = args.iters
+    if args.impl == "reference":
+        return run_reference(args, nx, ny, nz, iters, cfg)
+    return run_ours(args, nx, ny, nz, iters, cfg)
+
+
+if __name__ == "__main__":
+    sys.exit(main())

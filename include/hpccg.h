@@ -1,0 +1,222 @@
+/*
+ * hpccg.h -- C ABI of the B200-native HPCCG conjugate-gradient hot path.
+ *
+ * The library (libhpccg.so, built from paper_conf_sc_valero_laragmtv24_b200/
+ * csrc/) runs every step of the path in hand-written sm_100a CUDA kernels:
+ * on-device problem generation, the 27-point SpMV, the ddot reductions and
+ * the waxpby updates, with the dots fused into the updates, and a z-slab
+ * ("chimney") decomposition across GPUs with NCCL halo-plane exchange and one
+ * scalar allreduce per dot (BASELINE.json north_star).
+ *
+ * Citations: "P:Lnnn" = line of the paper text (Valero-Lara et al., "JACC",
+ * SC'24 workshops, PAPER.md); "north_star" = BASELINE.json; "A<k>" = reading
+ * k in DESIGN.md (sec. Readings).  HPCCG = the Mantevo HPCCG 1.0 benchmark the
+ * paper names (P:L7), whose call signatures
+ * generate_matrix / HPC_sparsemv / ddot / waxpby / HPCCG this ABI follows.
+ *
+ * Conventions (all functions):
+ *  - Return HPCCG_OK (0) or a negative HPCCG_E* code; never abort or throw.
+ *    hpccg_strerror(code) names the code, hpccg_last_error() gives the
+ *    detail message of the calling thread's last failure.
+ *  - Every call is host-synchronous on return: device work it enqueued has
+ *    completed (JACC's constructs are synchronous).
+ *  - SPMD: with nranks > 1 every rank calls every function collectively, in
+ *    the same order, like HPCCG-MPI.
+ *  - "device" pointers are CUDA device pointers on the context's device
+ *    (e.g. torch.empty(..., device='cuda').data_ptr()); the caller owns them.
+ *    Objects returned through ** out-parameters are library-owned until the
+ *    matching hpccg_free / hpccg_finalize.
+ *  - fp64 everywhere ("All computations are double-precision").
+ *  - Loopback contexts (hpccg_init_loopback) host all nranks slabs in ONE
+ *    process on ONE device, for testing the decomposition without NCCL.  In
+ *    that mode every "local vector" argument is the concatenation, in rank
+ *    order, of the nranks per-rank local vectors, and every length n is the
+ *    per-rank length.
+ *  - One context per host thread (thread-compatible, not thread-safe).
+ */
+#ifndef HPCCG_H
+#define HPCCG_H
+
+#include <stdint.h>
+
+#if defined(__GNUC__)
+#define HPCCG_API __attribute__((visibility("default")))
+#else
+#define HPCCG_API
+#endif
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define HPCCG_OK 0
+#define HPCCG_EINVAL (-1)   /* bad argument (sizes < 1, n > local length, NULL) */
+#define HPCCG_ENOMEM (-2)   /* device or host allocation failed */
+#define HPCCG_ECUDA (-3)    /* a CUDA runtime call or kernel launch failed */
+#define HPCCG_ENCCL (-4)    /* an NCCL call failed (comm aborted) */
+#define HPCCG_ENOTSUP (-5)  /* not available in this build / configuration */
+
+#define HPCCG_UNIQUE_ID_BYTES 128
+
+/* which vector hpccg_vec / hpccg_set_vec / hpccg_get_vec address */
+#define HPCCG_VEC_X 0       /* iterate / initial guess, nrow_local */
+#define HPCCG_VEC_B 1       /* right-hand side b = A.1, nrow_local */
+#define HPCCG_VEC_XEXACT 2  /* exact solution (all ones), nrow_local */
+
+/* hpccg_set_option keys */
+#define HPCCG_OPT_GRAPH 0   /* 1 (default): replay each CG iteration as a CUDA graph */
+#define HPCCG_OPT_POLL 1    /* iterations between host polls of the device stop flag
+                               when tol > 0 (default 8); 0 = never poll */
+#define HPCCG_OPT_TIMING 2  /* 1: CUDA-event time every phase of every iteration into
+                               hpccg_get_stats / times[] (disables the graph); default 0 */
+
+typedef struct hpccg_ctx hpccg_ctx;         /* device, streams, comm (rank, nranks) */
+typedef struct hpccg_problem hpccg_problem; /* A (ELL-27), b, x, x_exact, CG work vectors */
+
+/* Per-solve statistics (filled by hpccg_solve, read with hpccg_get_stats). Times are
+ * milliseconds of device time measured with CUDA events on the stream each phase
+ * runs on; they are filled only with HPCCG_OPT_TIMING = 1 (else 0). */
+typedef struct hpccg_stats {
+    double total_ms;        /* whole solve (events around it; always filled) */
+    double spmv_ms;         /* sum over SpMV launches (incl. the fused p.Ap) */
+    double update_ms;       /* sum over fused x/r update + r.r launches */
+    double pupdate_ms;      /* sum over p = r + beta p launches */
+    double allreduce_ms;    /* sum over scalar allreduces (0 at nranks = 1) */
+    double exchange_ms;     /* sum over halo exchanges (0 at nranks = 1) */
+    int64_t spmv_launches;  /* SpMV passes (= niters + 1) */
+    int64_t iterations;     /* niters */
+    int64_t kernel_launches;/* kernels this library enqueued during the solve */
+} hpccg_stats;
+
+HPCCG_API const char *hpccg_strerror(int code);
+HPCCG_API const char *hpccg_last_error(void);
+HPCCG_API const char *hpccg_version(void);
+
+/* Number of kernels this library has enqueued on `ctx` since hpccg_init
+ * (graph replays count every kernel node).  Used for bench gpu_launches. */
+HPCCG_API int hpccg_launch_count(const hpccg_ctx *ctx, int64_t *count);
+
+/* ---------------------------------------------------------------- context */
+
+/* Fill `out` (HPCCG_UNIQUE_ID_BYTES bytes, host) with an NCCL unique id.
+ * Call on rank 0 only, then broadcast the bytes (e.g. torch.distributed).
+ * HPCCG_ENOTSUP if the library was built without NCCL. */
+HPCCG_API int hpccg_unique_id(void *out);
+
+/* Create a context on CUDA `device`.  `cuda_stream` (cudaStream_t, nullable)
+ * is the stream all work is enqueued on; NULL = a library-created stream.
+ * nranks == 1: single GPU, `unique_id` must be NULL.  nranks > 1: z-slab rank
+ * `rank` of `nranks` over NCCL; `unique_id` = the bytes from hpccg_unique_id
+ * on rank 0 (north_star "z-slab decomposition ... NCCL").  Collective. */
+HPCCG_API int hpccg_init(hpccg_ctx **ctx, int device, void *cuda_stream, int rank,
+               int nranks, const void *unique_id);
+
+/* Create a loopback context: all `nranks` z-slabs in this process on `device`;
+ * halo exchange = device-to-device plane copies, allreduce = fixed-rank-order
+ * sum kernel.  Same kernels and decomposition as the NCCL path. */
+HPCCG_API int hpccg_init_loopback(hpccg_ctx **ctx, int device, void *cuda_stream,
+                        int nranks);
+
+/* rank / nranks of the context; nslabs = slabs hosted by this process
+ * (1, or nranks for loopback). */
+HPCCG_API int hpccg_ctx_info(const hpccg_ctx *ctx, int *rank, int *nranks, int *nslabs);
+
+HPCCG_API void hpccg_finalize(hpccg_ctx *ctx);
+
+/* ---------------------------------------------------------------- problem */
+
+/* a.1 -- generate this rank's slab of the HPCCG problem ON THE DEVICE
+ * (HPCCG generate_matrix; north_star "on-device problem generation").
+ * Global grid nx x ny x (nz * nranks); rank r owns z-planes [r nz, (r+1) nz),
+ * i.e. global rows [r n, (r+1) n), n = nx ny nz, row id = z*ny*nx + y*nx + x.
+ * Row i holds, for sz, sy, sx in {-1,0,1} (that nesting = ascending column),
+ * the entry -1.0 (27.0 on the diagonal) iff the neighbour lies in the global
+ * grid (truncated stencil, A6); b_i = 28 - nnz_i (so A.1 = b, x_exact = 1),
+ * x = 0 (A5).  Storage: ELL-27 slot-major.
+ * Errors: HPCCG_EINVAL if nx, ny or nz < 1 or the local row count or the
+ * local-with-halo column count exceeds 2^31 - 1; HPCCG_ENOMEM. Collective. */
+HPCCG_API int hpccg_generate(hpccg_ctx *ctx, int nx, int ny, int nz, hpccg_problem **out);
+
+/* Sizes: nrow_local = n; ncol_local = n + 2 nx ny (the local-with-halo x
+ * length: [lower halo plane | n owned | upper halo plane]); nnz_local = stored
+ * entries of the slab(s) this process hosts; nrow_global / nnz_global over all
+ * ranks.  Any out-pointer may be NULL. */
+HPCCG_API int hpccg_info(const hpccg_problem *prob, int64_t *nrow_local,
+               int64_t *ncol_local, int64_t *nnz_local, int64_t *nrow_global,
+               int64_t *nnz_global);
+
+/* Borrowed device pointer to X, B or XEXACT (nrow_local doubles per slab,
+ * slabs concatenated in loopback mode).  Valid until hpccg_free. */
+HPCCG_API int hpccg_vec(hpccg_problem *prob, int which, double **dev_ptr);
+
+/* Copy a problem vector from / to HOST memory (nrow_local doubles per slab).
+ * Pinned host memory gives full PCIe bandwidth; pageable works. */
+HPCCG_API int hpccg_set_vec(hpccg_problem *prob, int which, const double *host_src);
+HPCCG_API int hpccg_get_vec(const hpccg_problem *prob, int which, double *host_dst);
+
+/* Copy slab `slab`'s ELL-27 matrix to HOST memory: val_host[27 * nrow_local]
+ * and col_host[27 * nrow_local], slot-major (entry (s, i) at s*nrow_local+i),
+ * columns as local-with-halo indices (global - (rank n - nx ny)); padding
+ * slots hold val 0.0, col = the row's own local-with-halo index.  For tests. */
+HPCCG_API int hpccg_copy_matrix(const hpccg_problem *prob, int slab, double *val_host,
+                      int32_t *col_host);
+
+HPCCG_API int hpccg_set_option(hpccg_problem *prob, int key, int64_t value);
+
+/* ------------------------------------------------------------- operations */
+
+/* a.2 + a.3 -- y = A x (HPCCG HPC_sparsemv; the paper's analogue is the
+ * matvecmul of Fig. 12).  x: device, ncol_local doubles in the
+ * local-with-halo layout; its two halo planes are OVERWRITTEN by the halo
+ * exchange this call performs (zero-filled at the global z boundary).
+ * y: device, nrow_local doubles; must not overlap x.  Per row, the stored
+ * entries are reduced in ascending column order as an fp64 FMA chain from
+ * +0.0 (A8), so the result is bitwise reproducible. */
+HPCCG_API int hpccg_spmv(hpccg_problem *prob, double *x, double *y);
+
+/* a.4/a.10 -- *result (HOST) = sum_i x_i y_i over all ranks (JACC DOT: Fig. 2
+ * P:L67-L69; HPCCG ddot + MPI_Allreduce).  x, y: device, n doubles
+ * each (x == y allowed).  Local sum: deterministic fixed-shape tree; then a
+ * sum-allreduce in fixed rank order (loopback) or via NCCL.  n >= 0. */
+HPCCG_API int hpccg_ddot(hpccg_ctx *ctx, int64_t n, const double *x, const double *y,
+               double *result);
+
+/* a.5/a.6/a.10 -- w = alpha x + beta y (HPCCG waxpby; JACC AXPY x += alpha y
+ * of Fig. 2 P:L64-L66 is hpccg_waxpby(n, 1, x, alpha, y, x)).  Device arrays
+ * of n doubles; w may alias x or y.  Canonical single-FMA forms (A10):
+ * alpha == 1 -> fma(beta, y, x); beta == 1 -> fma(alpha, x, y); otherwise
+ * fma(alpha, x, beta * y).  Purely local (no communication). */
+HPCCG_API int hpccg_waxpby(hpccg_ctx *ctx, int64_t n, double alpha, const double *x,
+                 double beta, const double *y, double *w);
+
+/* a.2-a.8 -- HPCCG's unpreconditioned CG (the paper's loop Fig. 12
+ * P:L450-L474; loop semantics A3/A4):
+ *   p = x; Ap = A p; r = b - Ap; rtrans = r.r; normr = sqrt(rtrans)
+ *   for (k = 1; k < max_iter && normr > tol; k++):
+ *     k == 1 ? p = r : { beta = (r.r) / rtrans_old; p = r + beta p }
+ *     normr = sqrt(rtrans); Ap = A p; alpha = rtrans / p.Ap;
+ *     x += alpha p; r -= alpha Ap; niters = k
+ * with guard A11 (rtrans == 0 or p.Ap == 0 -> alpha = 0, stop).  Uses the
+ * problem's b; the problem's X is the initial guess in and the iterate out.
+ * All scalars (alpha, beta, normr, stop flag) live on the device; no per-dot
+ * host round trip.  *niters, *normr: HOST out (nullable).  times (HOST,
+ * nullable, 6 entries, seconds): total, ddot, waxpby, spmv, allreduce,
+ * exchange -- phase entries need HPCCG_OPT_TIMING = 1 (ddot is fused into the
+ * waxpby/spmv kernels, so times[1] = 0).  max_iter >= 1, tol >= 0. */
+HPCCG_API int hpccg_solve(hpccg_problem *prob, int max_iter, double tol, int *niters,
+                double *normr, double times[6]);
+
+/* Statistics of the last hpccg_solve on `prob`. */
+HPCCG_API int hpccg_get_stats(const hpccg_problem *prob, hpccg_stats *out);
+
+/* a.9 -- *result (HOST) = max_i |x_i - x_exact_i| over all ranks (HPCCG
+ * compute_residual; north_star "final max|x-1|"). */
+HPCCG_API int hpccg_maxabsdiff(hpccg_problem *prob, double *result);
+
+HPCCG_API void hpccg_free(hpccg_problem *prob);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* HPCCG_H */

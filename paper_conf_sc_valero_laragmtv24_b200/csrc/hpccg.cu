@@ -1,0 +1,1055 @@
+// hpccg.cu -- C ABI (include/hpccg.h) and host orchestration of the B200
+// HPCCG CG hot path: contexts, on-device problem generation, the halo
+// exchange (NCCL or loopback), and the CG solve loop replayed as a CUDA graph
+// with every scalar kept on the device.  Design: DESIGN.md.
+#include <cuda_runtime.h>
+#include <math.h>
+#include <stdarg.h>
+#include <stdio.h>
+#include <string.h>
+
+#include <algorithm>
+#include <string>
+#include <vector>
+
+#include "hpccg.h"
+#include "kernels.cuh"
+
+#ifdef HPCCG_WITH_NCCL
+#include <nccl.h>
+#endif
+
+using namespace hpccg;
+
+namespace {
+
+thread_local std::string g_err;
+
+int fail(int code, const char *fmt, ...) {
+    char buf[512];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof buf, fmt, ap);
+    va_end(ap);
+    g_err = buf;
+    return code;
+}
+
+#define CU(call)                                                                       \
+    do {                                                                               \
+        cudaError_t e_ = (call);                                                       \
+        if (e_ != cudaSuccess)                                                         \
+            return fail(HPCCG_ECUDA, "%s failed: %s (%s:%d)", #call,                   \
+                        cudaGetErrorString(e_), __FILE__, __LINE__);                   \
+    } while (0)
+
+#define CHECK(expr)                        \
+    do {                                   \
+        int rc_ = (expr);                  \
+        if (rc_ != HPCCG_OK) return rc_;   \
+    } while (0)
+
+enum Mode { MODE_SINGLE = 0, MODE_NCCL = 1, MODE_LOOPBACK = 2 };
+enum Phase { PH_PUPDATE = 0, PH_SPMV, PH_UPDATE, PH_ALLREDUCE, PH_EXCHANGE, PH_N };
+
+int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
+
+// Grid of the streaming kernels: enough 256-thread blocks to cover n (in
+// elements per thread), capped at 8 resident blocks on each of the 148 SMs.
+int stream_grid(int64_t work) {
+    int64_t b = cdiv(std::max<int64_t>(work, 1), kBlock);
+    return (int)std::min<int64_t>(b, 148 * 8);
+}
+
+bool aligned16(const void *p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
+
+}  // namespace
+
+// ------------------------------------------------------------------ structs
+
+struct hpccg_ctx {
+    int device = 0;
+    cudaStream_t stream = nullptr;
+    bool own_stream = false;
+    cudaStream_t comm_stream = nullptr;
+    cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
+    int rank = 0, nranks = 1, nslabs = 1;
+    Mode mode = MODE_SINGLE;
+#ifdef HPCCG_WITH_NCCL
+    ncclComm_t comm = nullptr;
+#endif
+    // scratch for the API reductions (ddot / maxabsdiff): per slab loc / out
+    double *d_api = nullptr;             // [2 * nslabs]: loc[s], out[s]
+    double **d_api_src = nullptr;        // loopback allreduce tables
+    double **d_api_dst = nullptr;
+    Reduction red{};                     // partials + counter
+    int64_t red_cap = 0;
+    double *h_pinned = nullptr;          // 8 doubles, pinned
+    int64_t launches = 0;
+};
+
+struct Slab {
+    int rank = 0;
+    int64_t n = 0, plane = 0, ncol = 0;
+    unsigned long long nnz = 0;
+    double *val = nullptr;
+    int *col = nullptr;
+    double *b = nullptr, *x = nullptr, *xexact = nullptr, *r = nullptr, *Ap = nullptr;
+    double *p_alloc = nullptr, *p = nullptr;  // p: local-with-halo base (ncol)
+    CgScalars *sc = nullptr;
+    Reduction red{};
+};
+
+struct TimedOp {
+    int phase;
+    cudaEvent_t a, b;
+};
+
+struct hpccg_problem {
+    hpccg_ctx *ctx = nullptr;
+    int nx = 0, ny = 0, nz = 0;
+    std::vector<Slab> slabs;
+    unsigned long long nnz_global = 0;
+    // loopback allreduce tables (device arrays of device pointers)
+    double **d_tab = nullptr;  // [6][nslabs]: src pAp, dst pAp, src rr, dst rr, src red, dst red
+    // options
+    int opt_graph = 1, opt_poll = 8, opt_timing = 0;
+    // graph of one CG iteration
+    cudaGraphExec_t graph = nullptr;
+    int64_t graph_kernels = 0;
+    // timing
+    std::vector<cudaEvent_t> ev_pool;
+    size_t ev_used = 0;
+    std::vector<TimedOp> timed;
+    cudaEvent_t ev_t0 = nullptr, ev_t1 = nullptr;
+    int *h_done = nullptr;  // pinned poll flags [2]
+    cudaEvent_t ev_poll[2] = {nullptr, nullptr};
+    hpccg_stats stats{};
+};
+
+namespace {
+
+#ifdef HPCCG_WITH_NCCL
+int nccl_fail(hpccg_ctx *ctx, ncclResult_t r, const char *what) {
+    if (ctx->comm) {
+        ncclCommAbort(ctx->comm);
+        ctx->comm = nullptr;
+    }
+    return fail(HPCCG_ENCCL, "%s failed: %s", what, ncclGetErrorString(r));
+}
+#define NC(ctx, call)                                               \
+    do {                                                            \
+        ncclResult_t r_ = (call);                                   \
+        if (r_ != ncclSuccess) return nccl_fail((ctx), r_, #call);  \
+    } while (0)
+#endif
+
+int check_launch(hpccg_ctx *ctx, int nkernels = 1) {
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return fail(HPCCG_ECUDA, "kernel launch failed: %s", cudaGetErrorString(e));
+    ctx->launches += nkernels;
+    return HPCCG_OK;
+}
+
+// --------------------------------------------------------------- timing
+
+cudaEvent_t pool_event(hpccg_problem *p) {
+    if (p->ev_used == p->ev_pool.size()) {
+        cudaEvent_t e;
+        if (cudaEventCreate(&e) != cudaSuccess) return nullptr;
+        p->ev_pool.push_back(e);
+    }
+    return p->ev_pool[p->ev_used++];
+}
+
+struct PhaseTimer {  // records a begin/end event pair on `s` when timing is on
+    hpccg_problem *p;
+    cudaStream_t s;
+    int phase;
+    cudaEvent_t a = nullptr;
+    PhaseTimer(hpccg_problem *p_, cudaStream_t s_, int ph, bool on) : p(p_), s(s_), phase(ph) {
+        if (on) {
+            a = pool_event(p);
+            if (a) cudaEventRecord(a, s);
+        }
+    }
+    ~PhaseTimer() {
+        if (!a) return;
+        cudaEvent_t b = pool_event(p);
+        if (!b) return;
+        cudaEventRecord(b, s);
+        p->timed.push_back({phase, a, b});
+    }
+};
+
+// ------------------------------------------------------- comm primitives
+
+// Sum-allreduce (or max) of one scalar per slab: loc -> out, identical on all
+// slabs / ranks.  Single: plain device copy is unnecessary (kernels write
+// the global value directly), so this is only called for nslabs/nranks > 1.
+int allreduce_scalar(hpccg_ctx *ctx, double *const *h_src, double *const *h_dst,
+                     double *const *d_src, double *const *d_dst, bool is_max) {
+    if (ctx->mode == MODE_LOOPBACK) {
+        slab_allreduce_kernel<<<1, 32, 0, ctx->stream>>>(d_src, d_dst, ctx->nslabs, is_max);
+        return check_launch(ctx);
+    }
+#ifdef HPCCG_WITH_NCCL
+    if (ctx->mode == MODE_NCCL) {
+        NC(ctx, ncclAllReduce(h_src[0], h_dst[0], 1, ncclDouble, is_max ? ncclMax : ncclSum,
+                              ctx->comm, ctx->stream));
+        return HPCCG_OK;
+    }
+#endif
+    (void)h_src;
+    (void)h_dst;
+    return fail(HPCCG_ENOTSUP, "allreduce: no communicator");
+}
+
+// a.2 halo exchange of a local-with-halo vector per slab (bases xs[s]):
+// first owned plane -> rank-1's upper halo, last owned plane -> rank+1's
+// lower halo; the halo beyond the global z boundary is zero-filled.
+// `on` = the stream the exchange runs on.
+int exchange(hpccg_problem *p, double *const *xs, cudaStream_t on) {
+    hpccg_ctx *ctx = p->ctx;
+    const Slab &s0 = p->slabs[0];
+    const int64_t n = s0.n, plane = s0.plane;
+    const size_t pb = (size_t)plane * sizeof(double);
+    if (ctx->mode == MODE_SINGLE) {
+        CU(cudaMemsetAsync(xs[0], 0, pb, on));
+        CU(cudaMemsetAsync(xs[0] + plane + n, 0, pb, on));
+        return HPCCG_OK;
+    }
+    if (ctx->mode == MODE_LOOPBACK) {
+        const int P = ctx->nslabs;
+        for (int r = 0; r < P; ++r) {
+            if (r > 0)  // my first owned plane -> (r-1)'s upper halo
+                CU(cudaMemcpyAsync(xs[r - 1] + plane + n, xs[r] + plane, pb,
+                                   cudaMemcpyDeviceToDevice, on));
+            else
+                CU(cudaMemsetAsync(xs[r], 0, pb, on));
+            if (r < P - 1)  // my last owned plane -> (r+1)'s lower halo
+                CU(cudaMemcpyAsync(xs[r + 1], xs[r] + n, pb, cudaMemcpyDeviceToDevice, on));
+            else
+                CU(cudaMemsetAsync(xs[r] + plane + n, 0, pb, on));
+        }
+        return HPCCG_OK;
+    }
+#ifdef HPCCG_WITH_NCCL
+    const int r = ctx->rank, P = ctx->nranks;
+    double *x = xs[0];
+    if (r == 0) CU(cudaMemsetAsync(x, 0, pb, on));
+    if (r == P - 1) CU(cudaMemsetAsync(x + plane + n, 0, pb, on));
+    NC(ctx, ncclGroupStart());
+    if (r > 0) {
+        NC(ctx, ncclSend(x + plane, plane, ncclDouble, r - 1, ctx->comm, on));
+        NC(ctx, ncclRecv(x, plane, ncclDouble, r - 1, ctx->comm, on));
+    }
+    if (r < P - 1) {
+        NC(ctx, ncclSend(x + n, plane, ncclDouble, r + 1, ctx->comm, on));
+        NC(ctx, ncclRecv(x + plane + n, plane, ncclDouble, r + 1, ctx->comm, on));
+    }
+    NC(ctx, ncclGroupEnd());
+    return HPCCG_OK;
+#else
+    return fail(HPCCG_ENOTSUP, "built without NCCL");
+#endif
+}
+
+// ------------------------------------------------------------- launchers
+
+SpmvArgs spmv_args(const Slab &s, const double *x, double *y) {
+    SpmvArgs a{};
+    a.stride = s.n;
+    a.plane = s.plane;
+    a.val = s.val;
+    a.col = s.col;
+    a.x = x;
+    a.y = y;
+    a.sc = s.sc;
+    a.red = s.red;
+    return a;
+}
+
+template <bool kDot>
+int launch_spmv(hpccg_ctx *ctx, SpmvArgs a, int64_t r0, int64_t len0, int64_t r1, int64_t len1,
+                cudaStream_t st) {
+    a.r0 = r0;
+    a.len0 = len0;
+    a.r1 = r1;
+    a.len1 = len1;
+    a.nb0 = cdiv(len0, kBlock);
+    const int64_t blocks = a.nb0 + cdiv(len1, kBlock);
+    if (blocks == 0) return HPCCG_OK;
+    if (blocks > 0x7fffffffLL) return fail(HPCCG_EINVAL, "SpMV grid too large");
+    spmv27_kernel<kDot><<<(unsigned)blocks, kBlock, 0, st>>>(a);
+    return check_launch(ctx);
+}
+
+// y = A x for one slab over all rows (no dot).
+int spmv_plain(hpccg_ctx *ctx, const Slab &s, const double *x, double *y, cudaStream_t st) {
+    return launch_spmv<false>(ctx, spmv_args(s, x, y), 0, s.n, 0, 0, st);
+}
+
+int launch_pupdate(hpccg_ctx *ctx, const Slab &s) {
+    double *po = s.p + s.plane;
+    const bool vec = aligned16(s.r) && aligned16(po);
+    const int g = stream_grid(vec ? s.n / 2 : s.n);
+    if (vec)
+        cg_pupdate_kernel<true><<<g, kBlock, 0, ctx->stream>>>(s.n, s.r, po, s.sc);
+    else
+        cg_pupdate_kernel<false><<<g, kBlock, 0, ctx->stream>>>(s.n, s.r, po, s.sc);
+    return check_launch(ctx);
+}
+
+int launch_update(hpccg_ctx *ctx, const Slab &s, int single) {
+    UpdArgs a{};
+    a.n = s.n;
+    a.x = s.x;
+    a.r = s.r;
+    a.p = s.p + s.plane;
+    a.Ap = s.Ap;
+    a.sc = s.sc;
+    a.red = s.red;
+    a.single = single;
+    const bool vec = aligned16(a.x) && aligned16(a.r) && aligned16(a.p) && aligned16(a.Ap);
+    const int g = stream_grid(vec ? s.n / 2 : s.n);
+    if (vec)
+        cg_update_kernel<true><<<g, kBlock, 0, ctx->stream>>>(a);
+    else
+        cg_update_kernel<false><<<g, kBlock, 0, ctx->stream>>>(a);
+    return check_launch(ctx);
+}
+
+// CG SpMV of every slab with the p.Ap epilogue.  Multi-slab: the rows that
+// do not touch a halo plane (interior) run first, overlapped with the halo
+// exchange on the comm stream (NCCL), then the two boundary planes.
+int cg_spmv_all(hpccg_problem *p, bool timing) {
+    hpccg_ctx *ctx = p->ctx;
+    const bool single = ctx->mode == MODE_SINGLE;
+    if (single) {
+        const Slab &s = p->slabs[0];
+        PhaseTimer t(p, ctx->stream, PH_SPMV, timing);
+        SpmvArgs a = spmv_args(s, s.p, s.Ap);
+        a.single = 1;
+        a.part_base = 0;
+        a.total_blocks = (unsigned)cdiv(s.n, kBlock);
+        return launch_spmv<true>(ctx, a, 0, s.n, 0, 0, ctx->stream);
+    }
+    const Slab &s0 = p->slabs[0];
+    const int64_t n = s0.n, plane = s0.plane;
+    // interior rows: planes 1..nz-2; boundary: plane 0 and plane nz-1
+    const int64_t int_r0 = plane, int_len = std::max<int64_t>(n - 2 * plane, 0);
+    const int64_t b0_len = std::min<int64_t>(plane, n);
+    const int64_t b1_r0 = std::max<int64_t>(n - plane, plane), b1_len = n - b1_r0;
+    const unsigned nb_int = (unsigned)cdiv(int_len, kBlock);
+    const unsigned nb_bnd = (unsigned)(cdiv(b0_len, kBlock) + cdiv(b1_len, kBlock));
+    std::vector<double *> xs(p->slabs.size());
+    for (size_t i = 0; i < xs.size(); ++i) xs[i] = p->slabs[i].p;
+
+    if (ctx->mode == MODE_NCCL) {
+        CU(cudaEventRecord(ctx->ev_fork, ctx->stream));
+        CU(cudaStreamWaitEvent(ctx->comm_stream, ctx->ev_fork, 0));
+        {
+            PhaseTimer t(p, ctx->comm_stream, PH_EXCHANGE, timing);
+            CHECK(exchange(p, xs.data(), ctx->comm_stream));
+        }
+        CU(cudaEventRecord(ctx->ev_join, ctx->comm_stream));
+        const Slab &s = p->slabs[0];
+        PhaseTimer t(p, ctx->stream, PH_SPMV, timing);
+        SpmvArgs a = spmv_args(s, s.p, s.Ap);
+        a.single = 0;
+        a.total_blocks = nb_int + nb_bnd;
+        a.part_base = 0;
+        CHECK(launch_spmv<true>(ctx, a, int_r0, int_len, 0, 0, ctx->stream));
+        CU(cudaStreamWaitEvent(ctx->stream, ctx->ev_join, 0));
+        a.part_base = nb_int;
+        return launch_spmv<true>(ctx, a, 0, b0_len, b1_r0, b1_len, ctx->stream);
+    }
+    // loopback: exchange, then interior + boundary launches per slab
+    {
+        PhaseTimer t(p, ctx->stream, PH_EXCHANGE, timing);
+        CHECK(exchange(p, xs.data(), ctx->stream));
+    }
+    PhaseTimer t(p, ctx->stream, PH_SPMV, timing);
+    for (const Slab &s : p->slabs) {
+        SpmvArgs a = spmv_args(s, s.p, s.Ap);
+        a.single = 0;
+        a.total_blocks = nb_int + nb_bnd;
+        a.part_base = 0;
+        CHECK(launch_spmv<true>(ctx, a, int_r0, int_len, 0, 0, ctx->stream));
+        a.part_base = nb_int;
+        CHECK(launch_spmv<true>(ctx, a, 0, b0_len, b1_r0, b1_len, ctx->stream));
+    }
+    return HPCCG_OK;
+}
+
+double **tab(hpccg_problem *p, int which) { return p->d_tab + (size_t)which * p->ctx->nslabs; }
+
+int allreduce_cg(hpccg_problem *p, bool rr, bool timing) {
+    hpccg_ctx *ctx = p->ctx;
+    if (ctx->mode == MODE_SINGLE) return HPCCG_OK;
+    PhaseTimer t(p, ctx->stream, PH_ALLREDUCE, timing);
+    const Slab &s = p->slabs[0];
+    double *hs[1] = {rr ? &s.sc->loc_rr : &s.sc->loc_pAp};
+    double *hd[1] = {rr ? &s.sc->rr_cur : &s.sc->pAp};
+    return allreduce_scalar(ctx, hs, hd, tab(p, rr ? 2 : 0), tab(p, rr ? 3 : 1), false);
+}
+
+// One CG iteration (a.6, a.2, a.3+a.4, a.5, a.8) for every slab.
+int enqueue_iteration(hpccg_problem *p, bool timing) {
+    hpccg_ctx *ctx = p->ctx;
+    const int single = ctx->mode == MODE_SINGLE;
+    {
+        PhaseTimer t(p, ctx->stream, PH_PUPDATE, timing);
+        for (const Slab &s : p->slabs) CHECK(launch_pupdate(ctx, s));
+    }
+    CHECK(cg_spmv_all(p, timing));
+    CHECK(allreduce_cg(p, false, timing));
+    {
+        PhaseTimer t(p, ctx->stream, PH_UPDATE, timing);
+        for (const Slab &s : p->slabs) CHECK(launch_update(ctx, s, single));
+    }
+    CHECK(allreduce_cg(p, true, timing));
+    return HPCCG_OK;
+}
+
+// a.7: p = x; halo; Ap = A p; r = b - Ap; rtrans = r.r; normr; first check.
+int enqueue_init(hpccg_problem *p, int max_iter, double tol, bool timing) {
+    hpccg_ctx *ctx = p->ctx;
+    const int single = ctx->mode == MODE_SINGLE;
+    for (const Slab &s : p->slabs) {
+        copy_kernel<<<stream_grid(s.n), kBlock, 0, ctx->stream>>>(s.n, s.x, s.p + s.plane);
+        CHECK(check_launch(ctx));
+    }
+    std::vector<double *> xs(p->slabs.size());
+    for (size_t i = 0; i < xs.size(); ++i) xs[i] = p->slabs[i].p;
+    {
+        PhaseTimer t(p, ctx->stream, PH_EXCHANGE, timing);
+        CHECK(exchange(p, xs.data(), ctx->stream));
+    }
+    {
+        PhaseTimer t(p, ctx->stream, PH_SPMV, timing);
+        for (const Slab &s : p->slabs) CHECK(spmv_plain(ctx, s, s.p, s.Ap, ctx->stream));
+    }
+    {
+        PhaseTimer t(p, ctx->stream, PH_UPDATE, timing);
+        for (const Slab &s : p->slabs) {
+            InitResArgs a{};
+            a.n = s.n;
+            a.b = s.b;
+            a.Ap = s.Ap;
+            a.r = s.r;
+            a.sc = s.sc;
+            a.red = s.red;
+            a.single = single;
+            cg_initres_kernel<<<stream_grid(s.n), kBlock, 0, ctx->stream>>>(a);
+            CHECK(check_launch(ctx));
+        }
+    }
+    CHECK(allreduce_cg(p, true, timing));
+    for (const Slab &s : p->slabs) {
+        cg_initstate_kernel<<<1, 1, 0, ctx->stream>>>(s.sc, max_iter, tol);
+        CHECK(check_launch(ctx));
+    }
+    return HPCCG_OK;
+}
+
+int build_graph(hpccg_problem *p) {
+    hpccg_ctx *ctx = p->ctx;
+    if (p->graph) return HPCCG_OK;
+    cudaGraph_t g = nullptr;
+    const int64_t l0 = ctx->launches;
+    CU(cudaStreamBeginCapture(ctx->stream, cudaStreamCaptureModeThreadLocal));
+    int rc = enqueue_iteration(p, false);
+    cudaError_t e = cudaStreamEndCapture(ctx->stream, &g);
+    if (rc != HPCCG_OK) {
+        if (g) cudaGraphDestroy(g);
+        return rc;
+    }
+    if (e != cudaSuccess) return fail(HPCCG_ECUDA, "graph capture: %s", cudaGetErrorString(e));
+    p->graph_kernels = ctx->launches - l0;
+    ctx->launches = l0;  // captured, not launched
+    e = cudaGraphInstantiate(&p->graph, g, 0);
+    cudaGraphDestroy(g);
+    if (e != cudaSuccess) {
+        p->graph = nullptr;
+        return fail(HPCCG_ECUDA, "graph instantiate: %s", cudaGetErrorString(e));
+    }
+    return HPCCG_OK;
+}
+
+int alloc_zero(void **ptr, size_t bytes) {
+    if (bytes == 0) bytes = 16;
+    cudaError_t e = cudaMalloc(ptr, bytes);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        return fail(HPCCG_ENOMEM, "cudaMalloc(%zu) failed: %s", bytes, cudaGetErrorString(e));
+    }
+    e = cudaMemset(*ptr, 0, bytes);
+    if (e != cudaSuccess) return fail(HPCCG_ECUDA, "cudaMemset: %s", cudaGetErrorString(e));
+    return HPCCG_OK;
+}
+
+void free_slab(Slab &s) {
+    cudaFree(s.val);
+    cudaFree(s.col);
+    cudaFree(s.b);
+    cudaFree(s.x);
+    cudaFree(s.xexact);
+    cudaFree(s.r);
+    cudaFree(s.Ap);
+    cudaFree(s.p_alloc);
+    cudaFree(s.sc);
+    cudaFree(s.red.partials);
+    cudaFree(s.red.counter);
+    s = Slab{};
+}
+
+int ctx_common_init(hpccg_ctx *c, int device, void *stream) {
+    c->device = device;
+    CU(cudaSetDevice(device));
+    if (stream) {
+        c->stream = (cudaStream_t)stream;
+    } else {
+        CU(cudaStreamCreateWithFlags(&c->stream, cudaStreamNonBlocking));
+        c->own_stream = true;
+    }
+    CU(cudaStreamCreateWithFlags(&c->comm_stream, cudaStreamNonBlocking));
+    CU(cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming));
+    CU(cudaEventCreateWithFlags(&c->ev_join, cudaEventDisableTiming));
+    CHECK(alloc_zero((void **)&c->d_api, sizeof(double) * 2 * c->nslabs));
+    CHECK(alloc_zero((void **)&c->d_api_src, sizeof(double *) * c->nslabs));
+    CHECK(alloc_zero((void **)&c->d_api_dst, sizeof(double *) * c->nslabs));
+    std::vector<double *> src(c->nslabs), dst(c->nslabs);
+    for (int s = 0; s < c->nslabs; ++s) {
+        src[s] = c->d_api + s;
+        dst[s] = c->d_api + c->nslabs + s;
+    }
+    CU(cudaMemcpy(c->d_api_src, src.data(), sizeof(double *) * c->nslabs, cudaMemcpyHostToDevice));
+    CU(cudaMemcpy(c->d_api_dst, dst.data(), sizeof(double *) * c->nslabs, cudaMemcpyHostToDevice));
+    c->red_cap = 148 * 8 + 64;
+    CHECK(alloc_zero((void **)&c->red.partials, sizeof(double) * c->red_cap));
+    CHECK(alloc_zero((void **)&c->red.counter, sizeof(unsigned)));
+    CU(cudaMallocHost((void **)&c->h_pinned, 8 * sizeof(double)));
+    return HPCCG_OK;
+}
+
+// Reduce n-element vectors per slab with `launch(slab, x_s, y_s, out_s)` and
+// allreduce the per-slab results; result on host.
+template <class L>
+int api_reduce(hpccg_ctx *ctx, bool is_max, double *result, L launch) {
+    const bool single = ctx->mode == MODE_SINGLE;
+    for (int s = 0; s < ctx->nslabs; ++s) {
+        double *out = single ? ctx->d_api + ctx->nslabs : ctx->d_api + s;
+        CHECK(launch(s, out));
+    }
+    if (!single) {
+        double *hs[1] = {ctx->d_api};
+        double *hd[1] = {ctx->d_api + ctx->nslabs};
+        CHECK(allreduce_scalar(ctx, hs, hd, ctx->d_api_src, ctx->d_api_dst, is_max));
+    }
+    CU(cudaMemcpyAsync(ctx->h_pinned, ctx->d_api + ctx->nslabs, sizeof(double),
+                       cudaMemcpyDeviceToHost, ctx->stream));
+    CU(cudaStreamSynchronize(ctx->stream));
+    *result = ctx->h_pinned[0];
+    return HPCCG_OK;
+}
+
+}  // namespace
+
+// ====================================================================== ABI
+
+extern "C" {
+
+const char *hpccg_strerror(int code) {
+    switch (code) {
+        case HPCCG_OK: return "HPCCG_OK";
+        case HPCCG_EINVAL: return "HPCCG_EINVAL";
+        case HPCCG_ENOMEM: return "HPCCG_ENOMEM";
+        case HPCCG_ECUDA: return "HPCCG_ECUDA";
+        case HPCCG_ENCCL: return "HPCCG_ENCCL";
+        case HPCCG_ENOTSUP: return "HPCCG_ENOTSUP";
+        default: return "HPCCG_E?";
+    }
+}
+
+const char *hpccg_last_error(void) { return g_err.c_str(); }
+
+const char *hpccg_version(void) {
+#ifdef HPCCG_WITH_NCCL
+    return "hpccg-b200 0.1 (sm_100a, nccl)";
+#else
+    return "hpccg-b200 0.1 (sm_100a)";
+#endif
+}
+
+int hpccg_launch_count(const hpccg_ctx *ctx, int64_t *count) {
+    if (!ctx || !count) return fail(HPCCG_EINVAL, "NULL argument");
+    *count = ctx->launches;
+    return HPCCG_OK;
+}
+
+int hpccg_unique_id(void *out) {
+    if (!out) return fail(HPCCG_EINVAL, "NULL out");
+#ifdef HPCCG_WITH_NCCL
+    static_assert(sizeof(ncclUniqueId) == HPCCG_UNIQUE_ID_BYTES, "unique id size");
+    ncclResult_t r = ncclGetUniqueId((ncclUniqueId *)out);
+    if (r != ncclSuccess) return fail(HPCCG_ENCCL, "ncclGetUniqueId: %s", ncclGetErrorString(r));
+    return HPCCG_OK;
+#else
+    return fail(HPCCG_ENOTSUP, "built without NCCL");
+#endif
+}
+
+int hpccg_init(hpccg_ctx **out, int device, void *stream, int rank, int nranks,
+               const void *unique_id) {
+    if (!out || nranks < 1 || rank < 0 || rank >= nranks)
+        return fail(HPCCG_EINVAL, "hpccg_init: bad rank/nranks");
+    if ((nranks == 1) != (unique_id == nullptr))
+        return fail(HPCCG_EINVAL, "hpccg_init: unique_id must be NULL iff nranks == 1");
+    *out = nullptr;
+    hpccg_ctx *c = new hpccg_ctx();
+    c->rank = rank;
+    c->nranks = nranks;
+    c->nslabs = 1;
+    c->mode = nranks == 1 ? MODE_SINGLE : MODE_NCCL;
+    int rc = ctx_common_init(c, device, stream);
+    if (rc != HPCCG_OK) {
+        hpccg_finalize(c);
+        return rc;
+    }
+    if (nranks > 1) {
+#ifdef HPCCG_WITH_NCCL
+        ncclUniqueId id;
+        memcpy(&id, unique_id, sizeof id);
+        ncclResult_t r = ncclCommInitRank(&c->comm, nranks, id, rank);
+        if (r != ncclSuccess) {
+            c->comm = nullptr;
+            hpccg_finalize(c);
+            return fail(HPCCG_ENCCL, "ncclCommInitRank: %s", ncclGetErrorString(r));
+        }
+#else
+        hpccg_finalize(c);
+        return fail(HPCCG_ENOTSUP, "built without NCCL");
+#endif
+    }
+    *out = c;
+    return HPCCG_OK;
+}
+
+int hpccg_init_loopback(hpccg_ctx **out, int device, void *stream, int nranks) {
+    if (!out || nranks < 1) return fail(HPCCG_EINVAL, "hpccg_init_loopback: bad nranks");
+    *out = nullptr;
+    hpccg_ctx *c = new hpccg_ctx();
+    c->rank = 0;
+    c->nranks = nranks;
+    c->nslabs = nranks;
+    c->mode = nranks == 1 ? MODE_SINGLE : MODE_LOOPBACK;
+    int rc = ctx_common_init(c, device, stream);
+    if (rc != HPCCG_OK) {
+        hpccg_finalize(c);
+        return rc;
+    }
+    *out = c;
+    return HPCCG_OK;
+}
+
+int hpccg_ctx_info(const hpccg_ctx *ctx, int *rank, int *nranks, int *nslabs) {
+    if (!ctx) return fail(HPCCG_EINVAL, "NULL ctx");
+    if (rank) *rank = ctx->rank;
+    if (nranks) *nranks = ctx->nranks;
+    if (nslabs) *nslabs = ctx->nslabs;
+    return HPCCG_OK;
+}
+
+void hpccg_finalize(hpccg_ctx *c) {
+    if (!c) return;
+    cudaSetDevice(c->device);
+    if (c->stream) cudaStreamSynchronize(c->stream);
+#ifdef HPCCG_WITH_NCCL
+    if (c->comm) ncclCommDestroy(c->comm);
+#endif
+    cudaFree(c->d_api);
+    cudaFree(c->d_api_src);
+    cudaFree(c->d_api_dst);
+    cudaFree(c->red.partials);
+    cudaFree(c->red.counter);
+    if (c->h_pinned) cudaFreeHost(c->h_pinned);
+    if (c->ev_fork) cudaEventDestroy(c->ev_fork);
+    if (c->ev_join) cudaEventDestroy(c->ev_join);
+    if (c->comm_stream) cudaStreamDestroy(c->comm_stream);
+    if (c->own_stream && c->stream) cudaStreamDestroy(c->stream);
+    delete c;
+}
+
+int hpccg_generate(hpccg_ctx *ctx, int nx, int ny, int nz, hpccg_problem **out) {
+    if (!ctx || !out) return fail(HPCCG_EINVAL, "NULL argument");
+    if (nx < 1 || ny < 1 || nz < 1) return fail(HPCCG_EINVAL, "nx, ny, nz must be >= 1");
+    const int64_t plane = (int64_t)nx * ny, n = plane * nz, ncol = n + 2 * plane;
+    if (ncol >= 0x7fffffffLL) return fail(HPCCG_EINVAL, "local problem too large for int32 columns");
+    if ((int64_t)nz * ctx->nranks >= 0x7fffffffLL) return fail(HPCCG_EINVAL, "nz * nranks too large");
+    *out = nullptr;
+    CU(cudaSetDevice(ctx->device));
+    hpccg_problem *p = new hpccg_problem();
+    p->ctx = ctx;
+    p->nx = nx;
+    p->ny = ny;
+    p->nz = nz;
+    p->slabs.resize(ctx->nslabs);
+    auto bail = [&](int rc) {
+        hpccg_free(p);
+        return rc;
+    };
+    for (int si = 0; si < ctx->nslabs; ++si) {
+        Slab &s = p->slabs[si];
+        s.rank = ctx->mode == MODE_LOOPBACK ? si : ctx->rank;
+        s.n = n;
+        s.plane = plane;
+        s.ncol = ncol;
+        int rc;
+        if ((rc = alloc_zero((void **)&s.val, sizeof(double) * kSlots * n))) return bail(rc);
+        if ((rc = alloc_zero((void **)&s.col, sizeof(int) * kSlots * n))) return bail(rc);
+        if ((rc = alloc_zero((void **)&s.b, sizeof(double) * n))) return bail(rc);
+        if ((rc = alloc_zero((void **)&s.x, sizeof(double) * n))) return bail(rc);
+        if ((rc = alloc_zero((void **)&s.xexact, sizeof(double) * n))) return bail(rc);
+        if ((rc = alloc_zero((void **)&s.r, sizeof(double) * n))) return bail(rc);
+        if ((rc = alloc_zero((void **)&s.Ap, sizeof(double) * n))) return bail(rc);
+        // p: [lower halo | n owned | upper halo]; shift by one element when
+        // the plane is odd so the owned part is 16-B aligned (double2 loads).
+        if ((rc = alloc_zero((void **)&s.p_alloc, sizeof(double) * (ncol + 2)))) return bail(rc);
+        s.p = s.p_alloc + ((plane & 1) ? 1 : 0);
+        if ((rc = alloc_zero((void **)&s.sc, sizeof(CgScalars)))) return bail(rc);
+        const int64_t parts = cdiv(n, kBlock) + 2 * cdiv(plane, kBlock) + 148 * 8 + 64;
+        if ((rc = alloc_zero((void **)&s.red.partials, sizeof(double) * parts))) return bail(rc);
+        if ((rc = alloc_zero((void **)&s.red.counter, sizeof(unsigned)))) return bail(rc);
+
+        GenArgs g{};
+        g.nx = nx;
+        g.ny = ny;
+        g.nz = nz;
+        g.rank = s.rank;
+        g.nranks = ctx->nranks;
+        g.n = n;
+        g.plane = plane;
+        g.val = s.val;
+        g.col = s.col;
+        g.b = s.b;
+        g.x = s.x;
+        g.xexact = s.xexact;
+        g.nnz = &s.sc->nnz;
+        const int64_t blocks = cdiv(n, kBlock);
+        gen27_kernel<<<(unsigned)blocks, kBlock, 0, ctx->stream>>>(g);
+        if ((rc = check_launch(ctx))) return bail(rc);
+    }
+    if (cudaStreamSynchronize(ctx->stream) != cudaSuccess)
+        return bail(fail(HPCCG_ECUDA, "generate: %s", cudaGetErrorString(cudaGetLastError())));
+    unsigned long long local = 0;
+    for (Slab &s : p->slabs) {
+        if (cudaMemcpy(&s.nnz, &s.sc->nnz, sizeof s.nnz, cudaMemcpyDeviceToHost) != cudaSuccess)
+            return bail(fail(HPCCG_ECUDA, "generate: nnz readback"));
+        local += s.nnz;
+    }
+    p->nnz_global = local;
+#ifdef HPCCG_WITH_NCCL
+    if (ctx->mode == MODE_NCCL) {
+        unsigned long long *d = nullptr;
+        int rc;
+        if ((rc = alloc_zero((void **)&d, sizeof *d))) return bail(rc);
+        cudaMemcpy(d, &local, sizeof local, cudaMemcpyHostToDevice);
+        ncclResult_t r = ncclAllReduce(d, d, 1, ncclUint64, ncclSum, ctx->comm, ctx->stream);
+        if (r != ncclSuccess) {
+            cudaFree(d);
+            return bail(nccl_fail(ctx, r, "ncclAllReduce(nnz)"));
+        }
+        cudaStreamSynchronize(ctx->stream);
+        cudaMemcpy(&p->nnz_global, d, sizeof local, cudaMemcpyDeviceToHost);
+        cudaFree(d);
+    }
+#endif
+    // loopback allreduce pointer tables
+    if (ctx->mode == MODE_LOOPBACK) {
+        const int P = ctx->nslabs;
+        int rc;
+        if ((rc = alloc_zero((void **)&p->d_tab, sizeof(double *) * 6 * P))) return bail(rc);
+        std::vector<double *> t(6 * P);
+        for (int s = 0; s < P; ++s) {
+            CgScalars *sc = p->slabs[s].sc;
+            t[0 * P + s] = &sc->loc_pAp;
+            t[1 * P + s] = &sc->pAp;
+            t[2 * P + s] = &sc->loc_rr;
+            t[3 * P + s] = &sc->rr_cur;
+            t[4 * P + s] = &sc->red_loc;
+            t[5 * P + s] = &sc->red_out;
+        }
+        if (cudaMemcpy(p->d_tab, t.data(), sizeof(double *) * 6 * P, cudaMemcpyHostToDevice) !=
+            cudaSuccess)
+            return bail(fail(HPCCG_ECUDA, "generate: table upload"));
+    }
+    if (cudaMallocHost((void **)&p->h_done, 2 * sizeof(int)) != cudaSuccess)
+        return bail(fail(HPCCG_ENOMEM, "pinned alloc"));
+    if (cudaEventCreate(&p->ev_t0) != cudaSuccess || cudaEventCreate(&p->ev_t1) != cudaSuccess ||
+        cudaEventCreateWithFlags(&p->ev_poll[0], cudaEventDisableTiming) != cudaSuccess ||
+        cudaEventCreateWithFlags(&p->ev_poll[1], cudaEventDisableTiming) != cudaSuccess)
+        return bail(fail(HPCCG_ECUDA, "event create"));
+    *out = p;
+    return HPCCG_OK;
+}
+
+int hpccg_info(const hpccg_problem *p, int64_t *nrow_local, int64_t *ncol_local,
+               int64_t *nnz_local, int64_t *nrow_global, int64_t *nnz_global) {
+    if (!p) return fail(HPCCG_EINVAL, "NULL problem");
+    const Slab &s = p->slabs[0];
+    unsigned long long loc = 0;
+    for (const Slab &q : p->slabs) loc += q.nnz;
+    if (nrow_local) *nrow_local = s.n;
+    if (ncol_local) *ncol_local = s.ncol;
+    if (nnz_local) *nnz_local = (int64_t)loc;
+    if (nrow_global) *nrow_global = s.n * p->ctx->nranks;
+    if (nnz_global) *nnz_global = (int64_t)p->nnz_global;
+    return HPCCG_OK;
+}
+
+static double *slab_vec(const Slab &s, int which) {
+    switch (which) {
+        case HPCCG_VEC_X: return s.x;
+        case HPCCG_VEC_B: return s.b;
+        case HPCCG_VEC_XEXACT: return s.xexact;
+        default: return nullptr;
+    }
+}
+
+int hpccg_vec(hpccg_problem *p, int which, double **dev_ptr) {
+    if (!p || !dev_ptr) return fail(HPCCG_EINVAL, "NULL argument");
+    if (p->slabs.size() > 1)
+        return fail(HPCCG_ENOTSUP, "hpccg_vec: loopback slabs are separate allocations; "
+                                   "use hpccg_get_vec / hpccg_set_vec");
+    double *v = slab_vec(p->slabs[0], which);
+    if (!v) return fail(HPCCG_EINVAL, "bad vector id %d", which);
+    *dev_ptr = v;
+    return HPCCG_OK;
+}
+
+int hpccg_set_vec(hpccg_problem *p, int which, const double *host_src) {
+    if (!p || !host_src) return fail(HPCCG_EINVAL, "NULL argument");
+    CU(cudaSetDevice(p->ctx->device));
+    for (size_t i = 0; i < p->slabs.size(); ++i) {
+        const Slab &s = p->slabs[i];
+        double *v = slab_vec(s, which);
+        if (!v) return fail(HPCCG_EINVAL, "bad vector id %d", which);
+        CU(cudaMemcpyAsync(v, host_src + i * s.n, sizeof(double) * s.n, cudaMemcpyHostToDevice,
+                           p->ctx->stream));
+    }
+    CU(cudaStreamSynchronize(p->ctx->stream));
+    return HPCCG_OK;
+}
+
+int hpccg_get_vec(const hpccg_problem *p, int which, double *host_dst) {
+    if (!p || !host_dst) return fail(HPCCG_EINVAL, "NULL argument");
+    CU(cudaSetDevice(p->ctx->device));
+    for (size_t i = 0; i < p->slabs.size(); ++i) {
+        const Slab &s = p->slabs[i];
+        double *v = slab_vec(s, which);
+        if (!v) return fail(HPCCG_EINVAL, "bad vector id %d", which);
+        CU(cudaMemcpyAsync(host_dst + i * s.n, v, sizeof(double) * s.n, cudaMemcpyDeviceToHost,
+                           p->ctx->stream));
+    }
+    CU(cudaStreamSynchronize(p->ctx->stream));
+    return HPCCG_OK;
+}
+
+int hpccg_copy_matrix(const hpccg_problem *p, int slab, double *val_host, int32_t *col_host) {
+    if (!p || !val_host || !col_host) return fail(HPCCG_EINVAL, "NULL argument");
+    if (slab < 0 || slab >= (int)p->slabs.size()) return fail(HPCCG_EINVAL, "bad slab");
+    CU(cudaSetDevice(p->ctx->device));
+    const Slab &s = p->slabs[slab];
+    CU(cudaMemcpy(val_host, s.val, sizeof(double) * kSlots * s.n, cudaMemcpyDeviceToHost));
+    CU(cudaMemcpy(col_host, s.col, sizeof(int) * kSlots * s.n, cudaMemcpyDeviceToHost));
+    return HPCCG_OK;
+}
+
+int hpccg_set_option(hpccg_problem *p, int key, int64_t value) {
+    if (!p) return fail(HPCCG_EINVAL, "NULL problem");
+    switch (key) {
+        case HPCCG_OPT_GRAPH: p->opt_graph = value != 0; return HPCCG_OK;
+        case HPCCG_OPT_POLL:
+            if (value < 0) return fail(HPCCG_EINVAL, "poll must be >= 0");
+            p->opt_poll = (int)value;
+            return HPCCG_OK;
+        case HPCCG_OPT_TIMING: p->opt_timing = value != 0; return HPCCG_OK;
+        default: return fail(HPCCG_EINVAL, "unknown option %d", key);
+    }
+}
+
+int hpccg_spmv(hpccg_problem *p, double *x, double *y) {
+    if (!p || !x || !y) return fail(HPCCG_EINVAL, "NULL argument");
+    hpccg_ctx *ctx = p->ctx;
+    CU(cudaSetDevice(ctx->device));
+    const size_t P = p->slabs.size();
+    const Slab &s0 = p->slabs[0];
+    std::vector<double *> xs(P);
+    for (size_t i = 0; i < P; ++i) xs[i] = x + i * s0.ncol;
+    // halo exchange on the main stream (API call: no overlap needed)
+    CHECK(exchange(p, xs.data(), ctx->stream));
+    for (size_t i = 0; i < P; ++i) CHECK(spmv_plain(ctx, p->slabs[i], xs[i], y + i * s0.n, ctx->stream));
+    CU(cudaStreamSynchronize(ctx->stream));
+    return HPCCG_OK;
+}
+
+int hpccg_ddot(hpccg_ctx *ctx, int64_t n, const double *x, const double *y, double *result) {
+    if (!ctx || !result || n < 0 || (n > 0 && (!x || !y))) return fail(HPCCG_EINVAL, "bad argument");
+    CU(cudaSetDevice(ctx->device));
+    return api_reduce(ctx, false, result, [&](int s, double *out) {
+        const double *xs = x + (size_t)s * n, *ys = y + (size_t)s * n;
+        const bool vec = aligned16(xs) && aligned16(ys);
+        const int g = stream_grid(vec ? n / 2 : n);
+        if (vec)
+            dot_kernel<true><<<g, kBlock, 0, ctx->stream>>>(n, xs, ys, ctx->red, out);
+        else
+            dot_kernel<false><<<g, kBlock, 0, ctx->stream>>>(n, xs, ys, ctx->red, out);
+        return check_launch(ctx);
+    });
+}
+
+int hpccg_waxpby(hpccg_ctx *ctx, int64_t n, double alpha, const double *x, double beta,
+                 const double *y, double *w) {
+    if (!ctx || n < 0 || (n > 0 && (!x || !y || !w))) return fail(HPCCG_EINVAL, "bad argument");
+    CU(cudaSetDevice(ctx->device));
+    const int64_t tot = n * ctx->nslabs;
+    if (tot == 0) return HPCCG_OK;
+    const bool vec = aligned16(x) && aligned16(y) && aligned16(w);
+    const int g = stream_grid(vec ? tot / 2 : tot);
+    const int form = alpha == 1.0 ? 0 : (beta == 1.0 ? 1 : 2);
+    cudaStream_t st = ctx->stream;
+#define WAX(V, F) waxpby_kernel<V, F><<<g, kBlock, 0, st>>>(tot, alpha, x, beta, y, w)
+    if (vec) {
+        if (form == 0) WAX(true, 0); else if (form == 1) WAX(true, 1); else WAX(true, 2);
+    } else {
+        if (form == 0) WAX(false, 0); else if (form == 1) WAX(false, 1); else WAX(false, 2);
+    }
+#undef WAX
+    CHECK(check_launch(ctx));
+    CU(cudaStreamSynchronize(st));
+    return HPCCG_OK;
+}
+
+int hpccg_maxabsdiff(hpccg_problem *p, double *result) {
+    if (!p || !result) return fail(HPCCG_EINVAL, "NULL argument");
+    hpccg_ctx *ctx = p->ctx;
+    CU(cudaSetDevice(ctx->device));
+    return api_reduce(ctx, true, result, [&](int s, double *out) {
+        const Slab &sl = p->slabs[s];
+        maxabsdiff_kernel<<<stream_grid(sl.n), kBlock, 0, ctx->stream>>>(sl.n, sl.x, sl.xexact,
+                                                                         ctx->red, out);
+        return check_launch(ctx);
+    });
+}
+
+int hpccg_solve(hpccg_problem *p, int max_iter, double tol, int *niters, double *normr,
+                double times[6]) {
+    if (!p) return fail(HPCCG_EINVAL, "NULL problem");
+    if (max_iter < 1 || !(tol >= 0.0)) return fail(HPCCG_EINVAL, "max_iter >= 1 and tol >= 0 required");
+    hpccg_ctx *ctx = p->ctx;
+    CU(cudaSetDevice(ctx->device));
+    const bool timing = p->opt_timing != 0;
+    const bool use_graph = p->opt_graph && !timing;
+    p->ev_used = 0;
+    p->timed.clear();
+    const int64_t l0 = ctx->launches;
+    if (use_graph) CHECK(build_graph(p));
+
+    CU(cudaEventRecord(p->ev_t0, ctx->stream));
+    CHECK(enqueue_init(p, max_iter, tol, timing));
+    // at most max_iter - 1 iterations (A4); finished iterations turn the
+    // remaining launches into no-ops on the device (done flag)
+    const int64_t iters = (int64_t)max_iter - 1;
+    const int poll = (tol > 0.0) ? p->opt_poll : 0;
+    const int *d_done = &p->slabs[0].sc->done;
+    int64_t launched = 0;
+    int chunk = 0;
+    bool stop = false;
+    while (launched < iters && !stop) {
+        const int64_t m = poll > 0 ? std::min<int64_t>(poll, iters - launched) : iters - launched;
+        for (int64_t i = 0; i < m; ++i) {
+            if (use_graph) {
+                CU(cudaGraphLaunch(p->graph, ctx->stream));
+                ctx->launches += p->graph_kernels;
+            } else {
+                CHECK(enqueue_iteration(p, timing));
+            }
+        }
+        launched += m;
+        if (poll > 0 && launched < iters) {
+            // double-buffered poll: queue this chunk's flag copy, then look at
+            // the previous chunk's, so the GPU always has a chunk queued
+            const int slot = chunk & 1;
+            CU(cudaMemcpyAsync(&p->h_done[slot], d_done, sizeof(int), cudaMemcpyDeviceToHost,
+                               ctx->stream));
+            CU(cudaEventRecord(p->ev_poll[slot], ctx->stream));
+            if (chunk > 0) {
+                CU(cudaEventSynchronize(p->ev_poll[slot ^ 1]));
+                if (p->h_done[slot ^ 1]) stop = true;
+            }
+            ++chunk;
+        }
+    }
+    CU(cudaEventRecord(p->ev_t1, ctx->stream));
+    CU(cudaStreamSynchronize(ctx->stream));
+    CU(cudaGetLastError());
+
+    CgScalars hs;
+    CU(cudaMemcpy(&hs, p->slabs[0].sc, sizeof hs, cudaMemcpyDeviceToHost));
+    hpccg_stats st{};
+    float ms = 0.f;
+    CU(cudaEventElapsedTime(&ms, p->ev_t0, p->ev_t1));
+    st.total_ms = ms;
+    for (const TimedOp &t : p->timed) {
+        float e = 0.f;
+        if (cudaEventElapsedTime(&e, t.a, t.b) != cudaSuccess) continue;
+        switch (t.phase) {
+            case PH_PUPDATE: st.pupdate_ms += e; break;
+            case PH_SPMV: st.spmv_ms += e; break;
+            case PH_UPDATE: st.update_ms += e; break;
+            case PH_ALLREDUCE: st.allreduce_ms += e; break;
+            case PH_EXCHANGE: st.exchange_ms += e; break;
+        }
+    }
+    st.iterations = hs.niters;
+    st.spmv_launches = hs.niters + 1;
+    st.kernel_launches = ctx->launches - l0;
+    p->stats = st;
+    if (niters) *niters = hs.niters;
+    if (normr) *normr = hs.normr;
+    if (times) {
+        times[0] = st.total_ms * 1e-3;
+        times[1] = 0.0;
+        times[2] = (st.pupdate_ms + st.update_ms) * 1e-3;
+        times[3] = st.spmv_ms * 1e-3;
+        times[4] = st.allreduce_ms * 1e-3;
+        times[5] = st.exchange_ms * 1e-3;
+    }
+    return HPCCG_OK;
+}
+
+int hpccg_get_stats(const hpccg_problem *p, hpccg_stats *out) {
+    if (!p || !out) return fail(HPCCG_EINVAL, "NULL argument");
+    *out = p->stats;
+    return HPCCG_OK;
+}
+
+void hpccg_free(hpccg_problem *p) {
+    if (!p) return;
+    cudaSetDevice(p->ctx->device);
+    cudaStreamSynchronize(p->ctx->stream);
+    if (p->graph) cudaGraphExecDestroy(p->graph);
+    for (Slab &s : p->slabs) free_slab(s);
+    cudaFree(p->d_tab);
+    for (cudaEvent_t e : p->ev_pool) cudaEventDestroy(e);
+    if (p->ev_t0) cudaEventDestroy(p->ev_t0);
+    if (p->ev_t1) cudaEventDestroy(p->ev_t1);
+    if (p->ev_poll[0]) cudaEventDestroy(p->ev_poll[0]);
+    if (p->ev_poll[1]) cudaEventDestroy(p->ev_poll[1]);
+    if (p->h_done) cudaFreeHost(p->h_done);
+    delete p;
+}
+
+}  // extern "C"

@@ -1,0 +1,472 @@
+// kernels.cuh -- sm_100a device code of the HPCCG CG hot path.
+//
+// Every step of the path runs here: problem generation (a.1), the 27-point
+// ELL SpMV with the p.Ap epilogue (a.3, a.4), the fused x/r update + r.r
+// (a.5), the p update (a.6), init (a.7), device-side loop control (a.8),
+// max|x - x_exact| (a.9) and the BLAS-1 waxpby / ddot (a.10).
+// Step ids and readings A<k> refer to DESIGN.md.
+//
+// The path is HBM-bandwidth bound (SpMV ~0.16 flop/B, BLAS-1 1/12..1/8
+// flop/B): no tensor cores.  What matters is coalescing (slot-major ELL,
+// consecutive rows on consecutive lanes), memory-level parallelism (all 54
+// matrix loads of a row issued before the FMA chain), keeping the matrix
+// stream from evicting the x planes out of L1/L2 (L1::no_allocate +
+// L2 evict_first on the matrix, default caching on x), and scalars that
+// never leave the device.
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+namespace hpccg {
+
+constexpr int kSlots = 27;      // 3x3x3 stencil slots per ELL row
+constexpr int kDiagSlot = 13;   // (sz, sy, sx) = (0, 0, 0)
+constexpr int kBlock = 256;     // threads per block of every kernel
+constexpr int kWarps = kBlock / 32;
+
+// Device-resident CG state, one per slab (A4 loop semantics, DESIGN.md
+// "Device-side scalars").  rr_cur / rr_prev are GLOBAL (allreduced) values.
+struct CgScalars {
+    double rr_cur;    // r.r of the current r            (global)
+    double rr_prev;   // rtrans of the previous iteration (global)
+    double pAp;       // p.Ap of this iteration           (global)
+    double loc_rr;    // this slab's partial r.r   (allreduce input)
+    double loc_pAp;   // this slab's partial p.Ap  (allreduce input)
+    double normr;     // sqrt(rtrans) of the last iteration run
+    double tol;
+    double red_loc;   // generic reduction (ddot API, maxabsdiff): local
+    double red_out;   //   ... and global result
+    unsigned long long nnz;  // stored entries counted by gen27
+    int k;            // index of the next CG iteration
+    int niters;
+    int done;         // loop-exit flag, read by every CG kernel
+    int max_iter;
+};
+
+// Scratch for the deterministic single-pass grid reduction.
+struct Reduction {
+    double *partials;       // one slot per block (of all launches in the pass)
+    unsigned int *counter;  // blocks finished; reset to 0 by the last block
+};
+
+// ------------------------------------------------------------ PTX helpers
+
+__device__ __forceinline__ uint64_t policy_evict_first() {
+    uint64_t p;
+    asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+
+// Matrix stream: read once per SpMV -> do not allocate in L1, evict first
+// from L2 so it does not push the x planes / CG vectors out.
+__device__ __forceinline__ double ld_stream(const double *ptr, uint64_t pol) {
+    double v;
+    asm("ld.global.nc.L1::no_allocate.L2::cache_hint.f64 %0, [%1], %2;"
+        : "=d"(v) : "l"(ptr), "l"(pol));
+    return v;
+}
+
+__device__ __forceinline__ int ld_stream(const int *ptr, uint64_t pol) {
+    int v;
+    asm("ld.global.nc.L1::no_allocate.L2::cache_hint.s32 %0, [%1], %2;"
+        : "=r"(v) : "l"(ptr), "l"(pol));
+    return v;
+}
+
+__device__ __forceinline__ double warp_sum(double v) {
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+    return v;
+}
+
+__device__ __forceinline__ double warp_max(double v) {
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) v = fmax(v, __shfl_xor_sync(0xffffffffu, v, o));
+    return v;
+}
+
+// Block-wide reduction in a fixed order (butterfly per warp, then warp 0 over
+// the per-warp values).  Result valid in every thread of warp 0.
+template <bool kMax>
+__device__ __forceinline__ double block_reduce(double v, double *sh) {
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    v = kMax ? warp_max(v) : warp_sum(v);
+    if (lane == 0) sh[warp] = v;
+    __syncthreads();
+    if (warp == 0) {
+        v = (lane < kWarps) ? sh[lane] : (kMax ? 0.0 : 0.0);
+        v = kMax ? warp_max(v) : warp_sum(v);
+    }
+    return v;
+}
+
+// Deterministic single-pass grid reduction ("last block done"): every block
+// writes its partial to partials[part]; the block that finishes last sums all
+// `total` partials in a fixed order and calls fin(result) on thread 0.  The
+// result depends only on the grid shape, never on scheduling (no fp atomics).
+// kMax: max instead of sum (values are >= 0).
+template <bool kMax, class Fin>
+__device__ __forceinline__ void grid_reduce(double v, Reduction red, unsigned part,
+                                            unsigned total, Fin fin) {
+    __shared__ double sh[32];
+    __shared__ int is_last;
+    v = block_reduce<kMax>(v, sh);
+    if (threadIdx.x == 0) {
+        red.partials[part] = v;
+        __threadfence();
+        unsigned t = atomicAdd(red.counter, 1u);
+        is_last = (t == total - 1);
+    }
+    __syncthreads();
+    if (!is_last) return;
+    __threadfence();
+    double s = 0.0;
+    for (unsigned i = threadIdx.x; i < total; i += kBlock) {
+        double q = __ldcg(red.partials + i);
+        s = kMax ? fmax(s, q) : s + q;
+    }
+    __syncthreads();  // sh reuse
+    s = block_reduce<kMax>(s, sh);
+    if (threadIdx.x == 0) {
+        *red.counter = 0u;
+        fin(s);
+    }
+}
+
+// ------------------------------------------------------- a.1 generation
+
+struct GenArgs {
+    int nx, ny, nz;       // local slab dims
+    int rank, nranks;     // z-slab of the global nx x ny x (nz*nranks) grid
+    int64_t n, plane;     // rows, nx*ny
+    double *val;          // [27][n]
+    int *col;             // [27][n]  local-with-halo index
+    double *b, *x, *xexact;
+    unsigned long long *nnz;
+};
+
+// One thread per local row.  Slot s <-> (sz, sy, sx) = (s/9-1, s/3%3-1, s%3-1):
+// ascending column (A8).  Absent neighbour -> padding (0.0, own column).
+__global__ void __launch_bounds__(kBlock) gen27_kernel(GenArgs a) {
+    __shared__ double sh[32];
+    const int64_t i = (int64_t)blockIdx.x * kBlock + threadIdx.x;
+    double cnt_d = 0.0;
+    if (i < a.n) {
+        const int64_t iz = i / a.plane;
+        const int64_t rem = i - iz * a.plane;
+        const int iy = (int)(rem / a.nx);
+        const int ix = (int)(rem - (int64_t)iy * a.nx);
+        const int64_t gz = (int64_t)a.rank * a.nz + iz;
+        const int64_t nzg = (int64_t)a.nz * a.nranks;
+        const int64_t own = i + a.plane;  // local-with-halo index of row i
+        int cnt = 0;
+#pragma unroll
+        for (int s = 0; s < kSlots; ++s) {
+            const int sz = s / 9 - 1, sy = (s / 3) % 3 - 1, sx = s % 3 - 1;
+            const bool in = (ix + sx >= 0) && (ix + sx < a.nx) && (iy + sy >= 0) &&
+                            (iy + sy < a.ny) && (gz + sz >= 0) && (gz + sz < nzg);
+            const int64_t c = own + sz * a.plane + (int64_t)sy * a.nx + sx;
+            a.val[(int64_t)s * a.n + i] = in ? (s == kDiagSlot ? 27.0 : -1.0) : 0.0;
+            a.col[(int64_t)s * a.n + i] = (int)(in ? c : own);
+            cnt += in;
+        }
+        a.b[i] = 28.0 - (double)cnt;  // = row sum: A.1 = b, x_exact = 1
+        a.x[i] = 0.0;
+        a.xexact[i] = 1.0;
+        cnt_d = (double)cnt;
+    }
+    // exact integer count (<= 27*256 per block)
+    double bs = block_reduce<false>(cnt_d, sh);
+    if (threadIdx.x == 0) atomicAdd(a.nnz, (unsigned long long)bs);
+}
+
+// --------------------------------------------------------- a.3 SpMV (ELL-27)
+
+// Rows of up to two disjoint ranges [r0, r0+len0) and [r1, r1+len1) (the
+// interior / boundary split used to overlap the halo exchange).
+struct SpmvArgs {
+    int64_t r0, len0, r1, len1;
+    int64_t nb0;            // blocks covering range 0
+    int64_t stride;         // slot stride = n
+    int64_t plane;          // x[row + plane] is the row's own entry
+    const double *val;
+    const int *col;
+    const double *x;        // local-with-halo base (ncol entries)
+    double *y;              // n entries
+    // CG epilogue (kDot): partial p.Ap -> scalars
+    CgScalars *sc;
+    Reduction red;
+    unsigned part_base, total_blocks;
+    int single;             // 1: write the global pAp directly (no allreduce)
+};
+
+template <bool kDot>
+__global__ void __launch_bounds__(kBlock) spmv27_kernel(SpmvArgs a) {
+    if (kDot && a.sc->done) return;  // uniform over the grid
+    int64_t row, lim;
+    if ((int64_t)blockIdx.x < a.nb0) {
+        row = a.r0 + (int64_t)blockIdx.x * kBlock + threadIdx.x;
+        lim = a.r0 + a.len0;
+    } else {
+        row = a.r1 + ((int64_t)blockIdx.x - a.nb0) * kBlock + threadIdx.x;
+        lim = a.r1 + a.len1;
+    }
+    double d = 0.0;
+    if (row < lim) {
+        const uint64_t pol = policy_evict_first();
+        const double *v = a.val + row;
+        const int *c = a.col + row;
+        double vv[kSlots];
+        int cc[kSlots];
+#pragma unroll
+        for (int s = 0; s < kSlots; ++s) {
+            vv[s] = ld_stream(v + s * a.stride, pol);
+            cc[s] = ld_stream(c + s * a.stride, pol);
+        }
+        double sum = 0.0;  // FMA chain in ascending column from +0.0 (A8)
+#pragma unroll
+        for (int s = 0; s < kSlots; ++s) sum = fma(vv[s], __ldg(a.x + cc[s]), sum);
+        a.y[row] = sum;
+        if (kDot) d = sum * __ldg(a.x + row + a.plane);
+    }
+    if (kDot) {
+        CgScalars *sc = a.sc;
+        const int single = a.single;
+        grid_reduce<false>(d, a.red, a.part_base + blockIdx.x, a.total_blocks,
+                           [sc, single](double s) {
+                               if (single) sc->pAp = s; else sc->loc_pAp = s;
+                           });
+    }
+}
+
+// ------------------------------------------------ streaming vector kernels
+// Grid-stride loops over 2-element (16 B) vectors when every pointer is
+// 16-B aligned (kVec), scalar otherwise.  The element -> thread mapping is a
+// function of (n, grid) only, so the reductions are run-to-run deterministic.
+
+// a.6: p = r + beta p  (k == 1: p = r)            -- 24n B
+template <bool kVec>
+__global__ void __launch_bounds__(kBlock) cg_pupdate_kernel(int64_t n, const double *__restrict__ r,
+                                                           double *__restrict__ p,
+                                                           const CgScalars *sc) {
+    if (sc->done) return;
+    const bool first = (sc->k == 1);
+    const double beta = first ? 0.0 : sc->rr_cur / sc->rr_prev;
+    const int64_t tid = (int64_t)blockIdx.x * kBlock + threadIdx.x;
+    const int64_t nth = (int64_t)gridDim.x * kBlock;
+    if (kVec) {
+        const int64_t nv = n >> 1;
+        const double2 *r2 = reinterpret_cast<const double2 *>(r);
+        double2 *p2 = reinterpret_cast<double2 *>(p);
+        for (int64_t i = tid; i < nv; i += nth) {
+            double2 rv = __ldcs(r2 + i);
+            double2 pv = first ? rv : __ldcs(p2 + i);
+            if (!first) {
+                pv.x = fma(beta, pv.x, rv.x);
+                pv.y = fma(beta, pv.y, rv.y);
+            }
+            p2[i] = pv;
+        }
+        if (tid == 0 && (n & 1)) {
+            const int64_t i = n - 1;
+            p[i] = first ? r[i] : fma(beta, p[i], r[i]);
+        }
+    } else {
+        for (int64_t i = tid; i < n; i += nth) p[i] = first ? r[i] : fma(beta, p[i], r[i]);
+    }
+}
+
+// a.5: x += alpha p; r -= alpha Ap; partial r.r; then the loop control of
+// the NEXT iteration (A4 lagged check, A11 guard) in the last block.  48n B.
+struct UpdArgs {
+    int64_t n;
+    double *x, *r;
+    const double *p, *Ap;
+    CgScalars *sc;
+    Reduction red;
+    int single;
+};
+
+template <bool kVec>
+__global__ void __launch_bounds__(kBlock) cg_update_kernel(UpdArgs a) {
+    CgScalars *sc = a.sc;
+    if (sc->done) return;
+    const double rtrans = sc->rr_cur, pAp = sc->pAp;
+    const bool stop = (rtrans == 0.0) || (pAp == 0.0);  // A11
+    const double alpha = stop ? 0.0 : rtrans / pAp;
+    const int64_t tid = (int64_t)blockIdx.x * kBlock + threadIdx.x;
+    const int64_t nth = (int64_t)gridDim.x * kBlock;
+    double acc = 0.0;
+    if (kVec) {
+        const int64_t nv = a.n >> 1;
+        double2 *x2 = reinterpret_cast<double2 *>(a.x);
+        double2 *r2 = reinterpret_cast<double2 *>(a.r);
+        const double2 *p2 = reinterpret_cast<const double2 *>(a.p);
+        const double2 *q2 = reinterpret_cast<const double2 *>(a.Ap);
+        for (int64_t i = tid; i < nv; i += nth) {
+            double2 xv = x2[i], rv = r2[i];
+            const double2 pv = __ldcs(p2 + i), qv = __ldcs(q2 + i);
+            xv.x = fma(alpha, pv.x, xv.x);
+            xv.y = fma(alpha, pv.y, xv.y);
+            rv.x = fma(-alpha, qv.x, rv.x);
+            rv.y = fma(-alpha, qv.y, rv.y);
+            x2[i] = xv;
+            r2[i] = rv;
+            acc = fma(rv.x, rv.x, acc);
+            acc = fma(rv.y, rv.y, acc);
+        }
+        if (tid == 0 && (a.n & 1)) {
+            const int64_t i = a.n - 1;
+            a.x[i] = fma(alpha, a.p[i], a.x[i]);
+            const double rv = fma(-alpha, a.Ap[i], a.r[i]);
+            a.r[i] = rv;
+            acc = fma(rv, rv, acc);
+        }
+    } else {
+        for (int64_t i = tid; i < a.n; i += nth) {
+            a.x[i] = fma(alpha, a.p[i], a.x[i]);
+            const double rv = fma(-alpha, a.Ap[i], a.r[i]);
+            a.r[i] = rv;
+            acc = fma(rv, rv, acc);
+        }
+    }
+    const int single = a.single;
+    grid_reduce<false>(acc, a.red, blockIdx.x, gridDim.x,
+                       [sc, single, rtrans, stop](double s) {
+                           sc->rr_prev = rtrans;
+                           if (single) sc->rr_cur = s; else sc->loc_rr = s;
+                           const int k = sc->k;
+                           const double normr = sqrt(rtrans);
+                           sc->normr = normr;
+                           sc->niters = k;
+                           sc->k = k + 1;
+                           sc->done = stop || !((k + 1) < sc->max_iter && normr > sc->tol);
+                       });
+}
+
+// a.7 init: r = b - Ap (waxpby(1, b, -1, Ap) = fma(-1, Ap, b)) and r.r.
+struct InitResArgs {
+    int64_t n;
+    const double *b, *Ap;
+    double *r;
+    CgScalars *sc;
+    Reduction red;
+    int single;
+};
+
+__global__ void __launch_bounds__(kBlock) cg_initres_kernel(InitResArgs a) {
+    const int64_t tid = (int64_t)blockIdx.x * kBlock + threadIdx.x;
+    const int64_t nth = (int64_t)gridDim.x * kBlock;
+    double acc = 0.0;
+    for (int64_t i = tid; i < a.n; i += nth) {
+        const double rv = fma(-1.0, a.Ap[i], a.b[i]);
+        a.r[i] = rv;
+        acc = fma(rv, rv, acc);
+    }
+    CgScalars *sc = a.sc;
+    const int single = a.single;
+    grid_reduce<false>(acc, a.red, blockIdx.x, gridDim.x, [sc, single](double s) {
+        if (single) sc->rr_cur = s; else sc->loc_rr = s;
+    });
+}
+
+// a.7/a.8: after the (allreduced) initial r.r: k = 1, normr, first check.
+__global__ void cg_initstate_kernel(CgScalars *sc, int max_iter, double tol) {
+    const double rr = sc->rr_cur;
+    const double normr = sqrt(rr);
+    sc->rr_prev = rr;
+    sc->normr = normr;
+    sc->tol = tol;
+    sc->max_iter = max_iter;
+    sc->k = 1;
+    sc->niters = 0;
+    sc->done = !(1 < max_iter && normr > tol);
+}
+
+// Loopback allreduce: fixed rank-order sum (or max) of one scalar of every
+// slab, written back to every slab (deterministic, identical on all slabs).
+__global__ void slab_allreduce_kernel(const double *const *src, double *const *dst,
+                                      int nslabs, int is_max) {
+    if (threadIdx.x != 0 || blockIdx.x != 0) return;
+    double s = *src[0];
+    for (int r = 1; r < nslabs; ++r) s = is_max ? fmax(s, *src[r]) : s + *src[r];
+    for (int r = 0; r < nslabs; ++r) *dst[r] = s;
+}
+
+// ---------------------------------------------------------- a.10 BLAS-1
+
+// w = alpha x + beta y, canonical forms (A10).  form: 0 alpha==1, 1 beta==1,
+// 2 general.  24n B.
+template <bool kVec, int kForm>
+__global__ void __launch_bounds__(kBlock) waxpby_kernel(int64_t n, double alpha, const double *x,
+                                                       double beta, const double *y, double *w) {
+    const int64_t tid = (int64_t)blockIdx.x * kBlock + threadIdx.x;
+    const int64_t nth = (int64_t)gridDim.x * kBlock;
+    auto op = [alpha, beta](double xv, double yv) {
+        if (kForm == 0) return fma(beta, yv, xv);
+        if (kForm == 1) return fma(alpha, xv, yv);
+        return fma(alpha, xv, beta * yv);
+    };
+    if (kVec) {
+        const int64_t nv = n >> 1;
+        const double2 *x2 = reinterpret_cast<const double2 *>(x);
+        const double2 *y2 = reinterpret_cast<const double2 *>(y);
+        double2 *w2 = reinterpret_cast<double2 *>(w);
+        for (int64_t i = tid; i < nv; i += nth) {
+            const double2 xv = x2[i], yv = y2[i];
+            double2 o;
+            o.x = op(xv.x, yv.x);
+            o.y = op(xv.y, yv.y);
+            w2[i] = o;
+        }
+        if (tid == 0 && (n & 1)) w[n - 1] = op(x[n - 1], y[n - 1]);
+    } else {
+        for (int64_t i = tid; i < n; i += nth) w[i] = op(x[i], y[i]);
+    }
+}
+
+// sum_i x_i y_i -> *out (deterministic).  16n B (8n for x.x).
+template <bool kVec>
+__global__ void __launch_bounds__(kBlock) dot_kernel(int64_t n, const double *x, const double *y,
+                                                    Reduction red, double *out) {
+    const int64_t tid = (int64_t)blockIdx.x * kBlock + threadIdx.x;
+    const int64_t nth = (int64_t)gridDim.x * kBlock;
+    double acc = 0.0;
+    if (kVec) {
+        const int64_t nv = n >> 1;
+        const double2 *x2 = reinterpret_cast<const double2 *>(x);
+        const double2 *y2 = reinterpret_cast<const double2 *>(y);
+        double acc2 = 0.0;
+        for (int64_t i = tid; i < nv; i += nth) {
+            const double2 xv = __ldcs(x2 + i), yv = __ldcs(y2 + i);
+            acc = fma(xv.x, yv.x, acc);
+            acc2 = fma(xv.y, yv.y, acc2);
+        }
+        acc += acc2;
+        if (tid == 0 && (n & 1)) acc = fma(x[n - 1], y[n - 1], acc);
+    } else {
+        for (int64_t i = tid; i < n; i += nth) acc = fma(x[i], y[i], acc);
+    }
+    grid_reduce<false>(acc, red, blockIdx.x, gridDim.x, [out](double s) { *out = s; });
+}
+
+// a.9: max_i |x_i - xe_i| -> *out
+__global__ void __launch_bounds__(kBlock) maxabsdiff_kernel(int64_t n, const double *x,
+                                                           const double *xe, Reduction red,
+                                                           double *out) {
+    const int64_t tid = (int64_t)blockIdx.x * kBlock + threadIdx.x;
+    const int64_t nth = (int64_t)gridDim.x * kBlock;
+    double m = 0.0;
+    for (int64_t i = tid; i < n; i += nth) m = fmax(m, fabs(x[i] - xe[i]));
+    grid_reduce<true>(m, red, blockIdx.x, gridDim.x, [out](double s) { *out = s; });
+}
+
+// p = x for the owned part (init, waxpby(1, x, 0, x, p) = x exactly).
+__global__ void __launch_bounds__(kBlock) copy_kernel(int64_t n, const double *src, double *dst) {
+    const int64_t tid = (int64_t)blockIdx.x * kBlock + threadIdx.x;
+    const int64_t nth = (int64_t)gridDim.x * kBlock;
+    for (int64_t i = tid; i < n; i += nth) dst[i] = src[i];
+}
+
+}  // namespace hpccg

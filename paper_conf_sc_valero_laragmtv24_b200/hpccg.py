@@ -1,0 +1,344 @@
+"""Thin ctypes binding of libhpccg.so (include/hpccg.h).
+
+Argument marshalling only: every step of the path runs in the library's
+sm_100a kernels.  There is no CPU fallback -- if ``libhpccg.so`` is missing or
+fails to load, every entry point raises.  The module-level functions carry the
+C names (``hpccg_generate``, ``hpccg_spmv``, ...); ``Context`` / ``Problem``
+wrap them for convenience.  torch is used only for device memory and streams:
+device-vector arguments may be CUDA float64 torch tensors (contiguous) or raw
+device pointers (int).
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import re
+import threading
+
+import numpy as np
+
+_PKG = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_PKG, "libhpccg.so")
+HEADER = os.path.join(os.path.dirname(_PKG), "include", "hpccg.h")
+
+HPCCG_OK = 0
+HPCCG_EINVAL = -1
+HPCCG_ENOMEM = -2
+HPCCG_ECUDA = -3
+HPCCG_ENCCL = -4
+HPCCG_ENOTSUP = -5
+HPCCG_UNIQUE_ID_BYTES = 128
+HPCCG_VEC_X, HPCCG_VEC_B, HPCCG_VEC_XEXACT = 0, 1, 2
+HPCCG_OPT_GRAPH, HPCCG_OPT_POLL, HPCCG_OPT_TIMING = 0, 1, 2
+
+_lock = threading.Lock()
+_lib = None
+
+
+class HpccgError(RuntimeError):
+    def __init__(self, code: int, where: str, detail: str):
+        super().__init__(f"{where}: {detail or ''} [{code}]")
+        self.code = code
+
+
+class hpccg_stats(ctypes.Structure):
+    _fields_ = [("total_ms", ctypes.c_double), ("spmv_ms", ctypes.c_double),
+                ("update_ms", ctypes.c_double), ("pupdate_ms", ctypes.c_double),
+                ("allreduce_ms", ctypes.c_double), ("exchange_ms", ctypes.c_double),
+                ("spmv_launches", ctypes.c_int64), ("iterations", ctypes.c_int64),
+                ("kernel_launches", ctypes.c_int64)]
+
+    def as_dict(self):
+        return {k: getattr(self, k) for k, _ in self._fields_}
+
+
+_vp, _i, _i64, _d = ctypes.c_void_p, ctypes.c_int, ctypes.c_int64, ctypes.c_double
+_pi64 = ctypes.POINTER(ctypes.c_int64)
+_SIGS = {
+    "hpccg_strerror": ([_i], ctypes.c_char_p),
+    "hpccg_last_error": ([], ctypes.c_char_p),
+    "hpccg_version": ([], ctypes.c_char_p),
+    "hpccg_launch_count": ([_vp, _pi64], _i),
+    "hpccg_unique_id": ([_vp], _i),
+    "hpccg_init": ([ctypes.POINTER(_vp), _i, _vp, _i, _i, _vp], _i),
+    "hpccg_init_loopback": ([ctypes.POINTER(_vp), _i, _vp, _i], _i),
+    "hpccg_ctx_info": ([_vp, ctypes.POINTER(_i), ctypes.POINTER(_i), ctypes.POINTER(_i)], _i),
+    "hpccg_finalize": ([_vp], None),
+    "hpccg_generate": ([_vp, _i, _i, _i, ctypes.POINTER(_vp)], _i),
+    "hpccg_info": ([_vp, _pi64, _pi64, _pi64, _pi64, _pi64], _i),
+    "hpccg_vec": ([_vp, _i, ctypes.POINTER(_vp)], _i),
+    "hpccg_set_vec": ([_vp, _i, _vp], _i),
+    "hpccg_get_vec": ([_vp, _i, _vp], _i),
+    "hpccg_copy_matrix": ([_vp, _i, _vp, _vp], _i),
+    "hpccg_set_option": ([_vp, _i, _i64], _i),
+    "hpccg_spmv": ([_vp, _vp, _vp], _i),
+    "hpccg_ddot": ([_vp, _i64, _vp, _vp, ctypes.POINTER(_d)], _i),
+    "hpccg_waxpby": ([_vp, _i64, _d, _vp, _d, _vp, _vp], _i),
+    "hpccg_solve": ([_vp, _i, _d, ctypes.POINTER(_i), ctypes.POINTER(_d), _vp], _i),
+    "hpccg_get_stats": ([_vp, ctypes.POINTER(hpccg_stats)], _i),
+    "hpccg_maxabsdiff": ([_vp, ctypes.POINTER(_d)], _i),
+    "hpccg_free": ([_vp], None),
+}
+
+
+def header_symbols(path: str = HEADER):
+    """Every function the C header declares (HPCCG_API ... name(...))."""
+    txt = open(path).read()
+    return sorted(set(re.findall(r"HPCCG_API[^;(]*?\b(hpccg_\w+)\s*\(", txt)))
+
+
+def lib():
+    """Load libhpccg.so (raises if it is missing: there is no fallback)."""
+    global _lib
+    with _lock:
+        if _lib is not None:
+            return _lib
+        if not os.path.exists(LIB_PATH):
+            raise RuntimeError(f"{LIB_PATH} is missing: build it with "
+                               "`python -c 'import __graft_entry__ as g; g.build()'`")
+        L = ctypes.CDLL(LIB_PATH)
+        for name, (args, res) in _SIGS.items():
+            f = getattr(L, name)
+            f.argtypes = args
+            f.restype = res
+        _lib = L
+        return L
+
+
+def _check(rc: int, where: str):
+    if rc != HPCCG_OK:
+        L = lib()
+        raise HpccgError(rc, where, (L.hpccg_last_error() or b"").decode())
+
+
+def _ptr(t) -> int:
+    """Device pointer of a CUDA tensor (contiguous float64) or a raw int."""
+    if isinstance(t, int):
+        return t
+    import torch
+    if not isinstance(t, torch.Tensor):
+        raise TypeError("expected a torch CUDA tensor or a raw device pointer")
+    if not t.is_cuda or t.dtype != torch.float64 or not t.is_contiguous():
+        raise TypeError("device vectors must be contiguous CUDA float64 tensors")
+    return t.data_ptr()
+
+
+def _torch_sync():
+    """Order the library's stream after torch's pending work on user tensors."""
+    try:
+        import torch
+        if torch.cuda.is_available() and torch.cuda.is_initialized():
+            torch.cuda.current_stream().synchronize()
+    except Exception:  # pragma: no cover
+        pass
+
+
+# ------------------------------------------------------------ C-named calls
+
+def hpccg_version() -> str:
+    return lib().hpccg_version().decode()
+
+
+def hpccg_strerror(code: int) -> str:
+    return lib().hpccg_strerror(code).decode()
+
+
+def hpccg_unique_id() -> bytes:
+    buf = ctypes.create_string_buffer(HPCCG_UNIQUE_ID_BYTES)
+    _check(lib().hpccg_unique_id(buf), "hpccg_unique_id")
+    return buf.raw
+
+
+def hpccg_init(device: int = 0, stream: int | None = None, rank: int = 0, nranks: int = 1,
+               unique_id: bytes | None = None) -> int:
+    h = _vp()
+    uid = None
+    if unique_id is not None:
+        uid = ctypes.create_string_buffer(bytes(unique_id), HPCCG_UNIQUE_ID_BYTES)
+    _check(lib().hpccg_init(ctypes.byref(h), device, stream or None, rank, nranks, uid),
+           "hpccg_init")
+    return h.value
+
+
+def hpccg_init_loopback(device: int = 0, stream: int | None = None, nranks: int = 2) -> int:
+    h = _vp()
+    _check(lib().hpccg_init_loopback(ctypes.byref(h), device, stream or None, nranks),
+           "hpccg_init_loopback")
+    return h.value
+
+
+def hpccg_finalize(ctx: int) -> None:
+    lib().hpccg_finalize(ctx)
+
+
+def hpccg_generate(ctx: int, nx: int, ny: int, nz: int) -> int:
+    h = _vp()
+    _check(lib().hpccg_generate(ctx, nx, ny, nz, ctypes.byref(h)), "hpccg_generate")
+    return h.value
+
+
+def hpccg_info(prob: int) -> dict:
+    v = [ctypes.c_int64() for _ in range(5)]
+    _check(lib().hpccg_info(prob, *[ctypes.byref(x) for x in v]), "hpccg_info")
+    keys = ("nrow_local", "ncol_local", "nnz_local", "nrow_global", "nnz_global")
+    return {k: x.value for k, x in zip(keys, v)}
+
+
+def hpccg_spmv(prob: int, x, y) -> None:
+    _torch_sync()
+    _check(lib().hpccg_spmv(prob, _ptr(x), _ptr(y)), "hpccg_spmv")
+
+
+def hpccg_ddot(ctx: int, n: int, x, y) -> float:
+    _torch_sync()
+    r = ctypes.c_double()
+    _check(lib().hpccg_ddot(ctx, n, _ptr(x), _ptr(y), ctypes.byref(r)), "hpccg_ddot")
+    return r.value
+
+
+def hpccg_waxpby(ctx: int, n: int, alpha: float, x, beta: float, y, w) -> None:
+    _torch_sync()
+    _check(lib().hpccg_waxpby(ctx, n, float(alpha), _ptr(x), float(beta), _ptr(y), _ptr(w)),
+           "hpccg_waxpby")
+
+
+def hpccg_solve(prob: int, max_iter: int, tol: float) -> dict:
+    ni, nr = ctypes.c_int(), ctypes.c_double()
+    times = (ctypes.c_double * 6)()
+    _check(lib().hpccg_solve(prob, max_iter, float(tol), ctypes.byref(ni), ctypes.byref(nr),
+                             times), "hpccg_solve")
+    return {"niters": ni.value, "normr": nr.value, "times": list(times)}
+
+
+def hpccg_get_stats(prob: int) -> dict:
+    s = hpccg_stats()
+    _check(lib().hpccg_get_stats(prob, ctypes.byref(s)), "hpccg_get_stats")
+    return s.as_dict()
+
+
+def hpccg_maxabsdiff(prob: int) -> float:
+    r = ctypes.c_double()
+    _check(lib().hpccg_maxabsdiff(prob, ctypes.byref(r)), "hpccg_maxabsdiff")
+    return r.value
+
+
+def hpccg_free(prob: int) -> None:
+    lib().hpccg_free(prob)
+
+
+# --------------------------------------------------------------- wrappers
+
+class Context:
+    """A device + stream + communicator (single GPU, NCCL rank, or loopback)."""
+
+    def __init__(self, device: int = 0, stream: int | None = None, rank: int = 0,
+                 nranks: int = 1, unique_id: bytes | None = None, loopback: bool = False):
+        if loopback:
+            self.handle = hpccg_init_loopback(device, stream, nranks)
+        else:
+            self.handle = hpccg_init(device, stream, rank, nranks, unique_id)
+        r, n, s = ctypes.c_int(), ctypes.c_int(), ctypes.c_int()
+        _check(lib().hpccg_ctx_info(self.handle, ctypes.byref(r), ctypes.byref(n),
+                                    ctypes.byref(s)), "hpccg_ctx_info")
+        self.rank, self.nranks, self.nslabs = r.value, n.value, s.value
+
+    def ddot(self, n: int, x, y) -> float:
+        return hpccg_ddot(self.handle, n, x, y)
+
+    def waxpby(self, n: int, alpha: float, x, beta: float, y, w) -> None:
+        hpccg_waxpby(self.handle, n, alpha, x, beta, y, w)
+
+    @property
+    def launch_count(self) -> int:
+        c = ctypes.c_int64()
+        _check(lib().hpccg_launch_count(self.handle, ctypes.byref(c)), "hpccg_launch_count")
+        return c.value
+
+    def close(self):
+        if self.handle:
+            hpccg_finalize(self.handle)
+            self.handle = 0
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
+
+
+class Problem:
+    """One rank's (or, loopback, all ranks') slab of the HPCCG problem."""
+
+    def __init__(self, ctx: Context, nx: int, ny: int, nz: int):
+        self.ctx = ctx
+        self.nx, self.ny, self.nz = nx, ny, nz
+        self.handle = hpccg_generate(ctx.handle, nx, ny, nz)
+        self.info = hpccg_info(self.handle)
+
+    @property
+    def n(self) -> int:
+        return self.info["nrow_local"]
+
+    @property
+    def ncol(self) -> int:
+        return self.info["ncol_local"]
+
+    def set_option(self, key: int, value: int) -> None:
+        _check(lib().hpccg_set_option(self.handle, key, int(value)), "hpccg_set_option")
+
+    def spmv(self, x, y) -> None:
+        hpccg_spmv(self.handle, x, y)
+
+    def solve(self, max_iter: int, tol: float) -> dict:
+        return hpccg_solve(self.handle, max_iter, tol)
+
+    def stats(self) -> dict:
+        return hpccg_get_stats(self.handle)
+
+    def maxabsdiff(self) -> float:
+        return hpccg_maxabsdiff(self.handle)
+
+    def get_vec(self, which: int, out: np.ndarray | None = None) -> np.ndarray:
+        """Host copy (nslabs * n doubles).  `out` may be a pinned buffer."""
+        if out is None:
+            out = np.empty(self.ctx.nslabs * self.n, dtype=np.float64)
+        assert out.dtype == np.float64 and out.flags.c_contiguous
+        assert out.size >= self.ctx.nslabs * self.n
+        _check(lib().hpccg_get_vec(self.handle, which, out.ctypes.data), "hpccg_get_vec")
+        return out
+
+    def set_vec(self, which: int, src: np.ndarray) -> None:
+        src = np.ascontiguousarray(src, dtype=np.float64)
+        assert src.size >= self.ctx.nslabs * self.n
+        _check(lib().hpccg_set_vec(self.handle, which, src.ctypes.data), "hpccg_set_vec")
+
+    def get_vec_ptr(self, which: int, host_ptr: int) -> None:
+        _check(lib().hpccg_get_vec(self.handle, which, host_ptr), "hpccg_get_vec")
+
+    def set_vec_ptr(self, which: int, host_ptr: int) -> None:
+        _check(lib().hpccg_set_vec(self.handle, which, host_ptr), "hpccg_set_vec")
+
+    def vec_ptr(self, which: int) -> int:
+        h = _vp()
+        _check(lib().hpccg_vec(self.handle, which, ctypes.byref(h)), "hpccg_vec")
+        return h.value
+
+    def copy_matrix(self, slab: int = 0):
+        """(val, col) host arrays, slot-major [27, n]."""
+        n = self.n
+        val = np.empty(27 * n, dtype=np.float64)
+        col = np.empty(27 * n, dtype=np.int32)
+        _check(lib().hpccg_copy_matrix(self.handle, slab, val.ctypes.data, col.ctypes.data),
+               "hpccg_copy_matrix")
+        return val.reshape(27, n), col.reshape(27, n)
+
+    def free(self):
+        if self.handle:
+            hpccg_free(self.handle)
+            self.handle = 0
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.free()

@@ -1,0 +1,329 @@
+"""GPU parity tests (``-m gpu``): the CUDA path through the C-ABI versus the
+CPU oracle, on identical seeded inputs.
+
+Bars (BASELINE.json north_star):
+  generate  bitwise (integer/index work + exact fp64 constants)
+  SpMV      bitwise (canonical ascending-column FMA chain, A8) -- stricter
+            than the north_star's 1e-14 relative
+  waxpby    bitwise (canonical FMA forms, A10)
+  ddot      relative <= 1e-12 vs the compensated oracle (A9); exact on
+            integer inputs
+  CG        niters +-1; final max|x-1| and normr within 1e-10 (A7, A20)
+"""
+import numpy as np
+import pytest
+
+import oracle
+import synth
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+
+from paper_conf_sc_valero_laragmtv24_b200 import hpccg as H  # noqa: E402
+
+DDOT_RTOL = 1e-12
+CG_ATOL = 1e-10
+
+
+@pytest.fixture(scope="module")
+def ctx():
+    c = H.Context(0)
+    yield c
+    c.close()
+
+
+def ell_to_csr(val, col, n, plane, rank):
+    """GPU ELL (slot-major) -> CSR with GLOBAL columns; checks padding."""
+    v, c = val.T, col.T.astype(np.int64)               # n x 27, row-major
+    own = np.arange(n, dtype=np.int64)[:, None] + plane
+    pad = v == 0.0
+    assert np.all(c[pad] == np.broadcast_to(own, c.shape)[pad]), "padding col != own row"
+    keep = ~pad
+    row_ptr = np.concatenate([[0], np.cumsum(keep.sum(1))]).astype(np.int64)
+    cols = c[keep] - plane + rank * n
+    return row_ptr, cols, v[keep]
+
+
+def dev(a):
+    return torch.from_numpy(np.ascontiguousarray(a, dtype=np.float64)).cuda()
+
+
+def halo_vector(xg, n, plane, rank, nranks, fill=0.0):
+    """Local-with-halo slab of a global vector: [lower | owned | upper]."""
+    xl = np.full(n + 2 * plane, fill)
+    lo = rank * n - plane
+    for j in range(n + 2 * plane):
+        g = lo + j
+        if plane <= j < plane + n and 0 <= g < xg.size:
+            xl[j] = xg[g]
+    return xl
+
+
+# ------------------------------------------------------------- generation
+
+@pytest.mark.parametrize("dims", [(20, 30, 10), (7, 5, 6), (1, 1, 1), (2, 3, 1), (33, 9, 3),
+                                  (3, 3, 3)])
+def test_generate_bitwise(ctx, dims):
+    nx, ny, nz = dims
+    with H.Problem(ctx, nx, ny, nz) as p:
+        ref = oracle.generate(nx, ny, nz)
+        assert p.info["nnz_local"] == ref.nnz == p.info["nnz_global"]
+        assert p.info["nrow_local"] == ref.n and p.info["ncol_local"] == ref.n + 2 * nx * ny
+        val, col = p.copy_matrix()
+        rp, cols, vals = ell_to_csr(val, col, p.n, nx * ny, 0)
+        np.testing.assert_array_equal(rp, ref.row_ptr)
+        np.testing.assert_array_equal(cols, ref.cols)
+        np.testing.assert_array_equal(vals, ref.vals)
+        np.testing.assert_array_equal(p.get_vec(H.HPCCG_VEC_B), ref.b)
+        np.testing.assert_array_equal(p.get_vec(H.HPCCG_VEC_X), ref.x)
+        np.testing.assert_array_equal(p.get_vec(H.HPCCG_VEC_XEXACT), ref.xexact)
+
+
+@pytest.mark.parametrize("P", [2, 3, 4])
+def test_generate_loopback_slabs_bitwise(P):
+    nx, ny, nz = 6, 5, 3
+    with H.Context(0, nranks=P, loopback=True) as c, H.Problem(c, nx, ny, nz) as p:
+        assert p.info["nnz_global"] == oracle.generate(nx, ny, nz * P).nnz
+        b = p.get_vec(H.HPCCG_VEC_B)
+        for r in range(P):
+            ref = oracle.generate(nx, ny, nz, r, P)
+            val, col = p.copy_matrix(r)
+            rp, cols, vals = ell_to_csr(val, col, p.n, nx * ny, r)
+            np.testing.assert_array_equal(rp, ref.row_ptr)
+            np.testing.assert_array_equal(cols, ref.cols)
+            np.testing.assert_array_equal(vals, ref.vals)
+            np.testing.assert_array_equal(b[r * p.n:(r + 1) * p.n], ref.b)
+
+
+def test_generate_rejects_bad_sizes(ctx):
+    with pytest.raises(H.HpccgError) as e:
+        H.Problem(ctx, 0, 4, 4)
+    assert e.value.code == H.HPCCG_EINVAL
+
+
+# ------------------------------------------------------------------ SpMV
+
+@pytest.mark.parametrize("dims", [(20, 30, 10), (7, 5, 6), (1, 1, 1), (33, 9, 3), (64, 64, 16)])
+def test_spmv_bitwise_real(ctx, dims):
+    nx, ny, nz = dims
+    with H.Problem(ctx, nx, ny, nz) as p:
+        ref = oracle.generate(nx, ny, nz)
+        x = synth.uniform(ref.n, 21)
+        xl = halo_vector(x, ref.n, nx * ny, 0, 1, fill=np.nan)   # halos overwritten
+        y = torch.empty(ref.n, dtype=torch.float64, device="cuda")
+        p.spmv(dev(xl), y)
+        np.testing.assert_array_equal(y.cpu().numpy(), oracle.spmv(ref, x))
+
+
+def test_spmv_integer_exact_and_ones(ctx):
+    nx, ny, nz = 31, 17, 9        # n = 4743: ragged tail over 256-row blocks
+    with H.Problem(ctx, nx, ny, nz) as p:
+        ref = oracle.generate(nx, ny, nz)
+        y = torch.empty(ref.n, dtype=torch.float64, device="cuda")
+        p.spmv(dev(halo_vector(np.ones(ref.n), ref.n, nx * ny, 0, 1)), y)
+        np.testing.assert_array_equal(y.cpu().numpy(), ref.b)          # A.1 = b
+        x = synth.integers(ref.n, 3, -1000, 1000)
+        p.spmv(dev(halo_vector(x, ref.n, nx * ny, 0, 1)), y)
+        np.testing.assert_array_equal(y.cpu().numpy(), oracle.spmv(ref, x))
+
+
+@pytest.mark.parametrize("P", [2, 3])
+def test_spmv_loopback_halo_exchange(P):
+    """Stacked slab vectors with NaN halos: the exchange must fill them from
+    the neighbours' owned planes; result = global oracle rows, bitwise."""
+    nx, ny, nz = 9, 7, 4
+    with H.Context(0, nranks=P, loopback=True) as c, H.Problem(c, nx, ny, nz) as p:
+        g = oracle.generate(nx, ny, nz * P)
+        xg = synth.uniform(g.n, 33)
+        n, plane = p.n, nx * ny
+        xs = np.concatenate([halo_vector(xg, n, plane, r, P, fill=np.nan) for r in range(P)])
+        y = torch.empty(P * n, dtype=torch.float64, device="cuda")
+        p.spmv(dev(xs), y)
+        np.testing.assert_array_equal(y.cpu().numpy(), oracle.spmv(g, xg))
+
+
+# ------------------------------------------------------------------- ddot
+
+@pytest.mark.parametrize("n", [0, 1, 2, 3, 255, 257, 1000, 65537, 1_000_003])
+def test_ddot_vs_compensated_oracle(ctx, n):
+    x, y = synth.uniform(n, 5), synth.uniform(n, 6)
+    got = ctx.ddot(n, dev(x), dev(y))
+    exp = oracle.ddot(x, y)
+    assert abs(got - exp) <= DDOT_RTOL * max(abs(exp), np.abs(x * y).sum() * 1e-4, 1e-300)
+    gx = ctx.ddot(n, dev(x), dev(x))  # x == x, squared norm (positive terms)
+    ex = oracle.ddot(x, x)
+    assert abs(gx - ex) <= DDOT_RTOL * max(ex, 1e-300)
+
+
+def test_ddot_jacc_integer_exact(ctx):
+    """Fig. 2 inputs: the sum is an integer < 2^53 -> exact."""
+    n = 1_000_000
+    x, y = synth.jacc_vector(n, 42), synth.jacc_vector(n, 43)
+    exact = float(int(np.dot(x.astype(np.int64), y.astype(np.int64))))
+    assert ctx.ddot(n, dev(x), dev(y)) == exact == oracle.ddot(x, y)
+
+
+def test_ddot_misaligned_scalar_path(ctx):
+    n = 4097
+    buf = dev(synth.uniform(n + 1, 8))
+    x = buf[1:]                       # 8-B aligned only -> scalar kernel
+    got = ctx.ddot(n, x.data_ptr(), x.data_ptr())
+    exp = oracle.ddot(buf.cpu().numpy()[1:], buf.cpu().numpy()[1:])
+    assert abs(got - exp) <= DDOT_RTOL * exp
+
+
+def test_ddot_loopback_stacked():
+    P, n = 3, 10001
+    with H.Context(0, nranks=P, loopback=True) as c:
+        x, y = synth.uniform(P * n, 9), synth.uniform(P * n, 10)
+        got = c.ddot(n, dev(x), dev(y))
+        exp = oracle.ddot(x, y)
+        assert abs(got - exp) <= DDOT_RTOL * abs(exp)
+
+
+# ----------------------------------------------------------------- waxpby
+
+@pytest.mark.parametrize("alpha,beta", [(1.0, 0.37), (0.61, 1.0), (0.3, -0.7), (1.0, 0.0),
+                                        (1.0, -1.0)])
+@pytest.mark.parametrize("n", [1, 2, 7, 1000, 100_001])
+def test_waxpby_bitwise(ctx, alpha, beta, n):
+    x, y = synth.uniform(n, 11), synth.uniform(n, 12)
+    w = torch.empty(n, dtype=torch.float64, device="cuda")
+    ctx.waxpby(n, alpha, dev(x), beta, dev(y), w)
+    np.testing.assert_array_equal(w.cpu().numpy(), oracle.waxpby(alpha, x, beta, y))
+
+
+def test_waxpby_jacc_axpy_inplace_and_misaligned(ctx):
+    """JACC AXPY x += 2.5 y in place (aliasing w == x), Fig. 2 inputs; and
+    the scalar path on 8-B-aligned views."""
+    n = 1_000_000
+    x, y = synth.jacc_vector(n, 42), synth.jacc_vector(n, 43)
+    xd, yd = dev(x), dev(y)
+    ctx.waxpby(n, 1.0, xd, 2.5, yd, xd)
+    np.testing.assert_array_equal(xd.cpu().numpy(), oracle.waxpby(1.0, x, 2.5, y))
+    buf = dev(synth.uniform(n + 1, 13))
+    v = buf[1:]
+    out = torch.empty(n + 1, dtype=torch.float64, device="cuda")[1:]
+    ctx.waxpby(n, 0.3, v.data_ptr(), -0.7, v.data_ptr(), out.data_ptr())
+    h = buf.cpu().numpy()[1:]
+    np.testing.assert_array_equal(out.cpu().numpy(), oracle.waxpby(0.3, h, -0.7, h))
+
+
+# --------------------------------------------------------------------- CG
+
+def check_cg(res, err, oref, ref):
+    assert abs(res["niters"] - oref["niters"]) <= 1, (res["niters"], oref["niters"])
+    assert abs(err - oracle.maxabsdiff(oref["x"], ref.xexact)) <= CG_ATOL
+    assert abs(res["normr"] - oref["normr"]) <= CG_ATOL
+
+
+@pytest.mark.parametrize("dims", [(20, 30, 10), (3, 3, 3), (16, 16, 16), (33, 9, 3)])
+def test_cg_vs_oracle(ctx, dims):
+    with H.Problem(ctx, *dims) as p:
+        ref = oracle.generate(*dims)
+        oref = oracle.cg(ref, 150, 1e-12)
+        res = p.solve(150, 1e-12)
+        check_cg(res, p.maxabsdiff(), oref, ref)
+        x = p.get_vec(H.HPCCG_VEC_X)
+        assert np.max(np.abs(x - oref["x"])) <= CG_ATOL
+        if dims == (20, 30, 10):
+            assert res["niters"] == 50       # BASELINE configs[0] anchor
+
+
+def test_cg_modes_bitwise_identical_and_deterministic(ctx):
+    """Graph replay, plain launches and timed launches run the same kernels
+    in the same order: identical bits, run after run."""
+    dims = (24, 20, 12)
+    xs, outs = [], []
+    with H.Problem(ctx, *dims) as p:
+        for graph, timing in [(1, 0), (0, 0), (0, 1), (1, 0)]:
+            p.set_vec(H.HPCCG_VEC_X, np.zeros(p.n))
+            p.set_option(H.HPCCG_OPT_GRAPH, graph)
+            p.set_option(H.HPCCG_OPT_TIMING, timing)
+            r = p.solve(150, 1e-12)
+            outs.append((r["niters"], r["normr"]))
+            xs.append(p.get_vec(H.HPCCG_VEC_X))
+            st = p.stats()
+            assert st["spmv_launches"] == r["niters"] + 1
+            if timing:
+                assert st["spmv_ms"] > 0 and st["update_ms"] > 0 and st["pupdate_ms"] > 0
+    for o, x in zip(outs[1:], xs[1:]):
+        assert o == outs[0]
+        np.testing.assert_array_equal(x, xs[0])
+
+
+def test_cg_first_step_exact(ctx):
+    """x0 = 0: alpha1 = b.b / b.Ab exactly (integers < 2^53), x1 = fl(alpha1 b)."""
+    with H.Problem(ctx, 20, 30, 10) as p:
+        r = p.solve(2, 0.0)
+        assert r["niters"] == 1
+        b = p.get_vec(H.HPCCG_VEC_B)
+        alpha = 236928 / 4056976
+        np.testing.assert_array_equal(p.get_vec(H.HPCCG_VEC_X), alpha * b)
+        assert r["normr"] == np.sqrt(236928.0)
+
+
+def test_cg_max_iter_semantics_and_initial_guess(ctx):
+    with H.Problem(ctx, 8, 8, 8) as p:
+        ref = oracle.generate(8, 8, 8)
+        for m in [1, 2, 10, 37]:
+            p.set_vec(H.HPCCG_VEC_X, np.zeros(p.n))
+            r = p.solve(m, 0.0)
+            o = oracle.cg(ref, m, 0.0)
+            assert r["niters"] == o["niters"] == m - 1
+            assert abs(r["normr"] - o["normr"]) <= CG_ATOL
+        p.set_vec(H.HPCCG_VEC_X, np.ones(p.n))       # start at the solution
+        r = p.solve(50, 1e-12)
+        assert r["niters"] == 0 and r["normr"] == 0.0
+
+
+@pytest.mark.parametrize("dims", [(1, 1, 1), (2, 2, 2), (4, 1, 1)])
+def test_cg_degenerate_guard(ctx, dims):
+    """A11: exact convergence with tol = 0 must not produce NaN."""
+    with H.Problem(ctx, *dims) as p:
+        r = p.solve(60, 0.0)
+        x = p.get_vec(H.HPCCG_VEC_X)
+        assert np.all(np.isfinite(x)) and p.maxabsdiff() < 1e-14
+        assert r["niters"] < 59
+
+
+@pytest.mark.parametrize("P", [2, 4])
+def test_cg_loopback_matches_global_oracle(P):
+    """Chimney decomposition (A13, A20): P slabs solve the same global
+    problem -- niters +-1, x and normr within 1e-10 of the oracle."""
+    nx, ny, nz = 16, 12, 6
+    with H.Context(0, nranks=P, loopback=True) as c, H.Problem(c, nx, ny, nz) as p:
+        ref = oracle.generate(nx, ny, nz * P)
+        oref = oracle.cg(ref, 150, 1e-12)
+        res = p.solve(150, 1e-12)
+        check_cg(res, p.maxabsdiff(), oref, ref)
+        assert np.max(np.abs(p.get_vec(H.HPCCG_VEC_X) - oref["x"])) <= CG_ATOL
+
+
+# ------------------------------------------- full sizes (bench launch config)
+
+def test_full_128cubed_sampled_spmv_and_solve(ctx):
+    """BASELINE configs[1] (128^3): sampled SpMV rows bitwise vs the oracle's
+    row-at-a-time evaluation; CG to tol 1e-12 vs the full oracle CG (niters
+    +-1, 1e-10); the bench's 500-iteration tol-0 run stays at the solution."""
+    nx = ny = nz = 128
+    with H.Problem(ctx, nx, ny, nz) as p:
+        n, plane = p.n, nx * ny
+        assert p.info["nnz_global"] == (3 * 128 - 2) ** 3
+        x = synth.uniform(n, 77)
+        xl = np.zeros(n + 2 * plane)
+        xl[plane:plane + n] = x
+        y = torch.empty(n, dtype=torch.float64, device="cuda")
+        p.spmv(dev(xl), y)
+        rows = synth.sample_rows(n, 2000, 5)
+        np.testing.assert_array_equal(y.cpu().numpy()[rows],
+                                      oracle.spmv_rows(nx, ny, nz, rows, x))
+        res = p.solve(150, 1e-12)
+        ref = oracle.generate(nx, ny, nz)
+        oref = oracle.cg(ref, 150, 1e-12)
+        check_cg(res, p.maxabsdiff(), oref, ref)
+        p.set_vec(H.HPCCG_VEC_X, np.zeros(n))
+        r500 = p.solve(501, 0.0)
+        assert r500["niters"] == 500
+        assert p.maxabsdiff() < 1e-13 and 0 <= r500["normr"] < 1e-40
