@@ -37,11 +37,12 @@ sys.path.insert(0, ROOT)
 
 METRIC = "HPCCG CG GFLOP/s and SpMV HBM GB/s (fp64) at 1/2/4/8 B200 vs HBM roofline"
 WORKLOADS = {
-    # name: (nx, ny, nz per GPU, CG iterations, BASELINE config index)
-    "hpccg128": (128, 128, 128, 500, 1),
-    "hpccg20": (20, 30, 10, 149, 0),
-    "hpccg256": (256, 256, 256, 200, 2),
-    "hpccg512s": (512, 512, 512, 200, 3),
+    # name: (nx, ny, nz, CG iterations, BASELINE config index, scaling)
+    # weak: nz planes per GPU; strong: nz global planes split over the GPUs
+    "hpccg128": (128, 128, 128, 500, 1, "weak"),
+    "hpccg20": (20, 30, 10, 149, 0, "weak"),
+    "hpccg256": (256, 256, 256, 200, 2, "weak"),
+    "hpccg512s": (512, 512, 512, 200, 3, "strong"),
 }
 FALLBACK_HBM_GBS = 6650.0  # B200_PROFILING.md fallback, used only without MEASURED_PEAKS.json
 
@@ -168,11 +169,12 @@ def run_reference(args, nx, ny, nz, iters, cfg_index):
 
 # -------------------------------------------------------------------- ours
 
-def run_ours(args, nx, ny, nz, iters, cfg_index):
+def run_ours(args, nx, ny, nz, iters, cfg_index, scaling):
     import numpy as np
     import torch
     import torch.distributed as dist
 
+    from paper_conf_sc_valero_laragmtv24_b200 import dist as D
     from paper_conf_sc_valero_laragmtv24_b200 import hpccg as H
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -183,12 +185,12 @@ def run_ours(args, nx, ny, nz, iters, cfg_index):
     if not torch.cuda.is_available():
         raise SystemExit("bench.py needs a CUDA device (no CPU fallback)")
     torch.cuda.set_device(local)
+    slab = D.slab_for(nx, ny, nz, rank, world, scaling)
+    nz = slab.nz
     uid = None
     if world > 1:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-        obj = [H.hpccg_unique_id() if rank == 0 else None]
-        dist.broadcast_object_list(obj, src=0)
-        uid = obj[0]
+        uid = D.broadcast_unique_id(H.hpccg_unique_id)
 
     stream = torch.cuda.Stream()
     ctx = H.Context(local, stream=stream.cuda_stream, rank=rank, nranks=world, unique_id=uid)
@@ -235,14 +237,8 @@ def run_ours(args, nx, ny, nz, iters, cfg_index):
         barrier()
     launches = ctx.launch_count - l0
     ms = t0.elapsed_time(t1)
-    tmax = torch.tensor([ms], dtype=torch.float64, device="cuda")
-    flops_local = torch.tensor([cg_flops(niters_tot, nnz_local, n)], dtype=torch.float64,
-                               device="cuda")
-    if world > 1:
-        dist.all_reduce(tmax, op=dist.ReduceOp.MAX)
-        dist.all_reduce(flops_local, op=dist.ReduceOp.SUM)
-    ms_max = float(tmax.item())
-    value = float(flops_local.item()) / (ms_max * 1e-3) * 1e-9
+    ms_max, flops = D.max_time_sum_work(ms, cg_flops(niters_tot, nnz_local, n), "cuda")
+    value = flops / (ms_max * 1e-3) * 1e-9
 
     # ---- e2e: public API with host buffers (pinned) each step
     h_x0 = torch.zeros(n, dtype=torch.float64).pin_memory()
@@ -264,12 +260,8 @@ def run_ours(args, nx, ny, nz, iters, cfg_index):
         ni_e2e += r_e["niters"]
     t1.record(stream)
     barrier()
-    te = torch.tensor([t0.elapsed_time(t1)], dtype=torch.float64, device="cuda")
-    fe = torch.tensor([cg_flops(ni_e2e, nnz_local, n)], dtype=torch.float64, device="cuda")
-    if world > 1:
-        dist.all_reduce(te, op=dist.ReduceOp.MAX)
-        dist.all_reduce(fe, op=dist.ReduceOp.SUM)
-    e2e_value = float(fe.item()) / (float(te.item()) * 1e-3) * 1e-9
+    te, fe = D.max_time_sum_work(t0.elapsed_time(t1), cg_flops(ni_e2e, nnz_local, n), "cuda")
+    e2e_value = fe / (te * 1e-3) * 1e-9
     x_host_err = float(np.max(np.abs(h_x.numpy() - 1.0)))
 
     if rank == 0:
@@ -298,7 +290,7 @@ def run_ours(args, nx, ny, nz, iters, cfg_index):
         line = {
             "metric": METRIC, "value": round(value, 3), "unit": "GFLOP/s", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms_max / args.steps, 4),
-            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+            "higher_is_better": True, "scaling": scaling, "vs_baseline": None, "dtype": "f64",
             "data": "synthetic (HPCCG 27-point problem generated on device, b = A.1)",
             "config": {"workload": args.workload, "baseline_config": cfg_index,
                        "nx": nx, "ny": ny, "nz_per_gpu": nz, "iters": iters,
@@ -352,12 +344,14 @@ def main():
     args = ap.parse_args()
     if args.warmup < 3:
         raise SystemExit("--warmup must be >= 3")
-    nx, ny, nz, iters, cfg = WORKLOADS[args.workload]
+    nx, ny, nz, iters, cfg, scaling = WORKLOADS[args.workload]
     if args.iters:
         iters = args.iters
     if args.impl == "reference":
+        if scaling == "strong":
+            nz = nz // args.gpus
         return run_reference(args, nx, ny, nz, iters, cfg)
-    return run_ours(args, nx, ny, nz, iters, cfg)
+    return run_ours(args, nx, ny, nz, iters, cfg, scaling)
 
 
 if __name__ == "__main__":

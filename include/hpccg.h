@@ -69,6 +69,11 @@ extern "C" {
                                when tol > 0 (default 8); 0 = never poll */
 #define HPCCG_OPT_TIMING 2  /* 1: CUDA-event time every phase of every iteration into
                                hpccg_get_stats / times[] (disables the graph); default 0 */
+#define HPCCG_OPT_SPMV_MINB 3 /* SpMV register budget: min resident 256-thread blocks per
+                               SM (1..4; 0 = tuned default) -- a tuning knob */
+#define HPCCG_OPT_WHILE 4   /* 1 (default): with GRAPH, run the whole solve as one graph
+                               with a device-driven conditional WHILE node (single GPU /
+                               loopback); 0: replay a per-iteration graph with host polls */
 
 typedef struct hpccg_ctx hpccg_ctx;         /* device, streams, comm (rank, nranks) */
 typedef struct hpccg_problem hpccg_problem; /* A (ELL-27), b, x, x_exact, CG work vectors */

@@ -10,6 +10,7 @@
 
 #include <algorithm>
 #include <string>
+#include <unordered_map>
 #include <vector>
 
 #include "hpccg.h"
@@ -54,11 +55,11 @@ enum Phase { PH_PUPDATE = 0, PH_SPMV, PH_UPDATE, PH_ALLREDUCE, PH_EXCHANGE, PH_N
 
 int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
 
-// Grid of the streaming kernels: enough 256-thread blocks to cover n (in
-// elements per thread), capped at 8 resident blocks on each of the 148 SMs.
-int stream_grid(int64_t work) {
+// Blocks needed for `work` thread-units, capped at one resident wave
+// (SM count x blocks per SM from the occupancy calculator).
+int wave_grid(int64_t work, int wave) {
     int64_t b = cdiv(std::max<int64_t>(work, 1), kBlock);
-    return (int)std::min<int64_t>(b, 148 * 8);
+    return (int)std::max<int64_t>(1, std::min<int64_t>(b, wave));
 }
 
 bool aligned16(const void *p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
@@ -86,6 +87,8 @@ struct hpccg_ctx {
     int64_t red_cap = 0;
     double *h_pinned = nullptr;          // 8 doubles, pinned
     int64_t launches = 0;
+    int num_sms = 148;
+    std::unordered_map<const void *, int> occ;  // kernel -> resident blocks / SM
 };
 
 struct Slab {
@@ -113,10 +116,17 @@ struct hpccg_problem {
     // loopback allreduce tables (device arrays of device pointers)
     double **d_tab = nullptr;  // [6][nslabs]: src pAp, dst pAp, src rr, dst rr, src red, dst red
     // options
-    int opt_graph = 1, opt_poll = 8, opt_timing = 0;
-    // graph of one CG iteration
+    int opt_graph = 1, opt_poll = 8, opt_timing = 0, opt_minb = 0, opt_while = 1;
+    // graph of one CG iteration (per-iteration replay) ...
     cudaGraphExec_t graph = nullptr;
     int64_t graph_kernels = 0;
+    // ... or of the whole solve: init + while(!done) { iteration }
+    cudaGraphExec_t wgraph = nullptr;
+    cudaGraphConditionalHandle whandle = 0;
+    int wgraph_max_iter = -1;
+    double wgraph_tol = -1.0;
+    int64_t wgraph_init_kernels = 0, wgraph_body_kernels = 0;
+    bool while_failed = false;
     // timing
     std::vector<cudaEvent_t> ev_pool;
     size_t ev_used = 0;
@@ -149,6 +159,21 @@ int check_launch(hpccg_ctx *ctx, int nkernels = 1) {
     if (e != cudaSuccess) return fail(HPCCG_ECUDA, "kernel launch failed: %s", cudaGetErrorString(e));
     ctx->launches += nkernels;
     return HPCCG_OK;
+}
+
+template <class K>
+int wave(hpccg_ctx *ctx, K kernel) {
+    const void *key = reinterpret_cast<const void *>(kernel);
+    auto it = ctx->occ.find(key);
+    if (it != ctx->occ.end()) return it->second;
+    int b = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, kernel, kBlock, 0) != cudaSuccess || b < 1) {
+        cudaGetLastError();
+        b = 1;
+    }
+    const int w = b * ctx->num_sms;
+    ctx->occ[key] = w;
+    return w;
 }
 
 // --------------------------------------------------------------- timing
@@ -256,6 +281,9 @@ int exchange(hpccg_problem *p, double *const *xs, cudaStream_t on) {
 }
 
 // ------------------------------------------------------------- launchers
+// `check`: kernels test the device `done` flag first (plain launches and the
+// per-iteration graph, which may run past convergence).  The while-graph
+// never does, so its kernels skip that dependent load.
 
 SpmvArgs spmv_args(const Slab &s, const double *x, double *y) {
     SpmvArgs a{};
@@ -270,9 +298,23 @@ SpmvArgs spmv_args(const Slab &s, const double *x, double *y) {
     return a;
 }
 
+// kMinB of the SpMV (register budget): tuned on B200, see DESIGN.md sec. 7.
+constexpr int kSpmvMinBDefault = 2;
+
+template <bool kDot, bool kCheck>
+int launch_spmv_t(hpccg_ctx *ctx, int minb, const SpmvArgs &a, unsigned blocks, cudaStream_t st) {
+    switch (minb) {
+        case 1: spmv27_kernel<kDot, kCheck, 1><<<blocks, kBlock, 0, st>>>(a); break;
+        case 3: spmv27_kernel<kDot, kCheck, 3><<<blocks, kBlock, 0, st>>>(a); break;
+        case 4: spmv27_kernel<kDot, kCheck, 4><<<blocks, kBlock, 0, st>>>(a); break;
+        default: spmv27_kernel<kDot, kCheck, 2><<<blocks, kBlock, 0, st>>>(a); break;
+    }
+    return check_launch(ctx);
+}
+
 template <bool kDot>
-int launch_spmv(hpccg_ctx *ctx, SpmvArgs a, int64_t r0, int64_t len0, int64_t r1, int64_t len1,
-                cudaStream_t st) {
+int launch_spmv(hpccg_ctx *ctx, int minb, bool check, SpmvArgs a, int64_t r0, int64_t len0,
+                int64_t r1, int64_t len1, cudaStream_t st) {
     a.r0 = r0;
     a.len0 = len0;
     a.r1 = r1;
@@ -281,27 +323,42 @@ int launch_spmv(hpccg_ctx *ctx, SpmvArgs a, int64_t r0, int64_t len0, int64_t r1
     const int64_t blocks = a.nb0 + cdiv(len1, kBlock);
     if (blocks == 0) return HPCCG_OK;
     if (blocks > 0x7fffffffLL) return fail(HPCCG_EINVAL, "SpMV grid too large");
-    spmv27_kernel<kDot><<<(unsigned)blocks, kBlock, 0, st>>>(a);
-    return check_launch(ctx);
+    if (minb <= 0) minb = kSpmvMinBDefault;
+    return check ? launch_spmv_t<kDot, true>(ctx, minb, a, (unsigned)blocks, st)
+                 : launch_spmv_t<kDot, false>(ctx, minb, a, (unsigned)blocks, st);
 }
 
 // y = A x for one slab over all rows (no dot).
-int spmv_plain(hpccg_ctx *ctx, const Slab &s, const double *x, double *y, cudaStream_t st) {
-    return launch_spmv<false>(ctx, spmv_args(s, x, y), 0, s.n, 0, 0, st);
+int spmv_plain(hpccg_ctx *ctx, int minb, const Slab &s, const double *x, double *y,
+               cudaStream_t st) {
+    return launch_spmv<false>(ctx, minb, false, spmv_args(s, x, y), 0, s.n, 0, 0, st);
 }
 
-int launch_pupdate(hpccg_ctx *ctx, const Slab &s) {
-    double *po = s.p + s.plane;
-    const bool vec = aligned16(s.r) && aligned16(po);
-    const int g = stream_grid(vec ? s.n / 2 : s.n);
-    if (vec)
-        cg_pupdate_kernel<true><<<g, kBlock, 0, ctx->stream>>>(s.n, s.r, po, s.sc);
-    else
-        cg_pupdate_kernel<false><<<g, kBlock, 0, ctx->stream>>>(s.n, s.r, po, s.sc);
+template <bool kVec, bool kCheck>
+int launch_pupdate_t(hpccg_ctx *ctx, const Slab &s, double *po) {
+    auto k = cg_pupdate_kernel<kVec, kCheck>;
+    const int g = wave_grid(kVec ? cdiv(s.n, 4) : s.n, wave(ctx, k));
+    k<<<g, kBlock, 0, ctx->stream>>>(s.n, s.r, po, s.sc);
     return check_launch(ctx);
 }
 
-int launch_update(hpccg_ctx *ctx, const Slab &s, int single) {
+int launch_pupdate(hpccg_ctx *ctx, const Slab &s, bool check) {
+    double *po = s.p + s.plane;
+    const bool vec = aligned16(s.r) && aligned16(po);
+    if (vec) return check ? launch_pupdate_t<true, true>(ctx, s, po) : launch_pupdate_t<true, false>(ctx, s, po);
+    return check ? launch_pupdate_t<false, true>(ctx, s, po) : launch_pupdate_t<false, false>(ctx, s, po);
+}
+
+template <bool kVec, bool kCheck>
+int launch_update_t(hpccg_ctx *ctx, const UpdArgs &a) {
+    auto k = cg_update_kernel<kVec, kCheck>;
+    const int g = wave_grid(kVec ? cdiv(a.n, 4) : a.n, wave(ctx, k));
+    k<<<g, kBlock, 0, ctx->stream>>>(a);
+    return check_launch(ctx);
+}
+
+int launch_update(hpccg_ctx *ctx, const Slab &s, int single, bool check,
+                  unsigned long long cond) {
     UpdArgs a{};
     a.n = s.n;
     a.x = s.x;
@@ -311,29 +368,26 @@ int launch_update(hpccg_ctx *ctx, const Slab &s, int single) {
     a.sc = s.sc;
     a.red = s.red;
     a.single = single;
+    a.cond = cond;
     const bool vec = aligned16(a.x) && aligned16(a.r) && aligned16(a.p) && aligned16(a.Ap);
-    const int g = stream_grid(vec ? s.n / 2 : s.n);
-    if (vec)
-        cg_update_kernel<true><<<g, kBlock, 0, ctx->stream>>>(a);
-    else
-        cg_update_kernel<false><<<g, kBlock, 0, ctx->stream>>>(a);
-    return check_launch(ctx);
+    if (vec) return check ? launch_update_t<true, true>(ctx, a) : launch_update_t<true, false>(ctx, a);
+    return check ? launch_update_t<false, true>(ctx, a) : launch_update_t<false, false>(ctx, a);
 }
 
 // CG SpMV of every slab with the p.Ap epilogue.  Multi-slab: the rows that
 // do not touch a halo plane (interior) run first, overlapped with the halo
 // exchange on the comm stream (NCCL), then the two boundary planes.
-int cg_spmv_all(hpccg_problem *p, bool timing) {
+int cg_spmv_all(hpccg_problem *p, bool timing, bool check) {
     hpccg_ctx *ctx = p->ctx;
-    const bool single = ctx->mode == MODE_SINGLE;
-    if (single) {
+    const int minb = p->opt_minb;
+    if (ctx->mode == MODE_SINGLE) {
         const Slab &s = p->slabs[0];
         PhaseTimer t(p, ctx->stream, PH_SPMV, timing);
         SpmvArgs a = spmv_args(s, s.p, s.Ap);
         a.single = 1;
         a.part_base = 0;
         a.total_blocks = (unsigned)cdiv(s.n, kBlock);
-        return launch_spmv<true>(ctx, a, 0, s.n, 0, 0, ctx->stream);
+        return launch_spmv<true>(ctx, minb, check, a, 0, s.n, 0, 0, ctx->stream);
     }
     const Slab &s0 = p->slabs[0];
     const int64_t n = s0.n, plane = s0.plane;
@@ -360,10 +414,10 @@ int cg_spmv_all(hpccg_problem *p, bool timing) {
         a.single = 0;
         a.total_blocks = nb_int + nb_bnd;
         a.part_base = 0;
-        CHECK(launch_spmv<true>(ctx, a, int_r0, int_len, 0, 0, ctx->stream));
+        CHECK(launch_spmv<true>(ctx, minb, check, a, int_r0, int_len, 0, 0, ctx->stream));
         CU(cudaStreamWaitEvent(ctx->stream, ctx->ev_join, 0));
         a.part_base = nb_int;
-        return launch_spmv<true>(ctx, a, 0, b0_len, b1_r0, b1_len, ctx->stream);
+        return launch_spmv<true>(ctx, minb, check, a, 0, b0_len, b1_r0, b1_len, ctx->stream);
     }
     // loopback: exchange, then interior + boundary launches per slab
     {
@@ -376,9 +430,9 @@ int cg_spmv_all(hpccg_problem *p, bool timing) {
         a.single = 0;
         a.total_blocks = nb_int + nb_bnd;
         a.part_base = 0;
-        CHECK(launch_spmv<true>(ctx, a, int_r0, int_len, 0, 0, ctx->stream));
+        CHECK(launch_spmv<true>(ctx, minb, check, a, int_r0, int_len, 0, 0, ctx->stream));
         a.part_base = nb_int;
-        CHECK(launch_spmv<true>(ctx, a, 0, b0_len, b1_r0, b1_len, ctx->stream));
+        CHECK(launch_spmv<true>(ctx, minb, check, a, 0, b0_len, b1_r0, b1_len, ctx->stream));
     }
     return HPCCG_OK;
 }
@@ -395,30 +449,36 @@ int allreduce_cg(hpccg_problem *p, bool rr, bool timing) {
     return allreduce_scalar(ctx, hs, hd, tab(p, rr ? 2 : 0), tab(p, rr ? 3 : 1), false);
 }
 
-// One CG iteration (a.6, a.2, a.3+a.4, a.5, a.8) for every slab.
-int enqueue_iteration(hpccg_problem *p, bool timing) {
+// One CG iteration (a.6, a.2, a.3+a.4, a.5, a.8) for every slab.  `cond`:
+// while-graph condition handle (0 outside the while-graph).
+int enqueue_iteration(hpccg_problem *p, bool timing, bool check, unsigned long long cond) {
     hpccg_ctx *ctx = p->ctx;
     const int single = ctx->mode == MODE_SINGLE;
     {
         PhaseTimer t(p, ctx->stream, PH_PUPDATE, timing);
-        for (const Slab &s : p->slabs) CHECK(launch_pupdate(ctx, s));
+        for (const Slab &s : p->slabs) CHECK(launch_pupdate(ctx, s, check));
     }
-    CHECK(cg_spmv_all(p, timing));
+    CHECK(cg_spmv_all(p, timing, check));
     CHECK(allreduce_cg(p, false, timing));
     {
         PhaseTimer t(p, ctx->stream, PH_UPDATE, timing);
-        for (const Slab &s : p->slabs) CHECK(launch_update(ctx, s, single));
+        // every slab computes the same (allreduced) decision; slab 0 drives the
+        // while-graph condition
+        for (size_t i = 0; i < p->slabs.size(); ++i)
+            CHECK(launch_update(ctx, p->slabs[i], single, check, i == 0 ? cond : 0ull));
     }
     CHECK(allreduce_cg(p, true, timing));
     return HPCCG_OK;
 }
 
 // a.7: p = x; halo; Ap = A p; r = b - Ap; rtrans = r.r; normr; first check.
-int enqueue_init(hpccg_problem *p, int max_iter, double tol, bool timing) {
+int enqueue_init(hpccg_problem *p, int max_iter, double tol, bool timing,
+                 unsigned long long cond) {
     hpccg_ctx *ctx = p->ctx;
     const int single = ctx->mode == MODE_SINGLE;
     for (const Slab &s : p->slabs) {
-        copy_kernel<<<stream_grid(s.n), kBlock, 0, ctx->stream>>>(s.n, s.x, s.p + s.plane);
+        copy_kernel<<<wave_grid(s.n, wave(ctx, copy_kernel)), kBlock, 0, ctx->stream>>>(
+            s.n, s.x, s.p + s.plane);
         CHECK(check_launch(ctx));
     }
     std::vector<double *> xs(p->slabs.size());
@@ -429,7 +489,7 @@ int enqueue_init(hpccg_problem *p, int max_iter, double tol, bool timing) {
     }
     {
         PhaseTimer t(p, ctx->stream, PH_SPMV, timing);
-        for (const Slab &s : p->slabs) CHECK(spmv_plain(ctx, s, s.p, s.Ap, ctx->stream));
+        for (const Slab &s : p->slabs) CHECK(spmv_plain(ctx, p->opt_minb, s, s.p, s.Ap, ctx->stream));
     }
     {
         PhaseTimer t(p, ctx->stream, PH_UPDATE, timing);
@@ -442,13 +502,15 @@ int enqueue_init(hpccg_problem *p, int max_iter, double tol, bool timing) {
             a.sc = s.sc;
             a.red = s.red;
             a.single = single;
-            cg_initres_kernel<<<stream_grid(s.n), kBlock, 0, ctx->stream>>>(a);
+            cg_initres_kernel<<<wave_grid(s.n, wave(ctx, cg_initres_kernel)), kBlock, 0,
+                                ctx->stream>>>(a);
             CHECK(check_launch(ctx));
         }
     }
     CHECK(allreduce_cg(p, true, timing));
-    for (const Slab &s : p->slabs) {
-        cg_initstate_kernel<<<1, 1, 0, ctx->stream>>>(s.sc, max_iter, tol);
+    for (size_t i = 0; i < p->slabs.size(); ++i) {
+        cg_initstate_kernel<<<1, 1, 0, ctx->stream>>>(p->slabs[i].sc, max_iter, tol,
+                                                      i == 0 ? cond : 0ull);
         CHECK(check_launch(ctx));
     }
     return HPCCG_OK;
@@ -460,7 +522,7 @@ int build_graph(hpccg_problem *p) {
     cudaGraph_t g = nullptr;
     const int64_t l0 = ctx->launches;
     CU(cudaStreamBeginCapture(ctx->stream, cudaStreamCaptureModeThreadLocal));
-    int rc = enqueue_iteration(p, false);
+    int rc = enqueue_iteration(p, false, true, 0ull);
     cudaError_t e = cudaStreamEndCapture(ctx->stream, &g);
     if (rc != HPCCG_OK) {
         if (g) cudaGraphDestroy(g);
@@ -475,6 +537,80 @@ int build_graph(hpccg_problem *p) {
         p->graph = nullptr;
         return fail(HPCCG_ECUDA, "graph instantiate: %s", cudaGetErrorString(e));
     }
+    return HPCCG_OK;
+}
+
+// The whole solve as ONE graph: init, then a conditional WHILE node whose
+// body is one CG iteration; the update kernel's last block sets the condition
+// (= !done) on the device, so no host round trip until the solve ends.
+// (max_iter, tol) are baked into the init kernel: rebuilt when they change.
+int build_while_graph(hpccg_problem *p, int max_iter, double tol) {
+    hpccg_ctx *ctx = p->ctx;
+    if (p->wgraph && p->wgraph_max_iter == max_iter && p->wgraph_tol == tol) return HPCCG_OK;
+    if (p->wgraph) {
+        cudaGraphExecDestroy(p->wgraph);
+        p->wgraph = nullptr;
+    }
+    cudaGraph_t g = nullptr;
+    CU(cudaGraphCreate(&g, 0));
+    auto bail = [&](int rc) {
+        cudaGraphDestroy(g);
+        return rc;
+    };
+    cudaGraphConditionalHandle h;
+    if (cudaGraphConditionalHandleCreate(&h, g, 0, 0) != cudaSuccess)
+        return bail(fail(HPCCG_ECUDA, "cudaGraphConditionalHandleCreate: %s",
+                         cudaGetErrorString(cudaGetLastError())));
+    const int64_t l0 = ctx->launches;
+    // init, captured into g
+    if (cudaStreamBeginCaptureToGraph(ctx->stream, g, nullptr, nullptr, 0,
+                                      cudaStreamCaptureModeThreadLocal) != cudaSuccess)
+        return bail(fail(HPCCG_ECUDA, "begin capture (init): %s",
+                         cudaGetErrorString(cudaGetLastError())));
+    int rc = enqueue_init(p, max_iter, tol, false, (unsigned long long)h);
+    cudaStreamCaptureStatus cs;
+    const cudaGraphNode_t *deps = nullptr;
+    size_t ndeps = 0;
+    cudaGraph_t cg = nullptr;
+    if (rc == HPCCG_OK &&
+        cudaStreamGetCaptureInfo(ctx->stream, &cs, nullptr, &cg, &deps, &ndeps) != cudaSuccess)
+        rc = fail(HPCCG_ECUDA, "capture info");
+    std::vector<cudaGraphNode_t> tail(deps, deps + ndeps);
+    cudaGraph_t gout = nullptr;
+    cudaError_t e = cudaStreamEndCapture(ctx->stream, &gout);
+    if (rc != HPCCG_OK) return bail(rc);
+    if (e != cudaSuccess) return bail(fail(HPCCG_ECUDA, "end capture (init): %s", cudaGetErrorString(e)));
+    const int64_t l1 = ctx->launches;
+    // while node after the init tail
+    cudaGraphNodeParams cp{};
+    cp.type = cudaGraphNodeTypeConditional;
+    cp.conditional.handle = h;
+    cp.conditional.type = cudaGraphCondTypeWhile;
+    cp.conditional.size = 1;
+    cudaGraphNode_t wnode;
+    e = cudaGraphAddNode(&wnode, g, tail.data(), tail.size(), &cp);
+    if (e != cudaSuccess) return bail(fail(HPCCG_ECUDA, "add while node: %s", cudaGetErrorString(e)));
+    cudaGraph_t body = cp.conditional.phGraph_out[0];
+    if (cudaStreamBeginCaptureToGraph(ctx->stream, body, nullptr, nullptr, 0,
+                                      cudaStreamCaptureModeThreadLocal) != cudaSuccess)
+        return bail(fail(HPCCG_ECUDA, "begin capture (body): %s",
+                         cudaGetErrorString(cudaGetLastError())));
+    rc = enqueue_iteration(p, false, false, (unsigned long long)h);
+    e = cudaStreamEndCapture(ctx->stream, &gout);
+    if (rc != HPCCG_OK) return bail(rc);
+    if (e != cudaSuccess) return bail(fail(HPCCG_ECUDA, "end capture (body): %s", cudaGetErrorString(e)));
+    p->wgraph_init_kernels = l1 - l0;
+    p->wgraph_body_kernels = ctx->launches - l1;
+    ctx->launches = l0;
+    e = cudaGraphInstantiate(&p->wgraph, g, 0);
+    cudaGraphDestroy(g);
+    if (e != cudaSuccess) {
+        p->wgraph = nullptr;
+        return fail(HPCCG_ECUDA, "while-graph instantiate: %s", cudaGetErrorString(e));
+    }
+    p->whandle = h;
+    p->wgraph_max_iter = max_iter;
+    p->wgraph_tol = tol;
     return HPCCG_OK;
 }
 
@@ -508,6 +644,7 @@ void free_slab(Slab &s) {
 int ctx_common_init(hpccg_ctx *c, int device, void *stream) {
     c->device = device;
     CU(cudaSetDevice(device));
+    CU(cudaDeviceGetAttribute(&c->num_sms, cudaDevAttrMultiProcessorCount, device));
     if (stream) {
         c->stream = (cudaStream_t)stream;
     } else {
@@ -876,6 +1013,11 @@ int hpccg_set_option(hpccg_problem *p, int key, int64_t value) {
             p->opt_poll = (int)value;
             return HPCCG_OK;
         case HPCCG_OPT_TIMING: p->opt_timing = value != 0; return HPCCG_OK;
+        case HPCCG_OPT_SPMV_MINB:
+            if (value < 0 || value > 4) return fail(HPCCG_EINVAL, "spmv minb must be 0..4");
+            p->opt_minb = (int)value;
+            return HPCCG_OK;
+        case HPCCG_OPT_WHILE: p->opt_while = value != 0; return HPCCG_OK;
         default: return fail(HPCCG_EINVAL, "unknown option %d", key);
     }
 }
@@ -890,7 +1032,8 @@ int hpccg_spmv(hpccg_problem *p, double *x, double *y) {
     for (size_t i = 0; i < P; ++i) xs[i] = x + i * s0.ncol;
     // halo exchange on the main stream (API call: no overlap needed)
     CHECK(exchange(p, xs.data(), ctx->stream));
-    for (size_t i = 0; i < P; ++i) CHECK(spmv_plain(ctx, p->slabs[i], xs[i], y + i * s0.n, ctx->stream));
+    for (size_t i = 0; i < P; ++i)
+        CHECK(spmv_plain(ctx, p->opt_minb, p->slabs[i], xs[i], y + i * s0.n, ctx->stream));
     CU(cudaStreamSynchronize(ctx->stream));
     return HPCCG_OK;
 }
@@ -901,11 +1044,9 @@ int hpccg_ddot(hpccg_ctx *ctx, int64_t n, const double *x, const double *y, doub
     return api_reduce(ctx, false, result, [&](int s, double *out) {
         const double *xs = x + (size_t)s * n, *ys = y + (size_t)s * n;
         const bool vec = aligned16(xs) && aligned16(ys);
-        const int g = stream_grid(vec ? n / 2 : n);
-        if (vec)
-            dot_kernel<true><<<g, kBlock, 0, ctx->stream>>>(n, xs, ys, ctx->red, out);
-        else
-            dot_kernel<false><<<g, kBlock, 0, ctx->stream>>>(n, xs, ys, ctx->red, out);
+        auto k = vec ? dot_kernel<true> : dot_kernel<false>;
+        const int g = std::min<int>(wave_grid(vec ? cdiv(n, 4) : n, wave(ctx, k)), (int)ctx->red_cap);
+        k<<<g, kBlock, 0, ctx->stream>>>(n, xs, ys, ctx->red, out);
         return check_launch(ctx);
     });
 }
@@ -917,7 +1058,7 @@ int hpccg_waxpby(hpccg_ctx *ctx, int64_t n, double alpha, const double *x, doubl
     const int64_t tot = n * ctx->nslabs;
     if (tot == 0) return HPCCG_OK;
     const bool vec = aligned16(x) && aligned16(y) && aligned16(w);
-    const int g = stream_grid(vec ? tot / 2 : tot);
+    const int g = wave_grid(vec ? cdiv(tot, 4) : tot, wave(ctx, waxpby_kernel<true, 2>));
     const int form = alpha == 1.0 ? 0 : (beta == 1.0 ? 1 : 2);
     cudaStream_t st = ctx->stream;
 #define WAX(V, F) waxpby_kernel<V, F><<<g, kBlock, 0, st>>>(tot, alpha, x, beta, y, w)
@@ -938,7 +1079,8 @@ int hpccg_maxabsdiff(hpccg_problem *p, double *result) {
     CU(cudaSetDevice(ctx->device));
     return api_reduce(ctx, true, result, [&](int s, double *out) {
         const Slab &sl = p->slabs[s];
-        maxabsdiff_kernel<<<stream_grid(sl.n), kBlock, 0, ctx->stream>>>(sl.n, sl.x, sl.xexact,
+        const int g = std::min<int>(wave_grid(sl.n, wave(ctx, maxabsdiff_kernel)), (int)ctx->red_cap);
+        maxabsdiff_kernel<<<g, kBlock, 0, ctx->stream>>>(sl.n, sl.x, sl.xexact,
                                                                          ctx->red, out);
         return check_launch(ctx);
     });
@@ -952,44 +1094,53 @@ int hpccg_solve(hpccg_problem *p, int max_iter, double tol, int *niters, double 
     CU(cudaSetDevice(ctx->device));
     const bool timing = p->opt_timing != 0;
     const bool use_graph = p->opt_graph && !timing;
+    bool use_while = use_graph && p->opt_while && ctx->mode != MODE_NCCL && !p->while_failed;
     p->ev_used = 0;
     p->timed.clear();
     const int64_t l0 = ctx->launches;
-    if (use_graph) CHECK(build_graph(p));
+    if (use_while && build_while_graph(p, max_iter, tol) != HPCCG_OK) {
+        p->while_failed = true;  // keep the message in hpccg_last_error; fall back
+        use_while = false;
+    }
+    if (use_graph && !use_while) CHECK(build_graph(p));
 
     CU(cudaEventRecord(p->ev_t0, ctx->stream));
-    CHECK(enqueue_init(p, max_iter, tol, timing));
-    // at most max_iter - 1 iterations (A4); finished iterations turn the
-    // remaining launches into no-ops on the device (done flag)
-    const int64_t iters = (int64_t)max_iter - 1;
-    const int poll = (tol > 0.0) ? p->opt_poll : 0;
-    const int *d_done = &p->slabs[0].sc->done;
-    int64_t launched = 0;
-    int chunk = 0;
-    bool stop = false;
-    while (launched < iters && !stop) {
-        const int64_t m = poll > 0 ? std::min<int64_t>(poll, iters - launched) : iters - launched;
-        for (int64_t i = 0; i < m; ++i) {
-            if (use_graph) {
-                CU(cudaGraphLaunch(p->graph, ctx->stream));
-                ctx->launches += p->graph_kernels;
-            } else {
-                CHECK(enqueue_iteration(p, timing));
+    if (use_while) {
+        CU(cudaGraphLaunch(p->wgraph, ctx->stream));
+    } else {
+        CHECK(enqueue_init(p, max_iter, tol, timing, 0ull));
+        // at most max_iter - 1 iterations (A4); finished iterations turn the
+        // remaining launches into no-ops on the device (done flag)
+        const int64_t iters = (int64_t)max_iter - 1;
+        const int poll = (tol > 0.0) ? p->opt_poll : 0;
+        const int *d_done = &p->slabs[0].sc->done;
+        int64_t launched = 0;
+        int chunk = 0;
+        bool stop = false;
+        while (launched < iters && !stop) {
+            const int64_t m = poll > 0 ? std::min<int64_t>(poll, iters - launched) : iters - launched;
+            for (int64_t i = 0; i < m; ++i) {
+                if (use_graph) {
+                    CU(cudaGraphLaunch(p->graph, ctx->stream));
+                    ctx->launches += p->graph_kernels;
+                } else {
+                    CHECK(enqueue_iteration(p, timing, true, 0ull));
+                }
             }
-        }
-        launched += m;
-        if (poll > 0 && launched < iters) {
-            // double-buffered poll: queue this chunk's flag copy, then look at
-            // the previous chunk's, so the GPU always has a chunk queued
-            const int slot = chunk & 1;
-            CU(cudaMemcpyAsync(&p->h_done[slot], d_done, sizeof(int), cudaMemcpyDeviceToHost,
-                               ctx->stream));
-            CU(cudaEventRecord(p->ev_poll[slot], ctx->stream));
-            if (chunk > 0) {
-                CU(cudaEventSynchronize(p->ev_poll[slot ^ 1]));
-                if (p->h_done[slot ^ 1]) stop = true;
+            launched += m;
+            if (poll > 0 && launched < iters) {
+                // double-buffered poll: queue this chunk's flag copy, then look at
+                // the previous chunk's, so the GPU always has a chunk queued
+                const int slot = chunk & 1;
+                CU(cudaMemcpyAsync(&p->h_done[slot], d_done, sizeof(int), cudaMemcpyDeviceToHost,
+                                   ctx->stream));
+                CU(cudaEventRecord(p->ev_poll[slot], ctx->stream));
+                if (chunk > 0) {
+                    CU(cudaEventSynchronize(p->ev_poll[slot ^ 1]));
+                    if (p->h_done[slot ^ 1]) stop = true;
+                }
+                ++chunk;
             }
-            ++chunk;
         }
     }
     CU(cudaEventRecord(p->ev_t1, ctx->stream));
@@ -1013,6 +1164,7 @@ int hpccg_solve(hpccg_problem *p, int max_iter, double tol, int *niters, double 
             case PH_EXCHANGE: st.exchange_ms += e; break;
         }
     }
+    if (use_while) ctx->launches += p->wgraph_init_kernels + p->wgraph_body_kernels * hs.niters;
     st.iterations = hs.niters;
     st.spmv_launches = hs.niters + 1;
     st.kernel_launches = ctx->launches - l0;
@@ -1041,6 +1193,7 @@ void hpccg_free(hpccg_problem *p) {
     cudaSetDevice(p->ctx->device);
     cudaStreamSynchronize(p->ctx->stream);
     if (p->graph) cudaGraphExecDestroy(p->graph);
+    if (p->wgraph) cudaGraphExecDestroy(p->wgraph);
     for (Slab &s : p->slabs) free_slab(s);
     cudaFree(p->d_tab);
     for (cudaEvent_t e : p->ev_pool) cudaEventDestroy(e);

@@ -201,9 +201,14 @@ struct SpmvArgs {
     int single;             // 1: write the global pAp directly (no allreduce)
 };
 
-template <bool kDot>
-__global__ void __launch_bounds__(kBlock) spmv27_kernel(SpmvArgs a) {
-    if (kDot && a.sc->done) return;  // uniform over the grid
+// kDot: CG variant with the p.Ap epilogue.  kCheck: return at once when the
+// device `done` flag is set (plain / per-iteration-graph launches; the
+// while-graph never launches past convergence so it skips that load, whose
+// latency would otherwise sit in front of every block's first matrix load).
+// kMinB: __launch_bounds__ min blocks per SM (register budget 65536/(256 kMinB)).
+template <bool kDot, bool kCheck, int kMinB>
+__global__ void __launch_bounds__(kBlock, kMinB) spmv27_kernel(SpmvArgs a) {
+    if (kDot && kCheck && a.sc->done) return;  // uniform over the grid
     int64_t row, lim;
     if ((int64_t)blockIdx.x < a.nb0) {
         row = a.r0 + (int64_t)blockIdx.x * kBlock + threadIdx.x;
@@ -225,10 +230,17 @@ __global__ void __launch_bounds__(kBlock) spmv27_kernel(SpmvArgs a) {
             cc[s] = ld_stream(c + s * a.stride, pol);
         }
         double sum = 0.0;  // FMA chain in ascending column from +0.0 (A8)
+        double xd = 0.0;
 #pragma unroll
-        for (int s = 0; s < kSlots; ++s) sum = fma(vv[s], __ldg(a.x + cc[s]), sum);
+        for (int s = 0; s < kSlots; ++s) {
+            const double xv = __ldg(a.x + cc[s]);
+            if (s == kDiagSlot) xd = xv;
+            sum = fma(vv[s], xv, sum);
+        }
         a.y[row] = sum;
-        if (kDot) d = sum * __ldg(a.x + row + a.plane);
+        // p_i: the diagonal slot's gathered value when that slot really is the
+        // row's own column (always, for generated matrices); else reload it.
+        if (kDot) d = sum * (cc[kDiagSlot] == row + a.plane ? xd : __ldg(a.x + row + a.plane));
     }
     if (kDot) {
         CgScalars *sc = a.sc;
@@ -241,32 +253,41 @@ __global__ void __launch_bounds__(kBlock) spmv27_kernel(SpmvArgs a) {
 }
 
 // ------------------------------------------------ streaming vector kernels
-// Grid-stride loops over 2-element (16 B) vectors when every pointer is
-// 16-B aligned (kVec), scalar otherwise.  The element -> thread mapping is a
-// function of (n, grid) only, so the reductions are run-to-run deterministic.
+// Persistent grids (SM count x resident blocks, sized by the host from the
+// occupancy calculator) walk the vectors in 16-B double2 units, two units per
+// thread per trip with all loads issued before any arithmetic (memory-level
+// parallelism).  Scalar (8-B) path when a pointer is not 16-B aligned.  The
+// element -> thread mapping depends only on (n, grid): reductions are
+// run-to-run deterministic.
+
+__device__ __forceinline__ int64_t gtid() { return (int64_t)blockIdx.x * kBlock + threadIdx.x; }
+__device__ __forceinline__ int64_t gnth() { return (int64_t)gridDim.x * kBlock; }
 
 // a.6: p = r + beta p  (k == 1: p = r)            -- 24n B
-template <bool kVec>
+template <bool kVec, bool kCheck>
 __global__ void __launch_bounds__(kBlock) cg_pupdate_kernel(int64_t n, const double *__restrict__ r,
                                                            double *__restrict__ p,
                                                            const CgScalars *sc) {
-    if (sc->done) return;
+    if (kCheck && sc->done) return;
     const bool first = (sc->k == 1);
     const double beta = first ? 0.0 : sc->rr_cur / sc->rr_prev;
-    const int64_t tid = (int64_t)blockIdx.x * kBlock + threadIdx.x;
-    const int64_t nth = (int64_t)gridDim.x * kBlock;
+    const int64_t tid = gtid(), nth = gnth();
     if (kVec) {
         const int64_t nv = n >> 1;
         const double2 *r2 = reinterpret_cast<const double2 *>(r);
         double2 *p2 = reinterpret_cast<double2 *>(p);
-        for (int64_t i = tid; i < nv; i += nth) {
-            double2 rv = __ldcs(r2 + i);
-            double2 pv = first ? rv : __ldcs(p2 + i);
-            if (!first) {
-                pv.x = fma(beta, pv.x, rv.x);
-                pv.y = fma(beta, pv.y, rv.y);
+        for (int64_t i = tid; i < nv; i += 2 * nth) {
+            const int64_t j = i + nth;
+            const bool hj = j < nv;
+            double2 ra = __ldcs(r2 + i), pa = p2[i], rb = {0, 0}, pb = {0, 0};
+            if (hj) { rb = __ldcs(r2 + j); pb = p2[j]; }
+            if (first) { pa = ra; pb = rb; }
+            else {
+                pa.x = fma(beta, pa.x, ra.x); pa.y = fma(beta, pa.y, ra.y);
+                pb.x = fma(beta, pb.x, rb.x); pb.y = fma(beta, pb.y, rb.y);
             }
-            p2[i] = pv;
+            p2[i] = pa;
+            if (hj) p2[j] = pb;
         }
         if (tid == 0 && (n & 1)) {
             const int64_t i = n - 1;
@@ -278,7 +299,8 @@ __global__ void __launch_bounds__(kBlock) cg_pupdate_kernel(int64_t n, const dou
 }
 
 // a.5: x += alpha p; r -= alpha Ap; partial r.r; then the loop control of
-// the NEXT iteration (A4 lagged check, A11 guard) in the last block.  48n B.
+// the NEXT iteration (A4 lagged check, A11 guard) in the last block, which
+// also drives the while-graph's condition (`cond`, 0 = none).  48n B.
 struct UpdArgs {
     int64_t n;
     double *x, *r;
@@ -286,35 +308,48 @@ struct UpdArgs {
     CgScalars *sc;
     Reduction red;
     int single;
+    unsigned long long cond;  // cudaGraphConditionalHandle or 0
 };
 
-template <bool kVec>
+__device__ __forceinline__ void set_cond(unsigned long long h, int cont) {
+    if (h) cudaGraphSetConditional((cudaGraphConditionalHandle)h, cont ? 1u : 0u);
+}
+
+template <bool kVec, bool kCheck>
 __global__ void __launch_bounds__(kBlock) cg_update_kernel(UpdArgs a) {
     CgScalars *sc = a.sc;
-    if (sc->done) return;
+    if (kCheck && sc->done) return;
     const double rtrans = sc->rr_cur, pAp = sc->pAp;
     const bool stop = (rtrans == 0.0) || (pAp == 0.0);  // A11
     const double alpha = stop ? 0.0 : rtrans / pAp;
-    const int64_t tid = (int64_t)blockIdx.x * kBlock + threadIdx.x;
-    const int64_t nth = (int64_t)gridDim.x * kBlock;
-    double acc = 0.0;
+    const int64_t tid = gtid(), nth = gnth();
+    double acc = 0.0, acc2 = 0.0;
     if (kVec) {
         const int64_t nv = a.n >> 1;
         double2 *x2 = reinterpret_cast<double2 *>(a.x);
         double2 *r2 = reinterpret_cast<double2 *>(a.r);
         const double2 *p2 = reinterpret_cast<const double2 *>(a.p);
         const double2 *q2 = reinterpret_cast<const double2 *>(a.Ap);
-        for (int64_t i = tid; i < nv; i += nth) {
-            double2 xv = x2[i], rv = r2[i];
-            const double2 pv = __ldcs(p2 + i), qv = __ldcs(q2 + i);
-            xv.x = fma(alpha, pv.x, xv.x);
-            xv.y = fma(alpha, pv.y, xv.y);
-            rv.x = fma(-alpha, qv.x, rv.x);
-            rv.y = fma(-alpha, qv.y, rv.y);
-            x2[i] = xv;
-            r2[i] = rv;
-            acc = fma(rv.x, rv.x, acc);
-            acc = fma(rv.y, rv.y, acc);
+        for (int64_t i = tid; i < nv; i += 2 * nth) {
+            const int64_t j = i + nth;
+            const bool hj = j < nv;
+            double2 xa = x2[i], ra = r2[i], pa = __ldcs(p2 + i), qa = __ldcs(q2 + i);
+            double2 xb = {0, 0}, rb = {0, 0}, pb = {0, 0}, qb = {0, 0};
+            if (hj) { xb = x2[j]; rb = r2[j]; pb = __ldcs(p2 + j); qb = __ldcs(q2 + j); }
+            xa.x = fma(alpha, pa.x, xa.x); xa.y = fma(alpha, pa.y, xa.y);
+            ra.x = fma(-alpha, qa.x, ra.x); ra.y = fma(-alpha, qa.y, ra.y);
+            xb.x = fma(alpha, pb.x, xb.x); xb.y = fma(alpha, pb.y, xb.y);
+            rb.x = fma(-alpha, qb.x, rb.x); rb.y = fma(-alpha, qb.y, rb.y);
+            x2[i] = xa;
+            r2[i] = ra;
+            acc = fma(ra.x, ra.x, acc);
+            acc2 = fma(ra.y, ra.y, acc2);
+            if (hj) {
+                x2[j] = xb;
+                r2[j] = rb;
+                acc = fma(rb.x, rb.x, acc);
+                acc2 = fma(rb.y, rb.y, acc2);
+            }
         }
         if (tid == 0 && (a.n & 1)) {
             const int64_t i = a.n - 1;
@@ -323,6 +358,7 @@ __global__ void __launch_bounds__(kBlock) cg_update_kernel(UpdArgs a) {
             a.r[i] = rv;
             acc = fma(rv, rv, acc);
         }
+        acc += acc2;
     } else {
         for (int64_t i = tid; i < a.n; i += nth) {
             a.x[i] = fma(alpha, a.p[i], a.x[i]);
@@ -332,8 +368,9 @@ __global__ void __launch_bounds__(kBlock) cg_update_kernel(UpdArgs a) {
         }
     }
     const int single = a.single;
+    const unsigned long long cond = a.cond;
     grid_reduce<false>(acc, a.red, blockIdx.x, gridDim.x,
-                       [sc, single, rtrans, stop](double s) {
+                       [sc, single, rtrans, stop, cond](double s) {
                            sc->rr_prev = rtrans;
                            if (single) sc->rr_cur = s; else sc->loc_rr = s;
                            const int k = sc->k;
@@ -341,7 +378,9 @@ __global__ void __launch_bounds__(kBlock) cg_update_kernel(UpdArgs a) {
                            sc->normr = normr;
                            sc->niters = k;
                            sc->k = k + 1;
-                           sc->done = stop || !((k + 1) < sc->max_iter && normr > sc->tol);
+                           const int done = stop || !((k + 1) < sc->max_iter && normr > sc->tol);
+                           sc->done = done;
+                           set_cond(cond, !done);
                        });
 }
 
@@ -356,8 +395,7 @@ struct InitResArgs {
 };
 
 __global__ void __launch_bounds__(kBlock) cg_initres_kernel(InitResArgs a) {
-    const int64_t tid = (int64_t)blockIdx.x * kBlock + threadIdx.x;
-    const int64_t nth = (int64_t)gridDim.x * kBlock;
+    const int64_t tid = gtid(), nth = gnth();
     double acc = 0.0;
     for (int64_t i = tid; i < a.n; i += nth) {
         const double rv = fma(-1.0, a.Ap[i], a.b[i]);
@@ -372,7 +410,8 @@ __global__ void __launch_bounds__(kBlock) cg_initres_kernel(InitResArgs a) {
 }
 
 // a.7/a.8: after the (allreduced) initial r.r: k = 1, normr, first check.
-__global__ void cg_initstate_kernel(CgScalars *sc, int max_iter, double tol) {
+__global__ void cg_initstate_kernel(CgScalars *sc, int max_iter, double tol,
+                                    unsigned long long cond) {
     const double rr = sc->rr_cur;
     const double normr = sqrt(rr);
     sc->rr_prev = rr;
@@ -381,7 +420,9 @@ __global__ void cg_initstate_kernel(CgScalars *sc, int max_iter, double tol) {
     sc->max_iter = max_iter;
     sc->k = 1;
     sc->niters = 0;
-    sc->done = !(1 < max_iter && normr > tol);
+    const int done = !(1 < max_iter && normr > tol);
+    sc->done = done;
+    set_cond(cond, !done);
 }
 
 // Loopback allreduce: fixed rank-order sum (or max) of one scalar of every
@@ -401,8 +442,7 @@ __global__ void slab_allreduce_kernel(const double *const *src, double *const *d
 template <bool kVec, int kForm>
 __global__ void __launch_bounds__(kBlock) waxpby_kernel(int64_t n, double alpha, const double *x,
                                                        double beta, const double *y, double *w) {
-    const int64_t tid = (int64_t)blockIdx.x * kBlock + threadIdx.x;
-    const int64_t nth = (int64_t)gridDim.x * kBlock;
+    const int64_t tid = gtid(), nth = gnth();
     auto op = [alpha, beta](double xv, double yv) {
         if (kForm == 0) return fma(beta, yv, xv);
         if (kForm == 1) return fma(alpha, xv, yv);
@@ -413,12 +453,14 @@ __global__ void __launch_bounds__(kBlock) waxpby_kernel(int64_t n, double alpha,
         const double2 *x2 = reinterpret_cast<const double2 *>(x);
         const double2 *y2 = reinterpret_cast<const double2 *>(y);
         double2 *w2 = reinterpret_cast<double2 *>(w);
-        for (int64_t i = tid; i < nv; i += nth) {
-            const double2 xv = x2[i], yv = y2[i];
-            double2 o;
-            o.x = op(xv.x, yv.x);
-            o.y = op(xv.y, yv.y);
-            w2[i] = o;
+        for (int64_t i = tid; i < nv; i += 2 * nth) {
+            const int64_t j = i + nth;
+            const bool hj = j < nv;
+            const double2 xa = x2[i], ya = y2[i];
+            double2 xb = {0, 0}, yb = {0, 0};
+            if (hj) { xb = x2[j]; yb = y2[j]; }
+            w2[i] = make_double2(op(xa.x, ya.x), op(xa.y, ya.y));
+            if (hj) w2[j] = make_double2(op(xb.x, yb.x), op(xb.y, yb.y));
         }
         if (tid == 0 && (n & 1)) w[n - 1] = op(x[n - 1], y[n - 1]);
     } else {
@@ -430,18 +472,23 @@ __global__ void __launch_bounds__(kBlock) waxpby_kernel(int64_t n, double alpha,
 template <bool kVec>
 __global__ void __launch_bounds__(kBlock) dot_kernel(int64_t n, const double *x, const double *y,
                                                     Reduction red, double *out) {
-    const int64_t tid = (int64_t)blockIdx.x * kBlock + threadIdx.x;
-    const int64_t nth = (int64_t)gridDim.x * kBlock;
+    const int64_t tid = gtid(), nth = gnth();
     double acc = 0.0;
     if (kVec) {
         const int64_t nv = n >> 1;
         const double2 *x2 = reinterpret_cast<const double2 *>(x);
         const double2 *y2 = reinterpret_cast<const double2 *>(y);
         double acc2 = 0.0;
-        for (int64_t i = tid; i < nv; i += nth) {
-            const double2 xv = __ldcs(x2 + i), yv = __ldcs(y2 + i);
-            acc = fma(xv.x, yv.x, acc);
-            acc2 = fma(xv.y, yv.y, acc2);
+        for (int64_t i = tid; i < nv; i += 2 * nth) {
+            const int64_t j = i + nth;
+            const bool hj = j < nv;
+            const double2 xa = __ldcs(x2 + i), ya = __ldcs(y2 + i);
+            double2 xb = {0, 0}, yb = {0, 0};
+            if (hj) { xb = __ldcs(x2 + j); yb = __ldcs(y2 + j); }
+            acc = fma(xa.x, ya.x, acc);
+            acc2 = fma(xa.y, ya.y, acc2);
+            acc = fma(xb.x, yb.x, acc);     // zero-padded when j >= nv
+            acc2 = fma(xb.y, yb.y, acc2);
         }
         acc += acc2;
         if (tid == 0 && (n & 1)) acc = fma(x[n - 1], y[n - 1], acc);
@@ -455,8 +502,7 @@ __global__ void __launch_bounds__(kBlock) dot_kernel(int64_t n, const double *x,
 __global__ void __launch_bounds__(kBlock) maxabsdiff_kernel(int64_t n, const double *x,
                                                            const double *xe, Reduction red,
                                                            double *out) {
-    const int64_t tid = (int64_t)blockIdx.x * kBlock + threadIdx.x;
-    const int64_t nth = (int64_t)gridDim.x * kBlock;
+    const int64_t tid = gtid(), nth = gnth();
     double m = 0.0;
     for (int64_t i = tid; i < n; i += nth) m = fmax(m, fabs(x[i] - xe[i]));
     grid_reduce<true>(m, red, blockIdx.x, gridDim.x, [out](double s) { *out = s; });
@@ -464,8 +510,7 @@ __global__ void __launch_bounds__(kBlock) maxabsdiff_kernel(int64_t n, const dou
 
 // p = x for the owned part (init, waxpby(1, x, 0, x, p) = x exactly).
 __global__ void __launch_bounds__(kBlock) copy_kernel(int64_t n, const double *src, double *dst) {
-    const int64_t tid = (int64_t)blockIdx.x * kBlock + threadIdx.x;
-    const int64_t nth = (int64_t)gridDim.x * kBlock;
+    const int64_t tid = gtid(), nth = gnth();
     for (int64_t i = tid; i < n; i += nth) dst[i] = src[i];
 }
 

@@ -1,0 +1,78 @@
+"""Host-side plumbing of the multi-GPU z-slab path (north_star "z-slab
+decomposition across the 8 B200s").
+
+torch.distributed is only the bootstrap: it broadcasts the 128-byte NCCL
+unique id (the library then owns its NCCL communicator, halo exchange and
+scalar allreduces) and aggregates the bench timings (max over ranks).
+"""
+from __future__ import annotations
+
+from dataclasses import dataclass
+
+
+@dataclass(frozen=True)
+class Slab:
+    nx: int
+    ny: int
+    nz: int          # local z-planes of this rank
+    rank: int
+    nranks: int
+
+    @property
+    def n(self) -> int:
+        return self.nx * self.ny * self.nz
+
+    @property
+    def plane(self) -> int:
+        return self.nx * self.ny
+
+    @property
+    def row0(self) -> int:
+        """Global id of the first owned row."""
+        return self.rank * self.n
+
+    @property
+    def col_offset(self) -> int:
+        """Global id of local-with-halo index 0: [lower halo | owned | upper halo]."""
+        return self.row0 - self.plane
+
+    @property
+    def nz_global(self) -> int:
+        return self.nz * self.nranks
+
+
+def slab_for(nx: int, ny: int, nz: int, rank: int, nranks: int, scaling: str) -> Slab:
+    """weak: nz planes per rank (global nz * nranks); strong: the global nz is
+    split evenly (A13: 512^3 -> 512 / P planes per rank)."""
+    if nranks < 1 or not 0 <= rank < nranks:
+        raise ValueError("bad rank / nranks")
+    if scaling == "weak":
+        return Slab(nx, ny, nz, rank, nranks)
+    if scaling == "strong":
+        if nz % nranks:
+            raise ValueError(f"strong scaling needs nz ({nz}) divisible by nranks ({nranks})")
+        return Slab(nx, ny, nz // nranks, rank, nranks)
+    raise ValueError(scaling)
+
+
+def broadcast_unique_id(make_id, src: int = 0) -> bytes:
+    """Rank `src` calls make_id() (hpccg_unique_id); every rank returns it."""
+    import torch.distributed as dist
+    obj = [make_id() if dist.get_rank() == src else None]
+    dist.broadcast_object_list(obj, src=src)
+    uid = obj[0]
+    if not isinstance(uid, (bytes, bytearray)) or len(uid) != 128:
+        raise RuntimeError("bad NCCL unique id from rank %d" % src)
+    return bytes(uid)
+
+
+def max_time_sum_work(ms_local: float, work_local: float, device=None):
+    """(max over ranks of the device time, sum over ranks of the work)."""
+    import torch
+    import torch.distributed as dist
+    t = torch.tensor([ms_local], dtype=torch.float64, device=device)
+    w = torch.tensor([work_local], dtype=torch.float64, device=device)
+    if dist.is_available() and dist.is_initialized() and dist.get_world_size() > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        dist.all_reduce(w, op=dist.ReduceOp.SUM)
+    return float(t.item()), float(w.item())

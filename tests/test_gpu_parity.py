@@ -231,16 +231,20 @@ def test_cg_vs_oracle(ctx, dims):
             assert res["niters"] == 50       # BASELINE configs[0] anchor
 
 
-def test_cg_modes_bitwise_identical_and_deterministic(ctx):
-    """Graph replay, plain launches and timed launches run the same kernels
-    in the same order: identical bits, run after run."""
+@pytest.mark.parametrize("minb", [0, 1, 3, 4])
+def test_cg_modes_bitwise_identical_and_deterministic(ctx, minb):
+    """While-graph, per-iteration graph replay, plain launches and timed
+    launches run the same arithmetic in the same order: identical bits, run
+    after run, for every SpMV register-budget variant."""
     dims = (24, 20, 12)
     xs, outs = [], []
     with H.Problem(ctx, *dims) as p:
-        for graph, timing in [(1, 0), (0, 0), (0, 1), (1, 0)]:
+        p.set_option(H.HPCCG_OPT_SPMV_MINB, minb)
+        for graph, timing, wh in [(1, 0, 1), (1, 0, 0), (0, 0, 0), (0, 1, 0), (1, 0, 1)]:
             p.set_vec(H.HPCCG_VEC_X, np.zeros(p.n))
             p.set_option(H.HPCCG_OPT_GRAPH, graph)
             p.set_option(H.HPCCG_OPT_TIMING, timing)
+            p.set_option(H.HPCCG_OPT_WHILE, wh)
             r = p.solve(150, 1e-12)
             outs.append((r["niters"], r["normr"]))
             xs.append(p.get_vec(H.HPCCG_VEC_X))
@@ -251,6 +255,21 @@ def test_cg_modes_bitwise_identical_and_deterministic(ctx):
     for o, x in zip(outs[1:], xs[1:]):
         assert o == outs[0]
         np.testing.assert_array_equal(x, xs[0])
+
+
+@pytest.mark.parametrize("wh", [0, 1])
+def test_cg_tolerance_stop_in_both_graph_modes(ctx, wh):
+    """tol > 0: the while-graph stops on the device; the per-iteration graph
+    stops via the double-buffered host poll -- same niters / normr / x."""
+    with H.Problem(ctx, 20, 30, 10) as p:
+        p.set_option(H.HPCCG_OPT_WHILE, wh)
+        r = p.solve(150, 1e-12)
+        assert r["niters"] == 50
+        st = p.stats()
+        assert st["iterations"] == 50
+        assert st["kernel_launches"] >= 3 * 50
+        r2 = p.solve(150, 1e-12)      # re-run from the converged x: 0 or few iterations
+        assert r2["niters"] <= 2
 
 
 def test_cg_first_step_exact(ctx):
