@@ -74,6 +74,9 @@ extern "C" {
 #define HPCCG_OPT_WHILE 4   /* 1 (default): with GRAPH, run the whole solve as one graph
                                with a device-driven conditional WHILE node (single GPU /
                                loopback); 0: replay a per-iteration graph with host polls */
+#define HPCCG_OPT_L2_PERSIST 5 /* 1 (default): during hpccg_solve, mark the CG vectors
+                               (r, x, Ap, p) L2-persisting via an access-policy window on
+                               the stream (restored afterwards); 0: off */
 
 typedef struct hpccg_ctx hpccg_ctx;         /* device, streams, comm (rank, nranks) */
 typedef struct hpccg_problem hpccg_problem; /* A (ELL-27), b, x, x_exact, CG work vectors */

@@ -88,6 +88,7 @@ struct hpccg_ctx {
     double *h_pinned = nullptr;          // 8 doubles, pinned
     int64_t launches = 0;
     int num_sms = 148;
+    int max_persist_l2 = 0, max_window = 0;  // bytes (device attributes)
     std::unordered_map<const void *, int> occ;  // kernel -> resident blocks / SM
 };
 
@@ -99,6 +100,10 @@ struct Slab {
     int *col = nullptr;
     double *b = nullptr, *x = nullptr, *xexact = nullptr, *r = nullptr, *Ap = nullptr;
     double *p_alloc = nullptr, *p = nullptr;  // p: local-with-halo base (ncol)
+    // r, x, Ap and p live in one contiguous "arena" so one L2 access-policy
+    // window can keep the CG vectors resident
+    double *arena = nullptr;
+    size_t arena_bytes = 0;
     CgScalars *sc = nullptr;
     Reduction red{};
 };
@@ -116,7 +121,7 @@ struct hpccg_problem {
     // loopback allreduce tables (device arrays of device pointers)
     double **d_tab = nullptr;  // [6][nslabs]: src pAp, dst pAp, src rr, dst rr, src red, dst red
     // options
-    int opt_graph = 1, opt_poll = 8, opt_timing = 0, opt_minb = 0, opt_while = 1;
+    int opt_graph = 1, opt_poll = 8, opt_timing = 0, opt_minb = 0, opt_while = 1, opt_l2 = 1;
     // graph of one CG iteration (per-iteration replay) ...
     cudaGraphExec_t graph = nullptr;
     int64_t graph_kernels = 0;
@@ -299,7 +304,7 @@ SpmvArgs spmv_args(const Slab &s, const double *x, double *y) {
 }
 
 // kMinB of the SpMV (register budget): tuned on B200, see DESIGN.md sec. 7.
-constexpr int kSpmvMinBDefault = 2;
+constexpr int kSpmvMinBDefault = 4;
 
 template <bool kDot, bool kCheck>
 int launch_spmv_t(hpccg_ctx *ctx, int minb, const SpmvArgs &a, unsigned blocks, cudaStream_t st) {
@@ -516,6 +521,46 @@ int enqueue_init(hpccg_problem *p, int max_iter, double tol, bool timing,
     return HPCCG_OK;
 }
 
+// L2 residency of the CG vectors (r, x, Ap, p: 32n B): an access-policy
+// window marks the arena "persisting" while the matrix stream is loaded with
+// an evict_first policy, so at sizes where the vectors fit (<= ~3.9M rows)
+// the vector kernels and the x gathers run out of L2.  Applied to the stream
+// (and so to every kernel captured into a graph) only for the solve.
+struct L2Window {
+    hpccg_problem *p;
+    bool on = false;
+    explicit L2Window(hpccg_problem *p_) : p(p_) {
+        hpccg_ctx *ctx = p->ctx;
+        const Slab &s = p->slabs[0];
+        if (!p->opt_l2 || ctx->max_persist_l2 <= 0 || ctx->max_window <= 0) return;
+        const size_t win = std::min<size_t>(s.arena_bytes, (size_t)ctx->max_window);
+        const size_t keep = std::min<size_t>(win, (size_t)ctx->max_persist_l2);
+        if (cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, keep) != cudaSuccess) {
+            cudaGetLastError();
+            return;
+        }
+        cudaStreamAttrValue v{};
+        v.accessPolicyWindow.base_ptr = s.arena;
+        v.accessPolicyWindow.num_bytes = win;
+        v.accessPolicyWindow.hitRatio = (float)std::min(1.0, (double)keep / (double)win);
+        v.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+        v.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+        if (cudaStreamSetAttribute(ctx->stream, cudaStreamAttributeAccessPolicyWindow, &v) !=
+            cudaSuccess) {
+            cudaGetLastError();
+            return;
+        }
+        on = true;
+    }
+    ~L2Window() {
+        if (!on) return;
+        cudaStreamAttrValue v{};
+        v.accessPolicyWindow.num_bytes = 0;
+        cudaStreamSetAttribute(p->ctx->stream, cudaStreamAttributeAccessPolicyWindow, &v);
+        cudaGetLastError();
+    }
+};
+
 int build_graph(hpccg_problem *p) {
     hpccg_ctx *ctx = p->ctx;
     if (p->graph) return HPCCG_OK;
@@ -630,11 +675,8 @@ void free_slab(Slab &s) {
     cudaFree(s.val);
     cudaFree(s.col);
     cudaFree(s.b);
-    cudaFree(s.x);
     cudaFree(s.xexact);
-    cudaFree(s.r);
-    cudaFree(s.Ap);
-    cudaFree(s.p_alloc);
+    cudaFree(s.arena);
     cudaFree(s.sc);
     cudaFree(s.red.partials);
     cudaFree(s.red.counter);
@@ -645,6 +687,8 @@ int ctx_common_init(hpccg_ctx *c, int device, void *stream) {
     c->device = device;
     CU(cudaSetDevice(device));
     CU(cudaDeviceGetAttribute(&c->num_sms, cudaDevAttrMultiProcessorCount, device));
+    CU(cudaDeviceGetAttribute(&c->max_persist_l2, cudaDevAttrMaxPersistingL2CacheSize, device));
+    CU(cudaDeviceGetAttribute(&c->max_window, cudaDevAttrMaxAccessPolicyWindowSize, device));
     if (stream) {
         c->stream = (cudaStream_t)stream;
     } else {
@@ -847,14 +891,18 @@ int hpccg_generate(hpccg_ctx *ctx, int nx, int ny, int nz, hpccg_problem **out) 
         if ((rc = alloc_zero((void **)&s.val, sizeof(double) * kSlots * n))) return bail(rc);
         if ((rc = alloc_zero((void **)&s.col, sizeof(int) * kSlots * n))) return bail(rc);
         if ((rc = alloc_zero((void **)&s.b, sizeof(double) * n))) return bail(rc);
-        if ((rc = alloc_zero((void **)&s.x, sizeof(double) * n))) return bail(rc);
         if ((rc = alloc_zero((void **)&s.xexact, sizeof(double) * n))) return bail(rc);
-        if ((rc = alloc_zero((void **)&s.r, sizeof(double) * n))) return bail(rc);
-        if ((rc = alloc_zero((void **)&s.Ap, sizeof(double) * n))) return bail(rc);
-        // p: [lower halo | n owned | upper halo]; shift by one element when
+        // arena: [p (ncol + 2) | r | x | Ap], each segment 256-B aligned.
+        // p: [lower halo | n owned | upper halo]; shifted by one element when
         // the plane is odd so the owned part is 16-B aligned (double2 loads).
-        if ((rc = alloc_zero((void **)&s.p_alloc, sizeof(double) * (ncol + 2)))) return bail(rc);
+        const int64_t seg_p = cdiv(ncol + 2, 32) * 32, seg_v = cdiv(n, 32) * 32;
+        s.arena_bytes = sizeof(double) * (size_t)(seg_p + 3 * seg_v);
+        if ((rc = alloc_zero((void **)&s.arena, s.arena_bytes))) return bail(rc);
+        s.p_alloc = s.arena;
         s.p = s.p_alloc + ((plane & 1) ? 1 : 0);
+        s.r = s.arena + seg_p;
+        s.x = s.r + seg_v;
+        s.Ap = s.x + seg_v;
         if ((rc = alloc_zero((void **)&s.sc, sizeof(CgScalars)))) return bail(rc);
         const int64_t parts = cdiv(n, kBlock) + 2 * cdiv(plane, kBlock) + 148 * 8 + 64;
         if ((rc = alloc_zero((void **)&s.red.partials, sizeof(double) * parts))) return bail(rc);
@@ -1006,6 +1054,13 @@ int hpccg_copy_matrix(const hpccg_problem *p, int slab, double *val_host, int32_
 
 int hpccg_set_option(hpccg_problem *p, int key, int64_t value) {
     if (!p) return fail(HPCCG_EINVAL, "NULL problem");
+    // captured graphs bake in the launch configuration: rebuild on change
+    cudaSetDevice(p->ctx->device);
+    if (p->graph) cudaGraphExecDestroy(p->graph);
+    if (p->wgraph) cudaGraphExecDestroy(p->wgraph);
+    p->graph = nullptr;
+    p->wgraph = nullptr;
+    p->while_failed = false;
     switch (key) {
         case HPCCG_OPT_GRAPH: p->opt_graph = value != 0; return HPCCG_OK;
         case HPCCG_OPT_POLL:
@@ -1018,6 +1073,7 @@ int hpccg_set_option(hpccg_problem *p, int key, int64_t value) {
             p->opt_minb = (int)value;
             return HPCCG_OK;
         case HPCCG_OPT_WHILE: p->opt_while = value != 0; return HPCCG_OK;
+        case HPCCG_OPT_L2_PERSIST: p->opt_l2 = value != 0; return HPCCG_OK;
         default: return fail(HPCCG_EINVAL, "unknown option %d", key);
     }
 }
@@ -1098,6 +1154,7 @@ int hpccg_solve(hpccg_problem *p, int max_iter, double tol, int *niters, double 
     p->ev_used = 0;
     p->timed.clear();
     const int64_t l0 = ctx->launches;
+    L2Window l2win(p);
     if (use_while && build_while_graph(p, max_iter, tol) != HPCCG_OK) {
         p->while_failed = true;  // keep the message in hpccg_last_error; fall back
         use_while = false;

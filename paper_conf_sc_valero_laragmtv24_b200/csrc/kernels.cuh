@@ -208,7 +208,6 @@ struct SpmvArgs {
 // kMinB: __launch_bounds__ min blocks per SM (register budget 65536/(256 kMinB)).
 template <bool kDot, bool kCheck, int kMinB>
 __global__ void __launch_bounds__(kBlock, kMinB) spmv27_kernel(SpmvArgs a) {
-    if (kDot && kCheck && a.sc->done) return;  // uniform over the grid
     int64_t row, lim;
     if ((int64_t)blockIdx.x < a.nb0) {
         row = a.r0 + (int64_t)blockIdx.x * kBlock + threadIdx.x;
@@ -218,30 +217,45 @@ __global__ void __launch_bounds__(kBlock, kMinB) spmv27_kernel(SpmvArgs a) {
         lim = a.r1 + a.len1;
     }
     double d = 0.0;
+    // The done flag is read together with the first matrix loads and tested
+    // after them, so its latency never sits in front of the stream.
+    const int done = (kDot && kCheck) ? *(volatile const int *)&a.sc->done : 0;
     if (row < lim) {
         const uint64_t pol = policy_evict_first();
         const double *v = a.val + row;
         const int *c = a.col + row;
-        double vv[kSlots];
-        int cc[kSlots];
-#pragma unroll
-        for (int s = 0; s < kSlots; ++s) {
-            vv[s] = ld_stream(v + s * a.stride, pol);
-            cc[s] = ld_stream(c + s * a.stride, pol);
-        }
         double sum = 0.0;  // FMA chain in ascending column from +0.0 (A8)
         double xd = 0.0;
+        int cd = 0;
+        // three groups of 9 slots (one z-plane of the stencil each); all 18
+        // loads of a group are issued before its gathers and FMAs, and the
+        // compiler may hoist the next group's loads above them
 #pragma unroll
-        for (int s = 0; s < kSlots; ++s) {
-            const double xv = __ldg(a.x + cc[s]);
-            if (s == kDiagSlot) xd = xv;
-            sum = fma(vv[s], xv, sum);
+        for (int g = 0; g < 3; ++g) {
+            double vv[9];
+            int cc[9];
+#pragma unroll
+            for (int t = 0; t < 9; ++t) {
+                vv[t] = ld_stream(v + (9 * g + t) * a.stride, pol);
+                cc[t] = ld_stream(c + (9 * g + t) * a.stride, pol);
+            }
+            if (g == 0 && done) return;  // uniform over the grid, before any store
+#pragma unroll
+            for (int t = 0; t < 9; ++t) {
+                const double xv = __ldg(a.x + cc[t]);
+                if (9 * g + t == kDiagSlot) {
+                    xd = xv;
+                    cd = cc[t];
+                }
+                sum = fma(vv[t], xv, sum);
+            }
         }
         a.y[row] = sum;
         // p_i: the diagonal slot's gathered value when that slot really is the
         // row's own column (always, for generated matrices); else reload it.
-        if (kDot) d = sum * (cc[kDiagSlot] == row + a.plane ? xd : __ldg(a.x + row + a.plane));
+        if (kDot) d = sum * (cd == row + a.plane ? xd : __ldg(a.x + row + a.plane));
     }
+    if (done) return;
     if (kDot) {
         CgScalars *sc = a.sc;
         const int single = a.single;
@@ -268,7 +282,8 @@ template <bool kVec, bool kCheck>
 __global__ void __launch_bounds__(kBlock) cg_pupdate_kernel(int64_t n, const double *__restrict__ r,
                                                            double *__restrict__ p,
                                                            const CgScalars *sc) {
-    if (kCheck && sc->done) return;
+    // `done` is tested after each trip's loads (never in front of them)
+    const int done = kCheck ? *(volatile const int *)&sc->done : 0;
     const bool first = (sc->k == 1);
     const double beta = first ? 0.0 : sc->rr_cur / sc->rr_prev;
     const int64_t tid = gtid(), nth = gnth();
@@ -281,6 +296,7 @@ __global__ void __launch_bounds__(kBlock) cg_pupdate_kernel(int64_t n, const dou
             const bool hj = j < nv;
             double2 ra = __ldcs(r2 + i), pa = p2[i], rb = {0, 0}, pb = {0, 0};
             if (hj) { rb = __ldcs(r2 + j); pb = p2[j]; }
+            if (done) return;
             if (first) { pa = ra; pb = rb; }
             else {
                 pa.x = fma(beta, pa.x, ra.x); pa.y = fma(beta, pa.y, ra.y);
@@ -289,11 +305,13 @@ __global__ void __launch_bounds__(kBlock) cg_pupdate_kernel(int64_t n, const dou
             p2[i] = pa;
             if (hj) p2[j] = pb;
         }
+        if (done) return;
         if (tid == 0 && (n & 1)) {
             const int64_t i = n - 1;
             p[i] = first ? r[i] : fma(beta, p[i], r[i]);
         }
     } else {
+        if (done) return;
         for (int64_t i = tid; i < n; i += nth) p[i] = first ? r[i] : fma(beta, p[i], r[i]);
     }
 }
@@ -318,7 +336,9 @@ __device__ __forceinline__ void set_cond(unsigned long long h, int cont) {
 template <bool kVec, bool kCheck>
 __global__ void __launch_bounds__(kBlock) cg_update_kernel(UpdArgs a) {
     CgScalars *sc = a.sc;
-    if (kCheck && sc->done) return;
+    // `done` is tested after each trip's loads (never in front of them); it
+    // is uniform over the grid, so every block leaves before the reduction.
+    const int done = kCheck ? *(volatile const int *)&sc->done : 0;
     const double rtrans = sc->rr_cur, pAp = sc->pAp;
     const bool stop = (rtrans == 0.0) || (pAp == 0.0);  // A11
     const double alpha = stop ? 0.0 : rtrans / pAp;
@@ -336,6 +356,7 @@ __global__ void __launch_bounds__(kBlock) cg_update_kernel(UpdArgs a) {
             double2 xa = x2[i], ra = r2[i], pa = __ldcs(p2 + i), qa = __ldcs(q2 + i);
             double2 xb = {0, 0}, rb = {0, 0}, pb = {0, 0}, qb = {0, 0};
             if (hj) { xb = x2[j]; rb = r2[j]; pb = __ldcs(p2 + j); qb = __ldcs(q2 + j); }
+            if (done) return;
             xa.x = fma(alpha, pa.x, xa.x); xa.y = fma(alpha, pa.y, xa.y);
             ra.x = fma(-alpha, qa.x, ra.x); ra.y = fma(-alpha, qa.y, ra.y);
             xb.x = fma(alpha, pb.x, xb.x); xb.y = fma(alpha, pb.y, xb.y);
@@ -351,6 +372,7 @@ __global__ void __launch_bounds__(kBlock) cg_update_kernel(UpdArgs a) {
                 acc2 = fma(rb.y, rb.y, acc2);
             }
         }
+        if (done) return;
         if (tid == 0 && (a.n & 1)) {
             const int64_t i = a.n - 1;
             a.x[i] = fma(alpha, a.p[i], a.x[i]);
@@ -360,6 +382,7 @@ __global__ void __launch_bounds__(kBlock) cg_update_kernel(UpdArgs a) {
         }
         acc += acc2;
     } else {
+        if (done) return;
         for (int64_t i = tid; i < a.n; i += nth) {
             a.x[i] = fma(alpha, a.p[i], a.x[i]);
             const double rv = fma(-alpha, a.Ap[i], a.r[i]);

@@ -20,7 +20,8 @@ xptr = p.vec_ptr(H.HPCCG_VEC_X)
 spmv_bytes = 12.0 * nnz + 16.0 * n
 
 
-def run(minb, graph, timing, wh, reps=3):
+def run(minb, graph, timing, wh, reps=3, l2=1):
+    p.set_option(H.HPCCG_OPT_L2_PERSIST, l2)
     p.set_option(H.HPCCG_OPT_SPMV_MINB, minb)
     p.set_option(H.HPCCG_OPT_GRAPH, graph)
     p.set_option(H.HPCCG_OPT_TIMING, timing)
@@ -32,7 +33,7 @@ def run(minb, graph, timing, wh, reps=3):
         st = p.stats()
         if best is None or st["total_ms"] < best["total_ms"]:
             best = st
-    out = {"dims": dims, "minb": minb, "graph": graph, "timing": timing, "while": wh,
+    out = {"dims": dims, "minb": minb, "graph": graph, "timing": timing, "while": wh, "l2": l2,
            "t_iter_us": best["total_ms"] * 1e3 / iters}
     if timing:
         sp = best["spmv_ms"] / best["spmv_launches"]
@@ -41,9 +42,10 @@ def run(minb, graph, timing, wh, reps=3):
     print(json.dumps(out), flush=True)
 
 
-for minb in (1, 2, 3, 4):
-    run(minb, 0, 1, 0)
-for minb in (1, 2, 3, 4):
-    run(minb, 1, 0, 1)
+for l2 in (1, 0):
+    for minb in (1, 2, 3, 4):
+        run(minb, 0, 1, 0, l2=l2)
+    for minb in (1, 2, 3, 4):
+        run(minb, 1, 0, 1, l2=l2)
 run(0, 1, 0, 0)
 run(0, 0, 0, 0)
