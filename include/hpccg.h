@@ -94,6 +94,8 @@ typedef struct hpccg_stats {
     int64_t spmv_launches;  /* SpMV passes (= niters + 1) */
     int64_t iterations;     /* niters */
     int64_t kernel_launches;/* kernels this library enqueued during the solve */
+    int64_t l2_persist_bytes; /* L2 set aside for the CG vectors during the solve (0: none) */
+    int64_t graph_mode;     /* 2 while-graph, 1 per-iteration graph, 0 plain launches */
 } hpccg_stats;
 
 HPCCG_API const char *hpccg_strerror(int code);

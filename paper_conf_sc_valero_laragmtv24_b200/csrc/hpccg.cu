@@ -529,6 +529,7 @@ int enqueue_init(hpccg_problem *p, int max_iter, double tol, bool timing,
 struct L2Window {
     hpccg_problem *p;
     bool on = false;
+    size_t kept = 0;
     explicit L2Window(hpccg_problem *p_) : p(p_) {
         hpccg_ctx *ctx = p->ctx;
         const Slab &s = p->slabs[0];
@@ -551,6 +552,8 @@ struct L2Window {
             return;
         }
         on = true;
+        size_t got = 0;
+        kept = (cudaDeviceGetLimit(&got, cudaLimitPersistingL2CacheSize) == cudaSuccess) ? got : keep;
     }
     ~L2Window() {
         if (!on) return;
@@ -1225,6 +1228,8 @@ int hpccg_solve(hpccg_problem *p, int max_iter, double tol, int *niters, double 
     st.iterations = hs.niters;
     st.spmv_launches = hs.niters + 1;
     st.kernel_launches = ctx->launches - l0;
+    st.l2_persist_bytes = (int64_t)l2win.kept;
+    st.graph_mode = use_while ? 2 : (use_graph ? 1 : 0);
     p->stats = st;
     if (niters) *niters = hs.niters;
     if (normr) *normr = hs.normr;

@@ -294,8 +294,8 @@ __global__ void __launch_bounds__(kBlock) cg_pupdate_kernel(int64_t n, const dou
         for (int64_t i = tid; i < nv; i += 2 * nth) {
             const int64_t j = i + nth;
             const bool hj = j < nv;
-            double2 ra = __ldcs(r2 + i), pa = p2[i], rb = {0, 0}, pb = {0, 0};
-            if (hj) { rb = __ldcs(r2 + j); pb = p2[j]; }
+            double2 ra = r2[i], pa = p2[i], rb = {0, 0}, pb = {0, 0};
+            if (hj) { rb = r2[j]; pb = p2[j]; }
             if (done) return;
             if (first) { pa = ra; pb = rb; }
             else {
@@ -353,9 +353,9 @@ __global__ void __launch_bounds__(kBlock) cg_update_kernel(UpdArgs a) {
         for (int64_t i = tid; i < nv; i += 2 * nth) {
             const int64_t j = i + nth;
             const bool hj = j < nv;
-            double2 xa = x2[i], ra = r2[i], pa = __ldcs(p2 + i), qa = __ldcs(q2 + i);
+            double2 xa = x2[i], ra = r2[i], pa = p2[i], qa = q2[i];
             double2 xb = {0, 0}, rb = {0, 0}, pb = {0, 0}, qb = {0, 0};
-            if (hj) { xb = x2[j]; rb = r2[j]; pb = __ldcs(p2 + j); qb = __ldcs(q2 + j); }
+            if (hj) { xb = x2[j]; rb = r2[j]; pb = p2[j]; qb = q2[j]; }
             if (done) return;
             xa.x = fma(alpha, pa.x, xa.x); xa.y = fma(alpha, pa.y, xa.y);
             ra.x = fma(-alpha, qa.x, ra.x); ra.y = fma(-alpha, qa.y, ra.y);
