@@ -118,10 +118,12 @@ struct hpccg_problem {
     int nx = 0, ny = 0, nz = 0;
     std::vector<Slab> slabs;
     unsigned long long nnz_global = 0;
+    int64_t red_cap = 0;  // partial slots per slab reduction scratch
     // loopback allreduce tables (device arrays of device pointers)
     double **d_tab = nullptr;  // [6][nslabs]: src pAp, dst pAp, src rr, dst rr, src red, dst red
     // options
     int opt_graph = 1, opt_poll = 8, opt_timing = 0, opt_minb = 0, opt_while = 1, opt_l2 = 1;
+    int opt_vec_waves = 0;  // 0: one thread per double2 (full grid); k: k resident waves
     // graph of one CG iteration (per-iteration replay) ...
     cudaGraphExec_t graph = nullptr;
     int64_t graph_kernels = 0;
@@ -339,30 +341,41 @@ int spmv_plain(hpccg_ctx *ctx, int minb, const Slab &s, const double *x, double 
     return launch_spmv<false>(ctx, minb, false, spmv_args(s, x, y), 0, s.n, 0, 0, st);
 }
 
+// Blocks for `units` thread-units: the full grid, or `waves` resident waves.
+template <class K>
+int vec_grid(hpccg_ctx *ctx, K kernel, int64_t units, int waves, int64_t cap) {
+    int64_t b = cdiv(std::max<int64_t>(units, 1), kBlock);
+    if (waves > 0) b = std::min<int64_t>(b, (int64_t)waves * wave(ctx, kernel));
+    return (int)std::max<int64_t>(1, std::min<int64_t>(b, cap));
+}
+
 template <bool kVec, bool kCheck>
-int launch_pupdate_t(hpccg_ctx *ctx, const Slab &s, double *po) {
+int launch_pupdate_t(hpccg_ctx *ctx, int waves, const Slab &s, double *po) {
     auto k = cg_pupdate_kernel<kVec, kCheck>;
-    const int g = wave_grid(kVec ? cdiv(s.n, 4) : s.n, wave(ctx, k));
+    const int g = vec_grid(ctx, k, kVec ? cdiv(s.n, 2) : s.n, waves, 0x7fffffff);
     k<<<g, kBlock, 0, ctx->stream>>>(s.n, s.r, po, s.sc);
     return check_launch(ctx);
 }
 
-int launch_pupdate(hpccg_ctx *ctx, const Slab &s, bool check) {
+int launch_pupdate(hpccg_ctx *ctx, int waves, const Slab &s, bool check) {
     double *po = s.p + s.plane;
     const bool vec = aligned16(s.r) && aligned16(po);
-    if (vec) return check ? launch_pupdate_t<true, true>(ctx, s, po) : launch_pupdate_t<true, false>(ctx, s, po);
-    return check ? launch_pupdate_t<false, true>(ctx, s, po) : launch_pupdate_t<false, false>(ctx, s, po);
+    if (vec)
+        return check ? launch_pupdate_t<true, true>(ctx, waves, s, po)
+                     : launch_pupdate_t<true, false>(ctx, waves, s, po);
+    return check ? launch_pupdate_t<false, true>(ctx, waves, s, po)
+                 : launch_pupdate_t<false, false>(ctx, waves, s, po);
 }
 
 template <bool kVec, bool kCheck>
-int launch_update_t(hpccg_ctx *ctx, const UpdArgs &a) {
+int launch_update_t(hpccg_ctx *ctx, int waves, int64_t cap, const UpdArgs &a) {
     auto k = cg_update_kernel<kVec, kCheck>;
-    const int g = wave_grid(kVec ? cdiv(a.n, 4) : a.n, wave(ctx, k));
+    const int g = vec_grid(ctx, k, kVec ? cdiv(a.n, 2) : a.n, waves, cap);
     k<<<g, kBlock, 0, ctx->stream>>>(a);
     return check_launch(ctx);
 }
 
-int launch_update(hpccg_ctx *ctx, const Slab &s, int single, bool check,
+int launch_update(hpccg_ctx *ctx, int waves, int64_t cap, const Slab &s, int single, bool check,
                   unsigned long long cond) {
     UpdArgs a{};
     a.n = s.n;
@@ -375,8 +388,11 @@ int launch_update(hpccg_ctx *ctx, const Slab &s, int single, bool check,
     a.single = single;
     a.cond = cond;
     const bool vec = aligned16(a.x) && aligned16(a.r) && aligned16(a.p) && aligned16(a.Ap);
-    if (vec) return check ? launch_update_t<true, true>(ctx, a) : launch_update_t<true, false>(ctx, a);
-    return check ? launch_update_t<false, true>(ctx, a) : launch_update_t<false, false>(ctx, a);
+    if (vec)
+        return check ? launch_update_t<true, true>(ctx, waves, cap, a)
+                     : launch_update_t<true, false>(ctx, waves, cap, a);
+    return check ? launch_update_t<false, true>(ctx, waves, cap, a)
+                 : launch_update_t<false, false>(ctx, waves, cap, a);
 }
 
 // CG SpMV of every slab with the p.Ap epilogue.  Multi-slab: the rows that
@@ -461,7 +477,7 @@ int enqueue_iteration(hpccg_problem *p, bool timing, bool check, unsigned long l
     const int single = ctx->mode == MODE_SINGLE;
     {
         PhaseTimer t(p, ctx->stream, PH_PUPDATE, timing);
-        for (const Slab &s : p->slabs) CHECK(launch_pupdate(ctx, s, check));
+        for (const Slab &s : p->slabs) CHECK(launch_pupdate(ctx, p->opt_vec_waves, s, check));
     }
     CHECK(cg_spmv_all(p, timing, check));
     CHECK(allreduce_cg(p, false, timing));
@@ -470,7 +486,8 @@ int enqueue_iteration(hpccg_problem *p, bool timing, bool check, unsigned long l
         // every slab computes the same (allreduced) decision; slab 0 drives the
         // while-graph condition
         for (size_t i = 0; i < p->slabs.size(); ++i)
-            CHECK(launch_update(ctx, p->slabs[i], single, check, i == 0 ? cond : 0ull));
+            CHECK(launch_update(ctx, p->opt_vec_waves, p->red_cap, p->slabs[i], single, check,
+                                i == 0 ? cond : 0ull));
     }
     CHECK(allreduce_cg(p, true, timing));
     return HPCCG_OK;
@@ -908,6 +925,7 @@ int hpccg_generate(hpccg_ctx *ctx, int nx, int ny, int nz, hpccg_problem **out) 
         s.Ap = s.x + seg_v;
         if ((rc = alloc_zero((void **)&s.sc, sizeof(CgScalars)))) return bail(rc);
         const int64_t parts = cdiv(n, kBlock) + 2 * cdiv(plane, kBlock) + 148 * 8 + 64;
+        p->red_cap = parts;
         if ((rc = alloc_zero((void **)&s.red.partials, sizeof(double) * parts))) return bail(rc);
         if ((rc = alloc_zero((void **)&s.red.counter, sizeof(unsigned)))) return bail(rc);
 
@@ -1077,6 +1095,10 @@ int hpccg_set_option(hpccg_problem *p, int key, int64_t value) {
             return HPCCG_OK;
         case HPCCG_OPT_WHILE: p->opt_while = value != 0; return HPCCG_OK;
         case HPCCG_OPT_L2_PERSIST: p->opt_l2 = value != 0; return HPCCG_OK;
+        case HPCCG_OPT_VEC_WAVES:
+            if (value < 0 || value > 64) return fail(HPCCG_EINVAL, "vec waves must be 0..64");
+            p->opt_vec_waves = (int)value;
+            return HPCCG_OK;
         default: return fail(HPCCG_EINVAL, "unknown option %d", key);
     }
 }

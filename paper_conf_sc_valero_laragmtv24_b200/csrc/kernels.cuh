@@ -267,10 +267,10 @@ __global__ void __launch_bounds__(kBlock, kMinB) spmv27_kernel(SpmvArgs a) {
 }
 
 // ------------------------------------------------ streaming vector kernels
-// Persistent grids (SM count x resident blocks, sized by the host from the
-// occupancy calculator) walk the vectors in 16-B double2 units, two units per
-// thread per trip with all loads issued before any arithmetic (memory-level
-// parallelism).  Scalar (8-B) path when a pointer is not 16-B aligned.  The
+// Grids walk the vectors in 16-B double2 units, one unit per thread per trip;
+// by default one thread per unit (a full, non-persistent grid: 2048 resident
+// threads per SM keep enough loads in flight), or a persistent grid of
+// HPCCG_OPT_VEC_WAVES waves (SM count x resident blocks).  Scalar (8-B) path when a pointer is not 16-B aligned.  The
 // element -> thread mapping depends only on (n, grid): reductions are
 // run-to-run deterministic.
 
@@ -291,19 +291,17 @@ __global__ void __launch_bounds__(kBlock) cg_pupdate_kernel(int64_t n, const dou
         const int64_t nv = n >> 1;
         const double2 *r2 = reinterpret_cast<const double2 *>(r);
         double2 *p2 = reinterpret_cast<double2 *>(p);
-        for (int64_t i = tid; i < nv; i += 2 * nth) {
-            const int64_t j = i + nth;
-            const bool hj = j < nv;
-            double2 ra = r2[i], pa = p2[i], rb = {0, 0}, pb = {0, 0};
-            if (hj) { rb = r2[j]; pb = p2[j]; }
+        for (int64_t i = tid; i < nv; i += nth) {
+            const double2 ra = r2[i];
+            double2 pa = p2[i];
             if (done) return;
-            if (first) { pa = ra; pb = rb; }
-            else {
-                pa.x = fma(beta, pa.x, ra.x); pa.y = fma(beta, pa.y, ra.y);
-                pb.x = fma(beta, pb.x, rb.x); pb.y = fma(beta, pb.y, rb.y);
+            if (first) {
+                pa = ra;
+            } else {
+                pa.x = fma(beta, pa.x, ra.x);
+                pa.y = fma(beta, pa.y, ra.y);
             }
             p2[i] = pa;
-            if (hj) p2[j] = pb;
         }
         if (done) return;
         if (tid == 0 && (n & 1)) {
@@ -350,27 +348,18 @@ __global__ void __launch_bounds__(kBlock) cg_update_kernel(UpdArgs a) {
         double2 *r2 = reinterpret_cast<double2 *>(a.r);
         const double2 *p2 = reinterpret_cast<const double2 *>(a.p);
         const double2 *q2 = reinterpret_cast<const double2 *>(a.Ap);
-        for (int64_t i = tid; i < nv; i += 2 * nth) {
-            const int64_t j = i + nth;
-            const bool hj = j < nv;
-            double2 xa = x2[i], ra = r2[i], pa = p2[i], qa = q2[i];
-            double2 xb = {0, 0}, rb = {0, 0}, pb = {0, 0}, qb = {0, 0};
-            if (hj) { xb = x2[j]; rb = r2[j]; pb = p2[j]; qb = q2[j]; }
+        for (int64_t i = tid; i < nv; i += nth) {
+            double2 xa = x2[i], ra = r2[i];
+            const double2 pa = p2[i], qa = q2[i];
             if (done) return;
-            xa.x = fma(alpha, pa.x, xa.x); xa.y = fma(alpha, pa.y, xa.y);
-            ra.x = fma(-alpha, qa.x, ra.x); ra.y = fma(-alpha, qa.y, ra.y);
-            xb.x = fma(alpha, pb.x, xb.x); xb.y = fma(alpha, pb.y, xb.y);
-            rb.x = fma(-alpha, qb.x, rb.x); rb.y = fma(-alpha, qb.y, rb.y);
+            xa.x = fma(alpha, pa.x, xa.x);
+            xa.y = fma(alpha, pa.y, xa.y);
+            ra.x = fma(-alpha, qa.x, ra.x);
+            ra.y = fma(-alpha, qa.y, ra.y);
             x2[i] = xa;
             r2[i] = ra;
             acc = fma(ra.x, ra.x, acc);
             acc2 = fma(ra.y, ra.y, acc2);
-            if (hj) {
-                x2[j] = xb;
-                r2[j] = rb;
-                acc = fma(rb.x, rb.x, acc);
-                acc2 = fma(rb.y, rb.y, acc2);
-            }
         }
         if (done) return;
         if (tid == 0 && (a.n & 1)) {

@@ -1,0 +1,35 @@
+"""GPU probe: time hpccg_solve under option sets.
+usage: probe.py NX NY NZ ITERS 'opt=val,opt=val' ['opt=val,...' ...]
+opts: graph timing while minb l2 waves"""
+import json, os, sys
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+from paper_conf_sc_valero_laragmtv24_b200 import hpccg as H
+KEYS = {"graph": H.HPCCG_OPT_GRAPH, "timing": H.HPCCG_OPT_TIMING, "while": H.HPCCG_OPT_WHILE,
+        "minb": H.HPCCG_OPT_SPMV_MINB, "l2": H.HPCCG_OPT_L2_PERSIST, "waves": H.HPCCG_OPT_VEC_WAVES}
+nx, ny, nz, iters = (int(v) for v in sys.argv[1:5])
+ctx = H.Context(0)
+p = H.Problem(ctx, nx, ny, nz)
+n, nnz = p.n, p.info["nnz_local"]
+xptr = p.vec_ptr(H.HPCCG_VEC_X)
+for spec in sys.argv[5:]:
+    opts = dict(kv.split("=") for kv in spec.split(",") if kv)
+    for k, v in opts.items():
+        p.set_option(KEYS[k], int(v))
+    best = None
+    for _ in range(4):
+        ctx.waxpby(n, 0.0, xptr, 0.0, xptr, xptr)
+        r = p.solve(iters + 1, 0.0)
+        st = p.stats()
+        if best is None or st["total_ms"] < best["total_ms"]:
+            best = st
+    out = {"dims": [nx, ny, nz], "opts": opts, "t_iter_us": round(best["total_ms"] * 1e3 / iters, 2),
+           "gflops": round(iters * (2 * nnz + 10 * n) / (best["total_ms"] * 1e-3) / 1e9, 1),
+           "mode": best["graph_mode"], "err": p.maxabsdiff()}
+    if best["spmv_ms"] > 0:
+        sp = best["spmv_ms"] / best["spmv_launches"]
+        out.update(spmv_us=round(sp * 1e3, 2), spmv_gbs=round((12 * nnz + 16 * n) / (sp * 1e-3) / 1e9, 1),
+                   upd_us=round(best["update_ms"] * 1e3 / iters, 2),
+                   pupd_us=round(best["pupdate_ms"] * 1e3 / iters, 2))
+    print(json.dumps(out), flush=True)
+    for k in opts:
+        p.set_option(KEYS[k], {"graph": 1, "while": 1, "l2": 1}.get(k, 0))
