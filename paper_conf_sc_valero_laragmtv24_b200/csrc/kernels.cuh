@@ -219,7 +219,7 @@ __global__ void __launch_bounds__(kBlock, kMinB) spmv27_kernel(SpmvArgs a) {
     double d = 0.0;
     // The done flag is read together with the first matrix loads and tested
     // after them, so its latency never sits in front of the stream.
-    const int done = (kDot && kCheck) ? *(volatile const int *)&a.sc->done : 0;
+    const int done = (kDot && kCheck) ? __ldg(&a.sc->done) : 0;
     if (row < lim) {
         const uint64_t pol = policy_evict_first();
         const double *v = a.val + row;
@@ -267,6 +267,11 @@ __global__ void __launch_bounds__(kBlock, kMinB) spmv27_kernel(SpmvArgs a) {
 }
 
 // ------------------------------------------------ streaming vector kernels
+// Device scalars are read with ld.global.nc (__ldg): they are constant for the
+// kernel's lifetime, and the read-only path lets one L2 request per SM serve
+// every warp.  (Plain volatile reads from every warp all hit the one L2 slice
+// that owns the scalar line and serialise there -- measured: 2x slower
+// vector kernels.)
 // Grids walk the vectors in 16-B double2 units, one unit per thread per trip;
 // by default one thread per unit (a full, non-persistent grid: 2048 resident
 // threads per SM keep enough loads in flight), or a persistent grid of
@@ -283,9 +288,9 @@ __global__ void __launch_bounds__(kBlock) cg_pupdate_kernel(int64_t n, const dou
                                                            double *__restrict__ p,
                                                            const CgScalars *sc) {
     // `done` is tested after each trip's loads (never in front of them)
-    const int done = kCheck ? *(volatile const int *)&sc->done : 0;
-    const bool first = (sc->k == 1);
-    const double beta = first ? 0.0 : sc->rr_cur / sc->rr_prev;
+    const int done = kCheck ? __ldg(&sc->done) : 0;
+    const bool first = (__ldg(&sc->k) == 1);
+    const double beta = first ? 0.0 : __ldg(&sc->rr_cur) / __ldg(&sc->rr_prev);
     const int64_t tid = gtid(), nth = gnth();
     if (kVec) {
         const int64_t nv = n >> 1;
@@ -336,8 +341,8 @@ __global__ void __launch_bounds__(kBlock) cg_update_kernel(UpdArgs a) {
     CgScalars *sc = a.sc;
     // `done` is tested after each trip's loads (never in front of them); it
     // is uniform over the grid, so every block leaves before the reduction.
-    const int done = kCheck ? *(volatile const int *)&sc->done : 0;
-    const double rtrans = sc->rr_cur, pAp = sc->pAp;
+    const int done = kCheck ? __ldg(&sc->done) : 0;
+    const double rtrans = __ldg(&sc->rr_cur), pAp = __ldg(&sc->pAp);
     const bool stop = (rtrans == 0.0) || (pAp == 0.0);  // A11
     const double alpha = stop ? 0.0 : rtrans / pAp;
     const int64_t tid = gtid(), nth = gnth();
