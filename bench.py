@@ -203,7 +203,6 @@ def run_ours(args, nx, ny, nz, iters, cfg_index, scaling):
     n, nnz_local = prob.n, prob.info["nnz_local"]
     nnz_global = prob.info["nnz_global"]
     prob.set_option(H.HPCCG_OPT_GRAPH, 1)
-    prob.set_option(H.HPCCG_OPT_TIMING, 1 if args.phase_timing else 0)
     xptr = prob.vec_ptr(H.HPCCG_VEC_X)
 
     def barrier():
@@ -217,26 +216,45 @@ def run_ours(args, nx, ny, nz, iters, cfg_index, scaling):
         err = prob.maxabsdiff()
         return r, err
 
-    for _ in range(args.warmup):
-        step()
-    barrier()
-    spmv_ms = spmv_n = 0.0
-    niters_tot = 0
-    l0 = ctx.launch_count
-    with ClockSampler(local) as clk:
-        barrier()
+    def timed(k_steps):
+        """K steps between barriers; CUDA events on the library stream."""
         t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        acc = {"spmv_ms": 0.0, "spmv_n": 0, "niters": 0, "update_ms": 0.0, "pupdate_ms": 0.0}
+        barrier()
         t0.record(stream)
-        for _ in range(args.steps):
+        for _ in range(k_steps):
             r, err = step()
             st = prob.stats()
-            spmv_ms += st["spmv_ms"]
-            spmv_n += st["spmv_launches"]
-            niters_tot += r["niters"]
+            acc["spmv_ms"] += st["spmv_ms"]
+            acc["spmv_n"] += st["spmv_launches"]
+            acc["update_ms"] += st["update_ms"]
+            acc["pupdate_ms"] += st["pupdate_ms"]
+            acc["niters"] += r["niters"]
+            acc["graph_mode"] = st["graph_mode"]
         t1.record(stream)
         barrier()
-    launches = ctx.launch_count - l0
-    ms = t0.elapsed_time(t1)
+        acc["ms"] = t0.elapsed_time(t1)
+        acc["r"], acc["err"] = r, err
+        return acc
+
+    for _ in range(args.warmup):
+        step()
+    l0 = ctx.launch_count
+    with ClockSampler(local) as clk:
+        # (1) the product configuration: whole solve = one graph with a
+        #     device-driven while node; this region gives `value`
+        main = timed(args.steps)
+        launches = ctx.launch_count - l0
+        # (2) the same K steps with CUDA events around every phase (plain
+        #     launches): the SpMV roofline and the phase split come from here
+        prob.set_option(H.HPCCG_OPT_TIMING, 1)
+        step()
+        ev = timed(args.steps)
+        prob.set_option(H.HPCCG_OPT_TIMING, 0)
+    ms = main["ms"]
+    niters_tot = main["niters"]
+    r, err = main["r"], main["err"]
+    spmv_ms, spmv_n = ev["spmv_ms"], ev["spmv_n"]
     ms_max, flops = D.max_time_sum_work(ms, cg_flops(niters_tot, nnz_local, n), "cuda")
     value = flops / (ms_max * 1e-3) * 1e-9
 
@@ -253,6 +271,7 @@ def run_ours(args, nx, ny, nz, iters, cfg_index, scaling):
 
     step_e2e()
     barrier()
+    t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     t0.record(stream)
     ni_e2e = 0
     for _ in range(args.steps):
@@ -277,7 +296,12 @@ def run_ours(args, nx, ny, nz, iters, cfg_index, scaling):
                     "traffic": traffic_from_profiles(args.workload),
                     "algorithmic_bytes_per_launch": spmv_bytes, "avg_launch_us": round(avg_ms * 1e3, 2),
                     "peak_source": peak_src,
-                    "spmv_share_of_step": round(spmv_ms / ms, 4) if ms > 0 else None}
+                    "spmv_share_of_step": round(spmv_ms / ev["ms"], 4) if ev["ms"] > 0 else None,
+                    "measured_in": "events pass: the same K steps re-run with a CUDA event pair "
+                                   "around every phase launch (plain launches, bench.py region 2)",
+                    "events_pass_ms_per_step": round(ev["ms"] / args.steps, 4),
+                    "update_avg_us": round(ev["update_ms"] * 1e3 / max(ev["niters"], 1), 2),
+                    "pupdate_avg_us": round(ev["pupdate_ms"] * 1e3 / max(ev["niters"], 1), 2)}
         cpu = None
         if world == 1 and not args.no_cpu_baseline:
             cs = oracle_sample(nx, ny, nz, iters, args.cpu_budget)
@@ -295,8 +319,9 @@ def run_ours(args, nx, ny, nz, iters, cfg_index, scaling):
             "config": {"workload": args.workload, "baseline_config": cfg_index,
                        "nx": nx, "ny": ny, "nz_per_gpu": nz, "iters": iters,
                        "global_rows": n * world, "global_nnz": nnz_global,
-                       "parallelism": f"zslab{world}", "graph": not args.phase_timing,
-                       "phase_timing_events": bool(args.phase_timing),
+                       "parallelism": f"zslab{world}",
+                       "solve_graph": {2: "while-graph", 1: "per-iteration graph", 0: "plain"}.get(
+                           main.get("graph_mode"), "?"),
                        "l2": "inputs larger than L2 (ELL %.0f MB/GPU > 126 MB)" % (324e-6 * n),
                        "gen_ms": round(gen_ms, 3)},
             "t_iter_us": round(t_iter_us, 3),
@@ -336,8 +361,6 @@ def main():
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
     ap.add_argument("--workload", choices=sorted(WORKLOADS), default="hpccg128")
     ap.add_argument("--iters", type=int, default=None, help="override CG iterations per step")
-    ap.add_argument("--phase-timing", type=int, default=1,
-                    help="1: CUDA events around every phase (roofline from the timed region)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-budget", type=float, default=12.0, help="seconds of oracle CG")
     ap.add_argument("--ref-iters", type=int, default=5, help="oracle iterations per reference step")
