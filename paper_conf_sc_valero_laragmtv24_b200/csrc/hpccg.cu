@@ -100,7 +100,6 @@ struct Slab {
     int *col = nullptr;
     double *b = nullptr, *x = nullptr, *xexact = nullptr, *r = nullptr, *Ap = nullptr;
     double *p_alloc = nullptr, *p = nullptr;  // p: local-with-halo base (ncol)
-    double *p2 = nullptr;  // second p buffer (fused single-slab iteration)
     // r, x, Ap and p live in one contiguous "arena" so one L2 access-policy
     // window can keep the CG vectors resident
     double *arena = nullptr;
@@ -124,8 +123,7 @@ struct hpccg_problem {
     double **d_tab = nullptr;  // [6][nslabs]: src pAp, dst pAp, src rr, dst rr, src red, dst red
     // options
     int opt_graph = 1, opt_poll = 8, opt_timing = 0, opt_minb = 0, opt_while = 1, opt_l2 = 1;
-    int opt_vec_waves = 1;  // 0: one thread per double2 (full grid); k: k resident waves
-    int opt_fuse_p = 1;     // single slab: fold the p update into the SpMV
+    int opt_vec_waves = 0;  // 0: one thread per double2 (full grid); k: k resident waves
     // graph of one CG iteration (per-iteration replay) ...
     cudaGraphExec_t graph = nullptr;
     int64_t graph_kernels = 0;
@@ -310,40 +308,15 @@ SpmvArgs spmv_args(const Slab &s, const double *x, double *y) {
 // kMinB of the SpMV (register budget): tuned on B200, see DESIGN.md sec. 7.
 constexpr int kSpmvMinBDefault = 4;
 
-template <bool kDot, bool kCheck, bool kFuse = false>
+template <bool kDot, bool kCheck>
 int launch_spmv_t(hpccg_ctx *ctx, int minb, const SpmvArgs &a, unsigned blocks, cudaStream_t st) {
     switch (minb) {
-        case 1: spmv27_kernel<kDot, kCheck, 1, kFuse><<<blocks, kBlock, 0, st>>>(a); break;
-        case 3: spmv27_kernel<kDot, kCheck, 3, kFuse><<<blocks, kBlock, 0, st>>>(a); break;
-        case 4: spmv27_kernel<kDot, kCheck, 4, kFuse><<<blocks, kBlock, 0, st>>>(a); break;
-        default: spmv27_kernel<kDot, kCheck, 2, kFuse><<<blocks, kBlock, 0, st>>>(a); break;
+        case 1: spmv27_kernel<kDot, kCheck, 1><<<blocks, kBlock, 0, st>>>(a); break;
+        case 3: spmv27_kernel<kDot, kCheck, 3><<<blocks, kBlock, 0, st>>>(a); break;
+        case 4: spmv27_kernel<kDot, kCheck, 4><<<blocks, kBlock, 0, st>>>(a); break;
+        default: spmv27_kernel<kDot, kCheck, 2><<<blocks, kBlock, 0, st>>>(a); break;
     }
     return check_launch(ctx);
-}
-
-// Single slab, fused p update (kFuse): all rows, p.Ap epilogue.
-int launch_spmv_fused(hpccg_ctx *ctx, int minb, bool check, const Slab &s) {
-    SpmvArgs a{};
-    a.stride = s.n;
-    a.plane = s.plane;
-    a.val = s.val;
-    a.col = s.col;
-    a.x = s.p;
-    a.x_alt = s.p2;
-    a.r = s.r;
-    a.y = s.Ap;
-    a.sc = s.sc;
-    a.red = s.red;
-    a.single = 1;
-    a.r0 = 0;
-    a.len0 = s.n;
-    a.nb0 = cdiv(s.n, kBlock);
-    a.part_base = 0;
-    a.total_blocks = (unsigned)a.nb0;
-    if (a.nb0 > 0x7fffffffLL) return fail(HPCCG_EINVAL, "SpMV grid too large");
-    if (minb <= 0) minb = kSpmvMinBDefault;
-    return check ? launch_spmv_t<true, true, true>(ctx, minb, a, (unsigned)a.nb0, ctx->stream)
-                 : launch_spmv_t<true, false, true>(ctx, minb, a, (unsigned)a.nb0, ctx->stream);
 }
 
 template <bool kDot>
@@ -403,20 +376,18 @@ int launch_update_t(hpccg_ctx *ctx, int waves, int64_t cap, const UpdArgs &a) {
 }
 
 int launch_update(hpccg_ctx *ctx, int waves, int64_t cap, const Slab &s, int single, bool check,
-                  unsigned long long cond, bool fused = false) {
+                  unsigned long long cond) {
     UpdArgs a{};
     a.n = s.n;
     a.x = s.x;
     a.r = s.r;
     a.p = s.p + s.plane;
-    a.p_alt = fused ? s.p2 + s.plane : nullptr;
     a.Ap = s.Ap;
     a.sc = s.sc;
     a.red = s.red;
     a.single = single;
     a.cond = cond;
-    const bool vec = aligned16(a.x) && aligned16(a.r) && aligned16(a.p) && aligned16(a.Ap) &&
-                     (!a.p_alt || aligned16(a.p_alt));
+    const bool vec = aligned16(a.x) && aligned16(a.r) && aligned16(a.p) && aligned16(a.Ap);
     if (vec)
         return check ? launch_update_t<true, true>(ctx, waves, cap, a)
                      : launch_update_t<true, false>(ctx, waves, cap, a);
@@ -504,15 +475,6 @@ int allreduce_cg(hpccg_problem *p, bool rr, bool timing) {
 int enqueue_iteration(hpccg_problem *p, bool timing, bool check, unsigned long long cond) {
     hpccg_ctx *ctx = p->ctx;
     const int single = ctx->mode == MODE_SINGLE;
-    if (single && p->opt_fuse_p) {  // 2 kernels: SpMV with the p update folded in, update
-        const Slab &s = p->slabs[0];
-        {
-            PhaseTimer t(p, ctx->stream, PH_SPMV, timing);
-            CHECK(launch_spmv_fused(ctx, p->opt_minb, check, s));
-        }
-        PhaseTimer t(p, ctx->stream, PH_UPDATE, timing);
-        return launch_update(ctx, p->opt_vec_waves, p->red_cap, s, 1, check, cond, true);
-    }
     {
         PhaseTimer t(p, ctx->stream, PH_PUPDATE, timing);
         for (const Slab &s : p->slabs) CHECK(launch_pupdate(ctx, p->opt_vec_waves, s, check));
@@ -954,12 +916,11 @@ int hpccg_generate(hpccg_ctx *ctx, int nx, int ny, int nz, hpccg_problem **out) 
         // p: [lower halo | n owned | upper halo]; shifted by one element when
         // the plane is odd so the owned part is 16-B aligned (double2 loads).
         const int64_t seg_p = cdiv(ncol + 2, 32) * 32, seg_v = cdiv(n, 32) * 32;
-        s.arena_bytes = sizeof(double) * (size_t)(2 * seg_p + 3 * seg_v);
+        s.arena_bytes = sizeof(double) * (size_t)(seg_p + 3 * seg_v);
         if ((rc = alloc_zero((void **)&s.arena, s.arena_bytes))) return bail(rc);
         s.p_alloc = s.arena;
         s.p = s.p_alloc + ((plane & 1) ? 1 : 0);
-        s.p2 = s.p + seg_p;
-        s.r = s.arena + 2 * seg_p;
+        s.r = s.arena + seg_p;
         s.x = s.r + seg_v;
         s.Ap = s.x + seg_v;
         if ((rc = alloc_zero((void **)&s.sc, sizeof(CgScalars)))) return bail(rc);
@@ -1138,7 +1099,6 @@ int hpccg_set_option(hpccg_problem *p, int key, int64_t value) {
             if (value < 0 || value > 64) return fail(HPCCG_EINVAL, "vec waves must be 0..64");
             p->opt_vec_waves = (int)value;
             return HPCCG_OK;
-        case HPCCG_OPT_FUSE_P: p->opt_fuse_p = value != 0; return HPCCG_OK;
         default: return fail(HPCCG_EINVAL, "unknown option %d", key);
     }
 }

@@ -199,9 +199,6 @@ struct SpmvArgs {
     Reduction red;
     unsigned part_base, total_blocks;
     int single;             // 1: write the global pAp directly (no allreduce)
-    // kFuse (single slab): the p update is folded in -- see spmv27_kernel
-    const double *x_alt;    // the second p buffer (local-with-halo base)
-    const double *r;        // owned r (n entries), gathered as r[col - plane]
 };
 
 // kDot: CG variant with the p.Ap epilogue.  kCheck: return at once when the
@@ -209,12 +206,7 @@ struct SpmvArgs {
 // while-graph never launches past convergence so it skips that load, whose
 // latency would otherwise sit in front of every block's first matrix load).
 // kMinB: __launch_bounds__ min blocks per SM (register budget 65536/(256 kMinB)).
-// kFuse (single slab): a.6 folded into the SpMV.  Iteration k
-// reads p_old from buffer (k&1)^1 and gathers p_new_j = fma(beta, p_old_j,
-// r_j) (k == 1: r_j) -- the very expression cg_pupdate_kernel evaluates, so
-// the bits are identical -- and writes p_new_i of its own row into buffer
-// k&1.  Saves the p-update pass (24n B) and one launch per iteration.
-template <bool kDot, bool kCheck, int kMinB, bool kFuse = false>
+template <bool kDot, bool kCheck, int kMinB>
 __global__ void __launch_bounds__(kBlock, kMinB) spmv27_kernel(SpmvArgs a) {
     int64_t row, lim;
     if ((int64_t)blockIdx.x < a.nb0) {
@@ -228,17 +220,6 @@ __global__ void __launch_bounds__(kBlock, kMinB) spmv27_kernel(SpmvArgs a) {
     // The done flag is read together with the first matrix loads and tested
     // after them, so its latency never sits in front of the stream.
     const int done = (kDot && kCheck) ? __ldg(&a.sc->done) : 0;
-    const double *src = a.x;
-    double *dst = nullptr;
-    bool first = false;
-    double beta = 0.0;
-    if (kFuse) {
-        const int k = __ldg(&a.sc->k);
-        first = (k == 1);
-        beta = first ? 0.0 : __ldg(&a.sc->rr_cur) / __ldg(&a.sc->rr_prev);
-        src = (k & 1) ? a.x : a.x_alt;
-        dst = const_cast<double *>((k & 1) ? a.x_alt : a.x);
-    }
     if (row < lim) {
         const uint64_t pol = policy_evict_first();
         const double *v = a.val + row;
@@ -261,13 +242,7 @@ __global__ void __launch_bounds__(kBlock, kMinB) spmv27_kernel(SpmvArgs a) {
             if (g == 0 && done) return;  // uniform over the grid, before any store
 #pragma unroll
             for (int t = 0; t < 9; ++t) {
-                double xv;
-                if (kFuse) {
-                    const double rv = __ldg(a.r + (cc[t] - a.plane));
-                    xv = first ? rv : fma(beta, __ldg(src + cc[t]), rv);
-                } else {
-                    xv = __ldg(a.x + cc[t]);
-                }
+                const double xv = __ldg(a.x + cc[t]);
                 if (9 * g + t == kDiagSlot) {
                     xd = xv;
                     cd = cc[t];
@@ -278,17 +253,7 @@ __global__ void __launch_bounds__(kBlock, kMinB) spmv27_kernel(SpmvArgs a) {
         a.y[row] = sum;
         // p_i: the diagonal slot's gathered value when that slot really is the
         // row's own column (always, for generated matrices); else reload it.
-        double pi;
-        if (cd == row + a.plane) {
-            pi = xd;
-        } else if (kFuse) {
-            const double rv = __ldg(a.r + row);
-            pi = first ? rv : fma(beta, __ldg(src + row + a.plane), rv);
-        } else {
-            pi = __ldg(a.x + row + a.plane);
-        }
-        if (kFuse) dst[row + a.plane] = pi;
-        if (kDot) d = sum * pi;
+        if (kDot) d = sum * (cd == row + a.plane ? xd : __ldg(a.x + row + a.plane));
     }
     if (done) return;
     if (kDot) {
@@ -361,7 +326,6 @@ struct UpdArgs {
     int64_t n;
     double *x, *r;
     const double *p, *Ap;
-    const double *p_alt;  // fused path: iteration k's p is (k & 1) ? p_alt : p
     CgScalars *sc;
     Reduction red;
     int single;
@@ -379,7 +343,6 @@ __global__ void __launch_bounds__(kBlock) cg_update_kernel(UpdArgs a) {
     // is uniform over the grid, so every block leaves before the reduction.
     const int done = kCheck ? __ldg(&sc->done) : 0;
     const double rtrans = __ldg(&sc->rr_cur), pAp = __ldg(&sc->pAp);
-    const double *pv = (a.p_alt && (__ldg(&sc->k) & 1)) ? a.p_alt : a.p;
     const bool stop = (rtrans == 0.0) || (pAp == 0.0);  // A11
     const double alpha = stop ? 0.0 : rtrans / pAp;
     const int64_t tid = gtid(), nth = gnth();
@@ -388,7 +351,7 @@ __global__ void __launch_bounds__(kBlock) cg_update_kernel(UpdArgs a) {
         const int64_t nv = a.n >> 1;
         double2 *x2 = reinterpret_cast<double2 *>(a.x);
         double2 *r2 = reinterpret_cast<double2 *>(a.r);
-        const double2 *p2 = reinterpret_cast<const double2 *>(pv);
+        const double2 *p2 = reinterpret_cast<const double2 *>(a.p);
         const double2 *q2 = reinterpret_cast<const double2 *>(a.Ap);
         for (int64_t i = tid; i < nv; i += nth) {
             double2 xa = x2[i], ra = r2[i];
@@ -406,7 +369,7 @@ __global__ void __launch_bounds__(kBlock) cg_update_kernel(UpdArgs a) {
         if (done) return;
         if (tid == 0 && (a.n & 1)) {
             const int64_t i = a.n - 1;
-            a.x[i] = fma(alpha, pv[i], a.x[i]);
+            a.x[i] = fma(alpha, a.p[i], a.x[i]);
             const double rv = fma(-alpha, a.Ap[i], a.r[i]);
             a.r[i] = rv;
             acc = fma(rv, rv, acc);
@@ -415,7 +378,7 @@ __global__ void __launch_bounds__(kBlock) cg_update_kernel(UpdArgs a) {
     } else {
         if (done) return;
         for (int64_t i = tid; i < a.n; i += nth) {
-            a.x[i] = fma(alpha, pv[i], a.x[i]);
+            a.x[i] = fma(alpha, a.p[i], a.x[i]);
             const double rv = fma(-alpha, a.Ap[i], a.r[i]);
             a.r[i] = rv;
             acc = fma(rv, rv, acc);

@@ -5,8 +5,7 @@ import json, os, sys
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 from paper_conf_sc_valero_laragmtv24_b200 import hpccg as H
 KEYS = {"graph": H.HPCCG_OPT_GRAPH, "timing": H.HPCCG_OPT_TIMING, "while": H.HPCCG_OPT_WHILE,
-        "minb": H.HPCCG_OPT_SPMV_MINB, "l2": H.HPCCG_OPT_L2_PERSIST, "waves": H.HPCCG_OPT_VEC_WAVES,
-        "fuse": H.HPCCG_OPT_FUSE_P}
+        "minb": H.HPCCG_OPT_SPMV_MINB, "l2": H.HPCCG_OPT_L2_PERSIST, "waves": H.HPCCG_OPT_VEC_WAVES}
 nx, ny, nz, iters = (int(v) for v in sys.argv[1:5])
 ctx = H.Context(0)
 p = H.Problem(ctx, nx, ny, nz)
@@ -33,4 +32,4 @@ for spec in sys.argv[5:]:
                    pupd_us=round(best["pupdate_ms"] * 1e3 / iters, 2))
     print(json.dumps(out), flush=True)
     for k in opts:
-        p.set_option(KEYS[k], {"graph": 1, "while": 1, "l2": 1, "waves": 1, "fuse": 1}.get(k, 0))
+        p.set_option(KEYS[k], {"graph": 1, "while": 1, "l2": 1}.get(k, 0))
