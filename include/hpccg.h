@@ -77,8 +77,8 @@ extern "C" {
 #define HPCCG_OPT_L2_PERSIST 5 /* 1 (default): during hpccg_solve, mark the CG vectors
                                (r, x, Ap, p) L2-persisting via an access-policy window on
                                the stream (restored afterwards); 0: off */
-#define HPCCG_OPT_VEC_WAVES 6 /* CG vector kernels: 0 (default) one thread per 16-B unit;
-                               k > 0: a persistent grid of k resident waves */
+#define HPCCG_OPT_VEC_WAVES 6 /* CG vector kernels: 0 one thread per 16-B unit; k > 0
+                               (default 1): a persistent grid of k resident waves */
 
 typedef struct hpccg_ctx hpccg_ctx;         /* device, streams, comm (rank, nranks) */
 typedef struct hpccg_problem hpccg_problem; /* A (ELL-27), b, x, x_exact, CG work vectors */

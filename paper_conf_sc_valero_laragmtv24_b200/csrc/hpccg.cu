@@ -123,7 +123,7 @@ struct hpccg_problem {
     double **d_tab = nullptr;  // [6][nslabs]: src pAp, dst pAp, src rr, dst rr, src red, dst red
     // options
     int opt_graph = 1, opt_poll = 8, opt_timing = 0, opt_minb = 0, opt_while = 1, opt_l2 = 1;
-    int opt_vec_waves = 0;  // 0: one thread per double2 (full grid); k: k resident waves
+    int opt_vec_waves = 1;  // 0: one thread per double2 (full grid); k: k resident waves
     // graph of one CG iteration (per-iteration replay) ...
     cudaGraphExec_t graph = nullptr;
     int64_t graph_kernels = 0;

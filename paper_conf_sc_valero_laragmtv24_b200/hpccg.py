@@ -18,7 +18,7 @@ import threading
 import numpy as np
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_PKG, "libhpccg.so")
+LIB_PATH = os.environ.get("HPCCG_LIB") or os.path.join(_PKG, "libhpccg.so")  # override: A/B tools
 HEADER = os.path.join(os.path.dirname(_PKG), "include", "hpccg.h")
 
 HPCCG_OK = 0

@@ -4,6 +4,7 @@ opts: graph timing while minb l2 waves"""
 import json, os, sys
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 from paper_conf_sc_valero_laragmtv24_b200 import hpccg as H
+# option ids (an older libhpccg may lack some; those are skipped)
 KEYS = {"graph": H.HPCCG_OPT_GRAPH, "timing": H.HPCCG_OPT_TIMING, "while": H.HPCCG_OPT_WHILE,
         "minb": H.HPCCG_OPT_SPMV_MINB, "l2": H.HPCCG_OPT_L2_PERSIST, "waves": H.HPCCG_OPT_VEC_WAVES}
 nx, ny, nz, iters = (int(v) for v in sys.argv[1:5])
@@ -14,7 +15,10 @@ xptr = p.vec_ptr(H.HPCCG_VEC_X)
 for spec in sys.argv[5:]:
     opts = dict(kv.split("=") for kv in spec.split(",") if kv)
     for k, v in opts.items():
-        p.set_option(KEYS[k], int(v))
+        try:
+            p.set_option(KEYS[k], int(v))
+        except H.HpccgError:
+            pass
     best = None
     for _ in range(4):
         ctx.waxpby(n, 0.0, xptr, 0.0, xptr, xptr)
@@ -32,4 +36,7 @@ for spec in sys.argv[5:]:
                    pupd_us=round(best["pupdate_ms"] * 1e3 / iters, 2))
     print(json.dumps(out), flush=True)
     for k in opts:
-        p.set_option(KEYS[k], {"graph": 1, "while": 1, "l2": 1}.get(k, 0))
+        try:
+            p.set_option(KEYS[k], {"graph": 1, "while": 1, "l2": 1, "waves": 1}.get(k, 0))
+        except H.HpccgError:
+            pass
