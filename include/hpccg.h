@@ -77,6 +77,8 @@ extern "C" {
 #define HPCCG_OPT_L2_PERSIST 5 /* 1 (default): during hpccg_solve, mark the CG vectors
                                (r, x, Ap, p) L2-persisting via an access-policy window on
                                the stream (restored afterwards); 0: off */
+#define HPCCG_OPT_SPMV_ROWS 7 /* SpMV rows per thread: 2 (default; needs even n and plane,
+                               else 1 is used), 1 */
 #define HPCCG_OPT_VEC_WAVES 6 /* CG vector kernels: 0 one thread per 16-B unit; k > 0
                                (default 1): a persistent grid of k resident waves */
 

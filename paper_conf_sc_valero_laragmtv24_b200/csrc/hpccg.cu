@@ -124,6 +124,7 @@ struct hpccg_problem {
     // options
     int opt_graph = 1, opt_poll = 8, opt_timing = 0, opt_minb = 0, opt_while = 1, opt_l2 = 1;
     int opt_vec_waves = 1;  // 0: one thread per double2 (full grid); k: k resident waves
+    int opt_rows = 2;       // SpMV rows per thread (2 when aligned, else 1)
     // graph of one CG iteration (per-iteration replay) ...
     cudaGraphExec_t graph = nullptr;
     int64_t graph_kernels = 0;
@@ -319,26 +320,44 @@ int launch_spmv_t(hpccg_ctx *ctx, int minb, const SpmvArgs &a, unsigned blocks, 
     return check_launch(ctx);
 }
 
+// Rows per thread of the SpMV for these ranges: 2 (spmv27x2_kernel) when the
+// 16-B / 8-B slot loads are aligned (even n, even range starts, 16-B y).
+int spmv_rows_per_thread(int opt_rows, const SpmvArgs &a, int64_t r0, int64_t r1) {
+    if (opt_rows == 1) return 1;
+    const bool ok = (a.stride % 2 == 0) && (r0 % 2 == 0) && (r1 % 2 == 0) && aligned16(a.y) &&
+                    aligned16(a.val) && ((reinterpret_cast<uintptr_t>(a.col) & 7u) == 0);
+    return ok ? 2 : 1;
+}
+
+int64_t spmv_blocks(int64_t len, int rows) { return cdiv(cdiv(len, rows), kBlock); }
+
 template <bool kDot>
 int launch_spmv(hpccg_ctx *ctx, int minb, bool check, SpmvArgs a, int64_t r0, int64_t len0,
-                int64_t r1, int64_t len1, cudaStream_t st) {
+                int64_t r1, int64_t len1, cudaStream_t st, int rows = 1) {
     a.r0 = r0;
     a.len0 = len0;
     a.r1 = r1;
     a.len1 = len1;
-    a.nb0 = cdiv(len0, kBlock);
-    const int64_t blocks = a.nb0 + cdiv(len1, kBlock);
+    a.nb0 = spmv_blocks(len0, rows);
+    const int64_t blocks = a.nb0 + spmv_blocks(len1, rows);
     if (blocks == 0) return HPCCG_OK;
     if (blocks > 0x7fffffffLL) return fail(HPCCG_EINVAL, "SpMV grid too large");
+    if (rows == 2) {
+        if (check) spmv27x2_kernel<kDot, true><<<(unsigned)blocks, kBlock, 0, st>>>(a);
+        else spmv27x2_kernel<kDot, false><<<(unsigned)blocks, kBlock, 0, st>>>(a);
+        return check_launch(ctx);
+    }
     if (minb <= 0) minb = kSpmvMinBDefault;
     return check ? launch_spmv_t<kDot, true>(ctx, minb, a, (unsigned)blocks, st)
                  : launch_spmv_t<kDot, false>(ctx, minb, a, (unsigned)blocks, st);
 }
 
 // y = A x for one slab over all rows (no dot).
-int spmv_plain(hpccg_ctx *ctx, int minb, const Slab &s, const double *x, double *y,
+int spmv_plain(hpccg_ctx *ctx, int minb, int opt_rows, const Slab &s, const double *x, double *y,
                cudaStream_t st) {
-    return launch_spmv<false>(ctx, minb, false, spmv_args(s, x, y), 0, s.n, 0, 0, st);
+    SpmvArgs a = spmv_args(s, x, y);
+    return launch_spmv<false>(ctx, minb, false, a, 0, s.n, 0, 0, st,
+                              spmv_rows_per_thread(opt_rows, a, 0, 0));
 }
 
 // Blocks for `units` thread-units: the full grid, or `waves` resident waves.
@@ -405,10 +424,11 @@ int cg_spmv_all(hpccg_problem *p, bool timing, bool check) {
         const Slab &s = p->slabs[0];
         PhaseTimer t(p, ctx->stream, PH_SPMV, timing);
         SpmvArgs a = spmv_args(s, s.p, s.Ap);
+        const int rows = spmv_rows_per_thread(p->opt_rows, a, 0, 0);
         a.single = 1;
         a.part_base = 0;
-        a.total_blocks = (unsigned)cdiv(s.n, kBlock);
-        return launch_spmv<true>(ctx, minb, check, a, 0, s.n, 0, 0, ctx->stream);
+        a.total_blocks = (unsigned)spmv_blocks(s.n, rows);
+        return launch_spmv<true>(ctx, minb, check, a, 0, s.n, 0, 0, ctx->stream, rows);
     }
     const Slab &s0 = p->slabs[0];
     const int64_t n = s0.n, plane = s0.plane;
@@ -416,8 +436,9 @@ int cg_spmv_all(hpccg_problem *p, bool timing, bool check) {
     const int64_t int_r0 = plane, int_len = std::max<int64_t>(n - 2 * plane, 0);
     const int64_t b0_len = std::min<int64_t>(plane, n);
     const int64_t b1_r0 = std::max<int64_t>(n - plane, plane), b1_len = n - b1_r0;
-    const unsigned nb_int = (unsigned)cdiv(int_len, kBlock);
-    const unsigned nb_bnd = (unsigned)(cdiv(b0_len, kBlock) + cdiv(b1_len, kBlock));
+    const int rows = spmv_rows_per_thread(p->opt_rows, spmv_args(s0, s0.p, s0.Ap), int_r0, b1_r0);
+    const unsigned nb_int = (unsigned)spmv_blocks(int_len, rows);
+    const unsigned nb_bnd = (unsigned)(spmv_blocks(b0_len, rows) + spmv_blocks(b1_len, rows));
     std::vector<double *> xs(p->slabs.size());
     for (size_t i = 0; i < xs.size(); ++i) xs[i] = p->slabs[i].p;
 
@@ -435,10 +456,10 @@ int cg_spmv_all(hpccg_problem *p, bool timing, bool check) {
         a.single = 0;
         a.total_blocks = nb_int + nb_bnd;
         a.part_base = 0;
-        CHECK(launch_spmv<true>(ctx, minb, check, a, int_r0, int_len, 0, 0, ctx->stream));
+        CHECK(launch_spmv<true>(ctx, minb, check, a, int_r0, int_len, 0, 0, ctx->stream, rows));
         CU(cudaStreamWaitEvent(ctx->stream, ctx->ev_join, 0));
         a.part_base = nb_int;
-        return launch_spmv<true>(ctx, minb, check, a, 0, b0_len, b1_r0, b1_len, ctx->stream);
+        return launch_spmv<true>(ctx, minb, check, a, 0, b0_len, b1_r0, b1_len, ctx->stream, rows);
     }
     // loopback: exchange, then interior + boundary launches per slab
     {
@@ -451,9 +472,9 @@ int cg_spmv_all(hpccg_problem *p, bool timing, bool check) {
         a.single = 0;
         a.total_blocks = nb_int + nb_bnd;
         a.part_base = 0;
-        CHECK(launch_spmv<true>(ctx, minb, check, a, int_r0, int_len, 0, 0, ctx->stream));
+        CHECK(launch_spmv<true>(ctx, minb, check, a, int_r0, int_len, 0, 0, ctx->stream, rows));
         a.part_base = nb_int;
-        CHECK(launch_spmv<true>(ctx, minb, check, a, 0, b0_len, b1_r0, b1_len, ctx->stream));
+        CHECK(launch_spmv<true>(ctx, minb, check, a, 0, b0_len, b1_r0, b1_len, ctx->stream, rows));
     }
     return HPCCG_OK;
 }
@@ -511,7 +532,8 @@ int enqueue_init(hpccg_problem *p, int max_iter, double tol, bool timing,
     }
     {
         PhaseTimer t(p, ctx->stream, PH_SPMV, timing);
-        for (const Slab &s : p->slabs) CHECK(spmv_plain(ctx, p->opt_minb, s, s.p, s.Ap, ctx->stream));
+        for (const Slab &s : p->slabs)
+            CHECK(spmv_plain(ctx, p->opt_minb, p->opt_rows, s, s.p, s.Ap, ctx->stream));
     }
     {
         PhaseTimer t(p, ctx->stream, PH_UPDATE, timing);
@@ -1095,6 +1117,10 @@ int hpccg_set_option(hpccg_problem *p, int key, int64_t value) {
             return HPCCG_OK;
         case HPCCG_OPT_WHILE: p->opt_while = value != 0; return HPCCG_OK;
         case HPCCG_OPT_L2_PERSIST: p->opt_l2 = value != 0; return HPCCG_OK;
+        case HPCCG_OPT_SPMV_ROWS:
+            if (value != 1 && value != 2) return fail(HPCCG_EINVAL, "spmv rows must be 1 or 2");
+            p->opt_rows = (int)value;
+            return HPCCG_OK;
         case HPCCG_OPT_VEC_WAVES:
             if (value < 0 || value > 64) return fail(HPCCG_EINVAL, "vec waves must be 0..64");
             p->opt_vec_waves = (int)value;
@@ -1114,7 +1140,8 @@ int hpccg_spmv(hpccg_problem *p, double *x, double *y) {
     // halo exchange on the main stream (API call: no overlap needed)
     CHECK(exchange(p, xs.data(), ctx->stream));
     for (size_t i = 0; i < P; ++i)
-        CHECK(spmv_plain(ctx, p->opt_minb, p->slabs[i], xs[i], y + i * s0.n, ctx->stream));
+        CHECK(spmv_plain(ctx, p->opt_minb, p->opt_rows, p->slabs[i], xs[i], y + i * s0.n,
+                         ctx->stream));
     CU(cudaStreamSynchronize(ctx->stream));
     return HPCCG_OK;
 }

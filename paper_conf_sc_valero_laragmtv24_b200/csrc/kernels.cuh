@@ -74,6 +74,21 @@ __device__ __forceinline__ int ld_stream(const int *ptr, uint64_t pol) {
     return v;
 }
 
+// 16-B / 8-B vector forms for two adjacent rows (slot-major: same slot)
+__device__ __forceinline__ double2 ld_stream2(const double *ptr, uint64_t pol) {
+    double2 v;
+    asm("ld.global.nc.L1::no_allocate.L2::cache_hint.v2.f64 {%0, %1}, [%2], %3;"
+        : "=d"(v.x), "=d"(v.y) : "l"(ptr), "l"(pol));
+    return v;
+}
+
+__device__ __forceinline__ int2 ld_stream2(const int *ptr, uint64_t pol) {
+    int2 v;
+    asm("ld.global.nc.L1::no_allocate.L2::cache_hint.v2.s32 {%0, %1}, [%2], %3;"
+        : "=r"(v.x), "=r"(v.y) : "l"(ptr), "l"(pol));
+    return v;
+}
+
 __device__ __forceinline__ double warp_sum(double v) {
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
@@ -254,6 +269,83 @@ __global__ void __launch_bounds__(kBlock, kMinB) spmv27_kernel(SpmvArgs a) {
         // p_i: the diagonal slot's gathered value when that slot really is the
         // row's own column (always, for generated matrices); else reload it.
         if (kDot) d = sum * (cd == row + a.plane ? xd : __ldg(a.x + row + a.plane));
+    }
+    if (done) return;
+    if (kDot) {
+        CgScalars *sc = a.sc;
+        const int single = a.single;
+        grid_reduce<false>(d, a.red, a.part_base + blockIdx.x, a.total_blocks,
+                           [sc, single](double s) {
+                               if (single) sc->pAp = s; else sc->loc_pAp = s;
+                           });
+    }
+}
+
+// Two adjacent rows per thread: 16-B `val` and 8-B `col` loads (half the
+// load instructions of spmv27_kernel for the same bytes), 9 groups of 3 slots.
+// Half as many blocks also halves the per-block cost of the last-block
+// finisher (its fence + ticket round trip holds the block's SM slot) --
+// measured on B200 at 128^3: 105.8 us vs 108.4 us with the p.Ap epilogue
+// (tools/spmvbench.cu).  Needs even n (stride), even range starts and a 16-B
+// aligned y (the host checks); a range of odd length ends in a 1-row thread.
+// Same per-row FMA order as spmv27_kernel: identical bits.
+template <bool kDot, bool kCheck>
+__global__ void __launch_bounds__(kBlock, 4) spmv27x2_kernel(SpmvArgs a) {
+    int64_t row, lim;
+    if ((int64_t)blockIdx.x < a.nb0) {
+        row = a.r0 + ((int64_t)blockIdx.x * kBlock + threadIdx.x) * 2;
+        lim = a.r0 + a.len0;
+    } else {
+        row = a.r1 + (((int64_t)blockIdx.x - a.nb0) * kBlock + threadIdx.x) * 2;
+        lim = a.r1 + a.len1;
+    }
+    double d = 0.0;
+    const int done = (kDot && kCheck) ? __ldg(&a.sc->done) : 0;
+    if (row + 1 < lim) {
+        const uint64_t pol = policy_evict_first();
+        const double *v = a.val + row;
+        const int *c = a.col + row;
+        double s0 = 0.0, s1 = 0.0, x0 = 0.0, x1 = 0.0;
+        int c0 = 0, c1 = 0;
+#pragma unroll
+        for (int g = 0; g < 9; ++g) {
+            double2 vv[3];
+            int2 cc[3];
+#pragma unroll
+            for (int t = 0; t < 3; ++t) {
+                vv[t] = ld_stream2(v + (3 * g + t) * a.stride, pol);
+                cc[t] = ld_stream2(c + (3 * g + t) * a.stride, pol);
+            }
+            if (g == 0 && done) return;  // uniform over the grid, before any store
+#pragma unroll
+            for (int t = 0; t < 3; ++t) {
+                const double xa = __ldg(a.x + cc[t].x), xb = __ldg(a.x + cc[t].y);
+                if (3 * g + t == kDiagSlot) {
+                    x0 = xa;
+                    x1 = xb;
+                    c0 = cc[t].x;
+                    c1 = cc[t].y;
+                }
+                s0 = fma(vv[t].x, xa, s0);
+                s1 = fma(vv[t].y, xb, s1);
+            }
+        }
+        *reinterpret_cast<double2 *>(a.y + row) = make_double2(s0, s1);
+        if (kDot) {
+            const double p0 = c0 == row + a.plane ? x0 : __ldg(a.x + row + a.plane);
+            const double p1 = c1 == row + 1 + a.plane ? x1 : __ldg(a.x + row + 1 + a.plane);
+            d = fma(s1, p1, s0 * p0);
+        }
+    } else if (row < lim) {  // odd tail: one row, scalar loads
+        const uint64_t pol = policy_evict_first();
+        if (done) return;
+        double s0 = 0.0;
+#pragma unroll
+        for (int k = 0; k < kSlots; ++k)
+            s0 = fma(ld_stream(a.val + k * a.stride + row, pol),
+                     __ldg(a.x + ld_stream(a.col + k * a.stride + row, pol)), s0);
+        a.y[row] = s0;
+        if (kDot) d = s0 * __ldg(a.x + row + a.plane);
     }
     if (done) return;
     if (kDot) {

@@ -104,10 +104,14 @@ def test_generate_rejects_bad_sizes(ctx):
 
 # ------------------------------------------------------------------ SpMV
 
-@pytest.mark.parametrize("dims", [(20, 30, 10), (7, 5, 6), (1, 1, 1), (33, 9, 3), (64, 64, 16)])
-def test_spmv_bitwise_real(ctx, dims):
+@pytest.mark.parametrize("rows", [1, 2])
+@pytest.mark.parametrize("dims", [(20, 30, 10), (7, 5, 6), (1, 1, 1), (33, 9, 3), (64, 64, 16),
+                                  (6, 5, 3), (2, 1, 1)])
+def test_spmv_bitwise_real(ctx, dims, rows):
+    """Both SpMV kernels (1 and 2 rows per thread) give the oracle's bits."""
     nx, ny, nz = dims
     with H.Problem(ctx, nx, ny, nz) as p:
+        p.set_option(H.HPCCG_OPT_SPMV_ROWS, rows)
         ref = oracle.generate(nx, ny, nz)
         x = synth.uniform(ref.n, 21)
         xl = halo_vector(x, ref.n, nx * ny, 0, 1, fill=np.nan)   # halos overwritten

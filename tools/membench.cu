@@ -1,0 +1,124 @@
+// membench.cu -- memory-roofline probes on the B200 (not the product):
+// pure-read streams (plain / nc+no_allocate+evict_first / +L2::256B
+// prefetch), a 2:1 read:write stream, and L2-resident re-reads, so the SpMV
+// and vector-kernel numbers can be read against what this GPU really does.
+// nvcc -gencode arch=compute_100a,code=sm_100a -O3 -o membench membench.cu
+#include <cuda_runtime.h>
+#include <stdio.h>
+#include <stdint.h>
+
+__device__ __forceinline__ uint64_t pol_ef() {
+    uint64_t p;
+    asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+
+template <int kMode>
+__global__ void __launch_bounds__(256) read_kernel(const double2 *__restrict__ a, int64_t n2, double *out) {
+    const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const int64_t nth = (int64_t)gridDim.x * blockDim.x;
+    double s = 0.0;
+    const uint64_t pol = pol_ef();
+    for (int64_t i = tid; i < n2; i += 4 * nth) {
+        double2 v[4];
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+            const int64_t j = i + u * nth;
+            if (j < n2) {
+                if (kMode == 0) {
+                    v[u] = a[j];
+                } else if (kMode == 1) {
+                    asm("ld.global.nc.L1::no_allocate.L2::cache_hint.v2.f64 {%0,%1}, [%2], %3;"
+                        : "=d"(v[u].x), "=d"(v[u].y) : "l"(a + j), "l"(pol));
+                } else {
+                    asm("ld.global.nc.L1::no_allocate.L2::cache_hint.L2::256B.v2.f64 {%0,%1}, [%2], %3;"
+                        : "=d"(v[u].x), "=d"(v[u].y) : "l"(a + j), "l"(pol));
+                }
+            } else {
+                v[u] = make_double2(0, 0);
+            }
+        }
+#pragma unroll
+        for (int u = 0; u < 4; ++u) s += v[u].x + v[u].y;
+    }
+    if (s == 123.456) *out = s;
+}
+
+__global__ void __launch_bounds__(256) copy_kernel(const double2 *__restrict__ a, double2 *__restrict__ b, int64_t n2) {
+    const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const int64_t nth = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t i = tid; i < n2; i += nth) b[i] = a[i];
+}
+
+// 2 reads : 1 write (waxpby-like)
+__global__ void __launch_bounds__(256) triad_kernel(const double2 *__restrict__ a, const double2 *__restrict__ b,
+                                                    double2 *__restrict__ c, int64_t n2) {
+    const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const int64_t nth = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t i = tid; i < n2; i += nth) {
+        double2 x = a[i], y = b[i];
+        c[i] = make_double2(x.x + 0.5 * y.x, x.y + 0.5 * y.y);
+    }
+}
+
+template <class F>
+float timeit(F f, int reps) {
+    cudaEvent_t e0, e1;
+    cudaEventCreate(&e0);
+    cudaEventCreate(&e1);
+    f();
+    cudaDeviceSynchronize();
+    float best = 1e30f;
+    for (int r = 0; r < reps; ++r) {
+        cudaEventRecord(e0);
+        f();
+        cudaEventRecord(e1);
+        cudaEventSynchronize(e1);
+        float ms;
+        cudaEventElapsedTime(&ms, e0, e1);
+        if (ms < best) best = ms;
+    }
+    return best;
+}
+
+int main() {
+    int sms;
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0);
+    const size_t big = (size_t)1 << 30;  // 1 GiB per array
+    double2 *a, *b, *c;
+    double *out;
+    cudaMalloc(&a, big);
+    cudaMalloc(&b, big);
+    cudaMalloc(&c, big);
+    cudaMalloc(&out, 8);
+    cudaMemset(a, 0, big);
+    cudaMemset(b, 0, big);
+    const int64_t n2 = big / 16;
+    int occ;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, read_kernel<0>, 256, 0);
+    const int grid = sms * occ;
+    printf("{\"sms\": %d, \"occ_read\": %d}\n", sms, occ);
+    const char *names[3] = {"read_plain", "read_nc_ef", "read_nc_ef_256B"};
+    for (int m = 0; m < 3; ++m) {
+        float ms = timeit([&] {
+            if (m == 0) read_kernel<0><<<grid, 256>>>(a, n2, out);
+            if (m == 1) read_kernel<1><<<grid, 256>>>(a, n2, out);
+            if (m == 2) read_kernel<2><<<grid, 256>>>(a, n2, out);
+        }, 10);
+        printf("{\"probe\": \"%s\", \"bytes\": %zu, \"ms\": %.4f, \"GBs\": %.1f}\n", names[m], big, ms, big / ms / 1e6);
+    }
+    float ms = timeit([&] { copy_kernel<<<grid, 256>>>(a, b, n2); }, 10);
+    printf("{\"probe\": \"copy\", \"bytes\": %zu, \"ms\": %.4f, \"GBs\": %.1f}\n", 2 * big, ms, 2 * big / ms / 1e6);
+    ms = timeit([&] { triad_kernel<<<grid, 256>>>(a, b, c, n2); }, 10);
+    printf("{\"probe\": \"triad_2r1w\", \"bytes\": %zu, \"ms\": %.4f, \"GBs\": %.1f}\n", 3 * big, ms, 3 * big / ms / 1e6);
+    // L2-resident re-reads: 16, 32, 64 MB
+    for (size_t mb : {16, 32, 64, 96}) {
+        const size_t bytes = mb << 20;
+        const int64_t m2 = bytes / 16;
+        ms = timeit([&] { read_kernel<0><<<grid, 256>>>(a, m2, out); }, 20);
+        printf("{\"probe\": \"l2_read_%zuMB\", \"bytes\": %zu, \"ms\": %.4f, \"GBs\": %.1f}\n", mb, bytes, ms, bytes / ms / 1e6);
+        ms = timeit([&] { triad_kernel<<<grid, 256>>>(a, b, c, m2); }, 20);
+        printf("{\"probe\": \"l2_triad_%zuMB\", \"bytes\": %zu, \"ms\": %.4f, \"GBs\": %.1f}\n", mb, 3 * bytes, ms, 3 * bytes / ms / 1e6);
+    }
+    return 0;
+}
