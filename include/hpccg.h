@@ -79,6 +79,8 @@ extern "C" {
                                the stream (restored afterwards); 0: off */
 #define HPCCG_OPT_SPMV_ROWS 7 /* SpMV rows per thread: 2 (default; needs even n and plane,
                                else 1 is used), 1 */
+#define HPCCG_OPT_VEC_UNROLL 8 /* CG vector kernels: 16-B units per thread per trip with
+                               all loads in flight: 1, 2 or 4 (default 4) */
 #define HPCCG_OPT_VEC_WAVES 6 /* CG vector kernels: 0 one thread per 16-B unit; k > 0
                                (default 1): a persistent grid of k resident waves */
 

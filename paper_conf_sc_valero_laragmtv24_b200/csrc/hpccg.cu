@@ -125,6 +125,7 @@ struct hpccg_problem {
     int opt_graph = 1, opt_poll = 8, opt_timing = 0, opt_minb = 0, opt_while = 1, opt_l2 = 1;
     int opt_vec_waves = 1;  // 0: one thread per double2 (full grid); k: k resident waves
     int opt_rows = 2;       // SpMV rows per thread (2 when aligned, else 1)
+    int opt_unroll = 4;     // CG vector kernels: 16-B units per thread per trip
     // graph of one CG iteration (per-iteration replay) ...
     cudaGraphExec_t graph = nullptr;
     int64_t graph_kernels = 0;
@@ -368,34 +369,52 @@ int vec_grid(hpccg_ctx *ctx, K kernel, int64_t units, int waves, int64_t cap) {
     return (int)std::max<int64_t>(1, std::min<int64_t>(b, cap));
 }
 
-template <bool kVec, bool kCheck>
+template <bool kVec, bool kCheck, int kU>
 int launch_pupdate_t(hpccg_ctx *ctx, int waves, const Slab &s, double *po) {
-    auto k = cg_pupdate_kernel<kVec, kCheck>;
-    const int g = vec_grid(ctx, k, kVec ? cdiv(s.n, 2) : s.n, waves, 0x7fffffff);
+    auto k = cg_pupdate_kernel<kVec, kCheck, kU>;
+    const int g = vec_grid(ctx, k, kVec ? cdiv(s.n, 2 * kU) : s.n, waves, 0x7fffffff);
     k<<<g, kBlock, 0, ctx->stream>>>(s.n, s.r, po, s.sc);
     return check_launch(ctx);
 }
 
-int launch_pupdate(hpccg_ctx *ctx, int waves, const Slab &s, bool check) {
+template <bool kVec, bool kCheck>
+int launch_pupdate_u(hpccg_ctx *ctx, int waves, int unroll, const Slab &s, double *po) {
+    switch (unroll) {
+        case 1: return launch_pupdate_t<kVec, kCheck, 1>(ctx, waves, s, po);
+        case 2: return launch_pupdate_t<kVec, kCheck, 2>(ctx, waves, s, po);
+        default: return launch_pupdate_t<kVec, kCheck, 4>(ctx, waves, s, po);
+    }
+}
+
+int launch_pupdate(hpccg_ctx *ctx, int waves, int unroll, const Slab &s, bool check) {
     double *po = s.p + s.plane;
     const bool vec = aligned16(s.r) && aligned16(po);
     if (vec)
-        return check ? launch_pupdate_t<true, true>(ctx, waves, s, po)
-                     : launch_pupdate_t<true, false>(ctx, waves, s, po);
-    return check ? launch_pupdate_t<false, true>(ctx, waves, s, po)
-                 : launch_pupdate_t<false, false>(ctx, waves, s, po);
+        return check ? launch_pupdate_u<true, true>(ctx, waves, unroll, s, po)
+                     : launch_pupdate_u<true, false>(ctx, waves, unroll, s, po);
+    return check ? launch_pupdate_u<false, true>(ctx, waves, 1, s, po)
+                 : launch_pupdate_u<false, false>(ctx, waves, 1, s, po);
 }
 
-template <bool kVec, bool kCheck>
+template <bool kVec, bool kCheck, int kU>
 int launch_update_t(hpccg_ctx *ctx, int waves, int64_t cap, const UpdArgs &a) {
-    auto k = cg_update_kernel<kVec, kCheck>;
-    const int g = vec_grid(ctx, k, kVec ? cdiv(a.n, 2) : a.n, waves, cap);
+    auto k = cg_update_kernel<kVec, kCheck, kU>;
+    const int g = vec_grid(ctx, k, kVec ? cdiv(a.n, 2 * kU) : a.n, waves, cap);
     k<<<g, kBlock, 0, ctx->stream>>>(a);
     return check_launch(ctx);
 }
 
-int launch_update(hpccg_ctx *ctx, int waves, int64_t cap, const Slab &s, int single, bool check,
-                  unsigned long long cond) {
+template <bool kVec, bool kCheck>
+int launch_update_u(hpccg_ctx *ctx, int waves, int unroll, int64_t cap, const UpdArgs &a) {
+    switch (unroll) {
+        case 1: return launch_update_t<kVec, kCheck, 1>(ctx, waves, cap, a);
+        case 2: return launch_update_t<kVec, kCheck, 2>(ctx, waves, cap, a);
+        default: return launch_update_t<kVec, kCheck, 4>(ctx, waves, cap, a);
+    }
+}
+
+int launch_update(hpccg_ctx *ctx, int waves, int unroll, int64_t cap, const Slab &s, int single,
+                  bool check, unsigned long long cond) {
     UpdArgs a{};
     a.n = s.n;
     a.x = s.x;
@@ -408,10 +427,10 @@ int launch_update(hpccg_ctx *ctx, int waves, int64_t cap, const Slab &s, int sin
     a.cond = cond;
     const bool vec = aligned16(a.x) && aligned16(a.r) && aligned16(a.p) && aligned16(a.Ap);
     if (vec)
-        return check ? launch_update_t<true, true>(ctx, waves, cap, a)
-                     : launch_update_t<true, false>(ctx, waves, cap, a);
-    return check ? launch_update_t<false, true>(ctx, waves, cap, a)
-                 : launch_update_t<false, false>(ctx, waves, cap, a);
+        return check ? launch_update_u<true, true>(ctx, waves, unroll, cap, a)
+                     : launch_update_u<true, false>(ctx, waves, unroll, cap, a);
+    return check ? launch_update_u<false, true>(ctx, waves, 1, cap, a)
+                 : launch_update_u<false, false>(ctx, waves, 1, cap, a);
 }
 
 // CG SpMV of every slab with the p.Ap epilogue.  Multi-slab: the rows that
@@ -498,7 +517,8 @@ int enqueue_iteration(hpccg_problem *p, bool timing, bool check, unsigned long l
     const int single = ctx->mode == MODE_SINGLE;
     {
         PhaseTimer t(p, ctx->stream, PH_PUPDATE, timing);
-        for (const Slab &s : p->slabs) CHECK(launch_pupdate(ctx, p->opt_vec_waves, s, check));
+        for (const Slab &s : p->slabs)
+            CHECK(launch_pupdate(ctx, p->opt_vec_waves, p->opt_unroll, s, check));
     }
     CHECK(cg_spmv_all(p, timing, check));
     CHECK(allreduce_cg(p, false, timing));
@@ -507,8 +527,8 @@ int enqueue_iteration(hpccg_problem *p, bool timing, bool check, unsigned long l
         // every slab computes the same (allreduced) decision; slab 0 drives the
         // while-graph condition
         for (size_t i = 0; i < p->slabs.size(); ++i)
-            CHECK(launch_update(ctx, p->opt_vec_waves, p->red_cap, p->slabs[i], single, check,
-                                i == 0 ? cond : 0ull));
+            CHECK(launch_update(ctx, p->opt_vec_waves, p->opt_unroll, p->red_cap, p->slabs[i],
+                                single, check, i == 0 ? cond : 0ull));
     }
     CHECK(allreduce_cg(p, true, timing));
     return HPCCG_OK;
@@ -1117,6 +1137,10 @@ int hpccg_set_option(hpccg_problem *p, int key, int64_t value) {
             return HPCCG_OK;
         case HPCCG_OPT_WHILE: p->opt_while = value != 0; return HPCCG_OK;
         case HPCCG_OPT_L2_PERSIST: p->opt_l2 = value != 0; return HPCCG_OK;
+        case HPCCG_OPT_VEC_UNROLL:
+            if (value != 1 && value != 2 && value != 4) return fail(HPCCG_EINVAL, "unroll: 1, 2 or 4");
+            p->opt_unroll = (int)value;
+            return HPCCG_OK;
         case HPCCG_OPT_SPMV_ROWS:
             if (value != 1 && value != 2) return fail(HPCCG_EINVAL, "spmv rows must be 1 or 2");
             p->opt_rows = (int)value;

@@ -375,7 +375,10 @@ __device__ __forceinline__ int64_t gtid() { return (int64_t)blockIdx.x * kBlock 
 __device__ __forceinline__ int64_t gnth() { return (int64_t)gridDim.x * kBlock; }
 
 // a.6: p = r + beta p  (k == 1: p = r)            -- 24n B
-template <bool kVec, bool kCheck>
+// kU: 16-B units per thread per trip, all loads issued before any store
+// (memory-level parallelism for DRAM-resident vectors).  The per-thread
+// element order is the same for every kU, so kU never changes the bits.
+template <bool kVec, bool kCheck, int kU>
 __global__ void __launch_bounds__(kBlock) cg_pupdate_kernel(int64_t n, const double *__restrict__ r,
                                                            double *__restrict__ p,
                                                            const CgScalars *sc) {
@@ -386,19 +389,31 @@ __global__ void __launch_bounds__(kBlock) cg_pupdate_kernel(int64_t n, const dou
     const int64_t tid = gtid(), nth = gnth();
     if (kVec) {
         const int64_t nv = n >> 1;
-        const double2 *r2 = reinterpret_cast<const double2 *>(r);
-        double2 *p2 = reinterpret_cast<double2 *>(p);
-        for (int64_t i = tid; i < nv; i += nth) {
-            const double2 ra = r2[i];
-            double2 pa = p2[i];
-            if (done) return;
-            if (first) {
-                pa = ra;
-            } else {
-                pa.x = fma(beta, pa.x, ra.x);
-                pa.y = fma(beta, pa.y, ra.y);
+        const double2 *__restrict__ r2 = reinterpret_cast<const double2 *>(r);
+        double2 *__restrict__ p2 = reinterpret_cast<double2 *>(p);
+        for (int64_t b = tid; b < nv; b += kU * nth) {
+            double2 ra[kU], pa[kU];
+#pragma unroll
+            for (int u = 0; u < kU; ++u) {
+                const int64_t i = b + u * nth;
+                if (i < nv) {
+                    ra[u] = r2[i];
+                    pa[u] = p2[i];
+                }
             }
-            p2[i] = pa;
+            if (done) return;
+#pragma unroll
+            for (int u = 0; u < kU; ++u) {
+                const int64_t i = b + u * nth;
+                if (i < nv) {
+                    double2 q = ra[u];
+                    if (!first) {
+                        q.x = fma(beta, pa[u].x, ra[u].x);
+                        q.y = fma(beta, pa[u].y, ra[u].y);
+                    }
+                    p2[i] = q;
+                }
+            }
         }
         if (done) return;
         if (tid == 0 && (n & 1)) {
@@ -428,7 +443,7 @@ __device__ __forceinline__ void set_cond(unsigned long long h, int cont) {
     if (h) cudaGraphSetConditional((cudaGraphConditionalHandle)h, cont ? 1u : 0u);
 }
 
-template <bool kVec, bool kCheck>
+template <bool kVec, bool kCheck, int kU>
 __global__ void __launch_bounds__(kBlock) cg_update_kernel(UpdArgs a) {
     CgScalars *sc = a.sc;
     // `done` is tested after each trip's loads (never in front of them); it
@@ -441,22 +456,37 @@ __global__ void __launch_bounds__(kBlock) cg_update_kernel(UpdArgs a) {
     double acc = 0.0, acc2 = 0.0;
     if (kVec) {
         const int64_t nv = a.n >> 1;
-        double2 *x2 = reinterpret_cast<double2 *>(a.x);
-        double2 *r2 = reinterpret_cast<double2 *>(a.r);
-        const double2 *p2 = reinterpret_cast<const double2 *>(a.p);
-        const double2 *q2 = reinterpret_cast<const double2 *>(a.Ap);
-        for (int64_t i = tid; i < nv; i += nth) {
-            double2 xa = x2[i], ra = r2[i];
-            const double2 pa = p2[i], qa = q2[i];
+        double2 *__restrict__ x2 = reinterpret_cast<double2 *>(a.x);
+        double2 *__restrict__ r2 = reinterpret_cast<double2 *>(a.r);
+        const double2 *__restrict__ p2 = reinterpret_cast<const double2 *>(a.p);
+        const double2 *__restrict__ q2 = reinterpret_cast<const double2 *>(a.Ap);
+        for (int64_t b = tid; b < nv; b += kU * nth) {
+            double2 xa[kU], ra[kU], pa[kU], qa[kU];
+#pragma unroll
+            for (int u = 0; u < kU; ++u) {
+                const int64_t i = b + u * nth;
+                if (i < nv) {
+                    xa[u] = x2[i];
+                    ra[u] = r2[i];
+                    pa[u] = p2[i];
+                    qa[u] = q2[i];
+                }
+            }
             if (done) return;
-            xa.x = fma(alpha, pa.x, xa.x);
-            xa.y = fma(alpha, pa.y, xa.y);
-            ra.x = fma(-alpha, qa.x, ra.x);
-            ra.y = fma(-alpha, qa.y, ra.y);
-            x2[i] = xa;
-            r2[i] = ra;
-            acc = fma(ra.x, ra.x, acc);
-            acc2 = fma(ra.y, ra.y, acc2);
+#pragma unroll
+            for (int u = 0; u < kU; ++u) {
+                const int64_t i = b + u * nth;
+                if (i < nv) {
+                    xa[u].x = fma(alpha, pa[u].x, xa[u].x);
+                    xa[u].y = fma(alpha, pa[u].y, xa[u].y);
+                    ra[u].x = fma(-alpha, qa[u].x, ra[u].x);
+                    ra[u].y = fma(-alpha, qa[u].y, ra[u].y);
+                    x2[i] = xa[u];
+                    r2[i] = ra[u];
+                    acc = fma(ra[u].x, ra[u].x, acc);
+                    acc2 = fma(ra[u].y, ra[u].y, acc2);
+                }
+            }
         }
         if (done) return;
         if (tid == 0 && (a.n & 1)) {
