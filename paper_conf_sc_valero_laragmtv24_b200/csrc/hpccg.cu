@@ -580,11 +580,16 @@ int enqueue_init(hpccg_problem *p, int max_iter, double tol, bool timing,
     return HPCCG_OK;
 }
 
-// L2 residency of the CG vectors (r, x, Ap, p: 32n B): an access-policy
-// window marks the arena "persisting" while the matrix stream is loaded with
-// an evict_first policy, so at sizes where the vectors fit (<= ~3.9M rows)
-// the vector kernels and the x gathers run out of L2.  Applied to the stream
-// (and so to every kernel captured into a graph) only for the solve.
+// L2 residency of the CG vectors (r, x, Ap, p: ~32n B): when they fit in the
+// persisting L2 set-aside (cudaDevAttrMaxPersistingL2CacheSize, 74.6 MB on
+// B200: n <= ~2.3M rows), an access-policy window marks the arena
+// "persisting" while the matrix stream is loaded evict_first, so the vector
+// kernels and the x gathers run out of L2 (measured at 128^3: 123.5 vs 132
+// us/iteration).  When they do not fit, a window would pin a fraction of one
+// vector and shrink the L2 for everything else (measured at 256^3: 1382 vs
+// 1038 us/iteration), so it is not applied.  Applied to the stream (and so
+// to every kernel captured into a graph) only for the solve; the set-aside
+// is released and the persisting lines reset afterwards.
 struct L2Window {
     hpccg_problem *p;
     bool on = false;
@@ -593,34 +598,40 @@ struct L2Window {
         hpccg_ctx *ctx = p->ctx;
         const Slab &s = p->slabs[0];
         if (!p->opt_l2 || ctx->max_persist_l2 <= 0 || ctx->max_window <= 0) return;
-        const size_t win = std::min<size_t>(s.arena_bytes, (size_t)ctx->max_window);
-        const size_t keep = std::min<size_t>(win, (size_t)ctx->max_persist_l2);
-        if (cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, keep) != cudaSuccess) {
+        if (s.arena_bytes > (size_t)ctx->max_persist_l2 || s.arena_bytes > (size_t)ctx->max_window)
+            return;
+        if (cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, s.arena_bytes) != cudaSuccess) {
             cudaGetLastError();
             return;
         }
         cudaStreamAttrValue v{};
         v.accessPolicyWindow.base_ptr = s.arena;
-        v.accessPolicyWindow.num_bytes = win;
-        v.accessPolicyWindow.hitRatio = (float)std::min(1.0, (double)keep / (double)win);
+        v.accessPolicyWindow.num_bytes = s.arena_bytes;
+        v.accessPolicyWindow.hitRatio = 1.0f;
         v.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
         v.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
         if (cudaStreamSetAttribute(ctx->stream, cudaStreamAttributeAccessPolicyWindow, &v) !=
             cudaSuccess) {
             cudaGetLastError();
+            cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, 0);
             return;
         }
         on = true;
         size_t got = 0;
-        kept = (cudaDeviceGetLimit(&got, cudaLimitPersistingL2CacheSize) == cudaSuccess) ? got : keep;
+        kept = (cudaDeviceGetLimit(&got, cudaLimitPersistingL2CacheSize) == cudaSuccess) ? got : 0;
     }
-    ~L2Window() {
+    // call after the solve's work has completed
+    void release() {
         if (!on) return;
+        on = false;
         cudaStreamAttrValue v{};
         v.accessPolicyWindow.num_bytes = 0;
         cudaStreamSetAttribute(p->ctx->stream, cudaStreamAttributeAccessPolicyWindow, &v);
+        cudaCtxResetPersistingL2Cache();
+        cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, 0);
         cudaGetLastError();
     }
+    ~L2Window() { release(); }
 };
 
 int build_graph(hpccg_problem *p) {
@@ -1279,6 +1290,7 @@ int hpccg_solve(hpccg_problem *p, int max_iter, double tol, int *niters, double 
     CU(cudaEventRecord(p->ev_t1, ctx->stream));
     CU(cudaStreamSynchronize(ctx->stream));
     CU(cudaGetLastError());
+    l2win.release();
 
     CgScalars hs;
     CU(cudaMemcpy(&hs, p->slabs[0].sc, sizeof hs, cudaMemcpyDeviceToHost));

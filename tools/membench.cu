@@ -61,6 +61,22 @@ __global__ void __launch_bounds__(256) triad_kernel(const double2 *__restrict__ 
     }
 }
 
+// CG-update-like: read x, r, p, q; write x, r (4R:2W), double2 units
+__global__ void __launch_bounds__(256) upd_kernel(double2 *__restrict__ x, double2 *__restrict__ r,
+                                                  const double2 *__restrict__ p, const double2 *__restrict__ q,
+                                                  int64_t n2, double al) {
+    const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const int64_t nth = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t i = tid; i < n2; i += nth) {
+        double2 xa = x[i], ra = r[i];
+        const double2 pa = p[i], qa = q[i];
+        xa.x += al * pa.x; xa.y += al * pa.y;
+        ra.x -= al * qa.x; ra.y -= al * qa.y;
+        x[i] = xa;
+        r[i] = ra;
+    }
+}
+
 template <class F>
 float timeit(F f, int reps) {
     cudaEvent_t e0, e1;
@@ -119,6 +135,25 @@ int main() {
         printf("{\"probe\": \"l2_read_%zuMB\", \"bytes\": %zu, \"ms\": %.4f, \"GBs\": %.1f}\n", mb, bytes, ms, bytes / ms / 1e6);
         ms = timeit([&] { triad_kernel<<<grid, 256>>>(a, b, c, m2); }, 20);
         printf("{\"probe\": \"l2_triad_%zuMB\", \"bytes\": %zu, \"ms\": %.4f, \"GBs\": %.1f}\n", mb, 3 * bytes, ms, 3 * bytes / ms / 1e6);
+    }
+    // array spacing: 4 arrays of 128 MiB in one allocation, separated by
+    // exactly 2^27 B vs. 2^27 B + a skew
+    {
+        const size_t seg = (size_t)1 << 27;
+        char *base;
+        cudaMalloc(&base, 4 * seg + 4 * (1 << 22));
+        cudaMemset(base, 0, 4 * seg + 4 * (1 << 22));
+        const int64_t m2 = seg / 16;
+        for (size_t skew : {(size_t)0, (size_t)4096, (size_t)65536 + 256, (size_t)(1 << 21) + 8192}) {
+            double2 *v[4];
+            for (int k = 0; k < 4; ++k) v[k] = (double2 *)(base + k * (seg + skew));
+            int og;
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&og, upd_kernel, 256, 0);
+            ms = timeit([&] { upd_kernel<<<sms * og, 256>>>(v[0], v[1], v[2], v[3], m2, 0.5); }, 10);
+            printf("{\"probe\": \"upd_4r2w_skew%zu\", \"bytes\": %zu, \"ms\": %.4f, \"GBs\": %.1f}\n", skew, 6 * seg, ms, 6 * seg / ms / 1e6);
+            ms = timeit([&] { upd_kernel<<<(unsigned)((m2 + 255) / 256), 256>>>(v[0], v[1], v[2], v[3], m2, 0.5); }, 10);
+            printf("{\"probe\": \"upd_4r2w_fullgrid_skew%zu\", \"bytes\": %zu, \"ms\": %.4f, \"GBs\": %.1f}\n", skew, 6 * seg, ms, 6 * seg / ms / 1e6);
+        }
     }
     return 0;
 }
