@@ -290,7 +290,10 @@ def run_ours(args, nx, ny, nz, iters, cfg_index, scaling):
         if spmv_n > 0 and spmv_ms > 0:
             avg_ms = spmv_ms / spmv_n
             ach = spmv_bytes / (avg_ms * 1e-3) * 1e-9
-            roof = {"bound": "hbm", "kernel": "spmv27_kernel<true>", "achieved": round(ach, 1),
+            roof = {"bound": "hbm",
+                    "kernel": "spmv27x2_kernel<dot> (2 rows/thread; spmv27_kernel<dot> if n or the "
+                              "plane is odd)",
+                    "achieved": round(ach, 1),
                     "peak": peak, "unit": "GB/s", "frac": round(ach / peak, 4),
                     "frac_of_8TBs_nominal": round(ach / 8000.0, 4),
                     "traffic": traffic_from_profiles(args.workload),
