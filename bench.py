@@ -356,13 +356,102 @@ def traffic_from_profiles(workload):
         return None
 
 
+def run_blas1(args):
+    """BASELINE configs[4]: JACC BLAS-1 sweep, AXPY x += alpha y (hpccg_waxpby(n, 1, x,
+    alpha, y, x)) and DOT (hpccg_ddot, host-synchronous like JACC's constructs)
+    on the paper's inputs round(rand*100), alpha = 2.5 (Fig. 2), n = 1e3..1e9
+    per GPU; multi-GPU: DOT sharded n per rank + NCCL allreduce inside hpccg_ddot."""
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+
+    import synth
+    from paper_conf_sc_valero_laragmtv24_b200 import dist as D
+    from paper_conf_sc_valero_laragmtv24_b200 import hpccg as H
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    uid = None
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        uid = D.broadcast_unique_id(H.hpccg_unique_id)
+    stream = torch.cuda.Stream()
+    ctx = H.Context(local, stream=stream.cuda_stream, rank=rank, nranks=world, unique_id=uid)
+    sizes = [10 ** k for k in range(3, 10)]
+    if args.blas1_max:
+        sizes = [s for s in sizes if s <= args.blas1_max]
+    rows = []
+    for n in sizes:
+        # seeded inputs generated once on the host (splitmix64), per-rank shard
+        gen = min(n, 1 << 24)
+        xh = synth.jacc_vector(gen, 42 + rank)
+        yh = synth.jacc_vector(gen, 43 + rank)
+        x = torch.from_numpy(np.resize(xh, n)).cuda() if n > gen else torch.from_numpy(xh).cuda()
+        y = torch.from_numpy(np.resize(yh, n)).cuda() if n > gen else torch.from_numpy(yh).cuda()
+        torch.cuda.synchronize()
+        reps = max(3, min(200, int(2e9 / (24 * n))))
+        for _ in range(args.warmup):
+            ctx.waxpby(n, 1.0, x, 2.5, y, x)
+            ctx.ddot(n, x, y)
+        # AXPY, host-synchronous per call
+        if world > 1:
+            dist.barrier()
+        t0 = time.perf_counter()
+        for _ in range(reps):
+            ctx.waxpby(n, 1.0, x, 2.5, y, x)
+        t_axpy = (time.perf_counter() - t0) / reps
+        if world > 1:
+            dist.barrier()
+        t0 = time.perf_counter()
+        for _ in range(reps):
+            res = ctx.ddot(n, x, y)
+        t_dot = (time.perf_counter() - t0) / reps
+        tt = torch.tensor([t_axpy, t_dot], dtype=torch.float64, device="cuda")
+        if world > 1:
+            dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        t_axpy, t_dot = float(tt[0]), float(tt[1])
+        # exactness: x stays integer-valued (multiples of 0.5 scaled) -> dot exact
+        xc = x.cpu().numpy()
+        exact = None
+        if world == 1 and n <= 10 ** 8:
+            exact = float(np.dot((2 * xc).astype(np.int64), y.cpu().numpy().astype(np.int64))) / 2
+        rows.append({"n_per_gpu": n, "axpy_us": round(t_axpy * 1e6, 2),
+                     "axpy_GBs": round(world * 24.0 * n / t_axpy / 1e9, 1),
+                     "dot_us": round(t_dot * 1e6, 2),
+                     "dot_GBs": round(world * 16.0 * n / t_dot / 1e9, 1),
+                     "dot_exact": (res == exact) if exact is not None else None})
+        del x, y
+        torch.cuda.empty_cache()
+    if rank == 0:
+        peak, src = peaks()
+        big = rows[-1]
+        line = {"metric": "JACC BLAS-1 AXPY+DOT fp64 HBM GB/s (host-synchronous calls)",
+                "value": round((24.0 + 16.0) * big["n_per_gpu"] * world /
+                               ((big["axpy_us"] + big["dot_us"]) * 1e-6) / 1e9, 1),
+                "unit": "GB/s", "n_gpus": world, "steps": None, "warmup": args.warmup,
+                "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+                "data": "synthetic round(rand*100), alpha 2.5 (Fig. 2, P:L70-L73)",
+                "config": {"workload": "blas1", "baseline_config": 4, "sizes": sizes,
+                           "parallelism": f"shard{world}"},
+                "sweep": rows, "peak_hbm_GBs": peak, "peak_source": src,
+                "gpu_launches_per_call": {"axpy": 1, "dot": 1}}
+        print(json.dumps(line), flush=True)
+    ctx.close()
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
-    ap.add_argument("--workload", choices=sorted(WORKLOADS), default="hpccg128")
+    ap.add_argument("--workload", choices=sorted(WORKLOADS) + ["blas1"], default="hpccg128")
+    ap.add_argument("--blas1-max", type=int, default=None, help="largest BLAS-1 n")
     ap.add_argument("--iters", type=int, default=None, help="override CG iterations per step")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-budget", type=float, default=12.0, help="seconds of oracle CG")
@@ -370,6 +459,12 @@ def main():
     args = ap.parse_args()
     if args.warmup < 3:
         raise SystemExit("--warmup must be >= 3")
+    if args.workload == "blas1":
+        if args.impl == "reference":
+            print(json.dumps({"impl": "reference", "unavailable":
+                              "the blas1 sweep has no oracle arm; run the default workload"}))
+            return 0
+        return run_blas1(args)
     nx, ny, nz, iters, cfg, scaling = WORKLOADS[args.workload]
     if args.iters:
         iters = args.iters
