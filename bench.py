@@ -455,7 +455,7 @@ def main():
     ap.add_argument("--iters", type=int, default=None, help="override CG iterations per step")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-budget", type=float, default=12.0, help="seconds of oracle CG")
-    ap.add_argument("--ref-iters", type=int, default=5, help="oracle iterations per reference step")
+    ap.add_argument("--ref-iters", type=int, default=20, help="oracle iterations per reference step")
     args = ap.parse_args()
     if args.warmup < 3:
         raise SystemExit("--warmup must be >= 3")
