@@ -81,6 +81,10 @@ extern "C" {
                                else 1 is used), 1 */
 #define HPCCG_OPT_VEC_UNROLL 8 /* CG vector kernels: 16-B units per thread per trip with
                                all loads in flight: 1, 2 or 4 (default 4) */
+#define HPCCG_OPT_PERSISTENT 9 /* single GPU: run the whole solve as ONE cooperative kernel
+                               (grid barriers between phases): 0 never, 1 (default) when
+                               nrow_local <= HPCCG_OPT_PERSIST_ROWS, 2 always */
+#define HPCCG_OPT_PERSIST_ROWS 10 /* threshold for HPCCG_OPT_PERSISTENT = 1 (default 65536) */
 #define HPCCG_OPT_VEC_WAVES 6 /* CG vector kernels: 0 one thread per 16-B unit; k > 0
                                (default 1): a persistent grid of k resident waves */
 
@@ -101,7 +105,8 @@ typedef struct hpccg_stats {
     int64_t iterations;     /* niters */
     int64_t kernel_launches;/* kernels this library enqueued during the solve */
     int64_t l2_persist_bytes; /* L2 set aside for the CG vectors during the solve (0: none) */
-    int64_t graph_mode;     /* 2 while-graph, 1 per-iteration graph, 0 plain launches */
+    int64_t graph_mode;     /* 3 persistent kernel, 2 while-graph, 1 per-iteration graph,
+                               0 plain launches */
 } hpccg_stats;
 
 HPCCG_API const char *hpccg_strerror(int code);

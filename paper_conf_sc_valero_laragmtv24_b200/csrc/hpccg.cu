@@ -106,6 +106,7 @@ struct Slab {
     size_t arena_bytes = 0;
     CgScalars *sc = nullptr;
     Reduction red{};
+    unsigned *bar = nullptr;  // grid barrier state of the persistent solve
 };
 
 struct TimedOp {
@@ -126,6 +127,8 @@ struct hpccg_problem {
     int opt_vec_waves = 1;  // 0: one thread per double2 (full grid); k: k resident waves
     int opt_rows = 2;       // SpMV rows per thread (2 when aligned, else 1)
     int opt_unroll = 4;     // CG vector kernels: 16-B units per thread per trip
+    int opt_persist = 1;    // 0 never, 1 auto (n <= opt_persist_rows), 2 always (single slab)
+    int64_t opt_persist_rows = 65536;
     // graph of one CG iteration (per-iteration replay) ...
     cudaGraphExec_t graph = nullptr;
     int64_t graph_kernels = 0;
@@ -634,6 +637,35 @@ struct L2Window {
     ~L2Window() { release(); }
 };
 
+// The whole solve in one cooperative kernel (small single-slab problems).
+int launch_persistent(hpccg_problem *p, int max_iter, double tol) {
+    hpccg_ctx *ctx = p->ctx;
+    const Slab &s = p->slabs[0];
+    PersistArgs a{};
+    a.n = s.n;
+    a.stride = s.n;
+    a.plane = s.plane;
+    a.val = s.val;
+    a.col = s.col;
+    a.b = s.b;
+    a.x = s.x;
+    a.r = s.r;
+    a.p = s.p;
+    a.Ap = s.Ap;
+    a.part_rr = s.red.partials;
+    a.part_pAp = s.red.partials + p->red_cap / 2;
+    a.bar = s.bar;
+    a.sc = s.sc;
+    a.max_iter = max_iter;
+    a.tol = tol;
+    int64_t g = std::min<int64_t>(cdiv(s.n, kBlock), wave(ctx, cg_persistent_kernel));
+    g = std::max<int64_t>(1, std::min<int64_t>(g, p->red_cap / 2));
+    void *args[] = {&a};
+    CU(cudaLaunchCooperativeKernel((const void *)cg_persistent_kernel, dim3((unsigned)g), dim3(kBlock),
+                                   args, 0, ctx->stream));
+    return check_launch(ctx);
+}
+
 int build_graph(hpccg_problem *p) {
     hpccg_ctx *ctx = p->ctx;
     if (p->graph) return HPCCG_OK;
@@ -753,6 +785,7 @@ void free_slab(Slab &s) {
     cudaFree(s.sc);
     cudaFree(s.red.partials);
     cudaFree(s.red.counter);
+    cudaFree(s.bar);
     s = Slab{};
 }
 
@@ -981,6 +1014,7 @@ int hpccg_generate(hpccg_ctx *ctx, int nx, int ny, int nz, hpccg_problem **out) 
         p->red_cap = parts;
         if ((rc = alloc_zero((void **)&s.red.partials, sizeof(double) * parts))) return bail(rc);
         if ((rc = alloc_zero((void **)&s.red.counter, sizeof(unsigned)))) return bail(rc);
+        if ((rc = alloc_zero((void **)&s.bar, 64 * sizeof(unsigned)))) return bail(rc);
 
         GenArgs g{};
         g.nx = nx;
@@ -1148,6 +1182,14 @@ int hpccg_set_option(hpccg_problem *p, int key, int64_t value) {
             return HPCCG_OK;
         case HPCCG_OPT_WHILE: p->opt_while = value != 0; return HPCCG_OK;
         case HPCCG_OPT_L2_PERSIST: p->opt_l2 = value != 0; return HPCCG_OK;
+        case HPCCG_OPT_PERSISTENT:
+            if (value < 0 || value > 2) return fail(HPCCG_EINVAL, "persistent: 0, 1 or 2");
+            p->opt_persist = (int)value;
+            return HPCCG_OK;
+        case HPCCG_OPT_PERSIST_ROWS:
+            if (value < 0) return fail(HPCCG_EINVAL, "persist rows must be >= 0");
+            p->opt_persist_rows = value;
+            return HPCCG_OK;
         case HPCCG_OPT_VEC_UNROLL:
             if (value != 1 && value != 2 && value != 4) return fail(HPCCG_EINVAL, "unroll: 1, 2 or 4");
             p->opt_unroll = (int)value;
@@ -1237,7 +1279,11 @@ int hpccg_solve(hpccg_problem *p, int max_iter, double tol, int *niters, double 
     CU(cudaSetDevice(ctx->device));
     const bool timing = p->opt_timing != 0;
     const bool use_graph = p->opt_graph && !timing;
-    bool use_while = use_graph && p->opt_while && ctx->mode != MODE_NCCL && !p->while_failed;
+    const bool use_persist = !timing && ctx->mode == MODE_SINGLE &&
+                             (p->opt_persist == 2 ||
+                              (p->opt_persist == 1 && p->slabs[0].n <= p->opt_persist_rows));
+    bool use_while = !use_persist && use_graph && p->opt_while && ctx->mode != MODE_NCCL &&
+                     !p->while_failed;
     p->ev_used = 0;
     p->timed.clear();
     const int64_t l0 = ctx->launches;
@@ -1246,10 +1292,12 @@ int hpccg_solve(hpccg_problem *p, int max_iter, double tol, int *niters, double 
         p->while_failed = true;  // keep the message in hpccg_last_error; fall back
         use_while = false;
     }
-    if (use_graph && !use_while) CHECK(build_graph(p));
+    if (use_graph && !use_while && !use_persist) CHECK(build_graph(p));
 
     CU(cudaEventRecord(p->ev_t0, ctx->stream));
-    if (use_while) {
+    if (use_persist) {
+        CHECK(launch_persistent(p, max_iter, tol));
+    } else if (use_while) {
         CU(cudaGraphLaunch(p->wgraph, ctx->stream));
     } else {
         CHECK(enqueue_init(p, max_iter, tol, timing, 0ull));
@@ -1314,7 +1362,7 @@ int hpccg_solve(hpccg_problem *p, int max_iter, double tol, int *niters, double 
     st.spmv_launches = hs.niters + 1;
     st.kernel_launches = ctx->launches - l0;
     st.l2_persist_bytes = (int64_t)l2win.kept;
-    st.graph_mode = use_while ? 2 : (use_graph ? 1 : 0);
+    st.graph_mode = use_persist ? 3 : (use_while ? 2 : (use_graph ? 1 : 0));
     p->stats = st;
     if (niters) *niters = hs.niters;
     if (normr) *normr = hs.normr;

@@ -564,6 +564,148 @@ __global__ void cg_initstate_kernel(CgScalars *sc, int max_iter, double tol,
     set_cond(cond, !done);
 }
 
+// ------------------------------------------- persistent single-kernel solve
+// For small single-GPU problems (configs[0], 20x30x10: everything fits in
+// L2 and each kernel boundary costs more than the work), the whole HPCCG
+// solve -- init and every iteration -- runs in ONE cooperative kernel: the
+// phases are separated by a grid barrier (3 per iteration), every block sums
+// the per-block partials itself in a fixed order (so all blocks hold
+// bit-identical scalars and take identical loop decisions), and the loop
+// control of A4/A11 is evaluated in registers.  Data written by other blocks
+// inside the kernel (p, the partials) is read through L2 (ld.global.cg):
+// L1 is not coherent within a launch.
+
+struct PersistArgs {
+    int64_t n, stride, plane;
+    const double *val;
+    const int *col;
+    const double *b;
+    double *x, *r, *p, *Ap;      // p: local-with-halo base
+    double *part_rr, *part_pAp;  // gridDim.x partials each
+    unsigned *bar;               // [0] arrivals, [32] generation (separate lines)
+    CgScalars *sc;
+    int max_iter;
+    double tol;
+};
+
+// Grid-wide barrier for a cooperative launch (all blocks co-resident):
+// arrival counter + generation flag, release/acquire at gpu scope.
+__device__ __forceinline__ void grid_barrier(unsigned *bar, unsigned nblocks) {
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        unsigned *count = bar, *gen = bar + 32;
+        unsigned g;
+        asm volatile("ld.acquire.gpu.u32 %0, [%1];" : "=r"(g) : "l"(gen) : "memory");
+        __threadfence();
+        unsigned t;
+        asm volatile("atom.add.acq_rel.gpu.u32 %0, [%1], 1;" : "=r"(t) : "l"(count) : "memory");
+        if (t == nblocks - 1) {
+            asm volatile("st.relaxed.gpu.u32 [%0], %1;" ::"l"(count), "r"(0u) : "memory");
+            asm volatile("st.release.gpu.u32 [%0], %1;" ::"l"(gen), "r"(g + 1) : "memory");
+        } else {
+            unsigned cur;
+            do {
+                asm volatile("ld.acquire.gpu.u32 %0, [%1];" : "=r"(cur) : "l"(gen) : "memory");
+            } while (cur == g);
+        }
+        __threadfence();
+    }
+    __syncthreads();
+}
+
+// Sum of the gridDim.x partials in a fixed order; identical in every block.
+__device__ __forceinline__ double sum_partials(const double *part, double *sh) {
+    double s = 0.0;
+    for (unsigned i = threadIdx.x; i < gridDim.x; i += kBlock) s += __ldcg(part + i);
+    __syncthreads();
+    s = block_reduce<false>(s, sh);
+    if (threadIdx.x == 0) sh[31] = s;
+    __syncthreads();
+    s = sh[31];
+    __syncthreads();
+    return s;
+}
+
+__device__ __forceinline__ double block_partial(double v, double *sh) {
+    v = block_reduce<false>(v, sh);  // valid in warp 0
+    __syncthreads();
+    return v;
+}
+
+__global__ void __launch_bounds__(kBlock, 1) cg_persistent_kernel(PersistArgs a) {
+    __shared__ double sh[32];
+    const int64_t tid = gtid(), nth = gnth();
+    const unsigned nb = gridDim.x;
+    double *po = a.p + a.plane;
+    auto spmv_row = [&](int64_t i) {
+        double s = 0.0;
+#pragma unroll 9
+        for (int k = 0; k < kSlots; ++k)
+            s = fma(__ldg(a.val + k * a.stride + i), __ldcg(a.p + __ldg(a.col + k * a.stride + i)), s);
+        return s;
+    };
+    // ---- init (a.7): p = x; Ap = A p; r = b - Ap; rtrans = r.r
+    for (int64_t i = tid; i < a.n; i += nth) po[i] = a.x[i];
+    grid_barrier(a.bar, nb);
+    double acc = 0.0;
+    for (int64_t i = tid; i < a.n; i += nth) {
+        const double ap = spmv_row(i);
+        const double rv = fma(-1.0, ap, a.b[i]);
+        a.r[i] = rv;
+        acc = fma(rv, rv, acc);
+    }
+    acc = block_partial(acc, sh);
+    if (threadIdx.x == 0) a.part_rr[blockIdx.x] = acc;
+    grid_barrier(a.bar, nb);
+    double rr = sum_partials(a.part_rr, sh);
+    double rtrans = rr, normr = sqrt(rtrans);
+    int niters = 0;
+    // ---- HPCCG loop (a.8, A4 lag, A11 guard)
+    for (int k = 1; k < a.max_iter && normr > a.tol; ++k) {
+        double beta = 0.0;
+        if (k > 1) {
+            const double old = rtrans;
+            rtrans = rr;
+            beta = rtrans / old;
+        }
+        for (int64_t i = tid; i < a.n; i += nth) po[i] = (k == 1) ? a.r[i] : fma(beta, po[i], a.r[i]);
+        normr = sqrt(rtrans);
+        grid_barrier(a.bar, nb);
+        double d = 0.0;
+        for (int64_t i = tid; i < a.n; i += nth) {
+            const double ap = spmv_row(i);
+            a.Ap[i] = ap;
+            d = fma(ap, po[i], d);
+        }
+        d = block_partial(d, sh);
+        if (threadIdx.x == 0) a.part_pAp[blockIdx.x] = d;
+        grid_barrier(a.bar, nb);
+        const double pAp = sum_partials(a.part_pAp, sh);
+        const bool stop = (rtrans == 0.0) || (pAp == 0.0);
+        const double alpha = stop ? 0.0 : rtrans / pAp;
+        acc = 0.0;
+        for (int64_t i = tid; i < a.n; i += nth) {
+            a.x[i] = fma(alpha, po[i], a.x[i]);
+            const double rv = fma(-alpha, a.Ap[i], a.r[i]);
+            a.r[i] = rv;
+            acc = fma(rv, rv, acc);
+        }
+        acc = block_partial(acc, sh);
+        if (threadIdx.x == 0) a.part_rr[blockIdx.x] = acc;
+        grid_barrier(a.bar, nb);
+        rr = sum_partials(a.part_rr, sh);
+        niters = k;
+        if (stop) break;
+    }
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+        a.sc->niters = niters;
+        a.sc->normr = normr;
+        a.sc->rr_cur = rr;
+        a.sc->rr_prev = rtrans;
+        a.sc->done = 1;
+    }
+}
+
 // Loopback allreduce: fixed rank-order sum (or max) of one scalar of every
 // slab, written back to every slab (deterministic, identical on all slabs).
 __global__ void slab_allreduce_kernel(const double *const *src, double *const *dst,

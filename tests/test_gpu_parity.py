@@ -243,6 +243,7 @@ def test_cg_modes_bitwise_identical_and_deterministic(ctx, minb):
     dims = (24, 20, 12)
     xs, outs = [], []
     with H.Problem(ctx, *dims) as p:
+        p.set_option(H.HPCCG_OPT_PERSISTENT, 0)
         p.set_option(H.HPCCG_OPT_SPMV_MINB, minb)
         for graph, timing, wh in [(1, 0, 1), (1, 0, 0), (0, 0, 0), (0, 1, 0), (1, 0, 1)]:
             p.set_vec(H.HPCCG_VEC_X, np.zeros(p.n))
@@ -266,6 +267,7 @@ def test_cg_tolerance_stop_in_both_graph_modes(ctx, wh):
     """tol > 0: the while-graph stops on the device; the per-iteration graph
     stops via the double-buffered host poll -- same niters / normr / x."""
     with H.Problem(ctx, 20, 30, 10) as p:
+        p.set_option(H.HPCCG_OPT_PERSISTENT, 0)
         p.set_option(H.HPCCG_OPT_WHILE, wh)
         r = p.solve(150, 1e-12)
         assert r["niters"] == 50
@@ -274,6 +276,41 @@ def test_cg_tolerance_stop_in_both_graph_modes(ctx, wh):
         assert st["kernel_launches"] >= 3 * 50
         r2 = p.solve(150, 1e-12)      # re-run from the converged x: 0 or few iterations
         assert r2["niters"] <= 2
+
+
+@pytest.mark.parametrize("dims", [(20, 30, 10), (3, 3, 3), (16, 16, 16), (33, 9, 3), (1, 1, 1),
+                                  (2, 2, 2), (64, 32, 40)])
+def test_cg_persistent_kernel_vs_oracle(ctx, dims):
+    """The whole solve in one cooperative kernel (grid barriers): same
+    tolerances against the oracle; tol stop, guard and max_iter semantics."""
+    with H.Problem(ctx, *dims) as p:
+        p.set_option(H.HPCCG_OPT_PERSISTENT, 2)
+        ref = oracle.generate(*dims)
+        tol = 0.0 if dims in [(1, 1, 1), (2, 2, 2)] else 1e-12
+        oref = oracle.cg(ref, 150, tol)
+        res = p.solve(150, tol)
+        assert p.stats()["graph_mode"] == 3 and p.stats()["kernel_launches"] == 1
+        check_cg(res, p.maxabsdiff(), oref, ref)
+        assert np.max(np.abs(p.get_vec(H.HPCCG_VEC_X) - oref["x"])) <= CG_ATOL
+        if dims == (20, 30, 10):
+            assert res["niters"] == 50
+        p.set_vec(H.HPCCG_VEC_X, np.zeros(p.n))
+        r = p.solve(7, 0.0)
+        assert r["niters"] == 6
+        o = oracle.cg(ref, 7, 0.0)
+        assert abs(r["normr"] - o["normr"]) <= CG_ATOL
+        p.set_vec(H.HPCCG_VEC_X, np.ones(p.n))
+        assert p.solve(50, 1e-12)["niters"] == 0
+
+
+def test_cg_persistent_auto_threshold(ctx):
+    with H.Problem(ctx, 20, 30, 10) as p:       # 6000 rows <= 65536: persistent
+        p.solve(150, 1e-12)
+        assert p.stats()["graph_mode"] == 3
+        p.set_option(H.HPCCG_OPT_PERSIST_ROWS, 1000)
+        p.set_vec(H.HPCCG_VEC_X, np.zeros(p.n))
+        p.solve(150, 1e-12)
+        assert p.stats()["graph_mode"] == 2
 
 
 def test_cg_first_step_exact(ctx):

@@ -8,7 +8,8 @@ from paper_conf_sc_valero_laragmtv24_b200 import hpccg as H
 KEYS = {"graph": H.HPCCG_OPT_GRAPH, "timing": H.HPCCG_OPT_TIMING, "while": H.HPCCG_OPT_WHILE,
         "minb": H.HPCCG_OPT_SPMV_MINB, "l2": H.HPCCG_OPT_L2_PERSIST, "waves": H.HPCCG_OPT_VEC_WAVES,
         "rows": H.HPCCG_OPT_SPMV_ROWS,
-        "unroll": H.HPCCG_OPT_VEC_UNROLL}
+        "unroll": H.HPCCG_OPT_VEC_UNROLL,
+        "persist": H.HPCCG_OPT_PERSISTENT}
 nx, ny, nz, iters = (int(v) for v in sys.argv[1:5])
 ctx = H.Context(0)
 p = H.Problem(ctx, nx, ny, nz)
@@ -39,6 +40,6 @@ for spec in sys.argv[5:]:
     print(json.dumps(out), flush=True)
     for k in opts:
         try:
-            p.set_option(KEYS[k], {"graph": 1, "while": 1, "l2": 1, "waves": 1, "rows": 2, "unroll": 4}.get(k, 0))
+            p.set_option(KEYS[k], {"graph": 1, "while": 1, "l2": 1, "waves": 1, "rows": 2, "unroll": 4, "persist": 1}.get(k, 0))
         except H.HpccgError:
             pass
