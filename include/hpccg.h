@@ -85,6 +85,9 @@ extern "C" {
                                (grid barriers between phases): 0 never, 1 (default) when
                                nrow_local <= HPCCG_OPT_PERSIST_ROWS, 2 always */
 #define HPCCG_OPT_PERSIST_ROWS 10 /* threshold for HPCCG_OPT_PERSISTENT = 1 (default 65536) */
+#define HPCCG_OPT_PDL 11    /* 1 (default): single GPU, launch the CG kernels with
+                               programmatic dependent launch (the SpMV starts its matrix
+                               stream while the p update drains); 0: off */
 #define HPCCG_OPT_VEC_WAVES 6 /* CG vector kernels: 0 one thread per 16-B unit; k > 0
                                (default 1): a persistent grid of k resident waves */
 

@@ -11,6 +11,7 @@
 #include <algorithm>
 #include <string>
 #include <unordered_map>
+#include <utility>
 #include <vector>
 
 #include "hpccg.h"
@@ -128,6 +129,7 @@ struct hpccg_problem {
     int opt_rows = 2;       // SpMV rows per thread (2 when aligned, else 1)
     int opt_unroll = 4;     // CG vector kernels: 16-B units per thread per trip
     int opt_persist = 1;    // 0 never, 1 auto (n <= opt_persist_rows), 2 always (single slab)
+    int opt_pdl = 1;        // programmatic dependent launch between the CG kernels
     int64_t opt_persist_rows = 65536;
     // graph of one CG iteration (per-iteration replay) ...
     cudaGraphExec_t graph = nullptr;
@@ -171,6 +173,24 @@ int check_launch(hpccg_ctx *ctx, int nkernels = 1) {
     if (e != cudaSuccess) return fail(HPCCG_ECUDA, "kernel launch failed: %s", cudaGetErrorString(e));
     ctx->launches += nkernels;
     return HPCCG_OK;
+}
+
+// Launch with optional programmatic dependent launch (PDL): the kernel may be
+// scheduled while its stream predecessor drains; it calls pdl_wait() before
+// touching anything that predecessor writes (kernels.cuh).
+template <typename... KArgs, typename... Args>
+cudaError_t launch_k(bool pdl, void (*kernel)(KArgs...), dim3 grid, cudaStream_t st, Args &&...args) {
+    cudaLaunchConfig_t cfg{};
+    cfg.gridDim = grid;
+    cfg.blockDim = dim3(kBlock);
+    cfg.dynamicSmemBytes = 0;
+    cfg.stream = st;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = pdl ? at : nullptr;
+    cfg.numAttrs = pdl ? 1 : 0;
+    return cudaLaunchKernelEx(&cfg, kernel, std::forward<Args>(args)...);
 }
 
 template <class K>
@@ -314,12 +334,13 @@ SpmvArgs spmv_args(const Slab &s, const double *x, double *y) {
 constexpr int kSpmvMinBDefault = 4;
 
 template <bool kDot, bool kCheck>
-int launch_spmv_t(hpccg_ctx *ctx, int minb, const SpmvArgs &a, unsigned blocks, cudaStream_t st) {
+int launch_spmv_t(hpccg_ctx *ctx, int minb, const SpmvArgs &a, unsigned blocks, cudaStream_t st,
+                  bool pdl) {
     switch (minb) {
-        case 1: spmv27_kernel<kDot, kCheck, 1><<<blocks, kBlock, 0, st>>>(a); break;
-        case 3: spmv27_kernel<kDot, kCheck, 3><<<blocks, kBlock, 0, st>>>(a); break;
-        case 4: spmv27_kernel<kDot, kCheck, 4><<<blocks, kBlock, 0, st>>>(a); break;
-        default: spmv27_kernel<kDot, kCheck, 2><<<blocks, kBlock, 0, st>>>(a); break;
+        case 1: launch_k(pdl, spmv27_kernel<kDot, kCheck, 1>, dim3(blocks), st, a); break;
+        case 3: launch_k(pdl, spmv27_kernel<kDot, kCheck, 3>, dim3(blocks), st, a); break;
+        case 4: launch_k(pdl, spmv27_kernel<kDot, kCheck, 4>, dim3(blocks), st, a); break;
+        default: launch_k(pdl, spmv27_kernel<kDot, kCheck, 2>, dim3(blocks), st, a); break;
     }
     return check_launch(ctx);
 }
@@ -337,7 +358,7 @@ int64_t spmv_blocks(int64_t len, int rows) { return cdiv(cdiv(len, rows), kBlock
 
 template <bool kDot>
 int launch_spmv(hpccg_ctx *ctx, int minb, bool check, SpmvArgs a, int64_t r0, int64_t len0,
-                int64_t r1, int64_t len1, cudaStream_t st, int rows = 1) {
+                int64_t r1, int64_t len1, cudaStream_t st, int rows = 1, bool pdl = false) {
     a.r0 = r0;
     a.len0 = len0;
     a.r1 = r1;
@@ -347,13 +368,13 @@ int launch_spmv(hpccg_ctx *ctx, int minb, bool check, SpmvArgs a, int64_t r0, in
     if (blocks == 0) return HPCCG_OK;
     if (blocks > 0x7fffffffLL) return fail(HPCCG_EINVAL, "SpMV grid too large");
     if (rows == 2) {
-        if (check) spmv27x2_kernel<kDot, true><<<(unsigned)blocks, kBlock, 0, st>>>(a);
-        else spmv27x2_kernel<kDot, false><<<(unsigned)blocks, kBlock, 0, st>>>(a);
+        if (check) launch_k(pdl, spmv27x2_kernel<kDot, true>, dim3((unsigned)blocks), st, a);
+        else launch_k(pdl, spmv27x2_kernel<kDot, false>, dim3((unsigned)blocks), st, a);
         return check_launch(ctx);
     }
     if (minb <= 0) minb = kSpmvMinBDefault;
-    return check ? launch_spmv_t<kDot, true>(ctx, minb, a, (unsigned)blocks, st)
-                 : launch_spmv_t<kDot, false>(ctx, minb, a, (unsigned)blocks, st);
+    return check ? launch_spmv_t<kDot, true>(ctx, minb, a, (unsigned)blocks, st, pdl)
+                 : launch_spmv_t<kDot, false>(ctx, minb, a, (unsigned)blocks, st, pdl);
 }
 
 // y = A x for one slab over all rows (no dot).
@@ -373,51 +394,51 @@ int vec_grid(hpccg_ctx *ctx, K kernel, int64_t units, int waves, int64_t cap) {
 }
 
 template <bool kVec, bool kCheck, int kU>
-int launch_pupdate_t(hpccg_ctx *ctx, int waves, const Slab &s, double *po) {
+int launch_pupdate_t(hpccg_ctx *ctx, int waves, const Slab &s, double *po, bool pdl) {
     auto k = cg_pupdate_kernel<kVec, kCheck, kU>;
     const int g = vec_grid(ctx, k, kVec ? cdiv(s.n, 2 * kU) : s.n, waves, 0x7fffffff);
-    k<<<g, kBlock, 0, ctx->stream>>>(s.n, s.r, po, s.sc);
+    launch_k(pdl, k, dim3(g), ctx->stream, s.n, (const double *)s.r, po, (const CgScalars *)s.sc);
     return check_launch(ctx);
 }
 
 template <bool kVec, bool kCheck>
-int launch_pupdate_u(hpccg_ctx *ctx, int waves, int unroll, const Slab &s, double *po) {
+int launch_pupdate_u(hpccg_ctx *ctx, int waves, int unroll, const Slab &s, double *po, bool pdl) {
     switch (unroll) {
-        case 1: return launch_pupdate_t<kVec, kCheck, 1>(ctx, waves, s, po);
-        case 2: return launch_pupdate_t<kVec, kCheck, 2>(ctx, waves, s, po);
-        default: return launch_pupdate_t<kVec, kCheck, 4>(ctx, waves, s, po);
+        case 1: return launch_pupdate_t<kVec, kCheck, 1>(ctx, waves, s, po, pdl);
+        case 2: return launch_pupdate_t<kVec, kCheck, 2>(ctx, waves, s, po, pdl);
+        default: return launch_pupdate_t<kVec, kCheck, 4>(ctx, waves, s, po, pdl);
     }
 }
 
-int launch_pupdate(hpccg_ctx *ctx, int waves, int unroll, const Slab &s, bool check) {
+int launch_pupdate(hpccg_ctx *ctx, int waves, int unroll, const Slab &s, bool check, bool pdl) {
     double *po = s.p + s.plane;
     const bool vec = aligned16(s.r) && aligned16(po);
     if (vec)
-        return check ? launch_pupdate_u<true, true>(ctx, waves, unroll, s, po)
-                     : launch_pupdate_u<true, false>(ctx, waves, unroll, s, po);
-    return check ? launch_pupdate_u<false, true>(ctx, waves, 1, s, po)
-                 : launch_pupdate_u<false, false>(ctx, waves, 1, s, po);
+        return check ? launch_pupdate_u<true, true>(ctx, waves, unroll, s, po, pdl)
+                     : launch_pupdate_u<true, false>(ctx, waves, unroll, s, po, pdl);
+    return check ? launch_pupdate_u<false, true>(ctx, waves, 1, s, po, pdl)
+                 : launch_pupdate_u<false, false>(ctx, waves, 1, s, po, pdl);
 }
 
 template <bool kVec, bool kCheck, int kU>
-int launch_update_t(hpccg_ctx *ctx, int waves, int64_t cap, const UpdArgs &a) {
+int launch_update_t(hpccg_ctx *ctx, int waves, int64_t cap, const UpdArgs &a, bool pdl) {
     auto k = cg_update_kernel<kVec, kCheck, kU>;
     const int g = vec_grid(ctx, k, kVec ? cdiv(a.n, 2 * kU) : a.n, waves, cap);
-    k<<<g, kBlock, 0, ctx->stream>>>(a);
+    launch_k(pdl, k, dim3(g), ctx->stream, a);
     return check_launch(ctx);
 }
 
 template <bool kVec, bool kCheck>
-int launch_update_u(hpccg_ctx *ctx, int waves, int unroll, int64_t cap, const UpdArgs &a) {
+int launch_update_u(hpccg_ctx *ctx, int waves, int unroll, int64_t cap, const UpdArgs &a, bool pdl) {
     switch (unroll) {
-        case 1: return launch_update_t<kVec, kCheck, 1>(ctx, waves, cap, a);
-        case 2: return launch_update_t<kVec, kCheck, 2>(ctx, waves, cap, a);
-        default: return launch_update_t<kVec, kCheck, 4>(ctx, waves, cap, a);
+        case 1: return launch_update_t<kVec, kCheck, 1>(ctx, waves, cap, a, pdl);
+        case 2: return launch_update_t<kVec, kCheck, 2>(ctx, waves, cap, a, pdl);
+        default: return launch_update_t<kVec, kCheck, 4>(ctx, waves, cap, a, pdl);
     }
 }
 
 int launch_update(hpccg_ctx *ctx, int waves, int unroll, int64_t cap, const Slab &s, int single,
-                  bool check, unsigned long long cond) {
+                  bool check, unsigned long long cond, bool pdl) {
     UpdArgs a{};
     a.n = s.n;
     a.x = s.x;
@@ -430,10 +451,10 @@ int launch_update(hpccg_ctx *ctx, int waves, int unroll, int64_t cap, const Slab
     a.cond = cond;
     const bool vec = aligned16(a.x) && aligned16(a.r) && aligned16(a.p) && aligned16(a.Ap);
     if (vec)
-        return check ? launch_update_u<true, true>(ctx, waves, unroll, cap, a)
-                     : launch_update_u<true, false>(ctx, waves, unroll, cap, a);
-    return check ? launch_update_u<false, true>(ctx, waves, 1, cap, a)
-                 : launch_update_u<false, false>(ctx, waves, 1, cap, a);
+        return check ? launch_update_u<true, true>(ctx, waves, unroll, cap, a, pdl)
+                     : launch_update_u<true, false>(ctx, waves, unroll, cap, a, pdl);
+    return check ? launch_update_u<false, true>(ctx, waves, 1, cap, a, pdl)
+                 : launch_update_u<false, false>(ctx, waves, 1, cap, a, pdl);
 }
 
 // CG SpMV of every slab with the p.Ap epilogue.  Multi-slab: the rows that
@@ -450,7 +471,8 @@ int cg_spmv_all(hpccg_problem *p, bool timing, bool check) {
         a.single = 1;
         a.part_base = 0;
         a.total_blocks = (unsigned)spmv_blocks(s.n, rows);
-        return launch_spmv<true>(ctx, minb, check, a, 0, s.n, 0, 0, ctx->stream, rows);
+        return launch_spmv<true>(ctx, minb, check, a, 0, s.n, 0, 0, ctx->stream, rows,
+                                 p->opt_pdl != 0);
     }
     const Slab &s0 = p->slabs[0];
     const int64_t n = s0.n, plane = s0.plane;
@@ -518,10 +540,13 @@ int allreduce_cg(hpccg_problem *p, bool rr, bool timing) {
 int enqueue_iteration(hpccg_problem *p, bool timing, bool check, unsigned long long cond) {
     hpccg_ctx *ctx = p->ctx;
     const int single = ctx->mode == MODE_SINGLE;
+    // PDL only between back-to-back kernels (single slab; the multi-slab
+    // iteration has copies / NCCL calls between its kernels)
+    const bool pdl = single && p->opt_pdl;
     {
         PhaseTimer t(p, ctx->stream, PH_PUPDATE, timing);
         for (const Slab &s : p->slabs)
-            CHECK(launch_pupdate(ctx, p->opt_vec_waves, p->opt_unroll, s, check));
+            CHECK(launch_pupdate(ctx, p->opt_vec_waves, p->opt_unroll, s, check, pdl));
     }
     CHECK(cg_spmv_all(p, timing, check));
     CHECK(allreduce_cg(p, false, timing));
@@ -531,7 +556,7 @@ int enqueue_iteration(hpccg_problem *p, bool timing, bool check, unsigned long l
         // while-graph condition
         for (size_t i = 0; i < p->slabs.size(); ++i)
             CHECK(launch_update(ctx, p->opt_vec_waves, p->opt_unroll, p->red_cap, p->slabs[i],
-                                single, check, i == 0 ? cond : 0ull));
+                                single, check, i == 0 ? cond : 0ull, pdl));
     }
     CHECK(allreduce_cg(p, true, timing));
     return HPCCG_OK;
@@ -1182,6 +1207,7 @@ int hpccg_set_option(hpccg_problem *p, int key, int64_t value) {
             return HPCCG_OK;
         case HPCCG_OPT_WHILE: p->opt_while = value != 0; return HPCCG_OK;
         case HPCCG_OPT_L2_PERSIST: p->opt_l2 = value != 0; return HPCCG_OK;
+        case HPCCG_OPT_PDL: p->opt_pdl = value != 0; return HPCCG_OK;
         case HPCCG_OPT_PERSISTENT:
             if (value < 0 || value > 2) return fail(HPCCG_EINVAL, "persistent: 0, 1 or 2");
             p->opt_persist = (int)value;

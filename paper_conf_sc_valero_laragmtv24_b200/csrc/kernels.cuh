@@ -89,6 +89,16 @@ __device__ __forceinline__ int2 ld_stream2(const int *ptr, uint64_t pol) {
     return v;
 }
 
+// Programmatic dependent launch (PDL): a kernel launched with the
+// programmatic-stream-serialization attribute may start while its
+// predecessor drains; pdl_wait() (griddepcontrol.wait) blocks until the
+// predecessor grid has completed and its writes are visible, and is a no-op
+// for an ordinary launch.  pdl_trigger() lets the successor be scheduled.
+// Before pdl_wait() a kernel may only read data no in-flight predecessor
+// writes (the matrix).
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;"); }
+
 __device__ __forceinline__ double warp_sum(double v) {
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
@@ -232,9 +242,10 @@ __global__ void __launch_bounds__(kBlock, kMinB) spmv27_kernel(SpmvArgs a) {
         lim = a.r1 + a.len1;
     }
     double d = 0.0;
-    // The done flag is read together with the first matrix loads and tested
-    // after them, so its latency never sits in front of the stream.
-    const int done = (kDot && kCheck) ? __ldg(&a.sc->done) : 0;
+    // The first matrix loads are issued before waiting for the predecessor
+    // (PDL) and before the done flag is read, so neither latency sits in
+    // front of the stream.
+    int done = 0;
     if (row < lim) {
         const uint64_t pol = policy_evict_first();
         const double *v = a.val + row;
@@ -254,7 +265,11 @@ __global__ void __launch_bounds__(kBlock, kMinB) spmv27_kernel(SpmvArgs a) {
                 vv[t] = ld_stream(v + (9 * g + t) * a.stride, pol);
                 cc[t] = ld_stream(c + (9 * g + t) * a.stride, pol);
             }
-            if (g == 0 && done) return;  // uniform over the grid, before any store
+            if (g == 0) {
+                pdl_wait();
+                if (kDot && kCheck) done = __ldg(&a.sc->done);
+                if (done) return;  // uniform over the grid, before any store
+            }
 #pragma unroll
             for (int t = 0; t < 9; ++t) {
                 const double xv = __ldg(a.x + cc[t]);
@@ -269,7 +284,11 @@ __global__ void __launch_bounds__(kBlock, kMinB) spmv27_kernel(SpmvArgs a) {
         // p_i: the diagonal slot's gathered value when that slot really is the
         // row's own column (always, for generated matrices); else reload it.
         if (kDot) d = sum * (cd == row + a.plane ? xd : __ldg(a.x + row + a.plane));
+    } else {
+        pdl_wait();
+        if (kDot && kCheck) done = __ldg(&a.sc->done);
     }
+    pdl_trigger();
     if (done) return;
     if (kDot) {
         CgScalars *sc = a.sc;
@@ -300,7 +319,7 @@ __global__ void __launch_bounds__(kBlock, 4) spmv27x2_kernel(SpmvArgs a) {
         lim = a.r1 + a.len1;
     }
     double d = 0.0;
-    const int done = (kDot && kCheck) ? __ldg(&a.sc->done) : 0;
+    int done = 0;
     if (row + 1 < lim) {
         const uint64_t pol = policy_evict_first();
         const double *v = a.val + row;
@@ -316,7 +335,11 @@ __global__ void __launch_bounds__(kBlock, 4) spmv27x2_kernel(SpmvArgs a) {
                 vv[t] = ld_stream2(v + (3 * g + t) * a.stride, pol);
                 cc[t] = ld_stream2(c + (3 * g + t) * a.stride, pol);
             }
-            if (g == 0 && done) return;  // uniform over the grid, before any store
+            if (g == 0) {
+                pdl_wait();
+                if (kDot && kCheck) done = __ldg(&a.sc->done);
+                if (done) return;  // uniform over the grid, before any store
+            }
 #pragma unroll
             for (int t = 0; t < 3; ++t) {
                 const double xa = __ldg(a.x + cc[t].x), xb = __ldg(a.x + cc[t].y);
@@ -338,6 +361,8 @@ __global__ void __launch_bounds__(kBlock, 4) spmv27x2_kernel(SpmvArgs a) {
         }
     } else if (row < lim) {  // odd tail: one row, scalar loads
         const uint64_t pol = policy_evict_first();
+        pdl_wait();
+        if (kDot && kCheck) done = __ldg(&a.sc->done);
         if (done) return;
         double s0 = 0.0;
 #pragma unroll
@@ -346,7 +371,11 @@ __global__ void __launch_bounds__(kBlock, 4) spmv27x2_kernel(SpmvArgs a) {
                      __ldg(a.x + ld_stream(a.col + k * a.stride + row, pol)), s0);
         a.y[row] = s0;
         if (kDot) d = s0 * __ldg(a.x + row + a.plane);
+    } else {
+        pdl_wait();
+        if (kDot && kCheck) done = __ldg(&a.sc->done);
     }
+    pdl_trigger();
     if (done) return;
     if (kDot) {
         CgScalars *sc = a.sc;
@@ -382,6 +411,8 @@ template <bool kVec, bool kCheck, int kU>
 __global__ void __launch_bounds__(kBlock) cg_pupdate_kernel(int64_t n, const double *__restrict__ r,
                                                            double *__restrict__ p,
                                                            const CgScalars *sc) {
+    pdl_wait();
+    pdl_trigger();
     // `done` is tested after each trip's loads (never in front of them)
     const int done = kCheck ? __ldg(&sc->done) : 0;
     const bool first = (__ldg(&sc->k) == 1);
@@ -446,6 +477,8 @@ __device__ __forceinline__ void set_cond(unsigned long long h, int cont) {
 template <bool kVec, bool kCheck, int kU>
 __global__ void __launch_bounds__(kBlock) cg_update_kernel(UpdArgs a) {
     CgScalars *sc = a.sc;
+    pdl_wait();
+    pdl_trigger();
     // `done` is tested after each trip's loads (never in front of them); it
     // is uniform over the grid, so every block leaves before the reduction.
     const int done = kCheck ? __ldg(&sc->done) : 0;
