@@ -129,9 +129,11 @@ HPCCG_API int hpccg_unique_id(void *out);
 
 /* Create a context on CUDA `device`.  `cuda_stream` (cudaStream_t, nullable)
  * is the stream all work is enqueued on; NULL = a library-created stream.
- * nranks == 1: single GPU, `unique_id` must be NULL.  nranks > 1: z-slab rank
+ * unique_id == NULL: single GPU (nranks must be 1).  Otherwise z-slab rank
  * `rank` of `nranks` over NCCL; `unique_id` = the bytes from hpccg_unique_id
- * on rank 0 (north_star "z-slab decomposition ... NCCL").  Collective. */
+ * on rank 0 (north_star "z-slab decomposition ... NCCL").  nranks == 1 with a
+ * unique_id runs the multi-GPU code path on a 1-rank communicator (testing).
+ * Collective. */
 HPCCG_API int hpccg_init(hpccg_ctx **ctx, int device, void *cuda_stream, int rank,
                int nranks, const void *unique_id);
 

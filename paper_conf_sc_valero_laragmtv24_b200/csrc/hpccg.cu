@@ -917,20 +917,22 @@ int hpccg_init(hpccg_ctx **out, int device, void *stream, int rank, int nranks,
                const void *unique_id) {
     if (!out || nranks < 1 || rank < 0 || rank >= nranks)
         return fail(HPCCG_EINVAL, "hpccg_init: bad rank/nranks");
-    if ((nranks == 1) != (unique_id == nullptr))
-        return fail(HPCCG_EINVAL, "hpccg_init: unique_id must be NULL iff nranks == 1");
+    if (nranks > 1 && unique_id == nullptr)
+        return fail(HPCCG_EINVAL, "hpccg_init: nranks > 1 needs the rank-0 unique_id");
     *out = nullptr;
     hpccg_ctx *c = new hpccg_ctx();
     c->rank = rank;
     c->nranks = nranks;
     c->nslabs = 1;
-    c->mode = nranks == 1 ? MODE_SINGLE : MODE_NCCL;
+    // nranks == 1 with a unique_id: a 1-rank NCCL communicator running the
+    // multi-GPU code path (halo split, NCCL allreduces, per-iteration graph)
+    c->mode = unique_id == nullptr ? MODE_SINGLE : MODE_NCCL;
     int rc = ctx_common_init(c, device, stream);
     if (rc != HPCCG_OK) {
         hpccg_finalize(c);
         return rc;
     }
-    if (nranks > 1) {
+    if (c->mode == MODE_NCCL) {
 #ifdef HPCCG_WITH_NCCL
         ncclUniqueId id;
         memcpy(&id, unique_id, sizeof id);

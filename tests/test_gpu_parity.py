@@ -361,6 +361,33 @@ def test_cg_loopback_matches_global_oracle(P):
         assert np.max(np.abs(p.get_vec(H.HPCCG_VEC_X) - oref["x"])) <= CG_ATOL
 
 
+@pytest.mark.parametrize("dims", [(20, 30, 10), (16, 12, 6), (24, 20, 1)])
+def test_nccl_one_rank_code_path(dims):
+    """A 1-rank NCCL communicator runs the multi-GPU code path on one GPU:
+    interior/boundary SpMV split, halo exchange (zero-fill at the global
+    boundary), NCCL allreduces inside a captured per-iteration graph, host
+    polling.  Same tolerances against the oracle as the single-GPU path;
+    bitwise SpMV through hpccg_spmv."""
+    uid = H.hpccg_unique_id()
+    with H.Context(0, rank=0, nranks=1, unique_id=uid) as c, H.Problem(c, *dims) as p:
+        ref = oracle.generate(*dims)
+        assert p.info["nnz_global"] == ref.nnz
+        nx, ny, _ = dims
+        x = synth.uniform(ref.n, 4)
+        y = torch.empty(ref.n, dtype=torch.float64, device="cuda")
+        p.spmv(dev(halo_vector(x, ref.n, nx * ny, 0, 1, fill=np.nan)), y)
+        np.testing.assert_array_equal(y.cpu().numpy(), oracle.spmv(ref, x))
+        oref = oracle.cg(ref, 150, 1e-12)
+        for timing in (0, 1):
+            p.set_option(H.HPCCG_OPT_TIMING, timing)
+            p.set_vec(H.HPCCG_VEC_X, np.zeros(p.n))
+            res = p.solve(150, 1e-12)
+            assert p.stats()["graph_mode"] == (0 if timing else 1)
+            check_cg(res, p.maxabsdiff(), oref, ref)
+        d = c.ddot(ref.n, dev(x), dev(x))
+        assert abs(d - oracle.ddot(x, x)) <= DDOT_RTOL * oracle.ddot(x, x)
+
+
 # ------------------------------------------- full sizes (bench launch config)
 
 def test_full_128cubed_sampled_spmv_and_solve(ctx):
