@@ -188,20 +188,27 @@ def hpccg_info(prob: int) -> dict:
     return {k: x.value for k, x in zip(keys, v)}
 
 
+def _sync_if_tensors(*args):
+    """Order after torch's pending work only when torch tensors are passed
+    (raw device pointers: the caller owns the ordering)."""
+    if any(not isinstance(a, int) for a in args):
+        _torch_sync()
+
+
 def hpccg_spmv(prob: int, x, y) -> None:
-    _torch_sync()
+    _sync_if_tensors(x, y)
     _check(lib().hpccg_spmv(prob, _ptr(x), _ptr(y)), "hpccg_spmv")
 
 
 def hpccg_ddot(ctx: int, n: int, x, y) -> float:
-    _torch_sync()
+    _sync_if_tensors(x, y)
     r = ctypes.c_double()
     _check(lib().hpccg_ddot(ctx, n, _ptr(x), _ptr(y), ctypes.byref(r)), "hpccg_ddot")
     return r.value
 
 
 def hpccg_waxpby(ctx: int, n: int, alpha: float, x, beta: float, y, w) -> None:
-    _torch_sync()
+    _sync_if_tensors(x, y, w)
     _check(lib().hpccg_waxpby(ctx, n, float(alpha), _ptr(x), float(beta), _ptr(y), _ptr(w)),
            "hpccg_waxpby")
 
