@@ -241,6 +241,49 @@ HPCCG_API int hpccg_maxabsdiff(hpccg_problem *prob, double *result);
 
 HPCCG_API void hpccg_free(hpccg_problem *prob);
 
+/* ---------------------------------------------------------------------------
+ * f1 -- the paper's own CG workload: Fig. 12, an
+ * unpreconditioned CG on a "diagonal-dominant tridiagonal" matrix
+ * held as three coefficient arrays a0 (sub), a1 (diag), a2 (super), read as
+ * tridiag(1, 4, 1) (A18); initial state r = p = b = 0.5 * 1, x = 0
+ * (P:L475-L484); the loop runs while cond = r.r > tol (A3) and at most
+ * max_iter times.  The paper times one iteration at SIZE = 1e8.
+ * Single GPU only (the paper's runs are single-device): ENOTSUP on a
+ * multi-rank or loopback context.
+ * ------------------------------------------------------------------------- */
+typedef struct hpccg_tri hpccg_tri;
+
+#define HPCCG_TRI_X 0
+#define HPCCG_TRI_B 1
+#define HPCCG_TRI_R 2
+#define HPCCG_TRI_P 3
+#define HPCCG_TRI_A0 4
+#define HPCCG_TRI_A1 5
+#define HPCCG_TRI_A2 6
+
+/* Generate the size-n system on the device (a0[0] = a2[n-1] = 0).  Caller
+ * frees with hpccg_tri_free.  EINVAL if n < 1. */
+HPCCG_API int hpccg_tri_generate(hpccg_ctx *ctx, int64_t n, hpccg_tri **out);
+
+/* Borrowed device pointer (n doubles) to X, B, R, P or a coefficient array. */
+HPCCG_API int hpccg_tri_vec(hpccg_tri *t, int which, double **dev_ptr);
+
+/* y = A x (Fig. 12 matvecmul): y_i = a0_i x_{i-1} + a1_i x_i + a2_i x_{i+1}
+ * over the existing terms, ascending column, fp64 FMA chain from +0.0 (A8).
+ * x, y: device, n doubles, not overlapping. */
+HPCCG_API int hpccg_tri_spmv(hpccg_tri *t, const double *x, double *y);
+
+/* Reset x = 0, r = p = b and run the CG.  variant 0: the iteration exactly as
+ * Fig. 12 writes it -- copy r_old, matvec, 5 dots, 3 axpys (axpy(i, a, x, y):
+ * x[i] += a*y[i]), 2 more copies -- with every scalar on the device; variant
+ * 1: fused (matvec + p.s, x/r update + r.r, p update).  Both run as one graph
+ * with a device-driven WHILE node.  *iters, *cond (last r.r), *ms (device
+ * time of the whole solve): HOST out, nullable. */
+HPCCG_API int hpccg_tri_solve(hpccg_tri *t, int max_iter, double tol, int variant, int *iters,
+                              double *cond, double *ms);
+
+HPCCG_API void hpccg_tri_free(hpccg_tri *t);
+
 #ifdef __cplusplus
 }
 #endif

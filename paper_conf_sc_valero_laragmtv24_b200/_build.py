@@ -35,7 +35,7 @@ def nvcc() -> str:
 
 def sources():
     return sorted(glob.glob(os.path.join(CSRC, "*.cu")) + glob.glob(os.path.join(CSRC, "*.cuh"))
-                  + [os.path.join(INCLUDE, "hpccg.h")])
+                  + glob.glob(os.path.join(CSRC, "*.inc")) + [os.path.join(INCLUDE, "hpccg.h")])
 
 
 def up_to_date() -> bool:

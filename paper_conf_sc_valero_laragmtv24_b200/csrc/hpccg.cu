@@ -16,6 +16,7 @@
 
 #include "hpccg.h"
 #include "kernels.cuh"
+#include "tridiag.cuh"
 
 #ifdef HPCCG_WITH_NCCL
 #include <nccl.h>
@@ -1435,3 +1436,5 @@ void hpccg_free(hpccg_problem *p) {
 }
 
 }  // extern "C"
+
+#include "tridiag_host.inc"

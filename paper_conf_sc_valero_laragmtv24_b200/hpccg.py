@@ -29,6 +29,8 @@ HPCCG_ENCCL = -4
 HPCCG_ENOTSUP = -5
 HPCCG_UNIQUE_ID_BYTES = 128
 HPCCG_VEC_X, HPCCG_VEC_B, HPCCG_VEC_XEXACT = 0, 1, 2
+HPCCG_TRI_X, HPCCG_TRI_B, HPCCG_TRI_R, HPCCG_TRI_P = 0, 1, 2, 3
+HPCCG_TRI_A0, HPCCG_TRI_A1, HPCCG_TRI_A2 = 4, 5, 6
 HPCCG_OPT_GRAPH, HPCCG_OPT_POLL, HPCCG_OPT_TIMING = 0, 1, 2
 HPCCG_OPT_SPMV_MINB, HPCCG_OPT_WHILE, HPCCG_OPT_L2_PERSIST, HPCCG_OPT_VEC_WAVES = 3, 4, 5, 6
 HPCCG_OPT_SPMV_ROWS, HPCCG_OPT_VEC_UNROLL = 7, 8
@@ -82,6 +84,12 @@ _SIGS = {
     "hpccg_get_stats": ([_vp, ctypes.POINTER(hpccg_stats)], _i),
     "hpccg_maxabsdiff": ([_vp, ctypes.POINTER(_d)], _i),
     "hpccg_free": ([_vp], None),
+    "hpccg_tri_generate": ([_vp, _i64, ctypes.POINTER(_vp)], _i),
+    "hpccg_tri_vec": ([_vp, _i, ctypes.POINTER(_vp)], _i),
+    "hpccg_tri_spmv": ([_vp, _vp, _vp], _i),
+    "hpccg_tri_solve": ([_vp, _i, _d, _i, ctypes.POINTER(_i), ctypes.POINTER(_d),
+                         ctypes.POINTER(_d)], _i),
+    "hpccg_tri_free": ([_vp], None),
 }
 
 
@@ -135,6 +143,18 @@ def _torch_sync():
             torch.cuda.current_stream().synchronize()
     except Exception:  # pragma: no cover
         pass
+
+
+class _CudaArray:
+    def __init__(self, ptr: int, n: int):
+        self.__cuda_array_interface__ = {"shape": (n,), "typestr": "<f8", "data": (ptr, False),
+                                         "version": 3, "strides": None}
+
+
+def device_view(ptr: int, n: int):
+    """torch view (no copy) of n doubles of library-owned device memory."""
+    import torch
+    return torch.as_tensor(_CudaArray(ptr, n), device="cuda")
 
 
 # ------------------------------------------------------------ C-named calls
@@ -346,6 +366,51 @@ class Problem:
     def free(self):
         if self.handle:
             hpccg_free(self.handle)
+            self.handle = 0
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.free()
+
+
+# ------------------------------------------------- f1: Fig. 12 tridiagonal CG
+
+class Tri:
+    """The paper's own CG workload (Fig. 12) on the device (hpccg_tri_*)."""
+
+    def __init__(self, ctx: Context, n: int):
+        self.ctx, self.n = ctx, n
+        h = _vp()
+        _check(lib().hpccg_tri_generate(ctx.handle, n, ctypes.byref(h)), "hpccg_tri_generate")
+        self.handle = h.value
+
+    def vec_ptr(self, which: int) -> int:
+        h = _vp()
+        _check(lib().hpccg_tri_vec(self.handle, which, ctypes.byref(h)), "hpccg_tri_vec")
+        return h.value
+
+    def spmv(self, x, y) -> None:
+        _sync_if_tensors(x, y)
+        _check(lib().hpccg_tri_spmv(self.handle, _ptr(x), _ptr(y)), "hpccg_tri_spmv")
+
+    def solve(self, max_iter: int, tol: float, variant: int = 1) -> dict:
+        it, cond, ms = ctypes.c_int(), ctypes.c_double(), ctypes.c_double()
+        _check(lib().hpccg_tri_solve(self.handle, max_iter, float(tol), variant, ctypes.byref(it),
+                                     ctypes.byref(cond), ctypes.byref(ms)), "hpccg_tri_solve")
+        return {"iters": it.value, "cond": cond.value, "ms": ms.value}
+
+    def view(self, which: int):
+        """Zero-copy torch view of a device vector (valid until free())."""
+        return device_view(self.vec_ptr(which), self.n)
+
+    def get(self, which: int) -> np.ndarray:
+        return self.view(which).cpu().numpy()
+
+    def free(self):
+        if self.handle:
+            lib().hpccg_tri_free(self.handle)
             self.handle = 0
 
     def __enter__(self):

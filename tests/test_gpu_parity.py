@@ -414,3 +414,76 @@ def test_full_128cubed_sampled_spmv_and_solve(ctx):
         r500 = p.solve(501, 0.0)
         assert r500["niters"] == 500
         assert p.maxabsdiff() < 1e-13 and 0 <= r500["normr"] < 1e-40
+
+
+# ------------------------------------------ f1: the paper's tridiagonal CG
+
+@pytest.mark.parametrize("n", [1, 2, 3, 1000, 100_003])
+def test_tri_generate_and_spmv_bitwise(ctx, n):
+    with H.Tri(ctx, n) as t:
+        ref = oracle.Tri(n)
+        np.testing.assert_array_equal(t.get(H.HPCCG_TRI_A0), ref.a0)
+        np.testing.assert_array_equal(t.get(H.HPCCG_TRI_A1), ref.a1)
+        np.testing.assert_array_equal(t.get(H.HPCCG_TRI_A2), ref.a2)
+        np.testing.assert_array_equal(t.get(H.HPCCG_TRI_B), ref.b)
+        x = synth.uniform(n, 12)
+        y = torch.empty(n, dtype=torch.float64, device="cuda")
+        t.spmv(dev(x), y)
+        np.testing.assert_array_equal(y.cpu().numpy(), oracle.tri_spmv(ref, x))
+
+
+@pytest.mark.parametrize("variant", [0, 1])
+@pytest.mark.parametrize("n,tol", [(1000, 1e-12), (100_003, 1e-20), (7, 1e-30), (3_000_000, 1e-24)])
+def test_tri_cg_vs_oracle(ctx, variant, n, tol):
+    """Fig. 12 as written (variant 0) and fused (variant 1) against the
+    oracle's Fig. 12: iterations +-1, x within 1e-10, final r.r <= tol."""
+    with H.Tri(ctx, n) as t:
+        ref = oracle.Tri(n)
+        o = oracle.tri_cg(ref, 300, tol)
+        g = t.solve(300, tol, variant)
+        assert abs(g["iters"] - o["iters"]) <= 1
+        assert g["cond"] <= tol
+        assert np.max(np.abs(t.get(H.HPCCG_TRI_X) - o["x"])) <= CG_ATOL
+
+
+@pytest.mark.parametrize("variant", [0, 1])
+def test_tri_cg_first_step_and_fixed_count(ctx, variant):
+    """max_iter 1: x1 = alpha/2 with alpha = n/(6n-2) correctly rounded (exact
+    integer dots); tol 0 runs exactly max_iter iterations."""
+    from fractions import Fraction
+    n = 12345
+    with H.Tri(ctx, n) as t:
+        g = t.solve(1, 0.0, variant)
+        assert g["iters"] == 1
+        alpha = float(Fraction(n, 6 * n - 2))
+        np.testing.assert_array_equal(t.get(H.HPCCG_TRI_X), np.full(n, alpha / 2))
+        g = t.solve(17, 0.0, variant)
+        assert g["iters"] == 17
+
+
+def test_tri_full_size_sampled(ctx):
+    """SIZE = 1e8: sampled SpMV rows bitwise; one Fig. 12 iteration of
+    each variant agrees with the exact first step on sampled entries."""
+    from fractions import Fraction
+    n = 100_000_000
+    with H.Tri(ctx, n) as t:
+        x = torch.empty(n, dtype=torch.float64, device="cuda").uniform_(-1, 1)
+        y = torch.empty(n, dtype=torch.float64, device="cuda")
+        t.spmv(x, y)
+        rows = synth.sample_rows(n, 500, 9)
+        xs = x.cpu().numpy()
+        exp = []
+        for i in rows:
+            s = 0.0
+            if i > 0:
+                s = float(Fraction(xs[i - 1]) + Fraction(s))
+            s = float(Fraction(4.0) * Fraction(xs[i]) + Fraction(s))
+            if i < n - 1:
+                s = float(Fraction(xs[i + 1]) + Fraction(s))
+            exp.append(s)
+        np.testing.assert_array_equal(y.cpu().numpy()[rows], np.array(exp))
+        alpha = float(Fraction(n, 6 * n - 2))
+        for v in (0, 1):
+            g = t.solve(1, 0.0, v)
+            xv = t.view(H.HPCCG_TRI_X)
+            assert g["iters"] == 1 and float(xv[rows].max()) == float(xv[rows].min()) == alpha / 2
