@@ -445,14 +445,81 @@ def run_blas1(args):
     return 0
 
 
+def run_tridiag(args):
+    """the paper's own CG measurement: one iteration of Fig. 12's CG
+    on the tridiagonal matrix of SIZE = 1e8.  Reports the
+    time per iteration of Fig. 12 as written (variant 0: 3 copies, 1 matvec,
+    5 dots, 3 axpys; 208n bytes) and fused (variant 1: 112n bytes), with the
+    CPU oracle's time per iteration beside it (the paper quotes GPU/CPU ratios:
+    68x A100, 17x MI100, 4x Max 1550 vs a 64-core EPYC 7742)."""
+    import torch
+
+    from paper_conf_sc_valero_laragmtv24_b200 import hpccg as H
+
+    if int(os.environ.get("WORLD_SIZE", "1")) > 1 and int(os.environ.get("RANK", "0")) != 0:
+        return 0          # single-device workload (P:L330): other ranks idle
+    n = args.tri_n
+    torch.cuda.set_device(int(os.environ.get("LOCAL_RANK", "0")))
+    ctx = H.Context(int(os.environ.get("LOCAL_RANK", "0")))
+    t = H.Tri(ctx, n)
+    K = 20
+    res = {}
+    with ClockSampler(int(os.environ.get("LOCAL_RANK", "0"))) as clk:
+        for v in (0, 1):
+            for _ in range(args.warmup):
+                t.solve(K + 1, 0.0, v)
+            one = min(t.solve(1, 0.0, v)["ms"] for _ in range(args.steps))
+            many = min(t.solve(K + 1, 0.0, v)["ms"] for _ in range(args.steps))
+            res[v] = (many - one) / K
+    l0 = ctx.launch_count
+    t.solve(K + 1, 0.0, 1)
+    launches = ctx.launch_count - l0
+    t.free()
+    peak, src = peaks()
+    cpu = None
+    if not args.no_cpu_baseline:
+        import oracle
+        tr = oracle.Tri(n)
+        o1 = oracle.tri_cg(tr, 1, 0.0)["seconds"]
+        o3 = oracle.tri_cg(tr, 3, 0.0)["seconds"]
+        cpu_ms = max((o3 - o1) / 2, o1 / 2) * 1e3
+        cpu = {"value": round(cpu_ms, 3), "unit": "ms/iteration", "cores": oracle.get_threads(),
+               "kind": "oracle", "sample": f"oracle Fig. 12 CG (C, OpenMP, compensated dots) at "
+                                           f"n = {n}, 3 iterations"}
+    fused_ms = res[1]
+    line = {"metric": "Fig. 12 CG time per iteration, tridiagonal SIZE = 1e8 (fp64)",
+            "value": round(fused_ms, 4), "unit": "ms/iteration", "higher_is_better": False,
+            "n_gpus": 1, "steps": args.steps, "warmup": args.warmup, "scaling": "none",
+            "vs_baseline": None, "dtype": "f64",
+            "data": "synthetic tridiag(1,4,1), r = p = 0.5 (Fig. 12, P:L475-L484; A18)",
+            "config": {"workload": "tridiag", "n": n, "variant": "fused (1 matvec+dot, "
+                       "1 update+dot, 1 p update)"},
+            "fig12_as_written_ms": round(res[0], 4),
+            "bytes_per_iteration": {"fused": 112 * n, "fig12": 208 * n},
+            "GBs": {"fused": round(112 * n / (fused_ms * 1e-3) / 1e9, 1),
+                    "fig12": round(208 * n / (res[0] * 1e-3) / 1e9, 1)},
+            "roofline": {"bound": "hbm", "achieved": round(112 * n / (fused_ms * 1e-3) / 1e9, 1),
+                         "peak": peak, "unit": "GB/s",
+                         "frac": round(112 * n / (fused_ms * 1e-3) / 1e9 / peak, 4),
+                         "peak_source": src},
+            "gpu_launches_per_iteration": launches / (K + 1),
+            "clocks": clk.summary(), "cpu_baseline": cpu,
+            "speedup_vs_cpu_oracle": (round(cpu["value"] / fused_ms, 1) if cpu else None)}
+    print(json.dumps(line), flush=True)
+    ctx.close()
+    return 0
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
-    ap.add_argument("--workload", choices=sorted(WORKLOADS) + ["blas1"], default="hpccg128")
+    ap.add_argument("--workload", choices=sorted(WORKLOADS) + ["blas1", "tridiag"],
+                    default="hpccg128")
     ap.add_argument("--blas1-max", type=int, default=None, help="largest BLAS-1 n")
+    ap.add_argument("--tri-n", type=int, default=100_000_000, help="tridiag SIZE (P:L475)")
     ap.add_argument("--iters", type=int, default=None, help="override CG iterations per step")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-budget", type=float, default=12.0, help="seconds of oracle CG")
@@ -460,6 +527,12 @@ def main():
     args = ap.parse_args()
     if args.warmup < 3:
         raise SystemExit("--warmup must be >= 3")
+    if args.workload == "tridiag":
+        if args.impl == "reference":
+            print(json.dumps({"impl": "reference", "unavailable":
+                              "tridiag reports the oracle in cpu_baseline; no separate arm"}))
+            return 0
+        return run_tridiag(args)
     if args.workload == "blas1":
         if args.impl == "reference":
             print(json.dumps({"impl": "reference", "unavailable":
