@@ -798,7 +798,11 @@ int alloc_zero(void **ptr, size_t bytes) {
         cudaGetLastError();
         return fail(HPCCG_ENOMEM, "cudaMalloc(%zu) failed: %s", bytes, cudaGetErrorString(e));
     }
+    // cudaMemset runs on the legacy default stream, which does NOT order with
+    // the library's non-blocking stream: wait for it, or a following kernel
+    // on our stream can race with (and be overwritten by) the zero fill.
     e = cudaMemset(*ptr, 0, bytes);
+    if (e == cudaSuccess) e = cudaDeviceSynchronize();
     if (e != cudaSuccess) return fail(HPCCG_ECUDA, "cudaMemset: %s", cudaGetErrorString(e));
     return HPCCG_OK;
 }
@@ -1189,8 +1193,11 @@ int hpccg_copy_matrix(const hpccg_problem *p, int slab, double *val_host, int32_
     if (slab < 0 || slab >= (int)p->slabs.size()) return fail(HPCCG_EINVAL, "bad slab");
     CU(cudaSetDevice(p->ctx->device));
     const Slab &s = p->slabs[slab];
-    CU(cudaMemcpy(val_host, s.val, sizeof(double) * kSlots * s.n, cudaMemcpyDeviceToHost));
-    CU(cudaMemcpy(col_host, s.col, sizeof(int) * kSlots * s.n, cudaMemcpyDeviceToHost));
+    CU(cudaMemcpyAsync(val_host, s.val, sizeof(double) * kSlots * s.n, cudaMemcpyDeviceToHost,
+                       p->ctx->stream));
+    CU(cudaMemcpyAsync(col_host, s.col, sizeof(int) * kSlots * s.n, cudaMemcpyDeviceToHost,
+                       p->ctx->stream));
+    CU(cudaStreamSynchronize(p->ctx->stream));
     return HPCCG_OK;
 }
 

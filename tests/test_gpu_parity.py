@@ -487,3 +487,16 @@ def test_tri_full_size_sampled(ctx):
             g = t.solve(1, 0.0, v)
             xv = t.view(H.HPCCG_TRI_X)
             assert g["iters"] == 1 and float(xv[rows].max()) == float(xv[rows].min()) == alpha / 2
+
+
+def test_generate_after_other_problems_large(ctx):
+    """Regression: the zero fill of a new allocation (legacy default stream)
+    must complete before the generation kernel on the library's non-blocking
+    stream -- a 512^3 problem generated after smaller ones once came out all
+    zeros.  Checked at 384 x 384 x 256 after two smaller problems."""
+    for dims in [(64, 64, 64), (200, 100, 50), (384, 384, 256)]:
+        with H.Problem(ctx, *dims) as p:
+            nx, ny, nz = dims
+            assert p.info["nnz_global"] == (3 * nx - 2) * (3 * ny - 2) * (3 * nz - 2)
+            b = p.get_vec(H.HPCCG_VEC_B)
+            assert float(b.sum()) == 28 * p.n - p.info["nnz_global"]
