@@ -110,6 +110,8 @@ struct Slab {
     CgScalars *sc = nullptr;
     Reduction red{};
     unsigned *bar = nullptr;  // grid barrier state of the persistent solve
+    double *spmv_parts = nullptr;  // per-block p.Ap partials (single slab)
+    int64_t spmv_nparts = 0;
 };
 
 struct TimedOp {
@@ -440,7 +442,7 @@ int launch_update_u(hpccg_ctx *ctx, int waves, int unroll, int64_t cap, const Up
 }
 
 int launch_update(hpccg_ctx *ctx, int waves, int unroll, int64_t cap, const Slab &s, int single,
-                  bool check, unsigned long long cond, bool pdl) {
+                  bool check, unsigned long long cond, bool pdl, int rows) {
     UpdArgs a{};
     a.n = s.n;
     a.x = s.x;
@@ -451,6 +453,10 @@ int launch_update(hpccg_ctx *ctx, int waves, int unroll, int64_t cap, const Slab
     a.red = s.red;
     a.single = single;
     a.cond = cond;
+    if (single) {  // p.Ap partials of the single-slab SpMV (see cg_spmv_all)
+        a.pAp_parts = s.spmv_parts;
+        a.n_parts = (unsigned)spmv_blocks(s.n, spmv_rows_per_thread(rows, spmv_args(s, s.p, s.Ap), 0, 0));
+    }
     const bool vec = aligned16(a.x) && aligned16(a.r) && aligned16(a.p) && aligned16(a.Ap);
     if (vec)
         return check ? launch_update_u<true, true>(ctx, waves, unroll, cap, a, pdl)
@@ -473,6 +479,7 @@ int cg_spmv_all(hpccg_problem *p, bool timing, bool check) {
         a.single = 1;
         a.part_base = 0;
         a.total_blocks = (unsigned)spmv_blocks(s.n, rows);
+        a.parts_only = s.spmv_parts;  // the update kernel finishes p.Ap
         return launch_spmv<true>(ctx, minb, check, a, 0, s.n, 0, 0, ctx->stream, rows,
                                  p->opt_pdl != 0);
     }
@@ -558,7 +565,7 @@ int enqueue_iteration(hpccg_problem *p, bool timing, bool check, unsigned long l
         // while-graph condition
         for (size_t i = 0; i < p->slabs.size(); ++i)
             CHECK(launch_update(ctx, p->opt_vec_waves, p->opt_unroll, p->red_cap, p->slabs[i],
-                                single, check, i == 0 ? cond : 0ull, pdl));
+                                single, check, i == 0 ? cond : 0ull, pdl, p->opt_rows));
     }
     CHECK(allreduce_cg(p, true, timing));
     return HPCCG_OK;
@@ -817,6 +824,7 @@ void free_slab(Slab &s) {
     cudaFree(s.red.partials);
     cudaFree(s.red.counter);
     cudaFree(s.bar);
+    cudaFree(s.spmv_parts);
     s = Slab{};
 }
 
@@ -1053,6 +1061,7 @@ int hpccg_generate(hpccg_ctx *ctx, int nx, int ny, int nz, hpccg_problem **out) 
         if ((rc = alloc_zero((void **)&s.red.partials, sizeof(double) * parts))) return bail(rc);
         if ((rc = alloc_zero((void **)&s.red.counter, sizeof(unsigned)))) return bail(rc);
         if ((rc = alloc_zero((void **)&s.bar, 64 * sizeof(unsigned)))) return bail(rc);
+        if ((rc = alloc_zero((void **)&s.spmv_parts, sizeof(double) * parts))) return bail(rc);
 
         GenArgs g{};
         g.nx = nx;

@@ -224,6 +224,10 @@ struct SpmvArgs {
     Reduction red;
     unsigned part_base, total_blocks;
     int single;             // 1: write the global pAp directly (no allreduce)
+    // single slab: write the per-block p.Ap partials here and skip the
+    // last-block finisher (its fence + ticket costs ~6 us per SpMV on B200);
+    // the update kernel sums the partials itself.  nullptr: finisher.
+    double *parts_only;
 };
 
 // kDot: CG variant with the p.Ap epilogue.  kCheck: return at once when the
@@ -291,6 +295,12 @@ __global__ void __launch_bounds__(kBlock, kMinB) spmv27_kernel(SpmvArgs a) {
     pdl_trigger();
     if (done) return;
     if (kDot) {
+        if (a.parts_only) {  // block partial only; the update kernel sums them
+            __shared__ double shp[32];
+            d = block_reduce<false>(d, shp);
+            if (threadIdx.x == 0) a.parts_only[a.part_base + blockIdx.x] = d;
+            return;
+        }
         CgScalars *sc = a.sc;
         const int single = a.single;
         grid_reduce<false>(d, a.red, a.part_base + blockIdx.x, a.total_blocks,
@@ -378,6 +388,12 @@ __global__ void __launch_bounds__(kBlock, 4) spmv27x2_kernel(SpmvArgs a) {
     pdl_trigger();
     if (done) return;
     if (kDot) {
+        if (a.parts_only) {  // block partial only; the update kernel sums them
+            __shared__ double shp[32];
+            d = block_reduce<false>(d, shp);
+            if (threadIdx.x == 0) a.parts_only[a.part_base + blockIdx.x] = d;
+            return;
+        }
         CgScalars *sc = a.sc;
         const int single = a.single;
         grid_reduce<false>(d, a.red, a.part_base + blockIdx.x, a.total_blocks,
@@ -464,6 +480,8 @@ struct UpdArgs {
     int64_t n;
     double *x, *r;
     const double *p, *Ap;
+    const double *pAp_parts;  // non-null: p.Ap = fixed-order sum of these
+    unsigned n_parts;
     CgScalars *sc;
     Reduction red;
     int single;
@@ -482,7 +500,21 @@ __global__ void __launch_bounds__(kBlock) cg_update_kernel(UpdArgs a) {
     // `done` is tested after each trip's loads (never in front of them); it
     // is uniform over the grid, so every block leaves before the reduction.
     const int done = kCheck ? __ldg(&sc->done) : 0;
-    const double rtrans = __ldg(&sc->rr_cur), pAp = __ldg(&sc->pAp);
+    const double rtrans = __ldg(&sc->rr_cur);
+    double pAp;
+    if (a.pAp_parts) {
+        // every block sums the SpMV's partials in the same fixed order, so
+        // every block holds the bit-identical p.Ap (no grid-wide finisher)
+        __shared__ double shq[32];
+        double q = 0.0;
+        for (unsigned i = threadIdx.x; i < a.n_parts; i += kBlock) q += __ldcg(a.pAp_parts + i);
+        q = block_reduce<false>(q, shq);
+        if (threadIdx.x == 0) shq[31] = q;
+        __syncthreads();
+        pAp = shq[31];
+    } else {
+        pAp = __ldg(&sc->pAp);
+    }
     const bool stop = (rtrans == 0.0) || (pAp == 0.0);  // A11
     const double alpha = stop ? 0.0 : rtrans / pAp;
     const int64_t tid = gtid(), nth = gnth();
@@ -542,7 +574,8 @@ __global__ void __launch_bounds__(kBlock) cg_update_kernel(UpdArgs a) {
     const int single = a.single;
     const unsigned long long cond = a.cond;
     grid_reduce<false>(acc, a.red, blockIdx.x, gridDim.x,
-                       [sc, single, rtrans, stop, cond](double s) {
+                       [sc, single, rtrans, stop, cond, pAp](double s) {
+                           sc->pAp = pAp;
                            sc->rr_prev = rtrans;
                            if (single) sc->rr_cur = s; else sc->loc_rr = s;
                            const int k = sc->k;

@@ -9,6 +9,8 @@
 #include <stdlib.h>
 #include <string.h>
 #include <vector>
+#include <cooperative_groups.h>
+namespace cgx = cooperative_groups;
 
 constexpr int S = 27;
 
@@ -347,6 +349,110 @@ __global__ void __launch_bounds__(kBlk, kMinB) vdot2(A a, Red red) {
     }
 }
 
+// 2 rows / thread + p.Ap with a CLUSTER-level pre-reduction: the 8 CTAs of a
+// cluster hand their partials to CTA 0 through DSMEM (+ a DSMEM atomic
+// arrival count); only CTA 0 does the global fence + ticket.
+template <int kCl>
+__global__ void __launch_bounds__(256, 4) vdot2c(A a, Red red) {
+    auto cluster = cgx::this_cluster();
+    __shared__ double cl_part[kCl];
+    __shared__ unsigned cl_count;
+    const unsigned crank = cluster.block_rank();
+    if (threadIdx.x == 0) cl_count = 0;
+    cluster.sync();  // CTA 0's counter initialised before anyone arrives
+    const int64_t r2 = ((int64_t)blockIdx.x * 256 + threadIdx.x) * 2;
+    const uint64_t pol = pol_ef();
+    double d = 0.0;
+    if (r2 < a.n) {
+        double s0 = 0.0, s1 = 0.0, x0 = 0.0, x1 = 0.0;
+#pragma unroll
+        for (int g = 0; g < 9; ++g) {
+            double2 vv[3];
+            int2 cc[3];
+#pragma unroll
+            for (int t = 0; t < 3; ++t) {
+                vv[t] = lds2(a.val + (3 * g + t) * a.stride + r2, pol);
+                cc[t] = lds2(a.col + (3 * g + t) * a.stride + r2, pol);
+            }
+#pragma unroll
+            for (int t = 0; t < 3; ++t) {
+                const double xa = __ldg(a.x + cc[t].x), xb = __ldg(a.x + cc[t].y);
+                if (3 * g + t == 13) { x0 = xa; x1 = xb; }
+                s0 = fma(vv[t].x, xa, s0);
+                s1 = fma(vv[t].y, xb, s1);
+            }
+        }
+        *reinterpret_cast<double2 *>(a.y + r2) = make_double2(s0, s1);
+        d = fma(s1, x1, s0 * x0);
+    }
+    __shared__ double sh[32];
+    __shared__ int last;
+    d = wsum(d);
+    if ((threadIdx.x & 31) == 0) sh[threadIdx.x >> 5] = d;
+    __syncthreads();
+    if (threadIdx.x < 32) {
+        d = threadIdx.x < 8 ? sh[threadIdx.x] : 0.0;
+        d = wsum(d);
+    }
+    if (crank != 0) {
+        if (threadIdx.x == 0) {
+            double *rp = cluster.map_shared_rank(cl_part, 0);
+            unsigned *rc = cluster.map_shared_rank(&cl_count, 0);
+            rp[crank] = d;
+            asm volatile("red.release.cluster.add.u32 [%0], 1;" ::"l"(rc) : "memory");
+        }
+        return;
+    }
+    if (threadIdx.x == 0) {
+        cl_part[0] = d;
+        unsigned c;
+        do {
+            asm volatile("ld.acquire.cluster.u32 %0, [%1];" : "=r"(c) : "l"(&cl_count) : "memory");
+        } while (c != kCl - 1);
+        double cs = 0.0;
+        for (int k = 0; k < kCl; ++k) cs += cl_part[k];
+        const unsigned ncl = gridDim.x / kCl;
+        red.partials[blockIdx.x / kCl] = cs;
+        __threadfence();
+        last = atomicAdd(red.counter, 1u) == ncl - 1;
+    }
+    __syncthreads();
+    if (!last) return;
+    __threadfence();
+    const unsigned ncl = gridDim.x / kCl;
+    double s = 0.0;
+    for (unsigned i = threadIdx.x; i < ncl; i += 256) s += __ldcg(red.partials + i);
+    s = wsum(s);
+    __syncthreads();
+    if ((threadIdx.x & 31) == 0) sh[threadIdx.x >> 5] = s;
+    __syncthreads();
+    if (threadIdx.x < 32) {
+        s = threadIdx.x < 8 ? sh[threadIdx.x] : 0.0;
+        s = wsum(s);
+        if (threadIdx.x == 0) {
+            *red.counter = 0;
+            *red.out = s;
+        }
+    }
+}
+
+template <int kCl>
+void launch_vdot2c(A a, Red red, int64_t n) {
+    const unsigned blocks = (unsigned)(((n / 2 + 255) / 256 + kCl - 1) / kCl * kCl);
+    cudaLaunchConfig_t cfg{};
+    cfg.gridDim = dim3(blocks);
+    cfg.blockDim = dim3(256);
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeClusterDimension;
+    at[0].val.clusterDim.x = kCl;
+    at[0].val.clusterDim.y = 1;
+    at[0].val.clusterDim.z = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    cudaError_t e = cudaLaunchKernelEx(&cfg, vdot2c<kCl>, a, red);
+    if (e != cudaSuccess) printf("launch error %s\n", cudaGetErrorString(e));
+}
+
 template <class F>
 float timeit(F f, int reps) {
     cudaEvent_t e0, e1;
@@ -449,6 +555,23 @@ int main(int argc, char **argv) {
     RUN("vdot2_b256_m4", (vdot2<256, 4><<<(unsigned)((n / 2 + 255) / 256), 256>>>(a, red)));
     RUN("vdot2_b512_m2", (vdot2<512, 2><<<(unsigned)((n / 2 + 511) / 512), 512>>>(a, red)));
     RUN("vdot2_b1024_m1", (vdot2<1024, 1><<<(unsigned)((n / 2 + 1023) / 1024), 1024>>>(a, red)));
+    RUN("vdot2c_cl2", (launch_vdot2c<2>(a, red, n)));
+    RUN("vdot2c_cl4", (launch_vdot2c<4>(a, red, n)));
+    RUN("vdot2c_cl8", (launch_vdot2c<8>(a, red, n)));
+    {
+        double h_out;
+        cudaMemcpy(&h_out, red.out, 8, cudaMemcpyDeviceToHost);
+        launch_vdot2c<8>(a, red, n);
+        double h2;
+        cudaDeviceSynchronize();
+        cudaMemcpy(&h2, red.out, 8, cudaMemcpyDeviceToHost);
+        vdot2<256, 4><<<(unsigned)((n / 2 + 255) / 256), 256>>>(a, red);
+        double h3;
+        cudaDeviceSynchronize();
+        cudaMemcpy(&h3, red.out, 8, cudaMemcpyDeviceToHost);
+        printf("{\"dot_cluster8\": %.17g, \"dot_flat\": %.17g, \"rel\": %.3g, \"err\": \"%s\"}\n", h2, h3,
+               (h2 - h3) / h3, cudaGetErrorString(cudaGetLastError()));
+    }
     RUN("v0_b256_m4_again", (v0<256, 4><<<g256, 256>>>(a)));
     for (int w : {1, 2, 4}) {
         int occ;
