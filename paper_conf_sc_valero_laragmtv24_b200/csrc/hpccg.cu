@@ -454,8 +454,25 @@ int launch_update(hpccg_ctx *ctx, int waves, int unroll, int64_t cap, const Slab
     a.single = single;
     a.cond = cond;
     if (single) {  // p.Ap partials of the single-slab SpMV (see cg_spmv_all)
-        a.pAp_parts = s.spmv_parts;
-        a.n_parts = (unsigned)spmv_blocks(s.n, spmv_rows_per_thread(rows, spmv_args(s, s.p, s.Ap), 0, 0));
+        const unsigned np =
+            (unsigned)spmv_blocks(s.n, spmv_rows_per_thread(rows, spmv_args(s, s.p, s.Ap), 0, 0));
+        if (np <= kUpdSumMax) {  // every update block sums them
+            a.pAp_parts = s.spmv_parts;
+            a.n_parts = np;
+        } else {  // one finisher block, then the update reads sc->pAp
+            void (*fk)(const double *, unsigned, CgScalars *) = cg_pap_finish_kernel;
+            cudaLaunchConfig_t cfg{};
+            cfg.gridDim = dim3(1);
+            cfg.blockDim = dim3(1024);
+            cfg.stream = ctx->stream;
+            cudaLaunchAttribute at[1];
+            at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+            at[0].val.programmaticStreamSerializationAllowed = 1;
+            cfg.attrs = pdl ? at : nullptr;
+            cfg.numAttrs = pdl ? 1 : 0;
+            cudaLaunchKernelEx(&cfg, fk, (const double *)s.spmv_parts, np, s.sc);
+            CHECK(check_launch(ctx));
+        }
     }
     const bool vec = aligned16(a.x) && aligned16(a.r) && aligned16(a.p) && aligned16(a.Ap);
     if (vec)

@@ -492,6 +492,26 @@ __device__ __forceinline__ void set_cond(unsigned long long h, int cont) {
     if (h) cudaGraphSetConditional((cudaGraphConditionalHandle)h, cont ? 1u : 0u);
 }
 
+// p.Ap from the SpMV's block partials when there are too many for every
+// update block to sum them (> kUpdSumMax): one 1024-thread block, fixed order.
+constexpr unsigned kUpdSumMax = 4096;
+
+__global__ void __launch_bounds__(1024) cg_pap_finish_kernel(const double *parts, unsigned n_parts,
+                                                             CgScalars *sc) {
+    pdl_wait();
+    pdl_trigger();
+    __shared__ double sh[32];
+    double q = 0.0;
+    for (unsigned i = threadIdx.x; i < n_parts; i += 1024) q += __ldcg(parts + i);
+    q = warp_sum(q);
+    if ((threadIdx.x & 31) == 0) sh[threadIdx.x >> 5] = q;
+    __syncthreads();
+    if (threadIdx.x < 32) {
+        q = warp_sum(sh[threadIdx.x]);
+        if (threadIdx.x == 0) sc->pAp = q;
+    }
+}
+
 template <bool kVec, bool kCheck, int kU>
 __global__ void __launch_bounds__(kBlock) cg_update_kernel(UpdArgs a) {
     CgScalars *sc = a.sc;
