@@ -215,6 +215,18 @@ HPCCG_API int hpccg_ddot(hpccg_ctx *ctx, int64_t n, const double *x, const doubl
 HPCCG_API int hpccg_waxpby(hpccg_ctx *ctx, int64_t n, double alpha, const double *x,
                  double beta, const double *y, double *w);
 
+/* f3 -- JACC's multidimensional constructs on 2-D arrays (Fig. 2):
+ * column-major m x n arrays with leading dimension ld >= m (element (i, j) at
+ * i + j*ld; only the m x n block is touched).  waxpby2d: w = alpha x + beta y
+ * with the canonical forms of hpccg_waxpby (JACC's 2-D axpy x[i,j] += alpha
+ * y[i,j] is waxpby2d(m, n, ld, 1, x, alpha, y, x)); ddot2d: *result (HOST) =
+ * sum over (i, j) of x[i,j] y[i,j] over all ranks (deterministic tree +
+ * allreduce).  Loopback: the per-rank arrays are stacked (ld*n doubles each). */
+HPCCG_API int hpccg_waxpby2d(hpccg_ctx *ctx, int64_t m, int64_t n, int64_t ld, double alpha,
+                             const double *x, double beta, const double *y, double *w);
+HPCCG_API int hpccg_ddot2d(hpccg_ctx *ctx, int64_t m, int64_t n, int64_t ld, const double *x,
+                           const double *y, double *result);
+
 /* a.2-a.8 -- HPCCG's unpreconditioned CG (the paper's loop Fig. 12
  * P:L450-L474; loop semantics A3/A4):
  *   p = x; Ap = A p; r = b - Ap; rtrans = r.r; normr = sqrt(rtrans)

@@ -1326,6 +1326,45 @@ int hpccg_waxpby(hpccg_ctx *ctx, int64_t n, double alpha, const double *x, doubl
     return HPCCG_OK;
 }
 
+// f3: grid of 32 x 8 blocks covering m x n, capped at ~2 waves (grid-stride beyond)
+static dim3 grid2d(int64_t m, int64_t n, int64_t cap_blocks) {
+    int64_t gx = std::max<int64_t>(1, std::min<int64_t>(cdiv(m, kB2x), 256));
+    int64_t gy = std::max<int64_t>(1, std::min<int64_t>(cdiv(n, kB2y), cap_blocks / gx));
+    gy = std::max<int64_t>(1, std::min<int64_t>(gy, 65535));
+    return dim3((unsigned)gx, (unsigned)gy);
+}
+
+int hpccg_waxpby2d(hpccg_ctx *ctx, int64_t m, int64_t n, int64_t ld, double alpha, const double *x,
+                   double beta, const double *y, double *w) {
+    if (!ctx || m < 0 || n < 0 || ld < m || (m > 0 && n > 0 && (!x || !y || !w)))
+        return fail(HPCCG_EINVAL, "hpccg_waxpby2d: bad argument");
+    if (m == 0 || n == 0) return HPCCG_OK;
+    CU(cudaSetDevice(ctx->device));
+    const int form = alpha == 1.0 ? 0 : (beta == 1.0 ? 1 : 2);
+    const dim3 g = grid2d(m, (int64_t)n * ctx->nslabs, 2 * 148 * 8), b(kB2x, kB2y);
+    const int64_t nn = (int64_t)n * ctx->nslabs;  // loopback: slabs stacked column-wise
+    if (form == 0) waxpby2d_kernel<0><<<g, b, 0, ctx->stream>>>(m, nn, ld, alpha, x, beta, y, w);
+    else if (form == 1) waxpby2d_kernel<1><<<g, b, 0, ctx->stream>>>(m, nn, ld, alpha, x, beta, y, w);
+    else waxpby2d_kernel<2><<<g, b, 0, ctx->stream>>>(m, nn, ld, alpha, x, beta, y, w);
+    CHECK(check_launch(ctx));
+    CU(cudaStreamSynchronize(ctx->stream));
+    return HPCCG_OK;
+}
+
+int hpccg_ddot2d(hpccg_ctx *ctx, int64_t m, int64_t n, int64_t ld, const double *x, const double *y,
+                 double *result) {
+    if (!ctx || !result || m < 0 || n < 0 || ld < m || (m > 0 && n > 0 && (!x || !y)))
+        return fail(HPCCG_EINVAL, "hpccg_ddot2d: bad argument");
+    CU(cudaSetDevice(ctx->device));
+    return api_reduce(ctx, false, result, [&](int s, double *out) {
+        const double *xs = x + (size_t)s * ld * n, *ys = y + (size_t)s * ld * n;
+        const dim3 g = grid2d(std::max<int64_t>(m, 1), std::max<int64_t>(n, 1),
+                              std::min<int64_t>(ctx->red_cap, 2 * 148 * 8));
+        dot2d_kernel<<<g, dim3(kB2x, kB2y), 0, ctx->stream>>>(m, n, ld, xs, ys, ctx->red, out);
+        return check_launch(ctx);
+    });
+}
+
 int hpccg_maxabsdiff(hpccg_problem *p, double *result) {
     if (!p || !result) return fail(HPCCG_EINVAL, "NULL argument");
     hpccg_ctx *ctx = p->ctx;

@@ -865,6 +865,47 @@ __global__ void __launch_bounds__(kBlock) dot_kernel(int64_t n, const double *x,
     grid_reduce<false>(acc, red, blockIdx.x, gridDim.x, [out](double s) { *out = s; });
 }
 
+// ----------------------------------------------- f3: JACC 2-D AXPY / DOT
+// JACC's multidimensional parallel_for / parallel_reduce over (M, N) on
+// column-major arrays with leading dimension ld (Fig. 2; the CUDA
+// back end uses 16x16 thread blocks, Fig. 6).  Here the blocks are
+// 32 x 8: threadIdx.x walks the contiguous row index i, so a warp reads one
+// 256-B segment of a column (coalesced); grid-stride in both dimensions.
+constexpr int kB2x = 32, kB2y = 8;
+
+template <int kForm>
+__global__ void __launch_bounds__(kB2x *kB2y) waxpby2d_kernel(int64_t m, int64_t n, int64_t ld,
+                                                              double alpha, const double *x,
+                                                              double beta, const double *y,
+                                                              double *w) {
+    auto op = [alpha, beta](double xv, double yv) {
+        if (kForm == 0) return fma(beta, yv, xv);
+        if (kForm == 1) return fma(alpha, xv, yv);
+        return fma(alpha, xv, beta * yv);
+    };
+    for (int64_t j = (int64_t)blockIdx.y * kB2y + threadIdx.y; j < n; j += (int64_t)gridDim.y * kB2y)
+        for (int64_t i = (int64_t)blockIdx.x * kB2x + threadIdx.x; i < m;
+             i += (int64_t)gridDim.x * kB2x) {
+            const int64_t k = i + j * ld;
+            w[k] = op(x[k], y[k]);
+        }
+}
+
+__global__ void __launch_bounds__(kB2x *kB2y) dot2d_kernel(int64_t m, int64_t n, int64_t ld,
+                                                           const double *x, const double *y,
+                                                           Reduction red, double *out) {
+    double acc = 0.0;
+    for (int64_t j = (int64_t)blockIdx.y * kB2y + threadIdx.y; j < n; j += (int64_t)gridDim.y * kB2y)
+        for (int64_t i = (int64_t)blockIdx.x * kB2x + threadIdx.x; i < m;
+             i += (int64_t)gridDim.x * kB2x) {
+            const int64_t k = i + j * ld;
+            acc = fma(__ldcs(x + k), __ldcs(y + k), acc);
+        }
+    // flatten the 2-D block into the 1-D reduction helpers (256 threads)
+    grid_reduce<false>(acc, red, blockIdx.y * gridDim.x + blockIdx.x, gridDim.x * gridDim.y,
+                       [out](double v) { *out = v; });
+}
+
 // a.9: max_i |x_i - xe_i| -> *out
 __global__ void __launch_bounds__(kBlock) maxabsdiff_kernel(int64_t n, const double *x,
                                                            const double *xe, Reduction red,

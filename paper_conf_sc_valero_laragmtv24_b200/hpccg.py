@@ -84,6 +84,8 @@ _SIGS = {
     "hpccg_get_stats": ([_vp, ctypes.POINTER(hpccg_stats)], _i),
     "hpccg_maxabsdiff": ([_vp, ctypes.POINTER(_d)], _i),
     "hpccg_free": ([_vp], None),
+    "hpccg_waxpby2d": ([_vp, _i64, _i64, _i64, _d, _vp, _d, _vp, _vp], _i),
+    "hpccg_ddot2d": ([_vp, _i64, _i64, _i64, _vp, _vp, ctypes.POINTER(_d)], _i),
     "hpccg_tri_generate": ([_vp, _i64, ctypes.POINTER(_vp)], _i),
     "hpccg_tri_vec": ([_vp, _i, ctypes.POINTER(_vp)], _i),
     "hpccg_tri_spmv": ([_vp, _vp, _vp], _i),
@@ -233,6 +235,19 @@ def hpccg_waxpby(ctx: int, n: int, alpha: float, x, beta: float, y, w) -> None:
            "hpccg_waxpby")
 
 
+def hpccg_waxpby2d(ctx: int, m: int, n: int, ld: int, alpha: float, x, beta: float, y, w) -> None:
+    _sync_if_tensors(x, y, w)
+    _check(lib().hpccg_waxpby2d(ctx, m, n, ld, float(alpha), _ptr(x), float(beta), _ptr(y),
+                                _ptr(w)), "hpccg_waxpby2d")
+
+
+def hpccg_ddot2d(ctx: int, m: int, n: int, ld: int, x, y) -> float:
+    _sync_if_tensors(x, y)
+    r = ctypes.c_double()
+    _check(lib().hpccg_ddot2d(ctx, m, n, ld, _ptr(x), _ptr(y), ctypes.byref(r)), "hpccg_ddot2d")
+    return r.value
+
+
 def hpccg_solve(prob: int, max_iter: int, tol: float) -> dict:
     ni, nr = ctypes.c_int(), ctypes.c_double()
     times = (ctypes.c_double * 6)()
@@ -278,6 +293,12 @@ class Context:
 
     def waxpby(self, n: int, alpha: float, x, beta: float, y, w) -> None:
         hpccg_waxpby(self.handle, n, alpha, x, beta, y, w)
+
+    def waxpby2d(self, m: int, n: int, ld: int, alpha: float, x, beta: float, y, w) -> None:
+        hpccg_waxpby2d(self.handle, m, n, ld, alpha, x, beta, y, w)
+
+    def ddot2d(self, m: int, n: int, ld: int, x, y) -> float:
+        return hpccg_ddot2d(self.handle, m, n, ld, x, y)
 
     @property
     def launch_count(self) -> int:

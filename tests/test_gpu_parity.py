@@ -500,3 +500,37 @@ def test_generate_after_other_problems_large(ctx):
             assert p.info["nnz_global"] == (3 * nx - 2) * (3 * ny - 2) * (3 * nz - 2)
             b = p.get_vec(H.HPCCG_VEC_B)
             assert float(b.sum()) == 28 * p.n - p.info["nnz_global"]
+
+
+# ------------------------------------------------ f3: JACC 2-D AXPY / DOT
+
+@pytest.mark.parametrize("m,n,ld", [(1000, 1000, 1000), (37, 23, 50), (1, 1, 1), (3000, 7, 3001),
+                                    (5, 40000, 8)])
+@pytest.mark.parametrize("alpha,beta", [(1.0, 2.5), (0.3, -0.7), (0.61, 1.0)])
+def test_2d_waxpby_bitwise_and_ld(ctx, m, n, ld, alpha, beta):
+    x, y = synth.uniform(ld * n, 5), synth.uniform(ld * n, 6)
+    xd, yd = dev(x), dev(y)
+    wd = dev(np.full(ld * n, 7.0))
+    ctx.waxpby2d(m, n, ld, alpha, xd, beta, yd, wd)
+    ref = oracle.waxpby2d(m, n, ld, alpha, x, beta, y, out=np.full(ld * n, 7.0))
+    np.testing.assert_array_equal(wd.cpu().numpy(), ref)
+
+
+@pytest.mark.parametrize("m,n,ld", [(1000, 1000, 1000), (37, 23, 50), (3000, 7, 3001), (5, 40000, 8)])
+def test_2d_ddot(ctx, m, n, ld):
+    x, y = synth.uniform(ld * n, 7), synth.uniform(ld * n, 8)
+    got = ctx.ddot2d(m, n, ld, dev(x), dev(y))
+    exp = oracle.ddot2d(m, n, ld, x, y)
+    X, Y = x.reshape(n, ld)[:, :m], y.reshape(n, ld)[:, :m]
+    assert abs(got - exp) <= DDOT_RTOL * max(abs(exp), np.abs(X * Y).sum() * 1e-4)
+
+
+def test_2d_fig2_example_exact(ctx):
+    """Fig. 2's multidimensional example: SIZE = 1000, round(rand*100), 2.5."""
+    m = n = 1000
+    x, y = synth.jacc_vector(m * n, 42), synth.jacc_vector(m * n, 43)
+    xd, yd = dev(x), dev(y)
+    ctx.waxpby2d(m, n, m, 1.0, xd, 2.5, yd, xd)
+    xo = oracle.waxpby2d(m, n, m, 1.0, x, 2.5, y)
+    np.testing.assert_array_equal(xd.cpu().numpy(), xo)
+    assert ctx.ddot2d(m, n, m, xd, yd) == oracle.ddot2d(m, n, m, xo, y)

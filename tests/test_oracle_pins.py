@@ -382,3 +382,34 @@ def test_cg_nonzero_initial_guess():
     res = oracle.cg(p, 50, 1e-12, x0=np.ones(p.n))
     assert res["niters"] == 0 and res["normr"] == 0.0
     np.testing.assert_array_equal(res["x"], np.ones(p.n))
+
+
+# ------------------------------------------------ f3: JACC 2-D AXPY / DOT
+
+def test_2d_axpy_dot_fig2_inputs_exact():
+    """Fig. 2's multidimensional example: SIZE = 1000,
+    round(rand*100) inputs, alpha = 2.5 -> AXPY and DOT exact."""
+    cfg = json.load(open(os.path.join(GOLDEN, "paper_inputs.json")))["fig2_blas1_2d"]
+    m = n = cfg["size"]
+    x, y = synth.jacc_vector(m * n, 42), synth.jacc_vector(m * n, 43)
+    w = oracle.waxpby2d(m, n, m, 1.0, x, 2.5, y)
+    np.testing.assert_array_equal(2 * w, (2 * x + 5 * y))
+    assert oracle.ddot2d(m, n, m, x, y) == float(int(np.dot(x.astype(np.int64), y.astype(np.int64))))
+
+
+def test_2d_leading_dimension_semantics():
+    """Only the m x n block of an ld x n column-major array is touched; the
+    result equals the 1-D routines on that block (numpy column-major slice)."""
+    m, n, ld = 37, 23, 50
+    x, y = synth.uniform(ld * n, 1), synth.uniform(ld * n, 2)
+    w = oracle.waxpby2d(m, n, ld, 0.3, x, -0.7, y)
+    X = x.reshape(n, ld).T
+    Y = y.reshape(n, ld).T
+    W = w.reshape(n, ld).T
+    np.testing.assert_array_equal(W[m:, :], X[m:, :])          # padding untouched
+    blk = oracle.waxpby(0.3, np.ascontiguousarray(X[:m, :].T).ravel(), -0.7,
+                        np.ascontiguousarray(Y[:m, :].T).ravel())
+    np.testing.assert_array_equal(np.ascontiguousarray(W[:m, :].T).ravel(), blk)
+    ex = sum(Fraction(a) * Fraction(b) for a, b in zip(X[:m, :].ravel(), Y[:m, :].ravel()))
+    got = oracle.ddot2d(m, n, ld, x, y)
+    assert abs(Fraction(got) - ex) <= abs(ex) * Fraction(2.0 ** -52)
