@@ -1360,7 +1360,7 @@ int hpccg_ddot2d(hpccg_ctx *ctx, int64_t m, int64_t n, int64_t ld, const double 
         const double *xs = x + (size_t)s * ld * n, *ys = y + (size_t)s * ld * n;
         const dim3 g = grid2d(std::max<int64_t>(m, 1), std::max<int64_t>(n, 1),
                               std::min<int64_t>(ctx->red_cap, 2 * 148 * 8));
-        dot2d_kernel<<<g, dim3(kB2x, kB2y), 0, ctx->stream>>>(m, n, ld, xs, ys, ctx->red, out);
+        dot2d_kernel<<<g, dim3(kB2x * kB2y), 0, ctx->stream>>>(m, n, ld, xs, ys, ctx->red, out);
         return check_launch(ctx);
     });
 }

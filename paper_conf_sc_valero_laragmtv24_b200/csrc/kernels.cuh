@@ -891,13 +891,15 @@ __global__ void __launch_bounds__(kB2x *kB2y) waxpby2d_kernel(int64_t m, int64_t
         }
 }
 
+// launched with 1-D blocks of kB2x*kB2y threads (the reduction helpers index
+// threads by threadIdx.x); (tx, ty) is the 32 x 8 tile position
 __global__ void __launch_bounds__(kB2x *kB2y) dot2d_kernel(int64_t m, int64_t n, int64_t ld,
                                                            const double *x, const double *y,
                                                            Reduction red, double *out) {
+    const int tx = threadIdx.x % kB2x, ty = threadIdx.x / kB2x;
     double acc = 0.0;
-    for (int64_t j = (int64_t)blockIdx.y * kB2y + threadIdx.y; j < n; j += (int64_t)gridDim.y * kB2y)
-        for (int64_t i = (int64_t)blockIdx.x * kB2x + threadIdx.x; i < m;
-             i += (int64_t)gridDim.x * kB2x) {
+    for (int64_t j = (int64_t)blockIdx.y * kB2y + ty; j < n; j += (int64_t)gridDim.y * kB2y)
+        for (int64_t i = (int64_t)blockIdx.x * kB2x + tx; i < m; i += (int64_t)gridDim.x * kB2x) {
             const int64_t k = i + j * ld;
             acc = fma(__ldcs(x + k), __ldcs(y + k), acc);
         }
