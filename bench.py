@@ -429,6 +429,35 @@ def run_blas1(args):
                      "dot_exact": (res == exact) if exact is not None else None})
         del x, y
         torch.cuda.empty_cache()
+    # f3: the 2-D constructs (Fig. 2) at SIZE x SIZE, SIZE = 1000 in the paper
+    rows2d = []
+    for size in [100, 1000, 10000, 31623]:
+        if args.blas1_max and size * size > args.blas1_max:
+            continue
+        n = size * size
+        gen = min(n, 1 << 24)
+        xh, yh = synth.jacc_vector(gen, 42 + rank), synth.jacc_vector(gen, 43 + rank)
+        x = torch.from_numpy(np.resize(xh, n)).cuda()
+        y = torch.from_numpy(np.resize(yh, n)).cuda()
+        torch.cuda.synchronize()
+        xp, yp = x.data_ptr(), y.data_ptr()
+        reps = max(3, min(200, int(2e9 / (24 * n))))
+        for _ in range(args.warmup):
+            ctx.waxpby2d(size, size, size, 1.0, xp, 2.5, yp, xp)
+            ctx.ddot2d(size, size, size, xp, yp)
+        t0 = time.perf_counter()
+        for _ in range(reps):
+            ctx.waxpby2d(size, size, size, 1.0, xp, 2.5, yp, xp)
+        ta = (time.perf_counter() - t0) / reps
+        t0 = time.perf_counter()
+        for _ in range(reps):
+            ctx.ddot2d(size, size, size, xp, yp)
+        td = (time.perf_counter() - t0) / reps
+        rows2d.append({"size": size, "axpy2d_us": round(ta * 1e6, 2),
+                       "axpy2d_GBs": round(world * 24.0 * n / ta / 1e9, 1),
+                       "dot2d_us": round(td * 1e6, 2), "dot2d_GBs": round(world * 16.0 * n / td / 1e9, 1)})
+        del x, y
+        torch.cuda.empty_cache()
     if rank == 0:
         peak, src = peaks()
         big = rows[-1]
@@ -440,7 +469,7 @@ def run_blas1(args):
                 "data": "synthetic round(rand*100), alpha 2.5 (Fig. 2, P:L70-L73)",
                 "config": {"workload": "blas1", "baseline_config": 4, "sizes": sizes,
                            "parallelism": f"shard{world}"},
-                "sweep": rows, "peak_hbm_GBs": peak, "peak_source": src,
+                "sweep": rows, "sweep_2d": rows2d, "peak_hbm_GBs": peak, "peak_source": src,
                 "gpu_launches_per_call": {"axpy": 1, "dot": 1}}
         print(json.dumps(line), flush=True)
     ctx.close()
