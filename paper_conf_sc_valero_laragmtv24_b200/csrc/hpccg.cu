@@ -1340,6 +1340,9 @@ int hpccg_waxpby2d(hpccg_ctx *ctx, int64_t m, int64_t n, int64_t ld, double alph
         return fail(HPCCG_EINVAL, "hpccg_waxpby2d: bad argument");
     if (m == 0 || n == 0) return HPCCG_OK;
     CU(cudaSetDevice(ctx->device));
+    // a contiguous m x n array (ld == m) is the 1-D AXPY over m n elements
+    // (same memory pattern, identical bits): use the vectorised 1-D kernel
+    if (ld == m) return hpccg_waxpby(ctx, m * n, alpha, x, beta, y, w);
     const int form = alpha == 1.0 ? 0 : (beta == 1.0 ? 1 : 2);
     const dim3 g = grid2d(m, (int64_t)n * ctx->nslabs, 2 * 148 * 8), b(kB2x, kB2y);
     const int64_t nn = (int64_t)n * ctx->nslabs;  // loopback: slabs stacked column-wise
@@ -1356,6 +1359,7 @@ int hpccg_ddot2d(hpccg_ctx *ctx, int64_t m, int64_t n, int64_t ld, const double 
     if (!ctx || !result || m < 0 || n < 0 || ld < m || (m > 0 && n > 0 && (!x || !y)))
         return fail(HPCCG_EINVAL, "hpccg_ddot2d: bad argument");
     CU(cudaSetDevice(ctx->device));
+    if (ld == m) return hpccg_ddot(ctx, m * n, x, y, result);  // contiguous: the 1-D DOT
     return api_reduce(ctx, false, result, [&](int s, double *out) {
         const double *xs = x + (size_t)s * ld * n, *ys = y + (size_t)s * ld * n;
         const dim3 g = grid2d(std::max<int64_t>(m, 1), std::max<int64_t>(n, 1),

@@ -883,11 +883,23 @@ __global__ void __launch_bounds__(kB2x *kB2y) waxpby2d_kernel(int64_t m, int64_t
         if (kForm == 1) return fma(alpha, xv, yv);
         return fma(alpha, xv, beta * yv);
     };
+    const int64_t si = (int64_t)gridDim.x * kB2x;
     for (int64_t j = (int64_t)blockIdx.y * kB2y + threadIdx.y; j < n; j += (int64_t)gridDim.y * kB2y)
-        for (int64_t i = (int64_t)blockIdx.x * kB2x + threadIdx.x; i < m;
-             i += (int64_t)gridDim.x * kB2x) {
-            const int64_t k = i + j * ld;
-            w[k] = op(x[k], y[k]);
+        for (int64_t i0 = (int64_t)blockIdx.x * kB2x + threadIdx.x; i0 < m; i0 += 4 * si) {
+            double xv[4], yv[4];
+#pragma unroll
+            for (int u = 0; u < 4; ++u) {
+                const int64_t i = i0 + u * si;
+                if (i < m) {
+                    xv[u] = x[i + j * ld];
+                    yv[u] = y[i + j * ld];
+                }
+            }
+#pragma unroll
+            for (int u = 0; u < 4; ++u) {
+                const int64_t i = i0 + u * si;
+                if (i < m) w[i + j * ld] = op(xv[u], yv[u]);
+            }
         }
 }
 
@@ -898,10 +910,18 @@ __global__ void __launch_bounds__(kB2x *kB2y) dot2d_kernel(int64_t m, int64_t n,
                                                            Reduction red, double *out) {
     const int tx = threadIdx.x % kB2x, ty = threadIdx.x / kB2x;
     double acc = 0.0;
+    const int64_t si = (int64_t)gridDim.x * kB2x;
     for (int64_t j = (int64_t)blockIdx.y * kB2y + ty; j < n; j += (int64_t)gridDim.y * kB2y)
-        for (int64_t i = (int64_t)blockIdx.x * kB2x + tx; i < m; i += (int64_t)gridDim.x * kB2x) {
-            const int64_t k = i + j * ld;
-            acc = fma(__ldcs(x + k), __ldcs(y + k), acc);
+        for (int64_t i0 = (int64_t)blockIdx.x * kB2x + tx; i0 < m; i0 += 4 * si) {
+            double xv[4], yv[4];  // 4 independent loads per array in flight
+#pragma unroll
+            for (int u = 0; u < 4; ++u) {
+                const int64_t i = i0 + u * si;
+                xv[u] = i < m ? __ldcs(x + i + j * ld) : 0.0;
+                yv[u] = i < m ? __ldcs(y + i + j * ld) : 0.0;
+            }
+#pragma unroll
+            for (int u = 0; u < 4; ++u) acc = fma(xv[u], yv[u], acc);
         }
     // flatten the 2-D block into the 1-D reduction helpers (256 threads)
     grid_reduce<false>(acc, red, blockIdx.y * gridDim.x + blockIdx.x, gridDim.x * gridDim.y,
