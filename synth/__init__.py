@@ -56,3 +56,10 @@ def sample_rows(n: int, k: int, seed: int) -> np.ndarray:
     k = min(k, n)
     idx = (splitmix64(k, seed) % np.uint64(max(n, 1))).astype(np.int64)
     return np.unique(np.concatenate([idx, [0, n - 1]]).astype(np.int64))
+
+
+def lbm_state(S: int, seed: int, amp: float = 0.05) -> np.ndarray:
+    """A positive D2Q9 state (9 S^2 doubles, distribution k at k S^2 + x S + y):
+    1/9 (1 + amp U[-1,1)) everywhere -- density ~1, small random velocities.
+    (Input shaping only: no lattice constant of the method is used here.)"""
+    return (1.0 / 9.0) * (1.0 + amp * uniform(9 * S * S, seed))
