@@ -543,16 +543,75 @@ def run_tridiag(args):
     return 0
 
 
+def run_lbm(args):
+    """the paper's LBM measurement (Fig. 11): the D2Q9 pull step of
+    Fig. 10 on SIZE x SIZE = 1000^2, 2 lattices.  Reports ms/step,
+    MLUPS and HBM GB/s (144 B per interior site: 9 pulled loads + 9 stores),
+    with the CPU oracle's step time beside it (the paper: 20x A100, 14x MI100,
+    6.5x Max 1550 vs a 64-core EPYC 7742)."""
+    import torch
+
+    import synth
+    from paper_conf_sc_valero_laragmtv24_b200 import hpccg as H
+
+    if int(os.environ.get("WORLD_SIZE", "1")) > 1 and int(os.environ.get("RANK", "0")) != 0:
+        return 0
+    S = args.lbm_size
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    ctx = H.Context(local)
+    l = H.Lbm(ctx, S)
+    f0 = synth.lbm_state(S, 21)
+    l.set(0, f0)
+    l.set(1, f0)
+    K = 200
+    with ClockSampler(local) as clk:
+        for _ in range(args.warmup):
+            l.run(10, 0.8)
+        ms = min(l.run(K, 0.8) for _ in range(args.steps)) / K
+    l.free()
+    sites = (S - 2) ** 2
+    gbs = 144.0 * sites / (ms * 1e-3) / 1e9
+    peak, src = peaks()
+    cpu = None
+    if not args.no_cpu_baseline:
+        import numpy as np
+        import oracle
+        a, b, f = f0.copy(), f0.copy(), np.zeros_like(f0)
+        t0 = time.perf_counter()
+        for _ in range(5):
+            oracle.lbm_step(S, a, f, b, 0.8)
+            a, b = b, a
+        cms = (time.perf_counter() - t0) / 5 * 1e3
+        cpu = {"value": round(cms, 3), "unit": "ms/step", "cores": oracle.get_threads(),
+               "kind": "oracle", "sample": f"oracle Fig. 10 step (C, OpenMP) at {S}^2, 5 steps"}
+    line = {"metric": "D2Q9 pull LBM (Fig. 10) time per step, 1000^2 (fp64)",
+            "value": round(ms, 5), "unit": "ms/step", "higher_is_better": False, "n_gpus": 1,
+            "steps": args.steps, "warmup": args.warmup, "scaling": "none", "vs_baseline": None,
+            "dtype": "f64", "data": "synthetic positive D2Q9 state (seeded), tau 0.8",
+            "config": {"workload": "lbm", "size": S, "steps_per_sample": K},
+            "MLUPS": round(sites / (ms * 1e-3) / 1e6, 1),
+            "roofline": {"bound": "hbm", "achieved": round(gbs, 1), "peak": peak, "unit": "GB/s",
+                         "frac": round(gbs / peak, 4), "peak_source": src,
+                         "algorithmic_bytes_per_step": 144 * sites},
+            "clocks": clk.summary(), "cpu_baseline": cpu,
+            "speedup_vs_cpu_oracle": round(cpu["value"] / ms, 1) if cpu else None}
+    print(json.dumps(line), flush=True)
+    ctx.close()
+    return 0
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
-    ap.add_argument("--workload", choices=sorted(WORKLOADS) + ["blas1", "tridiag"],
+    ap.add_argument("--workload", choices=sorted(WORKLOADS) + ["blas1", "tridiag", "lbm"],
                     default="hpccg128")
     ap.add_argument("--blas1-max", type=int, default=None, help="largest BLAS-1 n")
     ap.add_argument("--tri-n", type=int, default=100_000_000, help="tridiag SIZE (P:L475)")
+    ap.add_argument("--lbm-size", type=int, default=1000, help="LBM SIZE (P:L411)")
     ap.add_argument("--iters", type=int, default=None, help="override CG iterations per step")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-budget", type=float, default=12.0, help="seconds of oracle CG")
@@ -560,6 +619,12 @@ def main():
     args = ap.parse_args()
     if args.warmup < 3:
         raise SystemExit("--warmup must be >= 3")
+    if args.workload == "lbm":
+        if args.impl == "reference":
+            print(json.dumps({"impl": "reference", "unavailable":
+                              "lbm reports the oracle in cpu_baseline; no separate arm"}))
+            return 0
+        return run_lbm(args)
     if args.workload == "tridiag":
         if args.impl == "reference":
             print(json.dumps({"impl": "reference", "unavailable":
