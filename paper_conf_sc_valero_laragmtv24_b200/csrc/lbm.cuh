@@ -21,11 +21,12 @@ template <bool kWriteF>
 __global__ void __launch_bounds__(kBlock) lbm_pull_kernel(int S, const double *__restrict__ f1,
                                                          double *__restrict__ f,
                                                          double *__restrict__ f2, double tau) {
+    // grid (ceil((S-2)/256), S-2): blockIdx.y -> row x, threads -> y (interior only, Fig. 10)
     const int64_t SS = (int64_t)S * S;
-    const int64_t site = (int64_t)blockIdx.x * kBlock + threadIdx.x;
-    if (site >= SS) return;
-    const int x = (int)(site / S), y = (int)(site - (int64_t)x * S);
-    if (x < 1 || x > S - 2 || y < 1 || y > S - 2) return;  // interior only (Fig. 10)
+    const int x = 1 + (int)blockIdx.y;
+    const int y = 1 + (int)(blockIdx.x * kBlock + threadIdx.x);
+    if (y > S - 2) return;
+    const int64_t site = (int64_t)x * S + y;
     double fk[9];
 #pragma unroll
     for (int k = 0; k < 9; ++k) {
