@@ -93,6 +93,7 @@ struct hpccg_ctx {
     int64_t launches = 0;
     int num_sms = 148;
     int max_persist_l2 = 0, max_window = 0;  // bytes (device attributes)
+    int max_cluster = 0;                     // CTAs of the one-cluster persistent solve
     std::unordered_map<const void *, int> occ;  // kernel -> resident blocks / SM
 };
 
@@ -136,6 +137,8 @@ struct hpccg_problem {
     int opt_persist = 1;    // 0 never, 1 auto (n <= opt_persist_rows), 2 always (single slab)
     int opt_pdl = 1;        // programmatic dependent launch between the CG kernels
     int64_t opt_persist_rows = 65536;
+    int64_t opt_cluster_rows = 16384;  // persistent solve as one cluster up to this many rows
+    int last_persist_mode = 3;
     // graph of one CG iteration (per-iteration replay) ...
     cudaGraphExec_t graph = nullptr;
     int64_t graph_kernels = 0;
@@ -710,11 +713,30 @@ int launch_persistent(hpccg_problem *p, int max_iter, double tol) {
     a.sc = s.sc;
     a.max_iter = max_iter;
     a.tol = tol;
-    int64_t g = std::min<int64_t>(cdiv(s.n, kBlock), wave(ctx, cg_persistent_kernel));
-    g = std::max<int64_t>(1, std::min<int64_t>(g, p->red_cap / 2));
-    void *args[] = {&a};
-    CU(cudaLaunchCooperativeKernel((const void *)cg_persistent_kernel, dim3((unsigned)g), dim3(kBlock),
-                                   args, 0, ctx->stream));
+    if (s.n <= p->opt_cluster_rows && ctx->max_cluster > 1) {
+        // one cluster of up to 16 CTAs, hardware cluster barrier between phases
+        const int64_t g = std::max<int64_t>(1, std::min<int64_t>(cdiv(s.n, kBlock), ctx->max_cluster));
+        cudaLaunchConfig_t cfg{};
+        cfg.gridDim = dim3((unsigned)g);
+        cfg.blockDim = dim3(kBlock);
+        cfg.stream = ctx->stream;
+        cudaLaunchAttribute at[1];
+        at[0].id = cudaLaunchAttributeClusterDimension;
+        at[0].val.clusterDim.x = (unsigned)g;
+        at[0].val.clusterDim.y = 1;
+        at[0].val.clusterDim.z = 1;
+        cfg.attrs = at;
+        cfg.numAttrs = 1;
+        CU(cudaLaunchKernelEx(&cfg, cg_persistent_kernel<true>, a));
+        p->last_persist_mode = 4;
+    } else {
+        int64_t g = std::min<int64_t>(cdiv(s.n, kBlock), wave(ctx, cg_persistent_kernel<false>));
+        g = std::max<int64_t>(1, std::min<int64_t>(g, p->red_cap / 2));
+        void *args[] = {&a};
+        CU(cudaLaunchCooperativeKernel((const void *)cg_persistent_kernel<false>, dim3((unsigned)g),
+                                       dim3(kBlock), args, 0, ctx->stream));
+        p->last_persist_mode = 3;
+    }
     return check_launch(ctx);
 }
 
@@ -852,6 +874,35 @@ int ctx_common_init(hpccg_ctx *c, int device, void *stream) {
     CU(cudaDeviceGetAttribute(&c->num_sms, cudaDevAttrMultiProcessorCount, device));
     CU(cudaDeviceGetAttribute(&c->max_persist_l2, cudaDevAttrMaxPersistingL2CacheSize, device));
     CU(cudaDeviceGetAttribute(&c->max_window, cudaDevAttrMaxAccessPolicyWindowSize, device));
+    {   // largest cluster the persistent kernel can form (16 with the non-portable opt-in)
+        int cc = 0;
+        CU(cudaDeviceGetAttribute(&cc, cudaDevAttrClusterLaunch, device));
+        c->max_cluster = 0;
+        if (cc) {
+            if (cudaFuncSetAttribute(cg_persistent_kernel<true>,
+                                     cudaFuncAttributeNonPortableClusterSizeAllowed, 1) != cudaSuccess)
+                cudaGetLastError();
+            for (int sz : {16, 8, 4, 2}) {
+                cudaLaunchConfig_t cfg{};
+                cfg.gridDim = dim3(sz);
+                cfg.blockDim = dim3(kBlock);
+                cudaLaunchAttribute at[1];
+                at[0].id = cudaLaunchAttributeClusterDimension;
+                at[0].val.clusterDim.x = sz;
+                at[0].val.clusterDim.y = 1;
+                at[0].val.clusterDim.z = 1;
+                cfg.attrs = at;
+                cfg.numAttrs = 1;
+                int ncl = 0;
+                if (cudaOccupancyMaxActiveClusters(&ncl, cg_persistent_kernel<true>, &cfg) == cudaSuccess &&
+                    ncl > 0) {
+                    c->max_cluster = sz;
+                    break;
+                }
+                cudaGetLastError();
+            }
+        }
+    }
     if (stream) {
         c->stream = (cudaStream_t)stream;
     } else {
@@ -1255,6 +1306,10 @@ int hpccg_set_option(hpccg_problem *p, int key, int64_t value) {
             if (value < 0 || value > 2) return fail(HPCCG_EINVAL, "persistent: 0, 1 or 2");
             p->opt_persist = (int)value;
             return HPCCG_OK;
+        case HPCCG_OPT_CLUSTER_ROWS:
+            if (value < 0) return fail(HPCCG_EINVAL, "cluster rows must be >= 0");
+            p->opt_cluster_rows = value;
+            return HPCCG_OK;
         case HPCCG_OPT_PERSIST_ROWS:
             if (value < 0) return fail(HPCCG_EINVAL, "persist rows must be >= 0");
             p->opt_persist_rows = value;
@@ -1474,7 +1529,7 @@ int hpccg_solve(hpccg_problem *p, int max_iter, double tol, int *niters, double 
     st.spmv_launches = hs.niters + 1;
     st.kernel_launches = ctx->launches - l0;
     st.l2_persist_bytes = (int64_t)l2win.kept;
-    st.graph_mode = use_persist ? 3 : (use_while ? 2 : (use_graph ? 1 : 0));
+    st.graph_mode = use_persist ? p->last_persist_mode : (use_while ? 2 : (use_graph ? 1 : 0));
     p->stats = st;
     if (niters) *niters = hs.niters;
     if (normr) *normr = hs.normr;

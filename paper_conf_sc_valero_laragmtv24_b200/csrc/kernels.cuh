@@ -15,6 +15,7 @@
 // never leave the device.
 #pragma once
 
+#include <cooperative_groups.h>
 #include <cuda_runtime.h>
 #include <stdint.h>
 
@@ -718,6 +719,16 @@ __device__ __forceinline__ double block_partial(double v, double *sh) {
     return v;
 }
 
+// kCluster: the whole grid is ONE thread-block cluster (<= 16 CTAs) and the
+// phases are separated by the hardware cluster barrier (~380 cycles on
+// Blackwell, and it invalidates L1) instead of the global-atomic grid barrier.
+template <bool kCluster>
+__device__ __forceinline__ void phase_barrier(unsigned *bar, unsigned nb) {
+    if (kCluster) cooperative_groups::this_cluster().sync();
+    else grid_barrier(bar, nb);
+}
+
+template <bool kCluster>
 __global__ void __launch_bounds__(kBlock, 1) cg_persistent_kernel(PersistArgs a) {
     __shared__ double sh[32];
     const int64_t tid = gtid(), nth = gnth();
@@ -732,7 +743,7 @@ __global__ void __launch_bounds__(kBlock, 1) cg_persistent_kernel(PersistArgs a)
     };
     // ---- init (a.7): p = x; Ap = A p; r = b - Ap; rtrans = r.r
     for (int64_t i = tid; i < a.n; i += nth) po[i] = a.x[i];
-    grid_barrier(a.bar, nb);
+    phase_barrier<kCluster>(a.bar, nb);
     double acc = 0.0;
     for (int64_t i = tid; i < a.n; i += nth) {
         const double ap = spmv_row(i);
@@ -742,7 +753,7 @@ __global__ void __launch_bounds__(kBlock, 1) cg_persistent_kernel(PersistArgs a)
     }
     acc = block_partial(acc, sh);
     if (threadIdx.x == 0) a.part_rr[blockIdx.x] = acc;
-    grid_barrier(a.bar, nb);
+    phase_barrier<kCluster>(a.bar, nb);
     double rr = sum_partials(a.part_rr, sh);
     double rtrans = rr, normr = sqrt(rtrans);
     int niters = 0;
@@ -756,7 +767,7 @@ __global__ void __launch_bounds__(kBlock, 1) cg_persistent_kernel(PersistArgs a)
         }
         for (int64_t i = tid; i < a.n; i += nth) po[i] = (k == 1) ? a.r[i] : fma(beta, po[i], a.r[i]);
         normr = sqrt(rtrans);
-        grid_barrier(a.bar, nb);
+        phase_barrier<kCluster>(a.bar, nb);
         double d = 0.0;
         for (int64_t i = tid; i < a.n; i += nth) {
             const double ap = spmv_row(i);
@@ -765,7 +776,7 @@ __global__ void __launch_bounds__(kBlock, 1) cg_persistent_kernel(PersistArgs a)
         }
         d = block_partial(d, sh);
         if (threadIdx.x == 0) a.part_pAp[blockIdx.x] = d;
-        grid_barrier(a.bar, nb);
+        phase_barrier<kCluster>(a.bar, nb);
         const double pAp = sum_partials(a.part_pAp, sh);
         const bool stop = (rtrans == 0.0) || (pAp == 0.0);
         const double alpha = stop ? 0.0 : rtrans / pAp;
@@ -778,7 +789,7 @@ __global__ void __launch_bounds__(kBlock, 1) cg_persistent_kernel(PersistArgs a)
         }
         acc = block_partial(acc, sh);
         if (threadIdx.x == 0) a.part_rr[blockIdx.x] = acc;
-        grid_barrier(a.bar, nb);
+        phase_barrier<kCluster>(a.bar, nb);
         rr = sum_partials(a.part_rr, sh);
         niters = k;
         if (stop) break;
