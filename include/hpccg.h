@@ -85,6 +85,9 @@ extern "C" {
                                (grid barriers between phases): 0 never, 1 (default) when
                                nrow_local <= HPCCG_OPT_PERSIST_ROWS, 2 always */
 #define HPCCG_OPT_PERSIST_ROWS 10 /* threshold for HPCCG_OPT_PERSISTENT = 1 (default 65536) */
+#define HPCCG_OPT_SMEM_SOLVE 13 /* 1 (default): a persistent solve whose rows fit in the
+                               shared memory of one 16-CTA cluster (~9.9k rows) keeps the whole
+                               problem on chip (distributed shared memory gathers); 0: off */
 #define HPCCG_OPT_CLUSTER_ROWS 12 /* up to this many rows (default 16384) the persistent solve
                                is ONE thread-block cluster (<= 16 CTAs) synchronised by the
                                hardware cluster barrier; above, a cooperative grid with a
@@ -112,8 +115,9 @@ typedef struct hpccg_stats {
     int64_t iterations;     /* niters */
     int64_t kernel_launches;/* kernels this library enqueued during the solve */
     int64_t l2_persist_bytes; /* L2 set aside for the CG vectors during the solve (0: none) */
-    int64_t graph_mode;     /* 4 one-cluster persistent kernel, 3 cooperative-grid persistent
-                               kernel, 2 while-graph, 1 per-iteration graph, 0 plain */
+    int64_t graph_mode;     /* 5 shared-memory-resident cluster kernel, 4 one-cluster
+                               persistent kernel, 3 cooperative-grid persistent kernel,
+                               2 while-graph, 1 per-iteration graph, 0 plain */
 } hpccg_stats;
 
 HPCCG_API const char *hpccg_strerror(int code);

@@ -94,6 +94,8 @@ struct hpccg_ctx {
     int num_sms = 148;
     int max_persist_l2 = 0, max_window = 0;  // bytes (device attributes)
     int max_cluster = 0;                     // CTAs of the one-cluster persistent solve
+    int smem_cluster = 0;                    // CTAs of the shared-memory-resident solve
+    int64_t smem_bytes = 0;                  // dynamic smem per CTA it may use
     std::unordered_map<const void *, int> occ;  // kernel -> resident blocks / SM
 };
 
@@ -138,6 +140,7 @@ struct hpccg_problem {
     int opt_pdl = 1;        // programmatic dependent launch between the CG kernels
     int64_t opt_persist_rows = 65536;
     int64_t opt_cluster_rows = 16384;  // persistent solve as one cluster up to this many rows
+    int opt_smem = 1;                  // persistent solve resident in cluster shared memory if it fits
     int last_persist_mode = 3;
     // graph of one CG iteration (per-iteration replay) ...
     cudaGraphExec_t graph = nullptr;
@@ -713,6 +716,41 @@ int launch_persistent(hpccg_problem *p, int max_iter, double tol) {
     a.sc = s.sc;
     a.max_iter = max_iter;
     a.tol = tol;
+    // whole problem in one cluster's shared memory when it fits
+    const int64_t bytes_per_row = kSlots * (sizeof(double) + sizeof(int)) + 5 * sizeof(double);
+    if (p->opt_smem && ctx->smem_cluster > 1) {
+        const int64_t R = cdiv(s.n, ctx->smem_cluster);
+        if (R * bytes_per_row <= ctx->smem_bytes) {
+            SmemArgs m{};
+            m.n = s.n;
+            m.stride = s.n;
+            m.plane = s.plane;
+            m.R = (int)R;
+            m.val = s.val;
+            m.col = s.col;
+            m.b = s.b;
+            m.x = s.x;
+            m.sc = s.sc;
+            m.max_iter = max_iter;
+            m.tol = tol;
+            const int64_t g = cdiv(s.n, R);
+            cudaLaunchConfig_t cfg{};
+            cfg.gridDim = dim3((unsigned)g);
+            cfg.blockDim = dim3(kBlock);
+            cfg.dynamicSmemBytes = (size_t)(R * bytes_per_row);
+            cfg.stream = ctx->stream;
+            cudaLaunchAttribute at[1];
+            at[0].id = cudaLaunchAttributeClusterDimension;
+            at[0].val.clusterDim.x = (unsigned)g;
+            at[0].val.clusterDim.y = 1;
+            at[0].val.clusterDim.z = 1;
+            cfg.attrs = at;
+            cfg.numAttrs = 1;
+            CU(cudaLaunchKernelEx(&cfg, cg_smem_cluster_kernel, m));
+            p->last_persist_mode = 5;
+            return check_launch(ctx);
+        }
+    }
     if (s.n <= p->opt_cluster_rows && ctx->max_cluster > 1) {
         // one cluster of up to 16 CTAs, hardware cluster barrier between phases
         const int64_t g = std::max<int64_t>(1, std::min<int64_t>(cdiv(s.n, kBlock), ctx->max_cluster));
@@ -874,6 +912,38 @@ int ctx_common_init(hpccg_ctx *c, int device, void *stream) {
     CU(cudaDeviceGetAttribute(&c->num_sms, cudaDevAttrMultiProcessorCount, device));
     CU(cudaDeviceGetAttribute(&c->max_persist_l2, cudaDevAttrMaxPersistingL2CacheSize, device));
     CU(cudaDeviceGetAttribute(&c->max_window, cudaDevAttrMaxAccessPolicyWindowSize, device));
+    {   // shared-memory-resident solve: largest dynamic smem and cluster size
+        int optin = 0;
+        CU(cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, device));
+        c->smem_bytes = optin - 1024;  // static smem of the kernel + slack
+        c->smem_cluster = 0;
+        if (cudaFuncSetAttribute(cg_smem_cluster_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 (int)c->smem_bytes) == cudaSuccess &&
+            cudaFuncSetAttribute(cg_smem_cluster_kernel, cudaFuncAttributeNonPortableClusterSizeAllowed,
+                                 1) == cudaSuccess) {
+            for (int sz : {16, 8}) {
+                cudaLaunchConfig_t cfg{};
+                cfg.gridDim = dim3(sz);
+                cfg.blockDim = dim3(kBlock);
+                cfg.dynamicSmemBytes = (size_t)c->smem_bytes;
+                cudaLaunchAttribute at[1];
+                at[0].id = cudaLaunchAttributeClusterDimension;
+                at[0].val.clusterDim.x = sz;
+                at[0].val.clusterDim.y = 1;
+                at[0].val.clusterDim.z = 1;
+                cfg.attrs = at;
+                cfg.numAttrs = 1;
+                int ncl = 0;
+                if (cudaOccupancyMaxActiveClusters(&ncl, cg_smem_cluster_kernel, &cfg) == cudaSuccess &&
+                    ncl > 0) {
+                    c->smem_cluster = sz;
+                    break;
+                }
+                cudaGetLastError();
+            }
+        }
+        cudaGetLastError();
+    }
     {   // largest cluster the persistent kernel can form (16 with the non-portable opt-in)
         int cc = 0;
         CU(cudaDeviceGetAttribute(&cc, cudaDevAttrClusterLaunch, device));
@@ -1306,6 +1376,7 @@ int hpccg_set_option(hpccg_problem *p, int key, int64_t value) {
             if (value < 0 || value > 2) return fail(HPCCG_EINVAL, "persistent: 0, 1 or 2");
             p->opt_persist = (int)value;
             return HPCCG_OK;
+        case HPCCG_OPT_SMEM_SOLVE: p->opt_smem = value != 0; return HPCCG_OK;
         case HPCCG_OPT_CLUSTER_ROWS:
             if (value < 0) return fail(HPCCG_EINVAL, "cluster rows must be >= 0");
             p->opt_cluster_rows = value;

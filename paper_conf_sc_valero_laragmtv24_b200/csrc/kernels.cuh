@@ -803,6 +803,134 @@ __global__ void __launch_bounds__(kBlock, 1) cg_persistent_kernel(PersistArgs a)
     }
 }
 
+// ----------------------------------- on-chip solve (tiny single-GPU problems)
+// The whole problem lives in the shared memory of ONE thread-block cluster
+// (<= 16 CTAs, 227 KB each): CTA c owns rows [c R, (c+1) R) -- its ELL slice,
+// b, x, r, p, Ap -- loaded once per solve.  The stencil gathers read p from
+// the owning CTA's shared memory (distributed shared memory when it is a
+// neighbour CTA), every reduction is 16 per-CTA partials read by every CTA in
+// rank order, and the phases are separated by the hardware cluster barrier.
+// Same HPCCG loop (A4, A11) as every other path; per-row FMA chain as A8.
+struct SmemArgs {
+    int64_t n, stride, plane;
+    int R;  // rows per CTA
+    const double *val;
+    const int *col;
+    const double *b;
+    double *x;  // in: initial guess, out: iterate
+    CgScalars *sc;
+    int max_iter;
+    double tol;
+};
+
+__device__ __forceinline__ double cluster_sum(double *mine, double v, double *sh) {
+    namespace cgx = cooperative_groups;
+    auto cl = cgx::this_cluster();
+    v = block_reduce<false>(v, sh);
+    if (threadIdx.x == 0) *mine = v;
+    cl.sync();
+    double s = 0.0;
+    if (threadIdx.x == 0) {
+        for (unsigned c = 0; c < cl.num_blocks(); ++c) s += *cl.map_shared_rank(mine, c);
+        sh[31] = s;
+    }
+    __syncthreads();
+    s = sh[31];
+    __syncthreads();
+    return s;
+}
+
+__global__ void __launch_bounds__(kBlock, 1) cg_smem_cluster_kernel(SmemArgs a) {
+    namespace cgx = cooperative_groups;
+    auto cl = cgx::this_cluster();
+    extern __shared__ double smem[];
+    __shared__ double sh[32];
+    __shared__ double part_pAp, part_rr;
+    const int R = a.R;
+    const unsigned me = cl.block_rank();
+    double *sval = smem;                        // [27][R]
+    double *sb = sval + (size_t)kSlots * R;     // [R] each
+    double *sx = sb + R, *sr = sx + R, *sp = sr + R, *sAp = sp + R;
+    int *scol = reinterpret_cast<int *>(sAp + R);  // [27][R]
+    const int64_t row0 = (int64_t)me * R;
+    const int nr = (int)max<int64_t>(0, min<int64_t>(R, a.n - row0));
+    // load this CTA's slice (global column ids -> owner CTA / offset later)
+    for (int k = 0; k < kSlots; ++k)
+        for (int i = threadIdx.x; i < nr; i += kBlock) {
+            sval[k * R + i] = a.val[k * a.stride + row0 + i];
+            scol[k * R + i] = a.col[k * a.stride + row0 + i];
+        }
+    for (int i = threadIdx.x; i < nr; i += kBlock) {
+        sb[i] = a.b[row0 + i];
+        sx[i] = a.x[row0 + i];
+    }
+    __syncthreads();
+    auto spmv_row = [&](int i) {  // y_i = sum_k val * p[col], p read from its owner CTA
+        double s = 0.0;
+#pragma unroll 9
+        for (int k = 0; k < kSlots; ++k) {
+            const int64_t g = (int64_t)scol[k * R + i] - a.plane;  // global row of the column
+            const unsigned owner = (unsigned)(g / R);
+            const int off = (int)(g - (int64_t)owner * R);
+            const double pv = owner == me ? sp[off] : *cl.map_shared_rank(sp + off, owner);
+            s = fma(sval[k * R + i], pv, s);
+        }
+        return s;
+    };
+    // ---- init (a.7)
+    for (int i = threadIdx.x; i < nr; i += kBlock) sp[i] = sx[i];
+    cl.sync();
+    double acc = 0.0;
+    for (int i = threadIdx.x; i < nr; i += kBlock) {
+        const double rv = fma(-1.0, spmv_row(i), sb[i]);
+        sr[i] = rv;
+        acc = fma(rv, rv, acc);
+    }
+    double rr = cluster_sum(&part_rr, acc, sh);
+    double rtrans = rr, normr = sqrt(rtrans);
+    int niters = 0;
+    for (int k = 1; k < a.max_iter && normr > a.tol; ++k) {
+        double beta = 0.0;
+        if (k > 1) {
+            const double old = rtrans;
+            rtrans = rr;
+            beta = rtrans / old;
+        }
+        // every CTA has finished reading the previous p (cluster_sum's barrier)
+        for (int i = threadIdx.x; i < nr; i += kBlock) sp[i] = (k == 1) ? sr[i] : fma(beta, sp[i], sr[i]);
+        normr = sqrt(rtrans);
+        cl.sync();
+        double d = 0.0;
+        for (int i = threadIdx.x; i < nr; i += kBlock) {
+            const double ap = spmv_row(i);
+            sAp[i] = ap;
+            d = fma(ap, sp[i], d);
+        }
+        const double pAp = cluster_sum(&part_pAp, d, sh);
+        const bool stop = (rtrans == 0.0) || (pAp == 0.0);
+        const double alpha = stop ? 0.0 : rtrans / pAp;
+        acc = 0.0;
+        for (int i = threadIdx.x; i < nr; i += kBlock) {
+            sx[i] = fma(alpha, sp[i], sx[i]);
+            const double rv = fma(-alpha, sAp[i], sr[i]);
+            sr[i] = rv;
+            acc = fma(rv, rv, acc);
+        }
+        rr = cluster_sum(&part_rr, acc, sh);
+        niters = k;
+        if (stop) break;
+    }
+    for (int i = threadIdx.x; i < nr; i += kBlock) a.x[row0 + i] = sx[i];
+    if (me == 0 && threadIdx.x == 0) {
+        a.sc->niters = niters;
+        a.sc->normr = normr;
+        a.sc->rr_cur = rr;
+        a.sc->rr_prev = rtrans;
+        a.sc->done = 1;
+    }
+    cl.sync();  // no CTA leaves while its shared memory may still be read
+}
+
 // Loopback allreduce: fixed rank-order sum (or max) of one scalar of every
 // slab, written back to every slab (deterministic, identical on all slabs).
 __global__ void slab_allreduce_kernel(const double *const *src, double *const *dst,

@@ -35,7 +35,7 @@ HPCCG_OPT_GRAPH, HPCCG_OPT_POLL, HPCCG_OPT_TIMING = 0, 1, 2
 HPCCG_OPT_SPMV_MINB, HPCCG_OPT_WHILE, HPCCG_OPT_L2_PERSIST, HPCCG_OPT_VEC_WAVES = 3, 4, 5, 6
 HPCCG_OPT_SPMV_ROWS, HPCCG_OPT_VEC_UNROLL = 7, 8
 HPCCG_OPT_PERSISTENT, HPCCG_OPT_PERSIST_ROWS, HPCCG_OPT_PDL = 9, 10, 11
-HPCCG_OPT_CLUSTER_ROWS = 12
+HPCCG_OPT_CLUSTER_ROWS, HPCCG_OPT_SMEM_SOLVE = 12, 13
 
 _lock = threading.Lock()
 _lib = None

@@ -289,7 +289,7 @@ def test_cg_persistent_kernel_vs_oracle(ctx, dims):
         tol = 0.0 if dims in [(1, 1, 1), (2, 2, 2)] else 1e-12
         oref = oracle.cg(ref, 150, tol)
         res = p.solve(150, tol)
-        assert p.stats()["graph_mode"] in (3, 4) and p.stats()["kernel_launches"] == 1
+        assert p.stats()["graph_mode"] in (3, 4, 5) and p.stats()["kernel_launches"] == 1
         check_cg(res, p.maxabsdiff(), oref, ref)
         assert np.max(np.abs(p.get_vec(H.HPCCG_VEC_X) - oref["x"])) <= CG_ATOL
         if dims == (20, 30, 10):
@@ -303,18 +303,20 @@ def test_cg_persistent_kernel_vs_oracle(ctx, dims):
         assert p.solve(50, 1e-12)["niters"] == 0
 
 
-@pytest.mark.parametrize("crows", [0, 1 << 30])
-def test_cg_persistent_grid_and_cluster_variants(ctx, crows):
-    """Both persistent variants (cooperative grid + global barrier; one
-    cluster + hardware cluster barrier) against the oracle."""
+@pytest.mark.parametrize("crows,smem,mode", [(0, 0, 3), (1 << 30, 0, 4), (0, 1, 5)])
+def test_cg_persistent_grid_and_cluster_variants(ctx, crows, smem, mode):
+    """The three persistent variants (cooperative grid + global barrier; one
+    cluster + hardware cluster barrier; the whole problem in one cluster's
+    shared memory) against the oracle."""
     dims = (20, 30, 10)
     with H.Problem(ctx, *dims) as p:
         p.set_option(H.HPCCG_OPT_PERSISTENT, 2)
         p.set_option(H.HPCCG_OPT_CLUSTER_ROWS, crows)
+        p.set_option(H.HPCCG_OPT_SMEM_SOLVE, smem)
         ref = oracle.generate(*dims)
         oref = oracle.cg(ref, 150, 1e-12)
         res = p.solve(150, 1e-12)
-        assert p.stats()["graph_mode"] == (4 if crows else 3)
+        assert p.stats()["graph_mode"] == mode
         check_cg(res, p.maxabsdiff(), oref, ref)
         assert res["niters"] == 50
 
@@ -322,7 +324,7 @@ def test_cg_persistent_grid_and_cluster_variants(ctx, crows):
 def test_cg_persistent_auto_threshold(ctx):
     with H.Problem(ctx, 20, 30, 10) as p:       # 6000 rows <= 65536: persistent
         p.solve(150, 1e-12)
-        assert p.stats()["graph_mode"] in (3, 4)
+        assert p.stats()["graph_mode"] in (3, 4, 5)
         p.set_option(H.HPCCG_OPT_PERSIST_ROWS, 1000)
         p.set_vec(H.HPCCG_VEC_X, np.zeros(p.n))
         p.solve(150, 1e-12)

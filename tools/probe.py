@@ -11,7 +11,8 @@ KEYS = {"graph": H.HPCCG_OPT_GRAPH, "timing": H.HPCCG_OPT_TIMING, "while": H.HPC
         "unroll": H.HPCCG_OPT_VEC_UNROLL,
         "persist": H.HPCCG_OPT_PERSISTENT,
         "pdl": H.HPCCG_OPT_PDL,
-        "crows": H.HPCCG_OPT_CLUSTER_ROWS}
+        "crows": H.HPCCG_OPT_CLUSTER_ROWS,
+        "smem": H.HPCCG_OPT_SMEM_SOLVE}
 nx, ny, nz, iters = (int(v) for v in sys.argv[1:5])
 ctx = H.Context(0)
 p = H.Problem(ctx, nx, ny, nz)
@@ -42,6 +43,6 @@ for spec in sys.argv[5:]:
     print(json.dumps(out), flush=True)
     for k in opts:
         try:
-            p.set_option(KEYS[k], {"graph": 1, "while": 1, "l2": 1, "waves": 1, "rows": 2, "unroll": 4, "persist": 1, "pdl": 1, "crows": 16384}.get(k, 0))
+            p.set_option(KEYS[k], {"graph": 1, "while": 1, "l2": 1, "waves": 1, "rows": 2, "unroll": 4, "persist": 1, "pdl": 1, "crows": 16384, "smem": 1}.get(k, 0))
         except H.HpccgError:
             pass
