@@ -853,7 +853,8 @@ __global__ void __launch_bounds__(kBlock, 1) cg_smem_cluster_kernel(SmemArgs a) 
     double *sx = sb + R, *sr = sx + R, *sp = sr + R, *sAp = sp + R;
     int *scol = reinterpret_cast<int *>(sAp + R);  // [27][R]
     const int64_t row0 = (int64_t)me * R;
-    const int nr = (int)max<int64_t>(0, min<int64_t>(R, a.n - row0));
+    const int64_t rem = a.n - row0;
+    const int nr = rem <= 0 ? 0 : (int)(rem < R ? rem : R);
     // load this CTA's slice (global column ids -> owner CTA / offset later)
     for (int k = 0; k < kSlots; ++k)
         for (int i = threadIdx.x; i < nr; i += kBlock) {
