@@ -829,13 +829,16 @@ __device__ __forceinline__ double cluster_sum(double *mine, double v, double *sh
     v = block_reduce<false>(v, sh);
     if (threadIdx.x == 0) *mine = v;
     cl.sync();
-    double s = 0.0;
-    if (threadIdx.x == 0) {
-        for (unsigned c = 0; c < cl.num_blocks(); ++c) s += *cl.map_shared_rank(mine, c);
-        sh[31] = s;
+    // lanes 0..C-1 of warp 0 fetch the C partials in parallel (one DSMEM
+    // round trip), then a fixed butterfly: identical sums in every CTA
+    if (threadIdx.x < 32) {
+        const unsigned c = threadIdx.x;
+        double q = c < cl.num_blocks() ? *cl.map_shared_rank(mine, c) : 0.0;
+        q = warp_sum(q);
+        if (threadIdx.x == 0) sh[31] = q;
     }
     __syncthreads();
-    s = sh[31];
+    const double s = sh[31];
     __syncthreads();
     return s;
 }
@@ -866,16 +869,19 @@ __global__ void __launch_bounds__(kBlock, 1) cg_smem_cluster_kernel(SmemArgs a) 
         sx[i] = a.x[row0 + i];
     }
     __syncthreads();
+    const int plane32 = (int)a.plane;
     auto spmv_row = [&](int i) {  // y_i = sum_k val * p[col], p read from its owner CTA
-        double s = 0.0;
-#pragma unroll 9
-        for (int k = 0; k < kSlots; ++k) {
-            const int64_t g = (int64_t)scol[k * R + i] - a.plane;  // global row of the column
-            const unsigned owner = (unsigned)(g / R);
-            const int off = (int)(g - (int64_t)owner * R);
-            const double pv = owner == me ? sp[off] : *cl.map_shared_rank(sp + off, owner);
-            s = fma(sval[k * R + i], pv, s);
+        double pv[kSlots];
+#pragma unroll
+        for (int k = 0; k < kSlots; ++k) {  // all 27 gathers issued before the FMA chain
+            const int g = scol[k * R + i] - plane32;  // global row of the column (< 2^31)
+            const unsigned owner = (unsigned)g / (unsigned)R;
+            const int off = g - (int)owner * R;
+            pv[k] = *cl.map_shared_rank(sp + off, owner);
         }
+        double s = 0.0;
+#pragma unroll
+        for (int k = 0; k < kSlots; ++k) s = fma(sval[k * R + i], pv[k], s);
         return s;
     };
     // ---- init (a.7)
