@@ -117,6 +117,7 @@ __device__ __forceinline__ double warp_max(double v) {
 template <bool kMax>
 __device__ __forceinline__ double block_reduce(double v, double *sh) {
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    __syncwarp();  // reconverge lanes that left a grid-stride loop at different trips
     v = kMax ? warp_max(v) : warp_sum(v);
     if (lane == 0) sh[warp] = v;
     __syncthreads();
