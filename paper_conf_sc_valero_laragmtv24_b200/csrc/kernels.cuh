@@ -120,6 +120,7 @@ __device__ __forceinline__ double block_reduce(double v, double *sh) {
     __syncwarp();  // reconverge lanes that left a grid-stride loop at different trips
     v = kMax ? warp_max(v) : warp_sum(v);
     if (lane == 0) sh[warp] = v;
+    __syncwarp();  // converged warp at the block barrier (compute-sanitizer synccheck)
     __syncthreads();
     if (warp == 0) {
         v = (lane < kWarps) ? sh[lane] : (kMax ? 0.0 : 0.0);
@@ -145,6 +146,7 @@ __device__ __forceinline__ void grid_reduce(double v, Reduction red, unsigned pa
         unsigned t = atomicAdd(red.counter, 1u);
         is_last = (t == total - 1);
     }
+    __syncwarp();
     __syncthreads();
     if (!is_last) return;
     __threadfence();
