@@ -137,17 +137,19 @@ __global__ void __launch_bounds__(kBlock) tri_dot_kernel(int64_t n, const double
     pdl_trigger();
     double acc = 0.0;
     const int64_t nth = gnth();
-    for (int64_t b0 = gtid(); b0 < n; b0 += kTriU * nth) {
+    const int64_t full = n / (kTriU * nth) * (kTriU * nth);  // trips where all kTriU are in range
+    int64_t b0 = gtid();
+    for (; b0 < full; b0 += kTriU * nth) {
         double xv[kTriU], yv[kTriU];
 #pragma unroll
         for (int u = 0; u < kTriU; ++u) {
-            const int64_t i = b0 + u * nth;
-            xv[u] = i < n ? x[i] : 0.0;
-            yv[u] = i < n ? y[i] : 0.0;
+            xv[u] = x[b0 + u * nth];
+            yv[u] = y[b0 + u * nth];
         }
 #pragma unroll
         for (int u = 0; u < kTriU; ++u) acc = fma(xv[u], yv[u], acc);
     }
+    for (int64_t i = b0; i < n; i += nth) acc = fma(x[i], y[i], acc);  // ragged tail, same order
     grid_reduce<false>(acc, red, blockIdx.x, gridDim.x, [out](double v) { *out = v; });
 }
 
