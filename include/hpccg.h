@@ -88,6 +88,10 @@ extern "C" {
 #define HPCCG_OPT_SMEM_SOLVE 13 /* 1 (default): a persistent solve whose rows fit in the
                                shared memory of one 16-CTA cluster (~9.9k rows) keeps the whole
                                problem on chip (distributed shared memory gathers); 0: off */
+#define HPCCG_OPT_TRACE 14  /* k > 0: record, for the first k iterations, each CG kernel's
+                               first-block start and last-block end on the device clock
+                               (%globaltimer; works inside graphs); read with
+                               hpccg_get_trace.  0 (default): off */
 #define HPCCG_OPT_CLUSTER_ROWS 12 /* up to this many rows (default 16384) the persistent solve
                                is ONE thread-block cluster (<= 16 CTAs) synchronised by the
                                hardware cluster barrier; above, a cooperative grid with a
@@ -251,6 +255,12 @@ HPCCG_API int hpccg_ddot2d(hpccg_ctx *ctx, int64_t m, int64_t n, int64_t ld, con
  * waxpby/spmv kernels, so times[1] = 0).  max_iter >= 1, tol >= 0. */
 HPCCG_API int hpccg_solve(hpccg_problem *prob, int max_iter, double tol, int *niters,
                 double *normr, double times[6]);
+
+/* Device trace of the last solve (HPCCG_OPT_TRACE = k): out[(i*3 + j)*2 + {0,1}]
+ * = start / end (ns, device clock) of kernel j (0 p update, 1 SpMV, 2 x/r update)
+ * in iteration i+1, for i < min(k, niters); 0 where a kernel did not run.
+ * `out` (HOST) holds 6*k uint64.  Single slab / first slab. */
+HPCCG_API int hpccg_get_trace(const hpccg_problem *prob, uint64_t *out, int64_t k);
 
 /* Statistics of the last hpccg_solve on `prob`. */
 HPCCG_API int hpccg_get_stats(const hpccg_problem *prob, hpccg_stats *out);

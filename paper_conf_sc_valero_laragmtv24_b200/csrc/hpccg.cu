@@ -114,6 +114,9 @@ struct Slab {
     CgScalars *sc = nullptr;
     Reduction red{};
     unsigned *bar = nullptr;  // grid barrier state of the persistent solve
+    TraceSlot *trace = nullptr;  // HPCCG_OPT_TRACE buffer: [trace_max][3]
+    int trace_max = 0;
+    bool trace_on = false;
     double *spmv_parts = nullptr;  // per-block p.Ap partials (single slab)
     int64_t spmv_nparts = 0;
 };
@@ -330,6 +333,8 @@ int exchange(hpccg_problem *p, double *const *xs, cudaStream_t on) {
 
 SpmvArgs spmv_args(const Slab &s, const double *x, double *y) {
     SpmvArgs a{};
+    a.trace = s.trace_on ? s.trace : nullptr;
+    a.trace_max = s.trace_max;
     a.stride = s.n;
     a.plane = s.plane;
     a.val = s.val;
@@ -408,7 +413,8 @@ template <bool kVec, bool kCheck, int kU>
 int launch_pupdate_t(hpccg_ctx *ctx, int waves, const Slab &s, double *po, bool pdl) {
     auto k = cg_pupdate_kernel<kVec, kCheck, kU>;
     const int g = vec_grid(ctx, k, kVec ? cdiv(s.n, 2 * kU) : s.n, waves, 0x7fffffff);
-    launch_k(pdl, k, dim3(g), ctx->stream, s.n, (const double *)s.r, po, (const CgScalars *)s.sc);
+    launch_k(pdl, k, dim3(g), ctx->stream, s.n, (const double *)s.r, po, (const CgScalars *)s.sc,
+             s.trace_on ? s.trace : (TraceSlot *)nullptr, s.trace_max);
     return check_launch(ctx);
 }
 
@@ -460,6 +466,8 @@ int launch_update(hpccg_ctx *ctx, int waves, int unroll, int64_t cap, const Slab
     a.red = s.red;
     a.single = single;
     a.cond = cond;
+    a.trace = s.trace_on ? s.trace : nullptr;
+    a.trace_max = s.trace_max;
     if (single) {  // p.Ap partials of the single-slab SpMV (see cg_spmv_all)
         const unsigned np =
             (unsigned)spmv_blocks(s.n, spmv_rows_per_thread(rows, spmv_args(s, s.p, s.Ap), 0, 0));
@@ -903,6 +911,7 @@ void free_slab(Slab &s) {
     cudaFree(s.red.counter);
     cudaFree(s.bar);
     cudaFree(s.spmv_parts);
+    cudaFree(s.trace);
     s = Slab{};
 }
 
@@ -1377,6 +1386,21 @@ int hpccg_set_option(hpccg_problem *p, int key, int64_t value) {
             p->opt_persist = (int)value;
             return HPCCG_OK;
         case HPCCG_OPT_SMEM_SOLVE: p->opt_smem = value != 0; return HPCCG_OK;
+        case HPCCG_OPT_TRACE: {
+            if (value < 0 || value > (1 << 20)) return fail(HPCCG_EINVAL, "trace: 0..2^20 iterations");
+            for (Slab &sl : p->slabs) {
+                cudaFree(sl.trace);
+                sl.trace = nullptr;
+                sl.trace_max = 0;
+                sl.trace_on = false;
+                if (value > 0) {
+                    CHECK(alloc_zero((void **)&sl.trace, sizeof(TraceSlot) * 3 * (size_t)value));
+                    sl.trace_max = (int)value;
+                    sl.trace_on = true;
+                }
+            }
+            return HPCCG_OK;
+        }
         case HPCCG_OPT_CLUSTER_ROWS:
             if (value < 0) return fail(HPCCG_EINVAL, "cluster rows must be >= 0");
             p->opt_cluster_rows = value;
@@ -1532,6 +1556,13 @@ int hpccg_solve(hpccg_problem *p, int max_iter, double tol, int *niters, double 
     }
     if (use_graph && !use_while && !use_persist) CHECK(build_graph(p));
 
+    if (p->slabs[0].trace_on) {  // t0 = +inf, t1 = 0 for every slot
+        const Slab &s0 = p->slabs[0];
+        std::vector<TraceSlot> init((size_t)3 * s0.trace_max, TraceSlot{~0ull, 0ull});
+        CU(cudaMemcpyAsync(s0.trace, init.data(), sizeof(TraceSlot) * init.size(),
+                           cudaMemcpyHostToDevice, ctx->stream));
+        CU(cudaStreamSynchronize(ctx->stream));
+    }
     CU(cudaEventRecord(p->ev_t0, ctx->stream));
     if (use_persist) {
         CHECK(launch_persistent(p, max_iter, tol));
@@ -1612,6 +1643,18 @@ int hpccg_solve(hpccg_problem *p, int max_iter, double tol, int *niters, double 
         times[4] = st.allreduce_ms * 1e-3;
         times[5] = st.exchange_ms * 1e-3;
     }
+    return HPCCG_OK;
+}
+
+int hpccg_get_trace(const hpccg_problem *p, uint64_t *out, int64_t k) {
+    if (!p || !out || k < 0) return fail(HPCCG_EINVAL, "bad argument");
+    const Slab &s = p->slabs[0];
+    if (!s.trace_on) return fail(HPCCG_EINVAL, "tracing is off (HPCCG_OPT_TRACE)");
+    const int64_t m = std::min<int64_t>(k, s.trace_max);
+    CU(cudaSetDevice(p->ctx->device));
+    CU(cudaMemcpy(out, s.trace, sizeof(TraceSlot) * 3 * (size_t)m, cudaMemcpyDeviceToHost));
+    for (int64_t i = 0; i < 6 * m; i += 2)
+        if (out[i] == ~0ull) out[i] = out[i + 1] = 0;  // kernel did not run
     return HPCCG_OK;
 }
 

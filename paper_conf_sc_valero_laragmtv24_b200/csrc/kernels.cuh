@@ -100,6 +100,27 @@ __device__ __forceinline__ int2 ld_stream2(const int *ptr, uint64_t pol) {
 __device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
 __device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;"); }
 
+// Device-side trace (HPCCG_OPT_TRACE): for traced iteration k and CG kernel j
+// (0 p update, 1 SpMV, 2 x/r update) the earliest block start and the latest
+// block end on %globaltimer (ns), so per-kernel times and the gaps between
+// kernels can be read even inside the while-graph (no events allowed there).
+struct TraceSlot {
+    unsigned long long t0, t1;
+};
+
+__device__ __forceinline__ unsigned long long gtimer() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
+
+__device__ __forceinline__ void trace_mark(TraceSlot *tr, int trace_max, int k, int j, bool end) {
+    if (!tr || threadIdx.x != 0 || k < 1 || k > trace_max) return;
+    TraceSlot *s = tr + (size_t)(k - 1) * 3 + j;
+    if (end) atomicMax(&s->t1, gtimer());
+    else atomicMin(&s->t0, gtimer());
+}
+
 __device__ __forceinline__ double warp_sum(double v) {
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
@@ -232,6 +253,8 @@ struct SpmvArgs {
     // last-block finisher (its fence + ticket costs ~6 us per SpMV on B200);
     // the update kernel sums the partials itself.  nullptr: finisher.
     double *parts_only;
+    TraceSlot *trace;  // HPCCG_OPT_TRACE (nullptr: off)
+    int trace_max;
 };
 
 // kDot: CG variant with the p.Ap epilogue.  kCheck: return at once when the
@@ -275,6 +298,7 @@ __global__ void __launch_bounds__(kBlock, kMinB) spmv27_kernel(SpmvArgs a) {
             }
             if (g == 0) {
                 pdl_wait();
+                if (kDot && a.trace) trace_mark(a.trace, a.trace_max, __ldg(&a.sc->k), 1, false);
                 if (kDot && kCheck) done = __ldg(&a.sc->done);
                 if (done) return;  // uniform over the grid, before any store
             }
@@ -298,6 +322,7 @@ __global__ void __launch_bounds__(kBlock, kMinB) spmv27_kernel(SpmvArgs a) {
     }
     pdl_trigger();
     if (done) return;
+    if (kDot && a.trace) trace_mark(a.trace, a.trace_max, __ldg(&a.sc->k), 1, true);
     if (kDot) {
         if (a.parts_only) {  // block partial only; the update kernel sums them
             __shared__ double shp[32];
@@ -351,6 +376,7 @@ __global__ void __launch_bounds__(kBlock, 4) spmv27x2_kernel(SpmvArgs a) {
             }
             if (g == 0) {
                 pdl_wait();
+                if (kDot && a.trace) trace_mark(a.trace, a.trace_max, __ldg(&a.sc->k), 1, false);
                 if (kDot && kCheck) done = __ldg(&a.sc->done);
                 if (done) return;  // uniform over the grid, before any store
             }
@@ -391,6 +417,7 @@ __global__ void __launch_bounds__(kBlock, 4) spmv27x2_kernel(SpmvArgs a) {
     }
     pdl_trigger();
     if (done) return;
+    if (kDot && a.trace) trace_mark(a.trace, a.trace_max, __ldg(&a.sc->k), 1, true);
     if (kDot) {
         if (a.parts_only) {  // block partial only; the update kernel sums them
             __shared__ double shp[32];
@@ -430,9 +457,12 @@ __device__ __forceinline__ int64_t gnth() { return (int64_t)gridDim.x * kBlock; 
 template <bool kVec, bool kCheck, int kU>
 __global__ void __launch_bounds__(kBlock) cg_pupdate_kernel(int64_t n, const double *__restrict__ r,
                                                            double *__restrict__ p,
-                                                           const CgScalars *sc) {
+                                                           const CgScalars *sc, TraceSlot *trace,
+                                                           int trace_max) {
     pdl_wait();
     pdl_trigger();
+    const int ktr = trace ? __ldg(&sc->k) : 0;
+    trace_mark(trace, trace_max, ktr, 0, false);
     // `done` is tested after each trip's loads (never in front of them)
     const int done = kCheck ? __ldg(&sc->done) : 0;
     const bool first = (__ldg(&sc->k) == 1);
@@ -475,6 +505,10 @@ __global__ void __launch_bounds__(kBlock) cg_pupdate_kernel(int64_t n, const dou
         if (done) return;
         for (int64_t i = tid; i < n; i += nth) p[i] = first ? r[i] : fma(beta, p[i], r[i]);
     }
+    if (trace) {
+        __syncthreads();  // the block's stores are issued before its end mark
+        trace_mark(trace, trace_max, ktr, 0, true);
+    }
 }
 
 // a.5: x += alpha p; r -= alpha Ap; partial r.r; then the loop control of
@@ -486,6 +520,8 @@ struct UpdArgs {
     const double *p, *Ap;
     const double *pAp_parts;  // non-null: p.Ap = fixed-order sum of these
     unsigned n_parts;
+    TraceSlot *trace;
+    int trace_max;
     CgScalars *sc;
     Reduction red;
     int single;
@@ -521,6 +557,8 @@ __global__ void __launch_bounds__(kBlock) cg_update_kernel(UpdArgs a) {
     CgScalars *sc = a.sc;
     pdl_wait();
     pdl_trigger();
+    const int ktr = a.trace ? __ldg(&sc->k) : 0;
+    trace_mark(a.trace, a.trace_max, ktr, 2, false);
     // `done` is tested after each trip's loads (never in front of them); it
     // is uniform over the grid, so every block leaves before the reduction.
     const int done = kCheck ? __ldg(&sc->done) : 0;
@@ -597,6 +635,7 @@ __global__ void __launch_bounds__(kBlock) cg_update_kernel(UpdArgs a) {
     }
     const int single = a.single;
     const unsigned long long cond = a.cond;
+    trace_mark(a.trace, a.trace_max, ktr, 2, true);
     grid_reduce<false>(acc, a.red, blockIdx.x, gridDim.x,
                        [sc, single, rtrans, stop, cond, pAp](double s) {
                            sc->pAp = pAp;

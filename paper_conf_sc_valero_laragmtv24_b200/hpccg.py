@@ -35,7 +35,7 @@ HPCCG_OPT_GRAPH, HPCCG_OPT_POLL, HPCCG_OPT_TIMING = 0, 1, 2
 HPCCG_OPT_SPMV_MINB, HPCCG_OPT_WHILE, HPCCG_OPT_L2_PERSIST, HPCCG_OPT_VEC_WAVES = 3, 4, 5, 6
 HPCCG_OPT_SPMV_ROWS, HPCCG_OPT_VEC_UNROLL = 7, 8
 HPCCG_OPT_PERSISTENT, HPCCG_OPT_PERSIST_ROWS, HPCCG_OPT_PDL = 9, 10, 11
-HPCCG_OPT_CLUSTER_ROWS, HPCCG_OPT_SMEM_SOLVE = 12, 13
+HPCCG_OPT_CLUSTER_ROWS, HPCCG_OPT_SMEM_SOLVE, HPCCG_OPT_TRACE = 12, 13, 14
 
 _lock = threading.Lock()
 _lib = None
@@ -83,6 +83,7 @@ _SIGS = {
     "hpccg_waxpby": ([_vp, _i64, _d, _vp, _d, _vp, _vp], _i),
     "hpccg_solve": ([_vp, _i, _d, ctypes.POINTER(_i), ctypes.POINTER(_d), _vp], _i),
     "hpccg_get_stats": ([_vp, ctypes.POINTER(hpccg_stats)], _i),
+    "hpccg_get_trace": ([_vp, _vp, _i64], _i),
     "hpccg_maxabsdiff": ([_vp, ctypes.POINTER(_d)], _i),
     "hpccg_free": ([_vp], None),
     "hpccg_waxpby2d": ([_vp, _i64, _i64, _i64, _d, _vp, _d, _vp, _vp], _i),
@@ -355,6 +356,12 @@ class Problem:
 
     def maxabsdiff(self) -> float:
         return hpccg_maxabsdiff(self.handle)
+
+    def trace(self, k: int) -> np.ndarray:
+        """[k, 3, 2] uint64 ns: (start, end) of p update / SpMV / update per iteration."""
+        out = np.zeros(6 * k, dtype=np.uint64)
+        _check(lib().hpccg_get_trace(self.handle, out.ctypes.data, k), "hpccg_get_trace")
+        return out.reshape(k, 3, 2)
 
     def get_vec(self, which: int, out: np.ndarray | None = None) -> np.ndarray:
         """Host copy (nslabs * n doubles).  `out` may be a pinned buffer."""
