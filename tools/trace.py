@@ -10,7 +10,8 @@ sys.argv += [] if len(sys.argv) > 5 else [""]
 nx, ny, nz, iters = (int(v) for v in sys.argv[1:5])
 KEYS = {"graph": H.HPCCG_OPT_GRAPH, "timing": H.HPCCG_OPT_TIMING, "while": H.HPCCG_OPT_WHILE,
         "pdl": H.HPCCG_OPT_PDL, "waves": H.HPCCG_OPT_VEC_WAVES, "unroll": H.HPCCG_OPT_VEC_UNROLL,
-        "rows": H.HPCCG_OPT_SPMV_ROWS, "l2": H.HPCCG_OPT_L2_PERSIST}
+        "rows": H.HPCCG_OPT_SPMV_ROWS, "l2": H.HPCCG_OPT_L2_PERSIST,
+        "wu": H.HPCCG_OPT_WHILE_UNROLL}
 ctx = H.Context(0)
 p = H.Problem(ctx, nx, ny, nz)
 p.set_option(H.HPCCG_OPT_PERSISTENT, 0)
@@ -43,4 +44,4 @@ for spec in sys.argv[5:]:
     p.set_option(H.HPCCG_OPT_TRACE, 0)
     for k in opts:
         p.set_option(KEYS[k], {"graph": 1, "while": 1, "pdl": 1, "waves": 1, "unroll": 4, "rows": 2,
-                               "l2": 1}.get(k, 0))
+                               "l2": 1, "wu": 1}.get(k, 0))
