@@ -93,7 +93,7 @@ extern "C" {
                                (%globaltimer; works inside graphs); read with
                                hpccg_get_trace.  0 (default): off */
 #define HPCCG_OPT_WHILE_UNROLL 15 /* CG iterations per execution of the WHILE body
-                               (default 1; > 1 amortises the conditional node's cost) */
+                               (default 4: amortises the conditional node's ~8 us) */
 #define HPCCG_OPT_CLUSTER_ROWS 12 /* up to this many rows (default 16384) the persistent solve
                                is ONE thread-block cluster (<= 16 CTAs) synchronised by the
                                hardware cluster barrier; above, a cooperative grid with a

@@ -144,7 +144,7 @@ struct hpccg_problem {
     int64_t opt_persist_rows = 65536;
     int64_t opt_cluster_rows = 16384;  // persistent solve as one cluster up to this many rows
     int opt_smem = 1;                  // persistent solve resident in cluster shared memory if it fits
-    int opt_while_unroll = 1;          // CG iterations per WHILE-body execution
+    int opt_while_unroll = 4;          // CG iterations per WHILE-body execution
     int last_persist_mode = 3;
     // graph of one CG iteration (per-iteration replay) ...
     cudaGraphExec_t graph = nullptr;

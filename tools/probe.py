@@ -44,6 +44,6 @@ for spec in sys.argv[5:]:
     print(json.dumps(out), flush=True)
     for k in opts:
         try:
-            p.set_option(KEYS[k], {"graph": 1, "while": 1, "l2": 1, "waves": 1, "rows": 2, "unroll": 4, "persist": 1, "pdl": 1, "crows": 16384, "smem": 1, "wu": 1}.get(k, 0))
+            p.set_option(KEYS[k], {"graph": 1, "while": 1, "l2": 1, "waves": 1, "rows": 2, "unroll": 4, "persist": 1, "pdl": 1, "crows": 16384, "smem": 1, "wu": 4}.get(k, 0))
         except H.HpccgError:
             pass

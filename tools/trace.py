@@ -44,4 +44,4 @@ for spec in sys.argv[5:]:
     p.set_option(H.HPCCG_OPT_TRACE, 0)
     for k in opts:
         p.set_option(KEYS[k], {"graph": 1, "while": 1, "pdl": 1, "waves": 1, "unroll": 4, "rows": 2,
-                               "l2": 1, "wu": 1}.get(k, 0))
+                               "l2": 1, "wu": 4}.get(k, 0))
