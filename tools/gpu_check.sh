@@ -15,4 +15,4 @@ if [ -n "${NCU}" ]; then
   timeout 900 ncu --set full --clock-control none --import-source on -k regex:"cg_update|cg_pupdate" -s 4 -c 2 \
      -o gpurun_out/prof_upd -f python bench.py --steps 1 --warmup 3 --iters 5 --no-cpu-baseline > gpurun_out/ncu_full_upd.log 2>&1
 fi
-tail -3 gpurun_out/*.log
+tail -n 3 gpurun_out/*.log

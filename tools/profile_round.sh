@@ -15,4 +15,4 @@ timeout 900 ncu --set full --clock-control none --import-source on -k regex:spmv
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:"cg_update|cg_pupdate" -s 6 -c 2 \
     -o gpurun_out/prof_vec -f python bench.py --steps 1 --warmup 3 --iters 5 --no-cpu-baseline \
     > gpurun_out/ncu_vec.log 2>&1
-tail -2 gpurun_out/*.log
+tail -n 2 gpurun_out/*.log
