@@ -92,6 +92,14 @@ extern "C" {
                                first-block start and last-block end on the device clock
                                (%globaltimer; works inside graphs); read with
                                hpccg_get_trace.  0 (default): off */
+#define HPCCG_OPT_CG_VARIANT 16 /* 0 (default): HPCCG's CG (SpMV + p.Ap, x/r update + r.r,
+                               p update; two reductions per iteration).  1: single-reduction
+                               (Chronopoulos-Gear) CG: same iterates in exact
+                               arithmetic, two kernels per iteration (one fused update of
+                               p, s = A p, x, r; the SpMV w = A r with r.r and w.r in its
+                               epilogue) and ONE allreduce of two values; needs 8n more bytes
+                               (s), small problems use the graph path instead of the
+                               persistent kernel.  Rounding differs: niters +-1 */
 #define HPCCG_OPT_WHILE_UNROLL 15 /* CG iterations per execution of the WHILE body
                                (default 4: amortises the conditional node's ~8 us) */
 #define HPCCG_OPT_CLUSTER_ROWS 12 /* up to this many rows (default 16384) the persistent solve

@@ -117,8 +117,9 @@ struct Slab {
     TraceSlot *trace = nullptr;  // HPCCG_OPT_TRACE buffer: [trace_max][3]
     int trace_max = 0;
     bool trace_on = false;
-    double *spmv_parts = nullptr;  // per-block p.Ap partials (single slab)
+    double *spmv_parts = nullptr;  // per-block p.Ap partials (single slab); f2: 2 arrays
     int64_t spmv_nparts = 0;
+    double *sv = nullptr;  // f2 single-reduction CG: s = A p recurrence vector (n)
 };
 
 struct TimedOp {
@@ -133,7 +134,7 @@ struct hpccg_problem {
     unsigned long long nnz_global = 0;
     int64_t red_cap = 0;  // partial slots per slab reduction scratch
     // loopback allreduce tables (device arrays of device pointers)
-    double **d_tab = nullptr;  // [6][nslabs]: src pAp, dst pAp, src rr, dst rr, src red, dst red
+    double **d_tab = nullptr;  // [8][nslabs]: src/dst pAp, src/dst rr, src/dst red, src/dst gd (f2)
     // options
     int opt_graph = 1, opt_poll = 8, opt_timing = 0, opt_minb = 0, opt_while = 1, opt_l2 = 1;
     int opt_vec_waves = 1;  // 0: one thread per double2 (full grid); k: k resident waves
@@ -145,6 +146,7 @@ struct hpccg_problem {
     int64_t opt_cluster_rows = 16384;  // persistent solve as one cluster up to this many rows
     int opt_smem = 1;                  // persistent solve resident in cluster shared memory if it fits
     int opt_while_unroll = 4;          // CG iterations per WHILE-body execution
+    int opt_variant = 0;               // 0 HPCCG CG, 1 single-reduction CG (f2)
     int last_persist_mode = 3;
     // graph of one CG iteration (per-iteration replay) ...
     cudaGraphExec_t graph = nullptr;
@@ -260,14 +262,14 @@ struct PhaseTimer {  // records a begin/end event pair on `s` when timing is on
 // slabs / ranks.  Single: plain device copy is unnecessary (kernels write
 // the global value directly), so this is only called for nslabs/nranks > 1.
 int allreduce_scalar(hpccg_ctx *ctx, double *const *h_src, double *const *h_dst,
-                     double *const *d_src, double *const *d_dst, bool is_max) {
+                     double *const *d_src, double *const *d_dst, bool is_max, int count = 1) {
     if (ctx->mode == MODE_LOOPBACK) {
-        slab_allreduce_kernel<<<1, 32, 0, ctx->stream>>>(d_src, d_dst, ctx->nslabs, is_max);
+        slab_allreduce_kernel<<<1, 32, 0, ctx->stream>>>(d_src, d_dst, ctx->nslabs, is_max, count);
         return check_launch(ctx);
     }
 #ifdef HPCCG_WITH_NCCL
     if (ctx->mode == MODE_NCCL) {
-        NC(ctx, ncclAllReduce(h_src[0], h_dst[0], 1, ncclDouble, is_max ? ncclMax : ncclSum,
+        NC(ctx, ncclAllReduce(h_src[0], h_dst[0], count, ncclDouble, is_max ? ncclMax : ncclSum,
                               ctx->comm, ctx->stream));
         return HPCCG_OK;
     }
@@ -350,14 +352,14 @@ SpmvArgs spmv_args(const Slab &s, const double *x, double *y) {
 // kMinB of the SpMV (register budget): tuned on B200, see DESIGN.md sec. 7.
 constexpr int kSpmvMinBDefault = 4;
 
-template <bool kDot, bool kCheck>
+template <int kDots, bool kCheck>
 int launch_spmv_t(hpccg_ctx *ctx, int minb, const SpmvArgs &a, unsigned blocks, cudaStream_t st,
                   bool pdl) {
     switch (minb) {
-        case 1: launch_k(pdl, spmv27_kernel<kDot, kCheck, 1>, dim3(blocks), st, a); break;
-        case 3: launch_k(pdl, spmv27_kernel<kDot, kCheck, 3>, dim3(blocks), st, a); break;
-        case 4: launch_k(pdl, spmv27_kernel<kDot, kCheck, 4>, dim3(blocks), st, a); break;
-        default: launch_k(pdl, spmv27_kernel<kDot, kCheck, 2>, dim3(blocks), st, a); break;
+        case 1: launch_k(pdl, spmv27_kernel<kDots, kCheck, 1>, dim3(blocks), st, a); break;
+        case 3: launch_k(pdl, spmv27_kernel<kDots, kCheck, 3>, dim3(blocks), st, a); break;
+        case 4: launch_k(pdl, spmv27_kernel<kDots, kCheck, 4>, dim3(blocks), st, a); break;
+        default: launch_k(pdl, spmv27_kernel<kDots, kCheck, 2>, dim3(blocks), st, a); break;
     }
     return check_launch(ctx);
 }
@@ -373,7 +375,7 @@ int spmv_rows_per_thread(int opt_rows, const SpmvArgs &a, int64_t r0, int64_t r1
 
 int64_t spmv_blocks(int64_t len, int rows) { return cdiv(cdiv(len, rows), kBlock); }
 
-template <bool kDot>
+template <int kDots>
 int launch_spmv(hpccg_ctx *ctx, int minb, bool check, SpmvArgs a, int64_t r0, int64_t len0,
                 int64_t r1, int64_t len1, cudaStream_t st, int rows = 1, bool pdl = false) {
     a.r0 = r0;
@@ -385,20 +387,20 @@ int launch_spmv(hpccg_ctx *ctx, int minb, bool check, SpmvArgs a, int64_t r0, in
     if (blocks == 0) return HPCCG_OK;
     if (blocks > 0x7fffffffLL) return fail(HPCCG_EINVAL, "SpMV grid too large");
     if (rows == 2) {
-        if (check) launch_k(pdl, spmv27x2_kernel<kDot, true>, dim3((unsigned)blocks), st, a);
-        else launch_k(pdl, spmv27x2_kernel<kDot, false>, dim3((unsigned)blocks), st, a);
+        if (check) launch_k(pdl, spmv27x2_kernel<kDots, true>, dim3((unsigned)blocks), st, a);
+        else launch_k(pdl, spmv27x2_kernel<kDots, false>, dim3((unsigned)blocks), st, a);
         return check_launch(ctx);
     }
     if (minb <= 0) minb = kSpmvMinBDefault;
-    return check ? launch_spmv_t<kDot, true>(ctx, minb, a, (unsigned)blocks, st, pdl)
-                 : launch_spmv_t<kDot, false>(ctx, minb, a, (unsigned)blocks, st, pdl);
+    return check ? launch_spmv_t<kDots, true>(ctx, minb, a, (unsigned)blocks, st, pdl)
+                 : launch_spmv_t<kDots, false>(ctx, minb, a, (unsigned)blocks, st, pdl);
 }
 
 // y = A x for one slab over all rows (no dot).
 int spmv_plain(hpccg_ctx *ctx, int minb, int opt_rows, const Slab &s, const double *x, double *y,
                cudaStream_t st) {
     SpmvArgs a = spmv_args(s, x, y);
-    return launch_spmv<false>(ctx, minb, false, a, 0, s.n, 0, 0, st,
+    return launch_spmv<0>(ctx, minb, false, a, 0, s.n, 0, 0, st,
                               spmv_rows_per_thread(opt_rows, a, 0, 0));
 }
 
@@ -513,7 +515,7 @@ int cg_spmv_all(hpccg_problem *p, bool timing, bool check) {
         a.part_base = 0;
         a.total_blocks = (unsigned)spmv_blocks(s.n, rows);
         a.parts_only = s.spmv_parts;  // the update kernel finishes p.Ap
-        return launch_spmv<true>(ctx, minb, check, a, 0, s.n, 0, 0, ctx->stream, rows,
+        return launch_spmv<1>(ctx, minb, check, a, 0, s.n, 0, 0, ctx->stream, rows,
                                  p->opt_pdl != 0);
     }
     const Slab &s0 = p->slabs[0];
@@ -542,10 +544,10 @@ int cg_spmv_all(hpccg_problem *p, bool timing, bool check) {
         a.single = 0;
         a.total_blocks = nb_int + nb_bnd;
         a.part_base = 0;
-        CHECK(launch_spmv<true>(ctx, minb, check, a, int_r0, int_len, 0, 0, ctx->stream, rows));
+        CHECK(launch_spmv<1>(ctx, minb, check, a, int_r0, int_len, 0, 0, ctx->stream, rows));
         CU(cudaStreamWaitEvent(ctx->stream, ctx->ev_join, 0));
         a.part_base = nb_int;
-        return launch_spmv<true>(ctx, minb, check, a, 0, b0_len, b1_r0, b1_len, ctx->stream, rows);
+        return launch_spmv<1>(ctx, minb, check, a, 0, b0_len, b1_r0, b1_len, ctx->stream, rows);
     }
     // loopback: exchange, then interior + boundary launches per slab
     {
@@ -558,9 +560,9 @@ int cg_spmv_all(hpccg_problem *p, bool timing, bool check) {
         a.single = 0;
         a.total_blocks = nb_int + nb_bnd;
         a.part_base = 0;
-        CHECK(launch_spmv<true>(ctx, minb, check, a, int_r0, int_len, 0, 0, ctx->stream, rows));
+        CHECK(launch_spmv<1>(ctx, minb, check, a, int_r0, int_len, 0, 0, ctx->stream, rows));
         a.part_base = nb_int;
-        CHECK(launch_spmv<true>(ctx, minb, check, a, 0, b0_len, b1_r0, b1_len, ctx->stream, rows));
+        CHECK(launch_spmv<1>(ctx, minb, check, a, 0, b0_len, b1_r0, b1_len, ctx->stream, rows));
     }
     return HPCCG_OK;
 }
@@ -648,6 +650,226 @@ int enqueue_init(hpccg_problem *p, int max_iter, double tol, bool timing,
         CHECK(check_launch(ctx));
     }
     return HPCCG_OK;
+}
+
+// ------------------------------------ f2: single-reduction CG orchestration
+// Buffers (same arena as HPCCG's CG): the GATHERED vector is r here, so r
+// lives in the halo buffer s.p; w = A r in s.Ap; p (not gathered) in s.r;
+// the s = A p recurrence in s.sv; x in s.x.
+
+// SpMV partial count of a single slab's CG SpMV (the update sums them).
+unsigned single_spmv_parts(const hpccg_problem *p, const Slab &s) {
+    return (unsigned)spmv_blocks(s.n, spmv_rows_per_thread(p->opt_rows, spmv_args(s, s.p, s.Ap), 0, 0));
+}
+
+// w = A r with the (gamma, delta) epilogue for every slab; multi-slab: halo
+// exchange overlapped with the interior rows (NCCL), per-slab finisher, and
+// ONE allreduce of the two values.  q: parity of the iteration (run flag).
+int cg_sr_spmv_all(hpccg_problem *p, bool timing, bool check, int q) {
+    hpccg_ctx *ctx = p->ctx;
+    const int minb = p->opt_minb;
+    const bool pdl = ctx->mode == MODE_SINGLE && p->opt_pdl;
+    auto finish = [&](const Slab &s, unsigned np, double *out) {
+        cudaLaunchConfig_t cfg{};
+        cfg.gridDim = dim3(1);
+        cfg.blockDim = dim3(kBlock);
+        cfg.stream = ctx->stream;
+        cudaLaunchAttribute at[1];
+        at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+        at[0].val.programmaticStreamSerializationAllowed = 1;
+        cfg.attrs = pdl ? at : nullptr;
+        cfg.numAttrs = pdl ? 1 : 0;
+        CU(cudaLaunchKernelEx(&cfg, cg_sr_finish_kernel, (const double *)s.spmv_parts, np, out));
+        return check_launch(ctx);
+    };
+    if (ctx->mode == MODE_SINGLE) {
+        const Slab &s = p->slabs[0];
+        PhaseTimer t(p, ctx->stream, PH_SPMV, timing);
+        SpmvArgs a = spmv_args(s, s.p, s.Ap);
+        a.trace = nullptr;
+        const int rows = spmv_rows_per_thread(p->opt_rows, a, 0, 0);
+        a.single = 1;
+        a.part_base = 0;
+        a.total_blocks = (unsigned)spmv_blocks(s.n, rows);
+        a.parts_only = s.spmv_parts;
+        a.sr_q = q;
+        CHECK(launch_spmv<2>(ctx, minb, check, a, 0, s.n, 0, 0, ctx->stream, rows, pdl));
+        // too many partials for every update block to sum: one finisher block
+        if (a.total_blocks > kUpdSumMax) CHECK(finish(s, a.total_blocks, s.sc->gd));
+        return HPCCG_OK;
+    }
+    const Slab &s0 = p->slabs[0];
+    const int64_t n = s0.n, plane = s0.plane;
+    const int64_t int_r0 = plane, int_len = std::max<int64_t>(n - 2 * plane, 0);
+    const int64_t b0_len = std::min<int64_t>(plane, n);
+    const int64_t b1_r0 = std::max<int64_t>(n - plane, plane), b1_len = n - b1_r0;
+    const int rows = spmv_rows_per_thread(p->opt_rows, spmv_args(s0, s0.p, s0.Ap), int_r0, b1_r0);
+    const unsigned nb_int = (unsigned)spmv_blocks(int_len, rows);
+    const unsigned nb_bnd = (unsigned)(spmv_blocks(b0_len, rows) + spmv_blocks(b1_len, rows));
+    std::vector<double *> xs(p->slabs.size());
+    for (size_t i = 0; i < xs.size(); ++i) xs[i] = p->slabs[i].p;
+    auto slab_spmv = [&](const Slab &s, bool interior) {
+        SpmvArgs a = spmv_args(s, s.p, s.Ap);
+        a.trace = nullptr;
+        a.single = 0;
+        a.total_blocks = nb_int + nb_bnd;
+        a.parts_only = s.spmv_parts;
+        a.sr_q = q;
+        if (interior) {
+            a.part_base = 0;
+            return launch_spmv<2>(ctx, minb, check, a, int_r0, int_len, 0, 0, ctx->stream, rows);
+        }
+        a.part_base = nb_int;
+        return launch_spmv<2>(ctx, minb, check, a, 0, b0_len, b1_r0, b1_len, ctx->stream, rows);
+    };
+    if (ctx->mode == MODE_NCCL) {
+        CU(cudaEventRecord(ctx->ev_fork, ctx->stream));
+        CU(cudaStreamWaitEvent(ctx->comm_stream, ctx->ev_fork, 0));
+        {
+            PhaseTimer t(p, ctx->comm_stream, PH_EXCHANGE, timing);
+            CHECK(exchange(p, xs.data(), ctx->comm_stream));
+        }
+        CU(cudaEventRecord(ctx->ev_join, ctx->comm_stream));
+        PhaseTimer t(p, ctx->stream, PH_SPMV, timing);
+        CHECK(slab_spmv(p->slabs[0], true));
+        CU(cudaStreamWaitEvent(ctx->stream, ctx->ev_join, 0));
+        CHECK(slab_spmv(p->slabs[0], false));
+    } else {
+        {
+            PhaseTimer t(p, ctx->stream, PH_EXCHANGE, timing);
+            CHECK(exchange(p, xs.data(), ctx->stream));
+        }
+        PhaseTimer t(p, ctx->stream, PH_SPMV, timing);
+        for (const Slab &s : p->slabs) {
+            CHECK(slab_spmv(s, true));
+            CHECK(slab_spmv(s, false));
+        }
+    }
+    for (const Slab &s : p->slabs) CHECK(finish(s, nb_int + nb_bnd, s.sc->loc_gd));
+    PhaseTimer t(p, ctx->stream, PH_ALLREDUCE, timing);
+    double *hs[1] = {p->slabs[0].sc->loc_gd};
+    double *hd[1] = {p->slabs[0].sc->gd};
+    return allreduce_scalar(ctx, hs, hd, tab(p, 6), tab(p, 7), false, 2);
+}
+
+template <bool kVec, int kU>
+int launch_sr_update_t(hpccg_ctx *ctx, int waves, const SrUpdArgs &a, bool pdl) {
+    auto k = cg_sr_update_kernel<kVec, kU>;
+    const int g = vec_grid(ctx, k, kVec ? cdiv(a.n, 2 * kU) : a.n, waves, 0x7fffffff);
+    launch_k(pdl, k, dim3(g), ctx->stream, a);
+    return check_launch(ctx);
+}
+
+int launch_sr_update(hpccg_problem *p, const Slab &s, int q, unsigned long long cond, bool pdl) {
+    hpccg_ctx *ctx = p->ctx;
+    SrUpdArgs a{};
+    a.n = s.n;
+    a.x = s.x;
+    a.r = s.p + s.plane;
+    a.p = s.r;
+    a.s = s.sv;
+    a.w = s.Ap;
+    a.sc = s.sc;
+    a.q = q;
+    a.cond = cond;
+    if (ctx->mode == MODE_SINGLE) {
+        const unsigned np = single_spmv_parts(p, s);
+        if (np <= kUpdSumMax) {
+            a.parts = s.spmv_parts;
+            a.n_parts = np;
+        }
+    }
+    const int waves = p->opt_vec_waves;
+    const bool vec = aligned16(a.x) && aligned16(a.r) && aligned16(a.p) && aligned16(a.s) &&
+                     aligned16(a.w);
+    if (!vec) return launch_sr_update_t<false, 1>(ctx, waves, a, pdl);
+    switch (p->opt_unroll) {
+        case 1: return launch_sr_update_t<true, 1>(ctx, waves, a, pdl);
+        case 2: return launch_sr_update_t<true, 2>(ctx, waves, a, pdl);
+        default: return launch_sr_update_t<true, 4>(ctx, waves, a, pdl);
+    }
+}
+
+// One f2 iteration of parity q: the fused update, then w = A r + (gamma, delta).
+int enqueue_iteration_sr(hpccg_problem *p, bool timing, bool check, unsigned long long cond, int q) {
+    hpccg_ctx *ctx = p->ctx;
+    const bool pdl = ctx->mode == MODE_SINGLE && p->opt_pdl;
+    {
+        PhaseTimer t(p, ctx->stream, PH_UPDATE, timing);
+        for (size_t i = 0; i < p->slabs.size(); ++i)
+            CHECK(launch_sr_update(p, p->slabs[i], q, i == 0 ? cond : 0ull, pdl));
+    }
+    return cg_sr_spmv_all(p, timing, check, q);
+}
+
+// f2 init: r = b - A x (r in the halo buffer), w = A r, (gamma, delta), state.
+int enqueue_init_sr(hpccg_problem *p, int max_iter, double tol, bool timing,
+                    unsigned long long cond) {
+    hpccg_ctx *ctx = p->ctx;
+    const int single = ctx->mode == MODE_SINGLE;
+    for (const Slab &s : p->slabs) {
+        copy_kernel<<<wave_grid(s.n, wave(ctx, copy_kernel)), kBlock, 0, ctx->stream>>>(
+            s.n, s.x, s.p + s.plane);
+        CHECK(check_launch(ctx));
+    }
+    std::vector<double *> xs(p->slabs.size());
+    for (size_t i = 0; i < xs.size(); ++i) xs[i] = p->slabs[i].p;
+    {
+        PhaseTimer t(p, ctx->stream, PH_EXCHANGE, timing);
+        CHECK(exchange(p, xs.data(), ctx->stream));
+    }
+    {
+        PhaseTimer t(p, ctx->stream, PH_SPMV, timing);
+        for (const Slab &s : p->slabs)
+            CHECK(spmv_plain(ctx, p->opt_minb, p->opt_rows, s, s.p, s.Ap, ctx->stream));
+    }
+    {
+        PhaseTimer t(p, ctx->stream, PH_UPDATE, timing);
+        for (const Slab &s : p->slabs) {  // r = b - A x0 (its r.r goes unused)
+            InitResArgs a{};
+            a.n = s.n;
+            a.b = s.b;
+            a.Ap = s.Ap;
+            a.r = s.p + s.plane;
+            a.sc = s.sc;
+            a.red = s.red;
+            a.single = single;
+            cg_initres_kernel<<<wave_grid(s.n, wave(ctx, cg_initres_kernel)), kBlock, 0,
+                                ctx->stream>>>(a);
+            CHECK(check_launch(ctx));
+        }
+    }
+    CHECK(cg_sr_spmv_all(p, timing, false, 0));
+    for (size_t i = 0; i < p->slabs.size(); ++i) {
+        const Slab &s = p->slabs[i];
+        const double *parts = nullptr;
+        unsigned np = 0;
+        if (single && single_spmv_parts(p, s) <= kUpdSumMax) {
+            parts = s.spmv_parts;
+            np = single_spmv_parts(p, s);
+        }
+        cg_sr_initstate_kernel<<<1, kBlock, 0, ctx->stream>>>(parts, np, s.sc, max_iter, tol,
+                                                             i == 0 ? cond : 0ull);
+        CHECK(check_launch(ctx));
+    }
+    return HPCCG_OK;
+}
+
+// Iterations captured per WHILE-body / per-iteration graph: f2 needs an even
+// count (each launch's iteration parity is baked into the captured node).
+int body_iterations(const hpccg_problem *p, int u) {
+    if (p->opt_variant == 0) return u;
+    return std::max(2, (u + 1) & ~1);
+}
+
+int enqueue_iteration_any(hpccg_problem *p, bool timing, bool check, unsigned long long cond, int k) {
+    if (p->opt_variant == 1) return enqueue_iteration_sr(p, timing, check, cond, k & 1);
+    return enqueue_iteration(p, timing, check, cond);
+}
+
+int enqueue_init_any(hpccg_problem *p, int max_iter, double tol, bool timing, unsigned long long cond) {
+    if (p->opt_variant == 1) return enqueue_init_sr(p, max_iter, tol, timing, cond);
+    return enqueue_init(p, max_iter, tol, timing, cond);
 }
 
 // L2 residency of the CG vectors (r, x, Ap, p: ~32n B): when they fit in the
@@ -793,7 +1015,9 @@ int build_graph(hpccg_problem *p) {
     cudaGraph_t g = nullptr;
     const int64_t l0 = ctx->launches;
     CU(cudaStreamBeginCapture(ctx->stream, cudaStreamCaptureModeThreadLocal));
-    int rc = enqueue_iteration(p, false, true, 0ull);
+    int rc = HPCCG_OK;
+    for (int k = 1; k <= body_iterations(p, 1) && rc == HPCCG_OK; ++k)
+        rc = enqueue_iteration_any(p, false, true, 0ull, k);
     cudaError_t e = cudaStreamEndCapture(ctx->stream, &g);
     if (rc != HPCCG_OK) {
         if (g) cudaGraphDestroy(g);
@@ -838,7 +1062,7 @@ int build_while_graph(hpccg_problem *p, int max_iter, double tol) {
                                       cudaStreamCaptureModeThreadLocal) != cudaSuccess)
         return bail(fail(HPCCG_ECUDA, "begin capture (init): %s",
                          cudaGetErrorString(cudaGetLastError())));
-    int rc = enqueue_init(p, max_iter, tol, false, (unsigned long long)h);
+    int rc = enqueue_init_any(p, max_iter, tol, false, (unsigned long long)h);
     cudaStreamCaptureStatus cs;
     const cudaGraphNode_t *deps = nullptr;
     size_t ndeps = 0;
@@ -870,9 +1094,9 @@ int build_while_graph(hpccg_problem *p, int max_iter, double tol) {
     // conditional node (~8 us measured with the device trace at 128^3) is paid
     // once per U iterations; with U > 1 the kernels test the device `done`
     // flag, so iterations after convergence inside a body are no-ops.
-    const int U = std::max(1, p->opt_while_unroll);
+    const int U = body_iterations(p, std::max(1, p->opt_while_unroll));
     for (int u = 0; u < U && rc == HPCCG_OK; ++u)
-        rc = enqueue_iteration(p, false, U > 1, (unsigned long long)h);
+        rc = enqueue_iteration_any(p, false, U > 1, (unsigned long long)h, 1 + u);
     e = cudaStreamEndCapture(ctx->stream, &gout);
     if (rc != HPCCG_OK) return bail(rc);
     if (e != cudaSuccess) return bail(fail(HPCCG_ECUDA, "end capture (body): %s", cudaGetErrorString(e)));
@@ -918,6 +1142,7 @@ void free_slab(Slab &s) {
     cudaFree(s.red.counter);
     cudaFree(s.bar);
     cudaFree(s.spmv_parts);
+    cudaFree(s.sv);
     cudaFree(s.trace);
     s = Slab{};
 }
@@ -1216,7 +1441,8 @@ int hpccg_generate(hpccg_ctx *ctx, int nx, int ny, int nz, hpccg_problem **out) 
         if ((rc = alloc_zero((void **)&s.red.partials, sizeof(double) * parts))) return bail(rc);
         if ((rc = alloc_zero((void **)&s.red.counter, sizeof(unsigned)))) return bail(rc);
         if ((rc = alloc_zero((void **)&s.bar, 64 * sizeof(unsigned)))) return bail(rc);
-        if ((rc = alloc_zero((void **)&s.spmv_parts, sizeof(double) * parts))) return bail(rc);
+        if ((rc = alloc_zero((void **)&s.spmv_parts, sizeof(double) * 2 * parts))) return bail(rc);
+        if ((rc = alloc_zero((void **)&s.sv, sizeof(double) * (size_t)(cdiv(n, 32) * 32)))) return bail(rc);
 
         GenArgs g{};
         g.nx = nx;
@@ -1265,8 +1491,8 @@ int hpccg_generate(hpccg_ctx *ctx, int nx, int ny, int nz, hpccg_problem **out) 
     if (ctx->mode == MODE_LOOPBACK) {
         const int P = ctx->nslabs;
         int rc;
-        if ((rc = alloc_zero((void **)&p->d_tab, sizeof(double *) * 6 * P))) return bail(rc);
-        std::vector<double *> t(6 * P);
+        if ((rc = alloc_zero((void **)&p->d_tab, sizeof(double *) * 8 * P))) return bail(rc);
+        std::vector<double *> t(8 * P);
         for (int s = 0; s < P; ++s) {
             CgScalars *sc = p->slabs[s].sc;
             t[0 * P + s] = &sc->loc_pAp;
@@ -1275,8 +1501,10 @@ int hpccg_generate(hpccg_ctx *ctx, int nx, int ny, int nz, hpccg_problem **out) 
             t[3 * P + s] = &sc->rr_cur;
             t[4 * P + s] = &sc->red_loc;
             t[5 * P + s] = &sc->red_out;
+            t[6 * P + s] = &sc->loc_gd[0];
+            t[7 * P + s] = &sc->gd[0];
         }
-        if (cudaMemcpy(p->d_tab, t.data(), sizeof(double *) * 6 * P, cudaMemcpyHostToDevice) !=
+        if (cudaMemcpy(p->d_tab, t.data(), sizeof(double *) * 8 * P, cudaMemcpyHostToDevice) !=
             cudaSuccess)
             return bail(fail(HPCCG_ECUDA, "generate: table upload"));
     }
@@ -1393,6 +1621,10 @@ int hpccg_set_option(hpccg_problem *p, int key, int64_t value) {
             p->opt_persist = (int)value;
             return HPCCG_OK;
         case HPCCG_OPT_SMEM_SOLVE: p->opt_smem = value != 0; return HPCCG_OK;
+        case HPCCG_OPT_CG_VARIANT:
+            if (value != 0 && value != 1) return fail(HPCCG_EINVAL, "cg variant: 0 or 1");
+            p->opt_variant = (int)value;
+            return HPCCG_OK;
         case HPCCG_OPT_WHILE_UNROLL:
             if (value < 1 || value > 64) return fail(HPCCG_EINVAL, "while unroll must be 1..64");
             p->opt_while_unroll = (int)value;
@@ -1552,7 +1784,7 @@ int hpccg_solve(hpccg_problem *p, int max_iter, double tol, int *niters, double 
     CU(cudaSetDevice(ctx->device));
     const bool timing = p->opt_timing != 0;
     const bool use_graph = p->opt_graph && !timing;
-    const bool use_persist = !timing && ctx->mode == MODE_SINGLE &&
+    const bool use_persist = !timing && ctx->mode == MODE_SINGLE && p->opt_variant == 0 &&
                              (p->opt_persist == 2 ||
                               (p->opt_persist == 1 && p->slabs[0].n <= p->opt_persist_rows));
     bool use_while = !use_persist && use_graph && p->opt_while && ctx->mode != MODE_NCCL &&
@@ -1580,9 +1812,10 @@ int hpccg_solve(hpccg_problem *p, int max_iter, double tol, int *niters, double 
     } else if (use_while) {
         CU(cudaGraphLaunch(p->wgraph, ctx->stream));
     } else {
-        CHECK(enqueue_init(p, max_iter, tol, timing, 0ull));
+        CHECK(enqueue_init_any(p, max_iter, tol, timing, 0ull));
         // at most max_iter - 1 iterations (A4); finished iterations turn the
         // remaining launches into no-ops on the device (done flag)
+        const int per_graph = body_iterations(p, 1);
         const int64_t iters = (int64_t)max_iter - 1;
         const int poll = (tol > 0.0) ? p->opt_poll : 0;
         const int *d_done = &p->slabs[0].sc->done;
@@ -1591,15 +1824,18 @@ int hpccg_solve(hpccg_problem *p, int max_iter, double tol, int *niters, double 
         bool stop = false;
         while (launched < iters && !stop) {
             const int64_t m = poll > 0 ? std::min<int64_t>(poll, iters - launched) : iters - launched;
-            for (int64_t i = 0; i < m; ++i) {
-                if (use_graph) {
+            int64_t i = 0;
+            while (i < m) {
+                if (use_graph) {  // per_graph iterations per replay
                     CU(cudaGraphLaunch(p->graph, ctx->stream));
                     ctx->launches += p->graph_kernels;
+                    i += per_graph;
                 } else {
-                    CHECK(enqueue_iteration(p, timing, true, 0ull));
+                    CHECK(enqueue_iteration_any(p, timing, true, 0ull, (int)(launched + i + 1)));
+                    ++i;
                 }
             }
-            launched += m;
+            launched += i;
             if (poll > 0 && launched < iters) {
                 // double-buffered poll: queue this chunk's flag copy, then look at
                 // the previous chunk's, so the GPU always has a chunk queued
@@ -1639,7 +1875,7 @@ int hpccg_solve(hpccg_problem *p, int max_iter, double tol, int *niters, double 
     }
     if (use_while) ctx->launches += p->wgraph_init_kernels + p->wgraph_body_kernels * hs.niters;
     st.iterations = hs.niters;
-    st.spmv_launches = hs.niters + 1;
+    st.spmv_launches = hs.niters + (p->opt_variant == 1 ? 2 : 1);
     st.kernel_launches = ctx->launches - l0;
     st.l2_persist_bytes = (int64_t)l2win.kept;
     st.graph_mode = use_persist ? p->last_persist_mode : (use_while ? 2 : (use_graph ? 1 : 0));

@@ -43,6 +43,17 @@ struct CgScalars {
     int niters;
     int done;         // loop-exit flag, read by every CG kernel
     int max_iter;
+    // f2 single-reduction CG (HPCCG_OPT_CG_VARIANT = 1).  Double-buffered by
+    // iteration parity q = k & 1: the update of iteration k reads slot q^1
+    // (written by iteration k-1, or by init for k = 1) and its block 0 writes
+    // slot q, so no block ever reads a slot another block of the same grid
+    // writes.
+    double sr_gamma[2];   // gamma_(k-1) = r_(k-1).r_(k-1) (global)
+    double sr_alpha[2];   // alpha_k
+    double gd[2];         // global (gamma, delta) when not summed from partials
+    double loc_gd[2];     // this slab's (gamma, delta) partial (allreduce input)
+    int sr_k[2];          // index of the next iteration
+    int sr_run[2];        // sr_run[q]: iteration k + 1 runs (written by iteration k)
 };
 
 // Scratch for the deterministic single-pass grid reduction.
@@ -255,14 +266,56 @@ struct SpmvArgs {
     double *parts_only;
     TraceSlot *trace;  // HPCCG_OPT_TRACE (nullptr: off)
     int trace_max;
+    int sr_q;          // kDots 2: parity of the iteration (run flag sr_run[sr_q])
 };
 
-// kDot: CG variant with the p.Ap epilogue.  kCheck: return at once when the
-// device `done` flag is set (plain / per-iteration-graph launches; the
-// while-graph never launches past convergence so it skips that load, whose
-// latency would otherwise sit in front of every block's first matrix load).
+template <int kDots, bool kCheck>
+__device__ __forceinline__ int spmv_done(const SpmvArgs &a) {
+    if (!kCheck || kDots == 0) return 0;
+    if (kDots == 2) return !__ldg(&a.sc->sr_run[a.sr_q]);
+    return __ldg(&a.sc->done);
+}
+
+// Block sums of two values in a fixed order; valid in thread 0.
+__device__ __forceinline__ double2 block_reduce2(double u, double v, double *sh /*[64]*/) {
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    __syncwarp();
+    u = warp_sum(u);
+    v = warp_sum(v);
+    if (lane == 0) {
+        sh[warp] = u;
+        sh[32 + warp] = v;
+    }
+    __syncwarp();
+    __syncthreads();
+    if (warp == 0) {
+        u = warp_sum(lane < kWarps ? sh[lane] : 0.0);
+        v = warp_sum(lane < kWarps ? sh[32 + lane] : 0.0);
+    }
+    return make_double2(u, v);
+}
+
+// kDots 2 epilogue: per-block (gamma, delta) partials.
+__device__ __forceinline__ void spmv_sr_partials(const SpmvArgs &a, double g, double d) {
+    __shared__ double sh2[64];
+    const double2 t = block_reduce2(g, d, sh2);
+    if (threadIdx.x == 0) {
+        a.parts_only[a.part_base + blockIdx.x] = t.x;
+        a.parts_only[a.total_blocks + a.part_base + blockIdx.x] = t.y;
+    }
+}
+
+// kDots: 0 plain y = A x; 1 CG epilogue p.Ap (x = p, y = Ap); 2 the f2
+// single-reduction epilogue gamma = x.x and delta = y.x (x = r, y = w = A r),
+// both from the diagonal slot's gathered value (no extra bytes), written as
+// per-block partials parts_only[b] and parts_only[total_blocks + b].
+// kCheck: return at once when the device `done` flag is set (kDots 2: when
+// the run flag sr_run[sr_q] says the next iteration does not run) -- plain /
+// per-iteration-graph launches; the while-graph never launches past
+// convergence so it skips that load, whose latency would otherwise sit in
+// front of every block's first matrix load).
 // kMinB: __launch_bounds__ min blocks per SM (register budget 65536/(256 kMinB)).
-template <bool kDot, bool kCheck, int kMinB>
+template <int kDots, bool kCheck, int kMinB>
 __global__ void __launch_bounds__(kBlock, kMinB) spmv27_kernel(SpmvArgs a) {
     int64_t row, lim;
     if ((int64_t)blockIdx.x < a.nb0) {
@@ -272,7 +325,8 @@ __global__ void __launch_bounds__(kBlock, kMinB) spmv27_kernel(SpmvArgs a) {
         row = a.r1 + ((int64_t)blockIdx.x - a.nb0) * kBlock + threadIdx.x;
         lim = a.r1 + a.len1;
     }
-    double d = 0.0;
+    constexpr bool kDot = kDots == 1;
+    double d = 0.0, dg = 0.0;  // kDots 1: p.Ap; kDots 2: delta (d) and gamma (dg)
     // The first matrix loads are issued before waiting for the predecessor
     // (PDL) and before the done flag is read, so neither latency sits in
     // front of the stream.
@@ -299,7 +353,7 @@ __global__ void __launch_bounds__(kBlock, kMinB) spmv27_kernel(SpmvArgs a) {
             if (g == 0) {
                 pdl_wait();
                 if (kDot && a.trace) trace_mark(a.trace, a.trace_max, __ldg(&a.sc->k), 1, false);
-                if (kDot && kCheck) done = __ldg(&a.sc->done);
+                done = spmv_done<kDots, kCheck>(a);
                 if (done) return;  // uniform over the grid, before any store
             }
 #pragma unroll
@@ -315,13 +369,21 @@ __global__ void __launch_bounds__(kBlock, kMinB) spmv27_kernel(SpmvArgs a) {
         a.y[row] = sum;
         // p_i: the diagonal slot's gathered value when that slot really is the
         // row's own column (always, for generated matrices); else reload it.
-        if (kDot) d = sum * (cd == row + a.plane ? xd : __ldg(a.x + row + a.plane));
+        if (kDots > 0) {
+            const double xi = cd == row + a.plane ? xd : __ldg(a.x + row + a.plane);
+            d = sum * xi;
+            if (kDots == 2) dg = xi * xi;
+        }
     } else {
         pdl_wait();
-        if (kDot && kCheck) done = __ldg(&a.sc->done);
+        done = spmv_done<kDots, kCheck>(a);
     }
     pdl_trigger();
     if (done) return;
+    if (kDots == 2) {
+        spmv_sr_partials(a, dg, d);
+        return;
+    }
     if (kDot && a.trace) trace_mark(a.trace, a.trace_max, __ldg(&a.sc->k), 1, true);
     if (kDot) {
         if (a.parts_only) {  // block partial only; the update kernel sums them
@@ -347,8 +409,9 @@ __global__ void __launch_bounds__(kBlock, kMinB) spmv27_kernel(SpmvArgs a) {
 // (tools/spmvbench.cu).  Needs even n (stride), even range starts and a 16-B
 // aligned y (the host checks); a range of odd length ends in a 1-row thread.
 // Same per-row FMA order as spmv27_kernel: identical bits.
-template <bool kDot, bool kCheck>
+template <int kDots, bool kCheck>
 __global__ void __launch_bounds__(kBlock, 4) spmv27x2_kernel(SpmvArgs a) {
+    constexpr bool kDot = kDots == 1;
     int64_t row, lim;
     if ((int64_t)blockIdx.x < a.nb0) {
         row = a.r0 + ((int64_t)blockIdx.x * kBlock + threadIdx.x) * 2;
@@ -357,7 +420,7 @@ __global__ void __launch_bounds__(kBlock, 4) spmv27x2_kernel(SpmvArgs a) {
         row = a.r1 + (((int64_t)blockIdx.x - a.nb0) * kBlock + threadIdx.x) * 2;
         lim = a.r1 + a.len1;
     }
-    double d = 0.0;
+    double d = 0.0, dg = 0.0;  // kDots 1: p.Ap; kDots 2: delta (d) and gamma (dg)
     int done = 0;
     if (row + 1 < lim) {
         const uint64_t pol = policy_evict_first();
@@ -377,7 +440,7 @@ __global__ void __launch_bounds__(kBlock, 4) spmv27x2_kernel(SpmvArgs a) {
             if (g == 0) {
                 pdl_wait();
                 if (kDot && a.trace) trace_mark(a.trace, a.trace_max, __ldg(&a.sc->k), 1, false);
-                if (kDot && kCheck) done = __ldg(&a.sc->done);
+                done = spmv_done<kDots, kCheck>(a);
                 if (done) return;  // uniform over the grid, before any store
             }
 #pragma unroll
@@ -394,15 +457,16 @@ __global__ void __launch_bounds__(kBlock, 4) spmv27x2_kernel(SpmvArgs a) {
             }
         }
         *reinterpret_cast<double2 *>(a.y + row) = make_double2(s0, s1);
-        if (kDot) {
+        if (kDots > 0) {
             const double p0 = c0 == row + a.plane ? x0 : __ldg(a.x + row + a.plane);
             const double p1 = c1 == row + 1 + a.plane ? x1 : __ldg(a.x + row + 1 + a.plane);
             d = fma(s1, p1, s0 * p0);
+            if (kDots == 2) dg = fma(p1, p1, p0 * p0);
         }
     } else if (row < lim) {  // odd tail: one row, scalar loads
         const uint64_t pol = policy_evict_first();
         pdl_wait();
-        if (kDot && kCheck) done = __ldg(&a.sc->done);
+        done = spmv_done<kDots, kCheck>(a);
         if (done) return;
         double s0 = 0.0;
 #pragma unroll
@@ -410,13 +474,21 @@ __global__ void __launch_bounds__(kBlock, 4) spmv27x2_kernel(SpmvArgs a) {
             s0 = fma(ld_stream(a.val + k * a.stride + row, pol),
                      __ldg(a.x + ld_stream(a.col + k * a.stride + row, pol)), s0);
         a.y[row] = s0;
-        if (kDot) d = s0 * __ldg(a.x + row + a.plane);
+        if (kDots > 0) {
+            const double xi = __ldg(a.x + row + a.plane);
+            d = s0 * xi;
+            if (kDots == 2) dg = xi * xi;
+        }
     } else {
         pdl_wait();
-        if (kDot && kCheck) done = __ldg(&a.sc->done);
+        done = spmv_done<kDots, kCheck>(a);
     }
     pdl_trigger();
     if (done) return;
+    if (kDots == 2) {
+        spmv_sr_partials(a, dg, d);
+        return;
+    }
     if (kDot && a.trace) trace_mark(a.trace, a.trace_max, __ldg(&a.sc->k), 1, true);
     if (kDot) {
         if (a.parts_only) {  // block partial only; the update kernel sums them
@@ -691,6 +763,189 @@ __global__ void cg_initstate_kernel(CgScalars *sc, int max_iter, double tol,
     const int done = !(1 < max_iter && normr > tol);
     sc->done = done;
     set_cond(cond, !done);
+}
+
+// ------------------------------- f2: single-reduction (Chronopoulos-Gear) CG
+// Same HPCCG loop control (A4 lag, A11 guard) as the kernels above; the
+// iteration is two kernels: this fused update, then the SpMV w = A r with the
+// (gamma, delta) epilogue (spmv27*_kernel<2>).  The update of iteration k
+//   beta = gamma / gamma_old, den = delta - (beta gamma) / alpha_old
+//   (k = 1: beta = 0, den = delta), alpha = gamma / den
+//   p = r + beta p; s = w + beta s; x = x + alpha p; r = r - alpha s
+// makes ONE pass over r, w, p, s, x (reads 5, writes 4: 72n B, the same bytes
+// as HPCCG's p update + x/r update) and needs no grid-wide reduction of its
+// own: every block sums the previous SpMV's (gamma, delta) partials in the
+// same fixed order, so every block holds bit-identical scalars, and block 0
+// writes the double-buffered loop state (CgScalars::sr_*).  The scalar
+// arithmetic uses explicit round-to-nearest intrinsics in the oracle's
+// order (no contraction), so it matches oracle_cg_sr step for step.
+// Multi-slab: a finisher sums the partials into loc_gd, one allreduce of
+// the two values gives gd (one collective per iteration instead of two).
+
+struct SrUpdArgs {
+    int64_t n;
+    double *x, *r, *p, *s;     // r: owned part of the gathered (halo) vector
+    const double *w;
+    const double *parts;       // non-null: (gamma, delta) = fixed-order sums of
+    unsigned n_parts;          //   parts[0, n_parts) and parts[n_parts, 2 n_parts)
+    CgScalars *sc;
+    int q;                     // parity of the iteration this launch runs
+    unsigned long long cond;   // while-graph condition handle (0: none)
+};
+
+// Fixed-order sums of the (gamma, delta) partials, identical in every block.
+__device__ __forceinline__ double2 sr_sum_parts(const double *parts, unsigned np, double *sh) {
+    double g = 0.0, d = 0.0;
+    for (unsigned i = threadIdx.x; i < np; i += kBlock) {
+        g += __ldg(parts + i);
+        d += __ldg(parts + np + i);
+    }
+    double2 t = block_reduce2(g, d, sh);
+    if (threadIdx.x == 0) {
+        sh[64] = t.x;
+        sh[65] = t.y;
+    }
+    __syncthreads();
+    t = make_double2(sh[64], sh[65]);
+    return t;
+}
+
+// (gamma, delta) partials of one slab -> out[0..1] (one block, fixed order):
+// multi-slab (allreduce input) or a single slab with > kUpdSumMax partials.
+__global__ void __launch_bounds__(kBlock) cg_sr_finish_kernel(const double *parts, unsigned n_parts,
+                                                              double *out) {
+    pdl_wait();
+    pdl_trigger();
+    __shared__ double sh[66];
+    const double2 t = sr_sum_parts(parts, n_parts, sh);
+    if (threadIdx.x == 0) {
+        out[0] = t.x;
+        out[1] = t.y;
+    }
+}
+
+template <bool kVec, int kU>
+__global__ void __launch_bounds__(kBlock) cg_sr_update_kernel(SrUpdArgs a) {
+    CgScalars *sc = a.sc;
+    const int q = a.q, qp = q ^ 1;
+    pdl_wait();
+    pdl_trigger();
+    if (!__ldg(&sc->sr_run[qp])) {  // iteration k does not run (uniform) ...
+        // ... and neither does k + 1: propagate, or slot q would keep the stale
+        // flag of iteration k - 1 for the launches of parity q that follow
+        if (blockIdx.x == 0 && threadIdx.x == 0) sc->sr_run[q] = 0;
+        return;
+    }
+    __shared__ double sh[66];
+    double2 gd;
+    if (a.parts) gd = sr_sum_parts(a.parts, a.n_parts, sh);
+    else gd = make_double2(__ldg(&sc->gd[0]), __ldg(&sc->gd[1]));
+    const double gamma = gd.x, delta = gd.y;
+    const int k = __ldg(&sc->sr_k[qp]);
+    const bool first = (k == 1);
+    const double beta = first ? 0.0 : __ddiv_rn(gamma, __ldg(&sc->sr_gamma[qp]));
+    const double den =
+        first ? delta : __dsub_rn(delta, __ddiv_rn(__dmul_rn(beta, gamma), __ldg(&sc->sr_alpha[qp])));
+    const bool stop = (gamma == 0.0) || (den == 0.0);  // A11
+    const double alpha = stop ? 0.0 : __ddiv_rn(gamma, den);
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+        const double normr = sqrt(gamma);  // ||r_(k-1)||: the lagged check (A4)
+        const int nrun = !stop && (k + 1 < __ldg(&sc->max_iter)) && normr > __ldg(&sc->tol);
+        sc->sr_gamma[q] = gamma;
+        sc->sr_alpha[q] = alpha;
+        sc->sr_k[q] = k + 1;
+        sc->sr_run[q] = nrun;
+        sc->normr = normr;
+        sc->niters = k;
+        sc->done = !nrun;
+        set_cond(a.cond, nrun);
+    }
+    const int64_t tid = gtid(), nth = gnth();
+    if (kVec) {
+        const int64_t nv = a.n >> 1;
+        double2 *__restrict__ x2 = reinterpret_cast<double2 *>(a.x);
+        double2 *__restrict__ r2 = reinterpret_cast<double2 *>(a.r);
+        double2 *__restrict__ p2 = reinterpret_cast<double2 *>(a.p);
+        double2 *__restrict__ s2 = reinterpret_cast<double2 *>(a.s);
+        const double2 *__restrict__ w2 = reinterpret_cast<const double2 *>(a.w);
+        for (int64_t b = tid; b < nv; b += kU * nth) {
+            double2 ra[kU], wa[kU], pa[kU], sa[kU], xa[kU];
+#pragma unroll
+            for (int u = 0; u < kU; ++u) {
+                const int64_t i = b + u * nth;
+                if (i < nv) {
+                    ra[u] = r2[i];
+                    wa[u] = w2[i];
+                    if (!first) {
+                        pa[u] = p2[i];
+                        sa[u] = s2[i];
+                    }
+                    xa[u] = x2[i];
+                }
+            }
+#pragma unroll
+            for (int u = 0; u < kU; ++u) {
+                const int64_t i = b + u * nth;
+                if (i < nv) {
+                    double2 pv = ra[u], sv = wa[u];
+                    if (!first) {
+                        pv.x = fma(beta, pa[u].x, ra[u].x);
+                        pv.y = fma(beta, pa[u].y, ra[u].y);
+                        sv.x = fma(beta, sa[u].x, wa[u].x);
+                        sv.y = fma(beta, sa[u].y, wa[u].y);
+                    }
+                    p2[i] = pv;
+                    s2[i] = sv;
+                    x2[i] = make_double2(fma(alpha, pv.x, xa[u].x), fma(alpha, pv.y, xa[u].y));
+                    r2[i] = make_double2(fma(-alpha, sv.x, ra[u].x), fma(-alpha, sv.y, ra[u].y));
+                }
+            }
+        }
+        if (tid == 0 && (a.n & 1)) {
+            const int64_t i = a.n - 1;
+            const double pv = first ? a.r[i] : fma(beta, a.p[i], a.r[i]);
+            const double sv = first ? a.w[i] : fma(beta, a.s[i], a.w[i]);
+            a.p[i] = pv;
+            a.s[i] = sv;
+            a.x[i] = fma(alpha, pv, a.x[i]);
+            a.r[i] = fma(-alpha, sv, a.r[i]);
+        }
+    } else {
+        for (int64_t i = tid; i < a.n; i += nth) {
+            const double pv = first ? a.r[i] : fma(beta, a.p[i], a.r[i]);
+            const double sv = first ? a.w[i] : fma(beta, a.s[i], a.w[i]);
+            a.p[i] = pv;
+            a.s[i] = sv;
+            a.x[i] = fma(alpha, pv, a.x[i]);
+            a.r[i] = fma(-alpha, sv, a.r[i]);
+        }
+    }
+}
+
+// f2 init, after w = A r0 and its (gamma, delta) partials (or gd): the loop
+// state slot 0 (read by iteration k = 1, parity 1), normr = ||r0||, first
+// check (A4).  One block.
+__global__ void __launch_bounds__(kBlock) cg_sr_initstate_kernel(const double *parts, unsigned n_parts,
+                                                                 CgScalars *sc, int max_iter,
+                                                                 double tol, unsigned long long cond) {
+    __shared__ double sh[66];
+    double gamma;
+    if (parts) gamma = sr_sum_parts(parts, n_parts, sh).x;
+    else gamma = sc->gd[0];
+    if (threadIdx.x != 0) return;
+    const double normr = sqrt(gamma);
+    const int run = (1 < max_iter) && normr > tol;
+    sc->tol = tol;
+    sc->max_iter = max_iter;
+    sc->sr_k[0] = 1;
+    sc->sr_gamma[0] = gamma;
+    sc->sr_alpha[0] = 0.0;
+    sc->sr_run[0] = run;
+    sc->sr_run[1] = 0;
+    sc->normr = normr;
+    sc->niters = 0;
+    sc->done = !run;
+    set_cond(cond, run);
 }
 
 // ------------------------------------------- persistent single-kernel solve
@@ -983,11 +1238,13 @@ __global__ void __launch_bounds__(kBlock, 1) cg_smem_cluster_kernel(SmemArgs a) 
 // Loopback allreduce: fixed rank-order sum (or max) of one scalar of every
 // slab, written back to every slab (deterministic, identical on all slabs).
 __global__ void slab_allreduce_kernel(const double *const *src, double *const *dst,
-                                      int nslabs, int is_max) {
+                                      int nslabs, int is_max, int count) {
     if (threadIdx.x != 0 || blockIdx.x != 0) return;
-    double s = *src[0];
-    for (int r = 1; r < nslabs; ++r) s = is_max ? fmax(s, *src[r]) : s + *src[r];
-    for (int r = 0; r < nslabs; ++r) *dst[r] = s;
+    for (int c = 0; c < count; ++c) {
+        double s = src[0][c];
+        for (int r = 1; r < nslabs; ++r) s = is_max ? fmax(s, src[r][c]) : s + src[r][c];
+        for (int r = 0; r < nslabs; ++r) dst[r][c] = s;
+    }
 }
 
 // ---------------------------------------------------------- a.10 BLAS-1
