@@ -100,6 +100,12 @@ extern "C" {
                                epilogue) and ONE allreduce of two values; needs 8n more bytes
                                (s), small problems use the graph path instead of the
                                persistent kernel.  Rounding differs: niters +-1 */
+#define HPCCG_OPT_FINISHER_FREE 17 /* 1 (default): single GPU, HPCCG variant: no grid-wide
+                               finisher in any CG kernel -- the x/r update writes per-block
+                               r.r partials that every block of the next p update sums in
+                               the finisher's fixed order (identical bits), and takes the
+                               loop decision itself; 0: the update's last block finishes
+                               r.r and the loop control */
 #define HPCCG_OPT_WHILE_UNROLL 15 /* CG iterations per execution of the WHILE body
                                (default 4: amortises the conditional node's ~8 us) */
 #define HPCCG_OPT_CLUSTER_ROWS 12 /* up to this many rows (default 16384) the persistent solve

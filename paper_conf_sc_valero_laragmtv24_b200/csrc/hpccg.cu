@@ -147,6 +147,7 @@ struct hpccg_problem {
     int opt_smem = 1;                  // persistent solve resident in cluster shared memory if it fits
     int opt_while_unroll = 4;          // CG iterations per WHILE-body execution
     int opt_variant = 0;               // 0 HPCCG CG, 1 single-reduction CG (f2)
+    int opt_ff = 1;                    // single slab: finisher-free HPCCG loop (consumer-side sums)
     int last_persist_mode = 3;
     // graph of one CG iteration (per-iteration replay) ...
     cudaGraphExec_t graph = nullptr;
@@ -569,6 +570,11 @@ int cg_spmv_all(hpccg_problem *p, bool timing, bool check) {
 
 double **tab(hpccg_problem *p, int which) { return p->d_tab + (size_t)which * p->ctx->nslabs; }
 
+// SpMV partial count of a single slab's CG SpMV (the update sums them).
+unsigned single_spmv_parts(const hpccg_problem *p, const Slab &s) {
+    return (unsigned)spmv_blocks(s.n, spmv_rows_per_thread(p->opt_rows, spmv_args(s, s.p, s.Ap), 0, 0));
+}
+
 int allreduce_cg(hpccg_problem *p, bool rr, bool timing) {
     hpccg_ctx *ctx = p->ctx;
     if (ctx->mode == MODE_SINGLE) return HPCCG_OK;
@@ -579,9 +585,92 @@ int allreduce_cg(hpccg_problem *p, bool rr, bool timing) {
     return allreduce_scalar(ctx, hs, hd, tab(p, rr ? 2 : 0), tab(p, rr ? 3 : 1), false);
 }
 
+// Single slab, HPCCG variant: the finisher-free loop (kernels.cuh
+// cg_pupdate1 / cg_update1) when its vectors are 16-B aligned (always, for
+// generated problems).
+bool ff_path(const hpccg_problem *p) {
+    if (p->ctx->mode != MODE_SINGLE || !p->opt_ff || p->opt_variant != 0) return false;
+    const Slab &s = p->slabs[0];
+    return aligned16(s.r) && aligned16(s.p + s.plane) && aligned16(s.x) && aligned16(s.Ap);
+}
+
+template <int kU>
+int enqueue_iteration_ff_u(hpccg_problem *p, bool timing, bool check, unsigned long long cond, int q) {
+    hpccg_ctx *ctx = p->ctx;
+    const Slab &s = p->slabs[0];
+    const bool pdl = p->opt_pdl != 0;
+    auto upd = cg_update1_kernel<kU>;
+    auto pup = cg_pupdate1_kernel<kU>;
+    // the update's grid fixes the r.r partials and so the bits: size it as
+    // the finisher path's update kernel is sized, so both paths agree bitwise
+    const int ug = vec_grid(ctx, cg_update_kernel<true, false, kU>, cdiv(s.n, 2 * kU),
+                            p->opt_vec_waves, p->red_cap);
+    TraceSlot *tr = s.trace_on ? s.trace : nullptr;
+    {
+        PhaseTimer t(p, ctx->stream, PH_PUPDATE, timing);
+        Pupd1Args a{};
+        a.n = s.n;
+        a.r = s.r;
+        a.p = s.p + s.plane;
+        a.rr_parts = s.red.partials;
+        a.n_rr = (unsigned)ug;
+        a.sc = s.sc;
+        a.q = q;
+        a.trace = tr;
+        a.trace_max = s.trace_max;
+        const int g = vec_grid(ctx, pup, cdiv(s.n, 2 * kU), p->opt_vec_waves, 0x7fffffff);
+        launch_k(pdl, pup, dim3(g), ctx->stream, a);
+        CHECK(check_launch(ctx));
+    }
+    CHECK(cg_spmv_all(p, timing, check));
+    PhaseTimer t(p, ctx->stream, PH_UPDATE, timing);
+    Upd1Args a{};
+    a.n = s.n;
+    a.x = s.x;
+    a.r = s.r;
+    a.p = s.p + s.plane;
+    a.Ap = s.Ap;
+    a.rr_parts = s.red.partials;
+    a.sc = s.sc;
+    a.q = q;
+    a.cond = cond;
+    a.trace = tr;
+    a.trace_max = s.trace_max;
+    const unsigned np = single_spmv_parts(p, s);
+    if (np <= kUpdSumMax) {
+        a.pAp_parts = s.spmv_parts;
+        a.n_parts = np;
+    } else {  // one finisher block writes sc->pAp
+        void (*fk)(const double *, unsigned, CgScalars *) = cg_pap_finish_kernel;
+        cudaLaunchConfig_t cfg{};
+        cfg.gridDim = dim3(1);
+        cfg.blockDim = dim3(1024);
+        cfg.stream = ctx->stream;
+        cudaLaunchAttribute at[1];
+        at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+        at[0].val.programmaticStreamSerializationAllowed = 1;
+        cfg.attrs = pdl ? at : nullptr;
+        cfg.numAttrs = pdl ? 1 : 0;
+        CU(cudaLaunchKernelEx(&cfg, fk, (const double *)s.spmv_parts, np, s.sc));
+        CHECK(check_launch(ctx));
+    }
+    launch_k(pdl, upd, dim3(ug), ctx->stream, a);
+    return check_launch(ctx);
+}
+
+int enqueue_iteration_ff(hpccg_problem *p, bool timing, bool check, unsigned long long cond, int q) {
+    switch (p->opt_unroll) {
+        case 1: return enqueue_iteration_ff_u<1>(p, timing, check, cond, q);
+        case 2: return enqueue_iteration_ff_u<2>(p, timing, check, cond, q);
+        default: return enqueue_iteration_ff_u<4>(p, timing, check, cond, q);
+    }
+}
+
 // One CG iteration (a.6, a.2, a.3+a.4, a.5, a.8) for every slab.  `cond`:
-// while-graph condition handle (0 outside the while-graph).
-int enqueue_iteration(hpccg_problem *p, bool timing, bool check, unsigned long long cond) {
+// while-graph condition handle (0 outside the while-graph); k: the
+// iteration's index (its parity drives the finisher-free loop's state).
+int enqueue_iteration(hpccg_problem *p, bool timing, bool check, unsigned long long cond, int k) {
+    if (ff_path(p)) return enqueue_iteration_ff(p, timing, check, cond, k & 1);
     hpccg_ctx *ctx = p->ctx;
     const int single = ctx->mode == MODE_SINGLE;
     // PDL only between back-to-back kernels (single slab; the multi-slab
@@ -656,11 +745,6 @@ int enqueue_init(hpccg_problem *p, int max_iter, double tol, bool timing,
 // Buffers (same arena as HPCCG's CG): the GATHERED vector is r here, so r
 // lives in the halo buffer s.p; w = A r in s.Ap; p (not gathered) in s.r;
 // the s = A p recurrence in s.sv; x in s.x.
-
-// SpMV partial count of a single slab's CG SpMV (the update sums them).
-unsigned single_spmv_parts(const hpccg_problem *p, const Slab &s) {
-    return (unsigned)spmv_blocks(s.n, spmv_rows_per_thread(p->opt_rows, spmv_args(s, s.p, s.Ap), 0, 0));
-}
 
 // w = A r with the (gamma, delta) epilogue for every slab; multi-slab: halo
 // exchange overlapped with the interior rows (NCCL), per-slab finisher, and
@@ -858,13 +942,13 @@ int enqueue_init_sr(hpccg_problem *p, int max_iter, double tol, bool timing,
 // Iterations captured per WHILE-body / per-iteration graph: f2 needs an even
 // count (each launch's iteration parity is baked into the captured node).
 int body_iterations(const hpccg_problem *p, int u) {
-    if (p->opt_variant == 0) return u;
+    if (p->opt_variant == 0 && !ff_path(p)) return u;
     return std::max(2, (u + 1) & ~1);
 }
 
 int enqueue_iteration_any(hpccg_problem *p, bool timing, bool check, unsigned long long cond, int k) {
     if (p->opt_variant == 1) return enqueue_iteration_sr(p, timing, check, cond, k & 1);
-    return enqueue_iteration(p, timing, check, cond);
+    return enqueue_iteration(p, timing, check, cond, k);
 }
 
 int enqueue_init_any(hpccg_problem *p, int max_iter, double tol, bool timing, unsigned long long cond) {
@@ -1621,6 +1705,7 @@ int hpccg_set_option(hpccg_problem *p, int key, int64_t value) {
             p->opt_persist = (int)value;
             return HPCCG_OK;
         case HPCCG_OPT_SMEM_SOLVE: p->opt_smem = value != 0; return HPCCG_OK;
+        case HPCCG_OPT_FINISHER_FREE: p->opt_ff = value != 0; return HPCCG_OK;
         case HPCCG_OPT_CG_VARIANT:
             if (value != 0 && value != 1) return fail(HPCCG_EINVAL, "cg variant: 0 or 1");
             p->opt_variant = (int)value;

@@ -53,7 +53,8 @@ struct CgScalars {
     double gd[2];         // global (gamma, delta) when not summed from partials
     double loc_gd[2];     // this slab's (gamma, delta) partial (allreduce input)
     int sr_k[2];          // index of the next iteration
-    int sr_run[2];        // sr_run[q]: iteration k + 1 runs (written by iteration k)
+    int run_q[2];         // run_q[q]: iteration k + 1 runs (written by iteration k);
+                          // also used by HPCCG's finisher-free single-slab loop
 };
 
 // Scratch for the deterministic single-pass grid reduction.
@@ -266,13 +267,13 @@ struct SpmvArgs {
     double *parts_only;
     TraceSlot *trace;  // HPCCG_OPT_TRACE (nullptr: off)
     int trace_max;
-    int sr_q;          // kDots 2: parity of the iteration (run flag sr_run[sr_q])
+    int sr_q;          // kDots 2: parity of the iteration (run flag run_q[sr_q])
 };
 
 template <int kDots, bool kCheck>
 __device__ __forceinline__ int spmv_done(const SpmvArgs &a) {
     if (!kCheck || kDots == 0) return 0;
-    if (kDots == 2) return !__ldg(&a.sc->sr_run[a.sr_q]);
+    if (kDots == 2) return !__ldg(&a.sc->run_q[a.sr_q]);
     return __ldg(&a.sc->done);
 }
 
@@ -310,7 +311,7 @@ __device__ __forceinline__ void spmv_sr_partials(const SpmvArgs &a, double g, do
 // both from the diagonal slot's gathered value (no extra bytes), written as
 // per-block partials parts_only[b] and parts_only[total_blocks + b].
 // kCheck: return at once when the device `done` flag is set (kDots 2: when
-// the run flag sr_run[sr_q] says the next iteration does not run) -- plain /
+// the run flag run_q[sr_q] says the next iteration does not run) -- plain /
 // per-iteration-graph launches; the while-graph never launches past
 // convergence so it skips that load, whose latency would otherwise sit in
 // front of every block's first matrix load).
@@ -724,6 +725,206 @@ __global__ void __launch_bounds__(kBlock) cg_update_kernel(UpdArgs a) {
                        });
 }
 
+// ------------------- single slab: HPCCG's loop without any grid finisher
+// The last-block finisher of cg_update_kernel (fence + atomic ticket + the
+// final sum, then the loop control) sits between every update and the next
+// p update (~5 us of the 128^3 iteration, DESIGN.md 7.1 trace).  On a single
+// slab the reduction can be finished by the CONSUMER instead, as the SpMV's
+// p.Ap already is: the update writes its per-block r.r partials, and every
+// block of the next p update sums them in the same fixed order as the
+// finisher did (identical bits).  The loop decision for iteration k + 1
+// (A4: normr = ||r_(k-1)|| lagged, A11: p.Ap) is known inside update k, so
+// block 0 of update k takes it.  Device loop state per kernel:
+//   p update k  (block 0) writes rr_cur = rtrans_k, normr, niters = k
+//   update k    (block 0) writes rr_prev = rtrans_k, pAp, k = k + 1, done,
+//               run_q[q] = "iteration k + 1 runs", the while-graph condition
+// and every kernel of iteration k reads only what earlier kernels wrote; the
+// run flag is double-buffered by iteration parity q = k & 1 (a launch's
+// parity is baked into the graph node), so no block reads a word another
+// block of its own grid writes.
+
+struct Pupd1Args {
+    int64_t n;
+    const double *r;
+    double *p;
+    const double *rr_parts;  // r.r partials of the previous update
+    unsigned n_rr;
+    const CgScalars *sc_in;
+    CgScalars *sc;
+    int q;
+    TraceSlot *trace;
+    int trace_max;
+};
+
+// Fixed-order sum of n partials (the order of grid_reduce's last block);
+// identical in every block.
+__device__ __forceinline__ double sum_parts_fixed(const double *parts, unsigned n, double *sh) {
+    double s = 0.0;
+    for (unsigned i = threadIdx.x; i < n; i += kBlock) s += __ldg(parts + i);
+    s = block_reduce<false>(s, sh);
+    if (threadIdx.x == 0) sh[32] = s;
+    __syncthreads();
+    return sh[32];
+}
+
+// iteration k does not run: propagate to parity q (block 0), uniform exit
+__device__ __forceinline__ bool run_check(CgScalars *sc, int q) {
+    if (__ldg(&sc->run_q[q ^ 1])) return true;
+    if (blockIdx.x == 0 && threadIdx.x == 0) sc->run_q[q] = 0;
+    return false;
+}
+
+// a.6 p = r + beta p for a single slab (HPCCG's k > 1 branch: rtrans = r.r,
+// beta = rtrans / oldrtrans; k == 1: p = r).  The first trip's loads are
+// issued before the scalar work so their latency overlaps the partial sums.
+template <int kU>
+__global__ void __launch_bounds__(kBlock) cg_pupdate1_kernel(Pupd1Args a) {
+    __shared__ double sh[33];
+    CgScalars *sc = a.sc;
+    pdl_wait();
+    pdl_trigger();
+    const int64_t tid = gtid(), nth = gnth(), nv = a.n >> 1;
+    const double2 *__restrict__ r2 = reinterpret_cast<const double2 *>(a.r);
+    double2 *__restrict__ p2 = reinterpret_cast<double2 *>(a.p);
+    double2 ra[kU], pa[kU];
+    auto load = [&](int64_t b) {
+#pragma unroll
+        for (int u = 0; u < kU; ++u) {
+            const int64_t i = b + u * nth;
+            if (i < nv) {
+                ra[u] = r2[i];
+                pa[u] = p2[i];
+            }
+        }
+    };
+    load(tid);
+    if (!run_check(sc, a.q)) return;
+    const int k = __ldg(&sc->k);
+    trace_mark(a.trace, a.trace_max, k, 0, false);
+    const bool first = (k == 1);
+    const double rtrans = first ? __ldg(&sc->rr_cur) : sum_parts_fixed(a.rr_parts, a.n_rr, sh);
+    const double beta = first ? 0.0 : rtrans / __ldg(&sc->rr_prev);
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+        if (!first) sc->rr_cur = rtrans;
+        sc->normr = sqrt(rtrans);
+        sc->niters = k;
+    }
+    for (int64_t b = tid; b < nv;) {
+#pragma unroll
+        for (int u = 0; u < kU; ++u) {
+            const int64_t i = b + u * nth;
+            if (i < nv) {
+                double2 v = ra[u];
+                if (!first) {
+                    v.x = fma(beta, pa[u].x, ra[u].x);
+                    v.y = fma(beta, pa[u].y, ra[u].y);
+                }
+                p2[i] = v;
+            }
+        }
+        b += kU * nth;
+        if (b < nv) load(b);
+    }
+    if (tid == 0 && (a.n & 1)) {
+        const int64_t i = a.n - 1;
+        a.p[i] = first ? a.r[i] : fma(beta, a.p[i], a.r[i]);
+    }
+    if (a.trace) {
+        __syncthreads();
+        trace_mark(a.trace, a.trace_max, k, 0, true);
+    }
+}
+
+// a.5 x += alpha p, r -= alpha Ap, per-block r.r partial (no finisher), and
+// the loop decision for iteration k + 1 (block 0).
+struct Upd1Args {
+    int64_t n;
+    double *x, *r;
+    const double *p, *Ap;
+    const double *pAp_parts;  // the SpMV's p.Ap partials (nullptr: sc->pAp)
+    unsigned n_parts;
+    double *rr_parts;         // out: gridDim.x r.r partials
+    CgScalars *sc;
+    int q;
+    unsigned long long cond;
+    TraceSlot *trace;
+    int trace_max;
+};
+
+template <int kU>
+__global__ void __launch_bounds__(kBlock) cg_update1_kernel(Upd1Args a) {
+    __shared__ double sh[33];
+    CgScalars *sc = a.sc;
+    pdl_wait();
+    pdl_trigger();
+    const int64_t tid = gtid(), nth = gnth(), nv = a.n >> 1;
+    double2 *__restrict__ x2 = reinterpret_cast<double2 *>(a.x);
+    double2 *__restrict__ r2 = reinterpret_cast<double2 *>(a.r);
+    const double2 *__restrict__ p2 = reinterpret_cast<const double2 *>(a.p);
+    const double2 *__restrict__ q2 = reinterpret_cast<const double2 *>(a.Ap);
+    double2 xa[kU], ra[kU], pa[kU], qa[kU];
+    auto load = [&](int64_t b) {
+#pragma unroll
+        for (int u = 0; u < kU; ++u) {
+            const int64_t i = b + u * nth;
+            if (i < nv) {
+                xa[u] = x2[i];
+                ra[u] = r2[i];
+                pa[u] = p2[i];
+                qa[u] = q2[i];
+            }
+        }
+    };
+    load(tid);
+    if (!run_check(sc, a.q)) return;
+    const int ktr = a.trace ? __ldg(&sc->niters) : 0;
+    trace_mark(a.trace, a.trace_max, ktr, 2, false);
+    const double rtrans = __ldg(&sc->rr_cur);
+    const double pAp = a.pAp_parts ? sum_parts_fixed(a.pAp_parts, a.n_parts, sh) : __ldg(&sc->pAp);
+    const bool stop = (rtrans == 0.0) || (pAp == 0.0);  // A11
+    const double alpha = stop ? 0.0 : rtrans / pAp;
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+        const int k = __ldg(&sc->k);
+        const int run = !stop && (k + 1) < __ldg(&sc->max_iter) && __ldg(&sc->normr) > __ldg(&sc->tol);
+        sc->pAp = pAp;
+        sc->rr_prev = rtrans;
+        sc->k = k + 1;
+        sc->run_q[a.q] = run;
+        sc->done = !run;
+        set_cond(a.cond, run);
+    }
+    double acc = 0.0, acc2 = 0.0;
+    for (int64_t b = tid; b < nv;) {
+#pragma unroll
+        for (int u = 0; u < kU; ++u) {
+            const int64_t i = b + u * nth;
+            if (i < nv) {
+                xa[u].x = fma(alpha, pa[u].x, xa[u].x);
+                xa[u].y = fma(alpha, pa[u].y, xa[u].y);
+                ra[u].x = fma(-alpha, qa[u].x, ra[u].x);
+                ra[u].y = fma(-alpha, qa[u].y, ra[u].y);
+                x2[i] = xa[u];
+                r2[i] = ra[u];
+                acc = fma(ra[u].x, ra[u].x, acc);
+                acc2 = fma(ra[u].y, ra[u].y, acc2);
+            }
+        }
+        b += kU * nth;
+        if (b < nv) load(b);
+    }
+    if (tid == 0 && (a.n & 1)) {
+        const int64_t i = a.n - 1;
+        a.x[i] = fma(alpha, a.p[i], a.x[i]);
+        const double rv = fma(-alpha, a.Ap[i], a.r[i]);
+        a.r[i] = rv;
+        acc = fma(rv, rv, acc);
+    }
+    acc += acc2;
+    trace_mark(a.trace, a.trace_max, ktr, 2, true);
+    acc = block_reduce<false>(acc, sh);
+    if (threadIdx.x == 0) a.rr_parts[blockIdx.x] = acc;
+}
+
 // a.7 init: r = b - Ap (waxpby(1, b, -1, Ap) = fma(-1, Ap, b)) and r.r.
 struct InitResArgs {
     int64_t n;
@@ -762,6 +963,8 @@ __global__ void cg_initstate_kernel(CgScalars *sc, int max_iter, double tol,
     sc->niters = 0;
     const int done = !(1 < max_iter && normr > tol);
     sc->done = done;
+    sc->run_q[0] = !done;  // finisher-free loop: iteration 1 (parity 1) runs
+    sc->run_q[1] = 0;
     set_cond(cond, !done);
 }
 
@@ -830,10 +1033,10 @@ __global__ void __launch_bounds__(kBlock) cg_sr_update_kernel(SrUpdArgs a) {
     const int q = a.q, qp = q ^ 1;
     pdl_wait();
     pdl_trigger();
-    if (!__ldg(&sc->sr_run[qp])) {  // iteration k does not run (uniform) ...
+    if (!__ldg(&sc->run_q[qp])) {  // iteration k does not run (uniform) ...
         // ... and neither does k + 1: propagate, or slot q would keep the stale
         // flag of iteration k - 1 for the launches of parity q that follow
-        if (blockIdx.x == 0 && threadIdx.x == 0) sc->sr_run[q] = 0;
+        if (blockIdx.x == 0 && threadIdx.x == 0) sc->run_q[q] = 0;
         return;
     }
     __shared__ double sh[66];
@@ -854,7 +1057,7 @@ __global__ void __launch_bounds__(kBlock) cg_sr_update_kernel(SrUpdArgs a) {
         sc->sr_gamma[q] = gamma;
         sc->sr_alpha[q] = alpha;
         sc->sr_k[q] = k + 1;
-        sc->sr_run[q] = nrun;
+        sc->run_q[q] = nrun;
         sc->normr = normr;
         sc->niters = k;
         sc->done = !nrun;
@@ -940,8 +1143,8 @@ __global__ void __launch_bounds__(kBlock) cg_sr_initstate_kernel(const double *p
     sc->sr_k[0] = 1;
     sc->sr_gamma[0] = gamma;
     sc->sr_alpha[0] = 0.0;
-    sc->sr_run[0] = run;
-    sc->sr_run[1] = 0;
+    sc->run_q[0] = run;
+    sc->run_q[1] = 0;
     sc->normr = normr;
     sc->niters = 0;
     sc->done = !run;

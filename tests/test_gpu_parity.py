@@ -591,3 +591,32 @@ def test_lbm_paper_size_conservation(ctx):
             oracle.lbm_step(S, a, f, b, 0.8)
             a, b = b, a
         np.testing.assert_array_equal(l.get(0), a)
+
+
+# ------------------------- single slab: finisher-free vs last-block finisher
+
+@pytest.mark.parametrize("unroll", [4, 2, 1])
+@pytest.mark.parametrize("dims,max_iter,tol", [((24, 20, 12), 150, 1e-12), ((33, 9, 3), 150, 1e-12),
+                                               ((64, 64, 32), 41, 0.0), ((8, 8, 8), 2, 0.0),
+                                               ((8, 8, 8), 6, 0.0), ((2, 2, 2), 60, 0.0)])
+def test_cg_finisher_free_loop_bitwise_vs_finisher(ctx, unroll, dims, max_iter, tol):
+    """HPCCG_OPT_FINISHER_FREE: the next p update sums the update's r.r
+    partials in the finisher's order and the update takes the loop decision;
+    niters, normr and x are bit-identical to the last-block-finisher loop in
+    the while-graph (even and odd iteration counts, A11 guard) and in the
+    per-iteration graph."""
+    outs = []
+    with H.Problem(ctx, *dims) as p:
+        p.set_option(H.HPCCG_OPT_PERSISTENT, 0)
+        p.set_option(H.HPCCG_OPT_VEC_UNROLL, unroll)
+        for ff, wh in [(0, 1), (1, 1), (1, 0), (0, 0)]:
+            p.set_option(H.HPCCG_OPT_FINISHER_FREE, ff)
+            p.set_option(H.HPCCG_OPT_WHILE, wh)
+            p.set_vec(H.HPCCG_VEC_X, np.zeros(p.n))
+            r = p.solve(max_iter, tol)
+            outs.append((r["niters"], r["normr"], p.get_vec(H.HPCCG_VEC_X)))
+    for o in outs[1:]:
+        assert o[:2] == outs[0][:2]
+        np.testing.assert_array_equal(o[2], outs[0][2])
+    if tol == 0.0 and dims != (2, 2, 2):
+        assert outs[0][0] == max_iter - 1

@@ -14,7 +14,8 @@ KEYS = {"graph": H.HPCCG_OPT_GRAPH, "timing": H.HPCCG_OPT_TIMING, "while": H.HPC
         "crows": H.HPCCG_OPT_CLUSTER_ROWS,
         "smem": H.HPCCG_OPT_SMEM_SOLVE,
         "wu": H.HPCCG_OPT_WHILE_UNROLL,
-        "var": H.HPCCG_OPT_CG_VARIANT}
+        "var": H.HPCCG_OPT_CG_VARIANT,
+        "ff": H.HPCCG_OPT_FINISHER_FREE}
 nx, ny, nz, iters = (int(v) for v in sys.argv[1:5])
 ctx = H.Context(0)
 p = H.Problem(ctx, nx, ny, nz)
@@ -45,6 +46,6 @@ for spec in sys.argv[5:]:
     print(json.dumps(out), flush=True)
     for k in opts:
         try:
-            p.set_option(KEYS[k], {"graph": 1, "while": 1, "l2": 1, "waves": 1, "rows": 2, "unroll": 4, "persist": 1, "pdl": 1, "crows": 16384, "smem": 1, "wu": 4, "var": 0}.get(k, 0))
+            p.set_option(KEYS[k], {"graph": 1, "while": 1, "l2": 1, "waves": 1, "rows": 2, "unroll": 4, "persist": 1, "pdl": 1, "crows": 16384, "smem": 1, "wu": 4, "var": 0, "ff": 1}.get(k, 0))
         except H.HpccgError:
             pass
