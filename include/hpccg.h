@@ -106,6 +106,8 @@ extern "C" {
                                the finisher's fixed order (identical bits), and takes the
                                loop decision itself; 0: the update's last block finishes
                                r.r and the loop control */
+#define HPCCG_OPT_SMEM_THREADS 18 /* threads per CTA of the shared-memory-resident solve:
+                               0 (default) auto (512 when a CTA holds > 256 rows), 256, 512 */
 #define HPCCG_OPT_WHILE_UNROLL 15 /* CG iterations per execution of the WHILE body
                                (default 4: amortises the conditional node's ~8 us) */
 #define HPCCG_OPT_CLUSTER_ROWS 12 /* up to this many rows (default 16384) the persistent solve

@@ -148,6 +148,7 @@ struct hpccg_problem {
     int opt_while_unroll = 4;          // CG iterations per WHILE-body execution
     int opt_variant = 0;               // 0 HPCCG CG, 1 single-reduction CG (f2)
     int opt_ff = 1;                    // single slab: finisher-free HPCCG loop (consumer-side sums)
+    int opt_smem_threads = 0;          // on-chip solve CTA width: 0 auto, 256, 512
     int last_persist_mode = 3;
     // graph of one CG iteration (per-iteration replay) ...
     cudaGraphExec_t graph = nullptr;
@@ -1010,6 +1011,19 @@ struct L2Window {
     ~L2Window() { release(); }
 };
 
+// Shared-memory-resident solve: bytes per row (ELL slice + vectors) and the
+// rows per CTA when the problem fits one cluster (0: it does not).
+int64_t smem_bytes_per_row(bool sr) {
+    return kSlots * (int64_t)(sizeof(double) + sizeof(int)) + (sr ? 6 : 5) * (int64_t)sizeof(double);
+}
+
+int64_t smem_rows(const hpccg_problem *p) {
+    const hpccg_ctx *ctx = p->ctx;
+    if (!p->opt_smem || ctx->smem_cluster <= 1 || ctx->mode != MODE_SINGLE) return 0;
+    const int64_t R = cdiv(p->slabs[0].n, ctx->smem_cluster);
+    return R * smem_bytes_per_row(p->opt_variant == 1) <= ctx->smem_bytes ? R : 0;
+}
+
 // The whole solve in one cooperative kernel (small single-slab problems).
 int launch_persistent(hpccg_problem *p, int max_iter, double tol) {
     hpccg_ctx *ctx = p->ctx;
@@ -1032,10 +1046,11 @@ int launch_persistent(hpccg_problem *p, int max_iter, double tol) {
     a.max_iter = max_iter;
     a.tol = tol;
     // whole problem in one cluster's shared memory when it fits
-    const int64_t bytes_per_row = kSlots * (sizeof(double) + sizeof(int)) + 5 * sizeof(double);
-    if (p->opt_smem && ctx->smem_cluster > 1) {
-        const int64_t R = cdiv(s.n, ctx->smem_cluster);
-        if (R * bytes_per_row <= ctx->smem_bytes) {
+    const bool sr = p->opt_variant == 1;
+    const int64_t bytes_per_row = smem_bytes_per_row(sr);
+    {
+        const int64_t R = smem_rows(p);
+        if (R > 0) {
             SmemArgs m{};
             m.n = s.n;
             m.stride = s.n;
@@ -1050,8 +1065,10 @@ int launch_persistent(hpccg_problem *p, int max_iter, double tol) {
             m.tol = tol;
             const int64_t g = cdiv(s.n, R);
             cudaLaunchConfig_t cfg{};
+            // auto: 512 threads when a CTA holds more than 256 rows (one trip)
+            const int nt = p->opt_smem_threads ? p->opt_smem_threads : (R > kBlock ? 512 : kBlock);
             cfg.gridDim = dim3((unsigned)g);
-            cfg.blockDim = dim3(kBlock);
+            cfg.blockDim = dim3(nt);
             cfg.dynamicSmemBytes = (size_t)(R * bytes_per_row);
             cfg.stream = ctx->stream;
             cudaLaunchAttribute at[1];
@@ -1061,7 +1078,13 @@ int launch_persistent(hpccg_problem *p, int max_iter, double tol) {
             at[0].val.clusterDim.z = 1;
             cfg.attrs = at;
             cfg.numAttrs = 1;
-            CU(cudaLaunchKernelEx(&cfg, cg_smem_cluster_kernel, m));
+            if (nt == 512) {
+                if (sr) CU(cudaLaunchKernelEx(&cfg, cg_smem_cluster_kernel<512, true>, m));
+                else CU(cudaLaunchKernelEx(&cfg, cg_smem_cluster_kernel<512, false>, m));
+            } else {
+                if (sr) CU(cudaLaunchKernelEx(&cfg, cg_smem_cluster_kernel<kBlock, true>, m));
+                else CU(cudaLaunchKernelEx(&cfg, cg_smem_cluster_kernel<kBlock, false>, m));
+            }
             p->last_persist_mode = 5;
             return check_launch(ctx);
         }
@@ -1242,14 +1265,21 @@ int ctx_common_init(hpccg_ctx *c, int device, void *stream) {
         CU(cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, device));
         c->smem_bytes = optin - 1024;  // static smem of the kernel + slack
         c->smem_cluster = 0;
-        if (cudaFuncSetAttribute(cg_smem_cluster_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                 (int)c->smem_bytes) == cudaSuccess &&
-            cudaFuncSetAttribute(cg_smem_cluster_kernel, cudaFuncAttributeNonPortableClusterSizeAllowed,
-                                 1) == cudaSuccess) {
+        bool attr_ok = true;
+        for (const void *k : {(const void *)cg_smem_cluster_kernel<kBlock, false>,
+                              (const void *)cg_smem_cluster_kernel<kBlock, true>,
+                              (const void *)cg_smem_cluster_kernel<512, false>,
+                              (const void *)cg_smem_cluster_kernel<512, true>})
+            attr_ok = attr_ok &&
+                      cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                           (int)c->smem_bytes) == cudaSuccess &&
+                      cudaFuncSetAttribute(k, cudaFuncAttributeNonPortableClusterSizeAllowed, 1) ==
+                          cudaSuccess;
+        if (attr_ok) {
             for (int sz : {16, 8}) {
                 cudaLaunchConfig_t cfg{};
                 cfg.gridDim = dim3(sz);
-                cfg.blockDim = dim3(kBlock);
+                cfg.blockDim = dim3(512);
                 cfg.dynamicSmemBytes = (size_t)c->smem_bytes;
                 cudaLaunchAttribute at[1];
                 at[0].id = cudaLaunchAttributeClusterDimension;
@@ -1259,7 +1289,8 @@ int ctx_common_init(hpccg_ctx *c, int device, void *stream) {
                 cfg.attrs = at;
                 cfg.numAttrs = 1;
                 int ncl = 0;
-                if (cudaOccupancyMaxActiveClusters(&ncl, cg_smem_cluster_kernel, &cfg) == cudaSuccess &&
+                if (cudaOccupancyMaxActiveClusters(&ncl, cg_smem_cluster_kernel<512, true>, &cfg) ==
+                        cudaSuccess &&
                     ncl > 0) {
                     c->smem_cluster = sz;
                     break;
@@ -1706,6 +1737,10 @@ int hpccg_set_option(hpccg_problem *p, int key, int64_t value) {
             return HPCCG_OK;
         case HPCCG_OPT_SMEM_SOLVE: p->opt_smem = value != 0; return HPCCG_OK;
         case HPCCG_OPT_FINISHER_FREE: p->opt_ff = value != 0; return HPCCG_OK;
+        case HPCCG_OPT_SMEM_THREADS:
+            if (value != 0 && value != 256 && value != 512) return fail(HPCCG_EINVAL, "smem threads: 0, 256, 512");
+            p->opt_smem_threads = (int)value;
+            return HPCCG_OK;
         case HPCCG_OPT_CG_VARIANT:
             if (value != 0 && value != 1) return fail(HPCCG_EINVAL, "cg variant: 0 or 1");
             p->opt_variant = (int)value;
@@ -1869,7 +1904,9 @@ int hpccg_solve(hpccg_problem *p, int max_iter, double tol, int *niters, double 
     CU(cudaSetDevice(ctx->device));
     const bool timing = p->opt_timing != 0;
     const bool use_graph = p->opt_graph && !timing;
-    const bool use_persist = !timing && ctx->mode == MODE_SINGLE && p->opt_variant == 0 &&
+    // f2 (single-reduction) has a persistent form only on chip (smem cluster)
+    const bool use_persist = !timing && ctx->mode == MODE_SINGLE &&
+                             (p->opt_variant == 0 || smem_rows(p) > 0) &&
                              (p->opt_persist == 2 ||
                               (p->opt_persist == 1 && p->slabs[0].n <= p->opt_persist_rows));
     bool use_while = !use_persist && use_graph && p->opt_while && ctx->mode != MODE_NCCL &&

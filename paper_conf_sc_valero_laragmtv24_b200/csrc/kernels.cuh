@@ -614,8 +614,16 @@ __global__ void __launch_bounds__(1024) cg_pap_finish_kernel(const double *parts
     pdl_wait();
     pdl_trigger();
     __shared__ double sh[32];
-    double q = 0.0;
-    for (unsigned i = threadIdx.x; i < n_parts; i += 1024) q += __ldcg(parts + i);
+    // 8 independent loads in flight per thread (32768 partials at 256^3:
+    // one L2 round trip per 8 instead of a dependent chain of 32)
+    double acc[8] = {0.0, 0.0, 0.0, 0.0, 0.0, 0.0, 0.0, 0.0};
+    unsigned i = threadIdx.x;
+    for (; i + 7u * 1024u < n_parts; i += 8u * 1024u) {
+#pragma unroll
+        for (int u = 0; u < 8; ++u) acc[u] += __ldcg(parts + i + u * 1024u);
+    }
+    for (; i < n_parts; i += 1024) acc[0] += __ldcg(parts + i);
+    double q = ((acc[0] + acc[1]) + (acc[2] + acc[3])) + ((acc[4] + acc[5]) + (acc[6] + acc[7]));
     q = warp_sum(q);
     if ((threadIdx.x & 31) == 0) sh[threadIdx.x >> 5] = q;
     __syncthreads();
@@ -1323,116 +1331,228 @@ struct SmemArgs {
     double tol;
 };
 
-__device__ __forceinline__ double cluster_sum(double *mine, double v, double *sh) {
-    namespace cgx = cooperative_groups;
-    auto cl = cgx::this_cluster();
-    v = block_reduce<false>(v, sh);
-    if (threadIdx.x == 0) *mine = v;
-    cl.sync();
-    // lanes 0..C-1 of warp 0 fetch the C partials in parallel (one DSMEM
-    // round trip), then a fixed butterfly: identical sums in every CTA
-    if (threadIdx.x < 32) {
-        const unsigned c = threadIdx.x;
-        double q = c < cl.num_blocks() ? *cl.map_shared_rank(mine, c) : 0.0;
-        q = warp_sum(q);
-        if (threadIdx.x == 0) sh[31] = q;
+// Block sum of two values over NT threads in a fixed order (butterfly per
+// warp, then warp 0 over the per-warp values); valid in warp 0.
+template <int NT>
+__device__ __forceinline__ double2 blk_sum2(double u, double v, double *sh /*[64]*/) {
+    constexpr int W = NT / 32;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    __syncwarp();
+    u = warp_sum(u);
+    v = warp_sum(v);
+    if (lane == 0) {
+        sh[warp] = u;
+        sh[32 + warp] = v;
     }
+    __syncwarp();
     __syncthreads();
-    const double s = sh[31];
-    __syncthreads();
-    return s;
+    if (warp == 0) {
+        u = warp_sum(lane < W ? sh[lane] : 0.0);
+        v = warp_sum(lane < W ? sh[32 + lane] : 0.0);
+    }
+    return make_double2(u, v);
 }
 
-__global__ void __launch_bounds__(kBlock, 1) cg_smem_cluster_kernel(SmemArgs a) {
+// Cluster-wide sums of (u, v): per-CTA block sums, one cluster barrier, then
+// lanes 0..C-1 of warp 0 fetch the C partials in parallel (one DSMEM round
+// trip) and a fixed butterfly: bit-identical sums in every CTA.  `mine` is
+// this CTA's partial slot (2 doubles); the next write to it is separated from
+// these reads by at least one more cluster barrier (callers' phase structure).
+template <int NT>
+__device__ __forceinline__ double2 cluster_sum2(double *mine, double u, double v, double *sh) {
+    namespace cgx = cooperative_groups;
+    auto cl = cgx::this_cluster();
+    const double2 t = blk_sum2<NT>(u, v, sh);
+    if (threadIdx.x == 0) {
+        mine[0] = t.x;
+        mine[1] = t.y;
+    }
+    cl.sync();
+    if (threadIdx.x < 32) {
+        const unsigned c = threadIdx.x;
+        double qu = 0.0, qv = 0.0;
+        if (c < cl.num_blocks()) {
+            const double *m = cl.map_shared_rank(mine, c);
+            qu = m[0];
+            qv = m[1];
+        }
+        qu = warp_sum(qu);
+        qv = warp_sum(qv);
+        if (threadIdx.x == 0) {
+            sh[64] = qu;
+            sh[65] = qv;
+        }
+    }
+    __syncthreads();
+    const double2 r = make_double2(sh[64], sh[65]);
+    __syncthreads();
+    return r;
+}
+
+// ----------------------------------- on-chip solve (tiny single-GPU problems)
+// The whole problem lives in the shared memory of ONE thread-block cluster
+// (<= 16 CTAs, 227 KB each): CTA c owns rows [c R, (c+1) R) -- its ELL slice,
+// b and the CG vectors -- loaded once per solve.  The stencil gathers read the
+// gathered vector from the owning CTA's shared memory (distributed shared
+// memory when it is a neighbour CTA), every reduction is C per-CTA partials
+// read by every CTA in rank order, and the phases are separated by the
+// hardware cluster barrier.  NT threads per CTA (512 when R > 256, so each
+// thread's rows are gathered in one trip).
+//   kSR = false: HPCCG's CG (A4, A11), 3 cluster barriers per iteration;
+//   kSR = true:  the single-reduction CG of f2 (oracle_cg_sr), 2 per iteration.
+// Per-row FMA chain as A8.
+template <int NT, bool kSR>
+__global__ void __launch_bounds__(NT, 1) cg_smem_cluster_kernel(SmemArgs a) {
     namespace cgx = cooperative_groups;
     auto cl = cgx::this_cluster();
     extern __shared__ double smem[];
-    __shared__ double sh[32];
-    __shared__ double part_pAp, part_rr;
+    __shared__ double sh[66];
+    __shared__ double part_a[2], part_b[2];
     const int R = a.R;
     const unsigned me = cl.block_rank();
     double *sval = smem;                        // [27][R]
     double *sb = sval + (size_t)kSlots * R;     // [R] each
-    double *sx = sb + R, *sr = sx + R, *sp = sr + R, *sAp = sp + R;
-    int *scol = reinterpret_cast<int *>(sAp + R);  // [27][R]
+    double *sx = sb + R, *sr = sx + R, *sp = sr + R, *sq = sp + R;  // sq: Ap (HPCCG) / w (SR)
+    double *ss = sq + R;                        // SR: s = A p recurrence
+    int *scol = reinterpret_cast<int *>(ss + (kSR ? R : 0));  // [27][R]
     const int64_t row0 = (int64_t)me * R;
     const int64_t rem = a.n - row0;
     const int nr = rem <= 0 ? 0 : (int)(rem < R ? rem : R);
-    // load this CTA's slice (global column ids -> owner CTA / offset later)
     for (int k = 0; k < kSlots; ++k)
-        for (int i = threadIdx.x; i < nr; i += kBlock) {
+        for (int i = threadIdx.x; i < nr; i += NT) {
             sval[k * R + i] = a.val[k * a.stride + row0 + i];
             scol[k * R + i] = a.col[k * a.stride + row0 + i];
         }
-    for (int i = threadIdx.x; i < nr; i += kBlock) {
+    for (int i = threadIdx.x; i < nr; i += NT) {
         sb[i] = a.b[row0 + i];
         sx[i] = a.x[row0 + i];
     }
     __syncthreads();
     const int plane32 = (int)a.plane;
-    auto spmv_row = [&](int i) {  // y_i = sum_k val * p[col], p read from its owner CTA
+    // y_i = sum_k val * g[col], g = the gathered vector, read from its owner CTA
+    auto spmv_row = [&](const double *g, int i) {
         double pv[kSlots];
 #pragma unroll
         for (int k = 0; k < kSlots; ++k) {  // all 27 gathers issued before the FMA chain
-            const int g = scol[k * R + i] - plane32;  // global row of the column (< 2^31)
-            const unsigned owner = (unsigned)g / (unsigned)R;
-            const int off = g - (int)owner * R;
-            pv[k] = *cl.map_shared_rank(sp + off, owner);
+            const int c = scol[k * R + i] - plane32;  // global row of the column (< 2^31)
+            const unsigned owner = (unsigned)c / (unsigned)R;
+            const int off = c - (int)owner * R;
+            pv[k] = *cl.map_shared_rank(g + off, owner);
         }
         double s = 0.0;
 #pragma unroll
         for (int k = 0; k < kSlots; ++k) s = fma(sval[k * R + i], pv[k], s);
         return s;
     };
-    // ---- init (a.7)
-    for (int i = threadIdx.x; i < nr; i += kBlock) sp[i] = sx[i];
-    cl.sync();
-    double acc = 0.0;
-    for (int i = threadIdx.x; i < nr; i += kBlock) {
-        const double rv = fma(-1.0, spmv_row(i), sb[i]);
-        sr[i] = rv;
-        acc = fma(rv, rv, acc);
-    }
-    double rr = cluster_sum(&part_rr, acc, sh);
-    double rtrans = rr, normr = sqrt(rtrans);
     int niters = 0;
-    for (int k = 1; k < a.max_iter && normr > a.tol; ++k) {
-        double beta = 0.0;
-        if (k > 1) {
-            const double old = rtrans;
-            rtrans = rr;
-            beta = rtrans / old;
-        }
-        // every CTA has finished reading the previous p (cluster_sum's barrier)
-        for (int i = threadIdx.x; i < nr; i += kBlock) sp[i] = (k == 1) ? sr[i] : fma(beta, sp[i], sr[i]);
-        normr = sqrt(rtrans);
+    double normr, rr_out, rr_prev_out;
+    if (!kSR) {
+        // ---- init (a.7): p = x; Ap = A p; r = b - Ap; rtrans = r.r
+        for (int i = threadIdx.x; i < nr; i += NT) sp[i] = sx[i];
         cl.sync();
-        double d = 0.0;
-        for (int i = threadIdx.x; i < nr; i += kBlock) {
-            const double ap = spmv_row(i);
-            sAp[i] = ap;
-            d = fma(ap, sp[i], d);
-        }
-        const double pAp = cluster_sum(&part_pAp, d, sh);
-        const bool stop = (rtrans == 0.0) || (pAp == 0.0);
-        const double alpha = stop ? 0.0 : rtrans / pAp;
-        acc = 0.0;
-        for (int i = threadIdx.x; i < nr; i += kBlock) {
-            sx[i] = fma(alpha, sp[i], sx[i]);
-            const double rv = fma(-alpha, sAp[i], sr[i]);
+        double acc = 0.0;
+        for (int i = threadIdx.x; i < nr; i += NT) {
+            const double rv = fma(-1.0, spmv_row(sp, i), sb[i]);
             sr[i] = rv;
             acc = fma(rv, rv, acc);
         }
-        rr = cluster_sum(&part_rr, acc, sh);
-        niters = k;
-        if (stop) break;
+        double rr = cluster_sum2<NT>(part_b, acc, 0.0, sh).x;
+        double rtrans = rr;
+        normr = sqrt(rtrans);
+        for (int k = 1; k < a.max_iter && normr > a.tol; ++k) {
+            double beta = 0.0;
+            if (k > 1) {
+                const double old = rtrans;
+                rtrans = rr;
+                beta = rtrans / old;
+            }
+            // every CTA has finished reading the previous p (cluster_sum2's barrier)
+            for (int i = threadIdx.x; i < nr; i += NT) sp[i] = (k == 1) ? sr[i] : fma(beta, sp[i], sr[i]);
+            normr = sqrt(rtrans);
+            cl.sync();
+            double d = 0.0;
+            for (int i = threadIdx.x; i < nr; i += NT) {
+                const double ap = spmv_row(sp, i);
+                sq[i] = ap;
+                d = fma(ap, sp[i], d);
+            }
+            const double pAp = cluster_sum2<NT>(part_a, d, 0.0, sh).x;
+            const bool stop = (rtrans == 0.0) || (pAp == 0.0);
+            const double alpha = stop ? 0.0 : rtrans / pAp;
+            acc = 0.0;
+            for (int i = threadIdx.x; i < nr; i += NT) {
+                sx[i] = fma(alpha, sp[i], sx[i]);
+                const double rv = fma(-alpha, sq[i], sr[i]);
+                sr[i] = rv;
+                acc = fma(rv, rv, acc);
+            }
+            rr = cluster_sum2<NT>(part_b, acc, 0.0, sh).x;
+            niters = k;
+            if (stop) break;
+        }
+        rr_out = rr;
+        rr_prev_out = rtrans;
+    } else {
+        // ---- init: r = b - A x0 (x0 gathered from sr), w = A r, (gamma, delta)
+        for (int i = threadIdx.x; i < nr; i += NT) sr[i] = sx[i];
+        cl.sync();
+        for (int i = threadIdx.x; i < nr; i += NT) sq[i] = fma(-1.0, spmv_row(sr, i), sb[i]);
+        cl.sync();  // every CTA has finished gathering x0 from sr
+        for (int i = threadIdx.x; i < nr; i += NT) sr[i] = sq[i];
+        cl.sync();
+        double g = 0.0, dl = 0.0;
+        for (int i = threadIdx.x; i < nr; i += NT) {
+            const double w = spmv_row(sr, i);
+            sq[i] = w;
+            g = fma(sr[i], sr[i], g);
+            dl = fma(w, sr[i], dl);
+        }
+        double2 gd = cluster_sum2<NT>(part_a, g, dl, sh);
+        double gamma = gd.x, delta = gd.y, gamma_old = 0.0, alpha_old = 0.0;
+        normr = sqrt(gamma);
+        for (int k = 1; k < a.max_iter && normr > a.tol; ++k) {
+            const bool first = (k == 1);
+            const double beta = first ? 0.0 : __ddiv_rn(gamma, gamma_old);
+            const double den = first ? delta : __dsub_rn(delta, __ddiv_rn(__dmul_rn(beta, gamma), alpha_old));
+            const bool stop = (gamma == 0.0) || (den == 0.0);  // A11
+            const double alpha = stop ? 0.0 : __ddiv_rn(gamma, den);
+            normr = sqrt(gamma);
+            // every CTA has finished gathering r (cluster_sum2's barrier)
+            for (int i = threadIdx.x; i < nr; i += NT) {
+                const double pv = first ? sr[i] : fma(beta, sp[i], sr[i]);
+                const double sv = first ? sq[i] : fma(beta, ss[i], sq[i]);
+                sp[i] = pv;
+                ss[i] = sv;
+                sx[i] = fma(alpha, pv, sx[i]);
+                sr[i] = fma(-alpha, sv, sr[i]);
+            }
+            niters = k;
+            // the next iteration would not run (A4, A11): skip its SpMV
+            if (stop || !(k + 1 < a.max_iter && normr > a.tol)) break;
+            cl.sync();
+            g = 0.0;
+            dl = 0.0;
+            for (int i = threadIdx.x; i < nr; i += NT) {
+                const double w = spmv_row(sr, i);
+                sq[i] = w;
+                g = fma(sr[i], sr[i], g);
+                dl = fma(w, sr[i], dl);
+            }
+            gd = cluster_sum2<NT>((k & 1) ? part_b : part_a, g, dl, sh);
+            gamma_old = gamma;
+            gamma = gd.x;
+            delta = gd.y;
+            alpha_old = alpha;
+        }
+        rr_out = gamma;
+        rr_prev_out = gamma_old;
     }
-    for (int i = threadIdx.x; i < nr; i += kBlock) a.x[row0 + i] = sx[i];
+    for (int i = threadIdx.x; i < nr; i += NT) a.x[row0 + i] = sx[i];
     if (me == 0 && threadIdx.x == 0) {
         a.sc->niters = niters;
         a.sc->normr = normr;
-        a.sc->rr_cur = rr;
-        a.sc->rr_prev = rtrans;
+        a.sc->rr_cur = rr_out;
+        a.sc->rr_prev = rr_prev_out;
         a.sc->done = 1;
     }
     cl.sync();  // no CTA leaves while its shared memory may still be read

@@ -41,15 +41,21 @@ def check(res, p, oref, ref):
     assert np.max(np.abs(p.get_vec(H.HPCCG_VEC_X) - oref["x"])) <= CG_ATOL
 
 
+@pytest.mark.parametrize("persist", [0, 1])
 @pytest.mark.parametrize("dims", [(20, 30, 10), (3, 3, 3), (16, 16, 16), (33, 9, 3), (31, 17, 9),
                                   (64, 32, 40)])
-def test_sr_cg_vs_oracle(ctx, dims):
+def test_sr_cg_vs_oracle(ctx, dims, persist):
+    """persist 0: the while-graph of 2-kernel iterations; persist 1: problems
+    that fit one cluster's shared memory run the on-chip single-reduction
+    kernel (2 cluster barriers per iteration), larger ones the while-graph."""
     with H.Problem(ctx, *dims) as p:
         sr(p)
+        p.set_option(H.HPCCG_OPT_PERSISTENT, persist)
         ref = oracle.generate(*dims)
         oref = oracle.cg_sr(ref, 150, 1e-12)
         res = p.solve(150, 1e-12)
-        assert p.stats()["graph_mode"] == 2          # while-graph (no persistent kernel)
+        n = dims[0] * dims[1] * dims[2]
+        assert p.stats()["graph_mode"] == (5 if persist and n <= 9000 else 2)
         check(res, p, oref, ref)
         # same solution as HPCCG's CG
         assert abs(res["niters"] - oracle.cg(ref, 150, 1e-12)["niters"]) <= 1
@@ -57,11 +63,13 @@ def test_sr_cg_vs_oracle(ctx, dims):
             assert res["niters"] == 50
 
 
-def test_sr_first_step_exact(ctx):
+@pytest.mark.parametrize("persist", [0, 1])
+def test_sr_first_step_exact(ctx, persist):
     """x0 = 0: gamma0 = b.b, delta0 = (Ab).b exact integers -> alpha1 correctly
     rounded, x1 = fl(alpha1 b) bitwise, normr = sqrt(b.b)."""
     with H.Problem(ctx, 20, 30, 10) as p:
         sr(p)
+        p.set_option(H.HPCCG_OPT_PERSISTENT, persist)
         r = p.solve(2, 0.0)
         assert r["niters"] == 1
         b = p.get_vec(H.HPCCG_VEC_B)
@@ -78,6 +86,7 @@ def test_sr_launch_modes_bitwise_identical(ctx, rows):
     outs, xs = [], []
     with H.Problem(ctx, *dims) as p:
         sr(p)
+        p.set_option(H.HPCCG_OPT_PERSISTENT, 0)
         p.set_option(H.HPCCG_OPT_SPMV_ROWS, rows)
         cfgs = [dict(wu=4), dict(wu=1), dict(wu=3), dict(wu=6), dict(wh=0), dict(graph=0),
                 dict(timing=1), dict(unroll=1), dict(unroll=2), dict(pdl=0)]
@@ -101,13 +110,14 @@ def test_sr_launch_modes_bitwise_identical(ctx, rows):
         np.testing.assert_array_equal(x, xs[0])
 
 
-@pytest.mark.parametrize("wh", [0, 1])
-def test_sr_max_iter_semantics_odd_and_even(ctx, wh):
+@pytest.mark.parametrize("wh,persist", [(0, 0), (1, 0), (1, 1)])
+def test_sr_max_iter_semantics_odd_and_even(ctx, wh, persist):
     """A4 with the parity-double-buffered loop state: at most max_iter - 1
-    iterations for odd and even counts, in the while-graph and in the
-    per-iteration graph (which replays iteration PAIRS)."""
+    iterations for odd and even counts, in the while-graph, in the
+    per-iteration graph (which replays iteration PAIRS) and on chip."""
     with H.Problem(ctx, 8, 8, 8) as p:
         sr(p)
+        p.set_option(H.HPCCG_OPT_PERSISTENT, persist)
         p.set_option(H.HPCCG_OPT_WHILE, wh)
         ref = oracle.generate(8, 8, 8)
         for m in [1, 2, 3, 4, 10, 37]:
@@ -126,6 +136,7 @@ def test_sr_max_iter_semantics_odd_and_even(ctx, wh):
 def test_sr_tolerance_stop(ctx, wh):
     with H.Problem(ctx, 20, 30, 10) as p:
         sr(p)
+        p.set_option(H.HPCCG_OPT_PERSISTENT, 0)
         p.set_option(H.HPCCG_OPT_WHILE, wh)
         r = p.solve(150, 1e-12)
         assert r["niters"] == 50
@@ -133,10 +144,12 @@ def test_sr_tolerance_stop(ctx, wh):
         assert p.solve(150, 1e-12)["niters"] <= 2
 
 
+@pytest.mark.parametrize("persist", [0, 1])
 @pytest.mark.parametrize("dims", [(1, 1, 1), (2, 2, 2), (4, 1, 1)])
-def test_sr_degenerate_guard(ctx, dims):
+def test_sr_degenerate_guard(ctx, dims, persist):
     with H.Problem(ctx, *dims) as p:
         sr(p)
+        p.set_option(H.HPCCG_OPT_PERSISTENT, persist)
         r = p.solve(60, 0.0)
         assert np.all(np.isfinite(p.get_vec(H.HPCCG_VEC_X))) and p.maxabsdiff() < 1e-14
         assert r["niters"] < 59

@@ -11,7 +11,7 @@ nx, ny, nz, iters = (int(v) for v in sys.argv[1:5])
 KEYS = {"graph": H.HPCCG_OPT_GRAPH, "timing": H.HPCCG_OPT_TIMING, "while": H.HPCCG_OPT_WHILE,
         "pdl": H.HPCCG_OPT_PDL, "waves": H.HPCCG_OPT_VEC_WAVES, "unroll": H.HPCCG_OPT_VEC_UNROLL,
         "rows": H.HPCCG_OPT_SPMV_ROWS, "l2": H.HPCCG_OPT_L2_PERSIST,
-        "wu": H.HPCCG_OPT_WHILE_UNROLL}
+        "wu": H.HPCCG_OPT_WHILE_UNROLL, "ff": H.HPCCG_OPT_FINISHER_FREE}
 ctx = H.Context(0)
 p = H.Problem(ctx, nx, ny, nz)
 p.set_option(H.HPCCG_OPT_PERSISTENT, 0)
