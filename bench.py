@@ -115,18 +115,25 @@ def cg_flops(niters, nnz, n):
 
 # ------------------------------------------------------------ oracle (CPU)
 
-def oracle_sample(nx, ny, nz, iters_cap, budget_s):
+def oracle_cg_timed(prob, max_iter, sr=False):
+    """One oracle CG solve (HPCCG's, or f2's single-reduction) -> (result, seconds)."""
+    import oracle
+    t0 = time.perf_counter()
+    r = oracle.cg_sr(prob, max_iter, 0.0) if sr else oracle.cg(prob, max_iter, 0.0)
+    return r, time.perf_counter() - t0
+
+
+def oracle_sample(nx, ny, nz, iters_cap, budget_s, sr=False):
     """Time the CPU oracle (as it stands) on a bounded sample of the
     workload: the same generated problem, m CG iterations, all host cores."""
     import oracle
     t0 = time.perf_counter()
     prob = oracle.generate(nx, ny, nz)
     gen_s = time.perf_counter() - t0
-    r1 = oracle.cg(prob, 2, 0.0)           # calibrate: 1 iteration
-    per_it = max(r1["times"][0], 1e-6)
+    _, per_it = oracle_cg_timed(prob, 2, sr)   # calibrate: 1 iteration
+    per_it = max(per_it, 1e-6)
     m = int(max(1, min(iters_cap, budget_s / per_it)))
-    r = oracle.cg(prob, m + 1, 0.0)
-    t = r["times"][0]
+    r, t = oracle_cg_timed(prob, m + 1, sr)
     gflops = cg_flops(r["niters"], prob.nnz, prob.n) / t * 1e-9
     return {"value": gflops, "iters": r["niters"], "seconds": t, "gen_s": gen_s,
             "cores": oracle.get_threads(), "prob": prob}
@@ -140,12 +147,13 @@ def run_reference(args, nx, ny, nz, iters, cfg_index):
     oracle.build()
     prob = oracle.generate(nx, ny, nz)
     m = max(1, min(iters, args.ref_iters))
+    sr = args.cg_variant == "sr"
     for _ in range(args.warmup):
-        oracle.cg(prob, m + 1, 0.0)
+        oracle_cg_timed(prob, m + 1, sr)
     tot, flops = 0.0, 0.0
     for _ in range(args.steps):
-        r = oracle.cg(prob, m + 1, 0.0)
-        tot += r["times"][0]
+        r, t = oracle_cg_timed(prob, m + 1, sr)
+        tot += t
         flops += cg_flops(r["niters"], prob.nnz, prob.n)
     val = flops / tot * 1e-9
     sample = (f"oracle CG on the {nx}x{ny}x{nz} problem, {m} iterations per step "
@@ -203,6 +211,8 @@ def run_ours(args, nx, ny, nz, iters, cfg_index, scaling):
     n, nnz_local = prob.n, prob.info["nnz_local"]
     nnz_global = prob.info["nnz_global"]
     prob.set_option(H.HPCCG_OPT_GRAPH, 1)
+    sr = args.cg_variant == "sr"
+    prob.set_option(H.HPCCG_OPT_CG_VARIANT, 1 if sr else 0)
     xptr = prob.vec_ptr(H.HPCCG_VEC_X)
 
     def barrier():
@@ -291,8 +301,9 @@ def run_ours(args, nx, ny, nz, iters, cfg_index, scaling):
             avg_ms = spmv_ms / spmv_n
             ach = spmv_bytes / (avg_ms * 1e-3) * 1e-9
             roof = {"bound": "hbm",
-                    "kernel": "spmv27x2_kernel<dot> (2 rows/thread; spmv27_kernel<dot> if n or the "
-                              "plane is odd)",
+                    "kernel": ("spmv27x2_kernel<2> (w = A r with the r.r, w.r epilogue, f2)" if sr else
+                               "spmv27x2_kernel<1> (p.Ap epilogue)") +
+                              " -- 2 rows/thread; spmv27_kernel if n or the plane is odd",
                     "achieved": round(ach, 1),
                     "peak": peak, "unit": "GB/s", "frac": round(ach / peak, 4),
                     "frac_of_8TBs_nominal": round(ach / 8000.0, 4),
@@ -310,7 +321,7 @@ def run_ours(args, nx, ny, nz, iters, cfg_index, scaling):
             # the oracle's CSR needs ~430 B/row of host RAM: above 2^25 rows it
             # is timed on the 256^3 problem instead (said in `sample`)
             ox, oy, oz = (nx, ny, nz) if n <= (1 << 25) else (256, 256, 256)
-            cs = oracle_sample(ox, oy, oz, iters, args.cpu_budget)
+            cs = oracle_sample(ox, oy, oz, iters, args.cpu_budget, sr)
             nx_s = f"{ox}x{oy}x{oz}"
             cpu = {"value": round(cs["value"], 4), "unit": "GFLOP/s", "cores": cs["cores"],
                    "kind": "oracle",
@@ -327,7 +338,10 @@ def run_ours(args, nx, ny, nz, iters, cfg_index, scaling):
                        "nx": nx, "ny": ny, "nz_per_gpu": nz, "iters": iters,
                        "global_rows": n * world, "global_nnz": nnz_global,
                        "parallelism": f"zslab{world}",
-                       "solve_graph": {2: "while-graph", 1: "per-iteration graph", 0: "plain"}.get(
+                       "cg_variant": "single-reduction (Chronopoulos-Gear, f2)" if sr else "HPCCG",
+                       "solve_graph": {5: "on-chip cluster kernel", 4: "one-cluster persistent kernel",
+                                       3: "cooperative persistent kernel", 2: "while-graph",
+                                       1: "per-iteration graph", 0: "plain"}.get(
                            main.get("graph_mode"), "?"),
                        "l2": "inputs larger than L2 (ELL %.0f MB/GPU > 126 MB)" % (324e-6 * n),
                        "gen_ms": round(gen_ms, 3)},
@@ -613,6 +627,8 @@ def main():
     ap.add_argument("--tri-n", type=int, default=100_000_000, help="tridiag SIZE (P:L475)")
     ap.add_argument("--lbm-size", type=int, default=1000, help="LBM SIZE (P:L411)")
     ap.add_argument("--iters", type=int, default=None, help="override CG iterations per step")
+    ap.add_argument("--cg-variant", choices=["hpccg", "sr"], default="hpccg",
+                    help="hpccg: HPCCG's CG (default); sr: single-reduction CG (SURVEY f2)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-budget", type=float, default=12.0, help="seconds of oracle CG")
     ap.add_argument("--ref-iters", type=int, default=20, help="oracle iterations per reference step")
