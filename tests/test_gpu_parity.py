@@ -620,3 +620,67 @@ def test_cg_finisher_free_loop_bitwise_vs_finisher(ctx, unroll, dims, max_iter, 
         np.testing.assert_array_equal(o[2], outs[0][2])
     if tol == 0.0 and dims != (2, 2, 2):
         assert outs[0][0] == max_iter - 1
+
+
+# ------------------------- full sizes of BASELINE configs[2] and configs[3]
+
+def test_full_256cubed_vs_oracle(ctx):
+    """BASELINE configs[2] at one GPU (256^3, the bench's hpccg256 launch
+    configuration): sampled SpMV rows bitwise; CG to tol 1e-12 vs the full
+    oracle CG (niters +-1, x / normr within 1e-10); the 200-iteration tol-0
+    bench step stays at the solution."""
+    nx = ny = nz = 256
+    with H.Problem(ctx, nx, ny, nz) as p:
+        n, plane = p.n, nx * ny
+        assert p.info["nnz_global"] == (3 * 256 - 2) ** 3
+        x = synth.uniform(n, 91)
+        xl = np.zeros(n + 2 * plane)
+        xl[plane:plane + n] = x
+        y = torch.empty(n, dtype=torch.float64, device="cuda")
+        p.spmv(dev(xl), y)
+        rows = synth.sample_rows(n, 3000, 6)
+        np.testing.assert_array_equal(y.cpu().numpy()[rows], oracle.spmv_rows(nx, ny, nz, rows, x))
+        del y
+        res = p.solve(150, 1e-12)
+        ref = oracle.generate(nx, ny, nz)
+        oref = oracle.cg(ref, 150, 1e-12)
+        check_cg(res, p.maxabsdiff(), oref, ref)
+        assert np.max(np.abs(p.get_vec(H.HPCCG_VEC_X) - oref["x"])) <= CG_ATOL
+        del ref
+        p.set_vec(H.HPCCG_VEC_X, np.zeros(n))
+        r200 = p.solve(201, 0.0)
+        assert r200["niters"] == 200 and p.maxabsdiff() < 1e-13
+
+
+def test_full_512cubed_sampled_and_properties(ctx):
+    """BASELINE configs[3] at one GPU (512^3 = 134M rows, nnz 3.61e9 > 2^31:
+    64-bit slot offsets, A14).  The oracle's CSR would need ~50 GB of host RAM,
+    so: sampled SpMV rows bitwise vs the oracle's row-at-a-time evaluation, A.1
+    == b exactly (integer arithmetic, every row), and the CG solution checked
+    by properties that hold at any size -- max|x - 1| at the rounding floor,
+    the true residual ||b - A x|| (our SpMV, verified above) small relative to
+    ||b|| (A7), and the lagged normr below tol."""
+    nx = ny = nz = 512
+    with H.Problem(ctx, nx, ny, nz) as p:
+        n, plane = p.n, nx * ny
+        assert p.info["nnz_global"] == (3 * 512 - 2) ** 3
+        xl = torch.zeros(n + 2 * plane, dtype=torch.float64, device="cuda")
+        xs = synth.uniform(1 << 20, 93)
+        xl[plane:plane + n] = torch.from_numpy(np.resize(xs, n)).cuda()
+        y = torch.empty(n, dtype=torch.float64, device="cuda")
+        p.spmv(xl, y)
+        rows = synth.sample_rows(n, 2000, 7)
+        xh = xl[plane:plane + n].cpu().numpy()
+        np.testing.assert_array_equal(y.cpu().numpy()[rows], oracle.spmv_rows(nx, ny, nz, rows, xh))
+        b = torch.from_numpy(p.get_vec(H.HPCCG_VEC_B)).cuda()
+        xl.zero_()
+        xl[plane:plane + n] = 1.0
+        p.spmv(xl, y)
+        assert torch.equal(y, b)                         # A.1 == b, every row
+        res = p.solve(150, 1e-12)
+        assert 100 <= res["niters"] <= 130               # 256^3: 112 (oracle-checked above)
+        assert res["normr"] <= 1e-12
+        assert p.maxabsdiff() < 1e-13
+        xl[plane:plane + n] = torch.from_numpy(p.get_vec(H.HPCCG_VEC_X)).cuda()
+        p.spmv(xl, y)
+        assert float(torch.linalg.norm(b - y)) <= 1e-13 * float(torch.linalg.norm(b))
