@@ -108,6 +108,17 @@ extern "C" {
                                r.r and the loop control */
 #define HPCCG_OPT_SMEM_THREADS 18 /* threads per CTA of the shared-memory-resident solve:
                                0 (default) auto (512 when a CTA holds > 256 rows), 256, 512 */
+#define HPCCG_OPT_HALO_PEER 19 /* multi-slab: 1 = the halo exchange and the scalar allreduces
+                               run as this library's own kernels over PEER MEMORY -- each slab
+                               pushes its boundary planes straight into its neighbours' halo
+                               planes and signals them (flag + system-scope release), and each
+                               allreduce posts the local value into slot [rank] of every peer and
+                               sums the P slots in rank order -- instead of NCCL send/recv /
+                               ncclAllReduce (or the loopback copies).  NCCL contexts map the
+                               peers' buffers with CUDA IPC (collective: every rank sets it);
+                               loopback contexts use the sibling slabs.  0 (default): off.
+                               Bit-identical to the loopback reduction order.  Waits time out
+                               after ~2 s with HPCCG_ECUDA instead of hanging. */
 #define HPCCG_OPT_WHILE_UNROLL 15 /* CG iterations per execution of the WHILE body
                                (default 4: amortises the conditional node's ~8 us) */
 #define HPCCG_OPT_CLUSTER_ROWS 12 /* up to this many rows (default 16384) the persistent solve

@@ -120,6 +120,8 @@ struct Slab {
     double *spmv_parts = nullptr;  // per-block p.Ap partials (single slab); f2: 2 arrays
     int64_t spmv_nparts = 0;
     double *sv = nullptr;  // f2 single-reduction CG: s = A p recurrence vector (n)
+    PeerSync *psync = nullptr;  // HALO_PEER: this slab's flags / allreduce slots
+    PeerTab *ptab = nullptr;    // HALO_PEER: device copy of the peer table
 };
 
 struct TimedOp {
@@ -149,6 +151,8 @@ struct hpccg_problem {
     int opt_variant = 0;               // 0 HPCCG CG, 1 single-reduction CG (f2)
     int opt_ff = 1;                    // single slab: finisher-free HPCCG loop (consumer-side sums)
     int opt_smem_threads = 0;          // on-chip solve CTA width: 0 auto, 256, 512
+    int opt_peer = 0;                  // multi-slab: halo push + allreduce over peer memory
+    std::vector<void *> ipc_opened;    // peers' buffers mapped with cudaIpcOpenMemHandle
     int last_persist_mode = 3;
     // graph of one CG iteration (per-iteration replay) ...
     cudaGraphExec_t graph = nullptr;
@@ -331,6 +335,59 @@ int exchange(hpccg_problem *p, double *const *xs, cudaStream_t on) {
 #endif
 }
 
+// HALO_PEER (multi-slab, opt_peer): the halo exchange as our own push /
+// wait kernels over peer memory (kernels.cuh "peer-memory z-slab exchange").
+bool peer_on(const hpccg_problem *p) { return p->opt_peer && p->ctx->mode != MODE_SINGLE; }
+
+// push every hosted slab's boundary planes of x (local-with-halo bases xs)
+int halo_push(hpccg_problem *p, double *const *xs, cudaStream_t on) {
+    hpccg_ctx *ctx = p->ctx;
+    const Slab &s0 = p->slabs[0];
+    const int g = wave_grid(2 * s0.plane, wave(ctx, halo_push_kernel));
+    for (size_t i = 0; i < p->slabs.size(); ++i) {
+        halo_push_kernel<<<g, kBlock, 0, on>>>(p->slabs[i].ptab, xs[i], s0.n, s0.plane);
+        CHECK(check_launch(ctx));
+    }
+    return HPCCG_OK;
+}
+
+int halo_wait(hpccg_problem *p, cudaStream_t on) {
+    for (const Slab &s : p->slabs) {
+        halo_wait_kernel<<<1, 32, 0, on>>>(s.ptab);
+        CHECK(check_launch(p->ctx));
+    }
+    return HPCCG_OK;
+}
+
+// exchange of the internal gathered vector before an SpMV that does not
+// overlap it (init): copies / NCCL, or push + wait
+int halo_exchange(hpccg_problem *p, double *const *xs, cudaStream_t on) {
+    if (!peer_on(p)) return exchange(p, xs, on);
+    CHECK(halo_push(p, xs, on));
+    return halo_wait(p, on);
+}
+
+// allreduce of `count` doubles per slab (src -> dst, identical on all slabs)
+// over peer memory: posts of every hosted slab, then the collects (loopback
+// hosts all slabs in one stream, so every post must precede every collect)
+int peer_allreduce(hpccg_problem *p, double *const *src, double *const *dst, int count, bool is_max) {
+    hpccg_ctx *ctx = p->ctx;
+    const size_t P = p->slabs.size();
+    if (P == 1) {
+        peer_allreduce_kernel<<<1, 32, 0, ctx->stream>>>(p->slabs[0].ptab, src[0], dst[0], count, is_max, 1, 1);
+        return check_launch(ctx);
+    }
+    for (size_t i = 0; i < P; ++i) {
+        peer_allreduce_kernel<<<1, 32, 0, ctx->stream>>>(p->slabs[i].ptab, src[i], dst[i], count, is_max, 1, 0);
+        CHECK(check_launch(ctx));
+    }
+    for (size_t i = 0; i < P; ++i) {
+        peer_allreduce_kernel<<<1, 32, 0, ctx->stream>>>(p->slabs[i].ptab, src[i], dst[i], count, is_max, 0, 1);
+        CHECK(check_launch(ctx));
+    }
+    return HPCCG_OK;
+}
+
 // ------------------------------------------------------------- launchers
 // `check`: kernels test the device `done` flag first (plain launches and the
 // per-iteration graph, which may run past convergence).  The while-graph
@@ -502,6 +559,50 @@ int launch_update(hpccg_ctx *ctx, int waves, int unroll, int64_t cap, const Slab
                  : launch_update_u<false, false>(ctx, waves, 1, cap, a, pdl);
 }
 
+// Multi-slab SpMV around the halo exchange: the interior rows (planes
+// 1..nz-2, no halo reads) overlap the exchange, the two boundary planes
+// follow it.  NCCL: send/recv on the comm stream; HALO_PEER: our push kernel
+// on the comm stream (NCCL ctx) or in stream order before the interiors
+// (loopback), then a wait kernel before the boundaries; loopback copies: the
+// exchange first.  slab_spmv(slab, interior) launches one part.
+template <class F>
+int spmv_overlapped(hpccg_problem *p, bool timing, double *const *xs, F slab_spmv) {
+    hpccg_ctx *ctx = p->ctx;
+    const bool peer = peer_on(p);
+    if (ctx->mode == MODE_NCCL) {
+        CU(cudaEventRecord(ctx->ev_fork, ctx->stream));
+        CU(cudaStreamWaitEvent(ctx->comm_stream, ctx->ev_fork, 0));
+        {
+            PhaseTimer t(p, ctx->comm_stream, PH_EXCHANGE, timing);
+            if (peer) CHECK(halo_push(p, xs, ctx->comm_stream));
+            else CHECK(exchange(p, xs, ctx->comm_stream));
+        }
+        CU(cudaEventRecord(ctx->ev_join, ctx->comm_stream));
+        PhaseTimer t(p, ctx->stream, PH_SPMV, timing);
+        CHECK(slab_spmv(p->slabs[0], true));
+        if (peer) CHECK(halo_wait(p, ctx->stream));
+        CU(cudaStreamWaitEvent(ctx->stream, ctx->ev_join, 0));
+        return slab_spmv(p->slabs[0], false);
+    }
+    {
+        PhaseTimer t(p, ctx->stream, PH_EXCHANGE, timing);
+        if (peer) CHECK(halo_push(p, xs, ctx->stream));
+        else CHECK(exchange(p, xs, ctx->stream));
+    }
+    PhaseTimer t(p, ctx->stream, PH_SPMV, timing);
+    if (peer) {
+        for (const Slab &s : p->slabs) CHECK(slab_spmv(s, true));
+        CHECK(halo_wait(p, ctx->stream));
+        for (const Slab &s : p->slabs) CHECK(slab_spmv(s, false));
+        return HPCCG_OK;
+    }
+    for (const Slab &s : p->slabs) {
+        CHECK(slab_spmv(s, true));
+        CHECK(slab_spmv(s, false));
+    }
+    return HPCCG_OK;
+}
+
 // CG SpMV of every slab with the p.Ap epilogue.  Multi-slab: the rows that
 // do not touch a halo plane (interior) run first, overlapped with the halo
 // exchange on the comm stream (NCCL), then the two boundary planes.
@@ -532,41 +633,18 @@ int cg_spmv_all(hpccg_problem *p, bool timing, bool check) {
     std::vector<double *> xs(p->slabs.size());
     for (size_t i = 0; i < xs.size(); ++i) xs[i] = p->slabs[i].p;
 
-    if (ctx->mode == MODE_NCCL) {
-        CU(cudaEventRecord(ctx->ev_fork, ctx->stream));
-        CU(cudaStreamWaitEvent(ctx->comm_stream, ctx->ev_fork, 0));
-        {
-            PhaseTimer t(p, ctx->comm_stream, PH_EXCHANGE, timing);
-            CHECK(exchange(p, xs.data(), ctx->comm_stream));
-        }
-        CU(cudaEventRecord(ctx->ev_join, ctx->comm_stream));
-        const Slab &s = p->slabs[0];
-        PhaseTimer t(p, ctx->stream, PH_SPMV, timing);
+    auto slab_spmv = [&](const Slab &s, bool interior) {
         SpmvArgs a = spmv_args(s, s.p, s.Ap);
         a.single = 0;
         a.total_blocks = nb_int + nb_bnd;
-        a.part_base = 0;
-        CHECK(launch_spmv<1>(ctx, minb, check, a, int_r0, int_len, 0, 0, ctx->stream, rows));
-        CU(cudaStreamWaitEvent(ctx->stream, ctx->ev_join, 0));
+        if (interior) {
+            a.part_base = 0;
+            return launch_spmv<1>(ctx, minb, check, a, int_r0, int_len, 0, 0, ctx->stream, rows);
+        }
         a.part_base = nb_int;
         return launch_spmv<1>(ctx, minb, check, a, 0, b0_len, b1_r0, b1_len, ctx->stream, rows);
-    }
-    // loopback: exchange, then interior + boundary launches per slab
-    {
-        PhaseTimer t(p, ctx->stream, PH_EXCHANGE, timing);
-        CHECK(exchange(p, xs.data(), ctx->stream));
-    }
-    PhaseTimer t(p, ctx->stream, PH_SPMV, timing);
-    for (const Slab &s : p->slabs) {
-        SpmvArgs a = spmv_args(s, s.p, s.Ap);
-        a.single = 0;
-        a.total_blocks = nb_int + nb_bnd;
-        a.part_base = 0;
-        CHECK(launch_spmv<1>(ctx, minb, check, a, int_r0, int_len, 0, 0, ctx->stream, rows));
-        a.part_base = nb_int;
-        CHECK(launch_spmv<1>(ctx, minb, check, a, 0, b0_len, b1_r0, b1_len, ctx->stream, rows));
-    }
-    return HPCCG_OK;
+    };
+    return spmv_overlapped(p, timing, xs.data(), slab_spmv);
 }
 
 double **tab(hpccg_problem *p, int which) { return p->d_tab + (size_t)which * p->ctx->nslabs; }
@@ -581,6 +659,14 @@ int allreduce_cg(hpccg_problem *p, bool rr, bool timing) {
     if (ctx->mode == MODE_SINGLE) return HPCCG_OK;
     PhaseTimer t(p, ctx->stream, PH_ALLREDUCE, timing);
     const Slab &s = p->slabs[0];
+    if (peer_on(p)) {
+        std::vector<double *> src, dst;
+        for (const Slab &sl : p->slabs) {
+            src.push_back(rr ? &sl.sc->loc_rr : &sl.sc->loc_pAp);
+            dst.push_back(rr ? &sl.sc->rr_cur : &sl.sc->pAp);
+        }
+        return peer_allreduce(p, src.data(), dst.data(), 1, false);
+    }
     double *hs[1] = {rr ? &s.sc->loc_rr : &s.sc->loc_pAp};
     double *hd[1] = {rr ? &s.sc->rr_cur : &s.sc->pAp};
     return allreduce_scalar(ctx, hs, hd, tab(p, rr ? 2 : 0), tab(p, rr ? 3 : 1), false);
@@ -710,7 +796,7 @@ int enqueue_init(hpccg_problem *p, int max_iter, double tol, bool timing,
     for (size_t i = 0; i < xs.size(); ++i) xs[i] = p->slabs[i].p;
     {
         PhaseTimer t(p, ctx->stream, PH_EXCHANGE, timing);
-        CHECK(exchange(p, xs.data(), ctx->stream));
+        CHECK(halo_exchange(p, xs.data(), ctx->stream));
     }
     {
         PhaseTimer t(p, ctx->stream, PH_SPMV, timing);
@@ -807,31 +893,17 @@ int cg_sr_spmv_all(hpccg_problem *p, bool timing, bool check, int q) {
         a.part_base = nb_int;
         return launch_spmv<2>(ctx, minb, check, a, 0, b0_len, b1_r0, b1_len, ctx->stream, rows);
     };
-    if (ctx->mode == MODE_NCCL) {
-        CU(cudaEventRecord(ctx->ev_fork, ctx->stream));
-        CU(cudaStreamWaitEvent(ctx->comm_stream, ctx->ev_fork, 0));
-        {
-            PhaseTimer t(p, ctx->comm_stream, PH_EXCHANGE, timing);
-            CHECK(exchange(p, xs.data(), ctx->comm_stream));
-        }
-        CU(cudaEventRecord(ctx->ev_join, ctx->comm_stream));
-        PhaseTimer t(p, ctx->stream, PH_SPMV, timing);
-        CHECK(slab_spmv(p->slabs[0], true));
-        CU(cudaStreamWaitEvent(ctx->stream, ctx->ev_join, 0));
-        CHECK(slab_spmv(p->slabs[0], false));
-    } else {
-        {
-            PhaseTimer t(p, ctx->stream, PH_EXCHANGE, timing);
-            CHECK(exchange(p, xs.data(), ctx->stream));
-        }
-        PhaseTimer t(p, ctx->stream, PH_SPMV, timing);
-        for (const Slab &s : p->slabs) {
-            CHECK(slab_spmv(s, true));
-            CHECK(slab_spmv(s, false));
-        }
-    }
+    CHECK(spmv_overlapped(p, timing, xs.data(), slab_spmv));
     for (const Slab &s : p->slabs) CHECK(finish(s, nb_int + nb_bnd, s.sc->loc_gd));
     PhaseTimer t(p, ctx->stream, PH_ALLREDUCE, timing);
+    if (peer_on(p)) {
+        std::vector<double *> src, dst;
+        for (const Slab &sl : p->slabs) {
+            src.push_back(sl.sc->loc_gd);
+            dst.push_back(sl.sc->gd);
+        }
+        return peer_allreduce(p, src.data(), dst.data(), 2, false);
+    }
     double *hs[1] = {p->slabs[0].sc->loc_gd};
     double *hd[1] = {p->slabs[0].sc->gd};
     return allreduce_scalar(ctx, hs, hd, tab(p, 6), tab(p, 7), false, 2);
@@ -901,7 +973,7 @@ int enqueue_init_sr(hpccg_problem *p, int max_iter, double tol, bool timing,
     for (size_t i = 0; i < xs.size(); ++i) xs[i] = p->slabs[i].p;
     {
         PhaseTimer t(p, ctx->stream, PH_EXCHANGE, timing);
-        CHECK(exchange(p, xs.data(), ctx->stream));
+        CHECK(halo_exchange(p, xs.data(), ctx->stream));
     }
     {
         PhaseTimer t(p, ctx->stream, PH_SPMV, timing);
@@ -1250,6 +1322,8 @@ void free_slab(Slab &s) {
     cudaFree(s.bar);
     cudaFree(s.spmv_parts);
     cudaFree(s.sv);
+    cudaFree(s.psync);
+    cudaFree(s.ptab);
     cudaFree(s.trace);
     s = Slab{};
 }
@@ -1378,6 +1452,91 @@ int api_reduce(hpccg_ctx *ctx, bool is_max, double *result, L launch) {
     }
     CU(cudaStreamSynchronize(ctx->stream));
     *result = *(volatile double *)ctx->h_pinned;
+    return HPCCG_OK;
+}
+
+// HALO_PEER setup (collective): every slab's PeerSync, and the peer tables.
+// Loopback: the neighbours' buffers are sibling slabs in this process.  NCCL
+// (one slab per rank, one GPU each): every rank exports its CG arena (which
+// holds the halo'd vector) and its PeerSync with cudaIpcGetMemHandle, the
+// handles are all-gathered over the library's communicator, and the peers'
+// buffers are mapped with cudaIpcOpenMemHandle (NVLink P2P); the arena layout
+// is identical on every rank, so a peer's vector is at the same offset.
+int enable_peer(hpccg_problem *p) {
+    hpccg_ctx *ctx = p->ctx;
+    const int P = ctx->nranks;
+    if (P > kMaxPeers) return fail(HPCCG_ENOTSUP, "peer mode supports up to %d ranks", kMaxPeers);
+    for (Slab &sl : p->slabs)
+        if (!sl.psync) CHECK(alloc_zero((void **)&sl.psync, sizeof(PeerSync)));
+    const Slab &s0 = p->slabs[0];
+    const int64_t n = s0.n, plane = s0.plane;
+    std::vector<PeerSync *> sync(P, nullptr);
+    std::vector<double *> pvec(P, nullptr);  // each rank's local-with-halo vector base
+    if (ctx->mode == MODE_LOOPBACK) {
+        for (int q = 0; q < P; ++q) {
+            sync[q] = p->slabs[q].psync;
+            pvec[q] = p->slabs[q].p;
+        }
+    } else if (ctx->mode == MODE_NCCL) {
+#ifdef HPCCG_WITH_NCCL
+        const int r = ctx->rank;
+        const size_t hb = sizeof(cudaIpcMemHandle_t);
+        std::vector<unsigned char> mine(2 * hb), all(2 * hb * P);
+        cudaIpcMemHandle_t h[2];
+        CU(cudaIpcGetMemHandle(&h[0], s0.arena));
+        CU(cudaIpcGetMemHandle(&h[1], s0.psync));
+        memcpy(mine.data(), h, 2 * hb);
+        unsigned char *d = nullptr;
+        CU(cudaMalloc((void **)&d, 2 * hb * (P + 1)));
+        CU(cudaMemcpy(d, mine.data(), 2 * hb, cudaMemcpyHostToDevice));
+        ncclResult_t nr = ncclAllGather(d, d + 2 * hb, 2 * hb, ncclUint8, ctx->comm, ctx->stream);
+        if (nr != ncclSuccess) {
+            cudaFree(d);
+            return nccl_fail(ctx, nr, "ncclAllGather(ipc handles)");
+        }
+        CU(cudaStreamSynchronize(ctx->stream));
+        CU(cudaMemcpy(all.data(), d + 2 * hb, 2 * hb * P, cudaMemcpyDeviceToHost));
+        cudaFree(d);
+        for (int q = 0; q < P; ++q) {
+            if (q == r) {
+                sync[q] = s0.psync;
+                pvec[q] = s0.p;
+                continue;
+            }
+            cudaIpcMemHandle_t hq[2];
+            memcpy(hq, all.data() + 2 * hb * q, 2 * hb);
+            void *ps = nullptr;
+            CU(cudaIpcOpenMemHandle(&ps, hq[1], cudaIpcMemLazyEnablePeerAccess));
+            p->ipc_opened.push_back(ps);
+            sync[q] = (PeerSync *)ps;
+            if (q == r - 1 || q == r + 1) {  // neighbours: their halo'd vector
+                void *pa = nullptr;
+                CU(cudaIpcOpenMemHandle(&pa, hq[0], cudaIpcMemLazyEnablePeerAccess));
+                p->ipc_opened.push_back(pa);
+                pvec[q] = (double *)pa + (s0.p - s0.arena);
+            }
+        }
+#else
+        return fail(HPCCG_ENOTSUP, "built without NCCL");
+#endif
+    } else {
+        return HPCCG_OK;  // single GPU: nothing to exchange
+    }
+    for (size_t i = 0; i < p->slabs.size(); ++i) {
+        Slab &sl = p->slabs[i];
+        const int r = ctx->mode == MODE_LOOPBACK ? (int)i : ctx->rank;
+        PeerTab t{};
+        t.rank = r;
+        t.nranks = P;
+        t.mine = sl.psync;
+        t.lo = r > 0 ? sync[r - 1] : nullptr;
+        t.hi = r < P - 1 ? sync[r + 1] : nullptr;
+        t.halo_to_lo = r > 0 ? pvec[r - 1] + plane + n : nullptr;
+        t.halo_to_hi = r < P - 1 ? pvec[r + 1] : nullptr;
+        for (int q = 0; q < P; ++q) t.all[q] = sync[q];
+        if (!sl.ptab) CHECK(alloc_zero((void **)&sl.ptab, sizeof(PeerTab)));
+        CU(cudaMemcpy(sl.ptab, &t, sizeof t, cudaMemcpyHostToDevice));
+    }
     return HPCCG_OK;
 }
 
@@ -1737,6 +1896,10 @@ int hpccg_set_option(hpccg_problem *p, int key, int64_t value) {
             return HPCCG_OK;
         case HPCCG_OPT_SMEM_SOLVE: p->opt_smem = value != 0; return HPCCG_OK;
         case HPCCG_OPT_FINISHER_FREE: p->opt_ff = value != 0; return HPCCG_OK;
+        case HPCCG_OPT_HALO_PEER:
+            if (value && p->ctx->mode != MODE_SINGLE && !p->slabs[0].ptab) CHECK(enable_peer(p));
+            p->opt_peer = value != 0;
+            return HPCCG_OK;
         case HPCCG_OPT_SMEM_THREADS:
             if (value != 0 && value != 256 && value != 512) return fail(HPCCG_EINVAL, "smem threads: 0, 256, 512");
             p->opt_smem_threads = (int)value;
@@ -1977,6 +2140,12 @@ int hpccg_solve(hpccg_problem *p, int max_iter, double tol, int *niters, double 
     CU(cudaStreamSynchronize(ctx->stream));
     CU(cudaGetLastError());
     l2win.release();
+    if (peer_on(p))
+        for (const Slab &sl : p->slabs) {
+            int perr = 0;
+            CU(cudaMemcpy(&perr, &sl.psync->error, sizeof perr, cudaMemcpyDeviceToHost));
+            if (perr) return fail(HPCCG_ECUDA, "peer-memory wait timed out (slab %d)", sl.rank);
+        }
 
     CgScalars hs;
     CU(cudaMemcpy(&hs, p->slabs[0].sc, sizeof hs, cudaMemcpyDeviceToHost));
@@ -2039,6 +2208,7 @@ void hpccg_free(hpccg_problem *p) {
     cudaStreamSynchronize(p->ctx->stream);
     if (p->graph) cudaGraphExecDestroy(p->graph);
     if (p->wgraph) cudaGraphExecDestroy(p->wgraph);
+    for (void *q : p->ipc_opened) cudaIpcCloseMemHandle(q);
     for (Slab &s : p->slabs) free_slab(s);
     cudaFree(p->d_tab);
     for (cudaEvent_t e : p->ev_pool) cudaEventDestroy(e);

@@ -1570,6 +1570,147 @@ __global__ void slab_allreduce_kernel(const double *const *src, double *const *d
     }
 }
 
+// ------------------------------- peer-memory z-slab exchange (HALO_PEER)
+// The multi-slab iteration's two collectives done by our own kernels over
+// peer memory (NVLink P2P on a multi-GPU node; sibling slabs' buffers in
+// loopback): the halo exchange is a PUSH -- each slab stores its first and
+// last owned planes straight into its neighbours' halo planes and then
+// signals them -- and each scalar allreduce is a POST of the local value into
+// slot [rank] of every peer followed by a COLLECT that waits for the P slots
+// and sums them in rank order (deterministic, bit-identical on every rank, and
+// bit-identical to the loopback allreduce kernel).  Counters advance in
+// lockstep on every slab (every slab runs every exchange and allreduce), so a
+// flag / tag is the count of the operation it completes.  Two slot sets
+// (count parity) suffice: a rank cannot post allreduce m + 2 before every rank
+// has collected m (it needs all ranks' m + 1 posts, made after their collect
+// of m).  Memory model: pushes / posts, then fence.sc.sys, then a st.release.sys
+// of the flag / tag; waits are ld.acquire.sys spins, bounded by a %globaltimer
+// timeout that records an error instead of hanging the GPU.
+
+constexpr int kMaxPeers = 64;
+
+struct PeerSync {                      // one per slab, in that slab's device memory
+    unsigned long long flag_from_lo;   // exchanges pushed to me by rank - 1
+    unsigned long long flag_from_hi;   //   ... by rank + 1
+    unsigned long long recv_count;     // exchanges I have waited for
+    unsigned long long push_count;     // exchanges I have pushed
+    unsigned long long ar_count;       // allreduces I have collected
+    unsigned long long ar_posted;      // allreduces I have posted
+    unsigned int push_ticket;          // blocks of the current push done
+    int error;                         // 1: a wait timed out
+    unsigned long long ar_tag[2][kMaxPeers];
+    double ar_val[2][kMaxPeers][2];
+};
+
+struct PeerTab {                       // device copy per slab; pointers may be peers'
+    int rank, nranks;
+    double *halo_to_lo;                // rank-1's upper halo plane (gets my first owned plane)
+    double *halo_to_hi;                // rank+1's lower halo plane (gets my last owned plane)
+    PeerSync *mine, *lo, *hi;
+    PeerSync *all[kMaxPeers];          // every rank's PeerSync (allreduce posts)
+};
+
+__device__ __forceinline__ void st_release_sys(unsigned long long *p, unsigned long long v) {
+    asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+
+__device__ __forceinline__ unsigned long long ld_acquire_sys(const unsigned long long *p) {
+    unsigned long long v;
+    asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+
+// spin until *flag >= target; false (and the error flag) after ~2 s
+__device__ __forceinline__ bool spin_until(const unsigned long long *flag, unsigned long long target,
+                                           PeerSync *mine) {
+    const unsigned long long t0 = gtimer();
+    while (ld_acquire_sys(flag) < target) {
+        if (gtimer() - t0 > 2000000000ull) {
+            mine->error = 1;
+            return false;
+        }
+        __nanosleep(64);
+    }
+    return true;
+}
+
+// a.2 push: my first owned plane -> rank-1's upper halo, my last owned plane
+// -> rank+1's lower halo (x = local-with-halo base); the last block signals.
+__global__ void __launch_bounds__(kBlock) halo_push_kernel(const PeerTab *t, const double *x, int64_t n,
+                                                         int64_t plane) {
+    const int64_t tid = gtid(), nth = gnth();
+    double *lo = t->halo_to_lo, *hi = t->halo_to_hi;
+    for (int64_t i = tid; i < 2 * plane; i += nth) {
+        if (i < plane) {
+            if (lo) lo[i] = x[plane + i];
+        } else if (hi) {
+            hi[i - plane] = x[n + (i - plane)];
+        }
+    }
+    __shared__ int last;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        __threadfence_system();  // my pushes before the ticket (and so before the flag)
+        const unsigned tk = atomicAdd(&t->mine->push_ticket, 1u);
+        last = (tk == gridDim.x - 1);
+    }
+    __syncthreads();
+    if (!last || threadIdx.x != 0) return;
+    __threadfence_system();
+    t->mine->push_ticket = 0u;
+    const unsigned long long c = t->mine->push_count + 1;
+    t->mine->push_count = c;
+    if (t->lo) st_release_sys(&t->lo->flag_from_hi, c);
+    if (t->hi) st_release_sys(&t->hi->flag_from_lo, c);
+}
+
+// a.2 wait: both neighbours have pushed this exchange (one thread).
+__global__ void halo_wait_kernel(const PeerTab *t) {
+    if (threadIdx.x != 0) return;
+    PeerSync *m = t->mine;
+    const unsigned long long target = m->recv_count + 1;
+    if (t->rank > 0 && !spin_until(&m->flag_from_lo, target, m)) return;
+    if (t->rank < t->nranks - 1 && !spin_until(&m->flag_from_hi, target, m)) return;
+    m->recv_count = target;
+}
+
+// a.4/a.5 allreduce over peer memory of `count` (<= 2) doubles: post (my
+// values into slot [rank] of every rank, then the tag) and / or collect (wait
+// for the P tags, sum in rank order -- or max -- into dst).  One warp.
+__global__ void peer_allreduce_kernel(const PeerTab *t, const double *src, double *dst, int count,
+                                      int is_max, int post, int collect) {
+    PeerSync *m = t->mine;
+    const int P = t->nranks, lane = threadIdx.x;
+    if (post) {
+        const unsigned long long c = m->ar_posted + 1;
+        const int q = (int)(c & 1);
+        for (int r = lane; r < P; r += 32) {
+            PeerSync *dstp = t->all[r];
+            for (int j = 0; j < count; ++j) dstp->ar_val[q][t->rank][j] = src[j];
+            __threadfence_system();
+            st_release_sys(&dstp->ar_tag[q][t->rank], c);
+        }
+        __syncwarp();
+        if (lane == 0) m->ar_posted = c;
+    }
+    if (collect) {
+        const unsigned long long c = m->ar_count + 1;
+        const int q = (int)(c & 1);
+        for (int r = lane; r < P; r += 32)
+            if (!spin_until(&m->ar_tag[q][r], c, m)) break;
+        __syncwarp();
+        if (lane == 0) {
+            __threadfence();
+            for (int j = 0; j < count; ++j) {
+                double s = m->ar_val[q][0][j];
+                for (int r = 1; r < P; ++r) s = is_max ? fmax(s, m->ar_val[q][r][j]) : s + m->ar_val[q][r][j];
+                dst[j] = s;
+            }
+            m->ar_count = c;
+        }
+    }
+}
+
 // ---------------------------------------------------------- a.10 BLAS-1
 
 // w = alpha x + beta y, canonical forms (A10).  form: 0 alpha==1, 1 beta==1,

@@ -684,3 +684,67 @@ def test_full_512cubed_sampled_and_properties(ctx):
         xl[plane:plane + n] = torch.from_numpy(p.get_vec(H.HPCCG_VEC_X)).cuda()
         p.spmv(xl, y)
         assert float(torch.linalg.norm(b - y)) <= 1e-13 * float(torch.linalg.norm(b))
+
+
+# ---------------------- peer-memory z-slab exchange (HPCCG_OPT_HALO_PEER)
+
+@pytest.mark.parametrize("variant", [0, 1])
+@pytest.mark.parametrize("P", [2, 3, 4])
+def test_peer_halo_and_allreduce_loopback_bitwise(P, variant):
+    """The halo push / wait kernels and the post / collect allreduce over peer
+    memory (sibling slabs in loopback) reproduce the copy-exchange +
+    loopback-allreduce path BIT FOR BIT (same rank-order sums), for HPCCG's CG
+    and the single-reduction variant, in the while-graph, the per-iteration
+    graph and plain timed launches; and match the global oracle."""
+    nx, ny, nz = 16, 12, 6
+    with H.Context(0, nranks=P, loopback=True) as c, H.Problem(c, nx, ny, nz) as p:
+        p.set_option(H.HPCCG_OPT_CG_VARIANT, variant)
+        outs = []
+        for peer, wh, timing in [(0, 1, 0), (1, 1, 0), (1, 0, 0), (1, 0, 1), (0, 0, 1)]:
+            p.set_option(H.HPCCG_OPT_HALO_PEER, peer)
+            p.set_option(H.HPCCG_OPT_WHILE, wh)
+            p.set_option(H.HPCCG_OPT_TIMING, timing)
+            p.set_vec(H.HPCCG_VEC_X, np.zeros(p.n * P))
+            r = p.solve(150, 1e-12)
+            outs.append((r["niters"], r["normr"], p.get_vec(H.HPCCG_VEC_X)))
+            if timing:
+                st = p.stats()
+                assert st["exchange_ms"] > 0 and st["allreduce_ms"] > 0
+        for o in outs[1:]:
+            assert o[:2] == outs[0][:2]
+            np.testing.assert_array_equal(o[2], outs[0][2])
+        ref = oracle.generate(nx, ny, nz * P)
+        oref = (oracle.cg_sr if variant else oracle.cg)(ref, 150, 1e-12)
+        assert abs(outs[0][0] - oref["niters"]) <= 1
+        assert np.max(np.abs(outs[0][2] - oref["x"])) <= CG_ATOL
+
+
+def test_peer_mode_max_iter_and_repeat_solves():
+    """Counters stay in lockstep across solves of different lengths (flags and
+    tags are operation counts, never reset)."""
+    P = 3
+    with H.Context(0, nranks=P, loopback=True) as c, H.Problem(c, 8, 8, 4) as p:
+        ref = oracle.generate(8, 8, 4 * P)
+        p.set_option(H.HPCCG_OPT_HALO_PEER, 1)
+        for m in [1, 2, 7, 3, 20]:
+            p.set_vec(H.HPCCG_VEC_X, np.zeros(p.n * P))
+            r = p.solve(m, 0.0)
+            o = oracle.cg(ref, m, 0.0)
+            assert r["niters"] == o["niters"] == m - 1
+            assert np.max(np.abs(p.get_vec(H.HPCCG_VEC_X) - o["x"])) <= CG_ATOL
+
+
+def test_peer_mode_nccl_one_rank():
+    """1-rank NCCL communicator with HALO_PEER: no neighbours (no pushes land
+    anywhere), the allreduce posts to its own slots and collects them."""
+    dims = (16, 12, 6)
+    uid = H.hpccg_unique_id()
+    with H.Context(0, rank=0, nranks=1, unique_id=uid) as c, H.Problem(c, *dims) as p:
+        p.set_option(H.HPCCG_OPT_HALO_PEER, 1)
+        ref = oracle.generate(*dims)
+        for variant in (0, 1):
+            p.set_option(H.HPCCG_OPT_CG_VARIANT, variant)
+            p.set_vec(H.HPCCG_VEC_X, np.zeros(p.n))
+            res = p.solve(150, 1e-12)
+            oref = (oracle.cg_sr if variant else oracle.cg)(ref, 150, 1e-12)
+            check_cg(res, p.maxabsdiff(), oref, ref)
