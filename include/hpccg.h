@@ -184,6 +184,31 @@ HPCCG_API int hpccg_init(hpccg_ctx **ctx, int device, void *cuda_stream, int ran
 HPCCG_API int hpccg_init_loopback(hpccg_ctx **ctx, int device, void *cuda_stream,
                         int nranks);
 
+/* Create a PEER-ONLY context: z-slab rank `rank` of `nranks`, one slab per
+ * process, NO NCCL.  The CG solve's halo exchange and scalar allreduces run
+ * as this library's kernels over peer memory (HPCCG_OPT_HALO_PEER) once the
+ * problem is attached to its peers: every rank calls hpccg_peer_export, the
+ * caller all-gathers the blobs (any transport, e.g. torch.distributed), and
+ * every rank calls hpccg_peer_attach with them.  Ranks may share one GPU
+ * (CUDA IPC within a device) or sit on NVLink peers.  Problem sizes are
+ * global by closed form (no collective): nnz_global = (3nx-2)(3ny-2)(3 nz
+ * nranks - 2).  hpccg_spmv / hpccg_ddot on caller-owned vectors need a
+ * transport and return HPCCG_ENOTSUP; hpccg_maxabsdiff works after attach. */
+HPCCG_API int hpccg_init_peer(hpccg_ctx **ctx, int device, void *cuda_stream, int rank, int nranks);
+
+#define HPCCG_PEER_BLOB_BYTES 256
+
+/* This rank's peer blob (HPCCG_PEER_BLOB_BYTES, host): CUDA IPC handles of its
+ * CG vector arena and its peer-sync block.  One slab per process (NCCL or
+ * peer-only contexts); not collective. */
+HPCCG_API int hpccg_peer_export(hpccg_problem *prob, void *blob);
+
+/* Map the peers' buffers from `blobs` (nranks x HPCCG_PEER_BLOB_BYTES, rank
+ * order, as exported) and switch HPCCG_OPT_HALO_PEER on.  Collective over the
+ * ranks in the sense that every rank must attach before any solves.  Once per
+ * problem; HPCCG_EINVAL if already attached. */
+HPCCG_API int hpccg_peer_attach(hpccg_problem *prob, const void *blobs);
+
 /* rank / nranks of the context; nslabs = slabs hosted by this process
  * (1, or nranks for loopback). */
 HPCCG_API int hpccg_ctx_info(const hpccg_ctx *ctx, int *rank, int *nranks, int *nslabs);

@@ -53,7 +53,7 @@ int fail(int code, const char *fmt, ...) {
         if (rc_ != HPCCG_OK) return rc_;   \
     } while (0)
 
-enum Mode { MODE_SINGLE = 0, MODE_NCCL = 1, MODE_LOOPBACK = 2 };
+enum Mode { MODE_SINGLE = 0, MODE_NCCL = 1, MODE_LOOPBACK = 2, MODE_PEER = 3 };
 enum Phase { PH_PUPDATE = 0, PH_SPMV, PH_UPDATE, PH_ALLREDUCE, PH_EXCHANGE, PH_N };
 
 int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
@@ -282,7 +282,7 @@ int allreduce_scalar(hpccg_ctx *ctx, double *const *h_src, double *const *h_dst,
 #endif
     (void)h_src;
     (void)h_dst;
-    return fail(HPCCG_ENOTSUP, "allreduce: no communicator");
+    return fail(HPCCG_ENOTSUP, "allreduce: no communicator (peer-only contexts reduce per problem)");
 }
 
 // a.2 halo exchange of a local-with-halo vector per slab (bases xs[s]):
@@ -314,6 +314,8 @@ int exchange(hpccg_problem *p, double *const *xs, cudaStream_t on) {
         }
         return HPCCG_OK;
     }
+    if (ctx->mode == MODE_PEER)
+        return fail(HPCCG_ENOTSUP, "peer-only context: no halo transport for caller-owned vectors");
 #ifdef HPCCG_WITH_NCCL
     const int r = ctx->rank, P = ctx->nranks;
     double *x = xs[0];
@@ -338,6 +340,7 @@ int exchange(hpccg_problem *p, double *const *xs, cudaStream_t on) {
 // HALO_PEER (multi-slab, opt_peer): the halo exchange as our own push /
 // wait kernels over peer memory (kernels.cuh "peer-memory z-slab exchange").
 bool peer_on(const hpccg_problem *p) { return p->opt_peer && p->ctx->mode != MODE_SINGLE; }
+bool one_slab_per_process(const hpccg_ctx *ctx) { return ctx->mode == MODE_NCCL || ctx->mode == MODE_PEER; }
 
 // push every hosted slab's boundary planes of x (local-with-halo bases xs)
 int halo_push(hpccg_problem *p, double *const *xs, cudaStream_t on) {
@@ -569,7 +572,7 @@ template <class F>
 int spmv_overlapped(hpccg_problem *p, bool timing, double *const *xs, F slab_spmv) {
     hpccg_ctx *ctx = p->ctx;
     const bool peer = peer_on(p);
-    if (ctx->mode == MODE_NCCL) {
+    if (one_slab_per_process(ctx)) {
         CU(cudaEventRecord(ctx->ev_fork, ctx->stream));
         CU(cudaStreamWaitEvent(ctx->comm_stream, ctx->ev_fork, 0));
         {
@@ -996,6 +999,11 @@ int enqueue_init_sr(hpccg_problem *p, int max_iter, double tol, bool timing,
             CHECK(check_launch(ctx));
         }
     }
+    // HALO_PEER: a push must not land before every neighbour has finished
+    // reading the previous exchange (the SpMV of A x just above); an allreduce
+    // is that barrier (every rank posts only after its SpMV) -- everywhere
+    // else in the solve one already separates consecutive exchanges
+    if (peer_on(p)) CHECK(allreduce_cg(p, true, timing));
     CHECK(cg_sr_spmv_all(p, timing, false, 0));
     for (size_t i = 0; i < p->slabs.size(); ++i) {
         const Slab &s = p->slabs[i];
@@ -1455,73 +1463,40 @@ int api_reduce(hpccg_ctx *ctx, bool is_max, double *result, L launch) {
     return HPCCG_OK;
 }
 
-// HALO_PEER setup (collective): every slab's PeerSync, and the peer tables.
-// Loopback: the neighbours' buffers are sibling slabs in this process.  NCCL
-// (one slab per rank, one GPU each): every rank exports its CG arena (which
-// holds the halo'd vector) and its PeerSync with cudaIpcGetMemHandle, the
-// handles are all-gathered over the library's communicator, and the peers'
-// buffers are mapped with cudaIpcOpenMemHandle (NVLink P2P); the arena layout
-// is identical on every rank, so a peer's vector is at the same offset.
-int enable_peer(hpccg_problem *p) {
-    hpccg_ctx *ctx = p->ctx;
-    const int P = ctx->nranks;
-    if (P > kMaxPeers) return fail(HPCCG_ENOTSUP, "peer mode supports up to %d ranks", kMaxPeers);
+// HALO_PEER setup: every slab's PeerSync, then the peer tables.  Loopback:
+// the neighbours' buffers are sibling slabs in this process.  One slab per
+// process (NCCL or peer-only contexts): every rank exports its CG arena (which
+// holds the halo'd vector) and its PeerSync as CUDA IPC handles (a "blob"),
+// the blobs are all-gathered (over NCCL inside the library, or by the caller
+// for peer-only contexts: hpccg_peer_export / hpccg_peer_attach) and the
+// peers' buffers are mapped with cudaIpcOpenMemHandle (NVLink P2P between
+// GPUs); the arena layout is identical on every rank, so a peer's vector sits
+// at the same offset.
+int peer_alloc(hpccg_problem *p) {
+    if (p->ctx->nranks > kMaxPeers) return fail(HPCCG_ENOTSUP, "peer mode supports up to %d ranks", kMaxPeers);
     for (Slab &sl : p->slabs)
         if (!sl.psync) CHECK(alloc_zero((void **)&sl.psync, sizeof(PeerSync)));
+    return HPCCG_OK;
+}
+
+int peer_export(hpccg_problem *p, unsigned char *blob) {
+    CHECK(peer_alloc(p));
     const Slab &s0 = p->slabs[0];
-    const int64_t n = s0.n, plane = s0.plane;
-    std::vector<PeerSync *> sync(P, nullptr);
-    std::vector<double *> pvec(P, nullptr);  // each rank's local-with-halo vector base
-    if (ctx->mode == MODE_LOOPBACK) {
-        for (int q = 0; q < P; ++q) {
-            sync[q] = p->slabs[q].psync;
-            pvec[q] = p->slabs[q].p;
-        }
-    } else if (ctx->mode == MODE_NCCL) {
-#ifdef HPCCG_WITH_NCCL
-        const int r = ctx->rank;
-        const size_t hb = sizeof(cudaIpcMemHandle_t);
-        std::vector<unsigned char> mine(2 * hb), all(2 * hb * P);
-        cudaIpcMemHandle_t h[2];
-        CU(cudaIpcGetMemHandle(&h[0], s0.arena));
-        CU(cudaIpcGetMemHandle(&h[1], s0.psync));
-        memcpy(mine.data(), h, 2 * hb);
-        unsigned char *d = nullptr;
-        CU(cudaMalloc((void **)&d, 2 * hb * (P + 1)));
-        CU(cudaMemcpy(d, mine.data(), 2 * hb, cudaMemcpyHostToDevice));
-        ncclResult_t nr = ncclAllGather(d, d + 2 * hb, 2 * hb, ncclUint8, ctx->comm, ctx->stream);
-        if (nr != ncclSuccess) {
-            cudaFree(d);
-            return nccl_fail(ctx, nr, "ncclAllGather(ipc handles)");
-        }
-        CU(cudaStreamSynchronize(ctx->stream));
-        CU(cudaMemcpy(all.data(), d + 2 * hb, 2 * hb * P, cudaMemcpyDeviceToHost));
-        cudaFree(d);
-        for (int q = 0; q < P; ++q) {
-            if (q == r) {
-                sync[q] = s0.psync;
-                pvec[q] = s0.p;
-                continue;
-            }
-            cudaIpcMemHandle_t hq[2];
-            memcpy(hq, all.data() + 2 * hb * q, 2 * hb);
-            void *ps = nullptr;
-            CU(cudaIpcOpenMemHandle(&ps, hq[1], cudaIpcMemLazyEnablePeerAccess));
-            p->ipc_opened.push_back(ps);
-            sync[q] = (PeerSync *)ps;
-            if (q == r - 1 || q == r + 1) {  // neighbours: their halo'd vector
-                void *pa = nullptr;
-                CU(cudaIpcOpenMemHandle(&pa, hq[0], cudaIpcMemLazyEnablePeerAccess));
-                p->ipc_opened.push_back(pa);
-                pvec[q] = (double *)pa + (s0.p - s0.arena);
-            }
-        }
-#else
-        return fail(HPCCG_ENOTSUP, "built without NCCL");
-#endif
-    } else {
-        return HPCCG_OK;  // single GPU: nothing to exchange
-    }
+    memset(blob, 0, HPCCG_PEER_BLOB_BYTES);
+    cudaIpcMemHandle_t h[2];
+    CU(cudaIpcGetMemHandle(&h[0], s0.arena));
+    CU(cudaIpcGetMemHandle(&h[1], s0.psync));
+    memcpy(blob, h, sizeof h);
+    return HPCCG_OK;
+}
+
+// sync[q] / pvec[q]: rank q's PeerSync and local-with-halo vector base (may
+// be null for non-neighbours' vectors) -> device tables of the hosted slabs
+int peer_build_tables(hpccg_problem *p, const std::vector<PeerSync *> &sync,
+                      const std::vector<double *> &pvec) {
+    hpccg_ctx *ctx = p->ctx;
+    const int P = ctx->nranks;
+    const int64_t n = p->slabs[0].n, plane = p->slabs[0].plane;
     for (size_t i = 0; i < p->slabs.size(); ++i) {
         Slab &sl = p->slabs[i];
         const int r = ctx->mode == MODE_LOOPBACK ? (int)i : ctx->rank;
@@ -1538,6 +1513,76 @@ int enable_peer(hpccg_problem *p) {
         CU(cudaMemcpy(sl.ptab, &t, sizeof t, cudaMemcpyHostToDevice));
     }
     return HPCCG_OK;
+}
+
+// blobs: nranks x HPCCG_PEER_BLOB_BYTES in rank order (one slab per process)
+int peer_attach(hpccg_problem *p, const unsigned char *blobs) {
+    hpccg_ctx *ctx = p->ctx;
+    CHECK(peer_alloc(p));
+    const int P = ctx->nranks, r = ctx->rank;
+    const Slab &s0 = p->slabs[0];
+    std::vector<PeerSync *> sync(P, nullptr);
+    std::vector<double *> pvec(P, nullptr);
+    for (int q = 0; q < P; ++q) {
+        if (q == r) {
+            sync[q] = s0.psync;
+            pvec[q] = s0.p;
+            continue;
+        }
+        cudaIpcMemHandle_t hq[2];
+        memcpy(hq, blobs + (size_t)HPCCG_PEER_BLOB_BYTES * q, sizeof hq);
+        void *ps = nullptr;
+        CU(cudaIpcOpenMemHandle(&ps, hq[1], cudaIpcMemLazyEnablePeerAccess));
+        p->ipc_opened.push_back(ps);
+        sync[q] = (PeerSync *)ps;
+        if (q == r - 1 || q == r + 1) {  // neighbours: their halo'd vector
+            void *pa = nullptr;
+            CU(cudaIpcOpenMemHandle(&pa, hq[0], cudaIpcMemLazyEnablePeerAccess));
+            p->ipc_opened.push_back(pa);
+            pvec[q] = (double *)pa + (s0.p - s0.arena);
+        }
+    }
+    return peer_build_tables(p, sync, pvec);
+}
+
+// HPCCG_OPT_HALO_PEER = 1 (collective): loopback and NCCL contexts build the
+// tables themselves; peer-only contexts are attached by the caller.
+int enable_peer(hpccg_problem *p) {
+    hpccg_ctx *ctx = p->ctx;
+    CHECK(peer_alloc(p));
+    const int P = ctx->nranks;
+    if (ctx->mode == MODE_LOOPBACK) {
+        std::vector<PeerSync *> sync(P);
+        std::vector<double *> pvec(P);
+        for (int q = 0; q < P; ++q) {
+            sync[q] = p->slabs[q].psync;
+            pvec[q] = p->slabs[q].p;
+        }
+        return peer_build_tables(p, sync, pvec);
+    }
+    if (ctx->mode == MODE_NCCL) {
+#ifdef HPCCG_WITH_NCCL
+        const size_t B = HPCCG_PEER_BLOB_BYTES;
+        std::vector<unsigned char> mine(B), all(B * P);
+        CHECK(peer_export(p, mine.data()));
+        unsigned char *d = nullptr;
+        CU(cudaMalloc((void **)&d, B * (P + 1)));
+        CU(cudaMemcpy(d, mine.data(), B, cudaMemcpyHostToDevice));
+        ncclResult_t nr = ncclAllGather(d, d + B, B, ncclUint8, ctx->comm, ctx->stream);
+        if (nr != ncclSuccess) {
+            cudaFree(d);
+            return nccl_fail(ctx, nr, "ncclAllGather(ipc handles)");
+        }
+        CU(cudaStreamSynchronize(ctx->stream));
+        CU(cudaMemcpy(all.data(), d + B, B * P, cudaMemcpyDeviceToHost));
+        cudaFree(d);
+        return peer_attach(p, all.data());
+#else
+        return fail(HPCCG_ENOTSUP, "built without NCCL");
+#endif
+    }
+    if (ctx->mode == MODE_PEER) return fail(HPCCG_EINVAL, "peer-only context: call hpccg_peer_attach");
+    return HPCCG_OK;  // single GPU: nothing to exchange
 }
 
 }  // namespace
@@ -1621,6 +1666,44 @@ int hpccg_init(hpccg_ctx **out, int device, void *stream, int rank, int nranks,
 #endif
     }
     *out = c;
+    return HPCCG_OK;
+}
+
+int hpccg_init_peer(hpccg_ctx **out, int device, void *stream, int rank, int nranks) {
+    if (!out || nranks < 1 || rank < 0 || rank >= nranks || nranks > kMaxPeers)
+        return fail(HPCCG_EINVAL, "hpccg_init_peer: bad rank/nranks");
+    *out = nullptr;
+    hpccg_ctx *c = new hpccg_ctx();
+    c->rank = rank;
+    c->nranks = nranks;
+    c->nslabs = 1;
+    c->mode = MODE_PEER;
+    int rc = ctx_common_init(c, device, stream);
+    if (rc != HPCCG_OK) {
+        hpccg_finalize(c);
+        return rc;
+    }
+    *out = c;
+    return HPCCG_OK;
+}
+
+int hpccg_peer_export(hpccg_problem *p, void *blob) {
+    if (!p || !blob) return fail(HPCCG_EINVAL, "NULL argument");
+    if (!one_slab_per_process(p->ctx)) return fail(HPCCG_EINVAL, "peer export: one slab per process only");
+    CU(cudaSetDevice(p->ctx->device));
+    return peer_export(p, (unsigned char *)blob);
+}
+
+int hpccg_peer_attach(hpccg_problem *p, const void *blobs) {
+    if (!p || !blobs) return fail(HPCCG_EINVAL, "NULL argument");
+    if (!one_slab_per_process(p->ctx)) return fail(HPCCG_EINVAL, "peer attach: one slab per process only");
+    if (p->slabs[0].ptab) return fail(HPCCG_EINVAL, "peer attach: already attached");
+    CU(cudaSetDevice(p->ctx->device));
+    CHECK(peer_attach(p, (const unsigned char *)blobs));
+    if (p->graph) cudaGraphExecDestroy(p->graph);
+    if (p->wgraph) cudaGraphExecDestroy(p->wgraph);
+    p->graph = p->wgraph = nullptr;
+    p->opt_peer = 1;
     return HPCCG_OK;
 }
 
@@ -1745,6 +1828,9 @@ int hpccg_generate(hpccg_ctx *ctx, int nx, int ny, int nz, hpccg_problem **out) 
         local += s.nnz;
     }
     p->nnz_global = local;
+    if (ctx->mode == MODE_PEER)  // no collective transport here: the closed form (pinned by the oracle)
+        p->nnz_global = (unsigned long long)(3LL * nx - 2) * (unsigned long long)(3LL * ny - 2) *
+                        (unsigned long long)(3LL * nz * ctx->nranks - 2);
 #ifdef HPCCG_WITH_NCCL
     if (ctx->mode == MODE_NCCL) {
         unsigned long long *d = nullptr;
@@ -2050,6 +2136,23 @@ int hpccg_maxabsdiff(hpccg_problem *p, double *result) {
     if (!p || !result) return fail(HPCCG_EINVAL, "NULL argument");
     hpccg_ctx *ctx = p->ctx;
     CU(cudaSetDevice(ctx->device));
+    if (ctx->mode == MODE_PEER) {  // local max, then the problem's peer allreduce (max)
+        if (!peer_on(p)) return fail(HPCCG_EINVAL, "peer-only context: call hpccg_peer_attach");
+        const Slab &sl = p->slabs[0];
+        const int g = std::min<int>(wave_grid(sl.n, wave(ctx, maxabsdiff_kernel)), (int)ctx->red_cap);
+        maxabsdiff_kernel<<<g, kBlock, 0, ctx->stream>>>(sl.n, sl.x, sl.xexact, ctx->red, &sl.sc->red_loc);
+        CHECK(check_launch(ctx));
+        double *src[1] = {&sl.sc->red_loc}, *dst[1] = {&sl.sc->red_out};
+        CHECK(peer_allreduce(p, src, dst, 1, true));
+        CU(cudaMemcpyAsync(ctx->h_pinned, &sl.sc->red_out, sizeof(double), cudaMemcpyDeviceToHost,
+                           ctx->stream));
+        CU(cudaStreamSynchronize(ctx->stream));
+        int perr = 0;
+        CU(cudaMemcpy(&perr, &sl.psync->error, sizeof perr, cudaMemcpyDeviceToHost));
+        if (perr) return fail(HPCCG_ECUDA, "peer-memory wait timed out");
+        *result = *(volatile double *)ctx->h_pinned;
+        return HPCCG_OK;
+    }
     return api_reduce(ctx, true, result, [&](int s, double *out) {
         const Slab &sl = p->slabs[s];
         const int g = std::min<int>(wave_grid(sl.n, wave(ctx, maxabsdiff_kernel)), (int)ctx->red_cap);
@@ -2063,6 +2166,8 @@ int hpccg_solve(hpccg_problem *p, int max_iter, double tol, int *niters, double 
                 double times[6]) {
     if (!p) return fail(HPCCG_EINVAL, "NULL problem");
     if (max_iter < 1 || !(tol >= 0.0)) return fail(HPCCG_EINVAL, "max_iter >= 1 and tol >= 0 required");
+    if (p->ctx->mode == MODE_PEER && !peer_on(p))
+        return fail(HPCCG_EINVAL, "peer-only context: call hpccg_peer_attach before solving");
     hpccg_ctx *ctx = p->ctx;
     CU(cudaSetDevice(ctx->device));
     const bool timing = p->opt_timing != 0;
@@ -2072,7 +2177,9 @@ int hpccg_solve(hpccg_problem *p, int max_iter, double tol, int *niters, double 
                              (p->opt_variant == 0 || smem_rows(p) > 0) &&
                              (p->opt_persist == 2 ||
                               (p->opt_persist == 1 && p->slabs[0].n <= p->opt_persist_rows));
-    bool use_while = !use_persist && use_graph && p->opt_while && ctx->mode != MODE_NCCL &&
+    // NCCL calls cannot live in a conditional graph body; with HALO_PEER the
+    // multi-GPU iteration is our own kernels only, so it can
+    bool use_while = !use_persist && use_graph && p->opt_while && (ctx->mode != MODE_NCCL || peer_on(p)) &&
                      !p->while_failed;
     p->ev_used = 0;
     p->timed.clear();

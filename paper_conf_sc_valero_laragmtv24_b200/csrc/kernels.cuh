@@ -1583,7 +1583,11 @@ __global__ void slab_allreduce_kernel(const double *const *src, double *const *d
 // flag / tag is the count of the operation it completes.  Two slot sets
 // (count parity) suffice: a rank cannot post allreduce m + 2 before every rank
 // has collected m (it needs all ranks' m + 1 posts, made after their collect
-// of m).  Memory model: pushes / posts, then fence.sc.sys, then a st.release.sys
+// of m).  A push overwrites the neighbour's halo with no handshake, so the
+// caller must separate consecutive exchanges by an allreduce (a rank posts
+// only after its boundary SpMV has read the previous halo): the CG iterations
+// do by construction, and the f2 init adds one between its two exchanges.
+// Memory model: pushes / posts, then fence.sc.sys, then a st.release.sys
 // of the flag / tag; waits are ld.acquire.sys spins, bounded by a %globaltimer
 // timeout that records an error instead of hanging the GPU.
 

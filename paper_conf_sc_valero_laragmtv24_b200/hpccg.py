@@ -71,6 +71,9 @@ _SIGS = {
     "hpccg_unique_id": ([_vp], _i),
     "hpccg_init": ([ctypes.POINTER(_vp), _i, _vp, _i, _i, _vp], _i),
     "hpccg_init_loopback": ([ctypes.POINTER(_vp), _i, _vp, _i], _i),
+    "hpccg_init_peer": ([ctypes.POINTER(_vp), _i, _vp, _i, _i], _i),
+    "hpccg_peer_export": ([_vp, _vp], _i),
+    "hpccg_peer_attach": ([_vp, _vp], _i),
     "hpccg_ctx_info": ([_vp, ctypes.POINTER(_i), ctypes.POINTER(_i), ctypes.POINTER(_i)], _i),
     "hpccg_finalize": ([_vp], None),
     "hpccg_generate": ([_vp, _i, _i, _i, ctypes.POINTER(_vp)], _i),
@@ -202,6 +205,31 @@ def hpccg_init_loopback(device: int = 0, stream: int | None = None, nranks: int 
     return h.value
 
 
+def hpccg_init_peer(device: int = 0, stream: int | None = None, rank: int = 0,
+                    nranks: int = 2) -> int:
+    h = _vp()
+    _check(lib().hpccg_init_peer(ctypes.byref(h), device, stream or None, rank, nranks),
+           "hpccg_init_peer")
+    return h.value
+
+
+HPCCG_PEER_BLOB_BYTES = 256
+
+
+def hpccg_peer_export(prob: int) -> bytes:
+    buf = ctypes.create_string_buffer(HPCCG_PEER_BLOB_BYTES)
+    _check(lib().hpccg_peer_export(prob, buf), "hpccg_peer_export")
+    return buf.raw
+
+
+def hpccg_peer_attach(prob: int, blobs) -> None:
+    data = b"".join(bytes(b) for b in blobs)
+    if any(len(b) != HPCCG_PEER_BLOB_BYTES for b in blobs):
+        raise ValueError("peer blobs must be %d bytes each" % HPCCG_PEER_BLOB_BYTES)
+    buf = ctypes.create_string_buffer(data, len(data))
+    _check(lib().hpccg_peer_attach(prob, buf), "hpccg_peer_attach")
+
+
 def hpccg_finalize(ctx: int) -> None:
     lib().hpccg_finalize(ctx)
 
@@ -287,9 +315,12 @@ class Context:
     """A device + stream + communicator (single GPU, NCCL rank, or loopback)."""
 
     def __init__(self, device: int = 0, stream: int | None = None, rank: int = 0,
-                 nranks: int = 1, unique_id: bytes | None = None, loopback: bool = False):
+                 nranks: int = 1, unique_id: bytes | None = None, loopback: bool = False,
+                 peer: bool = False):
         if loopback:
             self.handle = hpccg_init_loopback(device, stream, nranks)
+        elif peer:      # peer-only (no NCCL): attach problems with peer_export / peer_attach
+            self.handle = hpccg_init_peer(device, stream, rank, nranks)
         else:
             self.handle = hpccg_init(device, stream, rank, nranks, unique_id)
         r, n, s = ctypes.c_int(), ctypes.c_int(), ctypes.c_int()
@@ -358,6 +389,14 @@ class Problem:
 
     def maxabsdiff(self) -> float:
         return hpccg_maxabsdiff(self.handle)
+
+    def peer_export(self) -> bytes:
+        """This rank's CUDA-IPC blob (one slab per process)."""
+        return hpccg_peer_export(self.handle)
+
+    def peer_attach(self, blobs) -> None:
+        """Map every rank's blob (rank order) and switch HALO_PEER on."""
+        hpccg_peer_attach(self.handle, blobs)
 
     def trace(self, k: int) -> np.ndarray:
         """[k, 3, 2] uint64 ns: (start, end) of p update / SpMV / update per iteration."""

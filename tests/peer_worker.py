@@ -1,0 +1,30 @@
+"""Child-process body of tests/test_gpu_peer_ipc.py (not a test module).
+
+One z-slab rank in its own process on GPU 0, in a PEER-ONLY context (no
+NCCL): export the CUDA-IPC blob, receive every rank's blob from the parent,
+attach, solve, and report.  Ranks on one GPU exercise the real multi-process
+path of HPCCG_OPT_HALO_PEER -- IPC export / open, peer tables, cross-process
+flags and allreduce slots -- that NCCL cannot (it refuses two ranks on one
+GPU)."""
+
+
+def run(rank, nranks, dims, variant, max_iter, tol, to_parent, from_parent):
+    try:
+        import numpy as np
+        from paper_conf_sc_valero_laragmtv24_b200 import hpccg as H
+        with H.Context(0, rank=rank, nranks=nranks, peer=True) as c, H.Problem(c, *dims) as p:
+            p.set_option(H.HPCCG_OPT_CG_VARIANT, variant)
+            to_parent.put(("blob", rank, p.peer_export()))
+            blobs = from_parent.get(timeout=120)
+            p.peer_attach(blobs)
+            out = []
+            for wh in (1, 0):
+                p.set_option(H.HPCCG_OPT_WHILE, wh)
+                p.set_vec(H.HPCCG_VEC_X, np.zeros(p.n))
+                r = p.solve(max_iter, tol)
+                out.append({"niters": r["niters"], "normr": r["normr"], "err": p.maxabsdiff(),
+                            "x": p.get_vec(H.HPCCG_VEC_X), "mode": p.stats()["graph_mode"],
+                            "nnz_global": p.info["nnz_global"]})
+            to_parent.put(("done", rank, out))
+    except Exception as e:  # reported to the parent, which fails the test
+        to_parent.put(("error", rank, repr(e)))

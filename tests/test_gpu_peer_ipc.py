@@ -1,0 +1,81 @@
+"""Two z-slab ranks as two PROCESSES on one GPU, peer-only contexts: the
+multi-process HALO_PEER path (CUDA IPC export / open, neighbour halo pushes
+and allreduce posts into another process's memory, release/acquire flags)
+against the global oracle and bit-for-bit against the same decomposition in
+one process (loopback + HALO_PEER, whose reduction order it shares)."""
+import multiprocessing as mp
+
+import numpy as np
+import pytest
+
+import oracle
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+
+from paper_conf_sc_valero_laragmtv24_b200 import hpccg as H  # noqa: E402
+
+
+def run_ranks(nranks, dims, variant, max_iter, tol, timeout=240):
+    import peer_worker
+    ctx = mp.get_context("spawn")
+    to_parent = ctx.Queue()
+    inbox = [ctx.Queue() for _ in range(nranks)]
+    procs = [ctx.Process(target=peer_worker.run,
+                         args=(r, nranks, dims, variant, max_iter, tol, to_parent, inbox[r]))
+             for r in range(nranks)]
+    for pr in procs:
+        pr.start()
+    try:
+        blobs, done = {}, {}
+        while len(blobs) < nranks:
+            kind, r, payload = to_parent.get(timeout=timeout)
+            assert kind == "blob", payload
+            blobs[r] = payload
+        for q in inbox:
+            q.put([blobs[r] for r in range(nranks)])
+        while len(done) < nranks:
+            kind, r, payload = to_parent.get(timeout=timeout)
+            assert kind == "done", payload
+            done[r] = payload
+        return [done[r] for r in range(nranks)]
+    finally:
+        for pr in procs:
+            pr.join(timeout=30)
+            if pr.is_alive():
+                pr.kill()
+
+
+@pytest.mark.parametrize("variant", [0, 1])
+def test_two_processes_one_gpu_peer_cg(variant):
+    P, dims = 2, (16, 12, 6)
+    res = run_ranks(P, dims, variant, 150, 1e-12)
+    ref = oracle.generate(dims[0], dims[1], dims[2] * P)
+    oref = (oracle.cg_sr if variant else oracle.cg)(ref, 150, 1e-12)
+    with H.Context(0, nranks=P, loopback=True) as c, H.Problem(c, *dims) as p:
+        p.set_option(H.HPCCG_OPT_CG_VARIANT, variant)
+        p.set_option(H.HPCCG_OPT_HALO_PEER, 1)
+        rl = p.solve(150, 1e-12)
+        xl = p.get_vec(H.HPCCG_VEC_X)
+    for k in range(2):                       # while-graph, per-iteration graph
+        outs = [res[r][k] for r in range(P)]
+        assert outs[0]["mode"] == (2 if k == 0 else 1)
+        assert outs[0]["nnz_global"] == ref.nnz
+        x = np.concatenate([o["x"] for o in outs])
+        for o in outs:                       # every rank took the same decisions
+            assert (o["niters"], o["normr"]) == (rl["niters"], rl["normr"])
+            assert o["err"] == outs[0]["err"]
+        np.testing.assert_array_equal(x, xl)
+        assert abs(outs[0]["niters"] - oref["niters"]) <= 1
+        assert np.max(np.abs(x - oref["x"])) <= 1e-10
+
+
+def test_three_processes_fixed_iterations():
+    P, dims = 3, (8, 8, 4)
+    res = run_ranks(P, dims, 0, 12, 0.0)
+    ref = oracle.generate(8, 8, 4 * P)
+    oref = oracle.cg(ref, 12, 0.0)
+    x = np.concatenate([res[r][0]["x"] for r in range(P)])
+    assert all(res[r][0]["niters"] == 11 for r in range(P))
+    assert np.max(np.abs(x - oref["x"])) <= 1e-10
