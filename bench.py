@@ -213,8 +213,19 @@ def run_ours(args, nx, ny, nz, iters, cfg_index, scaling):
     prob.set_option(H.HPCCG_OPT_GRAPH, 1)
     sr = args.cg_variant == "sr"
     prob.set_option(H.HPCCG_OPT_CG_VARIANT, 1 if sr else 0)
-    if args.halo == "peer":   # collective: every rank maps its neighbours' buffers (CUDA IPC)
-        prob.set_option(H.HPCCG_OPT_HALO_PEER, 1)
+    halo = "none (1 slab)"
+    if world > 1:
+        halo = "NCCL send/recv + ncclAllReduce"
+        if args.halo in ("peer", "auto"):
+            # collective: every rank maps its neighbours' buffers (CUDA IPC over NVLink);
+            # auto falls back to NCCL if the mapping is refused
+            try:
+                prob.set_option(H.HPCCG_OPT_HALO_PEER, 1)
+                halo = "peer-memory push + post/collect allreduce kernels (while-graph)"
+            except H.HpccgError as e:
+                if args.halo == "peer":
+                    raise
+                halo = "NCCL (peer mapping refused: %s)" % e
     xptr = prob.vec_ptr(H.HPCCG_VEC_X)
 
     def barrier():
@@ -341,8 +352,7 @@ def run_ours(args, nx, ny, nz, iters, cfg_index, scaling):
                        "global_rows": n * world, "global_nnz": nnz_global,
                        "parallelism": f"zslab{world}",
                        "cg_variant": "single-reduction (Chronopoulos-Gear, f2)" if sr else "HPCCG",
-                       "halo": ("peer-memory push + post/collect allreduce kernels" if args.halo == "peer"
-                                else "NCCL send/recv + ncclAllReduce") if world > 1 else "none (1 slab)",
+                       "halo": halo,
                        "solve_graph": {5: "on-chip cluster kernel", 4: "one-cluster persistent kernel",
                                        3: "cooperative persistent kernel", 2: "while-graph",
                                        1: "per-iteration graph", 0: "plain"}.get(
@@ -631,8 +641,9 @@ def main():
     ap.add_argument("--tri-n", type=int, default=100_000_000, help="tridiag SIZE (P:L475)")
     ap.add_argument("--lbm-size", type=int, default=1000, help="LBM SIZE (P:L411)")
     ap.add_argument("--iters", type=int, default=None, help="override CG iterations per step")
-    ap.add_argument("--halo", choices=["nccl", "peer"], default="nccl",
-                    help="multi-GPU exchange: NCCL (default) or our peer-memory kernels (HALO_PEER)")
+    ap.add_argument("--halo", choices=["auto", "nccl", "peer"], default="auto",
+                    help="multi-GPU exchange: our peer-memory kernels (HALO_PEER; auto falls back "
+                         "to NCCL if CUDA IPC is refused) or NCCL")
     ap.add_argument("--cg-variant", choices=["hpccg", "sr"], default="hpccg",
                     help="hpccg: HPCCG's CG (default); sr: single-reduction CG (SURVEY f2)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
