@@ -127,7 +127,10 @@ extern "C" {
                                global-memory barrier */
 #define HPCCG_OPT_PDL 11    /* 1 (default): single GPU, launch the CG kernels with
                                programmatic dependent launch (the SpMV starts its matrix
-                               stream while the p update drains); 0: off */
+                               stream while the p update drains; the SpMV lets the x/r update
+                               be scheduled right after its own dependency wait, so the update
+                               prefetches x, r, p during the SpMV's tail); 2: PDL with the
+                               SpMV triggering only after its rows; 0: off */
 #define HPCCG_OPT_VEC_WAVES 6 /* CG vector kernels: 0 one thread per 16-B unit; k > 0
                                (default 1): a persistent grid of k resident waves */
 

@@ -122,6 +122,7 @@ struct Slab {
     double *sv = nullptr;  // f2 single-reduction CG: s = A p recurrence vector (n)
     PeerSync *psync = nullptr;  // HALO_PEER: this slab's flags / allreduce slots
     PeerTab *ptab = nullptr;    // HALO_PEER: device copy of the peer table
+    int early_trigger = 1;      // HPCCG_OPT_PDL 1: SpMV triggers its successor early
 };
 
 struct TimedOp {
@@ -408,6 +409,7 @@ SpmvArgs spmv_args(const Slab &s, const double *x, double *y) {
     a.y = y;
     a.sc = s.sc;
     a.red = s.red;
+    a.early_trigger = s.early_trigger;
     return a;
 }
 
@@ -1975,7 +1977,11 @@ int hpccg_set_option(hpccg_problem *p, int key, int64_t value) {
             return HPCCG_OK;
         case HPCCG_OPT_WHILE: p->opt_while = value != 0; return HPCCG_OK;
         case HPCCG_OPT_L2_PERSIST: p->opt_l2 = value != 0; return HPCCG_OK;
-        case HPCCG_OPT_PDL: p->opt_pdl = value != 0; return HPCCG_OK;
+        case HPCCG_OPT_PDL:
+            if (value < 0 || value > 2) return fail(HPCCG_EINVAL, "pdl: 0, 1 or 2");
+            p->opt_pdl = value != 0;
+            for (Slab &sl : p->slabs) sl.early_trigger = value == 1;
+            return HPCCG_OK;
         case HPCCG_OPT_PERSISTENT:
             if (value < 0 || value > 2) return fail(HPCCG_EINVAL, "persistent: 0, 1 or 2");
             p->opt_persist = (int)value;

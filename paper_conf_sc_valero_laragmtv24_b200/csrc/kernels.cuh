@@ -268,6 +268,9 @@ struct SpmvArgs {
     TraceSlot *trace;  // HPCCG_OPT_TRACE (nullptr: off)
     int trace_max;
     int sr_q;          // kDots 2: parity of the iteration (run flag run_q[sr_q])
+    int early_trigger; // PDL: let the successor be scheduled right after pdl_wait
+                       // (it may then prefetch its inputs that this grid does not
+                       // write during this grid's tail); 0: after the rows
 };
 
 template <int kDots, bool kCheck>
@@ -353,6 +356,7 @@ __global__ void __launch_bounds__(kBlock, kMinB) spmv27_kernel(SpmvArgs a) {
             }
             if (g == 0) {
                 pdl_wait();
+                if (a.early_trigger) pdl_trigger();
                 if (kDot && a.trace) trace_mark(a.trace, a.trace_max, __ldg(&a.sc->k), 1, false);
                 done = spmv_done<kDots, kCheck>(a);
                 if (done) return;  // uniform over the grid, before any store
@@ -379,7 +383,7 @@ __global__ void __launch_bounds__(kBlock, kMinB) spmv27_kernel(SpmvArgs a) {
         pdl_wait();
         done = spmv_done<kDots, kCheck>(a);
     }
-    pdl_trigger();
+    pdl_trigger();  // (a second launch_dependents after an early one is a no-op)
     if (done) return;
     if (kDots == 2) {
         spmv_sr_partials(a, dg, d);
@@ -440,6 +444,7 @@ __global__ void __launch_bounds__(kBlock, 4) spmv27x2_kernel(SpmvArgs a) {
             }
             if (g == 0) {
                 pdl_wait();
+                if (a.early_trigger) pdl_trigger();
                 if (kDot && a.trace) trace_mark(a.trace, a.trace_max, __ldg(&a.sc->k), 1, false);
                 done = spmv_done<kDots, kCheck>(a);
                 if (done) return;  // uniform over the grid, before any store
@@ -484,7 +489,7 @@ __global__ void __launch_bounds__(kBlock, 4) spmv27x2_kernel(SpmvArgs a) {
         pdl_wait();
         done = spmv_done<kDots, kCheck>(a);
     }
-    pdl_trigger();
+    pdl_trigger();  // (a second launch_dependents after an early one is a no-op)
     if (done) return;
     if (kDots == 2) {
         spmv_sr_partials(a, dg, d);
@@ -863,15 +868,13 @@ template <int kU>
 __global__ void __launch_bounds__(kBlock) cg_update1_kernel(Upd1Args a) {
     __shared__ double sh[33];
     CgScalars *sc = a.sc;
-    pdl_wait();
-    pdl_trigger();
     const int64_t tid = gtid(), nth = gnth(), nv = a.n >> 1;
     double2 *__restrict__ x2 = reinterpret_cast<double2 *>(a.x);
     double2 *__restrict__ r2 = reinterpret_cast<double2 *>(a.r);
     const double2 *__restrict__ p2 = reinterpret_cast<const double2 *>(a.p);
     const double2 *__restrict__ q2 = reinterpret_cast<const double2 *>(a.Ap);
     double2 xa[kU], ra[kU], pa[kU], qa[kU];
-    auto load = [&](int64_t b) {
+    auto load_xrp = [&](int64_t b) {
 #pragma unroll
         for (int u = 0; u < kU; ++u) {
             const int64_t i = b + u * nth;
@@ -879,11 +882,27 @@ __global__ void __launch_bounds__(kBlock) cg_update1_kernel(Upd1Args a) {
                 xa[u] = x2[i];
                 ra[u] = r2[i];
                 pa[u] = p2[i];
-                qa[u] = q2[i];
             }
         }
     };
-    load(tid);
+    auto load_q = [&](int64_t b) {
+#pragma unroll
+        for (int u = 0; u < kU; ++u) {
+            const int64_t i = b + u * nth;
+            if (i < nv) qa[u] = q2[i];
+        }
+    };
+    auto load = [&](int64_t b) {
+        load_xrp(b);
+        load_q(b);
+    };
+    // x, r (previous update) and p (p update) are complete before the SpMV's
+    // blocks pass their pdl_wait, so before this grid can launch: read them
+    // during the SpMV's tail; Ap only after the SpMV has completed
+    load_xrp(tid);
+    pdl_wait();
+    pdl_trigger();
+    load_q(tid);
     if (!run_check(sc, a.q)) return;
     const int ktr = a.trace ? __ldg(&sc->niters) : 0;
     trace_mark(a.trace, a.trace_max, ktr, 2, false);
