@@ -848,7 +848,7 @@ int cg_sr_spmv_all(hpccg_problem *p, bool timing, bool check, int q) {
     auto finish = [&](const Slab &s, unsigned np, double *out) {
         cudaLaunchConfig_t cfg{};
         cfg.gridDim = dim3(1);
-        cfg.blockDim = dim3(kBlock);
+        cfg.blockDim = dim3(1024);
         cfg.stream = ctx->stream;
         cudaLaunchAttribute at[1];
         at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;

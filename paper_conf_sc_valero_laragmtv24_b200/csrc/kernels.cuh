@@ -772,8 +772,18 @@ struct Pupd1Args {
 // Fixed-order sum of n partials (the order of grid_reduce's last block);
 // identical in every block.
 __device__ __forceinline__ double sum_parts_fixed(const double *parts, unsigned n, double *sh) {
+    // the same left-to-right order per thread as the finisher, with 8 loads
+    // in flight per batch instead of a dependent chain
     double s = 0.0;
-    for (unsigned i = threadIdx.x; i < n; i += kBlock) s += __ldg(parts + i);
+    unsigned i = threadIdx.x;
+    for (; i + 7u * kBlock < n; i += 8u * kBlock) {
+        double v[8];
+#pragma unroll
+        for (int u = 0; u < 8; ++u) v[u] = __ldg(parts + i + u * kBlock);
+#pragma unroll
+        for (int u = 0; u < 8; ++u) s += v[u];
+    }
+    for (; i < n; i += kBlock) s += __ldg(parts + i);
     s = block_reduce<false>(s, sh);
     if (threadIdx.x == 0) sh[32] = s;
     __syncthreads();
@@ -794,23 +804,34 @@ template <int kU>
 __global__ void __launch_bounds__(kBlock) cg_pupdate1_kernel(Pupd1Args a) {
     __shared__ double sh[33];
     CgScalars *sc = a.sc;
-    pdl_wait();
-    pdl_trigger();
     const int64_t tid = gtid(), nth = gnth(), nv = a.n >> 1;
     const double2 *__restrict__ r2 = reinterpret_cast<const double2 *>(a.r);
     double2 *__restrict__ p2 = reinterpret_cast<double2 *>(a.p);
     double2 ra[kU], pa[kU];
-    auto load = [&](int64_t b) {
+    auto load_p = [&](int64_t b) {
 #pragma unroll
         for (int u = 0; u < kU; ++u) {
             const int64_t i = b + u * nth;
-            if (i < nv) {
-                ra[u] = r2[i];
-                pa[u] = p2[i];
-            }
+            if (i < nv) pa[u] = p2[i];
         }
     };
-    load(tid);
+    auto load_r = [&](int64_t b) {
+#pragma unroll
+        for (int u = 0; u < kU; ++u) {
+            const int64_t i = b + u * nth;
+            if (i < nv) ra[u] = r2[i];
+        }
+    };
+    auto load = [&](int64_t b) {
+        load_r(b);
+        load_p(b);
+    };
+    // p (this kernel's own output one iteration ago) is complete before the
+    // update's blocks pass their wait: read it during the update's tail
+    load_p(tid);
+    pdl_wait();
+    pdl_trigger();
+    load_r(tid);
     if (!run_check(sc, a.q)) return;
     const int k = __ldg(&sc->k);
     trace_mark(a.trace, a.trace_max, k, 0, false);
@@ -1026,7 +1047,21 @@ struct SrUpdArgs {
 // Fixed-order sums of the (gamma, delta) partials, identical in every block.
 __device__ __forceinline__ double2 sr_sum_parts(const double *parts, unsigned np, double *sh) {
     double g = 0.0, d = 0.0;
-    for (unsigned i = threadIdx.x; i < np; i += kBlock) {
+    unsigned i = threadIdx.x;
+    for (; i + 3u * kBlock < np; i += 4u * kBlock) {  // 8 loads in flight
+        double vg[4], vd[4];
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+            vg[u] = __ldg(parts + i + u * kBlock);
+            vd[u] = __ldg(parts + np + i + u * kBlock);
+        }
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+            g += vg[u];
+            d += vd[u];
+        }
+    }
+    for (; i < np; i += kBlock) {
         g += __ldg(parts + i);
         d += __ldg(parts + np + i);
     }
@@ -1042,15 +1077,40 @@ __device__ __forceinline__ double2 sr_sum_parts(const double *parts, unsigned np
 
 // (gamma, delta) partials of one slab -> out[0..1] (one block, fixed order):
 // multi-slab (allreduce input) or a single slab with > kUpdSumMax partials.
-__global__ void __launch_bounds__(kBlock) cg_sr_finish_kernel(const double *parts, unsigned n_parts,
-                                                              double *out) {
+// 1024 threads, 8 loads in flight per thread (65536 partials at 256^3).
+__global__ void __launch_bounds__(1024) cg_sr_finish_kernel(const double *parts, unsigned n_parts,
+                                                            double *out) {
     pdl_wait();
     pdl_trigger();
-    __shared__ double sh[66];
-    const double2 t = sr_sum_parts(parts, n_parts, sh);
-    if (threadIdx.x == 0) {
-        out[0] = t.x;
-        out[1] = t.y;
+    __shared__ double sh[64];
+    double g[4] = {0.0, 0.0, 0.0, 0.0}, d[4] = {0.0, 0.0, 0.0, 0.0};
+    unsigned i = threadIdx.x;
+    for (; i + 3u * 1024u < n_parts; i += 4u * 1024u) {
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+            g[u] += __ldcg(parts + i + u * 1024u);
+            d[u] += __ldcg(parts + n_parts + i + u * 1024u);
+        }
+    }
+    for (; i < n_parts; i += 1024u) {
+        g[0] += __ldcg(parts + i);
+        d[0] += __ldcg(parts + n_parts + i);
+    }
+    double gs = (g[0] + g[1]) + (g[2] + g[3]), ds = (d[0] + d[1]) + (d[2] + d[3]);
+    gs = warp_sum(gs);
+    ds = warp_sum(ds);
+    if ((threadIdx.x & 31) == 0) {
+        sh[threadIdx.x >> 5] = gs;
+        sh[32 + (threadIdx.x >> 5)] = ds;
+    }
+    __syncthreads();
+    if (threadIdx.x < 32) {
+        gs = warp_sum(sh[threadIdx.x]);
+        ds = warp_sum(sh[32 + threadIdx.x]);
+        if (threadIdx.x == 0) {
+            out[0] = gs;
+            out[1] = ds;
+        }
     }
 }
 
@@ -1058,6 +1118,21 @@ template <bool kVec, int kU>
 __global__ void __launch_bounds__(kBlock) cg_sr_update_kernel(SrUpdArgs a) {
     CgScalars *sc = a.sc;
     const int q = a.q, qp = q ^ 1;
+    // r, p, s, x were written by the previous update, complete before the
+    // SpMV's blocks passed their wait: warm L2/L1 with the first trip while
+    // the SpMV drains (w, the SpMV's output, only after the wait)
+    if (kVec) {
+        const int64_t nv0 = a.n >> 1;
+        for (int u = 0; u < kU; ++u) {
+            const int64_t i = gtid() + u * gnth();
+            if (i < nv0) {
+                asm volatile("prefetch.global.L2 [%0];" ::"l"(a.r + 2 * i));
+                asm volatile("prefetch.global.L2 [%0];" ::"l"(a.x + 2 * i));
+                asm volatile("prefetch.global.L2 [%0];" ::"l"(a.p + 2 * i));
+                asm volatile("prefetch.global.L2 [%0];" ::"l"(a.s + 2 * i));
+            }
+        }
+    }
     pdl_wait();
     pdl_trigger();
     if (!__ldg(&sc->run_q[qp])) {  // iteration k does not run (uniform) ...
