@@ -17,7 +17,11 @@ __constant__ double kLbmCy[9] = {0, 0, 1, 0, -1, 1, 1, -1, -1};
 __constant__ double kLbmW[9] = {4.0 / 9, 1.0 / 9, 1.0 / 9, 1.0 / 9, 1.0 / 9,
                                 1.0 / 36, 1.0 / 36, 1.0 / 36, 1.0 / 36};
 
-template <bool kWriteF>
+// kPol: cache policy of the lattice streams -- 0: loads and stores
+// streaming (evict-first); 1 (default): loads streaming, stores cached (the
+// lattice just written, 72 MB at 1000^2, stays largely in the 126 MB L2 for
+// the next step's pulls: 26.7 vs 29.3 us/step measured); 2: both cached.
+template <bool kWriteF, int kPol>
 __global__ void __launch_bounds__(kBlock) lbm_pull_kernel(int S, const double *__restrict__ f1,
                                                          double *__restrict__ f,
                                                          double *__restrict__ f2, double tau) {
@@ -25,13 +29,18 @@ __global__ void __launch_bounds__(kBlock) lbm_pull_kernel(int S, const double *_
     const int64_t SS = (int64_t)S * S;
     const int x = 1 + (int)blockIdx.y;
     const int y = 1 + (int)(blockIdx.x * kBlock + threadIdx.x);
+    // PDL: this step's blocks are scheduled during the previous step's tail
+    // and wait here until it has completed (every pull may read its output)
+    pdl_wait();
+    pdl_trigger();
     if (y > S - 2) return;
     const int64_t site = (int64_t)x * S + y;
     double fk[9];
 #pragma unroll
     for (int k = 0; k < 9; ++k) {
         const int xs = x - (int)kLbmCx[k], ys = y - (int)kLbmCy[k];
-        fk[k] = __ldcs(f1 + k * SS + (int64_t)xs * S + ys);
+        const double *src = f1 + k * SS + (int64_t)xs * S + ys;
+        fk[k] = kPol == 2 ? __ldg(src) : __ldcs(src);
     }
     if (kWriteF) {
 #pragma unroll
@@ -55,7 +64,9 @@ __global__ void __launch_bounds__(kBlock) lbm_pull_kernel(int S, const double *_
         t = __dadd_rn(t, __dmul_rn(__dmul_rn(4.5, cu), cu));
         t = __dsub_rn(t, __dmul_rn(1.5, usq));
         const double feq = __dmul_rn(__dmul_rn(kLbmW[k], p), t);
-        __stcs(f2 + k * SS + site, __dadd_rn(__dmul_rn(fk[k], keep), __ddiv_rn(feq, tau)));
+        const double out = __dadd_rn(__dmul_rn(fk[k], keep), __ddiv_rn(feq, tau));
+        if (kPol == 0) __stcs(f2 + k * SS + site, out);
+        else f2[k * SS + site] = out;
     }
 }
 
