@@ -56,7 +56,19 @@ def peaks():
 
 
 class ClockSampler:
-    """nvidia-smi clocks + throttle reasons sampled during the timed region."""
+    """SM clock + throttle reasons sampled DURING the timed region: NVML polled
+    every 5 ms from a thread (short regions still get samples), else
+    `nvidia-smi -lms 100` filtered to samples with the GPU busy."""
+
+    def __new__(cls, index: int):
+        if cls is ClockSampler:
+            try:
+                import pynvml
+                pynvml.nvmlInit()
+                return super().__new__(NvmlClockSampler)
+            except Exception:
+                pass
+        return super().__new__(cls)
     Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
          "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
          "clocks_event_reasons.sw_power_cap,utilization.gpu")
@@ -107,6 +119,44 @@ class ClockSampler:
                         reasons.add(nm)
         return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": mx,
                 "reasons": sorted(reasons), "samples": len(sm)}
+
+
+class NvmlClockSampler(ClockSampler):
+    REASONS = {"hw_slowdown": 0x8, "sw_thermal_slowdown": 0x20, "hw_thermal_slowdown": 0x40,
+               "sw_power_cap": 0x4}
+
+    def __init__(self, index: int):
+        self.index, self.samples, self.stop = index, [], None
+
+    def __enter__(self):
+        import pynvml
+        self.nv = pynvml
+        self.h = pynvml.nvmlDeviceGetHandleByIndex(self.index)
+        self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+        self.stop = threading.Event()
+
+        def poll():
+            while not self.stop.is_set():
+                try:
+                    mhz = self.nv.nvmlDeviceGetClockInfo(self.h, self.nv.NVML_CLOCK_SM)
+                    rs = self.nv.nvmlDeviceGetCurrentClocksThrottleReasons(self.h)
+                    self.samples.append((mhz, rs))
+                except Exception:
+                    pass
+                time.sleep(0.005)
+        self.t = threading.Thread(target=poll, daemon=True)
+        self.t.start()
+        return self
+
+    def __exit__(self, *a):
+        self.stop.set()
+        self.t.join(timeout=2)
+
+    def summary(self):
+        reasons = sorted({nm for _, rs in self.samples for nm, bit in self.REASONS.items() if rs & bit})
+        mhz = [m for m, _ in self.samples]
+        return {"sm_mhz": statistics.median(mhz) if mhz else None, "sm_max_mhz": self.max_mhz,
+                "reasons": reasons, "samples": len(mhz), "source": "nvml 5 ms"}
 
 
 def cg_flops(niters, nnz, n):
@@ -227,6 +277,21 @@ def run_ours(args, nx, ny, nz, iters, cfg_index, scaling):
                     raise
                 halo = "NCCL (peer mapping refused: %s)" % e
     xptr = prob.vec_ptr(H.HPCCG_VEC_X)
+    # working set (ELL 324 B/row + 6 vectors): when it fits in L2, flush L2
+    # between timed steps (outside the timed events) so no step starts warm
+    l2_bytes = torch.cuda.get_device_properties(local).L2_cache_size
+    work_bytes = (324 + 6 * 8) * n
+    flush_buf = None
+    if work_bytes < l2_bytes:
+        flush_buf = torch.empty(2 * l2_bytes // 8, dtype=torch.float64, device="cuda")
+    l2_note = ("L2 flushed between timed steps (a %d MB write; working set %.1f MB < L2 %.0f MB); "
+               "per-step events" % (2 * l2_bytes >> 20, work_bytes / 1e6, l2_bytes / 1e6)
+               if flush_buf is not None else
+               "inputs larger than L2 (ELL %.0f MB/GPU > %.0f MB)" % (324e-6 * n, l2_bytes / 1e6))
+
+    def flush():
+        with torch.cuda.stream(stream):
+            flush_buf.zero_()
 
     def barrier():
         if world > 1:
@@ -240,10 +305,30 @@ def run_ours(args, nx, ny, nz, iters, cfg_index, scaling):
         return r, err
 
     def timed(k_steps):
-        """K steps between barriers; CUDA events on the library stream."""
+        """K steps between barriers; CUDA events on the library stream (one
+        pair per step, L2 flushed outside them, when the problem fits in L2)."""
         t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         acc = {"spmv_ms": 0.0, "spmv_n": 0, "niters": 0, "update_ms": 0.0, "pupdate_ms": 0.0}
         barrier()
+        if flush_buf is not None:
+            ms = 0.0
+            for _ in range(k_steps):
+                flush()
+                t0.record(stream)
+                r, err = step()
+                t1.record(stream)
+                t1.synchronize()
+                ms += t0.elapsed_time(t1)
+                st = prob.stats()
+                acc["spmv_ms"] += st["spmv_ms"]
+                acc["spmv_n"] += st["spmv_launches"]
+                acc["update_ms"] += st["update_ms"]
+                acc["pupdate_ms"] += st["pupdate_ms"]
+                acc["niters"] += r["niters"]
+                acc["graph_mode"] = st["graph_mode"]
+            barrier()
+            acc["ms"], acc["r"], acc["err"] = ms, r, err
+            return acc
         t0.record(stream)
         for _ in range(k_steps):
             r, err = step()
@@ -295,14 +380,26 @@ def run_ours(args, nx, ny, nz, iters, cfg_index, scaling):
     step_e2e()
     barrier()
     t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    t0.record(stream)
-    ni_e2e = 0
-    for _ in range(args.steps):
-        r_e, _ = step_e2e()
-        ni_e2e += r_e["niters"]
-    t1.record(stream)
-    barrier()
-    te, fe = D.max_time_sum_work(t0.elapsed_time(t1), cg_flops(ni_e2e, nnz_local, n), "cuda")
+    ni_e2e, te_local = 0, 0.0
+    if flush_buf is not None:          # same L2 rule as the device-timed region
+        for _ in range(args.steps):
+            flush()
+            t0.record(stream)
+            r_e, _ = step_e2e()
+            t1.record(stream)
+            t1.synchronize()
+            te_local += t0.elapsed_time(t1)
+            ni_e2e += r_e["niters"]
+        barrier()
+    else:
+        t0.record(stream)
+        for _ in range(args.steps):
+            r_e, _ = step_e2e()
+            ni_e2e += r_e["niters"]
+        t1.record(stream)
+        barrier()
+        te_local = t0.elapsed_time(t1)
+    te, fe = D.max_time_sum_work(te_local, cg_flops(ni_e2e, nnz_local, n), "cuda")
     e2e_value = fe / (te * 1e-3) * 1e-9
     x_host_err = float(np.max(np.abs(h_x.numpy() - 1.0)))
 
@@ -329,6 +426,9 @@ def run_ours(args, nx, ny, nz, iters, cfg_index, scaling):
                     "events_pass_ms_per_step": round(ev["ms"] / args.steps, 4),
                     "update_avg_us": round(ev["update_ms"] * 1e3 / max(ev["niters"], 1), 2),
                     "pupdate_avg_us": round(ev["pupdate_ms"] * 1e3 / max(ev["niters"], 1), 2)}
+            if flush_buf is not None:
+                roof["note"] = ("latency-bound configuration (the problem fits in L2; the product path is "
+                                "one on-chip kernel): the fraction is not a meaningful target here")
         cpu = None
         if world == 1 and not args.no_cpu_baseline:
             # the oracle's CSR needs ~430 B/row of host RAM: above 2^25 rows it
@@ -357,7 +457,7 @@ def run_ours(args, nx, ny, nz, iters, cfg_index, scaling):
                                        3: "cooperative persistent kernel", 2: "while-graph",
                                        1: "per-iteration graph", 0: "plain"}.get(
                            main.get("graph_mode"), "?"),
-                       "l2": "inputs larger than L2 (ELL %.0f MB/GPU > 126 MB)" % (324e-6 * n),
+                       "l2": l2_note,
                        "gen_ms": round(gen_ms, 3)},
             "t_iter_us": round(t_iter_us, 3),
             "niters_per_step": niters_tot // args.steps,
