@@ -66,6 +66,19 @@ def broadcast_unique_id(make_id, src: int = 0) -> bytes:
     return bytes(uid)
 
 
+def allgather_peer_blobs(blob: bytes, nbytes: int = 256) -> list:
+    """Every rank's hpccg_peer_export blob, in rank order (for peer-only
+    contexts, which have no NCCL: hpccg_peer_attach takes the list)."""
+    import torch.distributed as dist
+    if len(blob) != nbytes:
+        raise ValueError("peer blob must be %d bytes" % nbytes)
+    got = [None] * dist.get_world_size()
+    dist.all_gather_object(got, bytes(blob))
+    if any(not isinstance(b, (bytes, bytearray)) or len(b) != nbytes for b in got):
+        raise RuntimeError("bad peer blob from a rank")
+    return [bytes(b) for b in got]
+
+
 def max_time_sum_work(ms_local: float, work_local: float, device=None):
     """(max over ranks of the device time, sum over ranks of the work)."""
     import torch

@@ -136,7 +136,23 @@ def _body_distributed_cg(rank, world, nx, ny, nz, max_iter, tol):
         assert oracle.maxabsdiff(xg, g.xexact) <= 1e-12
 
 
+def _body_peer_blobs(rank, world):
+    from paper_conf_sc_valero_laragmtv24_b200 import dist as D
+    blob = bytes([rank + 1]) * 256
+    got = D.allgather_peer_blobs(blob)
+    assert got == [bytes([r + 1]) * 256 for r in range(world)]
+    with pytest.raises(ValueError):
+        D.allgather_peer_blobs(b"short")
+
+
 # ------------------------------------------------------------------- tests
+
+def test_gloo_peer_blob_allgather():
+    """Peer-only contexts: the caller all-gathers the hpccg_peer_export blobs
+    (rank order) before hpccg_peer_attach."""
+    _run(_body_peer_blobs, 3)
+
+
 
 def test_slab_helpers():
     from paper_conf_sc_valero_laragmtv24_b200 import dist as D

@@ -296,6 +296,21 @@ def test_cg_first_step_exact():
         assert res["normr"] == math.sqrt(num)
 
 
+def test_cg_iterates_equal_exact_rational_cg():
+    """The k-th fp64 iterate of oracle_cg equals the k-th EXACT iterate of
+    textbook CG (Python Fractions, 4x3x3 grid, k <= 6) to rounding: pins the
+    trajectory beyond the first step, not just the end point."""
+    from test_oracle_sr_pins import exact_textbook_cg
+    p = oracle.generate(4, 3, 3)
+    A = p.to_scipy().toarray().astype(np.int64).tolist()
+    exact = exact_textbook_cg(A, p.b.astype(np.int64).tolist(), 6)
+    for k in range(1, 7):
+        res = oracle.cg(p, k + 1, 0.0)
+        assert res["niters"] == k
+        xe = np.array([float(v) for v in exact[k - 1]])
+        assert np.max(np.abs(res["x"] - xe)) <= 1e-14 * max(1.0, np.max(np.abs(xe)))
+
+
 def independent_cg(A, b, max_iter, tol):
     """Textbook CG written independently (numpy dot, HPCCG loop control)."""
     x = np.zeros_like(b)
