@@ -266,14 +266,18 @@ def run_ours(args, nx, ny, nz, iters, cfg_index, scaling):
     halo = "none (1 slab)"
     if world > 1:
         halo = "NCCL send/recv + ncclAllReduce"
-        if args.halo in ("peer", "auto"):
+        if args.halo in ("peer", "fused", "auto"):
             # collective: every rank maps its neighbours' buffers (CUDA IPC over NVLink);
-            # auto falls back to NCCL if the mapping is refused
+            # auto = fused for HPCCG's CG (the exchange and both allreduces inside the
+            # three CG kernels), else the separate peer kernels; falls back to NCCL if
+            # the mapping is refused
+            mode = 2 if (args.halo == "fused" or (args.halo == "auto" and not sr)) else 1
             try:
-                prob.set_option(H.HPCCG_OPT_HALO_PEER, 1)
-                halo = "peer-memory push + post/collect allreduce kernels (while-graph)"
+                prob.set_option(H.HPCCG_OPT_HALO_PEER, mode)
+                halo = ("peer memory fused into the CG kernels (HALO_PEER 2, while-graph)" if mode == 2
+                        else "peer-memory push + post/collect allreduce kernels (while-graph)")
             except H.HpccgError as e:
-                if args.halo == "peer":
+                if args.halo != "auto":
                     raise
                 halo = "NCCL (peer mapping refused: %s)" % e
     xptr = prob.vec_ptr(H.HPCCG_VEC_X)
@@ -774,9 +778,10 @@ def main():
     ap.add_argument("--tri-n", type=int, default=100_000_000, help="tridiag SIZE (P:L475)")
     ap.add_argument("--lbm-size", type=int, default=1000, help="LBM SIZE (P:L411)")
     ap.add_argument("--iters", type=int, default=None, help="override CG iterations per step")
-    ap.add_argument("--halo", choices=["auto", "nccl", "peer"], default="auto",
-                    help="multi-GPU exchange: our peer-memory kernels (HALO_PEER; auto falls back "
-                         "to NCCL if CUDA IPC is refused) or NCCL")
+    ap.add_argument("--halo", choices=["auto", "nccl", "peer", "fused"], default="auto",
+                    help="multi-GPU exchange: peer memory fused into the CG kernels (HALO_PEER 2, "
+                         "auto for HPCCG's CG), our separate peer-memory kernels (HALO_PEER 1, auto "
+                         "for --cg-variant sr), or NCCL; auto falls back to NCCL if CUDA IPC is refused")
     ap.add_argument("--cg-variant", choices=["hpccg", "sr"], default="hpccg",
                     help="hpccg: HPCCG's CG (default); sr: single-reduction CG (SURVEY f2)")
     ap.add_argument("--no-cpu-baseline", action="store_true")

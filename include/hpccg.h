@@ -117,6 +117,15 @@ extern "C" {
                                ncclAllReduce (or the loopback copies).  NCCL contexts map the
                                peers' buffers with CUDA IPC (collective: every rank sets it);
                                loopback contexts use the sibling slabs.  0 (default): off.
+                               2: the same exchange and allreduces FUSED into the CG kernels
+                               (HPCCG variant; no push / wait / allreduce kernels, no comm
+                               stream): the p update stores its boundary planes into the
+                               neighbours' halos as it computes them and raises their flags,
+                               the SpMV's boundary row blocks wait for the flags and its last
+                               block posts p.Ap to every rank, every block of the x/r update
+                               collects the P posts (rank order) and its last block posts r.r,
+                               which every block of the next p update collects -- 3 kernels
+                               per iteration; needs even nx*ny and n, else behaves as 1.
                                Bit-identical to the loopback reduction order.  Waits time out
                                after ~2 s with HPCCG_ECUDA instead of hanging. */
 #define HPCCG_OPT_WHILE_UNROLL 15 /* CG iterations per execution of the WHILE body
@@ -131,6 +140,12 @@ extern "C" {
                                be scheduled right after its own dependency wait, so the update
                                prefetches x, r, p during the SpMV's tail); 2: PDL with the
                                SpMV triggering only after its rows; 0: off */
+#define HPCCG_OPT_SERPENTINE 20 /* single GPU, finisher-free HPCCG loop: bit 0 = the p update
+                               walks the rows backwards (it starts where the x/r update ended,
+                               with r and p still in L2), bit 1 = the SpMV's blocks take the row
+                               blocks in reverse order.  Same rows per thread / block and the
+                               same partial slots: never changes results.  -1 (default):
+                               auto, 3 when the CG vectors exceed L2 (256^3), else 0 */
 #define HPCCG_OPT_VEC_WAVES 6 /* CG vector kernels: 0 one thread per 16-B unit; k > 0
                                (default 1): a persistent grid of k resident waves */
 

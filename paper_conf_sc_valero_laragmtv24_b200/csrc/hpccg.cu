@@ -151,6 +151,9 @@ struct hpccg_problem {
     int opt_while_unroll = 4;          // CG iterations per WHILE-body execution
     int opt_variant = 0;               // 0 HPCCG CG, 1 single-reduction CG (f2)
     int opt_ff = 1;                    // single slab: finisher-free HPCCG loop (consumer-side sums)
+    int opt_serp = -1;                 // HPCCG_OPT_SERPENTINE bit mask (-1 auto)
+    // HALO_PEER = 2, per slab: ((grid, unroll) key, blocks of the p update that push a plane)
+    std::vector<std::pair<uint64_t, unsigned>> fpush;
     int opt_smem_threads = 0;          // on-chip solve CTA width: 0 auto, 256, 512
     int opt_peer = 0;                  // multi-slab: halo push + allreduce over peer memory
     std::vector<void *> ipc_opened;    // peers' buffers mapped with cudaIpcOpenMemHandle
@@ -447,7 +450,8 @@ int launch_spmv(hpccg_ctx *ctx, int minb, bool check, SpmvArgs a, int64_t r0, in
     a.r1 = r1;
     a.len1 = len1;
     a.nb0 = spmv_blocks(len0, rows);
-    const int64_t blocks = a.nb0 + spmv_blocks(len1, rows);
+    a.nb01 = a.nb0 + spmv_blocks(len1, rows);
+    const int64_t blocks = a.nb01 + spmv_blocks(a.len2, rows);  // len2: kFused only
     if (blocks == 0) return HPCCG_OK;
     if (blocks > 0x7fffffffLL) return fail(HPCCG_EINVAL, "SpMV grid too large");
     if (rows == 2) {
@@ -608,6 +612,15 @@ int spmv_overlapped(hpccg_problem *p, bool timing, double *const *xs, F slab_spm
     return HPCCG_OK;
 }
 
+bool ff_path(const hpccg_problem *p);
+
+// HPCCG_OPT_SERPENTINE in effect: auto = both bits once the CG vectors no
+// longer fit in L2 (256^3: 1005.5 -> 999.0 us/iter; 128^3: no gain)
+int serpentine(const hpccg_problem *p) {
+    if (p->opt_serp >= 0) return p->opt_serp;
+    return p->slabs[0].arena_bytes > ((size_t)126 << 20) ? 3 : 0;
+}
+
 // CG SpMV of every slab with the p.Ap epilogue.  Multi-slab: the rows that
 // do not touch a halo plane (interior) run first, overlapped with the halo
 // exchange on the comm stream (NCCL), then the two boundary planes.
@@ -623,6 +636,7 @@ int cg_spmv_all(hpccg_problem *p, bool timing, bool check) {
         a.part_base = 0;
         a.total_blocks = (unsigned)spmv_blocks(s.n, rows);
         a.parts_only = s.spmv_parts;  // the update kernel finishes p.Ap
+        a.rev = ff_path(p) && (serpentine(p) & 2);
         return launch_spmv<1>(ctx, minb, check, a, 0, s.n, 0, 0, ctx->stream, rows,
                                  p->opt_pdl != 0);
     }
@@ -710,6 +724,7 @@ int enqueue_iteration_ff_u(hpccg_problem *p, bool timing, bool check, unsigned l
         a.q = q;
         a.trace = tr;
         a.trace_max = s.trace_max;
+        a.rev = serpentine(p) & 1;
         const int g = vec_grid(ctx, pup, cdiv(s.n, 2 * kU), p->opt_vec_waves, 0x7fffffff);
         launch_k(pdl, pup, dim3(g), ctx->stream, a);
         CHECK(check_launch(ctx));
@@ -758,11 +773,146 @@ int enqueue_iteration_ff(hpccg_problem *p, bool timing, bool check, unsigned lon
     }
 }
 
+// HALO_PEER = 2: the halo exchange and both scalar allreduces of the HPCCG
+// iteration fused into its three kernels (kernels.cuh "HALO_PEER = 2").
+// Needs the 2-rows-per-thread SpMV and 16-B aligned vectors; else the
+// HALO_PEER = 1 kernels run (same bits).
+bool fused_on(const hpccg_problem *p) {
+    if (p->opt_peer != 2 || !peer_on(p) || p->opt_variant != 0) return false;
+    const Slab &s = p->slabs[0];
+    if (!s.ptab || !aligned16(s.r) || !aligned16(s.p + s.plane) || !aligned16(s.x) || !aligned16(s.Ap))
+        return false;
+    const int64_t b1_r0 = std::max<int64_t>(s.n - s.plane, s.plane);
+    return spmv_rows_per_thread(p->opt_rows, spmv_args(s, s.p, s.Ap), s.plane, b1_r0) == 2;
+}
+
+// Blocks of a grid-stride vector grid (g blocks, 16-B unit i handled by
+// thread i mod (g * kBlock)) that hold a unit of rows [0, plane) or
+// [n - plane, n): the blocks that push a boundary plane.
+unsigned push_blocks(int64_t n, int64_t plane, int g, bool has_lo, bool has_hi) {
+    const int64_t nth = (int64_t)g * kBlock, nv = n >> 1;
+    std::vector<char> mark((size_t)g, 0);
+    auto units = [&](int64_t u0, int64_t u1) {  // units [u0, u1)
+        if (u1 <= u0) return;
+        if (u1 - u0 >= nth) {
+            std::fill(mark.begin(), mark.end(), 1);
+            return;
+        }
+        for (int64_t t = u0 % nth, m = 0; m < u1 - u0;) {  // thread ranges, wrapping at nth
+            const int64_t len = std::min(u1 - u0 - m, nth - t);
+            for (int64_t b = t / kBlock; b <= (t + len - 1) / kBlock; ++b) mark[(size_t)b] = 1;
+            m += len;
+            t = 0;
+        }
+    };
+    if (has_lo) units(0, std::min<int64_t>(cdiv(plane, 2), nv));  // units holding a row < plane
+    if (has_hi) units(std::max<int64_t>((n - plane) / 2, 0), nv); // ... a row >= n - plane
+    if ((n & 1) && (has_hi || (has_lo && n - 1 < plane))) mark[0] = 1;  // thread 0 does row n - 1
+    return (unsigned)std::count(mark.begin(), mark.end(), 1);
+}
+
+template <bool kCheck, int kU>
+int launch_pupdate_fused_t(hpccg_problem *p, const Slab &s) {
+    hpccg_ctx *ctx = p->ctx;
+    auto k = cg_pupdate_fused_kernel<kCheck, kU>;
+    PupdFArgs a{};
+    a.n = s.n;
+    a.plane = s.plane;
+    a.r = s.r;
+    a.p = s.p + s.plane;
+    a.sc = s.sc;
+    a.t = s.ptab;
+    const int g = vec_grid(ctx, k, cdiv(s.n, 2 * kU), p->opt_vec_waves, 0x7fffffff);
+    const int r = s.rank, P = ctx->nranks;
+    const uint64_t key = ((uint64_t)g << 16) | ((uint64_t)kU << 8) | 1u;
+    auto &cache = p->fpush[(size_t)(&s - p->slabs.data())];
+    if (cache.first != key) cache = {key, push_blocks(s.n, s.plane, g, r > 0, r < P - 1)};
+    a.n_push = cache.second;
+    k<<<g, kBlock, 0, ctx->stream>>>(a);
+    return check_launch(ctx);
+}
+
+template <bool kCheck, int kU>
+int launch_update_fused_t(hpccg_problem *p, const Slab &s, unsigned long long cond) {
+    hpccg_ctx *ctx = p->ctx;
+    UpdArgs a{};
+    a.n = s.n;
+    a.x = s.x;
+    a.r = s.r;
+    a.p = s.p + s.plane;
+    a.Ap = s.Ap;
+    a.sc = s.sc;
+    a.red = s.red;
+    a.cond = cond;
+    a.fpeer = s.ptab;
+    // HALO_PEER = 1's update grid (cg_update_kernel): same r.r partials, same bits
+    const int g = vec_grid(ctx, cg_update_kernel<true, kCheck, kU>, cdiv(s.n, 2 * kU), p->opt_vec_waves,
+                           p->red_cap);
+    cg_update_fused_kernel<kCheck, kU><<<g, kBlock, 0, ctx->stream>>>(a);
+    return check_launch(ctx);
+}
+
+int launch_update_fused(hpccg_problem *p, const Slab &s, bool check, unsigned long long cond) {
+    switch (p->opt_unroll) {
+        case 1: return check ? launch_update_fused_t<true, 1>(p, s, cond) : launch_update_fused_t<false, 1>(p, s, cond);
+        case 2: return check ? launch_update_fused_t<true, 2>(p, s, cond) : launch_update_fused_t<false, 2>(p, s, cond);
+        default: return check ? launch_update_fused_t<true, 4>(p, s, cond) : launch_update_fused_t<false, 4>(p, s, cond);
+    }
+}
+
+int launch_pupdate_fused(hpccg_problem *p, const Slab &s, bool check) {
+    switch (p->opt_unroll) {
+        case 1: return check ? launch_pupdate_fused_t<true, 1>(p, s) : launch_pupdate_fused_t<false, 1>(p, s);
+        case 2: return check ? launch_pupdate_fused_t<true, 2>(p, s) : launch_pupdate_fused_t<false, 2>(p, s);
+        default: return check ? launch_pupdate_fused_t<true, 4>(p, s) : launch_pupdate_fused_t<false, 4>(p, s);
+    }
+}
+
+// one launch per slab: interior row blocks, then plane 0, then plane nz-1
+// (the same blocks and partial slots as HALO_PEER = 1's two launches)
+int launch_spmv_fused(hpccg_problem *p, const Slab &s, bool check) {
+    const int64_t n = s.n, plane = s.plane;
+    SpmvArgs a = spmv_args(s, s.p, s.Ap);
+    a.single = 0;
+    a.fpeer = s.ptab;
+    a.r0 = plane;
+    a.len0 = std::max<int64_t>(n - 2 * plane, 0);
+    a.r1 = 0;
+    a.len1 = std::min<int64_t>(plane, n);
+    a.r2 = std::max<int64_t>(n - plane, plane);
+    a.len2 = n - a.r2;
+    a.nb0 = spmv_blocks(a.len0, 2);
+    a.nb01 = a.nb0 + spmv_blocks(a.len1, 2);
+    const int64_t blocks = a.nb01 + spmv_blocks(a.len2, 2);
+    a.part_base = 0;
+    a.total_blocks = (unsigned)blocks;
+    if (check) spmv27x2_kernel<1, true, true><<<(unsigned)blocks, kBlock, 0, p->ctx->stream>>>(a);
+    else spmv27x2_kernel<1, false, true><<<(unsigned)blocks, kBlock, 0, p->ctx->stream>>>(a);
+    return check_launch(p->ctx);
+}
+
+int enqueue_iteration_fused(hpccg_problem *p, bool timing, bool check, unsigned long long cond) {
+    hpccg_ctx *ctx = p->ctx;
+    {
+        PhaseTimer t(p, ctx->stream, PH_PUPDATE, timing);
+        for (const Slab &s : p->slabs) CHECK(launch_pupdate_fused(p, s, check));
+    }
+    {
+        PhaseTimer t(p, ctx->stream, PH_SPMV, timing);
+        for (const Slab &s : p->slabs) CHECK(launch_spmv_fused(p, s, check));
+    }
+    PhaseTimer t(p, ctx->stream, PH_UPDATE, timing);
+    for (size_t i = 0; i < p->slabs.size(); ++i)
+        CHECK(launch_update_fused(p, p->slabs[i], check, i == 0 ? cond : 0ull));
+    return HPCCG_OK;
+}
+
 // One CG iteration (a.6, a.2, a.3+a.4, a.5, a.8) for every slab.  `cond`:
 // while-graph condition handle (0 outside the while-graph); k: the
 // iteration's index (its parity drives the finisher-free loop's state).
 int enqueue_iteration(hpccg_problem *p, bool timing, bool check, unsigned long long cond, int k) {
     if (ff_path(p)) return enqueue_iteration_ff(p, timing, check, cond, k & 1);
+    if (fused_on(p)) return enqueue_iteration_fused(p, timing, check, cond);
     hpccg_ctx *ctx = p->ctx;
     const int single = ctx->mode == MODE_SINGLE;
     // PDL only between back-to-back kernels (single slab; the multi-slab
@@ -1768,6 +1918,7 @@ int hpccg_generate(hpccg_ctx *ctx, int nx, int ny, int nz, hpccg_problem **out) 
     p->ny = ny;
     p->nz = nz;
     p->slabs.resize(ctx->nslabs);
+    p->fpush.assign((size_t)ctx->nslabs, {0ull, 0u});
     auto bail = [&](int rc) {
         hpccg_free(p);
         return rc;
@@ -1988,9 +2139,14 @@ int hpccg_set_option(hpccg_problem *p, int key, int64_t value) {
             return HPCCG_OK;
         case HPCCG_OPT_SMEM_SOLVE: p->opt_smem = value != 0; return HPCCG_OK;
         case HPCCG_OPT_FINISHER_FREE: p->opt_ff = value != 0; return HPCCG_OK;
+        case HPCCG_OPT_SERPENTINE:
+            if (value < -1 || value > 3) return fail(HPCCG_EINVAL, "serpentine: bit mask 0..3 or -1 (auto)");
+            p->opt_serp = (int)value;
+            return HPCCG_OK;
         case HPCCG_OPT_HALO_PEER:
             if (value && p->ctx->mode != MODE_SINGLE && !p->slabs[0].ptab) CHECK(enable_peer(p));
-            p->opt_peer = value != 0;
+            if (value < 0 || value > 2) return fail(HPCCG_EINVAL, "halo peer: 0, 1 or 2");
+            p->opt_peer = (int)value;
             return HPCCG_OK;
         case HPCCG_OPT_SMEM_THREADS:
             if (value != 0 && value != 256 && value != 512) return fail(HPCCG_EINVAL, "smem threads: 0, 256, 512");

@@ -55,6 +55,7 @@ struct CgScalars {
     int sr_k[2];          // index of the next iteration
     int run_q[2];         // run_q[q]: iteration k + 1 runs (written by iteration k);
                           // also used by HPCCG's finisher-free single-slab loop
+    unsigned long long epoch;  // solves initialised so far (HALO_PEER = 2 tags)
 };
 
 // Scratch for the deterministic single-pass grid reduction.
@@ -243,6 +244,126 @@ __global__ void __launch_bounds__(kBlock) gen27_kernel(GenArgs a) {
     if (threadIdx.x == 0) atomicAdd(a.nnz, (unsigned long long)bs);
 }
 
+// ------------------------------- peer-memory z-slab exchange: shared state
+// (protocol: see "peer-memory z-slab exchange (HALO_PEER)" below)
+
+constexpr int kMaxPeers = 64;
+
+struct PeerSync {                      // one per slab, in that slab's device memory
+    unsigned long long flag_from_lo;   // exchanges pushed to me by rank - 1
+    unsigned long long flag_from_hi;   //   ... by rank + 1
+    unsigned long long recv_count;     // exchanges I have waited for
+    unsigned long long push_count;     // exchanges I have pushed
+    unsigned long long ar_count;       // allreduces I have collected
+    unsigned long long ar_posted;      // allreduces I have posted
+    unsigned int push_ticket;          // blocks of the current push done
+    int error;                         // 1: a wait timed out
+    unsigned long long ar_tag[2][kMaxPeers];
+    double ar_val[2][kMaxPeers][2];
+    // HALO_PEER = 2 (collectives fused into the CG kernels): separate words,
+    // tagged tag(epoch, seq) = epoch << 32 | seq instead of counted
+    unsigned long long fflag_from_lo;  // p pushed to me by rank - 1 (seq = k)
+    unsigned long long fflag_from_hi;  //   ... by rank + 1
+    unsigned int fpush_ticket;         // blocks of the current fused push done
+    unsigned int pad_;
+    unsigned long long far_tag[2][kMaxPeers];  // slot 1: p.Ap (seq 2k-1), 0: r.r (seq 2k)
+    double far_val[2][kMaxPeers];
+};
+
+struct PeerTab {                       // device copy per slab; pointers may be peers'
+    int rank, nranks;
+    double *halo_to_lo;                // rank-1's upper halo plane (gets my first owned plane)
+    double *halo_to_hi;                // rank+1's lower halo plane (gets my last owned plane)
+    PeerSync *mine, *lo, *hi;
+    PeerSync *all[kMaxPeers];          // every rank's PeerSync (allreduce posts)
+};
+
+__device__ __forceinline__ void st_release_sys(unsigned long long *p, unsigned long long v) {
+    asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+
+__device__ __forceinline__ unsigned long long ld_acquire_sys(const unsigned long long *p) {
+    unsigned long long v;
+    asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+
+// spin until *flag >= target; false (and the error flag) after ~2 s
+__device__ __forceinline__ bool spin_until(const unsigned long long *flag, unsigned long long target,
+                                           PeerSync *mine) {
+    if (ld_acquire_sys(flag) >= target) return true;  // the common case: one load
+    if (*(volatile int *)&mine->error) return false;  // an earlier wait timed out: do not hang again
+    const unsigned long long t0 = gtimer();
+    while (ld_acquire_sys(flag) < target) {
+        if (gtimer() - t0 > 2000000000ull) {
+            mine->error = 1;
+            return false;
+        }
+        __nanosleep(64);
+    }
+    return true;
+}
+
+// ---- HALO_PEER = 2: the exchange and the scalar allreduces fused into the
+// CG kernels themselves (no push / wait / allreduce kernels, no comm stream):
+//   p update k   collects r.r(k-1) (k > 1), computes p, stores its first /
+//                last owned plane straight into the neighbours' halo planes as
+//                it goes, and its last block raises their flags
+//   SpMV k       interior row blocks first; the boundary blocks (last in
+//                block order) wait for the flags, then gather the halo with
+//                L2-coherent loads; the last block posts the slab's p.Ap
+//   update k     every block collects the P p.Ap posts (rank order) -> alpha;
+//                the last block posts the slab's r.r
+// Flags / tags are tag(epoch, seq) (monotone: the epoch, counted by the init
+// kernel of every solve, is the same on every slab; seq = k for the halo of
+// iteration k, 2k - 1 for its p.Ap, 2k for its r.r), so every kernel knows
+// what it waits for from the device loop state alone.  Slots alternate by seq
+// parity; a rank cannot post seq m + 2 before every rank has collected m (the
+// post needs everyone's m + 1, made after their collect of m), and a push of
+// iteration k + 1 needs r.r(k), posted after the neighbour's SpMV k read the
+// halo.  The rank-order sums are those of peer_allreduce_kernel and the
+// partials those of the HALO_PEER = 1 path: the two modes are bit-identical.
+__device__ __forceinline__ unsigned long long ftag(unsigned long long epoch, unsigned long long seq) {
+    return (epoch << 32) | seq;
+}
+
+// post v as rank t->rank into slot q of every rank (one thread)
+__device__ __forceinline__ void fused_post(const PeerTab *t, int q, double v, unsigned long long tag) {
+    const int P = t->nranks, me = t->rank;
+    for (int r = 0; r < P; ++r) t->all[r]->far_val[q][me] = v;
+    __threadfence_system();
+    for (int r = 0; r < P; ++r) st_release_sys(&t->all[r]->far_tag[q][me], tag);
+}
+
+// wait for the P posts of slot q and sum them in rank order; the block's
+// result (*sh broadcasts it).  Lane r of warp 0 acquires rank r's tag and
+// reads its value (ordered after its own acquire), so the P latencies
+// overlap; lane 0 adds the shuffled values left to right (the order of
+// peer_allreduce_kernel).
+__device__ __forceinline__ double fused_collect_block(const PeerTab *t, int q, unsigned long long tag,
+                                                      double *sh) {
+    __syncthreads();  // sh reuse
+    if (threadIdx.x < 32) {
+        PeerSync *m = t->mine;
+        const int P = t->nranks, lane = threadIdx.x;
+        double s = 0.0;
+        for (int r0 = 0; r0 < P; r0 += 32) {
+            double v = 0.0;
+            if (r0 + lane < P) {
+                spin_until(&m->far_tag[q][r0 + lane], tag, m);
+                v = *(volatile double *)&m->far_val[q][r0 + lane];
+            }
+            for (int j = 0; j < 32 && r0 + j < P; ++j) {
+                const double w = __shfl_sync(0xffffffffu, v, j);
+                s = (r0 + j == 0) ? w : s + w;
+            }
+        }
+        if (lane == 0) *sh = s;
+    }
+    __syncthreads();
+    return *sh;
+}
+
 // --------------------------------------------------------- a.3 SpMV (ELL-27)
 
 // Rows of up to two disjoint ranges [r0, r0+len0) and [r1, r1+len1) (the
@@ -250,6 +371,8 @@ __global__ void __launch_bounds__(kBlock) gen27_kernel(GenArgs a) {
 struct SpmvArgs {
     int64_t r0, len0, r1, len1;
     int64_t nb0;            // blocks covering range 0
+    int64_t r2, len2;       // a third range (HALO_PEER = 2: interior, plane 0, plane nz-1)
+    int64_t nb01;           // blocks covering ranges 0 and 1
     int64_t stride;         // slot stride = n
     int64_t plane;          // x[row + plane] is the row's own entry
     const double *val;
@@ -271,7 +394,17 @@ struct SpmvArgs {
     int early_trigger; // PDL: let the successor be scheduled right after pdl_wait
                        // (it may then prefetch its inputs that this grid does not
                        // write during this grid's tail); 0: after the rows
+    const PeerTab *fpeer;  // HALO_PEER = 2 (spmv27x2_kernel<., ., true>): blocks of ranges
+                           // 1 and 2 wait for the halo flags; the finisher posts p.Ap
+    int rev;           // 1: block b takes the rows (and the partial slot) of block
+                       // gridDim - 1 - b, i.e. the grid walks the rows backwards
+                       // (same rows per block, same partials: identical bits)
 };
+
+// the row block this CTA handles (HPCCG_OPT_SERPENTINE)
+__device__ __forceinline__ int64_t spmv_bid(const SpmvArgs &a) {
+    return a.rev ? (int64_t)gridDim.x - 1 - blockIdx.x : (int64_t)blockIdx.x;
+}
 
 template <int kDots, bool kCheck>
 __device__ __forceinline__ int spmv_done(const SpmvArgs &a) {
@@ -304,8 +437,8 @@ __device__ __forceinline__ void spmv_sr_partials(const SpmvArgs &a, double g, do
     __shared__ double sh2[64];
     const double2 t = block_reduce2(g, d, sh2);
     if (threadIdx.x == 0) {
-        a.parts_only[a.part_base + blockIdx.x] = t.x;
-        a.parts_only[a.total_blocks + a.part_base + blockIdx.x] = t.y;
+        a.parts_only[a.part_base + spmv_bid(a)] = t.x;
+        a.parts_only[a.total_blocks + a.part_base + spmv_bid(a)] = t.y;
     }
 }
 
@@ -322,11 +455,12 @@ __device__ __forceinline__ void spmv_sr_partials(const SpmvArgs &a, double g, do
 template <int kDots, bool kCheck, int kMinB>
 __global__ void __launch_bounds__(kBlock, kMinB) spmv27_kernel(SpmvArgs a) {
     int64_t row, lim;
-    if ((int64_t)blockIdx.x < a.nb0) {
-        row = a.r0 + (int64_t)blockIdx.x * kBlock + threadIdx.x;
+    const int64_t bid = spmv_bid(a);
+    if (bid < a.nb0) {
+        row = a.r0 + bid * kBlock + threadIdx.x;
         lim = a.r0 + a.len0;
     } else {
-        row = a.r1 + ((int64_t)blockIdx.x - a.nb0) * kBlock + threadIdx.x;
+        row = a.r1 + (bid - a.nb0) * kBlock + threadIdx.x;
         lim = a.r1 + a.len1;
     }
     constexpr bool kDot = kDots == 1;
@@ -394,12 +528,12 @@ __global__ void __launch_bounds__(kBlock, kMinB) spmv27_kernel(SpmvArgs a) {
         if (a.parts_only) {  // block partial only; the update kernel sums them
             __shared__ double shp[32];
             d = block_reduce<false>(d, shp);
-            if (threadIdx.x == 0) a.parts_only[a.part_base + blockIdx.x] = d;
+            if (threadIdx.x == 0) a.parts_only[a.part_base + bid] = d;
             return;
         }
         CgScalars *sc = a.sc;
         const int single = a.single;
-        grid_reduce<false>(d, a.red, a.part_base + blockIdx.x, a.total_blocks,
+        grid_reduce<false>(d, a.red, a.part_base + (unsigned)bid, a.total_blocks,
                            [sc, single](double s) {
                                if (single) sc->pAp = s; else sc->loc_pAp = s;
                            });
@@ -414,17 +548,32 @@ __global__ void __launch_bounds__(kBlock, kMinB) spmv27_kernel(SpmvArgs a) {
 // (tools/spmvbench.cu).  Needs even n (stride), even range starts and a 16-B
 // aligned y (the host checks); a range of odd length ends in a 1-row thread.
 // Same per-row FMA order as spmv27_kernel: identical bits.
-template <int kDots, bool kCheck>
-__global__ void __launch_bounds__(kBlock, 4) spmv27x2_kernel(SpmvArgs a) {
-    constexpr bool kDot = kDots == 1;
-    int64_t row, lim;
-    if ((int64_t)blockIdx.x < a.nb0) {
-        row = a.r0 + ((int64_t)blockIdx.x * kBlock + threadIdx.x) * 2;
-        lim = a.r0 + a.len0;
-    } else {
-        row = a.r1 + (((int64_t)blockIdx.x - a.nb0) * kBlock + threadIdx.x) * 2;
-        lim = a.r1 + a.len1;
+// HALO_PEER = 2 boundary block: wait until the neighbours whose halo planes
+// rows [first, last] read have pushed p of iteration k (uniform per block)
+__device__ __forceinline__ void fused_halo_wait(const SpmvArgs &a, int64_t first, int64_t last) {
+    if (threadIdx.x == 0) {
+        const PeerTab *t = a.fpeer;
+        const unsigned long long tg = ftag(__ldg(&a.sc->epoch), (unsigned long long)__ldg(&a.sc->k));
+        if (first < a.plane && t->rank > 0) spin_until(&t->mine->fflag_from_lo, tg, t->mine);
+        if (last >= a.stride - a.plane && t->rank < t->nranks - 1)
+            spin_until(&t->mine->fflag_from_hi, tg, t->mine);
     }
+    __syncthreads();
+}
+
+// kFused (HALO_PEER = 2, multi-slab CG SpMV): ranges 1 and 2 are the boundary
+// planes; their blocks (the last ones in block order) wait for the halo flags
+// before any load (fused_halo_wait) and gather through L2 (ld.global.cg: the
+// halo was written by a peer during this grid's lifetime, so the read-only
+// path is not allowed for it); interior blocks are unchanged.
+template <bool kCoh>
+__device__ __forceinline__ double ld_gather(const double *p) {
+    return kCoh ? __ldcg(p) : __ldg(p);
+}
+
+template <int kDots, bool kCheck, bool kFused, bool kCoh>
+__device__ __forceinline__ void spmv27x2_body(const SpmvArgs &a, int64_t row, int64_t lim, int64_t bid) {
+    constexpr bool kDot = kDots == 1;
     double d = 0.0, dg = 0.0;  // kDots 1: p.Ap; kDots 2: delta (d) and gamma (dg)
     int done = 0;
     if (row + 1 < lim) {
@@ -451,7 +600,7 @@ __global__ void __launch_bounds__(kBlock, 4) spmv27x2_kernel(SpmvArgs a) {
             }
 #pragma unroll
             for (int t = 0; t < 3; ++t) {
-                const double xa = __ldg(a.x + cc[t].x), xb = __ldg(a.x + cc[t].y);
+                const double xa = ld_gather<kCoh>(a.x + cc[t].x), xb = ld_gather<kCoh>(a.x + cc[t].y);
                 if (3 * g + t == kDiagSlot) {
                     x0 = xa;
                     x1 = xb;
@@ -464,8 +613,8 @@ __global__ void __launch_bounds__(kBlock, 4) spmv27x2_kernel(SpmvArgs a) {
         }
         *reinterpret_cast<double2 *>(a.y + row) = make_double2(s0, s1);
         if (kDots > 0) {
-            const double p0 = c0 == row + a.plane ? x0 : __ldg(a.x + row + a.plane);
-            const double p1 = c1 == row + 1 + a.plane ? x1 : __ldg(a.x + row + 1 + a.plane);
+            const double p0 = c0 == row + a.plane ? x0 : ld_gather<kCoh>(a.x + row + a.plane);
+            const double p1 = c1 == row + 1 + a.plane ? x1 : ld_gather<kCoh>(a.x + row + 1 + a.plane);
             d = fma(s1, p1, s0 * p0);
             if (kDots == 2) dg = fma(p1, p1, p0 * p0);
         }
@@ -478,10 +627,10 @@ __global__ void __launch_bounds__(kBlock, 4) spmv27x2_kernel(SpmvArgs a) {
 #pragma unroll
         for (int k = 0; k < kSlots; ++k)
             s0 = fma(ld_stream(a.val + k * a.stride + row, pol),
-                     __ldg(a.x + ld_stream(a.col + k * a.stride + row, pol)), s0);
+                     ld_gather<kCoh>(a.x + ld_stream(a.col + k * a.stride + row, pol)), s0);
         a.y[row] = s0;
         if (kDots > 0) {
-            const double xi = __ldg(a.x + row + a.plane);
+            const double xi = ld_gather<kCoh>(a.x + row + a.plane);
             d = s0 * xi;
             if (kDots == 2) dg = xi * xi;
         }
@@ -500,16 +649,50 @@ __global__ void __launch_bounds__(kBlock, 4) spmv27x2_kernel(SpmvArgs a) {
         if (a.parts_only) {  // block partial only; the update kernel sums them
             __shared__ double shp[32];
             d = block_reduce<false>(d, shp);
-            if (threadIdx.x == 0) a.parts_only[a.part_base + blockIdx.x] = d;
+            if (threadIdx.x == 0) a.parts_only[a.part_base + bid] = d;
             return;
         }
         CgScalars *sc = a.sc;
         const int single = a.single;
-        grid_reduce<false>(d, a.red, a.part_base + blockIdx.x, a.total_blocks,
-                           [sc, single](double s) {
+        const PeerTab *fp = kFused ? a.fpeer : nullptr;
+        grid_reduce<false>(d, a.red, a.part_base + (unsigned)bid, a.total_blocks,
+                           [sc, single, fp](double s) {
                                if (single) sc->pAp = s; else sc->loc_pAp = s;
+                               if (kFused)  // p.Ap(k) -> slot 1 of every rank
+                                   fused_post(fp, 1, s, ftag(sc->epoch, 2ull * (unsigned)sc->k - 1ull));
                            });
     }
+}
+
+
+template <int kDots, bool kCheck, bool kFused = false>
+__global__ void __launch_bounds__(kBlock, 4) spmv27x2_kernel(SpmvArgs a) {
+    int64_t row, lim;
+    const int64_t bid = spmv_bid(a);
+    bool bnd = false;
+    if (bid < a.nb0) {
+        row = a.r0 + (bid * kBlock + threadIdx.x) * 2;
+        lim = a.r0 + a.len0;
+    } else if (!kFused || bid < a.nb01) {
+        row = a.r1 + ((bid - a.nb0) * kBlock + threadIdx.x) * 2;
+        lim = a.r1 + a.len1;
+        bnd = kFused;
+    } else {
+        row = a.r2 + ((bid - a.nb01) * kBlock + threadIdx.x) * 2;
+        lim = a.r2 + a.len2;
+        bnd = true;
+    }
+    if (kFused && bnd) {
+        // `done` first: past convergence no neighbour pushes (uniform exit)
+        if (kCheck && __ldg(&a.sc->done)) return;
+        const int64_t first = row - 2 * (int64_t)threadIdx.x;
+        fused_halo_wait(a, first, min(first + 2 * kBlock, lim) - 1);
+    }
+    if (kFused && bnd) {
+        spmv27x2_body<kDots, kCheck, kFused, true>(a, row, lim, bid);
+        return;
+    }
+    spmv27x2_body<kDots, kCheck, kFused, false>(a, row, lim, bid);
 }
 
 // ------------------------------------------------ streaming vector kernels
@@ -589,6 +772,105 @@ __global__ void __launch_bounds__(kBlock) cg_pupdate_kernel(int64_t n, const dou
     }
 }
 
+// a.6 + a.2 fused (HALO_PEER = 2, multi-slab): r.r(k-1) collected from every
+// rank's post (k > 1), p = r + beta p, and the first / last owned plane of
+// the new p stored straight into the neighbours' halo planes as it is
+// computed; the blocks that pushed fence and take a ticket, the last of them
+// raises the neighbours' flags (n_push = how many blocks hold boundary units,
+// from the host).  The first trip's loads are issued before the collect.
+// 16-B units (the host falls back to HALO_PEER = 1 otherwise).
+struct PupdFArgs {
+    int64_t n, plane;
+    const double *r;
+    double *p;             // owned part (local-with-halo base + plane)
+    CgScalars *sc;
+    const PeerTab *t;
+    unsigned n_push;       // blocks that store into a neighbour's halo
+};
+
+template <bool kCheck, int kU>
+__global__ void __launch_bounds__(kBlock) cg_pupdate_fused_kernel(PupdFArgs a) {
+    __shared__ double sh;
+    __shared__ int last;
+    CgScalars *sc = a.sc;
+    const int64_t tid = gtid(), nth = gnth(), nv = a.n >> 1, n = a.n, plane = a.plane;
+    const double2 *__restrict__ r2 = reinterpret_cast<const double2 *>(a.r);
+    double2 *__restrict__ p2 = reinterpret_cast<double2 *>(a.p);
+    double2 ra[kU], pa[kU];
+    auto load = [&](int64_t b) {
+#pragma unroll
+        for (int u = 0; u < kU; ++u) {
+            const int64_t i = b + u * nth;
+            if (i < nv) {
+                ra[u] = r2[i];
+                pa[u] = p2[i];
+            }
+        }
+    };
+    load(tid);
+    if (kCheck && __ldg(&sc->done)) return;  // uniform: nobody pushes or posts
+    const int k = __ldg(&sc->k);
+    const unsigned long long epoch = __ldg(&sc->epoch);
+    const bool first = (k == 1);
+    double beta = 0.0;
+    if (!first) {
+        const double rtrans = fused_collect_block(a.t, 0, ftag(epoch, 2ull * (unsigned)(k - 1)), &sh);
+        beta = rtrans / __ldg(&sc->rr_prev);
+        if (blockIdx.x == 0 && threadIdx.x == 0) sc->rr_cur = rtrans;
+    }
+    double *lo = a.t->halo_to_lo, *hi = a.t->halo_to_hi;
+    int pushed = 0;
+    auto put = [&](int64_t i, double v) {  // row i of the new p
+        if (lo && i < plane) {
+            lo[i] = v;
+            pushed = 1;
+        }
+        if (hi && i >= n - plane) {
+            hi[i - (n - plane)] = v;
+            pushed = 1;
+        }
+    };
+    for (int64_t b = tid; b < nv;) {
+#pragma unroll
+        for (int u = 0; u < kU; ++u) {
+            const int64_t i = b + u * nth;
+            if (i < nv) {
+                double2 q = ra[u];
+                if (!first) {
+                    q.x = fma(beta, pa[u].x, ra[u].x);
+                    q.y = fma(beta, pa[u].y, ra[u].y);
+                }
+                p2[i] = q;
+                if (2 * i < plane || 2 * i + 1 >= n - plane) {
+                    put(2 * i, q.x);
+                    put(2 * i + 1, q.y);
+                }
+            }
+        }
+        b += kU * nth;
+        if (b < nv) load(b);
+    }
+    if (tid == 0 && (n & 1)) {
+        const int64_t i = n - 1;
+        const double v = first ? a.r[i] : fma(beta, a.p[i], a.r[i]);
+        a.p[i] = v;
+        put(i, v);
+    }
+    if (!__syncthreads_or(pushed)) return;
+    if (threadIdx.x == 0) {
+        __threadfence_system();  // this block's pushes before its ticket
+        const unsigned tk = atomicAdd(&a.t->mine->fpush_ticket, 1u);
+        last = (tk == a.n_push - 1);
+    }
+    __syncthreads();
+    if (!last || threadIdx.x != 0) return;
+    __threadfence_system();
+    a.t->mine->fpush_ticket = 0u;
+    const unsigned long long tg = ftag(epoch, (unsigned long long)k);
+    if (a.t->lo) st_release_sys(&a.t->lo->fflag_from_hi, tg);
+    if (a.t->hi) st_release_sys(&a.t->hi->fflag_from_lo, tg);
+}
+
 // a.5: x += alpha p; r -= alpha Ap; partial r.r; then the loop control of
 // the NEXT iteration (A4 lagged check, A11 guard) in the last block, which
 // also drives the while-graph's condition (`cond`, 0 = none).  48n B.
@@ -604,6 +886,7 @@ struct UpdArgs {
     Reduction red;
     int single;
     unsigned long long cond;  // cudaGraphConditionalHandle or 0
+    const PeerTab *fpeer;     // cg_update_fused_kernel (HALO_PEER = 2)
 };
 
 __device__ __forceinline__ void set_cond(unsigned long long h, int cont) {
@@ -738,6 +1021,85 @@ __global__ void __launch_bounds__(kBlock) cg_update_kernel(UpdArgs a) {
                        });
 }
 
+// a.5 fused (HALO_PEER = 2, multi-slab): the first trip's x, r, p, Ap loads,
+// then p.Ap collected from every rank's post -> alpha, x += alpha p,
+// r -= alpha Ap, and cg_update_kernel<true, ., kU>'s r.r partials and
+// finisher (same per-thread order and grid: same bits), whose last block
+// also posts the slab's r.r(k).
+template <bool kCheck, int kU>
+__global__ void __launch_bounds__(kBlock) cg_update_fused_kernel(UpdArgs a) {
+    __shared__ double shf;
+    CgScalars *sc = a.sc;
+    const int64_t tid = gtid(), nth = gnth(), nv = a.n >> 1;
+    double2 *__restrict__ x2 = reinterpret_cast<double2 *>(a.x);
+    double2 *__restrict__ r2 = reinterpret_cast<double2 *>(a.r);
+    const double2 *__restrict__ p2 = reinterpret_cast<const double2 *>(a.p);
+    const double2 *__restrict__ q2 = reinterpret_cast<const double2 *>(a.Ap);
+    double2 xa[kU], ra[kU], pa[kU], qa[kU];
+    auto load = [&](int64_t b) {
+#pragma unroll
+        for (int u = 0; u < kU; ++u) {
+            const int64_t i = b + u * nth;
+            if (i < nv) {
+                xa[u] = x2[i];
+                ra[u] = r2[i];
+                pa[u] = p2[i];
+                qa[u] = q2[i];
+            }
+        }
+    };
+    load(tid);
+    if (kCheck && __ldg(&sc->done)) return;  // uniform: nobody posted
+    const double rtrans = __ldg(&sc->rr_cur);
+    const double pAp =
+        fused_collect_block(a.fpeer, 1, ftag(__ldg(&sc->epoch), 2ull * (unsigned)__ldg(&sc->k) - 1ull), &shf);
+    const bool stop = (rtrans == 0.0) || (pAp == 0.0);  // A11
+    const double alpha = stop ? 0.0 : rtrans / pAp;
+    double acc = 0.0, acc2 = 0.0;
+    for (int64_t b = tid; b < nv;) {
+#pragma unroll
+        for (int u = 0; u < kU; ++u) {
+            const int64_t i = b + u * nth;
+            if (i < nv) {
+                xa[u].x = fma(alpha, pa[u].x, xa[u].x);
+                xa[u].y = fma(alpha, pa[u].y, xa[u].y);
+                ra[u].x = fma(-alpha, qa[u].x, ra[u].x);
+                ra[u].y = fma(-alpha, qa[u].y, ra[u].y);
+                x2[i] = xa[u];
+                r2[i] = ra[u];
+                acc = fma(ra[u].x, ra[u].x, acc);
+                acc2 = fma(ra[u].y, ra[u].y, acc2);
+            }
+        }
+        b += kU * nth;
+        if (b < nv) load(b);
+    }
+    if (tid == 0 && (a.n & 1)) {
+        const int64_t i = a.n - 1;
+        a.x[i] = fma(alpha, a.p[i], a.x[i]);
+        const double rv = fma(-alpha, a.Ap[i], a.r[i]);
+        a.r[i] = rv;
+        acc = fma(rv, rv, acc);
+    }
+    acc += acc2;
+    const unsigned long long cond = a.cond;
+    const PeerTab *fp = a.fpeer;
+    grid_reduce<false>(acc, a.red, blockIdx.x, gridDim.x, [sc, rtrans, stop, cond, pAp, fp](double s) {
+        sc->pAp = pAp;
+        sc->rr_prev = rtrans;
+        sc->loc_rr = s;
+        const int k = sc->k;
+        fused_post(fp, 0, s, ftag(sc->epoch, 2ull * (unsigned)k));  // r.r(k)
+        const double normr = sqrt(rtrans);
+        sc->normr = normr;
+        sc->niters = k;
+        sc->k = k + 1;
+        const int done = stop || !((k + 1) < sc->max_iter && normr > sc->tol);
+        sc->done = done;
+        set_cond(cond, !done);
+    });
+}
+
 // ------------------- single slab: HPCCG's loop without any grid finisher
 // The last-block finisher of cg_update_kernel (fence + atomic ticket + the
 // final sum, then the loop control) sits between every update and the next
@@ -767,6 +1129,7 @@ struct Pupd1Args {
     int q;
     TraceSlot *trace;
     int trace_max;
+    int rev;  // 1: each thread walks its trips last to first (no reduction: same bits)
 };
 
 // Fixed-order sum of n partials (the order of grid_reduce's last block);
@@ -826,12 +1189,16 @@ __global__ void __launch_bounds__(kBlock) cg_pupdate1_kernel(Pupd1Args a) {
         load_r(b);
         load_p(b);
     };
+    // HPCCG_OPT_SERPENTINE: walking the rows backwards starts where the x/r
+    // update (forwards) ended, so the first trips find r and p in L2
+    const int64_t step = kU * nth;
+    const int64_t b0 = (a.rev && tid < nv) ? tid + ((nv - 1 - tid) / step) * step : tid;
     // p (this kernel's own output one iteration ago) is complete before the
     // update's blocks pass their wait: read it during the update's tail
-    load_p(tid);
+    load_p(b0);
     pdl_wait();
     pdl_trigger();
-    load_r(tid);
+    load_r(b0);
     if (!run_check(sc, a.q)) return;
     const int k = __ldg(&sc->k);
     trace_mark(a.trace, a.trace_max, k, 0, false);
@@ -843,7 +1210,7 @@ __global__ void __launch_bounds__(kBlock) cg_pupdate1_kernel(Pupd1Args a) {
         sc->normr = sqrt(rtrans);
         sc->niters = k;
     }
-    for (int64_t b = tid; b < nv;) {
+    for (int64_t b = b0; b >= 0 && b < nv;) {
 #pragma unroll
         for (int u = 0; u < kU; ++u) {
             const int64_t i = b + u * nth;
@@ -856,8 +1223,8 @@ __global__ void __launch_bounds__(kBlock) cg_pupdate1_kernel(Pupd1Args a) {
                 p2[i] = v;
             }
         }
-        b += kU * nth;
-        if (b < nv) load(b);
+        b += a.rev ? -step : step;
+        if (b >= 0 && b < nv) load(b);
     }
     if (tid == 0 && (a.n & 1)) {
         const int64_t i = a.n - 1;
@@ -1013,6 +1380,7 @@ __global__ void cg_initstate_kernel(CgScalars *sc, int max_iter, double tol,
     sc->done = done;
     sc->run_q[0] = !done;  // finisher-free loop: iteration 1 (parity 1) runs
     sc->run_q[1] = 0;
+    sc->epoch = sc->epoch + 1;
     set_cond(cond, !done);
 }
 
@@ -1684,53 +2052,6 @@ __global__ void slab_allreduce_kernel(const double *const *src, double *const *d
 // Memory model: pushes / posts, then fence.sc.sys, then a st.release.sys
 // of the flag / tag; waits are ld.acquire.sys spins, bounded by a %globaltimer
 // timeout that records an error instead of hanging the GPU.
-
-constexpr int kMaxPeers = 64;
-
-struct PeerSync {                      // one per slab, in that slab's device memory
-    unsigned long long flag_from_lo;   // exchanges pushed to me by rank - 1
-    unsigned long long flag_from_hi;   //   ... by rank + 1
-    unsigned long long recv_count;     // exchanges I have waited for
-    unsigned long long push_count;     // exchanges I have pushed
-    unsigned long long ar_count;       // allreduces I have collected
-    unsigned long long ar_posted;      // allreduces I have posted
-    unsigned int push_ticket;          // blocks of the current push done
-    int error;                         // 1: a wait timed out
-    unsigned long long ar_tag[2][kMaxPeers];
-    double ar_val[2][kMaxPeers][2];
-};
-
-struct PeerTab {                       // device copy per slab; pointers may be peers'
-    int rank, nranks;
-    double *halo_to_lo;                // rank-1's upper halo plane (gets my first owned plane)
-    double *halo_to_hi;                // rank+1's lower halo plane (gets my last owned plane)
-    PeerSync *mine, *lo, *hi;
-    PeerSync *all[kMaxPeers];          // every rank's PeerSync (allreduce posts)
-};
-
-__device__ __forceinline__ void st_release_sys(unsigned long long *p, unsigned long long v) {
-    asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
-}
-
-__device__ __forceinline__ unsigned long long ld_acquire_sys(const unsigned long long *p) {
-    unsigned long long v;
-    asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
-    return v;
-}
-
-// spin until *flag >= target; false (and the error flag) after ~2 s
-__device__ __forceinline__ bool spin_until(const unsigned long long *flag, unsigned long long target,
-                                           PeerSync *mine) {
-    const unsigned long long t0 = gtimer();
-    while (ld_acquire_sys(flag) < target) {
-        if (gtimer() - t0 > 2000000000ull) {
-            mine->error = 1;
-            return false;
-        }
-        __nanosleep(64);
-    }
-    return true;
-}
 
 // a.2 push: my first owned plane -> rank-1's upper halo, my last owned plane
 // -> rank+1's lower halo (x = local-with-halo base); the last block signals.

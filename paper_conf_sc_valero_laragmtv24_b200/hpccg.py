@@ -37,7 +37,7 @@ HPCCG_OPT_SPMV_ROWS, HPCCG_OPT_VEC_UNROLL = 7, 8
 HPCCG_OPT_PERSISTENT, HPCCG_OPT_PERSIST_ROWS, HPCCG_OPT_PDL = 9, 10, 11
 HPCCG_OPT_CLUSTER_ROWS, HPCCG_OPT_SMEM_SOLVE, HPCCG_OPT_TRACE = 12, 13, 14
 HPCCG_OPT_WHILE_UNROLL, HPCCG_OPT_CG_VARIANT, HPCCG_OPT_FINISHER_FREE = 15, 16, 17
-HPCCG_OPT_SMEM_THREADS, HPCCG_OPT_HALO_PEER = 18, 19
+HPCCG_OPT_SMEM_THREADS, HPCCG_OPT_HALO_PEER, HPCCG_OPT_SERPENTINE = 18, 19, 20
 
 _lock = threading.Lock()
 _lib = None

@@ -8,7 +8,7 @@ flags and allreduce slots -- that NCCL cannot (it refuses two ranks on one
 GPU)."""
 
 
-def run(rank, nranks, dims, variant, max_iter, tol, to_parent, from_parent):
+def run(rank, nranks, dims, variant, max_iter, tol, to_parent, from_parent, halo=1):
     try:
         import numpy as np
         from paper_conf_sc_valero_laragmtv24_b200 import hpccg as H
@@ -17,6 +17,8 @@ def run(rank, nranks, dims, variant, max_iter, tol, to_parent, from_parent):
             to_parent.put(("blob", rank, p.peer_export()))
             blobs = from_parent.get(timeout=120)
             p.peer_attach(blobs)
+            if halo != 1:  # 2: exchange + allreduces fused into the CG kernels
+                p.set_option(H.HPCCG_OPT_HALO_PEER, halo)
             out = []
             for wh in (1, 0):
                 p.set_option(H.HPCCG_OPT_WHILE, wh)

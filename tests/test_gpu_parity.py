@@ -622,6 +622,34 @@ def test_cg_finisher_free_loop_bitwise_vs_finisher(ctx, unroll, dims, max_iter, 
         assert outs[0][0] == max_iter - 1
 
 
+@pytest.mark.parametrize("dims,max_iter,tol", [((24, 20, 12), 150, 1e-12), ((33, 9, 3), 150, 1e-12),
+                                               ((64, 64, 32), 41, 0.0), ((37, 29, 23), 30, 0.0)])
+def test_cg_serpentine_orders_bitwise(ctx, dims, max_iter, tol):
+    """HPCCG_OPT_SERPENTINE: the p update walking its trips backwards and the
+    SpMV taking its row blocks in reverse order (partials kept in row-block
+    slots) change only the traversal, never the bits: niters, normr and x are
+    identical for every mask, in the while-graph, the per-iteration graph and
+    plain timed launches."""
+    outs = []
+    with H.Problem(ctx, *dims) as p:
+        p.set_option(H.HPCCG_OPT_PERSISTENT, 0)
+        for serp in (0, 1, 2, 3):
+            p.set_option(H.HPCCG_OPT_SERPENTINE, serp)
+            for wh, timing in [(1, 0), (0, 0), (0, 1)]:
+                p.set_option(H.HPCCG_OPT_WHILE, wh)
+                p.set_option(H.HPCCG_OPT_TIMING, timing)
+                p.set_vec(H.HPCCG_VEC_X, np.zeros(p.n))
+                r = p.solve(max_iter, tol)
+                outs.append((r["niters"], r["normr"], p.get_vec(H.HPCCG_VEC_X)))
+        p.set_option(H.HPCCG_OPT_TIMING, 0)
+    for o in outs[1:]:
+        assert o[:2] == outs[0][:2]
+        np.testing.assert_array_equal(o[2], outs[0][2])
+    with pytest.raises(H.HpccgError):
+        with H.Problem(ctx, 4, 4, 4) as q:
+            q.set_option(H.HPCCG_OPT_SERPENTINE, 4)
+
+
 # ------------------------- full sizes of BASELINE configs[2] and configs[3]
 
 def test_full_256cubed_vs_oracle(ctx):
@@ -719,6 +747,79 @@ def test_peer_halo_and_allreduce_loopback_bitwise(P, variant):
         assert np.max(np.abs(outs[0][2] - oref["x"])) <= CG_ATOL
 
 
+@pytest.mark.parametrize("P,dims", [(2, (16, 12, 6)), (3, (16, 12, 6)), (4, (12, 10, 5)),
+                                    (2, (10, 6, 1)), (3, (8, 6, 2)), (2, (9, 7, 4)),
+                                    (3, (64, 64, 16)), (2, (96, 80, 40))])
+def test_peer_fused_loopback_bitwise(P, dims):
+    """HALO_PEER = 2: the halo push fused into the p update, the halo wait into
+    the SpMV's boundary blocks and both allreduces into the SpMV / update
+    finishers and the consumers' prologues reproduce the copy-exchange path
+    and HALO_PEER = 1 BIT FOR BIT (same blocks, partial slots and rank-order
+    sums) in every launch mode, and match the global oracle.  nz = 1 and 2
+    (boundary blocks touching both halos / no interior), an odd plane
+    (9 x 7: the 1-row SpMV, so HALO_PEER = 2 falls back to 1), and slabs
+    large enough that only some p-update blocks push (end ranks: one plane)."""
+    nx, ny, nz = dims
+    with H.Context(0, nranks=P, loopback=True) as c, H.Problem(c, nx, ny, nz) as p:
+        outs = []
+        for peer, wh, timing in [(0, 1, 0), (2, 1, 0), (2, 0, 0), (2, 0, 1), (1, 1, 0), (2, 1, 0)]:
+            p.set_option(H.HPCCG_OPT_HALO_PEER, peer)
+            p.set_option(H.HPCCG_OPT_WHILE, wh)
+            p.set_option(H.HPCCG_OPT_TIMING, timing)
+            p.set_vec(H.HPCCG_VEC_X, np.zeros(p.n * P))
+            r = p.solve(150, 1e-12)
+            outs.append((r["niters"], r["normr"], p.get_vec(H.HPCCG_VEC_X)))
+        # plain launches: an iteration is 3 kernels per slab when fused (no
+        # push / wait / allreduce kernels), 10 with HALO_PEER = 1
+        p.set_option(H.HPCCG_OPT_TIMING, 1)
+        per_iter = {}
+        for peer in (2, 1):
+            p.set_option(H.HPCCG_OPT_HALO_PEER, peer)
+            launches = []
+            for m in (5, 9):
+                p.set_vec(H.HPCCG_VEC_X, np.zeros(p.n * P))
+                p.solve(m, 0.0)
+                launches.append(p.stats()["kernel_launches"])
+            per_iter[peer] = (launches[1] - launches[0]) / (4 * P)
+        assert per_iter[1] == (10 if nz > 2 else 9)   # nz <= 2: no interior SpMV launch
+        assert per_iter[2] == (3 if (nx * ny) % 2 == 0 else 10)
+        p.set_option(H.HPCCG_OPT_TIMING, 0)
+        for o in outs[1:]:
+            assert o[:2] == outs[0][:2]
+            np.testing.assert_array_equal(o[2], outs[0][2])
+        ref = oracle.generate(nx, ny, nz * P)
+        oref = oracle.cg(ref, 150, 1e-12)
+        assert abs(outs[0][0] - oref["niters"]) <= 1
+        assert np.max(np.abs(outs[0][2] - oref["x"])) <= CG_ATOL
+
+
+def test_peer_fused_repeat_solves_and_mode_switches():
+    """Fused tags are (epoch, seq): solves of different lengths, tol-stopped
+    solves (kernels past convergence exit before waiting) and switches between
+    HALO_PEER 1 and 2 never wait on a stale flag or slot."""
+    P = 3
+    with H.Context(0, nranks=P, loopback=True) as c, H.Problem(c, 8, 8, 4) as p:
+        ref = oracle.generate(8, 8, 4 * P)
+        for m, mode, wh in [(1, 2, 1), (2, 2, 1), (7, 2, 0), (3, 1, 1), (20, 2, 1), (5, 2, 0), (9, 1, 0)]:
+            p.set_option(H.HPCCG_OPT_HALO_PEER, mode)
+            p.set_option(H.HPCCG_OPT_WHILE, wh)
+            p.set_vec(H.HPCCG_VEC_X, np.zeros(p.n * P))
+            r = p.solve(m, 0.0)
+            o = oracle.cg(ref, m, 0.0)
+            assert r["niters"] == o["niters"] == m - 1
+            assert np.max(np.abs(p.get_vec(H.HPCCG_VEC_X) - o["x"])) <= CG_ATOL
+        p.set_option(H.HPCCG_OPT_HALO_PEER, 2)
+        for wh in (1, 0):
+            p.set_option(H.HPCCG_OPT_WHILE, wh)
+            p.set_vec(H.HPCCG_VEC_X, np.zeros(p.n * P))
+            r = p.solve(150, 1e-10)  # stops early: the unrolled body / poll runs past it
+            o = oracle.cg(ref, 150, 1e-10)
+            assert abs(r["niters"] - o["niters"]) <= 1
+            assert np.max(np.abs(p.get_vec(H.HPCCG_VEC_X) - 1.0)) <= 1e-8
+        with pytest.raises(H.HpccgError):
+            p.set_option(H.HPCCG_OPT_HALO_PEER, 3)
+
+
 def test_peer_mode_max_iter_and_repeat_solves():
     """Counters stay in lockstep across solves of different lengths (flags and
     tags are operation counts, never reset)."""
@@ -742,7 +843,8 @@ def test_peer_mode_nccl_one_rank():
     with H.Context(0, rank=0, nranks=1, unique_id=uid) as c, H.Problem(c, *dims) as p:
         p.set_option(H.HPCCG_OPT_HALO_PEER, 1)
         ref = oracle.generate(*dims)
-        for variant in (0, 1):
+        for variant, halo in ((0, 1), (1, 1), (0, 2)):
+            p.set_option(H.HPCCG_OPT_HALO_PEER, halo)
             p.set_option(H.HPCCG_OPT_CG_VARIANT, variant)
             p.set_vec(H.HPCCG_VEC_X, np.zeros(p.n))
             res = p.solve(150, 1e-12)

@@ -17,13 +17,13 @@ torch = pytest.importorskip("torch")
 from paper_conf_sc_valero_laragmtv24_b200 import hpccg as H  # noqa: E402
 
 
-def run_ranks(nranks, dims, variant, max_iter, tol, timeout=240):
+def run_ranks(nranks, dims, variant, max_iter, tol, timeout=240, halo=1):
     import peer_worker
     ctx = mp.get_context("spawn")
     to_parent = ctx.Queue()
     inbox = [ctx.Queue() for _ in range(nranks)]
     procs = [ctx.Process(target=peer_worker.run,
-                         args=(r, nranks, dims, variant, max_iter, tol, to_parent, inbox[r]))
+                         args=(r, nranks, dims, variant, max_iter, tol, to_parent, inbox[r], halo))
              for r in range(nranks)]
     for pr in procs:
         pr.start()
@@ -79,3 +79,29 @@ def test_three_processes_fixed_iterations():
     x = np.concatenate([res[r][0]["x"] for r in range(P)])
     assert all(res[r][0]["niters"] == 11 for r in range(P))
     assert np.max(np.abs(x - oref["x"])) <= 1e-10
+
+
+@pytest.mark.parametrize("P,dims,max_iter,tol", [(2, (16, 12, 6), 150, 1e-12), (3, (8, 8, 4), 12, 0.0),
+                                                 (2, (10, 6, 1), 40, 0.0)])
+def test_processes_fused_peer_kernels(P, dims, max_iter, tol):
+    """HALO_PEER = 2 across processes: the p update pushes its boundary planes
+    into the other process's halo and raises its flag, the SpMV's boundary
+    blocks wait for it and post p.Ap, the update collects every rank's p.Ap
+    and posts r.r -- bit for bit the loopback HALO_PEER = 1 run, and within
+    the north_star tolerance of the global oracle (nz = 1: every row touches
+    both halos)."""
+    res = run_ranks(P, dims, 0, max_iter, tol, halo=2)
+    ref = oracle.generate(dims[0], dims[1], dims[2] * P)
+    oref = oracle.cg(ref, max_iter, tol)
+    with H.Context(0, nranks=P, loopback=True) as c, H.Problem(c, *dims) as p:
+        p.set_option(H.HPCCG_OPT_HALO_PEER, 1)
+        rl = p.solve(max_iter, tol)
+        xl = p.get_vec(H.HPCCG_VEC_X)
+    for k in range(2):                       # while-graph, per-iteration graph
+        outs = [res[r][k] for r in range(P)]
+        x = np.concatenate([o["x"] for o in outs])
+        for o in outs:
+            assert (o["niters"], o["normr"]) == (rl["niters"], rl["normr"])
+        np.testing.assert_array_equal(x, xl)
+        assert abs(outs[0]["niters"] - oref["niters"]) <= 1
+        assert np.max(np.abs(x - oref["x"])) <= 1e-10

@@ -2,6 +2,7 @@
 usage: probe.py NX NY NZ ITERS 'opt=val,opt=val' ['opt=val,...' ...]
 opts: graph timing while minb l2 waves"""
 import json, os, sys
+import numpy as np
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 from paper_conf_sc_valero_laragmtv24_b200 import hpccg as H
 # option ids (an older libhpccg may lack some; those are skipped)
@@ -15,12 +16,17 @@ KEYS = {"graph": H.HPCCG_OPT_GRAPH, "timing": H.HPCCG_OPT_TIMING, "while": H.HPC
         "smem": H.HPCCG_OPT_SMEM_SOLVE,
         "wu": H.HPCCG_OPT_WHILE_UNROLL,
         "var": H.HPCCG_OPT_CG_VARIANT,
-        "ff": H.HPCCG_OPT_FINISHER_FREE, "nt": H.HPCCG_OPT_SMEM_THREADS}
+        "ff": H.HPCCG_OPT_FINISHER_FREE, "nt": H.HPCCG_OPT_SMEM_THREADS,
+        "serp": H.HPCCG_OPT_SERPENTINE, "peer": H.HPCCG_OPT_HALO_PEER}
 nx, ny, nz, iters = (int(v) for v in sys.argv[1:5])
-ctx = H.Context(0)
+P = int(os.environ.get("PROBE_P", "1"))  # > 1: loopback slabs on one GPU
+if os.environ.get("PROBE_NCCL"):  # 1-rank NCCL communicator (the multi-GPU code path)
+    ctx = H.Context(0, rank=0, nranks=1, unique_id=H.hpccg_unique_id())
+else:
+    ctx = H.Context(0, nranks=P, loopback=True) if P > 1 else H.Context(0)
 p = H.Problem(ctx, nx, ny, nz)
-n, nnz = p.n, p.info["nnz_local"]
-xptr = p.vec_ptr(H.HPCCG_VEC_X)
+n, nnz = p.n * P, p.info["nnz_global"]
+xptr = p.vec_ptr(H.HPCCG_VEC_X) if P == 1 else None  # (noqa)
 for spec in sys.argv[5:]:
     opts = dict(kv.split("=") for kv in spec.split(",") if kv)
     for k, v in opts.items():
@@ -30,7 +36,10 @@ for spec in sys.argv[5:]:
             pass
     best = None
     for _ in range(4):
-        ctx.waxpby(n, 0.0, xptr, 0.0, xptr, xptr)
+        if P == 1:
+            ctx.waxpby(p.n, 0.0, xptr, 0.0, xptr, xptr)
+        else:
+            p.set_vec(H.HPCCG_VEC_X, np.zeros(n))
         r = p.solve(iters + 1, 0.0)
         st = p.stats()
         if best is None or st["total_ms"] < best["total_ms"]:
@@ -48,6 +57,6 @@ for spec in sys.argv[5:]:
     print(json.dumps(out), flush=True)
     for k in opts:
         try:
-            p.set_option(KEYS[k], {"graph": 1, "while": 1, "l2": 1, "waves": 1, "rows": 2, "unroll": 4, "persist": 1, "pdl": 1, "crows": 16384, "smem": 1, "wu": 4, "var": 0, "ff": 1, "nt": 0}.get(k, 0))
+            p.set_option(KEYS[k], {"graph": 1, "while": 1, "l2": 1, "waves": 1, "rows": 2, "unroll": 4, "persist": 1, "pdl": 1, "crows": 16384, "smem": 1, "wu": 4, "var": 0, "ff": 1, "nt": 0, "serp": -1, "peer": 0}.get(k, 0))
         except H.HpccgError:
             pass
