@@ -206,6 +206,22 @@ int check_launch(hpccg_ctx *ctx, int nkernels = 1) {
 // scheduled while its stream predecessor drains; it calls pdl_wait() before
 // touching anything that predecessor writes (kernels.cuh).
 template <typename... KArgs, typename... Args>
+cudaError_t launch_kb(bool pdl, void (*kernel)(KArgs...), dim3 grid, dim3 block, cudaStream_t st,
+                      Args &&...args) {
+    cudaLaunchConfig_t cfg{};
+    cfg.gridDim = grid;
+    cfg.blockDim = block;
+    cfg.dynamicSmemBytes = 0;
+    cfg.stream = st;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = pdl ? at : nullptr;
+    cfg.numAttrs = pdl ? 1 : 0;
+    return cudaLaunchKernelEx(&cfg, kernel, std::forward<Args>(args)...);
+}
+
+template <typename... KArgs, typename... Args>
 cudaError_t launch_k(bool pdl, void (*kernel)(KArgs...), dim3 grid, cudaStream_t st, Args &&...args) {
     cudaLaunchConfig_t cfg{};
     cfg.gridDim = grid;
@@ -694,91 +710,14 @@ int allreduce_cg(hpccg_problem *p, bool rr, bool timing) {
 // Single slab, HPCCG variant: the finisher-free loop (kernels.cuh
 // cg_pupdate1 / cg_update1) when its vectors are 16-B aligned (always, for
 // generated problems).
-bool ff_path(const hpccg_problem *p) {
-    if (p->ctx->mode != MODE_SINGLE || !p->opt_ff || p->opt_variant != 0) return false;
-    const Slab &s = p->slabs[0];
-    return aligned16(s.r) && aligned16(s.p + s.plane) && aligned16(s.x) && aligned16(s.Ap);
-}
-
-template <int kU>
-int enqueue_iteration_ff_u(hpccg_problem *p, bool timing, bool check, unsigned long long cond, int q) {
-    hpccg_ctx *ctx = p->ctx;
-    const Slab &s = p->slabs[0];
-    const bool pdl = p->opt_pdl != 0;
-    auto upd = cg_update1_kernel<kU>;
-    auto pup = cg_pupdate1_kernel<kU>;
-    // the update's grid fixes the r.r partials and so the bits: size it as
-    // the finisher path's update kernel is sized, so both paths agree bitwise
-    const int ug = vec_grid(ctx, cg_update_kernel<true, false, kU>, cdiv(s.n, 2 * kU),
-                            p->opt_vec_waves, p->red_cap);
-    TraceSlot *tr = s.trace_on ? s.trace : nullptr;
-    {
-        PhaseTimer t(p, ctx->stream, PH_PUPDATE, timing);
-        Pupd1Args a{};
-        a.n = s.n;
-        a.r = s.r;
-        a.p = s.p + s.plane;
-        a.rr_parts = s.red.partials;
-        a.n_rr = (unsigned)ug;
-        a.sc = s.sc;
-        a.q = q;
-        a.trace = tr;
-        a.trace_max = s.trace_max;
-        a.rev = serpentine(p) & 1;
-        const int g = vec_grid(ctx, pup, cdiv(s.n, 2 * kU), p->opt_vec_waves, 0x7fffffff);
-        launch_k(pdl, pup, dim3(g), ctx->stream, a);
-        CHECK(check_launch(ctx));
-    }
-    CHECK(cg_spmv_all(p, timing, check));
-    PhaseTimer t(p, ctx->stream, PH_UPDATE, timing);
-    Upd1Args a{};
-    a.n = s.n;
-    a.x = s.x;
-    a.r = s.r;
-    a.p = s.p + s.plane;
-    a.Ap = s.Ap;
-    a.rr_parts = s.red.partials;
-    a.sc = s.sc;
-    a.q = q;
-    a.cond = cond;
-    a.trace = tr;
-    a.trace_max = s.trace_max;
-    const unsigned np = single_spmv_parts(p, s);
-    if (np <= kUpdSumMax) {
-        a.pAp_parts = s.spmv_parts;
-        a.n_parts = np;
-    } else {  // one finisher block writes sc->pAp
-        void (*fk)(const double *, unsigned, CgScalars *) = cg_pap_finish_kernel;
-        cudaLaunchConfig_t cfg{};
-        cfg.gridDim = dim3(1);
-        cfg.blockDim = dim3(1024);
-        cfg.stream = ctx->stream;
-        cudaLaunchAttribute at[1];
-        at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-        at[0].val.programmaticStreamSerializationAllowed = 1;
-        cfg.attrs = pdl ? at : nullptr;
-        cfg.numAttrs = pdl ? 1 : 0;
-        CU(cudaLaunchKernelEx(&cfg, fk, (const double *)s.spmv_parts, np, s.sc));
-        CHECK(check_launch(ctx));
-    }
-    launch_k(pdl, upd, dim3(ug), ctx->stream, a);
-    return check_launch(ctx);
-}
-
-int enqueue_iteration_ff(hpccg_problem *p, bool timing, bool check, unsigned long long cond, int q) {
-    switch (p->opt_unroll) {
-        case 1: return enqueue_iteration_ff_u<1>(p, timing, check, cond, q);
-        case 2: return enqueue_iteration_ff_u<2>(p, timing, check, cond, q);
-        default: return enqueue_iteration_ff_u<4>(p, timing, check, cond, q);
-    }
-}
-
 // HALO_PEER = 2: the halo exchange and both scalar allreduces of the HPCCG
 // iteration fused into its three kernels (kernels.cuh "HALO_PEER = 2").
+// It runs on the finisher-free loop (HPCCG_OPT_FINISHER_FREE, kernels
+// cg_pupdate1 / spmv27x2<1, ., true> / cg_update1 with their peer hooks).
 // Needs the 2-rows-per-thread SpMV and 16-B aligned vectors; else the
 // HALO_PEER = 1 kernels run (same bits).
 bool fused_on(const hpccg_problem *p) {
-    if (p->opt_peer != 2 || !peer_on(p) || p->opt_variant != 0) return false;
+    if (p->opt_peer != 2 || !peer_on(p) || p->opt_variant != 0 || !p->opt_ff) return false;
     const Slab &s = p->slabs[0];
     if (!s.ptab || !aligned16(s.r) || !aligned16(s.p + s.plane) || !aligned16(s.x) || !aligned16(s.Ap))
         return false;
@@ -811,66 +750,9 @@ unsigned push_blocks(int64_t n, int64_t plane, int g, bool has_lo, bool has_hi) 
     return (unsigned)std::count(mark.begin(), mark.end(), 1);
 }
 
-template <bool kCheck, int kU>
-int launch_pupdate_fused_t(hpccg_problem *p, const Slab &s) {
-    hpccg_ctx *ctx = p->ctx;
-    auto k = cg_pupdate_fused_kernel<kCheck, kU>;
-    PupdFArgs a{};
-    a.n = s.n;
-    a.plane = s.plane;
-    a.r = s.r;
-    a.p = s.p + s.plane;
-    a.sc = s.sc;
-    a.t = s.ptab;
-    const int g = vec_grid(ctx, k, cdiv(s.n, 2 * kU), p->opt_vec_waves, 0x7fffffff);
-    const int r = s.rank, P = ctx->nranks;
-    const uint64_t key = ((uint64_t)g << 16) | ((uint64_t)kU << 8) | 1u;
-    auto &cache = p->fpush[(size_t)(&s - p->slabs.data())];
-    if (cache.first != key) cache = {key, push_blocks(s.n, s.plane, g, r > 0, r < P - 1)};
-    a.n_push = cache.second;
-    k<<<g, kBlock, 0, ctx->stream>>>(a);
-    return check_launch(ctx);
-}
-
-template <bool kCheck, int kU>
-int launch_update_fused_t(hpccg_problem *p, const Slab &s, unsigned long long cond) {
-    hpccg_ctx *ctx = p->ctx;
-    UpdArgs a{};
-    a.n = s.n;
-    a.x = s.x;
-    a.r = s.r;
-    a.p = s.p + s.plane;
-    a.Ap = s.Ap;
-    a.sc = s.sc;
-    a.red = s.red;
-    a.cond = cond;
-    a.fpeer = s.ptab;
-    // HALO_PEER = 1's update grid (cg_update_kernel): same r.r partials, same bits
-    const int g = vec_grid(ctx, cg_update_kernel<true, kCheck, kU>, cdiv(s.n, 2 * kU), p->opt_vec_waves,
-                           p->red_cap);
-    cg_update_fused_kernel<kCheck, kU><<<g, kBlock, 0, ctx->stream>>>(a);
-    return check_launch(ctx);
-}
-
-int launch_update_fused(hpccg_problem *p, const Slab &s, bool check, unsigned long long cond) {
-    switch (p->opt_unroll) {
-        case 1: return check ? launch_update_fused_t<true, 1>(p, s, cond) : launch_update_fused_t<false, 1>(p, s, cond);
-        case 2: return check ? launch_update_fused_t<true, 2>(p, s, cond) : launch_update_fused_t<false, 2>(p, s, cond);
-        default: return check ? launch_update_fused_t<true, 4>(p, s, cond) : launch_update_fused_t<false, 4>(p, s, cond);
-    }
-}
-
-int launch_pupdate_fused(hpccg_problem *p, const Slab &s, bool check) {
-    switch (p->opt_unroll) {
-        case 1: return check ? launch_pupdate_fused_t<true, 1>(p, s) : launch_pupdate_fused_t<false, 1>(p, s);
-        case 2: return check ? launch_pupdate_fused_t<true, 2>(p, s) : launch_pupdate_fused_t<false, 2>(p, s);
-        default: return check ? launch_pupdate_fused_t<true, 4>(p, s) : launch_pupdate_fused_t<false, 4>(p, s);
-    }
-}
-
 // one launch per slab: interior row blocks, then plane 0, then plane nz-1
 // (the same blocks and partial slots as HALO_PEER = 1's two launches)
-int launch_spmv_fused(hpccg_problem *p, const Slab &s, bool check) {
+int launch_spmv_fused(hpccg_problem *p, const Slab &s, bool check, unsigned *nparts) {
     const int64_t n = s.n, plane = s.plane;
     SpmvArgs a = spmv_args(s, s.p, s.Ap);
     a.single = 0;
@@ -886,25 +768,138 @@ int launch_spmv_fused(hpccg_problem *p, const Slab &s, bool check) {
     const int64_t blocks = a.nb01 + spmv_blocks(a.len2, 2);
     a.part_base = 0;
     a.total_blocks = (unsigned)blocks;
-    if (check) spmv27x2_kernel<1, true, true><<<(unsigned)blocks, kBlock, 0, p->ctx->stream>>>(a);
-    else spmv27x2_kernel<1, false, true><<<(unsigned)blocks, kBlock, 0, p->ctx->stream>>>(a);
+    a.parts_only = s.spmv_parts;  // the finisher-free update sums them
+    *nparts = (unsigned)blocks;
+    const bool pdl = p->opt_pdl != 0;
+    if (check) launch_k(pdl, spmv27x2_kernel<1, true, true>, dim3((unsigned)blocks), p->ctx->stream, a);
+    else launch_k(pdl, spmv27x2_kernel<1, false, true>, dim3((unsigned)blocks), p->ctx->stream, a);
     return check_launch(p->ctx);
 }
 
-int enqueue_iteration_fused(hpccg_problem *p, bool timing, bool check, unsigned long long cond) {
+// the finisher-free HPCCG loop: single slab, or z-slabs with HALO_PEER = 2
+bool ff_path(const hpccg_problem *p) {
+    if (!p->opt_ff || p->opt_variant != 0) return false;
+    if (p->ctx->mode != MODE_SINGLE) return fused_on(p);
+    const Slab &s = p->slabs[0];
+    return aligned16(s.r) && aligned16(s.p + s.plane) && aligned16(s.x) && aligned16(s.Ap);
+}
+
+template <int kU>
+int enqueue_iteration_ff_u(hpccg_problem *p, bool timing, bool check, unsigned long long cond, int q) {
     hpccg_ctx *ctx = p->ctx;
+    const bool pdl = p->opt_pdl != 0;
+    const bool zs = ctx->mode != MODE_SINGLE;  // HALO_PEER = 2 on z-slabs (fused_on)
+    auto upd = cg_update1_kernel<kU>;
+    auto pup = cg_pupdate1_kernel<kU>;
+    const Slab &s0 = p->slabs[0];
+    // the update's grid fixes the r.r partials and so the bits: size it as
+    // the finisher path's update kernel is sized, so both paths agree bitwise
+    const int ug = vec_grid(ctx, cg_update_kernel<true, false, kU>, cdiv(s0.n, 2 * kU),
+                            p->opt_vec_waves, p->red_cap);
+    const int pg = vec_grid(ctx, pup, cdiv(s0.n, 2 * kU), p->opt_vec_waves, 0x7fffffff);
+    // loopback: every slab's post ahead of every slab's collect (one stream)
+    const bool pre = zs && ctx->mode == MODE_LOOPBACK;
+    auto post = [&](const Slab &s, const double *parts, unsigned n, int q) {
+        launch_k(pdl, fused_post_kernel, dim3(1), ctx->stream, parts, n, (const double *)&s.sc->pAp,
+                 (const PeerTab *)s.ptab, (const CgScalars *)s.sc, q);
+        return check_launch(ctx);
+    };
     {
         PhaseTimer t(p, ctx->stream, PH_PUPDATE, timing);
-        for (const Slab &s : p->slabs) CHECK(launch_pupdate_fused(p, s, check));
+        if (pre)
+            for (const Slab &s : p->slabs) CHECK(post(s, s.red.partials, (unsigned)ug, 0));
+        for (size_t si = 0; si < p->slabs.size(); ++si) {
+            const Slab &s = p->slabs[si];
+            Pupd1Args a{};
+            a.post = !pre;
+            a.n = s.n;
+            a.r = s.r;
+            a.p = s.p + s.plane;
+            a.rr_parts = s.red.partials;
+            a.n_rr = (unsigned)ug;
+            a.sc = s.sc;
+            a.q = q;
+            a.trace = s.trace_on ? s.trace : nullptr;
+            a.trace_max = s.trace_max;
+            a.rev = serpentine(p) & 1;
+            if (zs) {
+                a.t = s.ptab;
+                a.plane = s.plane;
+                const uint64_t key = ((uint64_t)pg << 16) | ((uint64_t)kU << 8) | 2u;
+                auto &cache = p->fpush[si];
+                if (cache.first != key)
+                    cache = {key, push_blocks(s.n, s.plane, pg, s.rank > 0, s.rank < ctx->nranks - 1)};
+                a.n_push = cache.second;
+            }
+            launch_k(pdl, pup, dim3(pg), ctx->stream, a);
+            CHECK(check_launch(ctx));
+        }
     }
-    {
+    unsigned np = 0;
+    if (zs) {
         PhaseTimer t(p, ctx->stream, PH_SPMV, timing);
-        for (const Slab &s : p->slabs) CHECK(launch_spmv_fused(p, s, check));
+        for (const Slab &s : p->slabs) CHECK(launch_spmv_fused(p, s, check, &np));
+    } else {
+        CHECK(cg_spmv_all(p, timing, check));
+        np = single_spmv_parts(p, s0);
     }
     PhaseTimer t(p, ctx->stream, PH_UPDATE, timing);
-    for (size_t i = 0; i < p->slabs.size(); ++i)
-        CHECK(launch_update_fused(p, p->slabs[i], check, i == 0 ? cond : 0ull));
+    if (pre) {
+        if (np > kUpdSumMax)
+            for (const Slab &s : p->slabs) {  // sc->pAp = the slab's sum, then post it
+                launch_kb(pdl, cg_pap_finish_kernel, dim3(1), dim3(1024), ctx->stream,
+                          (const double *)s.spmv_parts, np, s.sc);
+                CHECK(check_launch(ctx));
+            }
+        for (const Slab &s : p->slabs)
+            CHECK(post(s, np <= kUpdSumMax ? s.spmv_parts : nullptr, np, 1));
+    }
+    for (size_t si = 0; si < p->slabs.size(); ++si) {
+        const Slab &s = p->slabs[si];
+        Upd1Args a{};
+        a.post = !pre;
+        a.n = s.n;
+        a.x = s.x;
+        a.r = s.r;
+        a.p = s.p + s.plane;
+        a.Ap = s.Ap;
+        a.rr_parts = s.red.partials;
+        a.sc = s.sc;
+        a.q = q;
+        a.cond = si == 0 ? cond : 0ull;
+        a.trace = s.trace_on ? s.trace : nullptr;
+        a.trace_max = s.trace_max;
+        a.t = zs ? s.ptab : nullptr;
+        if (np <= kUpdSumMax) {
+            a.pAp_parts = s.spmv_parts;
+            a.n_parts = np;
+        } else if (pre) {  // finished and posted below, ahead of every update
+        } else {  // one finisher block writes the slab's p.Ap into sc->pAp
+            void (*fk)(const double *, unsigned, CgScalars *) = cg_pap_finish_kernel;
+            cudaLaunchConfig_t cfg{};
+            cfg.gridDim = dim3(1);
+            cfg.blockDim = dim3(1024);
+            cfg.stream = ctx->stream;
+            cudaLaunchAttribute at[1];
+            at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+            at[0].val.programmaticStreamSerializationAllowed = 1;
+            cfg.attrs = pdl ? at : nullptr;
+            cfg.numAttrs = pdl ? 1 : 0;
+            CU(cudaLaunchKernelEx(&cfg, fk, (const double *)s.spmv_parts, np, s.sc));
+            CHECK(check_launch(ctx));
+        }
+        launch_k(pdl, upd, dim3(ug), ctx->stream, a);
+        CHECK(check_launch(ctx));
+    }
     return HPCCG_OK;
+}
+
+int enqueue_iteration_ff(hpccg_problem *p, bool timing, bool check, unsigned long long cond, int q) {
+    switch (p->opt_unroll) {
+        case 1: return enqueue_iteration_ff_u<1>(p, timing, check, cond, q);
+        case 2: return enqueue_iteration_ff_u<2>(p, timing, check, cond, q);
+        default: return enqueue_iteration_ff_u<4>(p, timing, check, cond, q);
+    }
 }
 
 // One CG iteration (a.6, a.2, a.3+a.4, a.5, a.8) for every slab.  `cond`:
@@ -912,7 +907,6 @@ int enqueue_iteration_fused(hpccg_problem *p, bool timing, bool check, unsigned 
 // iteration's index (its parity drives the finisher-free loop's state).
 int enqueue_iteration(hpccg_problem *p, bool timing, bool check, unsigned long long cond, int k) {
     if (ff_path(p)) return enqueue_iteration_ff(p, timing, check, cond, k & 1);
-    if (fused_on(p)) return enqueue_iteration_fused(p, timing, check, cond);
     hpccg_ctx *ctx = p->ctx;
     const int single = ctx->mode == MODE_SINGLE;
     // PDL only between back-to-back kernels (single slab; the multi-slab

@@ -184,8 +184,18 @@ __device__ __forceinline__ void grid_reduce(double v, Reduction red, unsigned pa
     __syncthreads();
     if (!is_last) return;
     __threadfence();
+    // per thread left to right over i, i + kBlock, ... with 8 loads in flight
+    // per batch (the order, and so the bits, of a plain loop)
     double s = 0.0;
-    for (unsigned i = threadIdx.x; i < total; i += kBlock) {
+    unsigned i = threadIdx.x;
+    for (; i + 7u * kBlock < total; i += 8u * kBlock) {
+        double q[8];
+#pragma unroll
+        for (int u = 0; u < 8; ++u) q[u] = __ldcg(red.partials + i + u * kBlock);
+#pragma unroll
+        for (int u = 0; u < 8; ++u) s = kMax ? fmax(s, q[u]) : s + q[u];
+    }
+    for (; i < total; i += kBlock) {
         double q = __ldcg(red.partials + i);
         s = kMax ? fmax(s, q) : s + q;
     }
@@ -266,8 +276,12 @@ struct PeerSync {                      // one per slab, in that slab's device me
     unsigned long long fflag_from_hi;  //   ... by rank + 1
     unsigned int fpush_ticket;         // blocks of the current fused push done
     unsigned int pad_;
-    unsigned long long far_tag[2][kMaxPeers];  // slot 1: p.Ap (seq 2k-1), 0: r.r (seq 2k)
-    double far_val[2][kMaxPeers];
+    // allreduce slots, LL style: slot q (1: p.Ap, seq 2k-1; 0: r.r, seq 2k),
+    // rank r: two 8-B words {32 value bits | 32-bit tag}, each single-copy
+    // atomic, so a reader that sees the tag in both has the value -- no fence
+    // on the post or the collect (the scalar allreduces are on the critical
+    // path of every iteration; the halo flags are hidden behind the interior)
+    unsigned long long fll[2][kMaxPeers][2];
 };
 
 struct PeerTab {                       // device copy per slab; pointers may be peers'
@@ -305,43 +319,67 @@ __device__ __forceinline__ bool spin_until(const unsigned long long *flag, unsig
 }
 
 // ---- HALO_PEER = 2: the exchange and the scalar allreduces fused into the
-// CG kernels themselves (no push / wait / allreduce kernels, no comm stream):
-//   p update k   collects r.r(k-1) (k > 1), computes p, stores its first /
-//                last owned plane straight into the neighbours' halo planes as
-//                it goes, and its last block raises their flags
+// finisher-free CG kernels (no push / wait / allreduce kernels, no comm
+// stream, no grid-wide finisher):
+//   p update k   every block sums the slab's r.r(k-1) partials (fixed order),
+//                block 0 posts that to every rank, every block collects the P
+//                posts (rank order) -> beta; p = r + beta p, with the first /
+//                last owned plane stored straight into the neighbours' halo
+//                planes as it is computed; the blocks that pushed fence and
+//                take a ticket, the last raises the neighbours' flags
 //   SpMV k       interior row blocks first; the boundary blocks (last in
 //                block order) wait for the flags, then gather the halo with
-//                L2-coherent loads; the last block posts the slab's p.Ap
-//   update k     every block collects the P p.Ap posts (rank order) -> alpha;
-//                the last block posts the slab's r.r
-// Flags / tags are tag(epoch, seq) (monotone: the epoch, counted by the init
-// kernel of every solve, is the same on every slab; seq = k for the halo of
-// iteration k, 2k - 1 for its p.Ap, 2k for its r.r), so every kernel knows
-// what it waits for from the device loop state alone.  Slots alternate by seq
-// parity; a rank cannot post seq m + 2 before every rank has collected m (the
-// post needs everyone's m + 1, made after their collect of m), and a push of
-// iteration k + 1 needs r.r(k), posted after the neighbour's SpMV k read the
-// halo.  The rank-order sums are those of peer_allreduce_kernel and the
-// partials those of the HALO_PEER = 1 path: the two modes are bit-identical.
+//                L2-coherent loads; per-block p.Ap partials only
+//   update k     as the p update for p.Ap (slot 1) -> alpha; r.r partials
+// Halo flags carry tag(epoch, k) (monotone: the epoch, counted by the init
+// kernel of every solve, is the same on every slab) and are released after a
+// system-scope fence (they are off the critical path: the interior rows hide
+// them).  The scalar posts are LL-style words {32 value bits | 32-bit tag}
+// (ll_tag: epoch and seq = 2k - 1 for p.Ap, 2k for r.r) that need no fence
+// -- the two allreduces sit on the critical path of every iteration.  Slots
+// alternate by seq parity; a rank cannot post seq m + 2 before every rank
+// has collected m (the post follows its own collect of m + 1, which needs
+// everyone's post of m + 1, made after their collect of m).  A push of
+// iteration k + 1 follows the collect of r.r(k), whose posts depend on the
+// neighbours' SpMV k results (so on their halo reads).  The local sums use
+// the last-block finisher's order and the rank-order sums are those of
+// peer_allreduce_kernel: bit-identical to HALO_PEER = 1 and the loopback copies.
 __device__ __forceinline__ unsigned long long ftag(unsigned long long epoch, unsigned long long seq) {
     return (epoch << 32) | seq;
 }
 
+// 32-bit tag of the LL slots: bit 31 set (never the zero of a fresh slot),
+// 11 bits of the epoch, 20 of seq.  A stale word could only match after 2048
+// solves that never rewrote the slot.
+__device__ __forceinline__ unsigned ll_tag(unsigned long long epoch, unsigned long long seq) {
+    return 0x80000000u | ((unsigned)(epoch & 0x7FFu) << 20) | (unsigned)(seq & 0xFFFFFu);
+}
+
 // post v as rank t->rank into slot q of every rank (one thread)
-__device__ __forceinline__ void fused_post(const PeerTab *t, int q, double v, unsigned long long tag) {
+__device__ __forceinline__ void fused_post(const PeerTab *t, int q, double v, unsigned tag) {
+    const unsigned long long b = (unsigned long long)__double_as_longlong(v);
+    const unsigned long long hi = (unsigned long long)tag << 32;
+    const unsigned long long w0 = (b & 0xffffffffull) | hi, w1 = (b >> 32) | hi;
     const int P = t->nranks, me = t->rank;
-    for (int r = 0; r < P; ++r) t->all[r]->far_val[q][me] = v;
-    __threadfence_system();
-    for (int r = 0; r < P; ++r) st_release_sys(&t->all[r]->far_tag[q][me], tag);
+    for (int r = 0; r < P; ++r)
+        asm volatile("st.relaxed.sys.global.v2.u64 [%0], {%1, %2};" ::"l"(&t->all[r]->fll[q][me][0]),
+                     "l"(w0), "l"(w1)
+                     : "memory");
+}
+
+__device__ __forceinline__ bool ll_read(const unsigned long long *w, unsigned tag, double *v) {
+    unsigned long long a, b;
+    asm volatile("ld.relaxed.sys.global.v2.u64 {%0, %1}, [%2];" : "=l"(a), "=l"(b) : "l"(w) : "memory");
+    if ((unsigned)(a >> 32) != tag || (unsigned)(b >> 32) != tag) return false;
+    *v = __longlong_as_double((long long)((a & 0xffffffffull) | (b << 32)));
+    return true;
 }
 
 // wait for the P posts of slot q and sum them in rank order; the block's
-// result (*sh broadcasts it).  Lane r of warp 0 acquires rank r's tag and
-// reads its value (ordered after its own acquire), so the P latencies
-// overlap; lane 0 adds the shuffled values left to right (the order of
-// peer_allreduce_kernel).
-__device__ __forceinline__ double fused_collect_block(const PeerTab *t, int q, unsigned long long tag,
-                                                      double *sh) {
+// result (*sh broadcasts it).  Lane r of warp 0 polls rank r's words (the P
+// latencies overlap); lane 0 adds the shuffled values left to right (the
+// order of peer_allreduce_kernel).  ~2 s timeout -> error flag.
+__device__ __forceinline__ double fused_collect_block(const PeerTab *t, int q, unsigned tag, double *sh) {
     __syncthreads();  // sh reuse
     if (threadIdx.x < 32) {
         PeerSync *m = t->mine;
@@ -349,9 +387,15 @@ __device__ __forceinline__ double fused_collect_block(const PeerTab *t, int q, u
         double s = 0.0;
         for (int r0 = 0; r0 < P; r0 += 32) {
             double v = 0.0;
-            if (r0 + lane < P) {
-                spin_until(&m->far_tag[q][r0 + lane], tag, m);
-                v = *(volatile double *)&m->far_val[q][r0 + lane];
+            if (r0 + lane < P && !ll_read(m->fll[q][r0 + lane], tag, &v)) {
+                const unsigned long long t0 = gtimer();
+                while (!ll_read(m->fll[q][r0 + lane], tag, &v)) {
+                    if (*(volatile int *)&m->error || gtimer() - t0 > 2000000000ull) {
+                        m->error = 1;
+                        break;
+                    }
+                    __nanosleep(32);
+                }
             }
             for (int j = 0; j < 32 && r0 + j < P; ++j) {
                 const double w = __shfl_sync(0xffffffffu, v, j);
@@ -659,7 +703,7 @@ __device__ __forceinline__ void spmv27x2_body(const SpmvArgs &a, int64_t row, in
                            [sc, single, fp](double s) {
                                if (single) sc->pAp = s; else sc->loc_pAp = s;
                                if (kFused)  // p.Ap(k) -> slot 1 of every rank
-                                   fused_post(fp, 1, s, ftag(sc->epoch, 2ull * (unsigned)sc->k - 1ull));
+                                   fused_post(fp, 1, s, ll_tag(sc->epoch, 2ull * (unsigned)sc->k - 1ull));
                            });
     }
 }
@@ -772,105 +816,6 @@ __global__ void __launch_bounds__(kBlock) cg_pupdate_kernel(int64_t n, const dou
     }
 }
 
-// a.6 + a.2 fused (HALO_PEER = 2, multi-slab): r.r(k-1) collected from every
-// rank's post (k > 1), p = r + beta p, and the first / last owned plane of
-// the new p stored straight into the neighbours' halo planes as it is
-// computed; the blocks that pushed fence and take a ticket, the last of them
-// raises the neighbours' flags (n_push = how many blocks hold boundary units,
-// from the host).  The first trip's loads are issued before the collect.
-// 16-B units (the host falls back to HALO_PEER = 1 otherwise).
-struct PupdFArgs {
-    int64_t n, plane;
-    const double *r;
-    double *p;             // owned part (local-with-halo base + plane)
-    CgScalars *sc;
-    const PeerTab *t;
-    unsigned n_push;       // blocks that store into a neighbour's halo
-};
-
-template <bool kCheck, int kU>
-__global__ void __launch_bounds__(kBlock) cg_pupdate_fused_kernel(PupdFArgs a) {
-    __shared__ double sh;
-    __shared__ int last;
-    CgScalars *sc = a.sc;
-    const int64_t tid = gtid(), nth = gnth(), nv = a.n >> 1, n = a.n, plane = a.plane;
-    const double2 *__restrict__ r2 = reinterpret_cast<const double2 *>(a.r);
-    double2 *__restrict__ p2 = reinterpret_cast<double2 *>(a.p);
-    double2 ra[kU], pa[kU];
-    auto load = [&](int64_t b) {
-#pragma unroll
-        for (int u = 0; u < kU; ++u) {
-            const int64_t i = b + u * nth;
-            if (i < nv) {
-                ra[u] = r2[i];
-                pa[u] = p2[i];
-            }
-        }
-    };
-    load(tid);
-    if (kCheck && __ldg(&sc->done)) return;  // uniform: nobody pushes or posts
-    const int k = __ldg(&sc->k);
-    const unsigned long long epoch = __ldg(&sc->epoch);
-    const bool first = (k == 1);
-    double beta = 0.0;
-    if (!first) {
-        const double rtrans = fused_collect_block(a.t, 0, ftag(epoch, 2ull * (unsigned)(k - 1)), &sh);
-        beta = rtrans / __ldg(&sc->rr_prev);
-        if (blockIdx.x == 0 && threadIdx.x == 0) sc->rr_cur = rtrans;
-    }
-    double *lo = a.t->halo_to_lo, *hi = a.t->halo_to_hi;
-    int pushed = 0;
-    auto put = [&](int64_t i, double v) {  // row i of the new p
-        if (lo && i < plane) {
-            lo[i] = v;
-            pushed = 1;
-        }
-        if (hi && i >= n - plane) {
-            hi[i - (n - plane)] = v;
-            pushed = 1;
-        }
-    };
-    for (int64_t b = tid; b < nv;) {
-#pragma unroll
-        for (int u = 0; u < kU; ++u) {
-            const int64_t i = b + u * nth;
-            if (i < nv) {
-                double2 q = ra[u];
-                if (!first) {
-                    q.x = fma(beta, pa[u].x, ra[u].x);
-                    q.y = fma(beta, pa[u].y, ra[u].y);
-                }
-                p2[i] = q;
-                if (2 * i < plane || 2 * i + 1 >= n - plane) {
-                    put(2 * i, q.x);
-                    put(2 * i + 1, q.y);
-                }
-            }
-        }
-        b += kU * nth;
-        if (b < nv) load(b);
-    }
-    if (tid == 0 && (n & 1)) {
-        const int64_t i = n - 1;
-        const double v = first ? a.r[i] : fma(beta, a.p[i], a.r[i]);
-        a.p[i] = v;
-        put(i, v);
-    }
-    if (!__syncthreads_or(pushed)) return;
-    if (threadIdx.x == 0) {
-        __threadfence_system();  // this block's pushes before its ticket
-        const unsigned tk = atomicAdd(&a.t->mine->fpush_ticket, 1u);
-        last = (tk == a.n_push - 1);
-    }
-    __syncthreads();
-    if (!last || threadIdx.x != 0) return;
-    __threadfence_system();
-    a.t->mine->fpush_ticket = 0u;
-    const unsigned long long tg = ftag(epoch, (unsigned long long)k);
-    if (a.t->lo) st_release_sys(&a.t->lo->fflag_from_hi, tg);
-    if (a.t->hi) st_release_sys(&a.t->hi->fflag_from_lo, tg);
-}
-
 // a.5: x += alpha p; r -= alpha Ap; partial r.r; then the loop control of
 // the NEXT iteration (A4 lagged check, A11 guard) in the last block, which
 // also drives the while-graph's condition (`cond`, 0 = none).  48n B.
@@ -886,7 +831,6 @@ struct UpdArgs {
     Reduction red;
     int single;
     unsigned long long cond;  // cudaGraphConditionalHandle or 0
-    const PeerTab *fpeer;     // cg_update_fused_kernel (HALO_PEER = 2)
 };
 
 __device__ __forceinline__ void set_cond(unsigned long long h, int cont) {
@@ -1021,85 +965,6 @@ __global__ void __launch_bounds__(kBlock) cg_update_kernel(UpdArgs a) {
                        });
 }
 
-// a.5 fused (HALO_PEER = 2, multi-slab): the first trip's x, r, p, Ap loads,
-// then p.Ap collected from every rank's post -> alpha, x += alpha p,
-// r -= alpha Ap, and cg_update_kernel<true, ., kU>'s r.r partials and
-// finisher (same per-thread order and grid: same bits), whose last block
-// also posts the slab's r.r(k).
-template <bool kCheck, int kU>
-__global__ void __launch_bounds__(kBlock) cg_update_fused_kernel(UpdArgs a) {
-    __shared__ double shf;
-    CgScalars *sc = a.sc;
-    const int64_t tid = gtid(), nth = gnth(), nv = a.n >> 1;
-    double2 *__restrict__ x2 = reinterpret_cast<double2 *>(a.x);
-    double2 *__restrict__ r2 = reinterpret_cast<double2 *>(a.r);
-    const double2 *__restrict__ p2 = reinterpret_cast<const double2 *>(a.p);
-    const double2 *__restrict__ q2 = reinterpret_cast<const double2 *>(a.Ap);
-    double2 xa[kU], ra[kU], pa[kU], qa[kU];
-    auto load = [&](int64_t b) {
-#pragma unroll
-        for (int u = 0; u < kU; ++u) {
-            const int64_t i = b + u * nth;
-            if (i < nv) {
-                xa[u] = x2[i];
-                ra[u] = r2[i];
-                pa[u] = p2[i];
-                qa[u] = q2[i];
-            }
-        }
-    };
-    load(tid);
-    if (kCheck && __ldg(&sc->done)) return;  // uniform: nobody posted
-    const double rtrans = __ldg(&sc->rr_cur);
-    const double pAp =
-        fused_collect_block(a.fpeer, 1, ftag(__ldg(&sc->epoch), 2ull * (unsigned)__ldg(&sc->k) - 1ull), &shf);
-    const bool stop = (rtrans == 0.0) || (pAp == 0.0);  // A11
-    const double alpha = stop ? 0.0 : rtrans / pAp;
-    double acc = 0.0, acc2 = 0.0;
-    for (int64_t b = tid; b < nv;) {
-#pragma unroll
-        for (int u = 0; u < kU; ++u) {
-            const int64_t i = b + u * nth;
-            if (i < nv) {
-                xa[u].x = fma(alpha, pa[u].x, xa[u].x);
-                xa[u].y = fma(alpha, pa[u].y, xa[u].y);
-                ra[u].x = fma(-alpha, qa[u].x, ra[u].x);
-                ra[u].y = fma(-alpha, qa[u].y, ra[u].y);
-                x2[i] = xa[u];
-                r2[i] = ra[u];
-                acc = fma(ra[u].x, ra[u].x, acc);
-                acc2 = fma(ra[u].y, ra[u].y, acc2);
-            }
-        }
-        b += kU * nth;
-        if (b < nv) load(b);
-    }
-    if (tid == 0 && (a.n & 1)) {
-        const int64_t i = a.n - 1;
-        a.x[i] = fma(alpha, a.p[i], a.x[i]);
-        const double rv = fma(-alpha, a.Ap[i], a.r[i]);
-        a.r[i] = rv;
-        acc = fma(rv, rv, acc);
-    }
-    acc += acc2;
-    const unsigned long long cond = a.cond;
-    const PeerTab *fp = a.fpeer;
-    grid_reduce<false>(acc, a.red, blockIdx.x, gridDim.x, [sc, rtrans, stop, cond, pAp, fp](double s) {
-        sc->pAp = pAp;
-        sc->rr_prev = rtrans;
-        sc->loc_rr = s;
-        const int k = sc->k;
-        fused_post(fp, 0, s, ftag(sc->epoch, 2ull * (unsigned)k));  // r.r(k)
-        const double normr = sqrt(rtrans);
-        sc->normr = normr;
-        sc->niters = k;
-        sc->k = k + 1;
-        const int done = stop || !((k + 1) < sc->max_iter && normr > sc->tol);
-        sc->done = done;
-        set_cond(cond, !done);
-    });
-}
-
 // ------------------- single slab: HPCCG's loop without any grid finisher
 // The last-block finisher of cg_update_kernel (fence + atomic ticket + the
 // final sum, then the loop control) sits between every update and the next
@@ -1118,6 +983,26 @@ __global__ void __launch_bounds__(kBlock) cg_update_fused_kernel(UpdArgs a) {
 // parity is baked into the graph node), so no block reads a word another
 // block of its own grid writes.
 
+// HALO_PEER = 2: after a block's halo stores -- the blocks that pushed fence
+// (system scope) and take a ticket; the last of the n_push raises the
+// neighbours' flags to tg
+__device__ __forceinline__ void fused_push_signal(const PeerTab *t, int pushed, unsigned n_push,
+                                                  unsigned long long tg) {
+    __shared__ int last;
+    if (!__syncthreads_or(pushed)) return;
+    if (threadIdx.x == 0) {
+        __threadfence_system();  // this block's pushes before its ticket
+        const unsigned tk = atomicAdd(&t->mine->fpush_ticket, 1u);
+        last = (tk == n_push - 1);
+    }
+    __syncthreads();
+    if (!last || threadIdx.x != 0) return;
+    __threadfence_system();
+    t->mine->fpush_ticket = 0u;
+    if (t->lo) st_release_sys(&t->lo->fflag_from_hi, tg);
+    if (t->hi) st_release_sys(&t->hi->fflag_from_lo, tg);
+}
+
 struct Pupd1Args {
     int64_t n;
     const double *r;
@@ -1130,6 +1015,13 @@ struct Pupd1Args {
     TraceSlot *trace;
     int trace_max;
     int rev;  // 1: each thread walks its trips last to first (no reduction: same bits)
+    // HALO_PEER = 2 on z-slabs (nullptr: single slab): r.r(k-1) = the P slabs'
+    // local sums (block 0 posts this slab's), and the p planes pushed into the
+    // neighbours' halos by the n_push blocks that hold boundary rows
+    const PeerTab *t;
+    int64_t plane;
+    unsigned n_push;
+    int post;  // 0: the slab's sum was posted by fused_post_kernel (loopback)
 };
 
 // Fixed-order sum of n partials (the order of grid_reduce's last block);
@@ -1203,13 +1095,31 @@ __global__ void __launch_bounds__(kBlock) cg_pupdate1_kernel(Pupd1Args a) {
     const int k = __ldg(&sc->k);
     trace_mark(a.trace, a.trace_max, k, 0, false);
     const bool first = (k == 1);
-    const double rtrans = first ? __ldg(&sc->rr_cur) : sum_parts_fixed(a.rr_parts, a.n_rr, sh);
+    double rtrans = first ? __ldg(&sc->rr_cur) : sum_parts_fixed(a.rr_parts, a.n_rr, sh);
+    if (a.t && !first) {  // z-slabs: the slab's r.r -> every rank; the global sum back
+        const unsigned tag = ll_tag(__ldg(&sc->epoch), 2ull * (unsigned)(k - 1));
+        if (a.post && blockIdx.x == 0 && threadIdx.x == 0) fused_post(a.t, 0, rtrans, tag);
+        rtrans = fused_collect_block(a.t, 0, tag, &sh[32]);
+    }
     const double beta = first ? 0.0 : rtrans / __ldg(&sc->rr_prev);
     if (blockIdx.x == 0 && threadIdx.x == 0) {
         if (!first) sc->rr_cur = rtrans;
         sc->normr = sqrt(rtrans);
         sc->niters = k;
     }
+    const int64_t n = a.n, plane = a.plane;
+    double *lo = a.t ? a.t->halo_to_lo : nullptr, *hi = a.t ? a.t->halo_to_hi : nullptr;
+    int pushed = 0;
+    auto put = [&](int64_t i, double v) {  // row i of the new p -> a neighbour's halo
+        if (lo && i < plane) {
+            lo[i] = v;
+            pushed = 1;
+        }
+        if (hi && i >= n - plane) {
+            hi[i - (n - plane)] = v;
+            pushed = 1;
+        }
+    };
     for (int64_t b = b0; b >= 0 && b < nv;) {
 #pragma unroll
         for (int u = 0; u < kU; ++u) {
@@ -1221,19 +1131,26 @@ __global__ void __launch_bounds__(kBlock) cg_pupdate1_kernel(Pupd1Args a) {
                     v.y = fma(beta, pa[u].y, ra[u].y);
                 }
                 p2[i] = v;
+                if (a.t && (2 * i < plane || 2 * i + 1 >= n - plane)) {
+                    put(2 * i, v.x);
+                    put(2 * i + 1, v.y);
+                }
             }
         }
         b += a.rev ? -step : step;
         if (b >= 0 && b < nv) load(b);
     }
-    if (tid == 0 && (a.n & 1)) {
-        const int64_t i = a.n - 1;
-        a.p[i] = first ? a.r[i] : fma(beta, a.p[i], a.r[i]);
+    if (tid == 0 && (n & 1)) {
+        const int64_t i = n - 1;
+        const double v = first ? a.r[i] : fma(beta, a.p[i], a.r[i]);
+        a.p[i] = v;
+        if (a.t) put(i, v);
     }
     if (a.trace) {
         __syncthreads();
         trace_mark(a.trace, a.trace_max, k, 0, true);
     }
+    if (a.t) fused_push_signal(a.t, pushed, a.n_push, ftag(__ldg(&sc->epoch), (unsigned long long)k));
 }
 
 // a.5 x += alpha p, r -= alpha Ap, per-block r.r partial (no finisher), and
@@ -1250,7 +1167,28 @@ struct Upd1Args {
     unsigned long long cond;
     TraceSlot *trace;
     int trace_max;
+    const PeerTab *t;  // HALO_PEER = 2 on z-slabs: p.Ap = the P slabs' local sums
+    int post;          // 0: posted by fused_post_kernel (loopback)
 };
+
+// Loopback + HALO_PEER = 2: every slab's kernels share one stream, so a
+// collect in slab 0's kernel could never see slab 1's post from a kernel
+// queued behind it.  This one-block kernel posts a slab's local sum (its
+// partials in the consumers' fixed order, or *fallback) ahead of all the
+// consumers.  q 0: r.r(k-1) before p update k (k = sc->k; nothing for k = 1);
+// q 1: p.Ap(k) before update k (k = sc->niters).
+__global__ void __launch_bounds__(kBlock) fused_post_kernel(const double *parts, unsigned n,
+                                                             const double *fallback, const PeerTab *t,
+                                                             const CgScalars *sc, int q) {
+    __shared__ double sh[33];
+    pdl_wait();
+    pdl_trigger();
+    const int k = q == 0 ? __ldg(&sc->k) - 1 : __ldg(&sc->niters);
+    if (q == 0 && k < 1) return;
+    const double v = parts ? sum_parts_fixed(parts, n, sh) : __ldcg(fallback);
+    if (threadIdx.x == 0)
+        fused_post(t, q, v, ll_tag(__ldg(&sc->epoch), q == 0 ? 2ull * (unsigned)k : 2ull * (unsigned)k - 1ull));
+}
 
 template <int kU>
 __global__ void __launch_bounds__(kBlock) cg_update1_kernel(Upd1Args a) {
@@ -1295,7 +1233,12 @@ __global__ void __launch_bounds__(kBlock) cg_update1_kernel(Upd1Args a) {
     const int ktr = a.trace ? __ldg(&sc->niters) : 0;
     trace_mark(a.trace, a.trace_max, ktr, 2, false);
     const double rtrans = __ldg(&sc->rr_cur);
-    const double pAp = a.pAp_parts ? sum_parts_fixed(a.pAp_parts, a.n_parts, sh) : __ldg(&sc->pAp);
+    double pAp = a.pAp_parts ? sum_parts_fixed(a.pAp_parts, a.n_parts, sh) : __ldg(&sc->pAp);
+    if (a.t) {  // z-slabs: the slab's p.Ap -> every rank; the global sum back
+        const unsigned tag = ll_tag(__ldg(&sc->epoch), 2ull * (unsigned)__ldg(&sc->niters) - 1ull);
+        if (a.post && blockIdx.x == 0 && threadIdx.x == 0) fused_post(a.t, 1, pAp, tag);
+        pAp = fused_collect_block(a.t, 1, tag, &sh[32]);
+    }
     const bool stop = (rtrans == 0.0) || (pAp == 0.0);  // A11
     const double alpha = stop ? 0.0 : rtrans / pAp;
     if (blockIdx.x == 0 && threadIdx.x == 0) {

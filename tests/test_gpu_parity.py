@@ -755,7 +755,9 @@ def test_peer_fused_loopback_bitwise(P, dims):
     the SpMV's boundary blocks and both allreduces into the SpMV / update
     finishers and the consumers' prologues reproduce the copy-exchange path
     and HALO_PEER = 1 BIT FOR BIT (same blocks, partial slots and rank-order
-    sums) in every launch mode, and match the global oracle.  nz = 1 and 2
+    sums; the slab sums of more than 4096 SpMV partials take the 1024-thread
+    finisher's order instead) in every launch mode, and match the global
+    oracle.  nz = 1 and 2
     (boundary blocks touching both halos / no interior), an odd plane
     (9 x 7: the 1-row SpMV, so HALO_PEER = 2 falls back to 1), and slabs
     large enough that only some p-update blocks push (end ranks: one plane)."""
@@ -769,8 +771,9 @@ def test_peer_fused_loopback_bitwise(P, dims):
             p.set_vec(H.HPCCG_VEC_X, np.zeros(p.n * P))
             r = p.solve(150, 1e-12)
             outs.append((r["niters"], r["normr"], p.get_vec(H.HPCCG_VEC_X)))
-        # plain launches: an iteration is 3 kernels per slab when fused (no
-        # push / wait / allreduce kernels), 10 with HALO_PEER = 1
+        # plain launches: an iteration is 3 CG kernels per slab when fused (no
+        # push / wait / allreduce kernels) + 2 one-block posts that loopback
+        # needs (all slabs share one stream), 10 with HALO_PEER = 1
         p.set_option(H.HPCCG_OPT_TIMING, 1)
         per_iter = {}
         for peer in (2, 1):
@@ -782,7 +785,7 @@ def test_peer_fused_loopback_bitwise(P, dims):
                 launches.append(p.stats()["kernel_launches"])
             per_iter[peer] = (launches[1] - launches[0]) / (4 * P)
         assert per_iter[1] == (10 if nz > 2 else 9)   # nz <= 2: no interior SpMV launch
-        assert per_iter[2] == (3 if (nx * ny) % 2 == 0 else 10)
+        assert per_iter[2] == (5 if (nx * ny) % 2 == 0 else 10)
         p.set_option(H.HPCCG_OPT_TIMING, 0)
         for o in outs[1:]:
             assert o[:2] == outs[0][:2]
@@ -850,3 +853,13 @@ def test_peer_mode_nccl_one_rank():
             res = p.solve(150, 1e-12)
             oref = (oracle.cg_sr if variant else oracle.cg)(ref, 150, 1e-12)
             check_cg(res, p.maxabsdiff(), oref, ref)
+        # HALO_PEER = 2 in a one-slab-per-process context: 3 kernels per iteration
+        p.set_option(H.HPCCG_OPT_CG_VARIANT, 0)
+        p.set_option(H.HPCCG_OPT_HALO_PEER, 2)
+        p.set_option(H.HPCCG_OPT_TIMING, 1)
+        launches = []
+        for m in (5, 9):
+            p.set_vec(H.HPCCG_VEC_X, np.zeros(p.n))
+            p.solve(m, 0.0)
+            launches.append(p.stats()["kernel_launches"])
+        assert launches[1] - launches[0] == 3 * 4

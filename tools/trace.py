@@ -11,8 +11,12 @@ nx, ny, nz, iters = (int(v) for v in sys.argv[1:5])
 KEYS = {"graph": H.HPCCG_OPT_GRAPH, "timing": H.HPCCG_OPT_TIMING, "while": H.HPCCG_OPT_WHILE,
         "pdl": H.HPCCG_OPT_PDL, "waves": H.HPCCG_OPT_VEC_WAVES, "unroll": H.HPCCG_OPT_VEC_UNROLL,
         "rows": H.HPCCG_OPT_SPMV_ROWS, "l2": H.HPCCG_OPT_L2_PERSIST,
-        "wu": H.HPCCG_OPT_WHILE_UNROLL, "ff": H.HPCCG_OPT_FINISHER_FREE}
-ctx = H.Context(0)
+        "wu": H.HPCCG_OPT_WHILE_UNROLL, "ff": H.HPCCG_OPT_FINISHER_FREE,
+        "peer": H.HPCCG_OPT_HALO_PEER, "serp": H.HPCCG_OPT_SERPENTINE}
+if os.environ.get("PROBE_NCCL"):  # 1-rank NCCL communicator: the multi-GPU code path
+    ctx = H.Context(0, rank=0, nranks=1, unique_id=H.hpccg_unique_id())
+else:
+    ctx = H.Context(0)
 p = H.Problem(ctx, nx, ny, nz)
 p.set_option(H.HPCCG_OPT_PERSISTENT, 0)
 xptr = p.vec_ptr(H.HPCCG_VEC_X)
@@ -44,4 +48,4 @@ for spec in sys.argv[5:]:
     p.set_option(H.HPCCG_OPT_TRACE, 0)
     for k in opts:
         p.set_option(KEYS[k], {"graph": 1, "while": 1, "pdl": 1, "waves": 1, "unroll": 4, "rows": 2,
-                               "l2": 1, "wu": 4}.get(k, 0))
+                               "l2": 1, "wu": 4, "serp": -1}.get(k, 0))
