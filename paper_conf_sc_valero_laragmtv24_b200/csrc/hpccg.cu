@@ -789,8 +789,8 @@ int enqueue_iteration_ff_u(hpccg_problem *p, bool timing, bool check, unsigned l
     hpccg_ctx *ctx = p->ctx;
     const bool pdl = p->opt_pdl != 0;
     const bool zs = ctx->mode != MODE_SINGLE;  // HALO_PEER = 2 on z-slabs (fused_on)
-    auto upd = cg_update1_kernel<kU>;
-    auto pup = cg_pupdate1_kernel<kU>;
+    auto upd = zs ? cg_update1_kernel<kU, true> : cg_update1_kernel<kU, false>;
+    auto pup = zs ? cg_pupdate1_kernel<kU, true> : cg_pupdate1_kernel<kU, false>;
     const Slab &s0 = p->slabs[0];
     // the update's grid fixes the r.r partials and so the bits: size it as
     // the finisher path's update kernel is sized, so both paths agree bitwise

@@ -184,18 +184,8 @@ __device__ __forceinline__ void grid_reduce(double v, Reduction red, unsigned pa
     __syncthreads();
     if (!is_last) return;
     __threadfence();
-    // per thread left to right over i, i + kBlock, ... with 8 loads in flight
-    // per batch (the order, and so the bits, of a plain loop)
     double s = 0.0;
-    unsigned i = threadIdx.x;
-    for (; i + 7u * kBlock < total; i += 8u * kBlock) {
-        double q[8];
-#pragma unroll
-        for (int u = 0; u < 8; ++u) q[u] = __ldcg(red.partials + i + u * kBlock);
-#pragma unroll
-        for (int u = 0; u < 8; ++u) s = kMax ? fmax(s, q[u]) : s + q[u];
-    }
-    for (; i < total; i += kBlock) {
+    for (unsigned i = threadIdx.x; i < total; i += kBlock) {
         double q = __ldcg(red.partials + i);
         s = kMax ? fmax(s, q) : s + q;
     }
@@ -727,10 +717,15 @@ __global__ void __launch_bounds__(kBlock, 4) spmv27x2_kernel(SpmvArgs a) {
         bnd = true;
     }
     if (kFused && bnd) {
-        // `done` first: past convergence no neighbour pushes (uniform exit)
-        if (kCheck && __ldg(&a.sc->done)) return;
-        const int64_t first = row - 2 * (int64_t)threadIdx.x;
-        fused_halo_wait(a, first, min(first + 2 * kBlock, lim) - 1);
+        // only blocks that read a halo some neighbour fills wait (and load
+        // coherently); `done` first: past convergence nobody pushes
+        const int64_t first = row - 2 * (int64_t)threadIdx.x, last = min(first + 2 * kBlock, lim) - 1;
+        const PeerTab *t = a.fpeer;
+        bnd = (first < a.plane && t->rank > 0) || (last >= a.stride - a.plane && t->rank < t->nranks - 1);
+        if (bnd) {
+            if (kCheck && __ldg(&a.sc->done)) return;  // uniform exit
+            fused_halo_wait(a, first, last);
+        }
     }
     if (kFused && bnd) {
         spmv27x2_body<kDots, kCheck, kFused, true>(a, row, lim, bid);
@@ -1055,7 +1050,9 @@ __device__ __forceinline__ bool run_check(CgScalars *sc, int q) {
 // a.6 p = r + beta p for a single slab (HPCCG's k > 1 branch: rtrans = r.r,
 // beta = rtrans / oldrtrans; k == 1: p = r).  The first trip's loads are
 // issued before the scalar work so their latency overlaps the partial sums.
-template <int kU>
+// kPeer: the HALO_PEER = 2 hooks (z-slabs); the single-slab instantiation
+// carries none of their code
+template <int kU, bool kPeer = false>
 __global__ void __launch_bounds__(kBlock) cg_pupdate1_kernel(Pupd1Args a) {
     __shared__ double sh[33];
     CgScalars *sc = a.sc;
@@ -1096,7 +1093,7 @@ __global__ void __launch_bounds__(kBlock) cg_pupdate1_kernel(Pupd1Args a) {
     trace_mark(a.trace, a.trace_max, k, 0, false);
     const bool first = (k == 1);
     double rtrans = first ? __ldg(&sc->rr_cur) : sum_parts_fixed(a.rr_parts, a.n_rr, sh);
-    if (a.t && !first) {  // z-slabs: the slab's r.r -> every rank; the global sum back
+    if (kPeer && !first) {  // z-slabs: the slab's r.r -> every rank; the global sum back
         const unsigned tag = ll_tag(__ldg(&sc->epoch), 2ull * (unsigned)(k - 1));
         if (a.post && blockIdx.x == 0 && threadIdx.x == 0) fused_post(a.t, 0, rtrans, tag);
         rtrans = fused_collect_block(a.t, 0, tag, &sh[32]);
@@ -1108,7 +1105,7 @@ __global__ void __launch_bounds__(kBlock) cg_pupdate1_kernel(Pupd1Args a) {
         sc->niters = k;
     }
     const int64_t n = a.n, plane = a.plane;
-    double *lo = a.t ? a.t->halo_to_lo : nullptr, *hi = a.t ? a.t->halo_to_hi : nullptr;
+    double *lo = kPeer ? a.t->halo_to_lo : nullptr, *hi = kPeer ? a.t->halo_to_hi : nullptr;
     int pushed = 0;
     auto put = [&](int64_t i, double v) {  // row i of the new p -> a neighbour's halo
         if (lo && i < plane) {
@@ -1131,7 +1128,7 @@ __global__ void __launch_bounds__(kBlock) cg_pupdate1_kernel(Pupd1Args a) {
                     v.y = fma(beta, pa[u].y, ra[u].y);
                 }
                 p2[i] = v;
-                if (a.t && (2 * i < plane || 2 * i + 1 >= n - plane)) {
+                if (kPeer && (2 * i < plane || 2 * i + 1 >= n - plane)) {
                     put(2 * i, v.x);
                     put(2 * i + 1, v.y);
                 }
@@ -1144,13 +1141,13 @@ __global__ void __launch_bounds__(kBlock) cg_pupdate1_kernel(Pupd1Args a) {
         const int64_t i = n - 1;
         const double v = first ? a.r[i] : fma(beta, a.p[i], a.r[i]);
         a.p[i] = v;
-        if (a.t) put(i, v);
+        if (kPeer) put(i, v);
     }
     if (a.trace) {
         __syncthreads();
         trace_mark(a.trace, a.trace_max, k, 0, true);
     }
-    if (a.t) fused_push_signal(a.t, pushed, a.n_push, ftag(__ldg(&sc->epoch), (unsigned long long)k));
+    if (kPeer) fused_push_signal(a.t, pushed, a.n_push, ftag(__ldg(&sc->epoch), (unsigned long long)k));
 }
 
 // a.5 x += alpha p, r -= alpha Ap, per-block r.r partial (no finisher), and
@@ -1190,7 +1187,7 @@ __global__ void __launch_bounds__(kBlock) fused_post_kernel(const double *parts,
         fused_post(t, q, v, ll_tag(__ldg(&sc->epoch), q == 0 ? 2ull * (unsigned)k : 2ull * (unsigned)k - 1ull));
 }
 
-template <int kU>
+template <int kU, bool kPeer = false>
 __global__ void __launch_bounds__(kBlock) cg_update1_kernel(Upd1Args a) {
     __shared__ double sh[33];
     CgScalars *sc = a.sc;
@@ -1234,7 +1231,7 @@ __global__ void __launch_bounds__(kBlock) cg_update1_kernel(Upd1Args a) {
     trace_mark(a.trace, a.trace_max, ktr, 2, false);
     const double rtrans = __ldg(&sc->rr_cur);
     double pAp = a.pAp_parts ? sum_parts_fixed(a.pAp_parts, a.n_parts, sh) : __ldg(&sc->pAp);
-    if (a.t) {  // z-slabs: the slab's p.Ap -> every rank; the global sum back
+    if (kPeer) {  // z-slabs: the slab's p.Ap -> every rank; the global sum back
         const unsigned tag = ll_tag(__ldg(&sc->epoch), 2ull * (unsigned)__ldg(&sc->niters) - 1ull);
         if (a.post && blockIdx.x == 0 && threadIdx.x == 0) fused_post(a.t, 1, pAp, tag);
         pAp = fused_collect_block(a.t, 1, tag, &sh[32]);
