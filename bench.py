@@ -272,14 +272,24 @@ def run_ours(args, nx, ny, nz, iters, cfg_index, scaling):
             # three CG kernels), else the separate peer kernels; falls back to NCCL if
             # the mapping is refused
             mode = 2 if (args.halo == "fused" or (args.halo == "auto" and not sr)) else 1
+            err = None
             try:
                 prob.set_option(H.HPCCG_OPT_HALO_PEER, mode)
+                # a short collective solve proves the peer mapping end to end (a wait
+                # that times out returns an error instead of hanging)
+                prob.solve(4, 0.0)
+            except H.HpccgError as e:
+                err = str(e)
+            ok = torch.tensor([0.0 if err else 1.0], device=torch.device("cuda", local))
+            dist.all_reduce(ok, op=dist.ReduceOp.MIN)   # every rank takes the same path
+            if ok.item() == 1.0:
                 halo = ("peer memory fused into the CG kernels (HALO_PEER 2, while-graph)" if mode == 2
                         else "peer-memory push + post/collect allreduce kernels (while-graph)")
-            except H.HpccgError as e:
+            else:
                 if args.halo != "auto":
-                    raise
-                halo = "NCCL (peer mapping refused: %s)" % e
+                    raise RuntimeError("peer-memory path failed: %s" % err)
+                prob.set_option(H.HPCCG_OPT_HALO_PEER, 0)
+                halo = "NCCL (peer path failed on some rank: %s)" % err
     xptr = prob.vec_ptr(H.HPCCG_VEC_X)
     # working set (ELL 324 B/row + 6 vectors): when it fits in L2, flush L2
     # between timed steps (outside the timed events) so no step starts warm
