@@ -717,9 +717,11 @@ int allreduce_cg(hpccg_problem *p, bool rr, bool timing) {
 // Needs the 2-rows-per-thread SpMV and 16-B aligned vectors; else the
 // HALO_PEER = 1 kernels run (same bits).
 bool fused_on(const hpccg_problem *p) {
-    if (p->opt_peer != 2 || !peer_on(p) || p->opt_variant != 0 || !p->opt_ff) return false;
+    if (p->opt_peer != 2 || !peer_on(p)) return false;
+    if (p->opt_variant == 0 && !p->opt_ff) return false;  // HPCCG: on the finisher-free loop
     const Slab &s = p->slabs[0];
-    if (!s.ptab || !aligned16(s.r) || !aligned16(s.p + s.plane) || !aligned16(s.x) || !aligned16(s.Ap))
+    if (!s.ptab || !aligned16(s.r) || !aligned16(s.p + s.plane) || !aligned16(s.x) || !aligned16(s.Ap) ||
+        !aligned16(s.sv))
         return false;
     const int64_t b1_r0 = std::max<int64_t>(s.n - s.plane, s.plane);
     return spmv_rows_per_thread(p->opt_rows, spmv_args(s, s.p, s.Ap), s.plane, b1_r0) == 2;
@@ -752,7 +754,8 @@ unsigned push_blocks(int64_t n, int64_t plane, int g, bool has_lo, bool has_hi) 
 
 // one launch per slab: interior row blocks, then plane 0, then plane nz-1
 // (the same blocks and partial slots as HALO_PEER = 1's two launches)
-int launch_spmv_fused(hpccg_problem *p, const Slab &s, bool check, unsigned *nparts) {
+template <int kDots = 1>
+int launch_spmv_fused(hpccg_problem *p, const Slab &s, bool check, unsigned *nparts, int sr_q = 0) {
     const int64_t n = s.n, plane = s.plane;
     SpmvArgs a = spmv_args(s, s.p, s.Ap);
     a.single = 0;
@@ -771,8 +774,10 @@ int launch_spmv_fused(hpccg_problem *p, const Slab &s, bool check, unsigned *npa
     a.parts_only = s.spmv_parts;  // the finisher-free update sums them
     *nparts = (unsigned)blocks;
     const bool pdl = p->opt_pdl != 0;
-    if (check) launch_k(pdl, spmv27x2_kernel<1, true, true>, dim3((unsigned)blocks), p->ctx->stream, a);
-    else launch_k(pdl, spmv27x2_kernel<1, false, true>, dim3((unsigned)blocks), p->ctx->stream, a);
+    a.sr_q = sr_q;
+    if (kDots == 2) a.trace = nullptr;
+    if (check) launch_k(pdl, spmv27x2_kernel<kDots, true, true>, dim3((unsigned)blocks), p->ctx->stream, a);
+    else launch_k(pdl, spmv27x2_kernel<kDots, false, true>, dim3((unsigned)blocks), p->ctx->stream, a);
     return check_launch(p->ctx);
 }
 
@@ -1096,9 +1101,72 @@ int launch_sr_update(hpccg_problem *p, const Slab &s, int q, unsigned long long 
     }
 }
 
+// f2 with HALO_PEER = 2 on z-slabs: the update collects (gamma, delta) from
+// every rank's post (block 0 posts the slab's; loopback: fused_post2_kernel
+// ahead of every update) and pushes the new r's boundary planes into the
+// neighbours' halos; the SpMV's boundary blocks wait for them; one post of
+// two values per iteration.
+template <int kU>
+int enqueue_iteration_sr_fused_u(hpccg_problem *p, bool timing, bool check, unsigned long long cond, int q) {
+    hpccg_ctx *ctx = p->ctx;
+    const bool pdl = p->opt_pdl != 0;
+    const bool pre = ctx->mode == MODE_LOOPBACK;
+    auto upd = cg_sr_update_kernel<true, kU, true>;
+    const Slab &s0 = p->slabs[0];
+    const int g = vec_grid(ctx, upd, cdiv(s0.n, 2 * kU), p->opt_vec_waves, 0x7fffffff);
+    // the slab sums come from cg_sr_finish_kernel (sc->loc_gd) as on the
+    // HALO_PEER 0 / 1 z-slab path, so all three modes give the same bits
+    {
+        PhaseTimer t(p, ctx->stream, PH_UPDATE, timing);
+        if (pre)
+            for (const Slab &s : p->slabs) {
+                launch_k(pdl, fused_post2_kernel, dim3(1), ctx->stream, (const double *)nullptr, 0u,
+                         (const double *)s.sc->loc_gd, (const PeerTab *)s.ptab, (const CgScalars *)s.sc, q);
+                CHECK(check_launch(ctx));
+            }
+        for (size_t si = 0; si < p->slabs.size(); ++si) {
+            const Slab &s = p->slabs[si];
+            SrUpdArgs a{};
+            a.n = s.n;
+            a.x = s.x;
+            a.r = s.p + s.plane;
+            a.p = s.r;
+            a.s = s.sv;
+            a.w = s.Ap;
+            a.sc = s.sc;
+            a.q = q;
+            a.cond = si == 0 ? cond : 0ull;
+            a.t = s.ptab;
+            a.plane = s.plane;
+            a.post = !pre;
+            const uint64_t key = ((uint64_t)g << 16) | ((uint64_t)kU << 8) | 3u;
+            auto &cache = p->fpush[si];
+            if (cache.first != key)
+                cache = {key, push_blocks(s.n, s.plane, g, s.rank > 0, s.rank < ctx->nranks - 1)};
+            a.n_push = cache.second;
+            launch_k(pdl, upd, dim3(g), ctx->stream, a);
+            CHECK(check_launch(ctx));
+        }
+    }
+    PhaseTimer t(p, ctx->stream, PH_SPMV, timing);
+    unsigned npo = 0;
+    for (const Slab &s : p->slabs) CHECK(launch_spmv_fused<2>(p, s, check, &npo, q));
+    for (const Slab &s : p->slabs) {  // the slab sums for the next update (its loc_gd)
+        launch_kb(pdl, cg_sr_finish_kernel, dim3(1), dim3(1024), ctx->stream, (const double *)s.spmv_parts, npo,
+                  s.sc->loc_gd);
+        CHECK(check_launch(ctx));
+    }
+    return HPCCG_OK;
+}
+
 // One f2 iteration of parity q: the fused update, then w = A r + (gamma, delta).
 int enqueue_iteration_sr(hpccg_problem *p, bool timing, bool check, unsigned long long cond, int q) {
     hpccg_ctx *ctx = p->ctx;
+    if (fused_on(p)) switch (p->opt_unroll) {
+            case 1: return enqueue_iteration_sr_fused_u<1>(p, timing, check, cond, q);
+            case 2: return enqueue_iteration_sr_fused_u<2>(p, timing, check, cond, q);
+            default: return enqueue_iteration_sr_fused_u<4>(p, timing, check, cond, q);
+        }
     const bool pdl = ctx->mode == MODE_SINGLE && p->opt_pdl;
     {
         PhaseTimer t(p, ctx->stream, PH_UPDATE, timing);

@@ -272,6 +272,7 @@ struct PeerSync {                      // one per slab, in that slab's device me
     // on the post or the collect (the scalar allreduces are on the critical
     // path of every iteration; the halo flags are hidden behind the interior)
     unsigned long long fll[2][kMaxPeers][2];
+    unsigned long long fll2[2][kMaxPeers][2];  // f2: delta beside gamma (in fll), seq = k
 };
 
 struct PeerTab {                       // device copy per slab; pointers may be peers'
@@ -369,15 +370,18 @@ __device__ __forceinline__ bool ll_read(const unsigned long long *w, unsigned ta
 // result (*sh broadcasts it).  Lane r of warp 0 polls rank r's words (the P
 // latencies overlap); lane 0 adds the shuffled values left to right (the
 // order of peer_allreduce_kernel).  ~2 s timeout -> error flag.
-__device__ __forceinline__ double fused_collect_block(const PeerTab *t, int q, unsigned tag, double *sh) {
+// `mine`: this slab's own value (every block holds it), used for slot [rank]
+// instead of waiting for its own block 0's post -- same bits.
+__device__ __forceinline__ double fused_collect_block(const PeerTab *t, int q, unsigned tag, double mine,
+                                                      double *sh) {
     __syncthreads();  // sh reuse
     if (threadIdx.x < 32) {
         PeerSync *m = t->mine;
         const int P = t->nranks, lane = threadIdx.x;
         double s = 0.0;
         for (int r0 = 0; r0 < P; r0 += 32) {
-            double v = 0.0;
-            if (r0 + lane < P && !ll_read(m->fll[q][r0 + lane], tag, &v)) {
+            double v = mine;
+            if (r0 + lane < P && r0 + lane != t->rank && !ll_read(m->fll[q][r0 + lane], tag, &v)) {
                 const unsigned long long t0 = gtimer();
                 while (!ll_read(m->fll[q][r0 + lane], tag, &v)) {
                     if (*(volatile int *)&m->error || gtimer() - t0 > 2000000000ull) {
@@ -396,6 +400,60 @@ __device__ __forceinline__ double fused_collect_block(const PeerTab *t, int q, u
     }
     __syncthreads();
     return *sh;
+}
+
+// f2 (HALO_PEER = 2): (gamma, delta) of one iteration in slot q = seq & 1 of
+// fll (gamma) and fll2 (delta); post by one thread, collect per block as above
+__device__ __forceinline__ void fused_post2(const PeerTab *t, int q, double2 v, unsigned tag) {
+    const unsigned long long hi = (unsigned long long)tag << 32;
+    const unsigned long long g = (unsigned long long)__double_as_longlong(v.x);
+    const unsigned long long d = (unsigned long long)__double_as_longlong(v.y);
+    const int P = t->nranks, me = t->rank;
+    for (int r = 0; r < P; ++r) {
+        asm volatile("st.relaxed.sys.global.v2.u64 [%0], {%1, %2};" ::"l"(&t->all[r]->fll[q][me][0]),
+                     "l"((g & 0xffffffffull) | hi), "l"((g >> 32) | hi)
+                     : "memory");
+        asm volatile("st.relaxed.sys.global.v2.u64 [%0], {%1, %2};" ::"l"(&t->all[r]->fll2[q][me][0]),
+                     "l"((d & 0xffffffffull) | hi), "l"((d >> 32) | hi)
+                     : "memory");
+    }
+}
+
+__device__ __forceinline__ double2 fused_collect2_block(const PeerTab *t, int q, unsigned tag, double2 mine,
+                                                        double *sh /*[2]*/) {
+    __syncthreads();  // sh reuse
+    if (threadIdx.x < 32) {
+        PeerSync *m = t->mine;
+        const int P = t->nranks, lane = threadIdx.x;
+        double sg = 0.0, sd = 0.0;
+        for (int r0 = 0; r0 < P; r0 += 32) {
+            double g = mine.x, d = mine.y;
+            const int src = r0 + lane;
+            if (src < P && src != t->rank) {
+                const unsigned long long t0 = gtimer();
+                bool okg = false, okd = false;
+                while (!(okg = okg || ll_read(m->fll[q][src], tag, &g)) |
+                       !(okd = okd || ll_read(m->fll2[q][src], tag, &d))) {
+                    if (*(volatile int *)&m->error || gtimer() - t0 > 2000000000ull) {
+                        m->error = 1;
+                        break;
+                    }
+                    __nanosleep(32);
+                }
+            }
+            for (int j = 0; j < 32 && r0 + j < P; ++j) {
+                const double wg = __shfl_sync(0xffffffffu, g, j), wd = __shfl_sync(0xffffffffu, d, j);
+                sg = (r0 + j == 0) ? wg : sg + wg;
+                sd = (r0 + j == 0) ? wd : sd + wd;
+            }
+        }
+        if (lane == 0) {
+            sh[0] = sg;
+            sh[1] = sd;
+        }
+    }
+    __syncthreads();
+    return make_double2(sh[0], sh[1]);
 }
 
 // --------------------------------------------------------- a.3 SpMV (ELL-27)
@@ -587,7 +645,8 @@ __global__ void __launch_bounds__(kBlock, kMinB) spmv27_kernel(SpmvArgs a) {
 __device__ __forceinline__ void fused_halo_wait(const SpmvArgs &a, int64_t first, int64_t last) {
     if (threadIdx.x == 0) {
         const PeerTab *t = a.fpeer;
-        const unsigned long long tg = ftag(__ldg(&a.sc->epoch), (unsigned long long)__ldg(&a.sc->k));
+        // iteration k's SpMV: niters = k (written by the p update / f2 update)
+        const unsigned long long tg = ftag(__ldg(&a.sc->epoch), (unsigned long long)__ldg(&a.sc->niters));
         if (first < a.plane && t->rank > 0) spin_until(&t->mine->fflag_from_lo, tg, t->mine);
         if (last >= a.stride - a.plane && t->rank < t->nranks - 1)
             spin_until(&t->mine->fflag_from_hi, tg, t->mine);
@@ -723,6 +782,9 @@ __global__ void __launch_bounds__(kBlock, 4) spmv27x2_kernel(SpmvArgs a) {
         const PeerTab *t = a.fpeer;
         bnd = (first < a.plane && t->rank > 0) || (last >= a.stride - a.plane && t->rank < t->nranks - 1);
         if (bnd) {
+            // niters / done are written by the predecessor (PDL): wait for it
+            // first (the body's second griddepcontrol.wait is a no-op)
+            pdl_wait();
             if (kCheck && __ldg(&a.sc->done)) return;  // uniform exit
             fused_halo_wait(a, first, last);
         }
@@ -1096,7 +1158,7 @@ __global__ void __launch_bounds__(kBlock) cg_pupdate1_kernel(Pupd1Args a) {
     if (kPeer && !first) {  // z-slabs: the slab's r.r -> every rank; the global sum back
         const unsigned tag = ll_tag(__ldg(&sc->epoch), 2ull * (unsigned)(k - 1));
         if (a.post && blockIdx.x == 0 && threadIdx.x == 0) fused_post(a.t, 0, rtrans, tag);
-        rtrans = fused_collect_block(a.t, 0, tag, &sh[32]);
+        rtrans = fused_collect_block(a.t, 0, tag, rtrans, &sh[32]);
     }
     const double beta = first ? 0.0 : rtrans / __ldg(&sc->rr_prev);
     if (blockIdx.x == 0 && threadIdx.x == 0) {
@@ -1234,7 +1296,7 @@ __global__ void __launch_bounds__(kBlock) cg_update1_kernel(Upd1Args a) {
     if (kPeer) {  // z-slabs: the slab's p.Ap -> every rank; the global sum back
         const unsigned tag = ll_tag(__ldg(&sc->epoch), 2ull * (unsigned)__ldg(&sc->niters) - 1ull);
         if (a.post && blockIdx.x == 0 && threadIdx.x == 0) fused_post(a.t, 1, pAp, tag);
-        pAp = fused_collect_block(a.t, 1, tag, &sh[32]);
+        pAp = fused_collect_block(a.t, 1, tag, pAp, &sh[32]);
     }
     const bool stop = (rtrans == 0.0) || (pAp == 0.0);  // A11
     const double alpha = stop ? 0.0 : rtrans / pAp;
@@ -1350,6 +1412,13 @@ struct SrUpdArgs {
     CgScalars *sc;
     int q;                     // parity of the iteration this launch runs
     unsigned long long cond;   // while-graph condition handle (0: none)
+    // HALO_PEER = 2 on z-slabs (kPeer): (gamma, delta) = the P slabs' sums
+    // (k > 1; block 0 posts this slab's unless `post` is 0), and the first /
+    // last owned plane of the new r pushed into the neighbours' halos
+    const PeerTab *t;
+    int64_t plane;
+    unsigned n_push;
+    int post;
 };
 
 // Fixed-order sums of the (gamma, delta) partials, identical in every block.
@@ -1422,7 +1491,22 @@ __global__ void __launch_bounds__(1024) cg_sr_finish_kernel(const double *parts,
     }
 }
 
-template <bool kVec, int kU>
+// Loopback + HALO_PEER = 2, f2: post a slab's (gamma, delta) of the previous
+// SpMV ahead of every update (see fused_post_kernel).  q: the parity of the
+// update about to run; nothing for its first iteration.
+__global__ void __launch_bounds__(kBlock) fused_post2_kernel(const double *parts, unsigned n,
+                                                              const double *fallback, const PeerTab *t,
+                                                              const CgScalars *sc, int q) {
+    __shared__ double sh[66];
+    pdl_wait();
+    pdl_trigger();
+    const int k = __ldg(&sc->sr_k[q ^ 1]);
+    if (k < 2 || !__ldg(&sc->run_q[q ^ 1])) return;
+    const double2 v = parts ? sr_sum_parts(parts, n, sh) : make_double2(__ldcg(fallback), __ldcg(fallback + 1));
+    if (threadIdx.x == 0) fused_post2(t, (k - 1) & 1, v, ll_tag(__ldg(&sc->epoch), (unsigned)(k - 1)));
+}
+
+template <bool kVec, int kU, bool kPeer = false>
 __global__ void __launch_bounds__(kBlock) cg_sr_update_kernel(SrUpdArgs a) {
     CgScalars *sc = a.sc;
     const int q = a.q, qp = q ^ 1;
@@ -1451,11 +1535,24 @@ __global__ void __launch_bounds__(kBlock) cg_sr_update_kernel(SrUpdArgs a) {
     }
     __shared__ double sh[66];
     double2 gd;
-    if (a.parts) gd = sr_sum_parts(a.parts, a.n_parts, sh);
-    else gd = make_double2(__ldg(&sc->gd[0]), __ldg(&sc->gd[1]));
-    const double gamma = gd.x, delta = gd.y;
     const int k = __ldg(&sc->sr_k[qp]);
     const bool first = (k == 1);
+    if (kPeer) {  // z-slabs: k = 1 takes the init's allreduced values
+        if (first) {
+            gd = make_double2(__ldg(&sc->gd[0]), __ldg(&sc->gd[1]));
+        } else {
+            gd = a.parts ? sr_sum_parts(a.parts, a.n_parts, sh)
+                         : make_double2(__ldcg(&sc->loc_gd[0]), __ldcg(&sc->loc_gd[1]));
+            const unsigned tag = ll_tag(__ldg(&sc->epoch), (unsigned)(k - 1));
+            if (a.post && blockIdx.x == 0 && threadIdx.x == 0) fused_post2(a.t, (k - 1) & 1, gd, tag);
+            gd = fused_collect2_block(a.t, (k - 1) & 1, tag, gd, &sh[64]);
+        }
+    } else if (a.parts) {
+        gd = sr_sum_parts(a.parts, a.n_parts, sh);
+    } else {
+        gd = make_double2(__ldg(&sc->gd[0]), __ldg(&sc->gd[1]));
+    }
+    const double gamma = gd.x, delta = gd.y;
     const double beta = first ? 0.0 : __ddiv_rn(gamma, __ldg(&sc->sr_gamma[qp]));
     const double den =
         first ? delta : __dsub_rn(delta, __ddiv_rn(__dmul_rn(beta, gamma), __ldg(&sc->sr_alpha[qp])));
@@ -1474,6 +1571,18 @@ __global__ void __launch_bounds__(kBlock) cg_sr_update_kernel(SrUpdArgs a) {
         set_cond(a.cond, nrun);
     }
     const int64_t tid = gtid(), nth = gnth();
+    double *lo = kPeer ? a.t->halo_to_lo : nullptr, *hi = kPeer ? a.t->halo_to_hi : nullptr;
+    int pushed = 0;
+    auto put = [&](int64_t i, double v) {  // row i of the new r -> a neighbour's halo
+        if (lo && i < a.plane) {
+            lo[i] = v;
+            pushed = 1;
+        }
+        if (hi && i >= a.n - a.plane) {
+            hi[i - (a.n - a.plane)] = v;
+            pushed = 1;
+        }
+    };
     if (kVec) {
         const int64_t nv = a.n >> 1;
         double2 *__restrict__ x2 = reinterpret_cast<double2 *>(a.x);
@@ -1510,7 +1619,12 @@ __global__ void __launch_bounds__(kBlock) cg_sr_update_kernel(SrUpdArgs a) {
                     p2[i] = pv;
                     s2[i] = sv;
                     x2[i] = make_double2(fma(alpha, pv.x, xa[u].x), fma(alpha, pv.y, xa[u].y));
-                    r2[i] = make_double2(fma(-alpha, sv.x, ra[u].x), fma(-alpha, sv.y, ra[u].y));
+                    const double2 rn = make_double2(fma(-alpha, sv.x, ra[u].x), fma(-alpha, sv.y, ra[u].y));
+                    r2[i] = rn;
+                    if (kPeer && (2 * i < a.plane || 2 * i + 1 >= a.n - a.plane)) {
+                        put(2 * i, rn.x);
+                        put(2 * i + 1, rn.y);
+                    }
                 }
             }
         }
@@ -1522,7 +1636,9 @@ __global__ void __launch_bounds__(kBlock) cg_sr_update_kernel(SrUpdArgs a) {
             a.s[i] = sv;
             a.x[i] = fma(alpha, pv, a.x[i]);
             a.r[i] = fma(-alpha, sv, a.r[i]);
+            if (kPeer) put(i, a.r[i]);
         }
+        if (kPeer) fused_push_signal(a.t, pushed, a.n_push, ftag(__ldg(&sc->epoch), (unsigned long long)k));
     } else {
         for (int64_t i = tid; i < a.n; i += nth) {
             const double pv = first ? a.r[i] : fma(beta, a.p[i], a.r[i]);
@@ -1558,6 +1674,7 @@ __global__ void __launch_bounds__(kBlock) cg_sr_initstate_kernel(const double *p
     sc->normr = normr;
     sc->niters = 0;
     sc->done = !run;
+    sc->epoch = sc->epoch + 1;
     set_cond(cond, run);
 }
 

@@ -149,7 +149,13 @@ __global__ void __launch_bounds__(kBlock) tri_dot_kernel(int64_t n, const double
 #pragma unroll
         for (int u = 0; u < kTriU; ++u) acc = fma(xv[u], yv[u], acc);
     }
-    for (int64_t i = b0; i < n; i += nth) acc = fma(x[i], y[i], acc);  // ragged tail, same order
+    // ragged tail (n - full < kTriU * nth: at most kTriU per thread), same
+    // order, a fixed trip count so no lane leaves early
+#pragma unroll
+    for (int t = 0; t < kTriU; ++t) {
+        const int64_t i = b0 + t * nth;
+        if (i < n) acc = fma(x[i], y[i], acc);
+    }
     grid_reduce<false>(acc, red, blockIdx.x, gridDim.x, [out](double v) { *out = v; });
 }
 

@@ -796,6 +796,33 @@ def test_peer_fused_loopback_bitwise(P, dims):
         assert np.max(np.abs(outs[0][2] - oref["x"])) <= CG_ATOL
 
 
+@pytest.mark.parametrize("P,dims", [(2, (16, 12, 6)), (3, (8, 6, 2)), (2, (10, 6, 1)), (3, (64, 64, 16))])
+def test_peer_fused_single_reduction_bitwise(P, dims):
+    """f2 (single-reduction CG) with HALO_PEER = 2: the update collects every
+    rank's (gamma, delta) post and pushes the new r's boundary planes, the
+    SpMV's boundary blocks wait for them -- bit for bit the copy path and
+    HALO_PEER = 1 in every launch mode, and the f2 oracle's tolerance."""
+    nx, ny, nz = dims
+    with H.Context(0, nranks=P, loopback=True) as c, H.Problem(c, nx, ny, nz) as p:
+        p.set_option(H.HPCCG_OPT_CG_VARIANT, 1)
+        outs = []
+        for peer, wh, timing in [(0, 1, 0), (2, 1, 0), (2, 0, 0), (2, 0, 1), (1, 1, 0)]:
+            p.set_option(H.HPCCG_OPT_HALO_PEER, peer)
+            p.set_option(H.HPCCG_OPT_WHILE, wh)
+            p.set_option(H.HPCCG_OPT_TIMING, timing)
+            p.set_vec(H.HPCCG_VEC_X, np.zeros(p.n * P))
+            r = p.solve(150, 1e-12)
+            outs.append((r["niters"], r["normr"], p.get_vec(H.HPCCG_VEC_X)))
+        p.set_option(H.HPCCG_OPT_TIMING, 0)
+        for o in outs[1:]:
+            assert o[:2] == outs[0][:2]
+            np.testing.assert_array_equal(o[2], outs[0][2])
+        ref = oracle.generate(nx, ny, nz * P)
+        oref = oracle.cg_sr(ref, 150, 1e-12)
+        assert abs(outs[0][0] - oref["niters"]) <= 1
+        assert np.max(np.abs(outs[0][2] - oref["x"])) <= CG_ATOL
+
+
 def test_peer_fused_repeat_solves_and_mode_switches():
     """Fused tags are (epoch, seq): solves of different lengths, tol-stopped
     solves (kernels past convergence exit before waiting) and switches between
@@ -846,7 +873,7 @@ def test_peer_mode_nccl_one_rank():
     with H.Context(0, rank=0, nranks=1, unique_id=uid) as c, H.Problem(c, *dims) as p:
         p.set_option(H.HPCCG_OPT_HALO_PEER, 1)
         ref = oracle.generate(*dims)
-        for variant, halo in ((0, 1), (1, 1), (0, 2)):
+        for variant, halo in ((0, 1), (1, 1), (0, 2), (1, 2)):
             p.set_option(H.HPCCG_OPT_HALO_PEER, halo)
             p.set_option(H.HPCCG_OPT_CG_VARIANT, variant)
             p.set_vec(H.HPCCG_VEC_X, np.zeros(p.n))

@@ -17,7 +17,7 @@ torch = pytest.importorskip("torch")
 from paper_conf_sc_valero_laragmtv24_b200 import hpccg as H  # noqa: E402
 
 
-def run_ranks(nranks, dims, variant, max_iter, tol, timeout=240, halo=1):
+def run_ranks(nranks, dims, variant, max_iter, tol, timeout=240, halo=1):  # noqa: PLR0913
     import peer_worker
     ctx = mp.get_context("spawn")
     to_parent = ctx.Queue()
@@ -98,6 +98,28 @@ def test_processes_fused_peer_kernels(P, dims, max_iter, tol):
         rl = p.solve(max_iter, tol)
         xl = p.get_vec(H.HPCCG_VEC_X)
     for k in range(2):                       # while-graph, per-iteration graph
+        outs = [res[r][k] for r in range(P)]
+        x = np.concatenate([o["x"] for o in outs])
+        for o in outs:
+            assert (o["niters"], o["normr"]) == (rl["niters"], rl["normr"])
+        np.testing.assert_array_equal(x, xl)
+        assert abs(outs[0]["niters"] - oref["niters"]) <= 1
+        assert np.max(np.abs(x - oref["x"])) <= 1e-10
+
+
+def test_processes_fused_peer_single_reduction():
+    """f2 with HALO_PEER = 2 across 2 processes: bit for bit the loopback
+    HALO_PEER = 1 run, within the tolerance of the f2 oracle."""
+    P, dims = 2, (16, 12, 6)
+    res = run_ranks(P, dims, 1, 150, 1e-12, halo=2)
+    ref = oracle.generate(dims[0], dims[1], dims[2] * P)
+    oref = oracle.cg_sr(ref, 150, 1e-12)
+    with H.Context(0, nranks=P, loopback=True) as c, H.Problem(c, *dims) as p:
+        p.set_option(H.HPCCG_OPT_CG_VARIANT, 1)
+        p.set_option(H.HPCCG_OPT_HALO_PEER, 1)
+        rl = p.solve(150, 1e-12)
+        xl = p.get_vec(H.HPCCG_VEC_X)
+    for k in range(2):
         outs = [res[r][k] for r in range(P)]
         x = np.concatenate([o["x"] for o in outs])
         for o in outs:
