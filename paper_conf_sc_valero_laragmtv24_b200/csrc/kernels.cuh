@@ -2190,8 +2190,9 @@ __global__ void peer_allreduce_kernel(const PeerTab *t, const double *src, doubl
 // ---------------------------------------------------------- a.10 BLAS-1
 
 // w = alpha x + beta y, canonical forms (A10).  form: 0 alpha==1, 1 beta==1,
-// 2 general.  24n B.
-template <bool kVec, int kForm>
+// 2 general.  24n B.  kU 16-B units per thread per trip, all loads issued
+// before the stores (plain loads: evict-first ones measured slower here).
+template <bool kVec, int kForm, int kU = 2>
 __global__ void __launch_bounds__(kBlock) waxpby_kernel(int64_t n, double alpha, const double *x,
                                                        double beta, const double *y, double *w) {
     const int64_t tid = gtid(), nth = gnth();
@@ -2205,14 +2206,21 @@ __global__ void __launch_bounds__(kBlock) waxpby_kernel(int64_t n, double alpha,
         const double2 *x2 = reinterpret_cast<const double2 *>(x);
         const double2 *y2 = reinterpret_cast<const double2 *>(y);
         double2 *w2 = reinterpret_cast<double2 *>(w);
-        for (int64_t i = tid; i < nv; i += 2 * nth) {
-            const int64_t j = i + nth;
-            const bool hj = j < nv;
-            const double2 xa = x2[i], ya = y2[i];
-            double2 xb = {0, 0}, yb = {0, 0};
-            if (hj) { xb = x2[j]; yb = y2[j]; }
-            w2[i] = make_double2(op(xa.x, ya.x), op(xa.y, ya.y));
-            if (hj) w2[j] = make_double2(op(xb.x, yb.x), op(xb.y, yb.y));
+        for (int64_t i = tid; i < nv; i += kU * nth) {
+            double2 xa[kU], ya[kU];
+#pragma unroll
+            for (int u = 0; u < kU; ++u) {
+                const int64_t j = i + u * nth;
+                if (j < nv) {
+                    xa[u] = x2[j];
+                    ya[u] = y2[j];
+                }
+            }
+#pragma unroll
+            for (int u = 0; u < kU; ++u) {
+                const int64_t j = i + u * nth;
+                if (j < nv) w2[j] = make_double2(op(xa[u].x, ya[u].x), op(xa[u].y, ya[u].y));
+            }
         }
         if (tid == 0 && (n & 1)) w[n - 1] = op(x[n - 1], y[n - 1]);
     } else {
@@ -2220,8 +2228,10 @@ __global__ void __launch_bounds__(kBlock) waxpby_kernel(int64_t n, double alpha,
     }
 }
 
-// sum_i x_i y_i -> *out (deterministic).  16n B (8n for x.x).
-template <bool kVec>
+// sum_i x_i y_i -> *out (deterministic: the element -> thread map and the
+// per-thread order depend only on (n, grid, kU)).  16n B (8n for x.x).  kU
+// 16-B units of x and y per thread per trip, all loads first, streamed.
+template <bool kVec, int kU = 2>
 __global__ void __launch_bounds__(kBlock) dot_kernel(int64_t n, const double *x, const double *y,
                                                     Reduction red, double *out) {
     const int64_t tid = gtid(), nth = gnth();
@@ -2231,16 +2241,23 @@ __global__ void __launch_bounds__(kBlock) dot_kernel(int64_t n, const double *x,
         const double2 *x2 = reinterpret_cast<const double2 *>(x);
         const double2 *y2 = reinterpret_cast<const double2 *>(y);
         double acc2 = 0.0;
-        for (int64_t i = tid; i < nv; i += 2 * nth) {
-            const int64_t j = i + nth;
-            const bool hj = j < nv;
-            const double2 xa = __ldcs(x2 + i), ya = __ldcs(y2 + i);
-            double2 xb = {0, 0}, yb = {0, 0};
-            if (hj) { xb = __ldcs(x2 + j); yb = __ldcs(y2 + j); }
-            acc = fma(xa.x, ya.x, acc);
-            acc2 = fma(xa.y, ya.y, acc2);
-            acc = fma(xb.x, yb.x, acc);     // zero-padded when j >= nv
-            acc2 = fma(xb.y, yb.y, acc2);
+        for (int64_t i = tid; i < nv; i += kU * nth) {
+            double2 xa[kU], ya[kU];
+#pragma unroll
+            for (int u = 0; u < kU; ++u) {
+                const int64_t j = i + u * nth;
+                xa[u] = make_double2(0.0, 0.0);   // zero-padded past nv
+                ya[u] = make_double2(0.0, 0.0);
+                if (j < nv) {
+                    xa[u] = __ldcs(x2 + j);
+                    ya[u] = __ldcs(y2 + j);
+                }
+            }
+#pragma unroll
+            for (int u = 0; u < kU; ++u) {
+                acc = fma(xa[u].x, ya[u].x, acc);
+                acc2 = fma(xa[u].y, ya[u].y, acc2);
+            }
         }
         acc += acc2;
         if (tid == 0 && (n & 1)) acc = fma(x[n - 1], y[n - 1], acc);
