@@ -27,7 +27,7 @@ class Shared:
         self.slots = [[[(0, None)] * P for _ in range(2)] for _ in range(P)]
         self.halo = [[None, None] for _ in range(P)]     # [owner][0 lower | 1 upper] = value
         self.flag = [[0, 0] for _ in range(P)]           # [owner][0 from lo | 1 from hi]
-        self.lock = threading.Lock()
+        self.barrier = threading.Barrier(P)   # the host sync at the end of every solve
         self.errors = []
 
 
@@ -110,14 +110,9 @@ def rank_main(sh, r, solves, iters, seed, deadline, one_slot=False):
         sh_barrier(sh, P)
 
 
-_bar = {}
-
-
 def sh_barrier(sh, P):
-    with sh.lock:
-        b = _bar.setdefault(id(sh), threading.Barrier(P))
     try:
-        b.wait(timeout=20)
+        sh.barrier.wait(timeout=20)
     except threading.BrokenBarrierError:
         sh.errors.append("solve-end barrier broken (a rank stopped early)")
 
