@@ -268,10 +268,10 @@ def run_ours(args, nx, ny, nz, iters, cfg_index, scaling):
         halo = "NCCL send/recv + ncclAllReduce"
         if args.halo in ("peer", "fused", "auto"):
             # collective: every rank maps its neighbours' buffers (CUDA IPC over NVLink);
-            # auto = fused for HPCCG's CG (the exchange and both allreduces inside the
-            # three CG kernels), else the separate peer kernels; falls back to NCCL if
-            # the mapping is refused
-            mode = 2 if (args.halo == "fused" or (args.halo == "auto" and not sr)) else 1
+            # auto = fused (the exchange and the allreduce(s) inside the CG kernels,
+            # either CG variant); peer = the separate peer kernels; auto falls back to
+            # NCCL if the mapping is refused
+            mode = 1 if args.halo == "peer" else 2
             err = None
             try:
                 prob.set_option(H.HPCCG_OPT_HALO_PEER, mode)
@@ -790,8 +790,8 @@ def main():
     ap.add_argument("--iters", type=int, default=None, help="override CG iterations per step")
     ap.add_argument("--halo", choices=["auto", "nccl", "peer", "fused"], default="auto",
                     help="multi-GPU exchange: peer memory fused into the CG kernels (HALO_PEER 2, "
-                         "auto for HPCCG's CG), our separate peer-memory kernels (HALO_PEER 1, auto "
-                         "for --cg-variant sr), or NCCL; auto falls back to NCCL if CUDA IPC is refused")
+                         "auto, both CG variants), our separate peer-memory kernels (HALO_PEER 1), "
+                         "or NCCL; auto falls back to NCCL if CUDA IPC is refused")
     ap.add_argument("--cg-variant", choices=["hpccg", "sr"], default="hpccg",
                     help="hpccg: HPCCG's CG (default); sr: single-reduction CG (SURVEY f2)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
