@@ -44,6 +44,9 @@ WORKLOADS = {
     "hpccg256": (256, 256, 256, 200, 2, "weak"),
     "hpccg512s": (512, 512, 512, 200, 3, "strong"),
 }
+BLAS1_METRIC = "JACC BLAS-1 AXPY+DOT fp64 HBM GB/s (host-synchronous calls)"
+TRI_METRIC = "Fig. 12 CG time per iteration, tridiagonal SIZE = 1e8 (fp64)"
+LBM_METRIC = "D2Q9 pull LBM (Fig. 10) time per step, 1000^2 (fp64)"
 FALLBACK_HBM_GBS = 6650.0  # B200_PROFILING.md fallback, used only without MEASURED_PEAKS.json
 
 
@@ -223,6 +226,107 @@ def run_reference(args, nx, ny, nz, iters, cfg_index):
     }
     print(json.dumps(line), flush=True)
     return 0
+
+
+def _reference_line(args, metric, value, unit, hib, ms_per_step, config, sample, scaling="none"):
+    """The reference arm's JSON line for the f1 / f4 / BLAS-1 workloads: the
+    oracle as it stands, on the host cores, in our arm's metric / unit / config."""
+    import oracle
+    line = {"metric": metric, "value": round(value, 5), "unit": unit, "impl": "reference",
+            "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": round(ms_per_step, 4), "higher_is_better": hib,
+            "scaling": scaling, "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": config,
+            "cpu_baseline": {"value": round(value, 5), "unit": unit, "cores": oracle.get_threads(),
+                             "kind": "oracle", "sample": sample},
+            "e2e": {"value": round(value, 5), "unit": unit, "h2d_bytes_per_step": 0,
+                    "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def run_reference_tridiag(args):
+    """Fig. 12 CG per-iteration time of the oracle at SIZE: each step
+    times a 1- and a 3-iteration oracle solve; per iteration = the difference / 2."""
+    if int(os.environ.get("RANK", "0")) != 0:
+        return 0
+    import oracle
+    oracle.build()
+    n = args.tri_n
+    tr = oracle.Tri(n)
+
+    def one():
+        o1 = oracle.tri_cg(tr, 1, 0.0)["seconds"]
+        o3 = oracle.tri_cg(tr, 3, 0.0)["seconds"]
+        return max((o3 - o1) / 2, o1 / 2) * 1e3
+
+    for _ in range(args.warmup):
+        one()
+    ms = sum(one() for _ in range(args.steps)) / args.steps
+    return _reference_line(args, TRI_METRIC, ms, "ms/iteration", False, ms,
+                           {"workload": "tridiag", "n": n},
+                           f"oracle Fig. 12 CG (C, OpenMP, compensated dots) at n = {n}: "
+                           f"(3-iteration - 1-iteration solve) / 2 per step")
+
+
+def run_reference_lbm(args):
+    """Fig. 10 D2Q9 pull step of the oracle at SIZE^2, one step per bench step."""
+    if int(os.environ.get("RANK", "0")) != 0:
+        return 0
+    import numpy as np
+    import oracle
+    import synth
+    oracle.build()
+    S = args.lbm_size
+    f0 = synth.lbm_state(S, 21)
+    a, b, f = f0.copy(), f0.copy(), np.zeros_like(f0)
+    for _ in range(args.warmup):
+        oracle.lbm_step(S, a, f, b, 0.8)
+        a, b = b, a
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        oracle.lbm_step(S, a, f, b, 0.8)
+        a, b = b, a
+    ms = (time.perf_counter() - t0) / args.steps * 1e3
+    return _reference_line(args, LBM_METRIC, ms, "ms/step", False, ms,
+                           {"workload": "lbm", "size": S},
+                           f"oracle Fig. 10 step (C, OpenMP) at {S}^2, one step per bench step")
+
+
+def run_reference_blas1(args):
+    """JACC AXPY + DOT of the oracle (Fig. 2 inputs) at a bounded n (the GPU arm's
+    headline is n = 1e9 per GPU; the host sample stops at 1e8 = 2.4 GB of vectors)."""
+    if int(os.environ.get("RANK", "0")) != 0:
+        return 0
+    import numpy as np
+    import oracle
+    import synth
+    oracle.build()
+    n = min(args.blas1_max or 10 ** 9, 10 ** 8)
+    gen = min(n, 1 << 24)
+    x = np.resize(synth.jacc_vector(gen, 42), n)
+    y = np.resize(synth.jacc_vector(gen, 43), n)
+    w = np.empty(n)
+
+    def one():
+        t0 = time.perf_counter()
+        oracle.waxpby(1.0, x, 2.5, y, w)
+        t1 = time.perf_counter()
+        oracle.ddot(x, y)
+        return t1 - t0, time.perf_counter() - t1
+
+    for _ in range(args.warmup):
+        one()
+    ta = td = 0.0
+    for _ in range(args.steps):
+        a, d = one()
+        ta, td = ta + a, td + d
+    ta, td = ta / args.steps, td / args.steps
+    gbs = (24.0 + 16.0) * n / (ta + td) / 1e9
+    return _reference_line(args, BLAS1_METRIC, gbs, "GB/s", True, (ta + td) * 1e3,
+                           {"workload": "blas1", "baseline_config": 4, "n": n},
+                           f"oracle waxpby (w = x + 2.5 y) + compensated ddot (C, OpenMP) at "
+                           f"n = {n} (bounded sample of the 1e9 headline)", scaling="weak")
 
 
 # -------------------------------------------------------------------- ours
@@ -636,7 +740,7 @@ def run_blas1(args):
     if rank == 0:
         peak, src = peaks()
         big = rows[-1]
-        line = {"metric": "JACC BLAS-1 AXPY+DOT fp64 HBM GB/s (host-synchronous calls)",
+        line = {"metric": BLAS1_METRIC,
                 "value": round((24.0 + 16.0) * big["n_per_gpu"] * world /
                                ((big["axpy_us"] + big["dot_us"]) * 1e-6) / 1e9, 1),
                 "unit": "GB/s", "n_gpus": world, "steps": None, "warmup": args.warmup,
@@ -695,7 +799,7 @@ def run_tridiag(args):
                "kind": "oracle", "sample": f"oracle Fig. 12 CG (C, OpenMP, compensated dots) at "
                                            f"n = {n}, 3 iterations"}
     fused_ms = res[1]
-    line = {"metric": "Fig. 12 CG time per iteration, tridiagonal SIZE = 1e8 (fp64)",
+    line = {"metric": TRI_METRIC,
             "value": round(fused_ms, 4), "unit": "ms/iteration", "higher_is_better": False,
             "n_gpus": 1, "steps": args.steps, "warmup": args.warmup, "scaling": "none",
             "vs_baseline": None, "dtype": "f64",
@@ -760,7 +864,7 @@ def run_lbm(args):
         cms = (time.perf_counter() - t0) / 5 * 1e3
         cpu = {"value": round(cms, 3), "unit": "ms/step", "cores": oracle.get_threads(),
                "kind": "oracle", "sample": f"oracle Fig. 10 step (C, OpenMP) at {S}^2, 5 steps"}
-    line = {"metric": "D2Q9 pull LBM (Fig. 10) time per step, 1000^2 (fp64)",
+    line = {"metric": LBM_METRIC,
             "value": round(ms, 5), "unit": "ms/step", "higher_is_better": False, "n_gpus": 1,
             "steps": args.steps, "warmup": args.warmup, "scaling": "none", "vs_baseline": None,
             "dtype": "f64", "data": "synthetic positive D2Q9 state (seeded), tau 0.8",
@@ -802,21 +906,15 @@ def main():
         raise SystemExit("--warmup must be >= 3")
     if args.workload == "lbm":
         if args.impl == "reference":
-            print(json.dumps({"impl": "reference", "unavailable":
-                              "lbm reports the oracle in cpu_baseline; no separate arm"}))
-            return 0
+            return run_reference_lbm(args)
         return run_lbm(args)
     if args.workload == "tridiag":
         if args.impl == "reference":
-            print(json.dumps({"impl": "reference", "unavailable":
-                              "tridiag reports the oracle in cpu_baseline; no separate arm"}))
-            return 0
+            return run_reference_tridiag(args)
         return run_tridiag(args)
     if args.workload == "blas1":
         if args.impl == "reference":
-            print(json.dumps({"impl": "reference", "unavailable":
-                              "the blas1 sweep has no oracle arm; run the default workload"}))
-            return 0
+            return run_reference_blas1(args)
         return run_blas1(args)
     nx, ny, nz, iters, cfg, scaling = WORKLOADS[args.workload]
     if args.iters:
