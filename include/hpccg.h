@@ -405,7 +405,12 @@ HPCCG_API int hpccg_lbm_set(hpccg_lbm *l, int which, const double *host);
 HPCCG_API int hpccg_lbm_get(const hpccg_lbm *l, int which, double *host);
 /* `steps` steps with relaxation time tau > 0: each step pulls lattice 0 into
  * lattice 1 (Fig. 10's f1 -> f2), then the two trade places, so lattice 0 is
- * always the newest state.  *ms (HOST, nullable) = device time. */
+ * always the newest state.  *ms (HOST, nullable) = device time.
+ * write_f: bit 0 materialises the streamed f into lattice 2; the other bits
+ * are tuning knobs (bits 1-2 cache policy, bit 3 no PDL; bit 4 runs the steps
+ * in fused pairs -- two steps per kernel, the intermediate lattice on chip,
+ * same bits; lattice 1 then keeps only its boundary sites and lattice 2 is
+ * scratch; ignored with bit 0). */
 HPCCG_API int hpccg_lbm_run(hpccg_lbm *l, int steps, double tau, int write_f, double *ms);
 HPCCG_API void hpccg_lbm_free(hpccg_lbm *l);
 

@@ -577,6 +577,57 @@ def test_lbm_bitwise_vs_oracle(ctx, S, steps, tau):
         np.testing.assert_array_equal(l.get(2), f)
 
 
+def _lbm_oracle(S, f1, f2, steps, tau):
+    a, b, f = f1.copy(), f2.copy(), np.zeros_like(f1)
+    for _ in range(steps):
+        oracle.lbm_step(S, a, f, b, tau)
+        a, b = b, a
+    return a, b
+
+
+def _edges(S, g):
+    g = g.reshape(9, S, S)
+    return np.concatenate([g[:, 0, :].ravel(), g[:, -1, :].ravel(), g[:, :, 0].ravel(),
+                           g[:, :, -1].ravel()])
+
+
+@pytest.mark.parametrize("S", [3, 4, 5, 17, 128, 129, 130, 257, 300])
+@pytest.mark.parametrize("steps", [1, 2, 3, 4, 5])
+def test_lbm_two_step_kernel_bitwise(ctx, S, steps):
+    """Tuning bit 4 runs the steps as fused pairs (lbm_pull2_kernel: step 1
+    into an on-chip ring, step 2 from it): lattice 0 bitwise equal to the
+    oracle's sequential steps for odd / even counts and sizes that cut the
+    126-column strips and 16-row chunks raggedly; lattice 1 keeps its boundary
+    sites (different from lattice 0's here, so a wrong boundary source fails)."""
+    f1 = synth.lbm_state(S, 31)
+    f2 = synth.lbm_state(S, 32)
+    with H.Lbm(ctx, S) as l:
+        l.set(0, f1)
+        l.set(1, f2)
+        l.run(steps, 0.7, 16)
+        a, b = _lbm_oracle(S, f1, f2, steps, 0.7)
+        np.testing.assert_array_equal(l.get(0), a)
+        np.testing.assert_array_equal(_edges(S, l.get(1)), _edges(S, b))
+
+
+@pytest.mark.parametrize("rows", [1, 2, 3, 7, 16, 33, 255])
+def test_lbm_two_step_rows_per_cta(ctx, rows):
+    """Every chunk height of the two-step kernel (tuning bits 8-15) gives the
+    same bits; repeated runs keep the lattice rotation consistent."""
+    S = 203
+    f1 = synth.lbm_state(S, 41)
+    f2 = synth.lbm_state(S, 42)
+    with H.Lbm(ctx, S) as l:
+        l.set(0, f1)
+        l.set(1, f2)
+        l.run(4, 1.1, rows << 8 | 16)
+        l.run(3, 1.1, rows << 8 | 16 | (5 << 16))
+        l.run(2, 1.1, rows << 8)   # without bit 4: one step per kernel
+        a, b = _lbm_oracle(S, f1, f2, 9, 1.1)
+        np.testing.assert_array_equal(l.get(0), a)
+        np.testing.assert_array_equal(_edges(S, l.get(1)), _edges(S, b))
+
+
 def test_lbm_paper_size_conservation(ctx):
     """S = 1000, 10 steps without materialising f: bitwise vs the
     oracle, and total mass of the interior preserved by collisions."""
