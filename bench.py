@@ -346,16 +346,32 @@ def run_ours(args, nx, ny, nz, iters, cfg_index, scaling):
         raise SystemExit(f"--gpus {args.gpus} but WORLD_SIZE={world}")
     if not torch.cuda.is_available():
         raise SystemExit("bench.py needs a CUDA device (no CPU fallback)")
+    # --share-device (a test of the N > 1 code path on a one-GPU box): every rank on
+    # cuda:0, torch.distributed over gloo, peer-only library contexts (NCCL refuses
+    # two ranks on one GPU); the ranks' kernels time-slice, so its numbers are not
+    # a scaling measurement
+    share = args.share_device and world > 1
+    if share:
+        local = 0
+    transport = "peer" if share else args.transport
+    if world > 1 and transport == "peer" and args.halo == "nccl":
+        raise SystemExit("--transport peer has no NCCL halo (use --halo fused or peer)")
+    coll_dev = "cpu" if share else "cuda"
     torch.cuda.set_device(local)
     slab = D.slab_for(nx, ny, nz, rank, world, scaling)
     nz = slab.nz
     uid = None
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-        uid = D.broadcast_unique_id(H.hpccg_unique_id)
+        if share:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if transport == "nccl":
+            uid = D.broadcast_unique_id(H.hpccg_unique_id)
 
     stream = torch.cuda.Stream()
-    ctx = H.Context(local, stream=stream.cuda_stream, rank=rank, nranks=world, unique_id=uid)
+    ctx = H.Context(local, stream=stream.cuda_stream, rank=rank, nranks=world, unique_id=uid,
+                    peer=(world > 1 and transport == "peer"))
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     e0.record(stream)
     prob = H.Problem(ctx, nx, ny, nz)
@@ -368,7 +384,16 @@ def run_ours(args, nx, ny, nz, iters, cfg_index, scaling):
     sr = args.cg_variant == "sr"
     prob.set_option(H.HPCCG_OPT_CG_VARIANT, 1 if sr else 0)
     halo = "none (1 slab)"
-    if world > 1:
+    if world > 1 and transport == "peer":
+        # peer-only context: no NCCL anywhere; every rank maps its neighbours' buffers
+        # from the exported CUDA-IPC blobs (gathered over torch.distributed)
+        prob.peer_attach(D.allgather_peer_blobs(prob.peer_export()))
+        mode = 1 if args.halo == "peer" else 2
+        prob.set_option(H.HPCCG_OPT_HALO_PEER, mode)
+        halo = ("peer memory fused into the CG kernels (HALO_PEER 2, while-graph), peer-only context"
+                if mode == 2 else
+                "peer-memory push + post/collect allreduce kernels (while-graph), peer-only context")
+    elif world > 1:
         halo = "NCCL send/recv + ncclAllReduce"
         if args.halo in ("peer", "fused", "auto"):
             # collective: every rank maps its neighbours' buffers (CUDA IPC over NVLink);
@@ -497,7 +522,7 @@ def run_ours(args, nx, ny, nz, iters, cfg_index, scaling):
     niters_tot = main["niters"]
     r, err = main["r"], main["err"]
     spmv_ms, spmv_n = ev["spmv_ms"], ev["spmv_n"]
-    ms_max, flops = D.max_time_sum_work(ms, cg_flops(niters_tot, nnz_local, n), "cuda")
+    ms_max, flops = D.max_time_sum_work(ms, cg_flops(niters_tot, nnz_local, n), coll_dev)
     value = flops / (ms_max * 1e-3) * 1e-9
 
     # ---- e2e: public API with host buffers (pinned) each step
@@ -533,7 +558,7 @@ def run_ours(args, nx, ny, nz, iters, cfg_index, scaling):
         t1.record(stream)
         barrier()
         te_local = t0.elapsed_time(t1)
-    te, fe = D.max_time_sum_work(te_local, cg_flops(ni_e2e, nnz_local, n), "cuda")
+    te, fe = D.max_time_sum_work(te_local, cg_flops(ni_e2e, nnz_local, n), coll_dev)
     e2e_value = fe / (te * 1e-3) * 1e-9
     x_host_err = float(np.max(np.abs(h_x.numpy() - 1.0)))
 
@@ -603,7 +628,8 @@ def run_ours(args, nx, ny, nz, iters, cfg_index, scaling):
                        "global_rows": n * world, "global_nnz": nnz_global,
                        "parallelism": f"zslab{world}",
                        "cg_variant": "single-reduction (Chronopoulos-Gear, f2)" if sr else "HPCCG",
-                       "halo": halo,
+                       "halo": halo, "transport": transport if world > 1 else None,
+                       "shared_device": bool(share),
                        "solve_graph": {5: "on-chip cluster kernel", 4: "one-cluster persistent kernel",
                                        3: "cooperative persistent kernel", 2: "while-graph",
                                        1: "per-iteration graph", 0: "plain"}.get(
@@ -896,6 +922,12 @@ def main():
                     help="multi-GPU exchange: peer memory fused into the CG kernels (HALO_PEER 2, "
                          "auto, both CG variants), our separate peer-memory kernels (HALO_PEER 1), "
                          "or NCCL; auto falls back to NCCL if CUDA IPC is refused")
+    ap.add_argument("--transport", choices=["nccl", "peer"], default="nccl",
+                    help="N > 1 library context: NCCL communicator (bootstrap + fallback), or "
+                         "peer-only (CUDA IPC blobs over torch.distributed, no NCCL)")
+    ap.add_argument("--share-device", action="store_true",
+                    help="test of the N > 1 code path on one GPU: all ranks on cuda:0, gloo, "
+                         "peer-only contexts (time-sliced kernels: not a scaling number)")
     ap.add_argument("--cg-variant", choices=["hpccg", "sr"], default="hpccg",
                     help="hpccg: HPCCG's CG (default); sr: single-reduction CG (SURVEY f2)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
