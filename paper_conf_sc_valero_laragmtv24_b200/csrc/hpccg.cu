@@ -1269,10 +1269,10 @@ struct L2Window {
     hpccg_problem *p;
     bool on = false;
     size_t kept = 0;
-    explicit L2Window(hpccg_problem *p_) : p(p_) {
+    L2Window(hpccg_problem *p_, bool want) : p(p_) {
         hpccg_ctx *ctx = p->ctx;
         const Slab &s = p->slabs[0];
-        if (!p->opt_l2 || ctx->max_persist_l2 <= 0 || ctx->max_window <= 0) return;
+        if (!want || !p->opt_l2 || ctx->max_persist_l2 <= 0 || ctx->max_window <= 0) return;
         if (s.arena_bytes > (size_t)ctx->max_persist_l2 || s.arena_bytes > (size_t)ctx->max_window)
             return;
         if (cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, s.arena_bytes) != cudaSuccess) {
@@ -2418,7 +2418,9 @@ int hpccg_solve(hpccg_problem *p, int max_iter, double tol, int *niters, double 
     p->ev_used = 0;
     p->timed.clear();
     const int64_t l0 = ctx->launches;
-    L2Window l2win(p);
+    // the persisting-L2 window costs two device-limit changes per solve; the
+    // persistent kernels keep their small working set on chip / in L2 anyway
+    L2Window l2win(p, !use_persist);
     if (use_while && build_while_graph(p, max_iter, tol) != HPCCG_OK) {
         p->while_failed = true;  // keep the message in hpccg_last_error; fall back
         use_while = false;

@@ -1937,14 +1937,24 @@ __global__ void __launch_bounds__(NT, 1) cg_smem_cluster_kernel(SmemArgs a) {
     const int64_t row0 = (int64_t)me * R;
     const int64_t rem = a.n - row0;
     const int nr = rem <= 0 ? 0 : (int)(rem < R ? rem : R);
-    for (int k = 0; k < kSlots; ++k)
-        for (int i = threadIdx.x; i < nr; i += NT) {
-            sval[k * R + i] = a.val[k * a.stride + row0 + i];
-            scol[k * R + i] = a.col[k * a.stride + row0 + i];
-        }
+    // matrix rows into shared memory: all 27 slots' loads of a row issued before
+    // any store (one HBM round trip per trip instead of one per slot)
     for (int i = threadIdx.x; i < nr; i += NT) {
-        sb[i] = a.b[row0 + i];
-        sx[i] = a.x[row0 + i];
+        double v[kSlots];
+        int cidx[kSlots];
+#pragma unroll
+        for (int k = 0; k < kSlots; ++k) {
+            v[k] = __ldcs(a.val + k * a.stride + row0 + i);
+            cidx[k] = __ldcs(a.col + k * a.stride + row0 + i);
+        }
+        const double bv = a.b[row0 + i], xv = a.x[row0 + i];
+#pragma unroll
+        for (int k = 0; k < kSlots; ++k) {
+            sval[k * R + i] = v[k];
+            scol[k * R + i] = cidx[k];
+        }
+        sb[i] = bv;
+        sx[i] = xv;
     }
     __syncthreads();
     const int plane32 = (int)a.plane;
