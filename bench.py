@@ -654,6 +654,16 @@ def run_ours(args, nx, ny, nz, iters, cfg_index, scaling):
     return 0
 
 
+def f1f4_traffic(key, field):
+    """DRAM bytes of the f1 / f4 hot path from the committed ncu summary
+    (profiles/r1_ncu_f1f4.json, tools/summarize_f1f4.py)."""
+    p = os.path.join(ROOT, "profiles", "r1_ncu_f1f4.json")
+    try:
+        return json.load(open(p)).get(key, {}).get(field)
+    except Exception:
+        return None
+
+
 def traffic_from_profiles(workload):
     """dram bytes per SpMV launch from the committed ncu --set full summary."""
     p = os.path.join(ROOT, "profiles", "spmv_traffic.json")
@@ -839,7 +849,12 @@ def run_tridiag(args):
             "roofline": {"bound": "hbm", "achieved": round(112 * n / (fused_ms * 1e-3) / 1e9, 1),
                          "peak": peak, "unit": "GB/s",
                          "frac": round(112 * n / (fused_ms * 1e-3) / 1e9 / peak, 4),
-                         "peak_source": src},
+                         "peak_source": src,
+                         "kernel": "the fused iteration (tri_spmv<true> + tri_update + tri_pupdate)",
+                         "traffic": (f1f4_traffic("tridiag", "dram_bytes_per_iteration")
+                                     if n == 100_000_000 else None),
+                         "traffic_unit": "DRAM bytes per iteration (ncu, SIZE 1e8)",
+                         "algorithmic_bytes_per_iteration": 112 * n},
             "gpu_launches_per_iteration": launches / (K + 1),
             "clocks": clk.summary(), "cpu_baseline": cpu,
             "speedup_vs_cpu_oracle": (round(cpu["value"] / fused_ms, 1) if cpu else None)}
@@ -898,7 +913,11 @@ def run_lbm(args):
             "MLUPS": round(sites / (ms * 1e-3) / 1e6, 1),
             "roofline": {"bound": "hbm", "achieved": round(gbs, 1), "peak": peak, "unit": "GB/s",
                          "frac": round(gbs / peak, 4), "peak_source": src,
-                         "algorithmic_bytes_per_step": 144 * sites},
+                         "algorithmic_bytes_per_step": 144 * sites,
+                         "kernel": "lbm_pull_kernel<0, 1>",
+                         "traffic": f1f4_traffic("lbm", "dram_bytes_per_launch") if S == 1000 else None,
+                         "traffic_note": "cold-cache ncu replay: the step's writes mostly stay in L2 "
+                                         "(read 72.0 MB = the pulled lattice once)"},
             "clocks": clk.summary(), "cpu_baseline": cpu,
             "speedup_vs_cpu_oracle": round(cpu["value"] / ms, 1) if cpu else None}
     print(json.dumps(line), flush=True)
