@@ -161,6 +161,103 @@ __global__ void __launch_bounds__(kBlk, kMinB) v4(A a) {
     *reinterpret_cast<double2 *>(a.y + r2) = make_double2(s0, s1);
 }
 
+// V5 / V6: the north_star's "shared-memory or TMA staging of x-planes".  A CTA
+// of 256 threads owns 512 rows [r0, r0 + 512) (2 rows / thread, the v4 matrix
+// stream); the x entries those rows can touch lie in three windows (z - 1,
+// z, z + 1 planes: r0 + (dz + 1) plane - (nx + 1) ... + 512 + nx + 1), staged
+// into shared memory -- V5 by three 1-D TMA bulk copies (cp.async.bulk, one
+// mbarrier, issued by one thread while every thread starts its matrix loads),
+// V6 by the CTA's threads (coalesced loads + __syncthreads).  Gathers take
+// slot s's window (s / 9, the generator's sz-major slot order) as a hint and
+// fall back to a global load when the column lies outside it, so any matrix
+// stays correct.  Same FMA order as v0: identical bits.
+struct StageArgs {
+    int64_t plane, ncol;
+    int nx, wmax;  // wmax: doubles per staged window (even)
+};
+
+__device__ __forceinline__ void stage_window(const A &a, const StageArgs &g, int64_t r0, int w,
+                                             int64_t &lo, int &len) {
+    int64_t b = r0 + (int64_t)w * g.plane - (g.nx + 1);  // local-with-halo index of the window start
+    int64_t e = r0 + (int64_t)w * g.plane + 512 + g.nx + 1;
+    b = b < 0 ? 0 : (b & ~(int64_t)1);                   // 16-B aligned start
+    e = e > g.ncol ? g.ncol : ((e + 1) & ~(int64_t)1);
+    lo = b;
+    len = (int)(e - b);
+    if (len > g.wmax) len = g.wmax;
+}
+
+template <bool kTma>
+__global__ void __launch_bounds__(256, 3) v56(A a, StageArgs g) {
+    extern __shared__ __align__(16) double xs[];
+    __shared__ __align__(8) unsigned long long mbar;
+    const int64_t r0 = (int64_t)blockIdx.x * 512;
+    int64_t lo[3];
+    int len[3];
+#pragma unroll
+    for (int w = 0; w < 3; ++w) stage_window(a, g, r0, w, lo[w], len[w]);
+    const unsigned mb = (unsigned)__cvta_generic_to_shared(&mbar);
+    if (kTma) {
+        if (threadIdx.x == 0) {
+            asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(mb));
+            asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+            const unsigned tx = (unsigned)(8 * (len[0] + len[1] + len[2]));
+            asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(mb), "r"(tx) : "memory");
+#pragma unroll
+            for (int w = 0; w < 3; ++w) {
+                const unsigned dst = (unsigned)__cvta_generic_to_shared(xs + w * g.wmax);
+                asm volatile(
+                    "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst),
+                    "l"(a.x + lo[w]), "r"((unsigned)(8 * len[w])), "r"(mb)
+                    : "memory");
+            }
+        }
+    } else {
+        for (int w = 0; w < 3; ++w)
+            for (int i = threadIdx.x; i < len[w]; i += 256) xs[w * g.wmax + i] = __ldg(a.x + lo[w] + i);
+    }
+    const int64_t r2 = r0 + 2 * threadIdx.x;
+    const uint64_t pol = pol_ef();
+    double s0 = 0.0, s1 = 0.0;
+    const bool live = r2 < a.n;
+#pragma unroll
+    for (int gi = 0; gi < 9; ++gi) {
+        double2 vv[3];
+        int2 cc[3];
+        if (live) {
+#pragma unroll
+            for (int t = 0; t < 3; ++t) {
+                vv[t] = lds2(a.val + (3 * gi + t) * a.stride + r2, pol);
+                cc[t] = lds2(a.col + (3 * gi + t) * a.stride + r2, pol);
+            }
+        }
+        if (gi == 0) {  // the staged windows are needed from here on
+            if (kTma) {
+                __syncthreads();  // mbarrier initialised before anyone waits on it
+                unsigned ok = 0;
+                while (!ok)
+                    asm volatile(
+                        "{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], 0; selp.u32 %0, 1, 0, p; }"
+                        : "=r"(ok) : "r"(mb) : "memory");
+            } else {
+                __syncthreads();
+            }
+        }
+        if (live) {
+#pragma unroll
+            for (int t = 0; t < 3; ++t) {
+                const int w = (3 * gi + t) / 9;
+                const int64_t o0 = (int64_t)cc[t].x - lo[w], o1 = (int64_t)cc[t].y - lo[w];
+                const double xa = (uint64_t)o0 < (uint64_t)len[w] ? xs[w * g.wmax + o0] : __ldg(a.x + cc[t].x);
+                const double xb = (uint64_t)o1 < (uint64_t)len[w] ? xs[w * g.wmax + o1] : __ldg(a.x + cc[t].y);
+                s0 = fma(vv[t].x, xa, s0);
+                s1 = fma(vv[t].y, xb, s1);
+            }
+        }
+    }
+    if (live) *reinterpret_cast<double2 *>(a.y + r2) = make_double2(s0, s1);
+}
+
 struct Red {
     double *partials;
     unsigned *counter;
@@ -573,6 +670,20 @@ int main(int argc, char **argv) {
                (h2 - h3) / h3, cudaGetErrorString(cudaGetLastError()));
     }
     RUN("v0_b256_m4_again", (v0<256, 4><<<g256, 256>>>(a)));
+    {   // x-plane staging (north_star): TMA bulk copies vs cooperative loads, vs v4
+        StageArgs sg{plane, ncol, nx, (512 + 2 * (nx + 1) + 4) & ~1};
+        const size_t sm = sizeof(double) * 3 * sg.wmax;
+        cudaFuncSetAttribute(v56<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+        cudaFuncSetAttribute(v56<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+        const unsigned g512 = (unsigned)((n + 511) / 512);
+        for (int rep = 0; rep < 2; ++rep) {
+            RUN("v4_b256_m4_ref", (v4<256, 4><<<(unsigned)((n / 2 + 255) / 256), 256>>>(a)));
+            RUN("v5_tma_staged_x", (v56<true><<<g512, 256, sm>>>(a, sg)));
+            RUN("v6_smem_staged_x", (v56<false><<<g512, 256, sm>>>(a, sg)));
+        }
+        printf("{\"staged_window_doubles\": %d, \"smem_bytes\": %zu, \"err\": \"%s\"}\n", sg.wmax, sm,
+               cudaGetErrorString(cudaGetLastError()));
+    }
     for (int w : {1, 2, 4}) {
         int occ;
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, v3<256, 4>, 256, 0);
