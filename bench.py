@@ -702,6 +702,8 @@ def run_blas1(args):
     if args.blas1_max:
         sizes = [s for s in sizes if s <= args.blas1_max]
     rows = []
+    clk = ClockSampler(local)
+    clk.__enter__()
     for n in sizes:
         # seeded inputs generated once on the host (splitmix64), per-rank shard
         gen = min(n, 1 << 24)
@@ -744,6 +746,7 @@ def run_blas1(args):
                      "dot_exact": (res == exact) if exact is not None else None})
         del x, y
         torch.cuda.empty_cache()
+    clk.__exit__(None, None, None)
     # f3: the 2-D constructs (Fig. 2) at SIZE x SIZE, SIZE = 1000 in the paper
     rows2d = []
     for size in [100, 1000, 10000, 31623]:
@@ -773,9 +776,33 @@ def run_blas1(args):
                        "dot2d_us": round(td * 1e6, 2), "dot2d_GBs": round(world * 16.0 * n / td / 1e9, 1)})
         del x, y
         torch.cuda.empty_cache()
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        # the oracle (as it stands) on a bounded sample: n = 1e8, one AXPY + one DOT
+        import oracle
+        nb = min(sizes[-1], 10 ** 8)
+        xb = np.resize(synth.jacc_vector(min(nb, 1 << 24), 42), nb)
+        yb = np.resize(synth.jacc_vector(min(nb, 1 << 24), 43), nb)
+        wb = np.empty(nb)
+        t0 = time.perf_counter()
+        oracle.waxpby(1.0, xb, 2.5, yb, wb)
+        t1 = time.perf_counter()
+        oracle.ddot(xb, yb)
+        t2 = time.perf_counter()
+        cpu = {"value": round(40.0 * nb / (t2 - t0) / 1e9, 2), "unit": "GB/s",
+               "cores": oracle.get_threads(), "kind": "oracle",
+               "sample": f"oracle waxpby + compensated ddot (C, OpenMP) at n = {nb}: "
+                         f"AXPY {round((t1 - t0) * 1e3, 2)} ms, DOT {round((t2 - t1) * 1e3, 2)} ms"}
+        del xb, yb, wb
     if rank == 0:
         peak, src = peaks()
         big = rows[-1]
+        ach = (24.0 + 16.0) * big["n_per_gpu"] / ((big["axpy_us"] + big["dot_us"]) * 1e-6) / 1e9
+        roof = {"bound": "hbm", "kernel": "waxpby_kernel + dot_kernel at n = %d per GPU (host-synchronous "
+                "calls, launch + sync included)" % big["n_per_gpu"],
+                "achieved": round(ach, 1), "peak": peak, "unit": "GB/s", "frac": round(ach / peak, 4),
+                "peak_source": src, "axpy_GBs": big["axpy_GBs"], "dot_GBs": big["dot_GBs"],
+                "traffic": None}
         line = {"metric": BLAS1_METRIC,
                 "value": round((24.0 + 16.0) * big["n_per_gpu"] * world /
                                ((big["axpy_us"] + big["dot_us"]) * 1e-6) / 1e9, 1),
@@ -785,6 +812,7 @@ def run_blas1(args):
                 "config": {"workload": "blas1", "baseline_config": 4, "sizes": sizes,
                            "parallelism": f"shard{world}"},
                 "sweep": rows, "sweep_2d": rows2d, "peak_hbm_GBs": peak, "peak_source": src,
+                "roofline": roof, "clocks": clk.summary(), "cpu_baseline": cpu,
                 "gpu_launches_per_call": {"axpy": 1, "dot": 1}}
         print(json.dumps(line), flush=True)
     ctx.close()
