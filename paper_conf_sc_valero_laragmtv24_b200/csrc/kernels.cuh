@@ -898,7 +898,7 @@ __device__ __forceinline__ void set_cond(unsigned long long h, int cont) {
 // update block to sum them (> kUpdSumMax): one 1024-thread block, fixed order.
 constexpr unsigned kUpdSumMax = 4096;
 
-__global__ void __launch_bounds__(1024) cg_pap_finish_kernel(const double *parts, unsigned n_parts,
+__global__ void __launch_bounds__(1024, 1) cg_pap_finish_kernel(const double *parts, unsigned n_parts,
                                                              CgScalars *sc) {
     pdl_wait();
     pdl_trigger();
@@ -907,6 +907,20 @@ __global__ void __launch_bounds__(1024) cg_pap_finish_kernel(const double *parts
     // one L2 round trip per 8 instead of a dependent chain of 32)
     double acc[8] = {0.0, 0.0, 0.0, 0.0, 0.0, 0.0, 0.0, 0.0};
     unsigned i = threadIdx.x;
+    // 3 trips' loads (24) in flight, then added trip by trip: the same order as
+    // the 8-wide loop below, so the same bits (262144 partials at 512^3).  The
+    // partials come from the previous grid (complete after pdl_wait), so the
+    // read-only path is valid -- and lets ptxas issue the whole batch at once
+    // (ld.cg loads were interleaved with the adds, ~4 in flight)
+    for (; i + 23u * 1024u < n_parts; i += 24u * 1024u) {
+        double v[24];
+#pragma unroll
+        for (int u = 0; u < 24; ++u) v[u] = __ldg(parts + i + u * 1024u);
+#pragma unroll
+        for (int t = 0; t < 3; ++t)
+#pragma unroll
+            for (int u = 0; u < 8; ++u) acc[u] += v[8 * t + u];
+    }
     for (; i + 7u * 1024u < n_parts; i += 8u * 1024u) {
 #pragma unroll
         for (int u = 0; u < 8; ++u) acc[u] += __ldcg(parts + i + u * 1024u);
@@ -1455,13 +1469,29 @@ __device__ __forceinline__ double2 sr_sum_parts(const double *parts, unsigned np
 // (gamma, delta) partials of one slab -> out[0..1] (one block, fixed order):
 // multi-slab (allreduce input) or a single slab with > kUpdSumMax partials.
 // 1024 threads, 8 loads in flight per thread (65536 partials at 256^3).
-__global__ void __launch_bounds__(1024) cg_sr_finish_kernel(const double *parts, unsigned n_parts,
+__global__ void __launch_bounds__(1024, 1) cg_sr_finish_kernel(const double *parts, unsigned n_parts,
                                                             double *out) {
     pdl_wait();
     pdl_trigger();
     __shared__ double sh[64];
     double g[4] = {0.0, 0.0, 0.0, 0.0}, d[4] = {0.0, 0.0, 0.0, 0.0};
     unsigned i = threadIdx.x;
+    // 3 trips' loads in flight, added trip by trip (same order as below)
+    for (; i + 11u * 1024u < n_parts; i += 12u * 1024u) {
+        double vg[12], vd[12];
+#pragma unroll
+        for (int u = 0; u < 12; ++u) {
+            vg[u] = __ldg(parts + i + u * 1024u);
+            vd[u] = __ldg(parts + n_parts + i + u * 1024u);
+        }
+#pragma unroll
+        for (int t = 0; t < 3; ++t)
+#pragma unroll
+            for (int u = 0; u < 4; ++u) {
+                g[u] += vg[4 * t + u];
+                d[u] += vd[4 * t + u];
+            }
+    }
     for (; i + 3u * 1024u < n_parts; i += 4u * 1024u) {
 #pragma unroll
         for (int u = 0; u < 4; ++u) {
