@@ -168,6 +168,36 @@ def test_ddot_jacc_integer_exact(ctx):
     assert ctx.ddot(n, dev(x), dev(y)) == exact == oracle.ddot(x, y)
 
 
+@pytest.mark.parametrize("n", [10 ** 9, 10 ** 9 - 3])
+def test_blas1_full_size_exact(ctx, n):
+    """BASELINE configs[4] at its largest size (n = 1e9 per GPU, and a ragged
+    1e9 - 3), the bench's calls: DOT of the Fig. 2 integer inputs equals the
+    exact integer (closed form over the inputs' 2^24 period), and the in-place
+    AXPY x += 2.5 y (exact: multiples of 0.5 < 2^53) matches on sampled
+    elements, the ragged tail, and its exact sum (DOT with y = 1)."""
+    import torch
+    P = 1 << 24
+    xb, yb = synth.jacc_vector(P, 42), synth.jacc_vector(P, 43)
+    reps, rem = divmod(n, P)
+    xi, yi = xb.astype(np.int64), yb.astype(np.int64)
+    exact_dot = reps * int(np.dot(xi, yi)) + int(np.dot(xi[:rem], yi[:rem]))
+    x = dev(xb).repeat(reps + 1)[:n].contiguous()
+    y = dev(yb).repeat(reps + 1)[:n].contiguous()
+    torch.cuda.synchronize()   # torch's kernels ran on its stream; the library has its own
+    assert ctx.ddot(n, x.data_ptr(), y.data_ptr()) == float(exact_dot)
+    ctx.waxpby(n, 1.0, x.data_ptr(), 2.5, y.data_ptr(), x.data_ptr())
+    rng = np.random.default_rng(5)
+    idx = np.concatenate([rng.integers(0, n, 4096), np.arange(n - 64, n), np.arange(64)])
+    got = x[torch.from_numpy(idx).cuda()].cpu().numpy()
+    np.testing.assert_array_equal(got, xb[idx % P] + 2.5 * yb[idx % P])
+    del y
+    ones = torch.ones(n, dtype=torch.float64, device="cuda")
+    torch.cuda.synchronize()
+    w = xb + 2.5 * yb
+    exact_sum = reps * float(np.sum(2 * w)) / 2 + float(np.sum(2 * w[:rem])) / 2
+    assert ctx.ddot(n, x.data_ptr(), ones.data_ptr()) == exact_sum
+
+
 def test_ddot_misaligned_scalar_path(ctx):
     n = 4097
     buf = dev(synth.uniform(n + 1, 8))
