@@ -383,6 +383,8 @@ def run_ours(args, nx, ny, nz, iters, cfg_index, scaling):
     prob.set_option(H.HPCCG_OPT_GRAPH, 1)
     sr = args.cg_variant == "sr"
     prob.set_option(H.HPCCG_OPT_CG_VARIANT, 1 if sr else 0)
+    dia = args.spmv_format == "dia"
+    prob.set_option(H.HPCCG_OPT_SPMV_FORMAT, 1 if dia else 0)
     halo = "none (1 slab)"
     if world > 1 and transport == "peer":
         # peer-only context: no NCCL anywhere; every rank maps its neighbours' buffers
@@ -564,7 +566,9 @@ def run_ours(args, nx, ny, nz, iters, cfg_index, scaling):
 
     if rank == 0:
         peak, peak_src = peaks()
-        spmv_bytes = 12.0 * nnz_local + 16.0 * n
+        # ELL-27: 8 B value + 4 B column per stored entry, x read + y written once;
+        # DIA-27 (--spmv-format dia): all 27 value slots (padding included), no columns
+        spmv_bytes = (216.0 * n if dia else 12.0 * nnz_local) + 16.0 * n
         roof = None
         if spmv_n > 0 and spmv_ms > 0:
             avg_ms = spmv_ms / spmv_n
@@ -572,11 +576,13 @@ def run_ours(args, nx, ny, nz, iters, cfg_index, scaling):
             roof = {"bound": "hbm",
                     "kernel": ("spmv27x2_kernel<2> (w = A r with the r.r, w.r epilogue, f2)" if sr else
                                "spmv27x2_kernel<1> (p.Ap epilogue)") +
-                              " -- 2 rows/thread; spmv27_kernel if n or the plane is odd",
+                              " -- 2 rows/thread; spmv27_kernel if n or the plane is odd" +
+                              ("; DIA-27 reading (columns formed from the stencil offsets, "
+                               "216n + 16n B per launch)" if dia else ""),
                     "achieved": round(ach, 1),
                     "peak": peak, "unit": "GB/s", "frac": round(ach / peak, 4),
                     "frac_of_8TBs_nominal": round(ach / 8000.0, 4),
-                    "traffic": traffic_from_profiles(args.workload),
+                    "traffic": traffic_from_profiles(args.workload + ("_dia" if dia else "")),
                     "algorithmic_bytes_per_launch": spmv_bytes, "avg_launch_us": round(avg_ms * 1e3, 2),
                     "peak_source": peak_src,
                     "spmv_share_of_step": round(spmv_ms / ev["ms"], 4) if ev["ms"] > 0 else None,
@@ -628,6 +634,8 @@ def run_ours(args, nx, ny, nz, iters, cfg_index, scaling):
                        "global_rows": n * world, "global_nnz": nnz_global,
                        "parallelism": f"zslab{world}",
                        "cg_variant": "single-reduction (Chronopoulos-Gear, f2)" if sr else "HPCCG",
+                       "spmv_format": "DIA-27 (val[27][n], columns from stencil offsets)" if dia
+                                      else "ELL-27 (val[27][n] + col[27][n])",
                        "halo": halo, "transport": transport if world > 1 else None,
                        "shared_device": bool(share),
                        "solve_graph": {5: "on-chip cluster kernel", 4: "one-cluster persistent kernel",
@@ -977,6 +985,8 @@ def main():
                          "peer-only contexts (time-sliced kernels: not a scaling number)")
     ap.add_argument("--cg-variant", choices=["hpccg", "sr"], default="hpccg",
                     help="hpccg: HPCCG's CG (default); sr: single-reduction CG (SURVEY f2)")
+    ap.add_argument("--spmv-format", choices=["ell", "dia"], default="ell",
+                    help="HPCCG_OPT_SPMV_FORMAT: ELL-27 (default) or the DIA-27 reading (no col[])")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-budget", type=float, default=12.0, help="seconds of oracle CG")
     ap.add_argument("--ref-iters", type=int, default=20, help="oracle iterations per reference step")

@@ -148,6 +148,15 @@ extern "C" {
                                auto, 3 when the CG vectors exceed L2 (256^3), else 0 */
 #define HPCCG_OPT_VEC_WAVES 6 /* CG vector kernels: 0 one thread per 16-B unit; k > 0
                                (default 1): a persistent grid of k resident waves */
+#define HPCCG_OPT_SPMV_FORMAT 21 /* how the 2-rows/thread SpMV reads A: 0 (default) ELL-27,
+                               val[27][n] + col[27][n] (12 B per slot); 1 DIA-27, val only:
+                               slot s's column is formed from its stencil offset
+                               (s/9-1)*nx*ny + (s/3%3-1)*nx + (s%3-1), a 0.0 value selecting
+                               the padding column -- bitwise identical results (8 B per
+                               slot).  Valid because hpccg_generate is the only source of
+                               A (A: diag 27, -1 per existing neighbour, BJ:north_star).
+                               Not used by the 1-row/thread, persistent, on-chip or
+                               HALO_PEER = 2 kernels (those read col[]). */
 
 typedef struct hpccg_ctx hpccg_ctx;         /* device, streams, comm (rank, nranks) */
 typedef struct hpccg_problem hpccg_problem; /* A (ELL-27), b, x, x_exact, CG work vectors */

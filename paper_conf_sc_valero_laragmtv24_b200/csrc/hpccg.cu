@@ -127,6 +127,8 @@ struct Slab {
     PeerSync *psync = nullptr;  // HALO_PEER: this slab's flags / allreduce slots
     PeerTab *ptab = nullptr;    // HALO_PEER: device copy of the peer table
     int early_trigger = 1;      // HPCCG_OPT_PDL 1: SpMV triggers its successor early
+    int nx = 0;                 // grid row stride (DIA-27 column formation)
+    int dia = 0;                // HPCCG_OPT_SPMV_FORMAT 1: DIA-27 SpMV (col[] not read)
 };
 
 struct TimedOp {
@@ -433,6 +435,8 @@ SpmvArgs spmv_args(const Slab &s, const double *x, double *y) {
     a.sc = s.sc;
     a.red = s.red;
     a.early_trigger = s.early_trigger;
+    a.nx = s.nx;
+    a.dia = s.dia;
     return a;
 }
 
@@ -475,8 +479,14 @@ int launch_spmv(hpccg_ctx *ctx, int minb, bool check, SpmvArgs a, int64_t r0, in
     if (blocks == 0) return HPCCG_OK;
     if (blocks > 0x7fffffffLL) return fail(HPCCG_EINVAL, "SpMV grid too large");
     if (rows == 2) {
-        if (check) launch_k(pdl, spmv27x2_kernel<kDots, true>, dim3((unsigned)blocks), st, a);
-        else launch_k(pdl, spmv27x2_kernel<kDots, false>, dim3((unsigned)blocks), st, a);
+        if (a.dia) {
+            if (check) launch_k(pdl, spmv27x2_kernel<kDots, true, false, true>, dim3((unsigned)blocks), st, a);
+            else launch_k(pdl, spmv27x2_kernel<kDots, false, false, true>, dim3((unsigned)blocks), st, a);
+        } else if (check) {
+            launch_k(pdl, spmv27x2_kernel<kDots, true>, dim3((unsigned)blocks), st, a);
+        } else {
+            launch_k(pdl, spmv27x2_kernel<kDots, false>, dim3((unsigned)blocks), st, a);
+        }
         return check_launch(ctx);
     }
     if (minb <= 0) minb = kSpmvMinBDefault;
@@ -1997,6 +2007,7 @@ int hpccg_generate(hpccg_ctx *ctx, int nx, int ny, int nz, hpccg_problem **out) 
         s.n = n;
         s.plane = plane;
         s.ncol = ncol;
+        s.nx = nx;
         int rc;
         if ((rc = alloc_zero((void **)&s.val, sizeof(double) * kSlots * n))) return bail(rc);
         if ((rc = alloc_zero((void **)&s.col, sizeof(int) * kSlots * n))) return bail(rc);
@@ -2206,6 +2217,10 @@ int hpccg_set_option(hpccg_problem *p, int key, int64_t value) {
             p->opt_persist = (int)value;
             return HPCCG_OK;
         case HPCCG_OPT_SMEM_SOLVE: p->opt_smem = value != 0; return HPCCG_OK;
+        case HPCCG_OPT_SPMV_FORMAT:
+            if (value != 0 && value != 1) return fail(HPCCG_EINVAL, "spmv format: 0 (ELL-27) or 1 (DIA-27)");
+            for (Slab &sl : p->slabs) sl.dia = (int)value;
+            return HPCCG_OK;
         case HPCCG_OPT_FINISHER_FREE: p->opt_ff = value != 0; return HPCCG_OK;
         case HPCCG_OPT_SERPENTINE:
             if (value < -1 || value > 3) return fail(HPCCG_EINVAL, "serpentine: bit mask 0..3 or -1 (auto)");

@@ -491,6 +491,8 @@ struct SpmvArgs {
     int rev;           // 1: block b takes the rows (and the partial slot) of block
                        // gridDim - 1 - b, i.e. the grid walks the rows backwards
                        // (same rows per block, same partials: identical bits)
+    int nx;            // kDia (HPCCG_OPT_SPMV_FORMAT 1): row stride of the grid
+    int dia;           // 1: spmv27x2_kernel<., ., false, true> (DIA-27, col[] not read)
 };
 
 // the row block this CTA handles (HPCCG_OPT_SERPENTINE)
@@ -664,7 +666,25 @@ __device__ __forceinline__ double ld_gather(const double *p) {
     return kCoh ? __ldcg(p) : __ldg(p);
 }
 
-template <int kDots, bool kCheck, bool kFused, bool kCoh>
+// kDia (HPCCG_OPT_SPMV_FORMAT = 1, DIA-27 reading of the same ELL): the column
+// of slot s is not loaded but formed from the stencil offset the generator
+// placed there (gen27_kernel: col = own + sz*plane + sy*nx + sx when the
+// neighbour exists, else the padding (0.0, own)); a zero value selects the
+// padding column, so every FMA sees the same (val, x) pair as the ELL kernel
+// and the result is bitwise identical.  Valid for matrices made by
+// hpccg_generate (the only source of matrices in this library): structurally
+// present entries are 27 or -1, never 0.  Saves the 4 B/slot index stream:
+// 216 B/row of values instead of 324 B/row of values + indices.
+template <bool kDia>
+__device__ __forceinline__ int2 spmv_cols(const SpmvArgs &a, const int *c, int s, double2 v, int64_t row,
+                                          uint64_t pol) {
+    if (!kDia) return ld_stream2(c + s * a.stride, pol);
+    const int own = (int)(row + a.plane);
+    const int off = (s / 9 - 1) * (int)a.plane + ((s / 3) % 3 - 1) * a.nx + (s % 3 - 1);
+    return make_int2(v.x != 0.0 ? own + off : own, v.y != 0.0 ? own + 1 + off : own + 1);
+}
+
+template <int kDots, bool kCheck, bool kFused, bool kCoh, bool kDia = false>
 __device__ __forceinline__ void spmv27x2_body(const SpmvArgs &a, int64_t row, int64_t lim, int64_t bid) {
     constexpr bool kDot = kDots == 1;
     double d = 0.0, dg = 0.0;  // kDots 1: p.Ap; kDots 2: delta (d) and gamma (dg)
@@ -682,7 +702,7 @@ __device__ __forceinline__ void spmv27x2_body(const SpmvArgs &a, int64_t row, in
 #pragma unroll
             for (int t = 0; t < 3; ++t) {
                 vv[t] = ld_stream2(v + (3 * g + t) * a.stride, pol);
-                cc[t] = ld_stream2(c + (3 * g + t) * a.stride, pol);
+                if (!kDia) cc[t] = ld_stream2(c + (3 * g + t) * a.stride, pol);
             }
             if (g == 0) {
                 pdl_wait();
@@ -693,6 +713,7 @@ __device__ __forceinline__ void spmv27x2_body(const SpmvArgs &a, int64_t row, in
             }
 #pragma unroll
             for (int t = 0; t < 3; ++t) {
+                if (kDia) cc[t] = spmv_cols<true>(a, c, 3 * g + t, vv[t], row, pol);
                 const double xa = ld_gather<kCoh>(a.x + cc[t].x), xb = ld_gather<kCoh>(a.x + cc[t].y);
                 if (3 * g + t == kDiagSlot) {
                     x0 = xa;
@@ -758,7 +779,7 @@ __device__ __forceinline__ void spmv27x2_body(const SpmvArgs &a, int64_t row, in
 }
 
 
-template <int kDots, bool kCheck, bool kFused = false>
+template <int kDots, bool kCheck, bool kFused = false, bool kDia = false>
 __global__ void __launch_bounds__(kBlock, 4) spmv27x2_kernel(SpmvArgs a) {
     int64_t row, lim;
     const int64_t bid = spmv_bid(a);
@@ -793,7 +814,7 @@ __global__ void __launch_bounds__(kBlock, 4) spmv27x2_kernel(SpmvArgs a) {
         spmv27x2_body<kDots, kCheck, kFused, true>(a, row, lim, bid);
         return;
     }
-    spmv27x2_body<kDots, kCheck, kFused, false>(a, row, lim, bid);
+    spmv27x2_body<kDots, kCheck, kFused, false, kDia>(a, row, lim, bid);
 }
 
 // ------------------------------------------------ streaming vector kernels
