@@ -155,8 +155,8 @@ extern "C" {
                                the padding column -- bitwise identical results (8 B per
                                slot).  Valid because hpccg_generate is the only source of
                                A (A: diag 27, -1 per existing neighbour, BJ:north_star).
-                               Not used by the 1-row/thread, persistent, on-chip or
-                               HALO_PEER = 2 kernels (those read col[]). */
+                               Not used by the 1-row/thread, persistent or on-chip
+                               kernels (those read col[]). */
 
 typedef struct hpccg_ctx hpccg_ctx;         /* device, streams, comm (rank, nranks) */
 typedef struct hpccg_problem hpccg_problem; /* A (ELL-27), b, x, x_exact, CG work vectors */

@@ -55,6 +55,7 @@ def build(force: bool = False, verbose: bool = False) -> str:
     if inc:
         cmd += ["-DHPCCG_WITH_NCCL", "-I", inc, "-L", lib, "-l:libnccl.so.2",
                 "-Xlinker", "-rpath=" + lib]
+    cmd += os.environ.get("HPCCG_NVCC_EXTRA", "").split()  # tuning builds (tools/)
     tmp = LIB + ".tmp.%d" % os.getpid()
     cmd += ["-o", tmp, os.path.join(CSRC, "hpccg.cu")]
     res = subprocess.run(cmd, capture_output=True, text=True)

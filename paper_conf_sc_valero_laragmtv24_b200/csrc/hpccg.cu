@@ -790,8 +790,14 @@ int launch_spmv_fused(hpccg_problem *p, const Slab &s, bool check, unsigned *npa
     const bool pdl = p->opt_pdl != 0;
     a.sr_q = sr_q;
     if (kDots == 2) a.trace = nullptr;
-    if (check) launch_k(pdl, spmv27x2_kernel<kDots, true, true>, dim3((unsigned)blocks), p->ctx->stream, a);
-    else launch_k(pdl, spmv27x2_kernel<kDots, false, true>, dim3((unsigned)blocks), p->ctx->stream, a);
+    if (a.dia) {
+        if (check) launch_k(pdl, spmv27x2_kernel<kDots, true, true, true>, dim3((unsigned)blocks), p->ctx->stream, a);
+        else launch_k(pdl, spmv27x2_kernel<kDots, false, true, true>, dim3((unsigned)blocks), p->ctx->stream, a);
+    } else if (check) {
+        launch_k(pdl, spmv27x2_kernel<kDots, true, true>, dim3((unsigned)blocks), p->ctx->stream, a);
+    } else {
+        launch_k(pdl, spmv27x2_kernel<kDots, false, true>, dim3((unsigned)blocks), p->ctx->stream, a);
+    }
     return check_launch(p->ctx);
 }
 

@@ -675,6 +675,12 @@ __device__ __forceinline__ double ld_gather(const double *p) {
 // hpccg_generate (the only source of matrices in this library): structurally
 // present entries are 27 or -1, never 0.  Saves the 4 B/slot index stream:
 // 216 B/row of values instead of 324 B/row of values + indices.
+#ifndef HPCCG_DIA_GROUP
+#define HPCCG_DIA_GROUP 9  // measured: 9 > 3 (27 spills at 64 registers), DESIGN.md sec. 7.1
+#endif
+constexpr int kDiaGroup = HPCCG_DIA_GROUP;  // 3 or 9
+static_assert(kSlots % kDiaGroup == 0, "DIA group must divide 27");
+
 template <bool kDia>
 __device__ __forceinline__ int2 spmv_cols(const SpmvArgs &a, const int *c, int s, double2 v, int64_t row,
                                           uint64_t pol) {
@@ -695,14 +701,17 @@ __device__ __forceinline__ void spmv27x2_body(const SpmvArgs &a, int64_t row, in
         const int *c = a.col + row;
         double s0 = 0.0, s1 = 0.0, x0 = 0.0, x1 = 0.0;
         int c0 = 0, c1 = 0;
+        // slots whose loads are issued together: 3 (ELL: 72 B per thread in
+        // flight); DIA has no index stream, so it takes kDiaGroup slots
+        constexpr int kG = kDia ? kDiaGroup : 3;
 #pragma unroll
-        for (int g = 0; g < 9; ++g) {
-            double2 vv[3];
-            int2 cc[3];
+        for (int g = 0; g < kSlots / kG; ++g) {
+            double2 vv[kG];
+            int2 cc[kG];
 #pragma unroll
-            for (int t = 0; t < 3; ++t) {
-                vv[t] = ld_stream2(v + (3 * g + t) * a.stride, pol);
-                if (!kDia) cc[t] = ld_stream2(c + (3 * g + t) * a.stride, pol);
+            for (int t = 0; t < kG; ++t) {
+                vv[t] = ld_stream2(v + (kG * g + t) * a.stride, pol);
+                if (!kDia) cc[t] = ld_stream2(c + (kG * g + t) * a.stride, pol);
             }
             if (g == 0) {
                 pdl_wait();
@@ -712,10 +721,10 @@ __device__ __forceinline__ void spmv27x2_body(const SpmvArgs &a, int64_t row, in
                 if (done) return;  // uniform over the grid, before any store
             }
 #pragma unroll
-            for (int t = 0; t < 3; ++t) {
-                if (kDia) cc[t] = spmv_cols<true>(a, c, 3 * g + t, vv[t], row, pol);
+            for (int t = 0; t < kG; ++t) {
+                if (kDia) cc[t] = spmv_cols<true>(a, c, kG * g + t, vv[t], row, pol);
                 const double xa = ld_gather<kCoh>(a.x + cc[t].x), xb = ld_gather<kCoh>(a.x + cc[t].y);
-                if (3 * g + t == kDiagSlot) {
+                if (kG * g + t == kDiagSlot) {
                     x0 = xa;
                     x1 = xb;
                     c0 = cc[t].x;
@@ -811,7 +820,7 @@ __global__ void __launch_bounds__(kBlock, 4) spmv27x2_kernel(SpmvArgs a) {
         }
     }
     if (kFused && bnd) {
-        spmv27x2_body<kDots, kCheck, kFused, true>(a, row, lim, bid);
+        spmv27x2_body<kDots, kCheck, kFused, true, kDia>(a, row, lim, bid);
         return;
     }
     spmv27x2_body<kDots, kCheck, kFused, false, kDia>(a, row, lim, bid);

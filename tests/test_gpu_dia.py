@@ -78,7 +78,7 @@ def _solve(p, fmt, max_iter, tol, while_graph=1, variant=0):
     p.set_option(H.HPCCG_OPT_SPMV_FORMAT, fmt)
     p.set_option(H.HPCCG_OPT_WHILE, while_graph)
     p.set_option(H.HPCCG_OPT_CG_VARIANT, variant)
-    p.set_vec(H.HPCCG_VEC_X, np.zeros(p.n))
+    p.set_vec(H.HPCCG_VEC_X, np.zeros(p.n * p.ctx.nslabs))
     r = p.solve(max_iter, tol)
     return r["niters"], r["normr"], p.get_vec(H.HPCCG_VEC_X)
 
@@ -124,3 +124,25 @@ def test_dia_full_128cubed_bitwise_to_ell(ctx):
         b = _solve(p, 1, 500, 0.0)
     assert a[:2] == b[:2]
     np.testing.assert_array_equal(a[2], b[2])
+
+
+@pytest.mark.parametrize("P,dims", [(2, (12, 10, 6)), (3, (8, 8, 2)), (2, (16, 16, 1))])
+def test_dia_fused_peer_path_bitwise(P, dims):
+    """HALO_PEER = 2 (halo push / wait and allreduces fused into the CG
+    kernels): the DIA reading of the boundary blocks' halo gathers (coherent
+    loads after the flag wait) gives the ELL run's bits, for both CG variants
+    and every exchange mode."""
+    nx, ny, nz = dims
+    with H.Context(0, nranks=P, loopback=True) as c, H.Problem(c, nx, ny, nz) as p:
+        for variant in (0, 1):
+            outs = []
+            for fmt, peer in [(0, 2), (1, 2), (1, 1), (1, 0)]:
+                p.set_option(H.HPCCG_OPT_HALO_PEER, peer)
+                p.set_option(H.HPCCG_OPT_SPMV_FORMAT, fmt)
+                p.set_option(H.HPCCG_OPT_CG_VARIANT, variant)
+                p.set_vec(H.HPCCG_VEC_X, np.zeros(p.n * P))
+                r = p.solve(150, 1e-12)
+                outs.append((r["niters"], r["normr"], p.get_vec(H.HPCCG_VEC_X)))
+            for o in outs[1:]:
+                assert o[:2] == outs[0][:2]
+                np.testing.assert_array_equal(o[2], outs[0][2])
