@@ -679,6 +679,10 @@ __device__ __forceinline__ double ld_gather(const double *p) {
 #define HPCCG_DIA_GROUP 9  // measured: 9 > 3 (27 spills at 64 registers), DESIGN.md sec. 7.1
 #endif
 constexpr int kDiaGroup = HPCCG_DIA_GROUP;  // 3 or 9
+#ifndef HPCCG_DIA_MINB
+#define HPCCG_DIA_MINB 4  // resident 256-thread blocks per SM (64 registers)
+#endif
+constexpr int kDiaMinB = HPCCG_DIA_MINB;
 static_assert(kSlots % kDiaGroup == 0, "DIA group must divide 27");
 
 template <bool kDia>
@@ -789,7 +793,7 @@ __device__ __forceinline__ void spmv27x2_body(const SpmvArgs &a, int64_t row, in
 
 
 template <int kDots, bool kCheck, bool kFused = false, bool kDia = false>
-__global__ void __launch_bounds__(kBlock, 4) spmv27x2_kernel(SpmvArgs a) {
+__global__ void __launch_bounds__(kBlock, kDia ? kDiaMinB : 4) spmv27x2_kernel(SpmvArgs a) {
     int64_t row, lim;
     const int64_t bid = spmv_bid(a);
     bool bnd = false;
