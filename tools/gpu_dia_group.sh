@@ -1,7 +1,11 @@
 #!/bin/bash
 # DIA-27 SpMV tuning: slots per load group (HPCCG_DIA_GROUP) x resident blocks
 # (HPCCG_DIA_MINB), libraries prebuilt as tools/libhpccg_g<G>_m<M>.so (git-ignored);
-# bench lines at 128^3 / 256^3, alternating.
+# bench lines at 128^3 / 256^3, alternating.  Build the variants here first:
+#   for v in "9 4" "9 3" "27 2"; do set -- $v; HPCCG_NVCC_EXTRA="-DHPCCG_DIA_GROUP=$1 -DHPCCG_DIA_MINB=$2" \
+#     python -c "from paper_conf_sc_valero_laragmtv24_b200 import _build; _build.build(force=True)"; \
+#     cp paper_conf_sc_valero_laragmtv24_b200/libhpccg.so tools/libhpccg_g$1_m$2.so; done
+# (then rebuild the default library).
 mkdir -p gpurun_out
 L=paper_conf_sc_valero_laragmtv24_b200/libhpccg.so
 cp $L /tmp/libhpccg_default.so
