@@ -82,9 +82,12 @@ extern "C" {
 #define HPCCG_OPT_VEC_UNROLL 8 /* CG vector kernels: 16-B units per thread per trip with
                                all loads in flight: 1, 2 or 4 (default 4) */
 #define HPCCG_OPT_PERSISTENT 9 /* single GPU: run the whole solve as ONE cooperative kernel
-                               (grid barriers between phases): 0 never, 1 (default) when
-                               nrow_local <= HPCCG_OPT_PERSIST_ROWS, 2 always */
-#define HPCCG_OPT_PERSIST_ROWS 10 /* threshold for HPCCG_OPT_PERSISTENT = 1 (default 65536) */
+                               (grid barriers between phases): 0 never, 1 (default) auto
+                               (HPCCG_OPT_PERSIST_ROWS), 2 always */
+#define HPCCG_OPT_PERSIST_ROWS 10 /* threshold for HPCCG_OPT_PERSISTENT = 1: -1 (default) only
+                               when the whole problem fits the on-chip (shared-memory) solve
+                               (the while-graph is faster above that); k >= 0:
+                               when nrow_local <= k */
 #define HPCCG_OPT_SMEM_SOLVE 13 /* 1 (default): a persistent solve whose rows fit in the
                                shared memory of one 16-CTA cluster (~9.9k rows) keeps the whole
                                problem on chip (distributed shared memory gathers); 0: off */

@@ -149,9 +149,12 @@ struct hpccg_problem {
     int opt_vec_waves = 1;  // 0: one thread per double2 (full grid); k: k resident waves
     int opt_rows = 2;       // SpMV rows per thread (2 when aligned, else 1)
     int opt_unroll = 4;     // CG vector kernels: 16-B units per thread per trip
-    int opt_persist = 1;    // 0 never, 1 auto (n <= opt_persist_rows), 2 always (single slab)
+    int opt_persist = 1;    // 0 never, 1 auto (see opt_persist_rows), 2 always (single slab)
     int opt_pdl = 1;        // programmatic dependent launch between the CG kernels
-    int64_t opt_persist_rows = 65536;
+    // auto threshold: -1 (default) = only when the on-chip (shared-memory) solve fits --
+    // the while-graph beats the grid / one-cluster persistent solves at every size
+    // above that; k >= 0 = when n <= k
+    int64_t opt_persist_rows = -1;
     int64_t opt_cluster_rows = 16384;  // persistent solve as one cluster up to this many rows
     int opt_smem = 1;                  // persistent solve resident in cluster shared memory if it fits
     int opt_while_unroll = 4;          // CG iterations per WHILE-body execution
@@ -2269,7 +2272,7 @@ int hpccg_set_option(hpccg_problem *p, int key, int64_t value) {
             p->opt_cluster_rows = value;
             return HPCCG_OK;
         case HPCCG_OPT_PERSIST_ROWS:
-            if (value < 0) return fail(HPCCG_EINVAL, "persist rows must be >= 0");
+            if (value < -1) return fail(HPCCG_EINVAL, "persist rows must be >= 0 or -1 (auto)");
             p->opt_persist_rows = value;
             return HPCCG_OK;
         case HPCCG_OPT_VEC_UNROLL:
@@ -2431,7 +2434,8 @@ int hpccg_solve(hpccg_problem *p, int max_iter, double tol, int *niters, double 
     const bool use_persist = !timing && ctx->mode == MODE_SINGLE &&
                              (p->opt_variant == 0 || smem_rows(p) > 0) &&
                              (p->opt_persist == 2 ||
-                              (p->opt_persist == 1 && p->slabs[0].n <= p->opt_persist_rows));
+                              (p->opt_persist == 1 && (p->opt_persist_rows < 0 ? smem_rows(p) > 0
+                                                                             : p->slabs[0].n <= p->opt_persist_rows)));
     // NCCL calls cannot live in a conditional graph body; with HALO_PEER the
     // multi-GPU iteration is our own kernels only, so it can
     bool use_while = !use_persist && use_graph && p->opt_while && (ctx->mode != MODE_NCCL || peer_on(p)) &&

@@ -352,13 +352,26 @@ def test_cg_persistent_grid_and_cluster_variants(ctx, crows, smem, mode):
 
 
 def test_cg_persistent_auto_threshold(ctx):
-    with H.Problem(ctx, 20, 30, 10) as p:       # 6000 rows <= 65536: persistent
+    with H.Problem(ctx, 20, 30, 10) as p:       # 6000 rows fit on chip: persistent
         p.solve(150, 1e-12)
         assert p.stats()["graph_mode"] in (3, 4, 5)
         p.set_option(H.HPCCG_OPT_PERSIST_ROWS, 1000)
         p.set_vec(H.HPCCG_VEC_X, np.zeros(p.n))
         p.solve(150, 1e-12)
         assert p.stats()["graph_mode"] == 2
+    # auto (-1): above the on-chip size the while-graph (faster there, DESIGN 7.1);
+    # an explicit threshold still selects the grid / one-cluster persistent solve
+    with H.Problem(ctx, 32, 32, 32) as p:
+        r0 = p.solve(150, 1e-12)
+        assert p.stats()["graph_mode"] == 2
+        p.set_option(H.HPCCG_OPT_PERSIST_ROWS, 65536)
+        p.set_vec(H.HPCCG_VEC_X, np.zeros(p.n))
+        r1 = p.solve(150, 1e-12)
+        assert p.stats()["graph_mode"] in (3, 4)
+        assert abs(r0["niters"] - r1["niters"]) <= 1
+        p.set_option(H.HPCCG_OPT_PERSIST_ROWS, -1)
+        with pytest.raises(H.HpccgError):
+            p.set_option(H.HPCCG_OPT_PERSIST_ROWS, -2)
 
 
 def test_cg_first_step_exact(ctx):
