@@ -158,8 +158,10 @@ extern "C" {
                                the padding column -- bitwise identical results (8 B per
                                slot).  Valid because hpccg_generate is the only source of
                                A (A: diag 27, -1 per existing neighbour, BJ:north_star).
-                               Not used by the 1-row/thread, persistent or on-chip
-                               kernels (those read col[]). */
+                               The on-chip (shared-memory) solve drops its column slice
+                               under 1 when the ELL slice does not fit (more rows on chip);
+                               the 1-row/thread SpMV and the grid / one-cluster persistent
+                               solves read col[]. */
 
 typedef struct hpccg_ctx hpccg_ctx;         /* device, streams, comm (rank, nranks) */
 typedef struct hpccg_problem hpccg_problem; /* A (ELL-27), b, x, x_exact, CG work vectors */

@@ -1330,15 +1330,25 @@ struct L2Window {
 
 // Shared-memory-resident solve: bytes per row (ELL slice + vectors) and the
 // rows per CTA when the problem fits one cluster (0: it does not).
-int64_t smem_bytes_per_row(bool sr) {
-    return kSlots * (int64_t)(sizeof(double) + sizeof(int)) + (sr ? 6 : 5) * (int64_t)sizeof(double);
+// (DIA-27 reading, HPCCG_OPT_SPMV_FORMAT 1: no column slice)
+int64_t smem_bytes_per_row(bool sr, bool dia) {
+    return kSlots * (int64_t)(sizeof(double) + (dia ? 0 : sizeof(int))) + (sr ? 6 : 5) * (int64_t)sizeof(double);
 }
 
 int64_t smem_rows(const hpccg_problem *p) {
     const hpccg_ctx *ctx = p->ctx;
     if (!p->opt_smem || ctx->smem_cluster <= 1 || ctx->mode != MODE_SINGLE) return 0;
     const int64_t R = cdiv(p->slabs[0].n, ctx->smem_cluster);
-    return R * smem_bytes_per_row(p->opt_variant == 1) <= ctx->smem_bytes ? R : 0;
+    const bool sr = p->opt_variant == 1;
+    // DIA (format 1) drops the column slice only where the ELL slice does not fit:
+    // on chip, forming the column from the value costs more than reading it (DESIGN 7.1)
+    if (R * smem_bytes_per_row(sr, false) <= ctx->smem_bytes) return R;
+    return p->slabs[0].dia && R * smem_bytes_per_row(sr, true) <= ctx->smem_bytes ? R : 0;
+}
+
+// the on-chip solve keeps no column slice (DIA reading): format 1 and the ELL slice does not fit
+bool smem_dia(const hpccg_problem *p, int64_t R) {
+    return p->slabs[0].dia && R * smem_bytes_per_row(p->opt_variant == 1, false) > p->ctx->smem_bytes;
 }
 
 // The whole solve in one cooperative kernel (small single-slab problems).
@@ -1364,15 +1374,17 @@ int launch_persistent(hpccg_problem *p, int max_iter, double tol) {
     a.tol = tol;
     // whole problem in one cluster's shared memory when it fits
     const bool sr = p->opt_variant == 1;
-    const int64_t bytes_per_row = smem_bytes_per_row(sr);
     {
         const int64_t R = smem_rows(p);
+        const int64_t bytes_per_row = smem_bytes_per_row(sr, smem_dia(p, R));
         if (R > 0) {
             SmemArgs m{};
             m.n = s.n;
             m.stride = s.n;
             m.plane = s.plane;
             m.R = (int)R;
+            m.nx = s.nx;
+            m.dia = smem_dia(p, R) ? 1 : 0;
             m.val = s.val;
             m.col = s.col;
             m.b = s.b;

@@ -1905,6 +1905,7 @@ __global__ void __launch_bounds__(kBlock, 1) cg_persistent_kernel(PersistArgs a)
 struct SmemArgs {
     int64_t n, stride, plane;
     int R;  // rows per CTA
+    int nx, dia;  // dia: DIA-27 reading (HPCCG_OPT_SPMV_FORMAT 1) -- no column slice in smem
     const double *val;
     const int *col;
     const double *b;
@@ -2009,13 +2010,13 @@ __global__ void __launch_bounds__(NT, 1) cg_smem_cluster_kernel(SmemArgs a) {
 #pragma unroll
         for (int k = 0; k < kSlots; ++k) {
             v[k] = __ldcs(a.val + k * a.stride + row0 + i);
-            cidx[k] = __ldcs(a.col + k * a.stride + row0 + i);
+            cidx[k] = a.dia ? 0 : __ldcs(a.col + k * a.stride + row0 + i);
         }
         const double bv = a.b[row0 + i], xv = a.x[row0 + i];
 #pragma unroll
         for (int k = 0; k < kSlots; ++k) {
             sval[k * R + i] = v[k];
-            scol[k * R + i] = cidx[k];
+            if (!a.dia) scol[k * R + i] = cidx[k];
         }
         sb[i] = bv;
         sx[i] = xv;
@@ -2025,9 +2026,14 @@ __global__ void __launch_bounds__(NT, 1) cg_smem_cluster_kernel(SmemArgs a) {
     // y_i = sum_k val * g[col], g = the gathered vector, read from its owner CTA
     auto spmv_row = [&](const double *g, int i) {
         double pv[kSlots];
+        const int own = (int)row0 + i;
 #pragma unroll
         for (int k = 0; k < kSlots; ++k) {  // all 27 gathers issued before the FMA chain
-            const int c = scol[k * R + i] - plane32;  // global row of the column (< 2^31)
+            // global row of the column (< 2^31); DIA: from the stencil offset, padding -> own
+            const int c = a.dia ? (sval[k * R + i] != 0.0
+                                       ? own + (k / 9 - 1) * plane32 + ((k / 3) % 3 - 1) * a.nx + (k % 3 - 1)
+                                       : own)
+                                : scol[k * R + i] - plane32;
             const unsigned owner = (unsigned)c / (unsigned)R;
             const int off = c - (int)owner * R;
             pv[k] = *cl.map_shared_rank(g + off, owner);

@@ -146,3 +146,32 @@ def test_dia_fused_peer_path_bitwise(P, dims):
             for o in outs[1:]:
                 assert o[:2] == outs[0][:2]
                 np.testing.assert_array_equal(o[2], outs[0][2])
+
+
+@pytest.mark.parametrize("variant", [0, 1])
+def test_dia_on_chip_solve(ctx, variant):
+    """The shared-memory-resident cluster solve under format 1 drops the
+    column slice where the ELL slice does not fit (216 + 40/48 B per row
+    instead of 324 + 40/48): same bits as ELL where both run on chip
+    (20x30x10, which keeps the column slice), and it takes problems the ELL
+    slice does not fit (30x20x20 = 12000 rows: ELL -> while-graph, DIA -> on
+    chip), which match the oracle."""
+    with H.Problem(ctx, 20, 30, 10) as p:
+        outs = []
+        for fmt in (0, 1):
+            outs.append(_solve(p, fmt, 150, 1e-12, variant=variant))
+            assert p.stats()["graph_mode"] == 5
+        assert outs[1][:2] == outs[0][:2]
+        np.testing.assert_array_equal(outs[1][2], outs[0][2])
+    dims = (30, 20, 20)
+    ref = oracle.generate(*dims)
+    oref = (oracle.cg_sr if variant else oracle.cg)(ref, 150, 1e-12)
+    with H.Problem(ctx, *dims) as p:
+        modes = []
+        for fmt in (0, 1):
+            it, nr, x = _solve(p, fmt, 150, 1e-12, variant=variant)
+            modes.append(p.stats()["graph_mode"])
+            assert abs(it - oref["niters"]) <= 1
+            assert abs(nr - oref["normr"]) <= 1e-10
+            assert np.max(np.abs(x - oref["x"])) <= 1e-10
+        assert modes == [2, 5]
