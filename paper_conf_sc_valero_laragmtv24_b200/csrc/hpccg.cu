@@ -1408,11 +1408,23 @@ int launch_persistent(hpccg_problem *p, int max_iter, double tol) {
             cfg.attrs = at;
             cfg.numAttrs = 1;
             if (nt == 512) {
-                if (sr) CU(cudaLaunchKernelEx(&cfg, cg_smem_cluster_kernel<512, true>, m));
-                else CU(cudaLaunchKernelEx(&cfg, cg_smem_cluster_kernel<512, false>, m));
+                if (m.dia) {
+                    if (sr) CU(cudaLaunchKernelEx(&cfg, cg_smem_cluster_kernel<512, true, true>, m));
+                    else CU(cudaLaunchKernelEx(&cfg, cg_smem_cluster_kernel<512, false, true>, m));
+                } else if (sr) {
+                    CU(cudaLaunchKernelEx(&cfg, cg_smem_cluster_kernel<512, true>, m));
+                } else {
+                    CU(cudaLaunchKernelEx(&cfg, cg_smem_cluster_kernel<512, false>, m));
+                }
             } else {
-                if (sr) CU(cudaLaunchKernelEx(&cfg, cg_smem_cluster_kernel<kBlock, true>, m));
-                else CU(cudaLaunchKernelEx(&cfg, cg_smem_cluster_kernel<kBlock, false>, m));
+                if (m.dia) {
+                    if (sr) CU(cudaLaunchKernelEx(&cfg, cg_smem_cluster_kernel<kBlock, true, true>, m));
+                    else CU(cudaLaunchKernelEx(&cfg, cg_smem_cluster_kernel<kBlock, false, true>, m));
+                } else if (sr) {
+                    CU(cudaLaunchKernelEx(&cfg, cg_smem_cluster_kernel<kBlock, true>, m));
+                } else {
+                    CU(cudaLaunchKernelEx(&cfg, cg_smem_cluster_kernel<kBlock, false>, m));
+                }
             }
             p->last_persist_mode = 5;
             return check_launch(ctx);
@@ -1602,7 +1614,11 @@ int ctx_common_init(hpccg_ctx *c, int device, void *stream) {
         for (const void *k : {(const void *)cg_smem_cluster_kernel<kBlock, false>,
                               (const void *)cg_smem_cluster_kernel<kBlock, true>,
                               (const void *)cg_smem_cluster_kernel<512, false>,
-                              (const void *)cg_smem_cluster_kernel<512, true>})
+                              (const void *)cg_smem_cluster_kernel<512, true>,
+                              (const void *)cg_smem_cluster_kernel<kBlock, false, true>,
+                              (const void *)cg_smem_cluster_kernel<kBlock, true, true>,
+                              (const void *)cg_smem_cluster_kernel<512, false, true>,
+                              (const void *)cg_smem_cluster_kernel<512, true, true>})
             attr_ok = attr_ok &&
                       cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                            (int)c->smem_bytes) == cudaSuccess &&

@@ -1905,7 +1905,7 @@ __global__ void __launch_bounds__(kBlock, 1) cg_persistent_kernel(PersistArgs a)
 struct SmemArgs {
     int64_t n, stride, plane;
     int R;  // rows per CTA
-    int nx, dia;  // dia: DIA-27 reading (HPCCG_OPT_SPMV_FORMAT 1) -- no column slice in smem
+    int nx, dia;  // dia: DIA-27 reading (HPCCG_OPT_SPMV_FORMAT 1) -- no column slice in smem (kDia)
     const double *val;
     const int *col;
     const double *b;
@@ -1985,7 +1985,7 @@ __device__ __forceinline__ double2 cluster_sum2(double *mine, double u, double v
 //   kSR = false: HPCCG's CG (A4, A11), 3 cluster barriers per iteration;
 //   kSR = true:  the single-reduction CG of f2 (oracle_cg_sr), 2 per iteration.
 // Per-row FMA chain as A8.
-template <int NT, bool kSR>
+template <int NT, bool kSR, bool kDia = false>
 __global__ void __launch_bounds__(NT, 1) cg_smem_cluster_kernel(SmemArgs a) {
     namespace cgx = cooperative_groups;
     auto cl = cgx::this_cluster();
@@ -2010,13 +2010,13 @@ __global__ void __launch_bounds__(NT, 1) cg_smem_cluster_kernel(SmemArgs a) {
 #pragma unroll
         for (int k = 0; k < kSlots; ++k) {
             v[k] = __ldcs(a.val + k * a.stride + row0 + i);
-            cidx[k] = a.dia ? 0 : __ldcs(a.col + k * a.stride + row0 + i);
+            cidx[k] = kDia ? 0 : __ldcs(a.col + k * a.stride + row0 + i);
         }
         const double bv = a.b[row0 + i], xv = a.x[row0 + i];
 #pragma unroll
         for (int k = 0; k < kSlots; ++k) {
             sval[k * R + i] = v[k];
-            if (!a.dia) scol[k * R + i] = cidx[k];
+            if (!kDia) scol[k * R + i] = cidx[k];
         }
         sb[i] = bv;
         sx[i] = xv;
@@ -2030,7 +2030,7 @@ __global__ void __launch_bounds__(NT, 1) cg_smem_cluster_kernel(SmemArgs a) {
 #pragma unroll
         for (int k = 0; k < kSlots; ++k) {  // all 27 gathers issued before the FMA chain
             // global row of the column (< 2^31); DIA: from the stencil offset, padding -> own
-            const int c = a.dia ? (sval[k * R + i] != 0.0
+            const int c = kDia ? (sval[k * R + i] != 0.0
                                        ? own + (k / 9 - 1) * plane32 + ((k / 3) % 3 - 1) * a.nx + (k % 3 - 1)
                                        : own)
                                 : scol[k * R + i] - plane32;
