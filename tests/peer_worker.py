@@ -30,3 +30,19 @@ def run(rank, nranks, dims, variant, max_iter, tol, to_parent, from_parent, halo
             to_parent.put(("done", rank, out))
     except Exception as e:  # reported to the parent, which fails the test
         to_parent.put(("error", rank, repr(e)))
+
+
+def run_maxabs(rank, nranks, dims, x_slab, xe_slab, to_parent, from_parent):
+    """a.9 across processes: set this rank's X (and X_EXACT) slab, then the
+    collective max|x - x_exact| (local kernel + peer MAX allreduce)."""
+    try:
+        from paper_conf_sc_valero_laragmtv24_b200 import hpccg as H
+        with H.Context(0, rank=rank, nranks=nranks, peer=True) as c, H.Problem(c, *dims) as p:
+            to_parent.put(("blob", rank, p.peer_export()))
+            p.peer_attach(from_parent.get(timeout=120))
+            p.set_vec(H.HPCCG_VEC_X, x_slab)
+            if xe_slab is not None:
+                p.set_vec(H.HPCCG_VEC_XEXACT, xe_slab)
+            to_parent.put(("done", rank, p.maxabsdiff()))
+    except Exception as e:
+        to_parent.put(("error", rank, repr(e)))

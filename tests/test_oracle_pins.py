@@ -428,3 +428,76 @@ def test_2d_leading_dimension_semantics():
     ex = sum(Fraction(a) * Fraction(b) for a, b in zip(X[:m, :].ravel(), Y[:m, :].ravel()))
     got = oracle.ddot2d(m, n, ld, x, y)
     assert abs(Fraction(got) - ex) <= abs(ex) * Fraction(2.0 ** -52)
+
+
+# ------------------------------------------------------------- a.9 verify
+
+def _maxabsdiff_exact(x, xe):
+    """Independent definition: for each i the EXACT difference as a rational,
+    rounded once to the nearest double (= what one IEEE subtraction returns),
+    then the largest magnitude; entries whose difference is NaN are skipped
+    (HPCCG's `if (diff > max)` never takes a NaN, reading A26)."""
+    best = Fraction(0)
+    for a, b in zip(x.tolist(), xe.tolist()):
+        if math.isnan(a) or math.isnan(b):
+            continue
+        d = abs(Fraction(float(np.float64(a))) - Fraction(float(np.float64(b))))
+        d = Fraction(float(d))                      # one correctly rounded subtraction
+        best = max(best, d)
+    return float(best)
+
+
+@pytest.mark.parametrize("pos", ["first", "middle", "last"])
+@pytest.mark.parametrize("sign", [1.0, -1.0])
+def test_maxabsdiff_planted_spike_closed_form(pos, sign):
+    """a.9 (HPCCG compute_residual; BJ:north_star "final max|x-1|"): x = 1 +
+    noise (|noise| < 2^-10) with ONE planted deviation d = sign * 0.75 -- the
+    result is exactly 0.75 (1 +- 0.75 and its difference with 1 are exact).
+    Breaks: a dropped fabs (sign -1), a loop that skips the first / last
+    element, a min instead of a max, a constant return."""
+    n = 4099
+    x = 1.0 + synth.uniform(n, 91, -2.0 ** -10, 2.0 ** -10)
+    j = {"first": 0, "middle": n // 2, "last": n - 1}[pos]
+    x[j] = 1.0 + sign * 0.75
+    xe = np.ones(n)
+    assert oracle.maxabsdiff(x, xe) == 0.75
+    assert oracle.maxabsdiff(x, xe) == np.max(np.abs(x - xe))
+
+
+def test_maxabsdiff_vs_exact_rational_general_xexact():
+    """Arbitrary x and x_exact (not only x_exact = 1): equal to the exact
+    rational definition above, bit for bit; both signs of the largest
+    deviation are exercised by the two seeds."""
+    for seed in (5, 6, 7):
+        x = synth.uniform(1537, seed, -3.0, 3.0)
+        xe = synth.uniform(1537, seed + 100, -3.0, 3.0)
+        assert oracle.maxabsdiff(x, xe) == _maxabsdiff_exact(x, xe)
+
+
+def test_maxabsdiff_zero_signed_zero_and_subnormals():
+    """x == x_exact -> exactly +0 (also with -0 against +0); a single
+    subnormal deviation is returned, not flushed to zero (either sign)."""
+    n = 257
+    xe = np.zeros(n)
+    x = np.zeros(n)
+    x[::2] = -0.0
+    r = oracle.maxabsdiff(x, xe)
+    assert r == 0.0 and not math.copysign(1.0, r) < 0
+    tiny = 5e-324
+    for j, s in ((0, 1.0), (n - 1, -1.0), (100, -1.0)):
+        y = x.copy()
+        y[j] = s * tiny
+        assert oracle.maxabsdiff(y, xe) == tiny
+    ones = np.ones(n)
+    assert oracle.maxabsdiff(ones, ones) == 0.0
+    assert oracle.maxabsdiff(np.ones(0), np.ones(0)) == 0.0
+
+
+def test_maxabsdiff_nan_entries_skipped():
+    """Reading A26: a NaN entry compares false against the running maximum
+    (HPCCG's `if (diff > max)`), so it is skipped; the finite entries still
+    decide the result."""
+    x = np.ones(64)
+    x[3] = np.nan
+    x[40] = 1.5
+    assert oracle.maxabsdiff(x, np.ones(64)) == 0.5 == _maxabsdiff_exact(x, np.ones(64))
