@@ -2,24 +2,36 @@
 """bench.py -- HPCCG CG hot path on B200 (BASELINE.json metric).
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
-                    [--workload hpccg128|hpccg20|hpccg256|hpccg512s]
+                    [--workload hpccg256|hpccg128|hpccg20|hpccg512s|blas1|tridiag|lbm]
 
 One STEP = one whole HPCCG solve on the synthetic on-device-generated problem:
-init (p = x, Ap = A p, r = b - Ap, r.r) + `iters` CG iterations (SpMV with
-fused p.Ap, fused x/r update + r.r, p update; device-side scalars; CUDA-graph
-replay) + the max|x - 1| verification -- rows a.2-a.9 of DESIGN.md.  The
-problem (a.1) is generated once per run (HPCCG times only the solve); its
-time is reported as config.gen_ms.  x is reset to 0 (x0, A5) before every
-step by our waxpby kernel.
+x0 = 0 (our waxpby kernel), init (p = x, Ap = A p, r = b - Ap, r.r), the CG
+iterations (SpMV with fused p.Ap, fused x/r update + r.r, p update; device-side
+scalars; one CUDA graph with a device-driven WHILE node) and the max|x - 1|
+verification -- rows a.2-a.9 of DESIGN.md.  The problem (a.1) is generated once
+per workload (HPCCG times only the solve): config.gen_ms.
+
+Default workload, at EVERY N: hpccg256 = BASELINE configs[2] (256^3 per GPU,
+weak scaling, 200 iterations, tol 0), the configuration north_star's targets
+are set on; so a scaling run's N = 1 point is this line.  Before timing, every
+workload runs a tol 1e-12 correctness solve of the GLOBAL problem and checks
+niters against SURVEY's independent counts (`correctness`).  The same line
+carries `sub_configs`: configs[1] (128^3, 500 iterations), configs[0]
+(20x30x10 at tol 1e-12 / 150, as BASELINE states it) at N = 1, and configs[3]
+(512^3 global, strong) at every N -- each with t_iter, GFLOP/s and e2e.
 
 value = CG GFLOP/s of the whole job = sum over ranks of niters (2 nnz + 10 n)
         / max-over-ranks device time of the K timed steps (exact nnz, A15).
 e2e   = the same metric through the public C-ABI with HOST buffers: every
         step copies x0 from pinned host memory in and the solution x back out.
 roofline = the SpMV kernel (dominant), algorithmic bytes 12 nnz + 16 n per
-        launch / its CUDA-event launch duration inside the timed region.
-Multi-GPU (torchrun): z-slab weak scaling, one rank per GPU, NCCL halo +
-        allreduce inside the library; torch.distributed only bootstraps.
+        launch / its CUDA-event launch duration (events pass); the fused vector
+        kernels (48n, 24n B) against 8 TB/s beside it (north_star's 75 % target).
+Multi-GPU (torchrun): z-slab, one rank per GPU; the halo exchange and the
+        allreduces run inside the library (peer memory fused into the CG kernels
+        by default, NCCL as the agreed fallback); torch.distributed only
+        bootstraps and aggregates.  `ranks` records, per rank, the transport,
+        exchange mode, NCCL's rank count and the correctness solve.
 """
 from __future__ import annotations
 
@@ -37,12 +49,17 @@ sys.path.insert(0, ROOT)
 
 METRIC = "HPCCG CG GFLOP/s and SpMV HBM GB/s (fp64) at 1/2/4/8 B200 vs HBM roofline"
 WORKLOADS = {
-    # name: (nx, ny, nz, CG iterations, BASELINE config index, scaling)
-    # weak: nz planes per GPU; strong: nz global planes split over the GPUs
-    "hpccg128": (128, 128, 128, 500, 1, "weak"),
-    "hpccg20": (20, 30, 10, 149, 0, "weak"),
-    "hpccg256": (256, 256, 256, 200, 2, "weak"),
-    "hpccg512s": (512, 512, 512, 200, 3, "strong"),
+    # weak: nz planes per GPU; strong: nz global planes split over the GPUs.
+    # tol 0 runs exactly max_iter - 1 iterations (HPCCG loop, A4); configs[0]
+    # is quoted at tol 1e-12 / 150 (50 iterations).  sub_steps: timed steps when
+    # the workload is a sub-record of another workload's line.
+    "hpccg256": dict(nx=256, ny=256, nz=256, max_iter=201, tol=0.0, cfg=2, scaling="weak", sub_steps=5,
+                     ref_iters=6),
+    "hpccg128": dict(nx=128, ny=128, nz=128, max_iter=501, tol=0.0, cfg=1, scaling="weak", sub_steps=10,
+                     ref_iters=20),
+    "hpccg20": dict(nx=20, ny=30, nz=10, max_iter=150, tol=1e-12, cfg=0, scaling="weak", sub_steps=20),
+    "hpccg512s": dict(nx=512, ny=512, nz=512, max_iter=101, tol=0.0, cfg=3, scaling="strong", sub_steps=3,
+                      ref_iters=6),
 }
 BLAS1_METRIC = "JACC BLAS-1 AXPY+DOT fp64 HBM GB/s (host-synchronous calls)"
 TRI_METRIC = "Fig. 12 CG time per iteration, tridiagonal SIZE = 1e8 (fp64)"
@@ -192,33 +209,54 @@ def oracle_sample(nx, ny, nz, iters_cap, budget_s, sr=False):
             "cores": oracle.get_threads(), "prob": prob}
 
 
-def run_reference(args, nx, ny, nz, iters, cfg_index):
+def run_reference(args, w):
+    """The reference arm for the CG workloads: the oracle as it stands, on the
+    host cores, in our arm's metric / unit.  A tol > 0 workload (configs[0])
+    runs its whole solve per step; a fixed-iteration one a bounded number of
+    its iterations per step (the same problem, `sample` says how many)."""
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return 0
     import oracle
     oracle.build()
+    nx, ny, nz = w["nx"], w["ny"], w["nz"]
+    if w["scaling"] == "strong":
+        nz = nz // args.gpus
+    if nx * ny * nz > (1 << 25):          # host RAM of the oracle's CSR: time the 256^3 problem
+        nx, ny, nz = 256, 256, 256
     prob = oracle.generate(nx, ny, nz)
-    m = max(1, min(iters, args.ref_iters))
     sr = args.cg_variant == "sr"
+    if w["tol"] > 0:
+        max_iter, tol = w["max_iter"], w["tol"]
+        what = f"the whole solve (tol {tol:g}, max_iter {max_iter}) per step"
+    else:
+        m = max(1, min(w["max_iter"] - 1, args.ref_iters or w.get("ref_iters", 20)))
+        max_iter, tol = m + 1, 0.0
+        what = f"{m} iterations per step (bounded sample of the {w['max_iter'] - 1}-iteration step)"
+
+    def one():
+        t0 = time.perf_counter()
+        r = oracle.cg_sr(prob, max_iter, tol) if sr else oracle.cg(prob, max_iter, tol)
+        return r, time.perf_counter() - t0
+
     for _ in range(args.warmup):
-        oracle_cg_timed(prob, m + 1, sr)
+        one()
     tot, flops = 0.0, 0.0
     for _ in range(args.steps):
-        r, t = oracle_cg_timed(prob, m + 1, sr)
+        r, t = one()
         tot += t
         flops += cg_flops(r["niters"], prob.nnz, prob.n)
     val = flops / tot * 1e-9
-    sample = (f"oracle CG on the {nx}x{ny}x{nz} problem, {m} iterations per step "
-              f"(bounded sample of the {iters}-iteration workload), OpenMP all host cores")
+    sample = (f"oracle CG (C, OpenMP, all host cores) on the {nx}x{ny}x{nz} problem, {what}"
+              + ("; one GPU's slab of the global problem" if args.gpus > 1 else ""))
     line = {
         "metric": METRIC, "value": round(val, 4), "unit": "GFLOP/s", "impl": "reference",
         "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
         "ms_per_step": round(tot / args.steps * 1e3, 3), "higher_is_better": True,
-        "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+        "scaling": w["scaling"], "vs_baseline": None, "dtype": "f64",
         "data": "synthetic (HPCCG generation, deterministic)",
-        "config": {"workload": args.workload, "baseline_config": cfg_index, "nx": nx, "ny": ny,
-                   "nz": nz, "iters_per_step": m},
+        "config": {"workload": args.workload, "baseline_config": w["cfg"], "nx": nx, "ny": ny,
+                   "nz": nz, "iters_per_step": r["niters"], "tol": tol},
         "cpu_baseline": {"value": round(val, 4), "unit": "GFLOP/s", "cores": oracle.get_threads(),
                          "kind": "oracle", "sample": sample},
         "e2e": {"value": round(val, 4), "unit": "GFLOP/s", "h2d_bytes_per_step": 0,
@@ -331,8 +369,237 @@ def run_reference_blas1(args):
 
 # -------------------------------------------------------------------- ours
 
-def run_ours(args, nx, ny, nz, iters, cfg_index, scaling):
+# tol = 1e-12 / max_iter 150 iteration counts of the GLOBAL problem (SURVEY 8(c)
+# pins: two independent numpy implementations, HPCCG loop semantics A4),
+# keyed by (nx, ny, nz_global): the N-rank correctness solve is checked against them
+EXPECTED_NITERS = {(20, 30, 10): 50, (32, 32, 32): 60, (64, 64, 64): 89, (128, 128, 128): 106,
+                   (256, 256, 256): 112, (256, 256, 512): 113, (256, 256, 1024): 114,
+                   (256, 256, 2048): 115, (512, 512, 512): 115}
+
+
+def _stats_add(acc, prob, r):
+    st = prob.stats()
+    acc["spmv_ms"] += st["spmv_ms"]
+    acc["spmv_n"] += st["spmv_launches"]
+    acc["update_ms"] += st["update_ms"]
+    acc["pupdate_ms"] += st["pupdate_ms"]
+    acc["niters"] += r["niters"]
+    acc["graph_mode"] = st["graph_mode"]
+
+
+class CgRunner:
+    """One generated problem and the bench's timing protocol around it: a step
+    is x0 = 0 (our waxpby kernel), one hpccg_solve(max_iter, tol), max|x - 1|.
+    Times are CUDA events on the library stream, max over ranks; L2 is flushed
+    between timed steps (outside the events) when the working set fits in L2."""
+
+    def __init__(self, H, D, ctx, prob, stream, world, coll_dev, max_iter, tol, local):
+        import torch
+        self.H, self.D, self.ctx, self.prob, self.stream = H, D, ctx, prob, stream
+        self.world, self.coll_dev, self.max_iter, self.tol = world, coll_dev, max_iter, tol
+        self.n = prob.n
+        self.nnz_local = prob.info["nnz_local"]
+        self.xptr = prob.vec_ptr(H.HPCCG_VEC_X)
+        l2_bytes = torch.cuda.get_device_properties(local).L2_cache_size
+        work_bytes = (324 + 6 * 8) * self.n
+        self.flush_buf = None
+        if work_bytes < l2_bytes:
+            self.flush_buf = torch.empty(2 * l2_bytes // 8, dtype=torch.float64, device="cuda")
+        self.l2_note = ("L2 flushed between timed steps (a %d MB write; working set %.1f MB < L2 %.0f MB); "
+                        "per-step events" % (2 * l2_bytes >> 20, work_bytes / 1e6, l2_bytes / 1e6)
+                        if self.flush_buf is not None else
+                        "inputs larger than L2 (ELL %.0f MB/GPU > %.0f MB)" % (324e-6 * self.n, l2_bytes / 1e6))
+
+    def flush(self):
+        import torch
+        with torch.cuda.stream(self.stream):
+            self.flush_buf.zero_()
+
+    def barrier(self):
+        import torch
+        import torch.distributed as dist
+        if self.world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    def step(self):
+        self.ctx.waxpby(self.n, 0.0, self.xptr, 0.0, self.xptr, self.xptr)   # x0 = 0 (A5)
+        r = self.prob.solve(self.max_iter, self.tol)
+        return r, self.prob.maxabsdiff()
+
+    def timed(self, k_steps, step=None):
+        """K steps between barriers; one event pair around all of them (inputs
+        larger than L2) or around each step (L2 flushed outside the events)."""
+        import torch
+        step = step or self.step
+        t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        acc = {"spmv_ms": 0.0, "spmv_n": 0, "niters": 0, "update_ms": 0.0, "pupdate_ms": 0.0, "ms": 0.0}
+        self.barrier()
+        if self.flush_buf is not None:
+            for _ in range(k_steps):
+                self.flush()
+                t0.record(self.stream)
+                r, err = step()
+                t1.record(self.stream)
+                t1.synchronize()
+                acc["ms"] += t0.elapsed_time(t1)
+                _stats_add(acc, self.prob, r)
+            self.barrier()
+        else:
+            t0.record(self.stream)
+            for _ in range(k_steps):
+                r, err = step()
+                _stats_add(acc, self.prob, r)
+            t1.record(self.stream)
+            self.barrier()
+            acc["ms"] = t0.elapsed_time(t1)
+        acc["r"], acc["err"] = r, err
+        return acc
+
+    def value(self, acc):
+        """(whole-job GFLOP/s, max-over-ranks ms) of a timed region."""
+        ms, flops = self.D.max_time_sum_work(acc["ms"], cg_flops(acc["niters"], self.nnz_local, self.n),
+                                             self.coll_dev)
+        return flops / (ms * 1e-3) * 1e-9, ms
+
+    def e2e(self, k_steps):
+        """The same metric through the public C-ABI with HOST buffers: every
+        step copies x0 in from pinned memory and x back out (+ max|x-1|)."""
+        import numpy as np
+        import torch
+        H, prob = self.H, self.prob
+        h_x0 = torch.zeros(self.n, dtype=torch.float64).pin_memory()
+        h_x = torch.empty(self.n, dtype=torch.float64).pin_memory()
+
+        def step_e2e():
+            prob.set_vec_ptr(H.HPCCG_VEC_X, h_x0.data_ptr())   # H2D 8n
+            r = prob.solve(self.max_iter, self.tol)
+            prob.get_vec_ptr(H.HPCCG_VEC_X, h_x.data_ptr())    # D2H 8n
+            return r, prob.maxabsdiff()                         # D2H 8 B
+
+        step_e2e()
+        acc = self.timed(k_steps, step_e2e)
+        val, _ = self.value(acc)
+        return {"value": round(val, 3), "unit": "GFLOP/s", "h2d_bytes_per_step": 8 * self.n,
+                "d2h_bytes_per_step": 8 * self.n + 8,
+                "max_abs_x_minus_1_host": float(np.max(np.abs(h_x.numpy() - 1.0)))}
+
+    def correctness(self, nx, ny, nz_global):
+        """tol 1e-12 / max_iter 150 solve of the global problem before any timing:
+        niters against SURVEY's independent counts, max|x-1| < 1e-13 (every rank
+        reports the same values: the loop decisions come from the allreduces)."""
+        self.ctx.waxpby(self.n, 0.0, self.xptr, 0.0, self.xptr, self.xptr)
+        r = self.prob.solve(150, 1e-12)
+        err = self.prob.maxabsdiff()
+        want = EXPECTED_NITERS.get((nx, ny, nz_global))
+        ok = err < 1e-13 and r["normr"] <= 1e-12 and (want is None or abs(r["niters"] - want) <= 1)
+        return {"tol": 1e-12, "max_iter": 150, "niters": r["niters"], "expected_niters": want,
+                "normr": r["normr"], "max_abs_x_minus_1": err, "ok": bool(ok),
+                "expected_from": "SURVEY 8(c) pins (independent numpy CG), niters +-1"}
+
+
+def measure_workload(H, D, ctx, stream, world, rank, local, coll_dev, name, steps, warmup,
+                     events=False, trace=False, clocks=False, opts=(), setup=None):
+    """Generate `name`'s problem, self-check it, time it; a dict of results."""
     import numpy as np
+    import torch
+    w = WORKLOADS[name]
+    slab = D.slab_for(w["nx"], w["ny"], w["nz"], rank, world, w["scaling"])
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    prob = H.Problem(ctx, slab.nx, slab.ny, slab.nz)
+    e1.record(stream)
+    torch.cuda.synchronize()
+    gen_ms = e0.elapsed_time(e1)
+    prob.set_option(H.HPCCG_OPT_GRAPH, 1)
+    for k, v in opts:
+        prob.set_option(k, v)
+    out = {"workload": name, "baseline_config": w["cfg"], "nx": slab.nx, "ny": slab.ny,
+           "nz_per_gpu": slab.nz, "global_rows": prob.n * world, "global_nnz": prob.info["nnz_global"],
+           "scaling": w["scaling"], "gen_ms": round(gen_ms, 3)}
+    if setup is not None:
+        out.update(setup(prob))
+    max_iter = w["max_iter"]
+    tol = w["tol"]
+    run = CgRunner(H, D, ctx, prob, stream, world, coll_dev, max_iter, tol, local)
+    out["tol"], out["max_iter"] = tol, max_iter
+    out["correctness"] = run.correctness(slab.nx, slab.ny, slab.nz_global)
+    for _ in range(warmup):
+        run.step()
+    l0 = ctx.launch_count
+    clk = ClockSampler(local) if clocks else None
+    if clk:
+        clk.__enter__()
+    main = run.timed(steps)
+    out["gpu_launches"] = ctx.launch_count - l0
+    ev = tr = None
+    if events:
+        # the same K steps with CUDA events around every phase (plain launches)
+        prob.set_option(H.HPCCG_OPT_TIMING, 1)
+        run.step()
+        ev = run.timed(steps)
+        prob.set_option(H.HPCCG_OPT_TIMING, 0)
+    if trace and world == 1 and main.get("graph_mode") == 2:
+        # one step of the product configuration with the device-side trace
+        # (%globaltimer, first-block start -> last-block end of each CG kernel)
+        k_tr = min(main["niters"] // max(steps, 1), 200)
+        prob.set_option(H.HPCCG_OPT_TRACE, k_tr)
+        run.step()
+        t = prob.trace(k_tr).astype("float64")[5:]
+        prob.set_option(H.HPCCG_OPT_TRACE, 0)
+        if len(t):
+            dur = np.median((t[:, :, 1] - t[:, :, 0]) / 1e3, axis=0)   # us
+            period = float(np.median(np.diff(t[:, 0, 0])) / 1e3) if len(t) > 1 else None
+            tr = {"period_us": round(period, 2) if period else None,
+                  "pupdate_us": round(float(dur[0]), 2), "spmv_us": round(float(dur[1]), 2),
+                  "update_us": round(float(dur[2]), 2)}
+    if clk:
+        clk.__exit__(None, None, None)
+        out["clocks"] = clk.summary()
+    val, ms_max = run.value(main)
+    out.update({"value": round(val, 3), "unit": "GFLOP/s", "steps": steps, "warmup": warmup,
+                "ms_per_step": round(ms_max / steps, 4),
+                "t_iter_us": round(ms_max * 1e3 / max(main["niters"], 1), 3),
+                "niters_per_step": main["niters"] // steps,
+                "max_abs_x_minus_1": main["err"], "normr": main["r"]["normr"],
+                "solve_graph": {5: "on-chip cluster kernel", 4: "one-cluster persistent kernel",
+                                3: "cooperative persistent kernel", 2: "while-graph",
+                                1: "per-iteration graph", 0: "plain"}.get(main.get("graph_mode"), "?"),
+                "l2": run.l2_note})
+    out["e2e"] = run.e2e(steps)
+    out["_ev"], out["_trace"], out["_n"], out["_nnz_local"] = ev, tr, prob.n, run.nnz_local
+    out["_prob"] = prob
+    return out
+
+
+def read_peak_gbs(ctx, stream, nbytes=4 << 30, reps=6):
+    """Live pure-read ceiling: our dot kernel (2 reads, no writes) over two
+    nbytes vectors, best of `reps` event-timed calls -- the SpMV reads 97 % of
+    its bytes, so this is its ceiling; the contract's `peak` (a copy) stays."""
+    import torch
+    n = nbytes // 8
+    x = torch.ones(n, dtype=torch.float64, device="cuda")
+    y = torch.ones(n, dtype=torch.float64, device="cuda")
+    torch.cuda.synchronize()
+    t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    best = None
+    for _ in range(reps + 2):
+        t0.record(stream)
+        ctx.ddot(n, x.data_ptr(), y.data_ptr())
+        t1.record(stream)
+        t1.synchronize()
+        ms = t0.elapsed_time(t1)
+        best = ms if best is None else min(best, ms)
+    del x, y
+    torch.cuda.empty_cache()
+    return 16.0 * n / (best * 1e-3) * 1e-9
+
+
+def _strip(d):
+    return {k: v for k, v in d.items() if not k.startswith("_")}
+
+
+def run_ours(args):
     import torch
     import torch.distributed as dist
 
@@ -356,10 +623,12 @@ def run_ours(args, nx, ny, nz, iters, cfg_index, scaling):
     transport = "peer" if share else args.transport
     if world > 1 and transport == "peer" and args.halo == "nccl":
         raise SystemExit("--transport peer has no NCCL halo (use --halo fused or peer)")
+    if world > 1 and transport == "nccl" and "NCCL_DEBUG" not in os.environ:
+        # keep NCCL's communicator-init lines (nRanks per comm) on stderr, off stdout
+        os.environ.update({"NCCL_DEBUG": "INFO", "NCCL_DEBUG_SUBSYS": "INIT",
+                           "NCCL_DEBUG_FILE": "/dev/stderr"})
     coll_dev = "cpu" if share else "cuda"
     torch.cuda.set_device(local)
-    slab = D.slab_for(nx, ny, nz, rank, world, scaling)
-    nz = slab.nz
     uid = None
     if world > 1:
         if share:
@@ -372,307 +641,188 @@ def run_ours(args, nx, ny, nz, iters, cfg_index, scaling):
     stream = torch.cuda.Stream()
     ctx = H.Context(local, stream=stream.cuda_stream, rank=rank, nranks=world, unique_id=uid,
                     peer=(world > 1 and transport == "peer"))
-    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    e0.record(stream)
-    prob = H.Problem(ctx, nx, ny, nz)
-    e1.record(stream)
-    torch.cuda.synchronize()
-    gen_ms = e0.elapsed_time(e1)
-    n, nnz_local = prob.n, prob.info["nnz_local"]
-    nnz_global = prob.info["nnz_global"]
-    prob.set_option(H.HPCCG_OPT_GRAPH, 1)
     sr = args.cg_variant == "sr"
-    prob.set_option(H.HPCCG_OPT_CG_VARIANT, 1 if sr else 0)
     dia = args.spmv_format == "dia"
-    prob.set_option(H.HPCCG_OPT_SPMV_FORMAT, 1 if dia else 0)
-    halo = "none (1 slab)"
-    if world > 1 and transport == "peer":
-        # peer-only context: no NCCL anywhere; every rank maps its neighbours' buffers
-        # from the exported CUDA-IPC blobs (gathered over torch.distributed)
-        prob.peer_attach(D.allgather_peer_blobs(prob.peer_export()))
-        mode = 1 if args.halo == "peer" else 2
-        prob.set_option(H.HPCCG_OPT_HALO_PEER, mode)
-        halo = ("peer memory fused into the CG kernels (HALO_PEER 2, while-graph), peer-only context"
-                if mode == 2 else
-                "peer-memory push + post/collect allreduce kernels (while-graph), peer-only context")
-    elif world > 1:
-        halo = "NCCL send/recv + ncclAllReduce"
-        if args.halo in ("peer", "fused", "auto"):
-            # collective: every rank maps its neighbours' buffers (CUDA IPC over NVLink);
-            # auto = fused (the exchange and the allreduce(s) inside the CG kernels,
-            # either CG variant); peer = the separate peer kernels; auto falls back to
-            # NCCL if the mapping is refused
-            mode = 1 if args.halo == "peer" else 2
-            err = None
-            try:
-                prob.set_option(H.HPCCG_OPT_HALO_PEER, mode)
-                # a short collective solve proves the peer mapping end to end (a wait
-                # that times out returns an error instead of hanging)
-                prob.solve(4, 0.0)
-            except H.HpccgError as e:
-                err = str(e)
-            ok = torch.tensor([0.0 if err else 1.0], device=torch.device("cuda", local))
-            dist.all_reduce(ok, op=dist.ReduceOp.MIN)   # every rank takes the same path
-            if ok.item() == 1.0:
-                halo = ("peer memory fused into the CG kernels (HALO_PEER 2, while-graph)" if mode == 2
-                        else "peer-memory push + post/collect allreduce kernels (while-graph)")
-            else:
-                if args.halo != "auto":
-                    raise RuntimeError("peer-memory path failed: %s" % err)
-                prob.set_option(H.HPCCG_OPT_HALO_PEER, 0)
-                halo = "NCCL (peer path failed on some rank: %s)" % err
-    xptr = prob.vec_ptr(H.HPCCG_VEC_X)
-    # working set (ELL 324 B/row + 6 vectors): when it fits in L2, flush L2
-    # between timed steps (outside the timed events) so no step starts warm
-    l2_bytes = torch.cuda.get_device_properties(local).L2_cache_size
-    work_bytes = (324 + 6 * 8) * n
-    flush_buf = None
-    if work_bytes < l2_bytes:
-        flush_buf = torch.empty(2 * l2_bytes // 8, dtype=torch.float64, device="cuda")
-    l2_note = ("L2 flushed between timed steps (a %d MB write; working set %.1f MB < L2 %.0f MB); "
-               "per-step events" % (2 * l2_bytes >> 20, work_bytes / 1e6, l2_bytes / 1e6)
-               if flush_buf is not None else
-               "inputs larger than L2 (ELL %.0f MB/GPU > %.0f MB)" % (324e-6 * n, l2_bytes / 1e6))
+    opts = [(H.HPCCG_OPT_CG_VARIANT, 1 if sr else 0), (H.HPCCG_OPT_SPMV_FORMAT, 1 if dia else 0)]
+    mode_want = 1 if args.halo == "peer" else 2
 
-    def flush():
-        with torch.cuda.stream(stream):
-            flush_buf.zero_()
+    def setup_multirank(prob):
+        """The exchange path every rank agrees on (recorded per rank)."""
+        if world == 1:
+            return {"halo": "none (1 slab)"}
+        if transport == "peer":
+            # peer-only context: no NCCL anywhere; every rank maps its neighbours'
+            # buffers from the exported CUDA-IPC blobs (gathered over torch.distributed)
+            prob.peer_attach(D.allgather_peer_blobs(prob.peer_export()))
+            prob.set_option(H.HPCCG_OPT_HALO_PEER, mode_want)
+            return {"halo": ("peer memory fused into the CG kernels (HALO_PEER 2, while-graph), "
+                             "peer-only context" if mode_want == 2 else
+                             "peer-memory push + post/collect allreduce kernels (while-graph), "
+                             "peer-only context"), "halo_mode": mode_want, "fallback": None}
+        if args.halo == "nccl":
+            return {"halo": "NCCL send/recv + ncclAllReduce", "halo_mode": 0, "fallback": None}
+        # NCCL context: every rank maps its neighbours' buffers (CUDA IPC over NVLink),
+        # then a short collective solve proves the mapping end to end; every rank takes
+        # the same path (auto falls back to NCCL if any rank fails either stage)
+        dec = D.decide_peer_path(
+            try_map=lambda: prob.set_option(H.HPCCG_OPT_HALO_PEER, mode_want),
+            try_proof=lambda: prob.solve(4, 0.0),
+            reset=lambda: prob.set_option(H.HPCCG_OPT_HALO_PEER, 0))
+        if not dec["peer"]:
+            if args.halo != "auto":
+                raise RuntimeError("peer-memory path failed: %s" % dec)
+            return {"halo": "NCCL send/recv + ncclAllReduce (peer path refused: %s)" % dec["why"],
+                    "halo_mode": 0, "fallback": dec}
+        return {"halo": ("peer memory fused into the CG kernels (HALO_PEER 2, while-graph)" if mode_want == 2
+                         else "peer-memory push + post/collect allreduce kernels (while-graph)"),
+                "halo_mode": mode_want, "fallback": None}
 
-    def barrier():
-        if world > 1:
-            dist.barrier()
-        torch.cuda.synchronize()
+    main = measure_workload(H, D, ctx, stream, world, rank, local, coll_dev, args.workload,
+                            args.steps, args.warmup, events=True, trace=not sr, clocks=True,
+                            opts=opts, setup=setup_multirank)
+    n, nnz_local = main["_n"], main["_nnz_local"]
+    ev, trace = main["_ev"], main["_trace"]
+    # per-rank record of what actually ran (transport, exchange mode, NCCL view)
+    cinfo = ctx.info()
+    me = {"rank": rank, "local_rank": local, "device": torch.cuda.get_device_name(local),
+          "pci_bus": torch.cuda.get_device_properties(local).pci_bus_id
+          if hasattr(torch.cuda.get_device_properties(local), "pci_bus_id") else None,
+          "transport": transport if world > 1 else None, "halo_mode": main.get("halo_mode", 0),
+          "lib_nranks": cinfo["nranks"], "lib_rank": cinfo["rank"],
+          "correct": main["correctness"]["ok"], "niters_tol": main["correctness"]["niters"]}
+    ranks = [me]
+    if world > 1:
+        ranks = [None] * world
+        dist.all_gather_object(ranks, me)
+    main["_prob"].free()
 
-    def step():
-        ctx.waxpby(n, 0.0, xptr, 0.0, xptr, xptr)        # x0 = 0 (A5)
-        r = prob.solve(iters + 1, 0.0)                     # `iters` iterations (A4)
-        err = prob.maxabsdiff()
-        return r, err
-
-    def timed(k_steps):
-        """K steps between barriers; CUDA events on the library stream (one
-        pair per step, L2 flushed outside them, when the problem fits in L2)."""
-        t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        acc = {"spmv_ms": 0.0, "spmv_n": 0, "niters": 0, "update_ms": 0.0, "pupdate_ms": 0.0}
-        barrier()
-        if flush_buf is not None:
-            ms = 0.0
-            for _ in range(k_steps):
-                flush()
-                t0.record(stream)
-                r, err = step()
-                t1.record(stream)
-                t1.synchronize()
-                ms += t0.elapsed_time(t1)
-                st = prob.stats()
-                acc["spmv_ms"] += st["spmv_ms"]
-                acc["spmv_n"] += st["spmv_launches"]
-                acc["update_ms"] += st["update_ms"]
-                acc["pupdate_ms"] += st["pupdate_ms"]
-                acc["niters"] += r["niters"]
-                acc["graph_mode"] = st["graph_mode"]
-            barrier()
-            acc["ms"], acc["r"], acc["err"] = ms, r, err
-            return acc
-        t0.record(stream)
-        for _ in range(k_steps):
-            r, err = step()
-            st = prob.stats()
-            acc["spmv_ms"] += st["spmv_ms"]
-            acc["spmv_n"] += st["spmv_launches"]
-            acc["update_ms"] += st["update_ms"]
-            acc["pupdate_ms"] += st["pupdate_ms"]
-            acc["niters"] += r["niters"]
-            acc["graph_mode"] = st["graph_mode"]
-        t1.record(stream)
-        barrier()
-        acc["ms"] = t0.elapsed_time(t1)
-        acc["r"], acc["err"] = r, err
-        return acc
-
-    for _ in range(args.warmup):
-        step()
-    l0 = ctx.launch_count
-    with ClockSampler(local) as clk:
-        # (1) the product configuration: whole solve = one graph with a
-        #     device-driven while node; this region gives `value`
-        main = timed(args.steps)
-        launches = ctx.launch_count - l0
-        # (2) the same K steps with CUDA events around every phase (plain
-        #     launches): the SpMV roofline and the phase split come from here
-        prob.set_option(H.HPCCG_OPT_TIMING, 1)
-        step()
-        ev = timed(args.steps)
-        prob.set_option(H.HPCCG_OPT_TIMING, 0)
-        # (3) one step of the product configuration with the device-side
-        #     trace (%globaltimer, first-block start -> last-block end of each
-        #     CG kernel inside the while-graph): per-kernel times with no events
-        trace = None
-        if world == 1 and not sr and main.get("graph_mode") == 2:
-            k_tr = min(iters, 200)
-            prob.set_option(H.HPCCG_OPT_TRACE, k_tr)
-            step()
-            tr = prob.trace(k_tr).astype("float64")[5:]
-            prob.set_option(H.HPCCG_OPT_TRACE, 0)
-            if len(tr):
-                dur = np.median((tr[:, :, 1] - tr[:, :, 0]) / 1e3, axis=0)   # us
-                period = float(np.median(np.diff(tr[:, 0, 0])) / 1e3) if len(tr) > 1 else None
-                trace = {"period_us": round(period, 2) if period else None,
-                         "pupdate_us": round(float(dur[0]), 2), "spmv_us": round(float(dur[1]), 2),
-                         "update_us": round(float(dur[2]), 2)}
-        # (4) the other SpMV reading of the same matrix (ELL-27 <-> DIA-27,
-        #     HPCCG_OPT_SPMV_FORMAT), same K steps in the product configuration:
-        #     reported beside the line, never as `value`
-        prob.set_option(H.HPCCG_OPT_SPMV_FORMAT, 0 if dia else 1)
-        step()
-        alt = timed(args.steps)
-        prob.set_option(H.HPCCG_OPT_SPMV_FORMAT, 1 if dia else 0)
-    ms = main["ms"]
-    niters_tot = main["niters"]
-    r, err = main["r"], main["err"]
-    spmv_ms, spmv_n = ev["spmv_ms"], ev["spmv_n"]
-    ms_max, flops = D.max_time_sum_work(ms, cg_flops(niters_tot, nnz_local, n), coll_dev)
-    value = flops / (ms_max * 1e-3) * 1e-9
-    alt_ms, alt_flops = D.max_time_sum_work(alt["ms"], cg_flops(alt["niters"], nnz_local, n), coll_dev)
-    alt_line = {"spmv_format": "ELL-27" if dia else "DIA-27 (HPCCG_OPT_SPMV_FORMAT 1)",
-                "value": round(alt_flops / (alt_ms * 1e-3) * 1e-9, 3), "unit": "GFLOP/s",
-                "t_iter_us": round(alt_ms * 1e3 / max(alt["niters"], 1), 3),
-                "same_normr_bits": alt["r"]["normr"] == r["normr"] and alt["niters"] == niters_tot,
-                "how": "the same K steps, same timing rules, the other reading of the same "
-                       "slot-major matrix (bench.py region 4); not the headline" +
-                       ("; this size runs the persistent / on-chip solve, which reads col[] in "
-                        "both readings" if main.get("graph_mode") in (3, 4, 5) else "")}
-
-    # ---- e2e: public API with host buffers (pinned) each step
-    h_x0 = torch.zeros(n, dtype=torch.float64).pin_memory()
-    h_x = torch.empty(n, dtype=torch.float64).pin_memory()
-
-    def step_e2e():
-        prob.set_vec_ptr(H.HPCCG_VEC_X, h_x0.data_ptr())   # H2D 8n
-        r = prob.solve(iters + 1, 0.0)
-        prob.get_vec_ptr(H.HPCCG_VEC_X, h_x.data_ptr())    # D2H 8n
-        err = prob.maxabsdiff()                             # D2H 8 B
-        return r, err
-
-    step_e2e()
-    barrier()
-    t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    ni_e2e, te_local = 0, 0.0
-    if flush_buf is not None:          # same L2 rule as the device-timed region
-        for _ in range(args.steps):
-            flush()
-            t0.record(stream)
-            r_e, _ = step_e2e()
-            t1.record(stream)
-            t1.synchronize()
-            te_local += t0.elapsed_time(t1)
-            ni_e2e += r_e["niters"]
-        barrier()
-    else:
-        t0.record(stream)
-        for _ in range(args.steps):
-            r_e, _ = step_e2e()
-            ni_e2e += r_e["niters"]
-        t1.record(stream)
-        barrier()
-        te_local = t0.elapsed_time(t1)
-    te, fe = D.max_time_sum_work(te_local, cg_flops(ni_e2e, nnz_local, n), coll_dev)
-    e2e_value = fe / (te * 1e-3) * 1e-9
-    x_host_err = float(np.max(np.abs(h_x.numpy() - 1.0)))
+    # sub-records: the other BASELINE configs of the same metric on this job
+    # (1-GPU configs at N = 1; the strong-scaling config at every N)
+    subs = {}
+    if not args.no_sub_configs:
+        names = (["hpccg128", "hpccg20", "hpccg512s"] if world == 1 else ["hpccg512s"])
+        for nm in names:
+            if nm == args.workload:
+                continue
+            k = max(1, min(args.steps, WORKLOADS[nm]["sub_steps"]))
+            sub = measure_workload(H, D, ctx, stream, world, rank, local, coll_dev, nm, k, 3,
+                                   opts=opts, setup=setup_multirank)
+            sub["_prob"].free()
+            subs[nm] = _strip(sub)
+            torch.cuda.empty_cache()
+    peak_read = read_peak_gbs(ctx, stream) if world == 1 else None
 
     if rank == 0:
         peak, peak_src = peaks()
         # ELL-27: 8 B value + 4 B column per stored entry, x read + y written once;
-        # DIA-27 (--spmv-format dia): all 27 value slots (padding included), no columns
+        # DIA-27 (--spmv-format dia, "effective"): all 27 value slots, no columns
         spmv_bytes = (216.0 * n if dia else 12.0 * nnz_local) + 16.0 * n
         roof = None
-        if spmv_n > 0 and spmv_ms > 0:
-            avg_ms = spmv_ms / spmv_n
+        if ev and ev["spmv_n"] > 0 and ev["spmv_ms"] > 0:
+            avg_ms = ev["spmv_ms"] / ev["spmv_n"]
             ach = spmv_bytes / (avg_ms * 1e-3) * 1e-9
             roof = {"bound": "hbm",
                     "kernel": ("spmv27x2_kernel<2> (w = A r with the r.r, w.r epilogue, f2)" if sr else
                                "spmv27x2_kernel<1> (p.Ap epilogue)") +
                               " -- 2 rows/thread; spmv27_kernel if n or the plane is odd" +
-                              ("; DIA-27 reading (columns formed from the stencil offsets, "
-                               "216n + 16n B per launch)" if dia else ""),
+                              ("; DIA-27 reading: EFFECTIVE, a different method (SURVEY 8(d): OUT), "
+                               "216n + 16n B per launch" if dia else ""),
                     "achieved": round(ach, 1),
                     "peak": peak, "unit": "GB/s", "frac": round(ach / peak, 4),
+                    "peak_source": peak_src,
                     "frac_of_8TBs_nominal": round(ach / 8000.0, 4),
                     "traffic": traffic_from_profiles(args.workload + ("_dia" if dia else "")),
                     "algorithmic_bytes_per_launch": spmv_bytes, "avg_launch_us": round(avg_ms * 1e3, 2),
-                    "peak_source": peak_src,
-                    "spmv_share_of_step": round(spmv_ms / ev["ms"], 4) if ev["ms"] > 0 else None,
+                    "spmv_share_of_step": round(ev["spmv_ms"] / ev["ms"], 4) if ev["ms"] > 0 else None,
                     "measured_in": "events pass: the same K steps re-run with a CUDA event pair "
-                                   "around every phase launch (plain launches, bench.py region 2)",
-                    "events_pass_ms_per_step": round(ev["ms"] / args.steps, 4),
-                    "update_avg_us": round(ev["update_ms"] * 1e3 / max(ev["niters"], 1), 2),
-                    "pupdate_avg_us": round(ev["pupdate_ms"] * 1e3 / max(ev["niters"], 1), 2)}
-            # the fused vector kernels against the same peak (north_star: >= 75 % of HBM peak
-            # on "SpMV and fused waxpby/ddot"): x/r update + r.r 48n B, p update 24n B
+                                   "around every phase launch on the library stream (plain launches)",
+                    "events_pass_ms_per_step": round(ev["ms"] / args.steps, 4)}
+            if peak_read:
+                roof["peak_read_GBs"] = round(peak_read, 1)
+                roof["frac_of_read_peak"] = round(ach / peak_read, 4)
+                roof["frac_note"] = ("peak is MEASURED_PEAKS' copy stream (half writes); the SpMV is "
+                                     "97 % reads, so frac > 1 is expected -- frac_of_read_peak divides "
+                                     "by a pure-read stream measured live here (our dot kernel, 2 x 4 GiB, best of 6)")
+            # the fused vector kernels (north_star: >= 75 % of the 8 TB/s HBM peak on
+            # "SpMV and fused waxpby/ddot"): x/r update + r.r 48n B, p update 24n B
+            vec = {}
+            u_bytes, p_bytes = (72.0 * n, None) if sr else (48.0 * n, 24.0 * n)
+            u_us = ev["update_ms"] * 1e3 / max(ev["niters"], 1)
+            p_us = ev["pupdate_ms"] * 1e3 / max(ev["niters"], 1)
+            for nm_k, by, us_ev, us_tr in (("update", u_bytes, u_us, trace and trace["update_us"]),
+                                           ("pupdate", p_bytes, p_us, trace and trace["pupdate_us"])):
+                if not by or us_ev <= 0:
+                    continue
+                g_ev = by / (us_ev * 1e-6) * 1e-9
+                rec = {"algorithmic_bytes": by, "events_us": round(us_ev, 2), "events_GBs": round(g_ev, 1),
+                       "events_frac_of_8TBs": round(g_ev / 8000.0, 4)}
+                if us_tr:
+                    g_tr = by / (us_tr * 1e-6) * 1e-9
+                    rec.update({"in_graph_us": us_tr, "in_graph_GBs": round(g_tr, 1),
+                                "in_graph_frac_of_8TBs": round(g_tr / 8000.0, 4),
+                                "in_graph_frac_of_measured": round(g_tr / peak, 4)})
+                vec[nm_k] = rec
+            roof["update_GBs"] = vec.get("update", {}).get("in_graph_GBs") or \
+                vec.get("update", {}).get("events_GBs")
+            roof["pupdate_GBs"] = vec.get("pupdate", {}).get("in_graph_GBs") or \
+                vec.get("pupdate", {}).get("events_GBs")
+            roof["vector_kernels"] = dict(vec, target_frac_of_8TBs=0.75,
+                                          how="in_graph = device trace (%globaltimer) of the product "
+                                              "while-graph; events = the events pass (plain launches)")
             if trace:
                 trace["spmv_GBs"] = round(spmv_bytes / (trace["spmv_us"] * 1e-6) * 1e-9, 1)
-                trace["update_GBs"] = round(48.0 * n / (trace["update_us"] * 1e-6) * 1e-9, 1)
-                trace["pupdate_GBs"] = round(24.0 * n / (trace["pupdate_us"] * 1e-6) * 1e-9, 1)
                 trace["how"] = ("device trace (%globaltimer) of one step of the product while-graph: "
                                 "median first-block-start -> last-block-end per kernel, iterations 6..")
                 roof["in_graph_trace"] = trace
-            if ev["update_ms"] > 0 and not sr:
-                u_us = ev["update_ms"] * 1e3 / max(ev["niters"], 1)
-                p_us = ev["pupdate_ms"] * 1e3 / max(ev["niters"], 1)
-                roof["update_GBs"] = round(48.0 * n / (u_us * 1e-6) * 1e-9, 1)
-                roof["pupdate_GBs"] = round(24.0 * n / (p_us * 1e-6) * 1e-9, 1) if p_us > 0 else None
-            elif ev["update_ms"] > 0:
-                u_us = ev["update_ms"] * 1e3 / max(ev["niters"], 1)
-                roof["update_GBs"] = round(72.0 * n / (u_us * 1e-6) * 1e-9, 1)
-            if flush_buf is not None:
-                roof["note"] = ("latency-bound configuration (the problem fits in L2; the product path is "
-                                "one on-chip kernel): the fraction is not a meaningful target here")
+            if main["l2"].startswith("L2 flushed"):
+                roof["note"] = ("latency-bound configuration (the problem fits in L2): the fraction is "
+                                "not a meaningful target here")
         cpu = None
         if world == 1 and not args.no_cpu_baseline:
             # the oracle's CSR needs ~430 B/row of host RAM: above 2^25 rows it
             # is timed on the 256^3 problem instead (said in `sample`)
-            ox, oy, oz = (nx, ny, nz) if n <= (1 << 25) else (256, 256, 256)
-            cs = oracle_sample(ox, oy, oz, iters, args.cpu_budget, sr)
-            nx_s = f"{ox}x{oy}x{oz}"
+            w = WORKLOADS[args.workload]
+            ox, oy, oz = (w["nx"], w["ny"], w["nz"]) if n <= (1 << 25) else (256, 256, 256)
+            it = main["niters_per_step"]
+            cs = oracle_sample(ox, oy, oz, it, args.cpu_budget, sr)
             cpu = {"value": round(cs["value"], 4), "unit": "GFLOP/s", "cores": cs["cores"],
                    "kind": "oracle",
-                   "sample": f"oracle CG (C, OpenMP) on the {nx_s} problem, "
+                   "sample": f"oracle CG (C, OpenMP) on the {ox}x{oy}x{oz} problem, "
                              f"{cs['iters']} iterations ({cs['seconds']:.1f} s) of the "
-                             f"{iters}-iteration step"}
-        t_iter_us = ms_max * 1e3 / max(niters_tot, 1)
+                             f"{it}-iteration step"}
+        wl = WORKLOADS[args.workload]
+        cfg = {k: main[k] for k in ("workload", "baseline_config", "nx", "ny", "nz_per_gpu", "global_rows",
+                                    "global_nnz", "tol", "max_iter", "solve_graph", "l2", "gen_ms")}
+        cfg.update({"iters": main["niters_per_step"], "parallelism": f"zslab{world}",
+                    "cg_variant": "single-reduction (Chronopoulos-Gear, f2)" if sr else "HPCCG",
+                    "spmv_format": ("DIA-27 (columns from stencil offsets) -- EFFECTIVE, a different "
+                                    "method (SURVEY 8(d): OUT)") if dia
+                    else "ELL-27 (val[27][n] + col[27][n])",
+                    "halo": main.get("halo"), "transport": transport if world > 1 else None,
+                    "shared_device": bool(share)})
         line = {
-            "metric": METRIC, "value": round(value, 3), "unit": "GFLOP/s", "n_gpus": world,
-            "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms_max / args.steps, 4),
-            "higher_is_better": True, "scaling": scaling, "vs_baseline": None, "dtype": "f64",
+            "metric": METRIC, "value": main["value"], "unit": "GFLOP/s", "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": main["ms_per_step"],
+            "higher_is_better": True, "scaling": wl["scaling"], "vs_baseline": None, "dtype": "f64",
             "data": "synthetic (HPCCG 27-point problem generated on device, b = A.1)",
-            "config": {"workload": args.workload, "baseline_config": cfg_index,
-                       "nx": nx, "ny": ny, "nz_per_gpu": nz, "iters": iters,
-                       "global_rows": n * world, "global_nnz": nnz_global,
-                       "parallelism": f"zslab{world}",
-                       "cg_variant": "single-reduction (Chronopoulos-Gear, f2)" if sr else "HPCCG",
-                       "spmv_format": "DIA-27 (val[27][n], columns from stencil offsets)" if dia
-                                      else "ELL-27 (val[27][n] + col[27][n])",
-                       "halo": halo, "transport": transport if world > 1 else None,
-                       "shared_device": bool(share),
-                       "solve_graph": {5: "on-chip cluster kernel", 4: "one-cluster persistent kernel",
-                                       3: "cooperative persistent kernel", 2: "while-graph",
-                                       1: "per-iteration graph", 0: "plain"}.get(
-                           main.get("graph_mode"), "?"),
-                       "l2": l2_note,
-                       "gen_ms": round(gen_ms, 3)},
-            "t_iter_us": round(t_iter_us, 3),
-            "alt_spmv_format": alt_line,
-            "niters_per_step": niters_tot // args.steps,
-            "max_abs_x_minus_1": err, "normr": r["normr"],
-            "gpu_launches": launches,
-            "clocks": clk.summary(),
-            "e2e": {"value": round(e2e_value, 3), "unit": "GFLOP/s", "h2d_bytes_per_step": 8 * n,
-                    "d2h_bytes_per_step": 8 * n + 8, "max_abs_x_minus_1_host": x_host_err},
+            "config": cfg,
+            "t_iter_us": main["t_iter_us"],
+            "niters_per_step": main["niters_per_step"],
+            "max_abs_x_minus_1": main["max_abs_x_minus_1"], "normr": main["normr"],
+            "correctness": main["correctness"],
+            "ranks": ranks,
+            "multi_gpu_ok": (all(r["correct"] and r["lib_nranks"] == world for r in ranks)
+                             and len({r["halo_mode"] for r in ranks}) == 1),
+            "gpu_launches": main["gpu_launches"],
+            "clocks": main.get("clocks"),
+            "e2e": main["e2e"],
             "roofline": roof,
             "cpu_baseline": cpu,
+            "sub_configs": subs,
         }
+        if main.get("fallback"):
+            line["peer_fallback"] = main["fallback"]
         print(json.dumps(line), flush=True)
-    prob.free()
     ctx.close()
     if world > 1:
         dist.destroy_process_group()
@@ -985,7 +1135,9 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
     ap.add_argument("--workload", choices=sorted(WORKLOADS) + ["blas1", "tridiag", "lbm"],
-                    default="hpccg128")
+                    default="hpccg256",
+                    help="hpccg256 (default, every N: configs[2], 256^3 per GPU, weak) -- its line "
+                         "carries configs[1] / [0] / [3] as sub_configs")
     ap.add_argument("--blas1-max", type=int, default=None, help="largest BLAS-1 n")
     ap.add_argument("--tri-n", type=int, default=100_000_000, help="tridiag SIZE (P:L475)")
     ap.add_argument("--lbm-size", type=int, default=1000, help="LBM SIZE (P:L411)")
@@ -1003,10 +1155,14 @@ def main():
     ap.add_argument("--cg-variant", choices=["hpccg", "sr"], default="hpccg",
                     help="hpccg: HPCCG's CG (default); sr: single-reduction CG (SURVEY f2)")
     ap.add_argument("--spmv-format", choices=["ell", "dia"], default="ell",
-                    help="HPCCG_OPT_SPMV_FORMAT: ELL-27 (default) or the DIA-27 reading (no col[])")
+                    help="HPCCG_OPT_SPMV_FORMAT: ELL-27 (default) or the DIA-27 reading (no col[]) -- "
+                         "EFFECTIVE numbers of a different method (SURVEY 8(d): OUT), never the headline")
+    ap.add_argument("--no-sub-configs", action="store_true",
+                    help="skip the configs[1] / [0] / [3] sub-records of the CG line")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-budget", type=float, default=12.0, help="seconds of oracle CG")
-    ap.add_argument("--ref-iters", type=int, default=20, help="oracle iterations per reference step")
+    ap.add_argument("--ref-iters", type=int, default=None,
+                    help="oracle iterations per reference step (default per workload)")
     args = ap.parse_args()
     if args.warmup < 3:
         raise SystemExit("--warmup must be >= 3")
@@ -1022,14 +1178,13 @@ def main():
         if args.impl == "reference":
             return run_reference_blas1(args)
         return run_blas1(args)
-    nx, ny, nz, iters, cfg, scaling = WORKLOADS[args.workload]
-    if args.iters:
-        iters = args.iters
+    w = dict(WORKLOADS[args.workload])
+    if args.iters:                       # fixed iteration count (tol 0), e.g. for tests
+        w.update(max_iter=args.iters + 1, tol=0.0)
+        WORKLOADS[args.workload] = w
     if args.impl == "reference":
-        if scaling == "strong":
-            nz = nz // args.gpus
-        return run_reference(args, nx, ny, nz, iters, cfg)
-    return run_ours(args, nx, ny, nz, iters, cfg, scaling)
+        return run_reference(args, w)
+    return run_ours(args)
 
 
 if __name__ == "__main__":

@@ -130,7 +130,16 @@ extern "C" {
                                which every block of the next p update collects -- 3 kernels
                                per iteration; needs even nx*ny and n, else behaves as 1.
                                Bit-identical to the loopback reduction order.  Waits time out
-                               after ~2 s with HPCCG_ECUDA instead of hanging. */
+                               after HPCCG_OPT_PEER_TIMEOUT_MS with HPCCG_ECUDA instead of
+                               hanging; hpccg_last_error() names the rank that gave up, what it
+                               waited for (halo plane / allreduce post) and the peer it waited
+                               on.  The record is sticky: a slab that timed out has lost step
+                               with its peers, so every later hpccg_solve of that problem
+                               returns HPCCG_ECUDA at once (recreate the problem).  The value
+                               is range-checked before any peer mapping is attempted. */
+#define HPCCG_OPT_PEER_TIMEOUT_MS 22 /* HALO_PEER waits: give up after this many milliseconds
+                               (1 .. 3600000; default 30000 -- above any host-side skew
+                               between ranks such as graph instantiation or a slow rank) */
 #define HPCCG_OPT_WHILE_UNROLL 15 /* CG iterations per execution of the WHILE body
                                (default 4: amortises the conditional node's ~8 us) */
 #define HPCCG_OPT_CLUSTER_ROWS 12 /* up to this many rows (default 16384) the persistent solve
@@ -242,7 +251,9 @@ HPCCG_API int hpccg_peer_export(hpccg_problem *prob, void *blob);
 HPCCG_API int hpccg_peer_attach(hpccg_problem *prob, const void *blobs);
 
 /* rank / nranks of the context; nslabs = slabs hosted by this process
- * (1, or nranks for loopback). */
+ * (1, or nranks for loopback).  NCCL contexts answer from the communicator
+ * itself (ncclCommUserRank / ncclCommCount), so a bench line can show how many
+ * ranks NCCL actually joined. */
 HPCCG_API int hpccg_ctx_info(const hpccg_ctx *ctx, int *rank, int *nranks, int *nslabs);
 
 HPCCG_API void hpccg_finalize(hpccg_ctx *ctx);

@@ -165,6 +165,7 @@ struct hpccg_problem {
     std::vector<std::pair<uint64_t, unsigned>> fpush;
     int opt_smem_threads = 0;          // on-chip solve CTA width: 0 auto, 256, 512
     int opt_peer = 0;                  // multi-slab: halo push + allreduce over peer memory
+    int64_t opt_peer_timeout_ms = 30000;  // give up a peer-memory wait after this long
     std::vector<void *> ipc_opened;    // peers' buffers mapped with cudaIpcOpenMemHandle
     int last_persist_mode = 3;
     // graph of one CG iteration (per-iteration replay) ...
@@ -1739,12 +1740,38 @@ int api_reduce(hpccg_ctx *ctx, bool is_max, double *result, L launch) {
 // peers' buffers are mapped with cudaIpcOpenMemHandle (NVLink P2P between
 // GPUs); the arena layout is identical on every rank, so a peer's vector sits
 // at the same offset.
+// the wait limit of every hosted slab's PeerSync (read by the spinning kernels)
+int peer_set_timeout(hpccg_problem *p) {
+    const unsigned long long ns = (unsigned long long)p->opt_peer_timeout_ms * 1000000ull;
+    for (Slab &sl : p->slabs)
+        if (sl.psync) CU(cudaMemcpy(&sl.psync->timeout_ns, &ns, sizeof ns, cudaMemcpyHostToDevice));
+    return HPCCG_OK;
+}
+
 int peer_alloc(hpccg_problem *p) {
     if (p->ctx->nranks > kMaxPeers) return fail(HPCCG_ENOTSUP, "peer mode supports up to %d ranks", kMaxPeers);
     for (Slab &sl : p->slabs)
         if (!sl.psync) CHECK(alloc_zero((void **)&sl.psync, sizeof(PeerSync)));
+    return peer_set_timeout(p);
+}
+
+// a timed-out wait -> HPCCG_ECUDA naming the rank, what it waited for and from whom
+int peer_check_error(hpccg_problem *p, const char *op) {
+    for (const Slab &sl : p->slabs) {
+        int e[2] = {0, 0};  // error, error_peer (adjacent fields)
+        CU(cudaMemcpy(e, &sl.psync->error, sizeof e, cudaMemcpyDeviceToHost));
+        if (!e[0]) continue;
+        static const char *what[] = {"?", "the halo plane of rank %d (lower neighbour)",
+                                     "the halo plane of rank %d (upper neighbour)",
+                                     "the allreduce post of rank %d", "the fused scalar post of rank %d"};
+        char w[96];
+        snprintf(w, sizeof w, what[e[0] >= 1 && e[0] <= 4 ? e[0] : 0], e[1]);
+        return fail(HPCCG_ECUDA, "%s: peer-memory wait timed out after %lld ms on rank %d, waiting for %s",
+                    op, (long long)p->opt_peer_timeout_ms, sl.rank, w);
+    }
     return HPCCG_OK;
 }
+
 
 int peer_export(hpccg_problem *p, unsigned char *blob) {
     CHECK(peer_alloc(p));
@@ -1993,8 +2020,16 @@ int hpccg_init_loopback(hpccg_ctx **out, int device, void *stream, int nranks) {
 
 int hpccg_ctx_info(const hpccg_ctx *ctx, int *rank, int *nranks, int *nslabs) {
     if (!ctx) return fail(HPCCG_EINVAL, "NULL ctx");
-    if (rank) *rank = ctx->rank;
-    if (nranks) *nranks = ctx->nranks;
+    int r = ctx->rank, n = ctx->nranks;
+#ifdef HPCCG_WITH_NCCL
+    if (ctx->mode == MODE_NCCL && ctx->comm) {  // the communicator's own view
+        ncclResult_t nr = ncclCommCount(ctx->comm, &n);
+        if (nr == ncclSuccess) nr = ncclCommUserRank(ctx->comm, &r);
+        if (nr != ncclSuccess) return fail(HPCCG_ENCCL, "ncclCommCount: %s", ncclGetErrorString(nr));
+    }
+#endif
+    if (rank) *rank = r;
+    if (nranks) *nranks = n;
     if (nslabs) *nslabs = ctx->nslabs;
     return HPCCG_OK;
 }
@@ -2264,10 +2299,14 @@ int hpccg_set_option(hpccg_problem *p, int key, int64_t value) {
             p->opt_serp = (int)value;
             return HPCCG_OK;
         case HPCCG_OPT_HALO_PEER:
-            if (value && p->ctx->mode != MODE_SINGLE && !p->slabs[0].ptab) CHECK(enable_peer(p));
             if (value < 0 || value > 2) return fail(HPCCG_EINVAL, "halo peer: 0, 1 or 2");
+            if (value && p->ctx->mode != MODE_SINGLE && !p->slabs[0].ptab) CHECK(enable_peer(p));
             p->opt_peer = (int)value;
             return HPCCG_OK;
+        case HPCCG_OPT_PEER_TIMEOUT_MS:
+            if (value < 1 || value > 3600000) return fail(HPCCG_EINVAL, "peer timeout: 1 .. 3600000 ms");
+            p->opt_peer_timeout_ms = value;
+            return peer_set_timeout(p);
         case HPCCG_OPT_SMEM_THREADS:
             if (value != 0 && value != 256 && value != 512) return fail(HPCCG_EINVAL, "smem threads: 0, 256, 512");
             p->opt_smem_threads = (int)value;
@@ -2433,9 +2472,7 @@ int hpccg_maxabsdiff(hpccg_problem *p, double *result) {
         CU(cudaMemcpyAsync(ctx->h_pinned, &sl.sc->red_out, sizeof(double), cudaMemcpyDeviceToHost,
                            ctx->stream));
         CU(cudaStreamSynchronize(ctx->stream));
-        int perr = 0;
-        CU(cudaMemcpy(&perr, &sl.psync->error, sizeof perr, cudaMemcpyDeviceToHost));
-        if (perr) return fail(HPCCG_ECUDA, "peer-memory wait timed out");
+        CHECK(peer_check_error(p, "hpccg_maxabsdiff"));
         *result = *(volatile double *)ctx->h_pinned;
         return HPCCG_OK;
     }
@@ -2470,6 +2507,14 @@ int hpccg_solve(hpccg_problem *p, int max_iter, double tol, int *niters, double 
                      !p->while_failed;
     p->ev_used = 0;
     p->timed.clear();
+    // a slab whose earlier peer wait timed out has lost step with its peers (the
+    // flag counts / epochs no longer agree): refuse to run instead of computing on
+    // stale halos (the peers then time out too and report it)
+    if (peer_on(p) && peer_check_error(p, "hpccg_solve") != HPCCG_OK) {
+        const std::string why = g_err;
+        return fail(HPCCG_ECUDA, "%s -- an earlier solve of this problem timed out: recreate it "
+                    "(hpccg_free + hpccg_generate)", why.c_str());
+    }
     const int64_t l0 = ctx->launches;
     // the persisting-L2 window costs two device-limit changes per solve; the
     // persistent kernels keep their small working set on chip / in L2 anyway
@@ -2536,12 +2581,7 @@ int hpccg_solve(hpccg_problem *p, int max_iter, double tol, int *niters, double 
     CU(cudaStreamSynchronize(ctx->stream));
     CU(cudaGetLastError());
     l2win.release();
-    if (peer_on(p))
-        for (const Slab &sl : p->slabs) {
-            int perr = 0;
-            CU(cudaMemcpy(&perr, &sl.psync->error, sizeof perr, cudaMemcpyDeviceToHost));
-            if (perr) return fail(HPCCG_ECUDA, "peer-memory wait timed out (slab %d)", sl.rank);
-        }
+    if (peer_on(p)) CHECK(peer_check_error(p, "hpccg_solve"));
 
     CgScalars hs;
     CU(cudaMemcpy(&hs, p->slabs[0].sc, sizeof hs, cudaMemcpyDeviceToHost));

@@ -257,7 +257,9 @@ struct PeerSync {                      // one per slab, in that slab's device me
     unsigned long long ar_count;       // allreduces I have collected
     unsigned long long ar_posted;      // allreduces I have posted
     unsigned int push_ticket;          // blocks of the current push done
-    int error;                         // 1: a wait timed out
+    int error;                         // != 0: a wait timed out (PEER_WAIT_* of the first one)
+    int error_peer;                    //   ... the rank it waited for
+    unsigned long long timeout_ns;     // give up a wait after this long (host-set; 0 = 30 s)
     unsigned long long ar_tag[2][kMaxPeers];
     double ar_val[2][kMaxPeers][2];
     // HALO_PEER = 2 (collectives fused into the CG kernels): separate words,
@@ -293,15 +295,28 @@ __device__ __forceinline__ unsigned long long ld_acquire_sys(const unsigned long
     return v;
 }
 
-// spin until *flag >= target; false (and the error flag) after ~2 s
+// what a timed-out wait was waiting for (PeerSync::error; hpccg_solve names it)
+enum : int { PEER_WAIT_HALO_LO = 1, PEER_WAIT_HALO_HI = 2, PEER_WAIT_ALLREDUCE = 3, PEER_WAIT_SCALAR = 4 };
+
+__device__ __forceinline__ unsigned long long peer_timeout_ns(const PeerSync *m) {
+    const unsigned long long t = *(const volatile unsigned long long *)&m->timeout_ns;
+    return t ? t : 30000000000ull;
+}
+
+// record the FIRST timeout of this slab (what, peer rank); later waits see it and return at once
+__device__ __forceinline__ void peer_fail(PeerSync *m, int what, int peer) {
+    if (atomicCAS(&m->error, 0, what) == 0) m->error_peer = peer;
+}
+
+// spin until *flag >= target; false (and the error record) after timeout_ns
 __device__ __forceinline__ bool spin_until(const unsigned long long *flag, unsigned long long target,
-                                           PeerSync *mine) {
+                                           PeerSync *mine, int what, int peer) {
     if (ld_acquire_sys(flag) >= target) return true;  // the common case: one load
     if (*(volatile int *)&mine->error) return false;  // an earlier wait timed out: do not hang again
-    const unsigned long long t0 = gtimer();
+    const unsigned long long t0 = gtimer(), lim = peer_timeout_ns(mine);
     while (ld_acquire_sys(flag) < target) {
-        if (gtimer() - t0 > 2000000000ull) {
-            mine->error = 1;
+        if (gtimer() - t0 > lim) {
+            peer_fail(mine, what, peer);
             return false;
         }
         __nanosleep(64);
@@ -382,10 +397,11 @@ __device__ __forceinline__ double fused_collect_block(const PeerTab *t, int q, u
         for (int r0 = 0; r0 < P; r0 += 32) {
             double v = mine;
             if (r0 + lane < P && r0 + lane != t->rank && !ll_read(m->fll[q][r0 + lane], tag, &v)) {
-                const unsigned long long t0 = gtimer();
+                const unsigned long long t0 = gtimer(), lim = peer_timeout_ns(m);
                 while (!ll_read(m->fll[q][r0 + lane], tag, &v)) {
-                    if (*(volatile int *)&m->error || gtimer() - t0 > 2000000000ull) {
-                        m->error = 1;
+                    if (*(volatile int *)&m->error) break;
+                    if (gtimer() - t0 > lim) {
+                        peer_fail(m, PEER_WAIT_SCALAR, r0 + lane);
                         break;
                     }
                     __nanosleep(32);
@@ -430,12 +446,13 @@ __device__ __forceinline__ double2 fused_collect2_block(const PeerTab *t, int q,
             double g = mine.x, d = mine.y;
             const int src = r0 + lane;
             if (src < P && src != t->rank) {
-                const unsigned long long t0 = gtimer();
+                const unsigned long long t0 = gtimer(), lim = peer_timeout_ns(m);
                 bool okg = false, okd = false;
                 while (!(okg = okg || ll_read(m->fll[q][src], tag, &g)) |
                        !(okd = okd || ll_read(m->fll2[q][src], tag, &d))) {
-                    if (*(volatile int *)&m->error || gtimer() - t0 > 2000000000ull) {
-                        m->error = 1;
+                    if (*(volatile int *)&m->error) break;
+                    if (gtimer() - t0 > lim) {
+                        peer_fail(m, PEER_WAIT_SCALAR, src);
                         break;
                     }
                     __nanosleep(32);
@@ -649,9 +666,10 @@ __device__ __forceinline__ void fused_halo_wait(const SpmvArgs &a, int64_t first
         const PeerTab *t = a.fpeer;
         // iteration k's SpMV: niters = k (written by the p update / f2 update)
         const unsigned long long tg = ftag(__ldg(&a.sc->epoch), (unsigned long long)__ldg(&a.sc->niters));
-        if (first < a.plane && t->rank > 0) spin_until(&t->mine->fflag_from_lo, tg, t->mine);
+        if (first < a.plane && t->rank > 0)
+            spin_until(&t->mine->fflag_from_lo, tg, t->mine, PEER_WAIT_HALO_LO, t->rank - 1);
         if (last >= a.stride - a.plane && t->rank < t->nranks - 1)
-            spin_until(&t->mine->fflag_from_hi, tg, t->mine);
+            spin_until(&t->mine->fflag_from_hi, tg, t->mine, PEER_WAIT_HALO_HI, t->rank + 1);
     }
     __syncthreads();
 }
@@ -2225,8 +2243,10 @@ __global__ void halo_wait_kernel(const PeerTab *t) {
     if (threadIdx.x != 0) return;
     PeerSync *m = t->mine;
     const unsigned long long target = m->recv_count + 1;
-    if (t->rank > 0 && !spin_until(&m->flag_from_lo, target, m)) return;
-    if (t->rank < t->nranks - 1 && !spin_until(&m->flag_from_hi, target, m)) return;
+    if (t->rank > 0 && !spin_until(&m->flag_from_lo, target, m, PEER_WAIT_HALO_LO, t->rank - 1)) return;
+    if (t->rank < t->nranks - 1 &&
+        !spin_until(&m->flag_from_hi, target, m, PEER_WAIT_HALO_HI, t->rank + 1))
+        return;
     m->recv_count = target;
 }
 
@@ -2253,7 +2273,7 @@ __global__ void peer_allreduce_kernel(const PeerTab *t, const double *src, doubl
         const unsigned long long c = m->ar_count + 1;
         const int q = (int)(c & 1);
         for (int r = lane; r < P; r += 32)
-            if (!spin_until(&m->ar_tag[q][r], c, m)) break;
+            if (!spin_until(&m->ar_tag[q][r], c, m, PEER_WAIT_ALLREDUCE, r)) break;
         __syncwarp();
         if (lane == 0) {
             __threadfence();

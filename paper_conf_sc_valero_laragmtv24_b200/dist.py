@@ -89,3 +89,44 @@ def max_time_sum_work(ms_local: float, work_local: float, device=None):
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         dist.all_reduce(w, op=dist.ReduceOp.SUM)
     return float(t.item()), float(w.item())
+
+
+def _attempt(fn):
+    """None if fn() returns, else the exception as one line."""
+    try:
+        fn()
+        return None
+    except Exception as e:  # noqa: BLE001 -- every failure is reported, none is fatal here
+        return f"{type(e).__name__}: {e}".replace("\n", " ")[:300]
+
+
+def _gather_objects(obj):
+    import torch.distributed as dist
+    out = [None] * dist.get_world_size()
+    dist.all_gather_object(out, obj)
+    return out
+
+
+def decide_peer_path(try_map, try_proof, reset, gather=None) -> dict:
+    """Agree, on every rank, whether the multi-GPU solve runs over peer memory
+    (HPCCG_OPT_HALO_PEER) or falls back to NCCL send/recv + allreduce.
+
+    Two collective stages, each followed by an all-gather of every rank's
+    outcome so all ranks take the SAME decision (a rank on the peer path and
+    one on NCCL would wait on each other forever):
+      1. try_map()   -- map the neighbours' buffers (CUDA IPC over NVLink);
+      2. try_proof() -- a short solve that exercises the mapping end to end.
+    If any rank failed a stage, every rank calls reset() (HALO_PEER = 0) and the
+    result names the stage, the failing ranks and their errors."""
+    gather = gather or _gather_objects
+    for stage, fn in (("map", try_map), ("proof", try_proof)):
+        errs = gather(_attempt(fn))
+        failed = {r: e for r, e in enumerate(errs) if e}
+        if failed:
+            reset_err = _attempt(reset)
+            first = min(failed)
+            return {"peer": False, "stage": stage, "failed_ranks": sorted(failed),
+                    "errors": {str(r): e for r, e in failed.items()}, "reset_error": reset_err,
+                    "why": f"{stage} failed on rank(s) {sorted(failed)}: {failed[first]}"}
+    return {"peer": True, "stage": "proof", "failed_ranks": [], "errors": {}, "reset_error": None,
+            "why": None}

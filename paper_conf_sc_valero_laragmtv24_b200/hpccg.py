@@ -38,7 +38,7 @@ HPCCG_OPT_PERSISTENT, HPCCG_OPT_PERSIST_ROWS, HPCCG_OPT_PDL = 9, 10, 11
 HPCCG_OPT_CLUSTER_ROWS, HPCCG_OPT_SMEM_SOLVE, HPCCG_OPT_TRACE = 12, 13, 14
 HPCCG_OPT_WHILE_UNROLL, HPCCG_OPT_CG_VARIANT, HPCCG_OPT_FINISHER_FREE = 15, 16, 17
 HPCCG_OPT_SMEM_THREADS, HPCCG_OPT_HALO_PEER, HPCCG_OPT_SERPENTINE = 18, 19, 20
-HPCCG_OPT_SPMV_FORMAT = 21
+HPCCG_OPT_SPMV_FORMAT, HPCCG_OPT_PEER_TIMEOUT_MS = 21, 22
 
 _lock = threading.Lock()
 _lib = None
@@ -324,10 +324,17 @@ class Context:
             self.handle = hpccg_init_peer(device, stream, rank, nranks)
         else:
             self.handle = hpccg_init(device, stream, rank, nranks, unique_id)
+        self.kind = "loopback" if loopback else "peer" if peer else "nccl" if nranks > 1 or unique_id \
+            else "single"
+        i = self.info()
+        self.rank, self.nranks, self.nslabs = i["rank"], i["nranks"], i["nslabs"]
+
+    def info(self) -> dict:
+        """hpccg_ctx_info (NCCL contexts: the communicator's own rank / count)."""
         r, n, s = ctypes.c_int(), ctypes.c_int(), ctypes.c_int()
         _check(lib().hpccg_ctx_info(self.handle, ctypes.byref(r), ctypes.byref(n),
                                     ctypes.byref(s)), "hpccg_ctx_info")
-        self.rank, self.nranks, self.nslabs = r.value, n.value, s.value
+        return {"rank": r.value, "nranks": n.value, "nslabs": s.value, "kind": self.kind}
 
     def ddot(self, n: int, x, y) -> float:
         return hpccg_ddot(self.handle, n, x, y)

@@ -46,3 +46,32 @@ def run_maxabs(rank, nranks, dims, x_slab, xe_slab, to_parent, from_parent):
             to_parent.put(("done", rank, p.maxabsdiff()))
     except Exception as e:
         to_parent.put(("error", rank, repr(e)))
+
+
+def run_timeout(rank, nranks, dims, halo, to_parent, from_parent):
+    """Rank 0 solves with a short peer-wait limit while rank 1 never joins: the
+    solve must fail with HPCCG_ECUDA naming both ranks (no hang), and a second
+    solve of the same problem must refuse at once (sticky record)."""
+    try:
+        import time
+
+        from paper_conf_sc_valero_laragmtv24_b200 import hpccg as H
+        with H.Context(0, rank=rank, nranks=nranks, peer=True) as c, H.Problem(c, *dims) as p:
+            to_parent.put(("blob", rank, p.peer_export()))
+            p.peer_attach(from_parent.get(timeout=120))
+            p.set_option(H.HPCCG_OPT_HALO_PEER, halo)
+            out = {}
+            if rank == 0:
+                p.set_option(H.HPCCG_OPT_PEER_TIMEOUT_MS, 300)
+                for k in ("first", "second"):
+                    t0 = time.perf_counter()
+                    try:
+                        p.solve(20, 0.0)
+                        out[k] = ("ok", 0, "", 0.0)
+                    except H.HpccgError as e:
+                        out[k] = ("error", e.code, str(e), time.perf_counter() - t0)
+            else:
+                from_parent.get(timeout=120)      # released after rank 0 reported
+            to_parent.put(("done", rank, out))
+    except Exception as e:
+        to_parent.put(("error", rank, repr(e)))

@@ -26,7 +26,7 @@ def _torchrun(n, *argv, port):
                                                  (2, "sr", "auto", 29613)])
 def test_bench_multirank_shared_device(n, variant, halo, port):
     r = _torchrun(n, "--workload", "hpccg20", "--iters", "30", "--steps", "3", "--warmup", "3",
-                  "--cg-variant", variant, "--halo", halo, port=port)
+                  "--cg-variant", variant, "--halo", halo, "--no-sub-configs", port=port)
     assert r.returncode == 0, r.stderr[-3000:]
     lines = [l for l in r.stdout.splitlines() if l.startswith("{")]
     assert len(lines) == 1, r.stdout[-2000:]
@@ -39,6 +39,15 @@ def test_bench_multirank_shared_device(n, variant, halo, port):
     assert d["niters_per_step"] == 30
     assert d["max_abs_x_minus_1"] < 1.0          # 30 iterations: on the way to x = 1
     assert d["e2e"]["value"] > 0 and d["gpu_launches"] > 0
+    # the N > 1 line verifies itself: the tol 1e-12 solve of the global problem,
+    # and per rank the transport / exchange mode / library rank count
+    cor = d["correctness"]
+    assert cor["ok"] and cor["max_abs_x_minus_1"] < 1e-13 and cor["normr"] <= 1e-12
+    ranks = d["ranks"]
+    assert [q["rank"] for q in ranks] == list(range(n))
+    assert all(q["transport"] == "peer" and q["lib_nranks"] == n and q["correct"] for q in ranks)
+    assert {q["halo_mode"] for q in ranks} == {1 if halo == "peer" else 2}
+    assert d["multi_gpu_ok"] is True
 
 
 @pytest.mark.gpu
@@ -46,8 +55,27 @@ def test_bench_multirank_strong_split():
     """Strong scaling (hpccg512s's split rule) on a reduced iteration count: the
     global 512 planes are split over the ranks (config nz_per_gpu = 512 / n)."""
     r = _torchrun(2, "--workload", "hpccg512s", "--iters", "3", "--steps", "1", "--warmup", "3",
-                  port=29614)
+                  "--no-sub-configs", port=29614)
     assert r.returncode == 0, r.stderr[-3000:]
     d = json.loads([l for l in r.stdout.splitlines() if l.startswith("{")][0])
     assert d["scaling"] == "strong" and d["config"]["nz_per_gpu"] == 256
     assert d["config"]["global_rows"] == 512 ** 3
+    cor = d["correctness"]              # 512^3 global at tol 1e-12: SURVEY's 115 (+-1)
+    assert cor["expected_niters"] == 115 and cor["ok"], cor
+
+
+@pytest.mark.gpu
+def test_bench_multirank_weak_256_correctness_and_subconfig():
+    """The default workload on 2 ranks (256^2 x 512 global): the correctness solve
+    must hit SURVEY's independent count (113 +- 1), and the strong-scaling
+    sub-record (512^3 split over the 2 ranks, its own 100 iterations; --iters
+    shortens only the main workload) is carried in sub_configs."""
+    r = _torchrun(2, "--steps", "1", "--warmup", "3", "--iters", "5", port=29615)
+    assert r.returncode == 0, r.stderr[-3000:]
+    d = json.loads([l for l in r.stdout.splitlines() if l.startswith("{")][0])
+    assert d["config"]["workload"] == "hpccg256" and d["scaling"] == "weak"
+    cor = d["correctness"]
+    assert cor["expected_niters"] == 113 and cor["ok"], cor
+    sub = d["sub_configs"]["hpccg512s"]
+    assert sub["scaling"] == "strong" and sub["nz_per_gpu"] == 256 and sub["correctness"]["ok"]
+    assert sub["value"] > 0 and sub["e2e"]["value"] > 0

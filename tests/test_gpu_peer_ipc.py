@@ -127,3 +127,60 @@ def test_processes_fused_peer_single_reduction():
         np.testing.assert_array_equal(x, xl)
         assert abs(outs[0]["niters"] - oref["niters"]) <= 1
         assert np.max(np.abs(x - oref["x"])) <= 1e-10
+
+
+@pytest.mark.parametrize("halo", [1, 2])
+def test_peer_wait_timeout_names_rank_and_is_sticky(halo):
+    """HPCCG_OPT_PEER_TIMEOUT_MS: a rank whose neighbour never joins gives up
+    after the limit with HPCCG_ECUDA naming itself, what it waited for and the
+    peer (no hang); the problem then refuses further solves at once."""
+    import peer_worker
+    P, dims = 2, (16, 12, 6)
+    mctx = mp.get_context("spawn")
+    to_parent = mctx.Queue()
+    inbox = [mctx.Queue() for _ in range(P)]
+    procs = [mctx.Process(target=peer_worker.run_timeout, args=(r, P, dims, halo, to_parent, inbox[r]))
+             for r in range(P)]
+    for pr in procs:
+        pr.start()
+    try:
+        blobs = {}
+        while len(blobs) < P:
+            kind, r, payload = to_parent.get(timeout=240)
+            assert kind == "blob", payload
+            blobs[r] = payload
+        for q in inbox:
+            q.put([blobs[r] for r in range(P)])
+        kind, r, out = to_parent.get(timeout=240)
+        assert kind == "done" and r == 0, out
+        inbox[1].put("go")
+        kind, r1, _ = to_parent.get(timeout=240)
+        assert kind == "done" and r1 == 1
+    finally:
+        for pr in procs:
+            pr.join(timeout=30)
+            if pr.is_alive():
+                pr.kill()
+    st, code, msg, secs = out["first"]
+    assert st == "error" and code == H.HPCCG_ECUDA, out
+    assert "timed out after 300 ms on rank 0" in msg and "rank 1" in msg, msg
+    assert secs < 20, secs
+    st2, code2, msg2, secs2 = out["second"]
+    assert st2 == "error" and code2 == H.HPCCG_ECUDA and "recreate" in msg2 and secs2 < 5, out
+
+
+def test_halo_peer_value_checked_before_mapping():
+    """An out-of-range HALO_PEER is refused (EINVAL) before any peer mapping or
+    collective is attempted (1-rank NCCL context)."""
+    uid = H.hpccg_unique_id()
+    with H.Context(0, rank=0, nranks=1, unique_id=uid) as c, H.Problem(c, 8, 8, 4) as p:
+        for bad in (3, -1):
+            with pytest.raises(H.HpccgError) as e:
+                p.set_option(H.HPCCG_OPT_HALO_PEER, bad)
+            assert e.value.code == H.HPCCG_EINVAL
+        with pytest.raises(H.HpccgError) as e:
+            p.set_option(H.HPCCG_OPT_PEER_TIMEOUT_MS, 0)
+        assert e.value.code == H.HPCCG_EINVAL
+        p.set_option(H.HPCCG_OPT_PEER_TIMEOUT_MS, 45000)
+        r = p.solve(50, 1e-12)
+        assert r["niters"] > 0

@@ -172,3 +172,37 @@ def test_gloo_bootstrap_unique_id_and_aggregation():
 @pytest.mark.parametrize("dims", [(9, 7, 4), (12, 10, 1)])
 def test_gloo_zslab_cg_matches_global_oracle(dims):
     _run(_body_distributed_cg, 2, *dims, 150, 1e-12)
+
+
+def _body_peer_decision(rank, world, fail_rank, fail_stage):
+    """bench.py's fallback decision (dist.decide_peer_path) over gloo: one rank's
+    IPC mapping (or proof solve) fails -> EVERY rank resets to NCCL and reports
+    the same stage and failing rank; nobody proceeds to the proof after a map
+    failure."""
+    from paper_conf_sc_valero_laragmtv24_b200 import dist as D
+    calls = []
+
+    def stage_fn(stage):
+        def fn():
+            calls.append(stage)
+            if rank == fail_rank and stage == fail_stage:
+                raise RuntimeError(f"hpccg_set_option: cudaIpcOpenMemHandle failed on rank {rank}")
+        return fn
+
+    dec = D.decide_peer_path(stage_fn("map"), stage_fn("proof"), stage_fn("reset"))
+    got = [None] * world
+    dist.all_gather_object(got, dec)
+    assert all(g == got[0] for g in got), got            # the same decision everywhere
+    if fail_rank is None:
+        assert dec["peer"] is True and calls == ["map", "proof"]
+        return
+    assert dec["peer"] is False and dec["stage"] == fail_stage
+    assert dec["failed_ranks"] == [fail_rank] and str(fail_rank) in dec["errors"]
+    assert f"rank {fail_rank}" in dec["why"]
+    want = ["map", "reset"] if fail_stage == "map" else ["map", "proof", "reset"]
+    assert calls == want, calls
+
+
+@pytest.mark.parametrize("fail_rank,fail_stage", [(None, None), (1, "map"), (0, "map"), (1, "proof")])
+def test_gloo_peer_path_fallback_decision(fail_rank, fail_stage):
+    _run(_body_peer_decision, 2, fail_rank, fail_stage)
