@@ -1,5 +1,13 @@
 """Turn gpurun_out/ ncu artefacts into committed profiles/ summaries.
-usage: python tools/summarize_profiles.py ROUND_TAG"""
+
+usage: python tools/summarize_profiles.py TAG [WORKLOAD]
+
+Reads gpurun_out/launches.csv (launch list) and gpurun_out/prof_<WORKLOAD>_{cold,warm}.ncu-rep
+(`ncu --set full` of the three CG kernels, tools/profile_round.sh) and writes
+profiles/<TAG>_ncu_<WORKLOAD>.json: per kernel the DRAM bytes per launch against
+its algorithmic bytes (SpMV 12 nnz + 16 n, x/r update 48 n, p update 24 n; DESIGN
+sec. 7), cold and warm cache; merges the SpMV's cold-cache DRAM bytes per launch
+into profiles/spmv_traffic.json[WORKLOAD] (bench.py roofline.traffic)."""
 import collections
 import csv
 import io
@@ -8,13 +16,23 @@ import os
 import subprocess
 import sys
 
-tag = sys.argv[1] if len(sys.argv) > 1 else "r1"
+tag = sys.argv[1] if len(sys.argv) > 1 else "r2"
+W = sys.argv[2] if len(sys.argv) > 2 else "hpccg256"
 G, P = "gpurun_out", "profiles"
 os.makedirs(P, exist_ok=True)
+DIMS = {"hpccg256": (256, 256, 256), "hpccg128": (128, 128, 128), "hpccg512s": (512, 512, 512),
+        "hpccg20": (20, 30, 10)}
+
+
+def nnz_of(nx, ny, nz):
+    return (3 * nx - 2) * (3 * ny - 2) * (3 * nz - 2)
 
 
 def launch_list():
-    rows = list(csv.reader(open(os.path.join(G, "launches.csv"))))
+    p = os.path.join(G, "launches.csv")
+    if not os.path.exists(p):
+        return []
+    rows = list(csv.reader(open(p)))
     hdr = None
     agg = collections.OrderedDict()
     for r in rows:
@@ -28,7 +46,8 @@ def launch_list():
             continue
         k = d["Kernel Name"]
         v = float(d["Metric Value"].replace(",", ""))
-        scale = {"ns": 1e-3, "us": 1.0, "usecond": 1.0, "nsecond": 1e-3, "ms": 1e3}.get(d["Metric Unit"], 1e-3)
+        scale = {"ns": 1e-3, "us": 1.0, "usecond": 1.0, "nsecond": 1e-3, "ms": 1e3,
+                 "msecond": 1e3}.get(d["Metric Unit"], 1e-3)
         agg.setdefault(k, []).append(v * scale)
     tot = sum(sum(v) for v in agg.values())
     out = []
@@ -47,6 +66,13 @@ KEYS = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum
         "lts__throughput.avg.pct_of_peak_sustained_elapsed",
         "smsp__average_warps_issue_stalled_long_scoreboard_per_issue_active.ratio",
         "smsp__average_warp_latency_per_inst_issued.ratio", "dram__bytes.sum.per_second"]
+MUL = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "nsecond": 1e-9, "usecond": 1e-6,
+       "msecond": 1e-3, "second": 1.0, "ns": 1e-9, "us": 1e-6, "ms": 1e-3, "s": 1.0}
+
+
+def num(v):
+    x, u = v.split()
+    return float(x.replace(",", "")) * MUL.get(u, 1.0)
 
 
 def full(rep):
@@ -68,26 +94,55 @@ def full(rep):
     return res
 
 
-summary = {"tag": tag, "launch_list": launch_list(),
-           "spmv_full": full("prof_spmv.ncu-rep"), "vector_full": full("prof_vec.ncu-rep")}
-json.dump(summary, open(os.path.join(P, f"{tag}_ncu_summary.json"), "w"), indent=1)
-# dram bytes per SpMV launch (for bench.py roofline.traffic)
-tr = {}
-for d in summary["spmv_full"]:
-    try:
-        rd, ru = d["dram__bytes_read.sum"].split()
-        wr, wu = d["dram__bytes_write.sum"].split()
-        mul = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}
-        tr = {"hpccg128": {"dram_bytes_per_launch": float(rd) * mul[ru] + float(wr) * mul[wu],
-                           "kernel": d["kernel"], "source": f"profiles/{tag}_ncu_summary.json"}}
-    except Exception:
-        pass
-if tr:
-    json.dump(tr, open(os.path.join(P, "spmv_traffic.json"), "w"), indent=1)
-for f in ["bench.json", "launches.csv", "smi.txt"]:
+def per_kernel(rows, n, nnz):
+    alg = {"spmv27x2_kernel": 12.0 * nnz + 16.0 * n, "cg_update1_kernel": 48.0 * n,
+           "cg_pupdate1_kernel": 24.0 * n}
+    out = {}
+    for d in rows:
+        name = next((k for k in alg if k in d["kernel"]), None)
+        if not name:
+            continue
+        dram = num(d["dram__bytes_read.sum"]) + num(d["dram__bytes_write.sum"])
+        t = num(d["gpu__time_duration.sum"])
+        rec = out.setdefault(name, {"kernel": d["kernel"], "launches": []})
+        rec["launches"].append({"dram_read": num(d["dram__bytes_read.sum"]),
+                                "dram_write": num(d["dram__bytes_write.sum"]),
+                                "dram_over_algorithmic": round(dram / alg[name], 4),
+                                "duration_us": round(t * 1e6, 2),
+                                "algorithmic_GBs": round(alg[name] / t / 1e9, 1),
+                                "l2_hit_pct": d.get("lts__t_sector_hit_rate.pct"),
+                                "dram_pct_of_peak": d.get("dram__throughput.avg.pct_of_peak_sustained_elapsed"),
+                                "registers": d.get("launch__registers_per_thread")})
+        rec["algorithmic_bytes"] = alg[name]
+    for rec in out.values():
+        ls = rec["launches"]
+        rec["dram_bytes_per_launch"] = sum(x["dram_read"] + x["dram_write"] for x in ls) / len(ls)
+        rec["dram_over_algorithmic"] = round(rec["dram_bytes_per_launch"] / rec["algorithmic_bytes"], 4)
+    return out
+
+
+nx, ny, nz = DIMS[W]
+n, nnz = nx * ny * nz, nnz_of(nx, ny, nz)
+summary = {"tag": tag, "workload": W, "n": n, "nnz": nnz, "launch_list": launch_list()}
+for cache in ("cold", "warm"):
+    rows = full(f"prof_{W}_{cache}.ncu-rep")
+    summary[f"{cache}_raw"] = rows
+    summary[cache] = per_kernel(rows, n, nnz)
+out = os.path.join(P, f"{tag}_ncu_{W}.json")
+json.dump(summary, open(out, "w"), indent=1)
+sp = summary.get("cold", {}).get("spmv27x2_kernel")
+if sp:
+    tp = os.path.join(P, "spmv_traffic.json")
+    tr = json.load(open(tp)) if os.path.exists(tp) else {}
+    tr[W] = {"dram_bytes_per_launch": sp["dram_bytes_per_launch"], "kernel": sp["kernel"],
+             "dram_over_algorithmic": sp["dram_over_algorithmic"], "cache": "cold (ncu default flush)",
+             "source": out}
+    json.dump(tr, open(tp, "w"), indent=1)
+for f in ["launches.csv", "smi.txt"]:
     if os.path.exists(os.path.join(G, f)):
-        with open(os.path.join(G, f)) as src, open(os.path.join(P, f"{tag}_{f}"), "w") as dst:
+        with open(os.path.join(G, f)) as src, open(os.path.join(P, f"{tag}_{W}_{f}"), "w") as dst:
             dst.write(src.read())
 print(json.dumps(summary["launch_list"][:8], indent=1))
-print(json.dumps(summary["spmv_full"], indent=1))
-print(json.dumps(summary["vector_full"], indent=1))
+for cache in ("cold", "warm"):
+    for k, v in summary[cache].items():
+        print(cache, k, v["dram_over_algorithmic"], [x["duration_us"] for x in v["launches"]])
