@@ -643,7 +643,9 @@ def run_ours(args):
                     peer=(world > 1 and transport == "peer"))
     sr = args.cg_variant == "sr"
     dia = args.spmv_format == "dia"
-    opts = [(H.HPCCG_OPT_CG_VARIANT, 1 if sr else 0), (H.HPCCG_OPT_SPMV_FORMAT, 1 if dia else 0)]
+    defer = not args.no_defer_x and not sr
+    opts = [(H.HPCCG_OPT_CG_VARIANT, 1 if sr else 0), (H.HPCCG_OPT_SPMV_FORMAT, 1 if dia else 0),
+            (H.HPCCG_OPT_DEFER_X, 1 if defer else 0)]
     mode_want = 1 if args.halo == "peer" else 2
 
     def setup_multirank(prob):
@@ -744,9 +746,11 @@ def run_ours(args):
                                      "97 % reads, so frac > 1 is expected -- frac_of_read_peak divides "
                                      "by a pure-read stream measured live here (our dot kernel, 2 x 4 GiB, best of 6)")
             # the fused vector kernels (north_star: >= 75 % of the 8 TB/s HBM peak on
-            # "SpMV and fused waxpby/ddot"): x/r update + r.r 48n B, p update 24n B
+            # "SpMV and fused waxpby/ddot"): x/r update + r.r 48n B, p update 24n B;
+            # with the deferred x update (default) r update + r.r 24n, x and p update 40n
             vec = {}
-            u_bytes, p_bytes = (72.0 * n, None) if sr else (48.0 * n, 24.0 * n)
+            u_bytes, p_bytes = ((72.0 * n, None) if sr else (24.0 * n, 40.0 * n) if defer
+                                else (48.0 * n, 24.0 * n))
             u_us = ev["update_ms"] * 1e3 / max(ev["niters"], 1)
             p_us = ev["pupdate_ms"] * 1e3 / max(ev["niters"], 1)
             for nm_k, by, us_ev, us_tr in (("update", u_bytes, u_us, trace and trace["update_us"]),
@@ -795,6 +799,8 @@ def run_ours(args):
                                     "global_nnz", "tol", "max_iter", "solve_graph", "l2", "gen_ms")}
         cfg.update({"iters": main["niters_per_step"], "parallelism": f"zslab{world}",
                     "cg_variant": "single-reduction (Chronopoulos-Gear, f2)" if sr else "HPCCG",
+                    "x_update": ("deferred into the next p update (HPCCG_OPT_DEFER_X 1): 12 nnz + 80n B "
+                                 "per iteration" if defer else "in the x/r update: 12 nnz + 88n B per iteration"),
                     "spmv_format": ("DIA-27 (columns from stencil offsets) -- EFFECTIVE, a different "
                                     "method (SURVEY 8(d): OUT)") if dia
                     else "ELL-27 (val[27][n] + col[27][n])",
@@ -1157,6 +1163,8 @@ def main():
     ap.add_argument("--spmv-format", choices=["ell", "dia"], default="ell",
                     help="HPCCG_OPT_SPMV_FORMAT: ELL-27 (default) or the DIA-27 reading (no col[]) -- "
                          "EFFECTIVE numbers of a different method (SURVEY 8(d): OUT), never the headline")
+    ap.add_argument("--no-defer-x", action="store_true",
+                    help="HPCCG_OPT_DEFER_X 0: update x in the x/r update (88n instead of 80n B/iteration)")
     ap.add_argument("--no-sub-configs", action="store_true",
                     help="skip the configs[1] / [0] / [3] sub-records of the CG line")
     ap.add_argument("--no-cpu-baseline", action="store_true")

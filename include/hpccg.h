@@ -137,6 +137,14 @@ extern "C" {
                                with its peers, so every later hpccg_solve of that problem
                                returns HPCCG_ECUDA at once (recreate the problem).  The value
                                is range-checked before any peer mapping is attempted. */
+#define HPCCG_OPT_DEFER_X 23 /* finisher-free HPCCG loop (single slab, or z-slabs with
+                               HALO_PEER 2): 1 (default) defers x += alpha p of iteration k
+                               into the p update of iteration k + 1 (which reads p_k anyway;
+                               cg_xfix_kernel applies the last one after the loop), so the
+                               x/r update moves 24n instead of 48n B and the p update 40n
+                               instead of 24n: 80n + 12 nnz B per iteration instead of 88n.
+                               Bitwise the same results (the same FMA on the same operands);
+                               0: x updated in the x/r update */
 #define HPCCG_OPT_PEER_TIMEOUT_MS 22 /* HALO_PEER waits: give up after this many milliseconds
                                (1 .. 3600000; default 30000 -- above any host-side skew
                                between ranks such as graph instantiation or a slow rank) */

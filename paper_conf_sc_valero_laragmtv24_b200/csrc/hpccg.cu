@@ -166,6 +166,7 @@ struct hpccg_problem {
     int opt_smem_threads = 0;          // on-chip solve CTA width: 0 auto, 256, 512
     int opt_peer = 0;                  // multi-slab: halo push + allreduce over peer memory
     int64_t opt_peer_timeout_ms = 30000;  // give up a peer-memory wait after this long
+    int opt_defer_x = 1;               // finisher-free loop: x update deferred into the p update
     std::vector<void *> ipc_opened;    // peers' buffers mapped with cudaIpcOpenMemHandle
     int last_persist_mode = 3;
     // graph of one CG iteration (per-iteration replay) ...
@@ -813,6 +814,22 @@ bool ff_path(const hpccg_problem *p) {
     return aligned16(s.r) && aligned16(s.p + s.plane) && aligned16(s.x) && aligned16(s.Ap);
 }
 
+// the deferred x update (HPCCG_OPT_DEFER_X) rides on the finisher-free loop
+bool defer_x_on(const hpccg_problem *p) { return p->opt_defer_x && ff_path(p); }
+
+// end of a solve on the finisher-free loop with the deferred x update: the
+// last iteration's x += alpha p (cg_xfix_kernel), every slab
+int enqueue_xfix(hpccg_problem *p) {
+    if (!defer_x_on(p)) return HPCCG_OK;
+    hpccg_ctx *ctx = p->ctx;
+    for (const Slab &s : p->slabs) {
+        launch_k(false, cg_xfix_kernel, dim3(wave_grid(s.n / 2 + 1, wave(ctx, cg_xfix_kernel))),
+                 ctx->stream, (int64_t)s.n, s.x, (const double *)(s.p + s.plane), (const CgScalars *)s.sc);
+        CHECK(check_launch(ctx));
+    }
+    return HPCCG_OK;
+}
+
 template <int kU>
 int enqueue_iteration_ff_u(hpccg_problem *p, bool timing, bool check, unsigned long long cond, int q) {
     hpccg_ctx *ctx = p->ctx;
@@ -851,6 +868,7 @@ int enqueue_iteration_ff_u(hpccg_problem *p, bool timing, bool check, unsigned l
             a.trace = s.trace_on ? s.trace : nullptr;
             a.trace_max = s.trace_max;
             a.rev = serpentine(p) & 1;
+            a.x = defer_x_on(p) ? s.x : nullptr;
             if (zs) {
                 a.t = s.ptab;
                 a.plane = s.plane;
@@ -899,6 +917,7 @@ int enqueue_iteration_ff_u(hpccg_problem *p, bool timing, bool check, unsigned l
         a.trace = s.trace_on ? s.trace : nullptr;
         a.trace_max = s.trace_max;
         a.t = zs ? s.ptab : nullptr;
+        a.defer_x = defer_x_on(p) ? 1 : 0;
         if (np <= kUpdSumMax) {
             a.pAp_parts = s.spmv_parts;
             a.n_parts = np;
@@ -1551,6 +1570,17 @@ int build_while_graph(hpccg_problem *p, int max_iter, double tol) {
     if (e != cudaSuccess) return bail(fail(HPCCG_ECUDA, "end capture (body): %s", cudaGetErrorString(e)));
     p->wgraph_init_kernels = l1 - l0;
     p->wgraph_body_kernels = (ctx->launches - l1) / U;
+    if (defer_x_on(p)) {  // after the WHILE node: the last iteration's deferred x update
+        const int64_t l2 = ctx->launches;
+        if (cudaStreamBeginCaptureToGraph(ctx->stream, g, &wnode, nullptr, 1,
+                                          cudaStreamCaptureModeThreadLocal) != cudaSuccess)
+            return bail(fail(HPCCG_ECUDA, "begin capture (tail): %s", cudaGetErrorString(cudaGetLastError())));
+        rc = enqueue_xfix(p);
+        e = cudaStreamEndCapture(ctx->stream, &gout);
+        if (rc != HPCCG_OK) return bail(rc);
+        if (e != cudaSuccess) return bail(fail(HPCCG_ECUDA, "end capture (tail): %s", cudaGetErrorString(e)));
+        p->wgraph_init_kernels += ctx->launches - l2;
+    }
     ctx->launches = l0;
     e = cudaGraphInstantiate(&p->wgraph, g, 0);
     cudaGraphDestroy(g);
@@ -2303,6 +2333,15 @@ int hpccg_set_option(hpccg_problem *p, int key, int64_t value) {
             if (value && p->ctx->mode != MODE_SINGLE && !p->slabs[0].ptab) CHECK(enable_peer(p));
             p->opt_peer = (int)value;
             return HPCCG_OK;
+        case HPCCG_OPT_DEFER_X:
+            if (value != 0 && value != 1) return fail(HPCCG_EINVAL, "defer x: 0 or 1");
+            if (p->opt_defer_x != (int)value) {  // graphs capture the choice
+                if (p->graph) cudaGraphExecDestroy(p->graph);
+                if (p->wgraph) cudaGraphExecDestroy(p->wgraph);
+                p->graph = p->wgraph = nullptr;
+            }
+            p->opt_defer_x = (int)value;
+            return HPCCG_OK;
         case HPCCG_OPT_PEER_TIMEOUT_MS:
             if (value < 1 || value > 3600000) return fail(HPCCG_EINVAL, "peer timeout: 1 .. 3600000 ms");
             p->opt_peer_timeout_ms = value;
@@ -2576,6 +2615,7 @@ int hpccg_solve(hpccg_problem *p, int max_iter, double tol, int *niters, double 
                 ++chunk;
             }
         }
+        CHECK(enqueue_xfix(p));
     }
     CU(cudaEventRecord(p->ev_t1, ctx->stream));
     CU(cudaStreamSynchronize(ctx->stream));

@@ -984,3 +984,57 @@ def test_peer_mode_nccl_one_rank():
             p.solve(m, 0.0)
             launches.append(p.stats()["kernel_launches"])
         assert launches[1] - launches[0] == 3 * 4
+
+
+# ------------------------------------------- deferred x update (DEFER_X)
+
+@pytest.mark.parametrize("dims,max_iter,tol", [((20, 30, 10), 150, 1e-12), ((31, 17, 9), 40, 0.0),
+                                               ((64, 64, 64), 150, 1e-12), ((33, 9, 3), 7, 0.0),
+                                               ((128, 128, 128), 21, 0.0)])
+def test_defer_x_bitwise_identical(ctx, dims, max_iter, tol):
+    """HPCCG_OPT_DEFER_X (x += alpha p moved into the next p update, the last
+    one into cg_xfix_kernel): the same FMA on the same operands, so x, niters
+    and normr are bit for bit those of the undeferred loop, in every launch
+    mode (while-graph, per-iteration graph, plain launches with events);
+    and within the north_star tolerance of the oracle."""
+    with H.Problem(ctx, *dims) as p:
+        p.set_option(H.HPCCG_OPT_PERSISTENT, 0)        # the graph / plain loops, not on-chip
+        outs = []
+        for defer in (0, 1):
+            p.set_option(H.HPCCG_OPT_DEFER_X, defer)
+            for mode in ("while", "graph", "timing"):
+                p.set_option(H.HPCCG_OPT_WHILE, 1 if mode == "while" else 0)
+                p.set_option(H.HPCCG_OPT_TIMING, 1 if mode == "timing" else 0)
+                p.set_vec(H.HPCCG_VEC_X, np.zeros(p.n))
+                r = p.solve(max_iter, tol)
+                outs.append((defer, mode, r["niters"], r["normr"], p.get_vec(H.HPCCG_VEC_X)))
+        p.set_option(H.HPCCG_OPT_TIMING, 0)
+        p.set_option(H.HPCCG_OPT_WHILE, 1)
+        for o in outs[1:]:
+            assert o[2:4] == outs[0][2:4], (o[:4], outs[0][:4])
+            np.testing.assert_array_equal(o[4], outs[0][4])
+        if p.n <= 300_000:
+            ref = oracle.generate(*dims)
+            oref = oracle.cg(ref, max_iter, tol)
+            assert abs(outs[-1][2] - oref["niters"]) <= 1
+            assert np.max(np.abs(outs[-1][4] - oref["x"])) <= CG_ATOL
+
+
+@pytest.mark.parametrize("P", [2, 3])
+def test_defer_x_fused_loopback_bitwise(P):
+    """The same on z-slabs with the exchange fused into the kernels (HALO_PEER 2)."""
+    dims = (16, 12, 6)
+    with H.Context(0, nranks=P, loopback=True) as c, H.Problem(c, *dims) as p:
+        p.set_option(H.HPCCG_OPT_HALO_PEER, 2)
+        res = []
+        for defer in (0, 1):
+            p.set_option(H.HPCCG_OPT_DEFER_X, defer)
+            p.set_vec(H.HPCCG_VEC_X, np.zeros(P * p.n))
+            r = p.solve(150, 1e-12)
+            res.append((r["niters"], r["normr"], p.get_vec(H.HPCCG_VEC_X)))
+        assert res[0][:2] == res[1][:2]
+        np.testing.assert_array_equal(res[0][2], res[1][2])
+        ref = oracle.generate(dims[0], dims[1], dims[2] * P)
+        oref = oracle.cg(ref, 150, 1e-12)
+        assert abs(res[1][0] - oref["niters"]) <= 1
+        assert np.max(np.abs(res[1][2] - oref["x"])) <= CG_ATOL
