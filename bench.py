@@ -385,6 +385,7 @@ def _stats_add(acc, prob, r):
     acc["pupdate_ms"] += st["pupdate_ms"]
     acc["niters"] += r["niters"]
     acc["graph_mode"] = st["graph_mode"]
+    acc["x_deferred"] = bool(st["x_deferred"])
 
 
 class CgRunner:
@@ -560,7 +561,7 @@ def measure_workload(H, D, ctx, stream, world, rank, local, coll_dev, name, step
     out.update({"value": round(val, 3), "unit": "GFLOP/s", "steps": steps, "warmup": warmup,
                 "ms_per_step": round(ms_max / steps, 4),
                 "t_iter_us": round(ms_max * 1e3 / max(main["niters"], 1), 3),
-                "niters_per_step": main["niters"] // steps,
+                "niters_per_step": main["niters"] // steps, "x_deferred": main.get("x_deferred"),
                 "max_abs_x_minus_1": main["err"], "normr": main["r"]["normr"],
                 "solve_graph": {5: "on-chip cluster kernel", 4: "one-cluster persistent kernel",
                                 3: "cooperative persistent kernel", 2: "while-graph",
@@ -643,9 +644,9 @@ def run_ours(args):
                     peer=(world > 1 and transport == "peer"))
     sr = args.cg_variant == "sr"
     dia = args.spmv_format == "dia"
-    defer = not args.no_defer_x and not sr
-    opts = [(H.HPCCG_OPT_CG_VARIANT, 1 if sr else 0), (H.HPCCG_OPT_SPMV_FORMAT, 1 if dia else 0),
-            (H.HPCCG_OPT_DEFER_X, 1 if defer else 0)]
+    opts = [(H.HPCCG_OPT_CG_VARIANT, 1 if sr else 0), (H.HPCCG_OPT_SPMV_FORMAT, 1 if dia else 0)]
+    if args.no_defer_x:
+        opts.append((H.HPCCG_OPT_DEFER_X, 0))
     mode_want = 1 if args.halo == "peer" else 2
 
     def setup_multirank(prob):
@@ -683,6 +684,7 @@ def run_ours(args):
                             args.steps, args.warmup, events=True, trace=not sr, clocks=True,
                             opts=opts, setup=setup_multirank)
     n, nnz_local = main["_n"], main["_nnz_local"]
+    defer = bool(main.get("x_deferred"))
     ev, trace = main["_ev"], main["_trace"]
     # per-rank record of what actually ran (transport, exchange mode, NCCL view)
     cinfo = ctx.info()
@@ -799,8 +801,9 @@ def run_ours(args):
                                     "global_nnz", "tol", "max_iter", "solve_graph", "l2", "gen_ms")}
         cfg.update({"iters": main["niters_per_step"], "parallelism": f"zslab{world}",
                     "cg_variant": "single-reduction (Chronopoulos-Gear, f2)" if sr else "HPCCG",
-                    "x_update": ("deferred into the next p update (HPCCG_OPT_DEFER_X 1): 12 nnz + 80n B "
-                                 "per iteration" if defer else "in the x/r update: 12 nnz + 88n B per iteration"),
+                    "x_update": ("deferred into the next p update (HPCCG_OPT_DEFER_X, auto: the CG vectors "
+                                 "exceed L2): 12 nnz + 80n B per iteration" if defer
+                                 else "in the x/r update: 12 nnz + 88n B per iteration"),
                     "spmv_format": ("DIA-27 (columns from stencil offsets) -- EFFECTIVE, a different "
                                     "method (SURVEY 8(d): OUT)") if dia
                     else "ELL-27 (val[27][n] + col[27][n])",

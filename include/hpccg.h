@@ -138,13 +138,15 @@ extern "C" {
                                returns HPCCG_ECUDA at once (recreate the problem).  The value
                                is range-checked before any peer mapping is attempted. */
 #define HPCCG_OPT_DEFER_X 23 /* finisher-free HPCCG loop (single slab, or z-slabs with
-                               HALO_PEER 2): 1 (default) defers x += alpha p of iteration k
+                               HALO_PEER 2): 1 defers x += alpha p of iteration k
                                into the p update of iteration k + 1 (which reads p_k anyway;
                                cg_xfix_kernel applies the last one after the loop), so the
                                x/r update moves 24n instead of 48n B and the p update 40n
                                instead of 24n: 80n + 12 nnz B per iteration instead of 88n.
                                Bitwise the same results (the same FMA on the same operands);
-                               0: x updated in the x/r update */
+                               0: x updated in the x/r update; -1 (default): auto, 1 when the
+                               CG vectors exceed L2 (256^3: 989 vs 1005 us/iteration; at 128^3
+                               the vectors are L2-resident and 0 is 0.4 % faster) */
 #define HPCCG_OPT_PEER_TIMEOUT_MS 22 /* HALO_PEER waits: give up after this many milliseconds
                                (1 .. 3600000; default 30000 -- above any host-side skew
                                between ranks such as graph instantiation or a slow rank) */
@@ -200,6 +202,7 @@ typedef struct hpccg_stats {
     int64_t graph_mode;     /* 5 shared-memory-resident cluster kernel, 4 one-cluster
                                persistent kernel, 3 cooperative-grid persistent kernel,
                                2 while-graph, 1 per-iteration graph, 0 plain */
+    int64_t x_deferred;     /* 1: the solve ran with the deferred x update (HPCCG_OPT_DEFER_X) */
 } hpccg_stats;
 
 HPCCG_API const char *hpccg_strerror(int code);

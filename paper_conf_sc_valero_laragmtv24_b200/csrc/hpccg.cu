@@ -166,7 +166,7 @@ struct hpccg_problem {
     int opt_smem_threads = 0;          // on-chip solve CTA width: 0 auto, 256, 512
     int opt_peer = 0;                  // multi-slab: halo push + allreduce over peer memory
     int64_t opt_peer_timeout_ms = 30000;  // give up a peer-memory wait after this long
-    int opt_defer_x = 1;               // finisher-free loop: x update deferred into the p update
+    int opt_defer_x = -1;              // finisher-free loop: x update deferred into the p update (-1 auto)
     std::vector<void *> ipc_opened;    // peers' buffers mapped with cudaIpcOpenMemHandle
     int last_persist_mode = 3;
     // graph of one CG iteration (per-iteration replay) ...
@@ -815,7 +815,12 @@ bool ff_path(const hpccg_problem *p) {
 }
 
 // the deferred x update (HPCCG_OPT_DEFER_X) rides on the finisher-free loop
-bool defer_x_on(const hpccg_problem *p) { return p->opt_defer_x && ff_path(p); }
+// (auto: when the CG vectors exceed L2 -- measured 256^3 989 vs 1005 us/iter,
+// 128^3, vectors L2-resident, 115.1 vs 114.7: the x traffic then costs nothing)
+bool defer_x_on(const hpccg_problem *p) {
+    const bool on = p->opt_defer_x < 0 ? p->slabs[0].arena_bytes > ((size_t)126 << 20) : p->opt_defer_x != 0;
+    return on && ff_path(p);
+}
 
 // end of a solve on the finisher-free loop with the deferred x update: the
 // last iteration's x += alpha p (cg_xfix_kernel), every slab
@@ -2334,7 +2339,7 @@ int hpccg_set_option(hpccg_problem *p, int key, int64_t value) {
             p->opt_peer = (int)value;
             return HPCCG_OK;
         case HPCCG_OPT_DEFER_X:
-            if (value != 0 && value != 1) return fail(HPCCG_EINVAL, "defer x: 0 or 1");
+            if (value < -1 || value > 1) return fail(HPCCG_EINVAL, "defer x: -1 (auto), 0 or 1");
             if (p->opt_defer_x != (int)value) {  // graphs capture the choice
                 if (p->graph) cudaGraphExecDestroy(p->graph);
                 if (p->wgraph) cudaGraphExecDestroy(p->wgraph);
@@ -2646,6 +2651,7 @@ int hpccg_solve(hpccg_problem *p, int max_iter, double tol, int *niters, double 
     st.kernel_launches = ctx->launches - l0;
     st.l2_persist_bytes = (int64_t)l2win.kept;
     st.graph_mode = use_persist ? p->last_persist_mode : (use_while ? 2 : (use_graph ? 1 : 0));
+    st.x_deferred = !use_persist && defer_x_on(p);
     p->stats = st;
     if (niters) *niters = hs.niters;
     if (normr) *normr = hs.normr;

@@ -56,7 +56,7 @@ class hpccg_stats(ctypes.Structure):
                 ("allreduce_ms", ctypes.c_double), ("exchange_ms", ctypes.c_double),
                 ("spmv_launches", ctypes.c_int64), ("iterations", ctypes.c_int64),
                 ("kernel_launches", ctypes.c_int64), ("l2_persist_bytes", ctypes.c_int64),
-                ("graph_mode", ctypes.c_int64)]
+                ("graph_mode", ctypes.c_int64), ("x_deferred", ctypes.c_int64)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}
