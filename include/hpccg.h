@@ -89,8 +89,10 @@ extern "C" {
                                (the while-graph is faster above that); k >= 0:
                                when nrow_local <= k */
 #define HPCCG_OPT_SMEM_SOLVE 13 /* 1 (default): a persistent solve whose rows fit in the
-                               shared memory of one 16-CTA cluster (~9.9k rows) keeps the whole
-                               problem on chip (distributed shared memory gathers); 0: off */
+                               shared memory of one 16-CTA cluster keeps the whole problem on
+                               chip (distributed shared memory gathers): ~9.9k rows with the ELL
+                               slice (HPCCG_OPT_SPMV_FORMAT 0), ~14k rows under format 1 (no column
+                               slice); 0: off */
 #define HPCCG_OPT_TRACE 14  /* k > 0: record, for the first k iterations, each CG kernel's
                                first-block start and last-block end on the device clock
                                (%globaltimer; works inside graphs); read with
@@ -174,8 +176,13 @@ extern "C" {
                                val[27][n] + col[27][n] (12 B per slot); 1 DIA-27, val only:
                                slot s's column is formed from its stencil offset
                                (s/9-1)*nx*ny + (s/3%3-1)*nx + (s%3-1), a 0.0 value selecting
-                               the padding column -- bitwise identical results (8 B per
-                               slot).  Valid because hpccg_generate is the only source of
+                               the padding column -- bitwise identical SpMV results (8 B per
+                               slot).  hpccg_solve's bits are format-invariant only where both
+                               formats take the same solve path: between ~9.9k and ~14k rows
+                               format 1 fits the on-chip cluster solve and format 0 takes the
+                               while-graph, whose reduction order differs (last bits of niters /
+                               normr / x; both within the oracle tolerances).  Format 1 is an
+                               "effective" reading (a different method per SURVEY 8(d)), opt-in.  Valid because hpccg_generate is the only source of
                                A (A: diag 27, -1 per existing neighbour, BJ:north_star).
                                The on-chip (shared-memory) solve drops its column slice
                                under 1 when the ELL slice does not fit (more rows on chip);
