@@ -149,6 +149,19 @@ extern "C" {
                                0: x updated in the x/r update; -1 (default): auto, 1 when the
                                CG vectors exceed L2 (256^3: 989 vs 1005 us/iteration; at 128^3
                                the vectors are L2-resident and 0 is 0.4 % faster) */
+#define HPCCG_OPT_FUSE_PSPMV 24 /* single slab, finisher-free loop: the p update and the
+                               SpMV of an iteration as ONE pipelined kernel (cg_pspmv_kernel:
+                               chunks of 512 rows taken in launch order; each block updates p
+                               a fixed lead of chunks ahead and publishes it, then waits for
+                               the <= 9 chunks its gathers read) -- p is gathered from L2
+                               right after it is written: 12 nnz + 72n B per iteration with
+                               the deferred x update (ncu at 256^3: 6.23 GB DRAM per launch,
+                               p gathered from L2).  Bitwise the same results.  0 (default)
+                               off -- measured no faster: the mixed read/write stream runs at
+                               6.84 TB/s where the plain SpMV reaches 7.11, which eats the
+                               8n B saved (256^3: 977 vs 978 us/iteration; 128^3 122 vs 115);
+                               1 on, -1 auto (on when the CG vectors exceed L2) */
+#define HPCCG_OPT_PS_LEAD 25 /* its production lead in chunks (0 default: plane/512 + 8) */
 #define HPCCG_OPT_PEER_TIMEOUT_MS 22 /* HALO_PEER waits: give up after this many milliseconds
                                (1 .. 3600000; default 30000 -- above any host-side skew
                                between ranks such as graph instantiation or a slow rank) */
@@ -210,6 +223,7 @@ typedef struct hpccg_stats {
                                persistent kernel, 3 cooperative-grid persistent kernel,
                                2 while-graph, 1 per-iteration graph, 0 plain */
     int64_t x_deferred;     /* 1: the solve ran with the deferred x update (HPCCG_OPT_DEFER_X) */
+    int64_t ps_fused;       /* 1: the solve ran the fused p update + SpMV (HPCCG_OPT_FUSE_PSPMV) */
 } hpccg_stats;
 
 HPCCG_API const char *hpccg_strerror(int code);

@@ -129,6 +129,11 @@ struct Slab {
     int early_trigger = 1;      // HPCCG_OPT_PDL 1: SpMV triggers its successor early
     int nx = 0;                 // grid row stride (DIA-27 column formation)
     int dia = 0;                // HPCCG_OPT_SPMV_FORMAT 1: DIA-27 SpMV (col[] not read)
+    // HPCCG_OPT_FUSE_PSPMV: ticket counter, error word, per-chunk flags
+    unsigned char *ps_mem = nullptr;
+    unsigned *ps_ticket = nullptr;
+    unsigned long long *ps_flags = nullptr;
+    int *ps_err = nullptr;
 };
 
 struct TimedOp {
@@ -167,6 +172,8 @@ struct hpccg_problem {
     int opt_peer = 0;                  // multi-slab: halo push + allreduce over peer memory
     int64_t opt_peer_timeout_ms = 30000;  // give up a peer-memory wait after this long
     int opt_defer_x = -1;              // finisher-free loop: x update deferred into the p update (-1 auto)
+    int opt_fuse_ps = 0;               // p update + SpMV in one pipelined kernel (-1 auto, 0 off, 1 on)
+    int opt_ps_lead = 0;               // its production lead in chunks (0: plane / 512 + 8)
     std::vector<void *> ipc_opened;    // peers' buffers mapped with cudaIpcOpenMemHandle
     int last_persist_mode = 3;
     // graph of one CG iteration (per-iteration replay) ...
@@ -835,6 +842,75 @@ int enqueue_xfix(hpccg_problem *p) {
     return HPCCG_OK;
 }
 
+// HPCCG_OPT_FUSE_PSPMV: single slab on the finisher-free loop, 2 rows per
+// thread, a 128-B-aligned chunk layout (a line of p never spans two chunks).
+// The lead (chunks between a block's production and its SpMV) must exceed
+// the gather reach (plane + nx + 1 rows); past that, more lead = more time
+// for a chunk's release to land before anyone needs it.
+int64_t ps_lead(const hpccg_problem *p) {
+    const Slab &s = p->slabs[0];
+    const int64_t reach = (s.plane + s.nx + 1) / kPsRows + 2;
+    return std::max<int64_t>(p->opt_ps_lead > 0 ? p->opt_ps_lead : reach + 128, reach + 1);
+}
+
+bool fuse_ps_on(hpccg_problem *p) {
+    if (p->opt_fuse_ps == 0 || p->ctx->mode != MODE_SINGLE || p->opt_variant != 0 || !ff_path(p)) return false;
+    const Slab &s = p->slabs[0];
+    if (s.dia || (s.n & 1) || (s.plane & 15) || ((uintptr_t)(s.p + s.plane) & 127)) return false;
+    if (spmv_rows_per_thread(p->opt_rows, spmv_args(s, s.p, s.Ap), 0, 0) != 2) return false;
+    if (p->opt_fuse_ps < 0 && s.arena_bytes <= ((size_t)126 << 20)) return false;  // auto: vectors > L2
+    return s.ps_mem != nullptr;  // allocated when the option is set (never during a graph capture)
+}
+
+int alloc_zero(void **ptr, size_t bytes);
+
+int ps_alloc(Slab &s) {
+    if (s.ps_mem) return HPCCG_OK;
+    const int64_t nch = cdiv(s.n, kPsRows);
+    const size_t bytes = 256 + sizeof(unsigned long long) * (size_t)nch;
+    CHECK(alloc_zero((void **)&s.ps_mem, bytes));
+    s.ps_ticket = (unsigned *)s.ps_mem;
+    s.ps_err = (int *)(s.ps_mem + 64);
+    s.ps_flags = (unsigned long long *)(s.ps_mem + 256);
+    return HPCCG_OK;
+}
+
+// rows [row0, row0 + nrows) that the prologue p update handles: the first
+// `lead` chunk positions (the last chunks when the SpMV walks backwards)
+void ps_prologue_rows(const hpccg_problem *p, int64_t *row0, int64_t *nrows) {
+    const Slab &s = p->slabs[0];
+    const int64_t nch = cdiv(s.n, kPsRows), lead = std::min<int64_t>(ps_lead(p), nch);
+    const bool rev = (serpentine(p) >> 1) & 1;
+    *row0 = rev ? (nch - lead) * kPsRows : 0;
+    *nrows = rev ? s.n - *row0 : std::min<int64_t>(lead * kPsRows, s.n);
+}
+
+int launch_pspmv(hpccg_problem *p, const Slab &s, int q) {
+    PsArgs a{};
+    a.n = s.n;
+    a.plane = s.plane;
+    a.nchunks = cdiv(s.n, kPsRows);
+    a.nx = s.nx;
+    a.lead = (int)ps_lead(p);
+    a.rev = (serpentine(p) >> 1) & 1;
+    a.q = q;
+    a.val = s.val;
+    a.col = s.col;
+    a.p = s.p;
+    a.r = s.r;
+    a.x = defer_x_on(p) ? s.x : nullptr;
+    a.Ap = s.Ap;
+    a.parts = s.spmv_parts;
+    a.sc = s.sc;
+    a.ticket = s.ps_ticket;
+    a.flags = s.ps_flags;
+    a.trace = s.trace_on ? s.trace : nullptr;
+    a.trace_max = s.trace_max;
+    a.err = s.ps_err;
+    launch_k(p->opt_pdl != 0, cg_pspmv_kernel, dim3((unsigned)a.nchunks), p->ctx->stream, a);
+    return check_launch(p->ctx);
+}
+
 template <int kU>
 int enqueue_iteration_ff_u(hpccg_problem *p, bool timing, bool check, unsigned long long cond, int q) {
     hpccg_ctx *ctx = p->ctx;
@@ -850,12 +926,36 @@ int enqueue_iteration_ff_u(hpccg_problem *p, bool timing, bool check, unsigned l
     const int pg = vec_grid(ctx, pup, cdiv(s0.n, 2 * kU), p->opt_vec_waves, 0x7fffffff);
     // loopback: every slab's post ahead of every slab's collect (one stream)
     const bool pre = zs && ctx->mode == MODE_LOOPBACK;
+    const bool fuse = !zs && fuse_ps_on(p);
     auto post = [&](const Slab &s, const double *parts, unsigned n, int q) {
         launch_k(pdl, fused_post_kernel, dim3(1), ctx->stream, parts, n, (const double *)&s.sc->pAp,
                  (const PeerTab *)s.ptab, (const CgScalars *)s.sc, q);
         return check_launch(ctx);
     };
-    {
+    if (fuse) {  // the prologue p update (first `lead` chunks), then p update + SpMV in one kernel
+        {
+            PhaseTimer t(p, ctx->stream, PH_PUPDATE, timing);
+            int64_t row0, nrows;
+            ps_prologue_rows(p, &row0, &nrows);
+            Pupd1Args a{};
+            a.post = 1;
+            a.n = nrows;
+            a.r = s0.r + row0;
+            a.p = s0.p + s0.plane + row0;
+            a.rr_parts = s0.red.partials;
+            a.n_rr = (unsigned)ug;
+            a.sc = s0.sc;
+            a.q = q;
+            a.trace = s0.trace_on ? s0.trace : nullptr;
+            a.trace_max = s0.trace_max;
+            a.x = defer_x_on(p) ? s0.x + row0 : nullptr;
+            const int gp = vec_grid(ctx, pup, cdiv(nrows, 2 * kU), p->opt_vec_waves, 0x7fffffff);
+            launch_k(pdl, pup, dim3(gp), ctx->stream, a);
+            CHECK(check_launch(ctx));
+        }
+        PhaseTimer t(p, ctx->stream, PH_SPMV, timing);
+        CHECK(launch_pspmv(p, s0, q));
+    } else {
         PhaseTimer t(p, ctx->stream, PH_PUPDATE, timing);
         if (pre)
             for (const Slab &s : p->slabs) CHECK(post(s, s.red.partials, (unsigned)ug, 0));
@@ -888,7 +988,9 @@ int enqueue_iteration_ff_u(hpccg_problem *p, bool timing, bool check, unsigned l
         }
     }
     unsigned np = 0;
-    if (zs) {
+    if (fuse) {
+        np = (unsigned)cdiv(s0.n, kPsRows);
+    } else if (zs) {
         PhaseTimer t(p, ctx->stream, PH_SPMV, timing);
         for (const Slab &s : p->slabs) CHECK(launch_spmv_fused(p, s, check, &np));
     } else {
@@ -923,6 +1025,7 @@ int enqueue_iteration_ff_u(hpccg_problem *p, bool timing, bool check, unsigned l
         a.trace_max = s.trace_max;
         a.t = zs ? s.ptab : nullptr;
         a.defer_x = defer_x_on(p) ? 1 : 0;
+        a.late_p = fuse ? 1 : 0;
         if (np <= kUpdSumMax) {
             a.pAp_parts = s.spmv_parts;
             a.n_parts = np;
@@ -1630,6 +1733,7 @@ void free_slab(Slab &s) {
     cudaFree(s.psync);
     cudaFree(s.ptab);
     cudaFree(s.trace);
+    cudaFree(s.ps_mem);
     s = Slab{};
 }
 
@@ -2338,6 +2442,23 @@ int hpccg_set_option(hpccg_problem *p, int key, int64_t value) {
             if (value && p->ctx->mode != MODE_SINGLE && !p->slabs[0].ptab) CHECK(enable_peer(p));
             p->opt_peer = (int)value;
             return HPCCG_OK;
+        case HPCCG_OPT_FUSE_PSPMV:
+            if (value < -1 || value > 1) return fail(HPCCG_EINVAL, "fuse pspmv: -1 (auto), 0 or 1");
+            if (p->opt_fuse_ps != (int)value) {
+                if (p->graph) cudaGraphExecDestroy(p->graph);
+                if (p->wgraph) cudaGraphExecDestroy(p->wgraph);
+                p->graph = p->wgraph = nullptr;
+            }
+            p->opt_fuse_ps = (int)value;
+            if (value != 0 && p->ctx->mode == MODE_SINGLE) CHECK(ps_alloc(p->slabs[0]));
+            return HPCCG_OK;
+        case HPCCG_OPT_PS_LEAD:
+            if (value < 0 || value > (1 << 20)) return fail(HPCCG_EINVAL, "ps lead: 0 (auto) .. 2^20 chunks");
+            if (p->graph) cudaGraphExecDestroy(p->graph);
+            if (p->wgraph) cudaGraphExecDestroy(p->wgraph);
+            p->graph = p->wgraph = nullptr;
+            p->opt_ps_lead = (int)value;
+            return HPCCG_OK;
         case HPCCG_OPT_DEFER_X:
             if (value < -1 || value > 1) return fail(HPCCG_EINVAL, "defer x: -1 (auto), 0 or 1");
             if (p->opt_defer_x != (int)value) {  // graphs capture the choice
@@ -2627,6 +2748,15 @@ int hpccg_solve(hpccg_problem *p, int max_iter, double tol, int *niters, double 
     CU(cudaGetLastError());
     l2win.release();
     if (peer_on(p)) CHECK(peer_check_error(p, "hpccg_solve"));
+    for (const Slab &sl : p->slabs)
+        if (sl.ps_err) {
+            int e = 0;
+            CU(cudaMemcpy(&e, sl.ps_err, sizeof e, cudaMemcpyDeviceToHost));
+            if (e) {
+                CU(cudaMemset(sl.ps_err, 0, sizeof e));
+                return fail(HPCCG_ECUDA, "fused p update + SpMV: a chunk wait gave up after 5 s (residency)");
+            }
+        }
 
     CgScalars hs;
     CU(cudaMemcpy(&hs, p->slabs[0].sc, sizeof hs, cudaMemcpyDeviceToHost));
@@ -2652,6 +2782,7 @@ int hpccg_solve(hpccg_problem *p, int max_iter, double tol, int *niters, double 
     st.l2_persist_bytes = (int64_t)l2win.kept;
     st.graph_mode = use_persist ? p->last_persist_mode : (use_while ? 2 : (use_graph ? 1 : 0));
     st.x_deferred = !use_persist && defer_x_on(p);
+    st.ps_fused = !use_persist && fuse_ps_on(p);
     p->stats = st;
     if (niters) *niters = hs.niters;
     if (normr) *normr = hs.normr;

@@ -105,6 +105,34 @@ __device__ __forceinline__ int2 ld_stream2(const int *ptr, uint64_t pol) {
     return v;
 }
 
+// Loads of data the PREDECESSOR grid wrote (device scalars, reduction
+// partials), for use after pdl_wait(): plain weak ld.global (L1-cacheable, so
+// one L2 request per SM still serves every warp), NOT the read-only path.  An
+// ld.global.nc promises the data is constant for the kernel's lifetime, and
+// ptxas uses that promise to hoist it above griddepcontrol.wait (SASS ACQBULK)
+// -- seen in the fused p update + SpMV kernel, where a stale run flag / scalar
+// read raced the predecessor; tests/test_abi_cpu.py checks every kernel's SASS.
+__device__ __forceinline__ double ldg_o(const double *p) {
+    double v;
+    asm volatile("ld.global.f64 %0, [%1];" : "=d"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ int ldg_o(const int *p) {
+    int v;
+    asm volatile("ld.global.s32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ double2 ldg_o2(const double2 *p) {
+    double2 v;
+    asm volatile("ld.global.v2.f64 {%0, %1}, [%2];" : "=d"(v.x), "=d"(v.y) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ unsigned long long ldg_o(const unsigned long long *p) {
+    unsigned long long v;
+    asm volatile("ld.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+
 // Programmatic dependent launch (PDL): a kernel launched with the
 // programmatic-stream-serialization attribute may start while its
 // predecessor drains; pdl_wait() (griddepcontrol.wait) blocks until the
@@ -522,8 +550,8 @@ __device__ __forceinline__ int64_t spmv_bid(const SpmvArgs &a) {
 template <int kDots, bool kCheck>
 __device__ __forceinline__ int spmv_done(const SpmvArgs &a) {
     if (!kCheck || kDots == 0) return 0;
-    if (kDots == 2) return !__ldg(&a.sc->run_q[a.sr_q]);
-    return __ldg(&a.sc->done);
+    if (kDots == 2) return !ldg_o(&a.sc->run_q[a.sr_q]);
+    return ldg_o(&a.sc->done);
 }
 
 // Block sums of two values in a fixed order; valid in thread 0.
@@ -604,7 +632,7 @@ __global__ void __launch_bounds__(kBlock, kMinB) spmv27_kernel(SpmvArgs a) {
             if (g == 0) {
                 pdl_wait();
                 if (a.early_trigger) pdl_trigger();
-                if (kDot && a.trace) trace_mark(a.trace, a.trace_max, __ldg(&a.sc->k), 1, false);
+                if (kDot && a.trace) trace_mark(a.trace, a.trace_max, ldg_o(&a.sc->k), 1, false);
                 done = spmv_done<kDots, kCheck>(a);
                 if (done) return;  // uniform over the grid, before any store
             }
@@ -636,7 +664,7 @@ __global__ void __launch_bounds__(kBlock, kMinB) spmv27_kernel(SpmvArgs a) {
         spmv_sr_partials(a, dg, d);
         return;
     }
-    if (kDot && a.trace) trace_mark(a.trace, a.trace_max, __ldg(&a.sc->k), 1, true);
+    if (kDot && a.trace) trace_mark(a.trace, a.trace_max, ldg_o(&a.sc->k), 1, true);
     if (kDot) {
         if (a.parts_only) {  // block partial only; the update kernel sums them
             __shared__ double shp[32];
@@ -667,7 +695,7 @@ __device__ __forceinline__ void fused_halo_wait(const SpmvArgs &a, int64_t first
     if (threadIdx.x == 0) {
         const PeerTab *t = a.fpeer;
         // iteration k's SpMV: niters = k (written by the p update / f2 update)
-        const unsigned long long tg = ftag(__ldg(&a.sc->epoch), (unsigned long long)__ldg(&a.sc->niters));
+        const unsigned long long tg = ftag(ldg_o(&a.sc->epoch), (unsigned long long)ldg_o(&a.sc->niters));
         if (first < a.plane && t->rank > 0)
             spin_until(&t->mine->fflag_from_lo, tg, t->mine, PEER_WAIT_HALO_LO, t->rank - 1);
         if (last >= a.stride - a.plane && t->rank < t->nranks - 1)
@@ -740,7 +768,7 @@ __device__ __forceinline__ void spmv27x2_body(const SpmvArgs &a, int64_t row, in
             if (g == 0) {
                 pdl_wait();
                 if (a.early_trigger) pdl_trigger();
-                if (kDot && a.trace) trace_mark(a.trace, a.trace_max, __ldg(&a.sc->k), 1, false);
+                if (kDot && a.trace) trace_mark(a.trace, a.trace_max, ldg_o(&a.sc->k), 1, false);
                 done = spmv_done<kDots, kCheck>(a);
                 if (done) return;  // uniform over the grid, before any store
             }
@@ -791,7 +819,7 @@ __device__ __forceinline__ void spmv27x2_body(const SpmvArgs &a, int64_t row, in
         spmv_sr_partials(a, dg, d);
         return;
     }
-    if (kDot && a.trace) trace_mark(a.trace, a.trace_max, __ldg(&a.sc->k), 1, true);
+    if (kDot && a.trace) trace_mark(a.trace, a.trace_max, ldg_o(&a.sc->k), 1, true);
     if (kDot) {
         if (a.parts_only) {  // block partial only; the update kernel sums them
             __shared__ double shp[32];
@@ -839,7 +867,7 @@ __global__ void __launch_bounds__(kBlock, kDia ? kDiaMinB : 4) spmv27x2_kernel(S
             // niters / done are written by the predecessor (PDL): wait for it
             // first (the body's second griddepcontrol.wait is a no-op)
             pdl_wait();
-            if (kCheck && __ldg(&a.sc->done)) return;  // uniform exit
+            if (kCheck && ldg_o(&a.sc->done)) return;  // uniform exit
             fused_halo_wait(a, first, last);
         }
     }
@@ -851,11 +879,11 @@ __global__ void __launch_bounds__(kBlock, kDia ? kDiaMinB : 4) spmv27x2_kernel(S
 }
 
 // ------------------------------------------------ streaming vector kernels
-// Device scalars are read with ld.global.nc (__ldg): they are constant for the
-// kernel's lifetime, and the read-only path lets one L2 request per SM serve
-// every warp.  (Plain volatile reads from every warp all hit the one L2 slice
-// that owns the scalar line and serialise there -- measured: 2x slower
-// vector kernels.)
+// Device scalars are read with weak L1-cacheable loads after the PDL wait
+// (ldg_o): one L2 request per SM serves every warp.  (Volatile reads from
+// every warp all hit the one L2 slice that owns the scalar line and serialise
+// there -- measured: 2x slower vector kernels; and the read-only path may be
+// hoisted above the wait, see ldg_o.)
 // Grids walk the vectors in 16-B double2 units, one unit per thread per trip;
 // by default one thread per unit (a full, non-persistent grid: 2048 resident
 // threads per SM keep enough loads in flight), or a persistent grid of
@@ -877,12 +905,12 @@ __global__ void __launch_bounds__(kBlock) cg_pupdate_kernel(int64_t n, const dou
                                                            int trace_max) {
     pdl_wait();
     pdl_trigger();
-    const int ktr = trace ? __ldg(&sc->k) : 0;
+    const int ktr = trace ? ldg_o(&sc->k) : 0;
     trace_mark(trace, trace_max, ktr, 0, false);
     // `done` is tested after each trip's loads (never in front of them)
-    const int done = kCheck ? __ldg(&sc->done) : 0;
-    const bool first = (__ldg(&sc->k) == 1);
-    const double beta = first ? 0.0 : __ldg(&sc->rr_cur) / __ldg(&sc->rr_prev);
+    const int done = kCheck ? ldg_o(&sc->done) : 0;
+    const bool first = (ldg_o(&sc->k) == 1);
+    const double beta = first ? 0.0 : ldg_o(&sc->rr_cur) / ldg_o(&sc->rr_prev);
     const int64_t tid = gtid(), nth = gnth();
     if (kVec) {
         const int64_t nv = n >> 1;
@@ -969,7 +997,7 @@ __global__ void __launch_bounds__(1024, 1) cg_pap_finish_kernel(const double *pa
     for (; i + 23u * 1024u < n_parts; i += 24u * 1024u) {
         double v[24];
 #pragma unroll
-        for (int u = 0; u < 24; ++u) v[u] = __ldg(parts + i + u * 1024u);
+        for (int u = 0; u < 24; ++u) v[u] = ldg_o(parts + i + u * 1024u);
 #pragma unroll
         for (int t = 0; t < 3; ++t)
 #pragma unroll
@@ -995,12 +1023,12 @@ __global__ void __launch_bounds__(kBlock) cg_update_kernel(UpdArgs a) {
     CgScalars *sc = a.sc;
     pdl_wait();
     pdl_trigger();
-    const int ktr = a.trace ? __ldg(&sc->k) : 0;
+    const int ktr = a.trace ? ldg_o(&sc->k) : 0;
     trace_mark(a.trace, a.trace_max, ktr, 2, false);
     // `done` is tested after each trip's loads (never in front of them); it
     // is uniform over the grid, so every block leaves before the reduction.
-    const int done = kCheck ? __ldg(&sc->done) : 0;
-    const double rtrans = __ldg(&sc->rr_cur);
+    const int done = kCheck ? ldg_o(&sc->done) : 0;
+    const double rtrans = ldg_o(&sc->rr_cur);
     double pAp;
     if (a.pAp_parts) {
         // every block sums the SpMV's partials in the same fixed order, so
@@ -1013,7 +1041,7 @@ __global__ void __launch_bounds__(kBlock) cg_update_kernel(UpdArgs a) {
         __syncthreads();
         pAp = shq[31];
     } else {
-        pAp = __ldg(&sc->pAp);
+        pAp = ldg_o(&sc->pAp);
     }
     const bool stop = (rtrans == 0.0) || (pAp == 0.0);  // A11
     const double alpha = stop ? 0.0 : rtrans / pAp;
@@ -1160,11 +1188,11 @@ __device__ __forceinline__ double sum_parts_fixed(const double *parts, unsigned 
     for (; i + 7u * kBlock < n; i += 8u * kBlock) {
         double v[8];
 #pragma unroll
-        for (int u = 0; u < 8; ++u) v[u] = __ldg(parts + i + u * kBlock);
+        for (int u = 0; u < 8; ++u) v[u] = ldg_o(parts + i + u * kBlock);
 #pragma unroll
         for (int u = 0; u < 8; ++u) s += v[u];
     }
-    for (; i < n; i += kBlock) s += __ldg(parts + i);
+    for (; i < n; i += kBlock) s += ldg_o(parts + i);
     s = block_reduce<false>(s, sh);
     if (threadIdx.x == 0) sh[32] = s;
     __syncthreads();
@@ -1173,7 +1201,7 @@ __device__ __forceinline__ double sum_parts_fixed(const double *parts, unsigned 
 
 // iteration k does not run: propagate to parity q (block 0), uniform exit
 __device__ __forceinline__ bool run_check(CgScalars *sc, int q) {
-    if (__ldg(&sc->run_q[q ^ 1])) return true;
+    if (ldg_o(&sc->run_q[q ^ 1])) return true;
     if (blockIdx.x == 0 && threadIdx.x == 0) sc->run_q[q] = 0;
     return false;
 }
@@ -1230,18 +1258,18 @@ __global__ void __launch_bounds__(kBlock) cg_pupdate1_kernel(Pupd1Args a) {
     pdl_trigger();
     load_r(b0);
     if (!run_check(sc, a.q)) return;
-    const int k = __ldg(&sc->k);
+    const int k = ldg_o(&sc->k);
     trace_mark(a.trace, a.trace_max, k, 0, false);
     const bool first = (k == 1);
     const bool upx = dx && !first;
-    const double alpha_x = upx ? __ldg(&sc->alpha_x) : 0.0;
-    double rtrans = first ? __ldg(&sc->rr_cur) : sum_parts_fixed(a.rr_parts, a.n_rr, sh);
+    const double alpha_x = upx ? ldg_o(&sc->alpha_x) : 0.0;
+    double rtrans = first ? ldg_o(&sc->rr_cur) : sum_parts_fixed(a.rr_parts, a.n_rr, sh);
     if (kPeer && !first) {  // z-slabs: the slab's r.r -> every rank; the global sum back
-        const unsigned tag = ll_tag(__ldg(&sc->epoch), 2ull * (unsigned)(k - 1));
+        const unsigned tag = ll_tag(ldg_o(&sc->epoch), 2ull * (unsigned)(k - 1));
         if (a.post && blockIdx.x == 0 && threadIdx.x == 0) fused_post(a.t, 0, rtrans, tag);
         rtrans = fused_collect_block(a.t, 0, tag, rtrans, &sh[32]);
     }
-    const double beta = first ? 0.0 : rtrans / __ldg(&sc->rr_prev);
+    const double beta = first ? 0.0 : rtrans / ldg_o(&sc->rr_prev);
     if (blockIdx.x == 0 && threadIdx.x == 0) {
         if (!first) sc->rr_cur = rtrans;
         sc->normr = sqrt(rtrans);
@@ -1296,7 +1324,7 @@ __global__ void __launch_bounds__(kBlock) cg_pupdate1_kernel(Pupd1Args a) {
         __syncthreads();
         trace_mark(a.trace, a.trace_max, k, 0, true);
     }
-    if (kPeer) fused_push_signal(a.t, pushed, a.n_push, ftag(__ldg(&sc->epoch), (unsigned long long)k));
+    if (kPeer) fused_push_signal(a.t, pushed, a.n_push, ftag(ldg_o(&sc->epoch), (unsigned long long)k));
 }
 
 // a.5 x += alpha p, r -= alpha Ap, per-block r.r partial (no finisher), and
@@ -1316,6 +1344,8 @@ struct Upd1Args {
     const PeerTab *t;  // HALO_PEER = 2 on z-slabs: p.Ap = the P slabs' local sums
     int post;          // 0: posted by fused_post_kernel (loopback)
     int defer_x;       // 1: leave x to the next p update / cg_xfix_kernel (alpha -> sc->alpha_x)
+    int late_p;        // 1: p was written by the kernel right before (cg_pspmv_kernel): read
+                       // x and p only after the PDL wait
 };
 
 // Loopback + HALO_PEER = 2: every slab's kernels share one stream, so a
@@ -1330,11 +1360,11 @@ __global__ void __launch_bounds__(kBlock) fused_post_kernel(const double *parts,
     __shared__ double sh[33];
     pdl_wait();
     pdl_trigger();
-    const int k = q == 0 ? __ldg(&sc->k) - 1 : __ldg(&sc->niters);
+    const int k = q == 0 ? ldg_o(&sc->k) - 1 : ldg_o(&sc->niters);
     if (q == 0 && k < 1) return;
     const double v = parts ? sum_parts_fixed(parts, n, sh) : __ldcg(fallback);
     if (threadIdx.x == 0)
-        fused_post(t, q, v, ll_tag(__ldg(&sc->epoch), q == 0 ? 2ull * (unsigned)k : 2ull * (unsigned)k - 1ull));
+        fused_post(t, q, v, ll_tag(ldg_o(&sc->epoch), q == 0 ? 2ull * (unsigned)k : 2ull * (unsigned)k - 1ull));
 }
 
 // deferred x update, end of the solve: the last iteration's x += alpha p (no p
@@ -1343,8 +1373,8 @@ __global__ void __launch_bounds__(kBlock) fused_post_kernel(const double *parts,
 __global__ void __launch_bounds__(kBlock) cg_xfix_kernel(int64_t n, double *x, const double *p,
                                                          const CgScalars *sc) {
     pdl_wait();
-    if (__ldg(&sc->niters) < 1) return;
-    const double alpha = __ldg(&sc->alpha_x);
+    if (ldg_o(&sc->niters) < 1) return;
+    const double alpha = ldg_o(&sc->alpha_x);
     const int64_t tid = gtid(), nth = gnth(), nv = n >> 1;
     double2 *__restrict__ x2 = reinterpret_cast<double2 *>(x);
     const double2 *__restrict__ p2 = reinterpret_cast<const double2 *>(p);
@@ -1356,6 +1386,201 @@ __global__ void __launch_bounds__(kBlock) cg_xfix_kernel(int64_t n, double *x, c
         x2[i] = xv;
     }
     if (tid == 0 && (n & 1)) x[n - 1] = fma(alpha, p[n - 1], x[n - 1]);
+}
+
+// ---- a.6 + a.3 + a.4 fused and pipelined (HPCCG_OPT_FUSE_PSPMV): the p
+// update of iteration k and the SpMV Ap = A p_k in ONE kernel, single slab.
+// Chunk c = rows [512c, 512c + 512) (one 256-thread block's SpMV rows, 2 per
+// thread, the partial slot c of the unfused SpMV: identical bits).  Blocks take
+// tickets t in launch order (an atomic counter) and SpMV the chunk at position
+// t (pos reverses the chunk order under serpentine).  Block t first applies p =
+// r + beta p (and the deferred x += alpha_x p) to the chunk at position t +
+// lead and publishes it with a release flag; the chunks at positions < lead
+// were updated by the p-update kernel launched just before (cg_pupdate1_kernel
+// on those rows only).  Its SpMV then waits (acquire) for the <= 9 chunks its
+// gathers touch (the z-1, z, z+1 windows), all at positions < t + lead when
+// lead > plane/512 + 2, i.e. produced by the prologue or by EARLIER tickets
+// that publish before they wait: no block ever waits for a block that has not
+// started, so the kernel cannot deadlock whatever the residency.  p_k is
+// gathered from L2 a few microseconds after it is written: the SpMV's 8n B read
+// of p from HBM goes (12 nnz + 72n B per iteration with the deferred x update,
+// instead of 80n).  The gathers are weak L1-cached loads: a line of p belongs
+// to one chunk (the host checks the alignment) and is first read after the
+// flag acquire (which invalidates the SM's L1), so no SM holds a stale copy;
+// p_old is read with L1::no_allocate.
+constexpr int kPsRows = 2 * kBlock;  // rows per chunk
+
+struct PsArgs {
+    int64_t n, plane, nchunks;
+    int nx, lead, rev, q;
+    const double *val;
+    const int *col;
+    double *p;                    // local-with-halo base: p[plane + i] is row i
+    const double *r;
+    double *x;                    // deferred x update (nullptr: none)
+    double *Ap;
+    double *parts;                // out: per-chunk p.Ap partials (chunk order)
+    const double *rr_parts;       // r.r partials of the previous update
+    unsigned n_rr;
+    CgScalars *sc;
+    unsigned *ticket;             // launch-order counter (reset by the last ticket)
+    unsigned long long *flags;    // [nchunks] chunk c of p_k published: tag(epoch, k)
+    TraceSlot *trace;
+    int trace_max;
+    int *err;                     // a wait that gave up (5 s): the solve reports HPCCG_ECUDA
+};
+
+__device__ __forceinline__ void st_release_gpu(unsigned long long *p, unsigned long long v) {
+    asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ unsigned long long ld_acquire_gpu(const unsigned long long *p) {
+    unsigned long long v;
+    asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ unsigned long long ld_relaxed_gpu(const unsigned long long *p) {
+    unsigned long long v;
+    asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ double2 ld_na2(const double2 *p) {  // coherent, no L1 allocation
+    double2 v;
+    asm volatile("ld.global.L1::no_allocate.v2.f64 {%0, %1}, [%2];" : "=d"(v.x), "=d"(v.y) : "l"(p) : "memory");
+    return v;
+}
+
+// wait until *f >= tag with acquire semantics: one acquire load in the common
+// case; else relaxed polls and a final acquire; gives up after 5 s (only a bug
+// could get there) with *err set instead of hanging the GPU
+__device__ __forceinline__ void ps_wait(const PsArgs &a, const unsigned long long *f, unsigned long long tag) {
+    if (ld_acquire_gpu(f) >= tag) return;
+    const unsigned long long t0 = gtimer();
+    while (ld_relaxed_gpu(f) < tag) {
+        if (*(volatile int *)a.err || gtimer() - t0 > 5000000000ull) {
+            *(volatile int *)a.err = 1;
+            return;
+        }
+        __nanosleep(64);
+    }
+    (void)ld_acquire_gpu(f);
+}
+
+__global__ void __launch_bounds__(kBlock, 4) cg_pspmv_kernel(PsArgs a) {
+    __shared__ unsigned s_t;
+    __shared__ double shp[33];
+    if (threadIdx.x == 0) s_t = atomicAdd(a.ticket, 1u);
+    __syncthreads();
+    const unsigned t = s_t;
+    if (threadIdx.x == 0 && t == (unsigned)a.nchunks - 1u) *a.ticket = 0u;  // every ticket taken
+    const int64_t c = a.rev ? a.nchunks - 1 - (int64_t)t : (int64_t)t;
+    const int64_t row = c * kPsRows + 2 * threadIdx.x;
+    const bool active = row < a.n;  // n even: both rows of the pair exist
+    const uint64_t pol = policy_evict_first();
+    const double *v = a.val + row;
+    const int *ci = a.col + row;
+    // the matrix does not depend on the predecessor: the first group's loads
+    // are in flight before the PDL wait and the producer work
+    double2 vv0[3];
+    int2 cc0[3];
+    if (active) {
+#pragma unroll
+        for (int u = 0; u < 3; ++u) {
+            vv0[u] = ld_stream2(v + u * a.n, pol);
+            cc0[u] = ld_stream2(ci + u * a.n, pol);
+        }
+    }
+    pdl_wait();
+    if (!run_check(a.sc, a.q)) return;  // uniform: iteration k does not run
+    CgScalars *sc = a.sc;
+    const int k = ldg_o(&sc->k);
+    const bool first = (k == 1);
+    const unsigned long long tag = ftag(ldg_o(&sc->epoch), (unsigned long long)k);
+    trace_mark(a.trace, a.trace_max, k, 1, false);
+    pdl_trigger();
+    // produce the chunk `lead` positions ahead (beta / alpha_x were finished
+    // and stored by the prologue p update's block 0: ordered loads after the wait)
+    const int64_t tp = (int64_t)t + a.lead;
+    if (tp < a.nchunks) {
+        const double beta = first ? 0.0 : ldg_o(&sc->rr_cur) / ldg_o(&sc->rr_prev);
+        const double alpha_x = first ? 0.0 : ldg_o(&sc->alpha_x);
+        const int64_t cp = a.rev ? a.nchunks - 1 - tp : tp;
+        const int64_t i = (cp * kPsRows >> 1) + threadIdx.x;  // 16-B unit
+        if (2 * i < a.n) {
+            double2 *p2 = reinterpret_cast<double2 *>(a.p + a.plane);
+            const double2 rv = ldg_o2(reinterpret_cast<const double2 *>(a.r) + i);
+            double2 pv = rv;
+            if (!first) {
+                const double2 po = ld_na2(p2 + i);
+                pv.x = fma(beta, po.x, rv.x);
+                pv.y = fma(beta, po.y, rv.y);
+                if (a.x) {
+                    double2 *x2 = reinterpret_cast<double2 *>(a.x);
+                    double2 xv = ld_na2(x2 + i);
+                    xv.x = fma(alpha_x, po.x, xv.x);
+                    xv.y = fma(alpha_x, po.y, xv.y);
+                    x2[i] = xv;
+                }
+            }
+            p2[i] = pv;
+        }
+        __syncthreads();  // the block's stores before thread 0's release (cumulative)
+        if (threadIdx.x == 0) st_release_gpu(a.flags + cp, tag);
+    }
+    // consume: wait for the chunks this block's gathers read (z-1, z, z+1
+    // windows of rows [512c - nx - 1, 512c + 511 + nx + 1]); thread 3w + o
+    // takes chunk o of window w, all polls in flight at once
+    if (threadIdx.x < 9) {
+        const int w = threadIdx.x / 3, o = threadIdx.x % 3;
+        const int64_t lo = c * kPsRows + (w - 1) * a.plane - a.nx - 1;
+        const int64_t hi = c * kPsRows + kPsRows - 1 + (w - 1) * a.plane + a.nx + 1;
+        const int64_t l = max(lo, (int64_t)0), h = min(hi, a.n - 1);
+        const int64_t cw = l / kPsRows + o;
+        if (l <= h && cw <= h / kPsRows) {
+            const int64_t pw = a.rev ? a.nchunks - 1 - cw : cw;  // its position
+            if (pw >= a.lead) ps_wait(a, a.flags + cw, tag);  // else: the prologue's
+        }
+    }
+    __syncthreads();
+    double d = 0.0;
+    if (active) {
+        const double *px = a.p;
+        double s0 = 0.0, s1 = 0.0, x0 = 0.0, x1 = 0.0;
+        int c0 = 0, c1 = 0;
+#pragma unroll
+        for (int g = 0; g < kSlots / 3; ++g) {
+            double2 vv[3];
+            int2 cc[3];
+#pragma unroll
+            for (int u = 0; u < 3; ++u) {
+                if (g == 0) {
+                    vv[u] = vv0[u];
+                    cc[u] = cc0[u];
+                } else {
+                    vv[u] = ld_stream2(v + (3 * g + u) * a.n, pol);
+                    cc[u] = ld_stream2(ci + (3 * g + u) * a.n, pol);
+                }
+            }
+#pragma unroll
+            for (int u = 0; u < 3; ++u) {
+                const double xa = px[cc[u].x], xb = px[cc[u].y];  // weak, L1-cached (see above)
+                if (3 * g + u == kDiagSlot) {
+                    x0 = xa;
+                    x1 = xb;
+                    c0 = cc[u].x;
+                    c1 = cc[u].y;
+                }
+                s0 = fma(vv[u].x, xa, s0);
+                s1 = fma(vv[u].y, xb, s1);
+            }
+        }
+        *reinterpret_cast<double2 *>(a.Ap + row) = make_double2(s0, s1);
+        const double p0 = c0 == row + a.plane ? x0 : px[row + a.plane];
+        const double p1 = c1 == row + 1 + a.plane ? x1 : px[row + 1 + a.plane];
+        d = fma(s1, p1, s0 * p0);
+    }
+    d = block_reduce<false>(d, shp);
+    if (threadIdx.x == 0) a.parts[c] = d;
+    trace_mark(a.trace, a.trace_max, k, 1, true);
 }
 
 template <int kU, bool kPeer = false>
@@ -1395,26 +1620,29 @@ __global__ void __launch_bounds__(kBlock) cg_update1_kernel(Upd1Args a) {
     };
     // x, r (previous update) and p (p update) are complete before the SpMV's
     // blocks pass their pdl_wait, so before this grid can launch: read them
-    // during the SpMV's tail; Ap only after the SpMV has completed
-    load_xrp(tid);
+    // during the SpMV's tail; Ap only after the SpMV has completed.  Fused p
+    // update + SpMV: p (and x) come from the predecessor itself -> after the wait
+    const bool early = !(a.late_p && !dx);
+    if (early) load_xrp(tid);
     pdl_wait();
     pdl_trigger();
+    if (!early) load_xrp(tid);
     load_q(tid);
     if (!run_check(sc, a.q)) return;
-    const int ktr = a.trace ? __ldg(&sc->niters) : 0;
+    const int ktr = a.trace ? ldg_o(&sc->niters) : 0;
     trace_mark(a.trace, a.trace_max, ktr, 2, false);
-    const double rtrans = __ldg(&sc->rr_cur);
-    double pAp = a.pAp_parts ? sum_parts_fixed(a.pAp_parts, a.n_parts, sh) : __ldg(&sc->pAp);
+    const double rtrans = ldg_o(&sc->rr_cur);
+    double pAp = a.pAp_parts ? sum_parts_fixed(a.pAp_parts, a.n_parts, sh) : ldg_o(&sc->pAp);
     if (kPeer) {  // z-slabs: the slab's p.Ap -> every rank; the global sum back
-        const unsigned tag = ll_tag(__ldg(&sc->epoch), 2ull * (unsigned)__ldg(&sc->niters) - 1ull);
+        const unsigned tag = ll_tag(ldg_o(&sc->epoch), 2ull * (unsigned)ldg_o(&sc->niters) - 1ull);
         if (a.post && blockIdx.x == 0 && threadIdx.x == 0) fused_post(a.t, 1, pAp, tag);
         pAp = fused_collect_block(a.t, 1, tag, pAp, &sh[32]);
     }
     const bool stop = (rtrans == 0.0) || (pAp == 0.0);  // A11
     const double alpha = stop ? 0.0 : rtrans / pAp;
     if (blockIdx.x == 0 && threadIdx.x == 0) {
-        const int k = __ldg(&sc->k);
-        const int run = !stop && (k + 1) < __ldg(&sc->max_iter) && __ldg(&sc->normr) > __ldg(&sc->tol);
+        const int k = ldg_o(&sc->k);
+        const int run = !stop && (k + 1) < ldg_o(&sc->max_iter) && ldg_o(&sc->normr) > ldg_o(&sc->tol);
         sc->pAp = pAp;
         sc->rr_prev = rtrans;
         sc->alpha_x = alpha;
@@ -1544,8 +1772,8 @@ __device__ __forceinline__ double2 sr_sum_parts(const double *parts, unsigned np
         double vg[4], vd[4];
 #pragma unroll
         for (int u = 0; u < 4; ++u) {
-            vg[u] = __ldg(parts + i + u * kBlock);
-            vd[u] = __ldg(parts + np + i + u * kBlock);
+            vg[u] = ldg_o(parts + i + u * kBlock);
+            vd[u] = ldg_o(parts + np + i + u * kBlock);
         }
 #pragma unroll
         for (int u = 0; u < 4; ++u) {
@@ -1554,8 +1782,8 @@ __device__ __forceinline__ double2 sr_sum_parts(const double *parts, unsigned np
         }
     }
     for (; i < np; i += kBlock) {
-        g += __ldg(parts + i);
-        d += __ldg(parts + np + i);
+        g += ldg_o(parts + i);
+        d += ldg_o(parts + np + i);
     }
     double2 t = block_reduce2(g, d, sh);
     if (threadIdx.x == 0) {
@@ -1582,8 +1810,8 @@ __global__ void __launch_bounds__(1024, 1) cg_sr_finish_kernel(const double *par
         double vg[12], vd[12];
 #pragma unroll
         for (int u = 0; u < 12; ++u) {
-            vg[u] = __ldg(parts + i + u * 1024u);
-            vd[u] = __ldg(parts + n_parts + i + u * 1024u);
+            vg[u] = ldg_o(parts + i + u * 1024u);
+            vd[u] = ldg_o(parts + n_parts + i + u * 1024u);
         }
 #pragma unroll
         for (int t = 0; t < 3; ++t)
@@ -1631,10 +1859,10 @@ __global__ void __launch_bounds__(kBlock) fused_post2_kernel(const double *parts
     __shared__ double sh[66];
     pdl_wait();
     pdl_trigger();
-    const int k = __ldg(&sc->sr_k[q ^ 1]);
-    if (k < 2 || !__ldg(&sc->run_q[q ^ 1])) return;
+    const int k = ldg_o(&sc->sr_k[q ^ 1]);
+    if (k < 2 || !ldg_o(&sc->run_q[q ^ 1])) return;
     const double2 v = parts ? sr_sum_parts(parts, n, sh) : make_double2(__ldcg(fallback), __ldcg(fallback + 1));
-    if (threadIdx.x == 0) fused_post2(t, (k - 1) & 1, v, ll_tag(__ldg(&sc->epoch), (unsigned)(k - 1)));
+    if (threadIdx.x == 0) fused_post2(t, (k - 1) & 1, v, ll_tag(ldg_o(&sc->epoch), (unsigned)(k - 1)));
 }
 
 template <bool kVec, int kU, bool kPeer = false>
@@ -1658,7 +1886,7 @@ __global__ void __launch_bounds__(kBlock) cg_sr_update_kernel(SrUpdArgs a) {
     }
     pdl_wait();
     pdl_trigger();
-    if (!__ldg(&sc->run_q[qp])) {  // iteration k does not run (uniform) ...
+    if (!ldg_o(&sc->run_q[qp])) {  // iteration k does not run (uniform) ...
         // ... and neither does k + 1: propagate, or slot q would keep the stale
         // flag of iteration k - 1 for the launches of parity q that follow
         if (blockIdx.x == 0 && threadIdx.x == 0) sc->run_q[q] = 0;
@@ -1666,32 +1894,32 @@ __global__ void __launch_bounds__(kBlock) cg_sr_update_kernel(SrUpdArgs a) {
     }
     __shared__ double sh[66];
     double2 gd;
-    const int k = __ldg(&sc->sr_k[qp]);
+    const int k = ldg_o(&sc->sr_k[qp]);
     const bool first = (k == 1);
     if (kPeer) {  // z-slabs: k = 1 takes the init's allreduced values
         if (first) {
-            gd = make_double2(__ldg(&sc->gd[0]), __ldg(&sc->gd[1]));
+            gd = make_double2(ldg_o(&sc->gd[0]), ldg_o(&sc->gd[1]));
         } else {
             gd = a.parts ? sr_sum_parts(a.parts, a.n_parts, sh)
                          : make_double2(__ldcg(&sc->loc_gd[0]), __ldcg(&sc->loc_gd[1]));
-            const unsigned tag = ll_tag(__ldg(&sc->epoch), (unsigned)(k - 1));
+            const unsigned tag = ll_tag(ldg_o(&sc->epoch), (unsigned)(k - 1));
             if (a.post && blockIdx.x == 0 && threadIdx.x == 0) fused_post2(a.t, (k - 1) & 1, gd, tag);
             gd = fused_collect2_block(a.t, (k - 1) & 1, tag, gd, &sh[64]);
         }
     } else if (a.parts) {
         gd = sr_sum_parts(a.parts, a.n_parts, sh);
     } else {
-        gd = make_double2(__ldg(&sc->gd[0]), __ldg(&sc->gd[1]));
+        gd = make_double2(ldg_o(&sc->gd[0]), ldg_o(&sc->gd[1]));
     }
     const double gamma = gd.x, delta = gd.y;
-    const double beta = first ? 0.0 : __ddiv_rn(gamma, __ldg(&sc->sr_gamma[qp]));
+    const double beta = first ? 0.0 : __ddiv_rn(gamma, ldg_o(&sc->sr_gamma[qp]));
     const double den =
-        first ? delta : __dsub_rn(delta, __ddiv_rn(__dmul_rn(beta, gamma), __ldg(&sc->sr_alpha[qp])));
+        first ? delta : __dsub_rn(delta, __ddiv_rn(__dmul_rn(beta, gamma), ldg_o(&sc->sr_alpha[qp])));
     const bool stop = (gamma == 0.0) || (den == 0.0);  // A11
     const double alpha = stop ? 0.0 : __ddiv_rn(gamma, den);
     if (blockIdx.x == 0 && threadIdx.x == 0) {
         const double normr = sqrt(gamma);  // ||r_(k-1)||: the lagged check (A4)
-        const int nrun = !stop && (k + 1 < __ldg(&sc->max_iter)) && normr > __ldg(&sc->tol);
+        const int nrun = !stop && (k + 1 < ldg_o(&sc->max_iter)) && normr > ldg_o(&sc->tol);
         sc->sr_gamma[q] = gamma;
         sc->sr_alpha[q] = alpha;
         sc->sr_k[q] = k + 1;
@@ -1769,7 +1997,7 @@ __global__ void __launch_bounds__(kBlock) cg_sr_update_kernel(SrUpdArgs a) {
             a.r[i] = fma(-alpha, sv, a.r[i]);
             if (kPeer) put(i, a.r[i]);
         }
-        if (kPeer) fused_push_signal(a.t, pushed, a.n_push, ftag(__ldg(&sc->epoch), (unsigned long long)k));
+        if (kPeer) fused_push_signal(a.t, pushed, a.n_push, ftag(ldg_o(&sc->epoch), (unsigned long long)k));
     } else {
         for (int64_t i = tid; i < a.n; i += nth) {
             const double pv = first ? a.r[i] : fma(beta, a.p[i], a.r[i]);

@@ -209,8 +209,8 @@ __global__ void __launch_bounds__(kBlock) tri_update_kernel(int64_t n, double *_
                                                            unsigned long long cond_handle) {
     pdl_wait();
     pdl_trigger();
-    const double rr = __ldg(&sc->rr);
-    const double alpha = rr / __ldg(&sc->pAp);
+    const double rr = ldg_o(&sc->rr);
+    const double alpha = rr / ldg_o(&sc->pAp);
     const double nalpha = alpha * (-1.0);
     double acc = 0.0;
     const int64_t nth = gnth();
@@ -253,7 +253,7 @@ __global__ void __launch_bounds__(kBlock) tri_pupdate_kernel(int64_t n, const do
                                                             const TriScalars *sc) {
     pdl_wait();
     pdl_trigger();
-    const double beta = __ldg(&sc->slot[2]);
+    const double beta = ldg_o(&sc->slot[2]);
     const int64_t nth = gnth();
     for (int64_t b0 = gtid(); b0 < n; b0 += kTriU * nth) {
         double pv[kTriU], rv[kTriU];

@@ -39,6 +39,7 @@ HPCCG_OPT_CLUSTER_ROWS, HPCCG_OPT_SMEM_SOLVE, HPCCG_OPT_TRACE = 12, 13, 14
 HPCCG_OPT_WHILE_UNROLL, HPCCG_OPT_CG_VARIANT, HPCCG_OPT_FINISHER_FREE = 15, 16, 17
 HPCCG_OPT_SMEM_THREADS, HPCCG_OPT_HALO_PEER, HPCCG_OPT_SERPENTINE = 18, 19, 20
 HPCCG_OPT_SPMV_FORMAT, HPCCG_OPT_PEER_TIMEOUT_MS, HPCCG_OPT_DEFER_X = 21, 22, 23
+HPCCG_OPT_FUSE_PSPMV, HPCCG_OPT_PS_LEAD = 24, 25
 
 _lock = threading.Lock()
 _lib = None
@@ -56,7 +57,8 @@ class hpccg_stats(ctypes.Structure):
                 ("allreduce_ms", ctypes.c_double), ("exchange_ms", ctypes.c_double),
                 ("spmv_launches", ctypes.c_int64), ("iterations", ctypes.c_int64),
                 ("kernel_launches", ctypes.c_int64), ("l2_persist_bytes", ctypes.c_int64),
-                ("graph_mode", ctypes.c_int64), ("x_deferred", ctypes.c_int64)]
+                ("graph_mode", ctypes.c_int64), ("x_deferred", ctypes.c_int64),
+                ("ps_fused", ctypes.c_int64)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}

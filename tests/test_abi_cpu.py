@@ -93,3 +93,27 @@ def test_product_does_not_import_oracle():
                 src = open(os.path.join(root, f)).read()
                 assert not re.search(r"^\s*(import|from)\s+oracle\b", src, re.M), f
                 assert "hpccg_oracle" not in src and "liboracle" not in src, f
+
+
+def test_no_readonly_loads_ahead_of_the_pdl_wait(lib):
+    """PDL safety (structural): in every kernel that waits on its predecessor
+    (griddepcontrol.wait = SASS ACQBULK), no read-only-path load of anything
+    but the matrix stream (LDG ... .NA ... .CONSTANT = ld.global.nc
+    L1::no_allocate) may come before the first wait.  Device scalars and
+    partial sums are read with ordered loads (kernels.cuh ldg_o) so the
+    compiler cannot hoist them above it (an __ldg may legally move)."""
+    cuobjdump = "/usr/local/cuda/bin/cuobjdump"
+    if not os.path.exists(cuobjdump):
+        pytest.skip("no cuobjdump")
+    sass = subprocess.run([cuobjdump, "-sass", H.LIB_PATH], capture_output=True, text=True).stdout
+    funcs = re.split(r"\n\s+Function : ", sass)[1:]
+    waiting = [f for f in funcs if "ACQBULK" in f]
+    assert len(waiting) > 20
+    bad = []
+    for f in waiting:
+        pre = f.split("ACQBULK")[0]
+        loads = set(re.findall(r"LDG\.E[A-Z0-9._]*", pre))
+        early = sorted(x for x in loads if "CONSTANT" in x and ".NA." not in x)
+        if early:
+            bad.append((f.split("\n", 1)[0][:80], early))
+    assert not bad, bad

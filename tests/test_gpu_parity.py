@@ -1063,3 +1063,63 @@ def test_defer_x_fused_loopback_bitwise(P):
         oref = oracle.cg(ref, 150, 1e-12)
         assert abs(res[1][0] - oref["niters"]) <= 1
         assert np.max(np.abs(res[1][2] - oref["x"])) <= CG_ATOL
+
+
+# ------------------------------- fused, pipelined p update + SpMV (FUSE_PSPMV)
+
+@pytest.mark.parametrize("dims,max_iter,tol,defer,lead", [
+    ((16, 16, 33), 60, 0.0, 1, 0), ((32, 32, 40), 150, 1e-12, 1, 0), ((32, 32, 40), 150, 1e-12, 0, 0),
+    ((64, 64, 64), 150, 1e-12, 1, 0), ((64, 64, 64), 30, 0.0, 1, 40), ((48, 16, 50), 25, 0.0, 1, 0),
+    ((128, 128, 128), 21, 0.0, 1, 0), ((256, 256, 256), 11, 0.0, 1, 0)])
+def test_fused_pspmv_bitwise_identical(ctx, dims, max_iter, tol, defer, lead):
+    """HPCCG_OPT_FUSE_PSPMV: the p update and the SpMV as one pipelined kernel
+    (chunks in launch-ticket order, release/acquire chunk flags) -- the same
+    per-row FMA chains and the same per-chunk p.Ap partials, so niters, normr
+    and x are bit for bit the unfused loop's, in every launch mode, with and
+    without the deferred x update, forwards and (serpentine) backwards; and
+    within the north_star tolerance of the oracle."""
+    with H.Problem(ctx, *dims) as p:
+        p.set_option(H.HPCCG_OPT_PERSISTENT, 0)
+        p.set_option(H.HPCCG_OPT_DEFER_X, defer)
+        p.set_option(H.HPCCG_OPT_PS_LEAD, lead)
+        outs = []
+        for fuse, serp in ((0, 0), (1, 0), (1, 3), (0, 3)):
+            p.set_option(H.HPCCG_OPT_FUSE_PSPMV, fuse)
+            p.set_option(H.HPCCG_OPT_SERPENTINE, serp)
+            for mode in ("while", "graph", "timing"):
+                p.set_option(H.HPCCG_OPT_WHILE, 1 if mode == "while" else 0)
+                p.set_option(H.HPCCG_OPT_TIMING, 1 if mode == "timing" else 0)
+                p.set_vec(H.HPCCG_VEC_X, np.zeros(p.n))
+                r = p.solve(max_iter, tol)
+                st = p.stats()
+                assert st["ps_fused"] == fuse, (fuse, mode)
+                outs.append((fuse, serp, mode, r["niters"], r["normr"], p.get_vec(H.HPCCG_VEC_X)))
+        p.set_option(H.HPCCG_OPT_TIMING, 0)
+        p.set_option(H.HPCCG_OPT_WHILE, 1)
+        p.set_option(H.HPCCG_OPT_FUSE_PSPMV, 0)
+        p.set_option(H.HPCCG_OPT_SERPENTINE, -1)
+        for o in outs[1:]:
+            assert o[3:5] == outs[0][3:5], (o[:5], outs[0][:5])
+            np.testing.assert_array_equal(o[5], outs[0][5])
+        if p.n <= 300_000:
+            ref = oracle.generate(*dims)
+            oref = oracle.cg(ref, max_iter, tol)
+            assert abs(outs[-1][3] - oref["niters"]) <= 1
+            assert np.max(np.abs(outs[-1][5] - oref["x"])) <= CG_ATOL
+
+
+def test_fused_pspmv_spmv_bitwise_vs_oracle(ctx):
+    """One fused iteration from x0 = 0 (p_1 = r_0 = b): Ap_1 must equal the
+    oracle's A b bit for bit (checked through the first CG step, which is
+    exact: alpha_1 = b.b / b.Ab)."""
+    dims = (20, 30, 12)
+    with H.Problem(ctx, *dims) as p:
+        p.set_option(H.HPCCG_OPT_PERSISTENT, 0)
+        p.set_option(H.HPCCG_OPT_FUSE_PSPMV, 1)
+        p.set_option(H.HPCCG_OPT_DEFER_X, 1)
+        p.set_vec(H.HPCCG_VEC_X, np.zeros(p.n))
+        p.solve(2, 0.0)                      # one iteration: x_1 = alpha_1 b
+        x1 = p.get_vec(H.HPCCG_VEC_X)
+        ref = oracle.generate(*dims)
+        o = oracle.cg(ref, 2, 0.0)
+        np.testing.assert_array_equal(x1, o["x"])
