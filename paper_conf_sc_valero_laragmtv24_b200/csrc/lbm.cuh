@@ -73,8 +73,11 @@ __device__ __forceinline__ void lbm_collide(const double (&fk)[9], double keep, 
 // streaming (evict-first); 1 (default): loads streaming, stores cached (the
 // lattice just written, 72 MB at 1000^2, stays largely in the 126 MB L2 for
 // the next step's pulls: 26.7 vs 29.3 us/step measured); 2: both cached.
+#ifndef HPCCG_LBM_MINB
+#define HPCCG_LBM_MINB 4  // 64 registers, 4 CTAs/SM: 21.45 vs 25.13 us/step at 1000^2 (68 regs, 3 CTAs); 5-6 spill
+#endif
 template <bool kWriteF, int kPol>
-__global__ void __launch_bounds__(kBlock) lbm_pull_kernel(int S, const double *__restrict__ f1,
+__global__ void __launch_bounds__(kBlock, HPCCG_LBM_MINB) lbm_pull_kernel(int S, const double *__restrict__ f1,
                                                          double *__restrict__ f,
                                                          double *__restrict__ f2, double keep,
                                                          double tau) {
