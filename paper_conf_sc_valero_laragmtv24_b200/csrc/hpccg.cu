@@ -916,7 +916,9 @@ int enqueue_iteration_ff_u(hpccg_problem *p, bool timing, bool check, unsigned l
     hpccg_ctx *ctx = p->ctx;
     const bool pdl = p->opt_pdl != 0;
     const bool zs = ctx->mode != MODE_SINGLE;  // HALO_PEER = 2 on z-slabs (fused_on)
-    auto upd = zs ? cg_update1_kernel<kU, true> : cg_update1_kernel<kU, false>;
+    const bool fuse = !zs && fuse_ps_on(p);
+    auto upd = zs ? cg_update1_kernel<kU, true> : fuse ? cg_update1_kernel<kU, false, true>
+                                                       : cg_update1_kernel<kU, false>;
     auto pup = zs ? cg_pupdate1_kernel<kU, true> : cg_pupdate1_kernel<kU, false>;
     const Slab &s0 = p->slabs[0];
     // the update's grid fixes the r.r partials and so the bits: size it as
@@ -926,7 +928,6 @@ int enqueue_iteration_ff_u(hpccg_problem *p, bool timing, bool check, unsigned l
     const int pg = vec_grid(ctx, pup, cdiv(s0.n, 2 * kU), p->opt_vec_waves, 0x7fffffff);
     // loopback: every slab's post ahead of every slab's collect (one stream)
     const bool pre = zs && ctx->mode == MODE_LOOPBACK;
-    const bool fuse = !zs && fuse_ps_on(p);
     auto post = [&](const Slab &s, const double *parts, unsigned n, int q) {
         launch_k(pdl, fused_post_kernel, dim3(1), ctx->stream, parts, n, (const double *)&s.sc->pAp,
                  (const PeerTab *)s.ptab, (const CgScalars *)s.sc, q);
@@ -1025,7 +1026,6 @@ int enqueue_iteration_ff_u(hpccg_problem *p, bool timing, bool check, unsigned l
         a.trace_max = s.trace_max;
         a.t = zs ? s.ptab : nullptr;
         a.defer_x = defer_x_on(p) ? 1 : 0;
-        a.late_p = fuse ? 1 : 0;
         if (np <= kUpdSumMax) {
             a.pAp_parts = s.spmv_parts;
             a.n_parts = np;

@@ -106,32 +106,18 @@ __device__ __forceinline__ int2 ld_stream2(const int *ptr, uint64_t pol) {
 }
 
 // Loads of data the PREDECESSOR grid wrote (device scalars, reduction
-// partials), for use after pdl_wait(): plain weak ld.global (L1-cacheable, so
-// one L2 request per SM still serves every warp), NOT the read-only path.  An
-// ld.global.nc promises the data is constant for the kernel's lifetime, and
-// ptxas uses that promise to hoist it above griddepcontrol.wait (SASS ACQBULK)
-// -- seen in the fused p update + SpMV kernel, where a stale run flag / scalar
-// read raced the predecessor; tests/test_abi_cpu.py checks every kernel's SASS.
-__device__ __forceinline__ double ldg_o(const double *p) {
-    double v;
-    asm volatile("ld.global.f64 %0, [%1];" : "=d"(v) : "l"(p) : "memory");
-    return v;
-}
-__device__ __forceinline__ int ldg_o(const int *p) {
-    int v;
-    asm volatile("ld.global.s32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
-    return v;
-}
-__device__ __forceinline__ double2 ldg_o2(const double2 *p) {
-    double2 v;
-    asm volatile("ld.global.v2.f64 {%0, %1}, [%2];" : "=d"(v.x), "=d"(v.y) : "l"(p) : "memory");
-    return v;
-}
-__device__ __forceinline__ unsigned long long ldg_o(const unsigned long long *p) {
-    unsigned long long v;
-    asm volatile("ld.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
-    return v;
-}
+// partials), after pdl_wait().  ldg_o: the read-only path (one L2 request per
+// SM serves every warp; plain loads cost 1.6 % at 128^3).  The compiler may
+// hoist an ld.global.nc above griddepcontrol.wait (SASS ACQBULK) -- the nc
+// contract says the data is constant for the kernel's lifetime -- and did so
+// in the fused p update + SpMV kernel, which therefore uses plain loads (ldp);
+// tests/test_abi_cpu.py fails the build if any kernel's SASS has a read-only
+// load ahead of its first ACQBULK.
+__device__ __forceinline__ double ldg_o(const double *p) { return __ldg(p); }
+__device__ __forceinline__ int ldg_o(const int *p) { return __ldg(p); }
+__device__ __forceinline__ unsigned long long ldg_o(const unsigned long long *p) { return __ldg(p); }
+template <class T>
+__device__ __forceinline__ T ldp(const T *p) { return *p; }  // plain weak load (never nc)
 
 // Programmatic dependent launch (PDL): a kernel launched with the
 // programmatic-stream-serialization attribute may start while its
@@ -1211,6 +1197,8 @@ __device__ __forceinline__ bool run_check(CgScalars *sc, int q) {
 // issued before the scalar work so their latency overlaps the partial sums.
 // kPeer: the HALO_PEER = 2 hooks (z-slabs); the single-slab instantiation
 // carries none of their code
+// (__launch_bounds__(kBlock, 4) -- 64 registers with spills -- measured slower
+// at 256^3: 992 vs 986 us/iteration)
 template <int kU, bool kPeer = false>
 __global__ void __launch_bounds__(kBlock) cg_pupdate1_kernel(Pupd1Args a) {
     __shared__ double sh[33];
@@ -1344,9 +1332,9 @@ struct Upd1Args {
     const PeerTab *t;  // HALO_PEER = 2 on z-slabs: p.Ap = the P slabs' local sums
     int post;          // 0: posted by fused_post_kernel (loopback)
     int defer_x;       // 1: leave x to the next p update / cg_xfix_kernel (alpha -> sc->alpha_x)
-    int late_p;        // 1: p was written by the kernel right before (cg_pspmv_kernel): read
-                       // x and p only after the PDL wait
 };
+// (kLateP: p was written by the kernel right before -- cg_pspmv_kernel -- so x
+// and p are read only after the PDL wait)
 
 // Loopback + HALO_PEER = 2: every slab's kernels share one stream, so a
 // collect in slab 0's kernel could never see slab 1's post from a kernel
@@ -1490,24 +1478,27 @@ __global__ void __launch_bounds__(kBlock, 4) cg_pspmv_kernel(PsArgs a) {
         }
     }
     pdl_wait();
-    if (!run_check(a.sc, a.q)) return;  // uniform: iteration k does not run
+    if (!ldp(&a.sc->run_q[a.q ^ 1])) {  // uniform: iteration k does not run (run_check)
+        if (t == 0 && threadIdx.x == 0) a.sc->run_q[a.q] = 0;
+        return;
+    }
     CgScalars *sc = a.sc;
-    const int k = ldg_o(&sc->k);
+    const int k = ldp(&sc->k);
     const bool first = (k == 1);
-    const unsigned long long tag = ftag(ldg_o(&sc->epoch), (unsigned long long)k);
+    const unsigned long long tag = ftag(ldp(&sc->epoch), (unsigned long long)k);
     trace_mark(a.trace, a.trace_max, k, 1, false);
     pdl_trigger();
     // produce the chunk `lead` positions ahead (beta / alpha_x were finished
     // and stored by the prologue p update's block 0: ordered loads after the wait)
     const int64_t tp = (int64_t)t + a.lead;
     if (tp < a.nchunks) {
-        const double beta = first ? 0.0 : ldg_o(&sc->rr_cur) / ldg_o(&sc->rr_prev);
-        const double alpha_x = first ? 0.0 : ldg_o(&sc->alpha_x);
+        const double beta = first ? 0.0 : ldp(&sc->rr_cur) / ldp(&sc->rr_prev);
+        const double alpha_x = first ? 0.0 : ldp(&sc->alpha_x);
         const int64_t cp = a.rev ? a.nchunks - 1 - tp : tp;
         const int64_t i = (cp * kPsRows >> 1) + threadIdx.x;  // 16-B unit
         if (2 * i < a.n) {
             double2 *p2 = reinterpret_cast<double2 *>(a.p + a.plane);
-            const double2 rv = ldg_o2(reinterpret_cast<const double2 *>(a.r) + i);
+            const double2 rv = ldp(reinterpret_cast<const double2 *>(a.r) + i);
             double2 pv = rv;
             if (!first) {
                 const double2 po = ld_na2(p2 + i);
@@ -1583,7 +1574,7 @@ __global__ void __launch_bounds__(kBlock, 4) cg_pspmv_kernel(PsArgs a) {
     trace_mark(a.trace, a.trace_max, k, 1, true);
 }
 
-template <int kU, bool kPeer = false>
+template <int kU, bool kPeer = false, bool kLateP = false>
 __global__ void __launch_bounds__(kBlock) cg_update1_kernel(Upd1Args a) {
     __shared__ double sh[33];
     CgScalars *sc = a.sc;
@@ -1622,7 +1613,7 @@ __global__ void __launch_bounds__(kBlock) cg_update1_kernel(Upd1Args a) {
     // blocks pass their pdl_wait, so before this grid can launch: read them
     // during the SpMV's tail; Ap only after the SpMV has completed.  Fused p
     // update + SpMV: p (and x) come from the predecessor itself -> after the wait
-    const bool early = !(a.late_p && !dx);
+    const bool early = !(kLateP && !dx);
     if (early) load_xrp(tid);
     pdl_wait();
     pdl_trigger();
