@@ -17,8 +17,9 @@ are set on; so a scaling run's N = 1 point is this line.  Before timing, every
 workload runs a tol 1e-12 correctness solve of the GLOBAL problem and checks
 niters against SURVEY's independent counts (`correctness`).  The same line
 carries `sub_configs`: configs[1] (128^3, 500 iterations), configs[0]
-(20x30x10 at tol 1e-12 / 150, as BASELINE states it) at N = 1, and configs[3]
-(512^3 global, strong) at every N -- each with t_iter, GFLOP/s and e2e.
+(20x30x10 at tol 1e-12 / 150, as BASELINE states it) at N = 1, configs[3]
+(512^3 global, strong) at every N -- each with t_iter, GFLOP/s and e2e -- and
+configs[4] (the JACC BLAS-1 AXPY/DOT sweep 1e3..1e9, DOT sharded at N > 1).
 
 value = CG GFLOP/s of the whole job = sum over ranks of niters (2 nnz + 10 n)
         / max-over-ranks device time of the K timed steps (exact nnz, A15).
@@ -714,6 +715,19 @@ def run_ours(args):
             sub["_prob"].free()
             subs[nm] = _strip(sub)
             torch.cuda.empty_cache()
+    # configs[4]: the JACC BLAS-1 sweep (AXPY + DOT, 1e3..1e9 per GPU; at N > 1 the
+    # DOT is sharded with the allreduce inside hpccg_ddot) -- needs a NCCL or single context
+    if not args.no_sub_configs and not (world > 1 and transport == "peer"):
+        rows = blas1_sweep(ctx, world, rank, [10 ** k for k in range(3, 10)], 3, reps_cap=50)
+        big = rows[-1]
+        subs["blas1"] = {
+            "workload": "blas1", "baseline_config": 4, "metric": BLAS1_METRIC, "unit": "GB/s",
+            "value": round((24.0 + 16.0) * big["n_per_gpu"] * world /
+                           ((big["axpy_us"] + big["dot_us"]) * 1e-6) / 1e9, 1),
+            "how": "AXPY x += 2.5 y then DOT x.y at n = 1e9 per GPU, host-synchronous calls (launch + "
+                   "sync included); inputs round(rand*100) (Fig. 2); max over ranks",
+            "all_dot_exact": all(r["dot_exact"] for r in rows) if world == 1 else None,
+            "sweep": rows}
     peak_read = read_peak_gbs(ctx, stream) if world == 1 else None
 
     if rank == 0:
@@ -859,6 +873,63 @@ def traffic_from_profiles(workload):
         return None
 
 
+def blas1_sweep(ctx, world, rank, sizes, warmup, reps_cap=200):
+    """The configs[4] sweep: per size, host-synchronous AXPY x += 2.5 y and DOT x.y
+    calls (JACC's synchronous constructs) on the paper's inputs
+    round(rand*100) (Fig. 2), each rank its own shard of n; the
+    seeded 2^24-element pattern is generated on the host and tiled ON THE DEVICE
+    (so n = 1e9 costs no 8 GB host copy).  Times: max over ranks.  DOT checked
+    against the exact integer (int64 closed form over the tiles) at every n."""
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+
+    import synth
+    P = 1 << 24
+    xb, yb = synth.jacc_vector(P, 42 + rank), synth.jacc_vector(P, 43 + rank)
+    xi, yi = xb.astype(np.int64), yb.astype(np.int64)
+    xb_d, yb_d = torch.from_numpy(xb).cuda(), torch.from_numpy(yb).cuda()
+    rows = []
+    for n in sizes:
+        reps_t, rem = divmod(n, P)
+        x = xb_d.repeat(reps_t + 1)[:n].contiguous()
+        y = yb_d.repeat(reps_t + 1)[:n].contiguous()
+        exact_dot = float(reps_t * int(np.dot(xi, yi)) + int(np.dot(xi[:rem], yi[:rem])))
+        torch.cuda.synchronize()
+        xp, yp = x.data_ptr(), y.data_ptr()   # raw pointers: no per-call torch sync
+        res0 = ctx.ddot(n, xp, yp)            # before any AXPY: the exact integer
+        reps = max(3, min(reps_cap, int(2e9 / (24 * n))))
+        for _ in range(warmup):
+            ctx.waxpby(n, 1.0, xp, 2.5, yp, xp)
+            ctx.ddot(n, xp, yp)
+        if world > 1:
+            dist.barrier()
+        t0 = time.perf_counter()
+        for _ in range(reps):
+            ctx.waxpby(n, 1.0, xp, 2.5, yp, xp)
+        t_axpy = (time.perf_counter() - t0) / reps
+        if world > 1:
+            dist.barrier()
+        t0 = time.perf_counter()
+        for _ in range(reps):
+            ctx.ddot(n, xp, yp)
+        t_dot = (time.perf_counter() - t0) / reps
+        tt = torch.tensor([t_axpy, t_dot], dtype=torch.float64, device="cuda")
+        if world > 1:
+            dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        t_axpy, t_dot = float(tt[0]), float(tt[1])
+        rows.append({"n_per_gpu": n, "axpy_us": round(t_axpy * 1e6, 2),
+                     "axpy_GBs": round(world * 24.0 * n / t_axpy / 1e9, 1),
+                     "dot_us": round(t_dot * 1e6, 2),
+                     "dot_GBs": round(world * 16.0 * n / t_dot / 1e9, 1),
+                     "dot_exact": (res0 == exact_dot) if world == 1 else None})
+        del x, y
+        torch.cuda.empty_cache()
+    del xb_d, yb_d
+    torch.cuda.empty_cache()
+    return rows
+
+
 def run_blas1(args):
     """BASELINE configs[4]: JACC BLAS-1 sweep, AXPY x += alpha y (hpccg_waxpby(n, 1, x,
     alpha, y, x)) and DOT (hpccg_ddot, host-synchronous like JACC's constructs)
@@ -885,51 +956,9 @@ def run_blas1(args):
     sizes = [10 ** k for k in range(3, 10)]
     if args.blas1_max:
         sizes = [s for s in sizes if s <= args.blas1_max]
-    rows = []
     clk = ClockSampler(local)
     clk.__enter__()
-    for n in sizes:
-        # seeded inputs generated once on the host (splitmix64), per-rank shard
-        gen = min(n, 1 << 24)
-        xh = synth.jacc_vector(gen, 42 + rank)
-        yh = synth.jacc_vector(gen, 43 + rank)
-        x = torch.from_numpy(np.resize(xh, n)).cuda() if n > gen else torch.from_numpy(xh).cuda()
-        y = torch.from_numpy(np.resize(yh, n)).cuda() if n > gen else torch.from_numpy(yh).cuda()
-        torch.cuda.synchronize()
-        xp, yp = x.data_ptr(), y.data_ptr()   # raw pointers: no per-call torch sync
-        reps = max(3, min(200, int(2e9 / (24 * n))))
-        for _ in range(args.warmup):
-            ctx.waxpby(n, 1.0, xp, 2.5, yp, xp)
-            ctx.ddot(n, xp, yp)
-        # AXPY, host-synchronous per call
-        if world > 1:
-            dist.barrier()
-        t0 = time.perf_counter()
-        for _ in range(reps):
-            ctx.waxpby(n, 1.0, xp, 2.5, yp, xp)
-        t_axpy = (time.perf_counter() - t0) / reps
-        if world > 1:
-            dist.barrier()
-        t0 = time.perf_counter()
-        for _ in range(reps):
-            res = ctx.ddot(n, xp, yp)
-        t_dot = (time.perf_counter() - t0) / reps
-        tt = torch.tensor([t_axpy, t_dot], dtype=torch.float64, device="cuda")
-        if world > 1:
-            dist.all_reduce(tt, op=dist.ReduceOp.MAX)
-        t_axpy, t_dot = float(tt[0]), float(tt[1])
-        # exactness: x stays integer-valued (multiples of 0.5 scaled) -> dot exact
-        xc = x.cpu().numpy()
-        exact = None
-        if world == 1 and n <= 10 ** 8:
-            exact = float(np.dot((2 * xc).astype(np.int64), y.cpu().numpy().astype(np.int64))) / 2
-        rows.append({"n_per_gpu": n, "axpy_us": round(t_axpy * 1e6, 2),
-                     "axpy_GBs": round(world * 24.0 * n / t_axpy / 1e9, 1),
-                     "dot_us": round(t_dot * 1e6, 2),
-                     "dot_GBs": round(world * 16.0 * n / t_dot / 1e9, 1),
-                     "dot_exact": (res == exact) if exact is not None else None})
-        del x, y
-        torch.cuda.empty_cache()
+    rows = blas1_sweep(ctx, world, rank, sizes, args.warmup)
     clk.__exit__(None, None, None)
     # f3: the 2-D constructs (Fig. 2) at SIZE x SIZE, SIZE = 1000 in the paper
     rows2d = []
