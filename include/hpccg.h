@@ -161,6 +161,15 @@ extern "C" {
                                6.84 TB/s where the plain SpMV reaches 7.11, which eats the
                                8n B saved (256^3: 977 vs 978 us/iteration; 128^3 122 vs 115);
                                1 on, -1 auto (on when the CG vectors exceed L2) */
+#define HPCCG_OPT_SPMV_TRIPS 26 /* single slab, finisher-free loop: 512-row trips per block of
+                               the CG SpMV (spmv27x2_trips_kernel; one p.Ap partial per block),
+                               so a slab with more than 4096 row blocks (256^3: 32768) needs no
+                               1024-thread p.Ap finisher kernel -- the update blocks sum the
+                               partials.  1 (default) off, 0 auto (the fewest trips that leave
+                               <= 4096 partials), T > 1 explicit.  Same Ap bits; the p.Ap sum
+                               takes another (fixed) tree.  Measured slower: 256^3 1066.7 (8
+                               trips) vs 984.7 us/iteration, 512^3 8593 vs 8019 -- a block's
+                               trips run back to back, so its loads drain between them */
 #define HPCCG_OPT_PS_LEAD 25 /* its production lead in chunks (0 default: plane/512 + 8) */
 #define HPCCG_OPT_PEER_TIMEOUT_MS 22 /* HALO_PEER waits: give up after this many milliseconds
                                (1 .. 3600000; default 30000 -- above any host-side skew

@@ -173,6 +173,7 @@ struct hpccg_problem {
     int64_t opt_peer_timeout_ms = 30000;  // give up a peer-memory wait after this long
     int opt_defer_x = -1;              // finisher-free loop: x update deferred into the p update (-1 auto)
     int opt_fuse_ps = 0;               // p update + SpMV in one pipelined kernel (-1 auto, 0 off, 1 on)
+    int opt_spmv_trips = 1;            // single-slab SpMV trips per block (0 auto, 1 off, T)
     int opt_ps_lead = 0;               // its production lead in chunks (0: plane / 512 + 8)
     std::vector<void *> ipc_opened;    // peers' buffers mapped with cudaIpcOpenMemHandle
     int last_persist_mode = 3;
@@ -666,6 +667,19 @@ int serpentine(const hpccg_problem *p) {
 // CG SpMV of every slab with the p.Ap epilogue.  Multi-slab: the rows that
 // do not touch a halo plane (interior) run first, overlapped with the halo
 // exchange on the comm stream (NCCL), then the two boundary planes.
+// HPCCG_OPT_SPMV_TRIPS: 512-row trips per block of the single-slab CG SpMV on
+// the finisher-free loop (spmv27x2_trips_kernel), so the update blocks can sum
+// the partials themselves (<= kUpdSumMax); 1: one trip (the finisher kernel
+// runs when the partials exceed kUpdSumMax)
+int spmv_trips(const hpccg_problem *p) {
+    const Slab &s = p->slabs[0];
+    if (p->ctx->mode != MODE_SINGLE || !ff_path(p) || s.dia || p->opt_spmv_trips == 1) return 1;
+    if (spmv_rows_per_thread(p->opt_rows, spmv_args(s, s.p, s.Ap), 0, 0) != 2) return 1;
+    const int64_t blocks = spmv_blocks(s.n, 2);
+    if (p->opt_spmv_trips > 1) return p->opt_spmv_trips;
+    return blocks > kUpdSumMax ? (int)cdiv(blocks, kUpdSumMax) : 1;
+}
+
 int cg_spmv_all(hpccg_problem *p, bool timing, bool check) {
     hpccg_ctx *ctx = p->ctx;
     const int minb = p->opt_minb;
@@ -679,6 +693,16 @@ int cg_spmv_all(hpccg_problem *p, bool timing, bool check) {
         a.total_blocks = (unsigned)spmv_blocks(s.n, rows);
         a.parts_only = s.spmv_parts;  // the update kernel finishes p.Ap
         a.rev = ff_path(p) && (serpentine(p) & 2);
+        const int trips = spmv_trips(p);
+        if (trips > 1) {
+            a.r0 = 0;
+            a.len0 = s.n;
+            a.trips = trips;
+            const unsigned g = (unsigned)cdiv(spmv_blocks(s.n, 2), trips);
+            if (check) launch_k(p->opt_pdl != 0, spmv27x2_trips_kernel<true>, dim3(g), ctx->stream, a);
+            else launch_k(p->opt_pdl != 0, spmv27x2_trips_kernel<false>, dim3(g), ctx->stream, a);
+            return check_launch(ctx);
+        }
         return launch_spmv<1>(ctx, minb, check, a, 0, s.n, 0, 0, ctx->stream, rows,
                                  p->opt_pdl != 0);
     }
@@ -712,6 +736,8 @@ double **tab(hpccg_problem *p, int which) { return p->d_tab + (size_t)which * p-
 
 // SpMV partial count of a single slab's CG SpMV (the update sums them).
 unsigned single_spmv_parts(const hpccg_problem *p, const Slab &s) {
+    const int trips = spmv_trips(p);
+    if (trips > 1) return (unsigned)cdiv(spmv_blocks(s.n, 2), trips);
     return (unsigned)spmv_blocks(s.n, spmv_rows_per_thread(p->opt_rows, spmv_args(s, s.p, s.Ap), 0, 0));
 }
 
@@ -2441,6 +2467,13 @@ int hpccg_set_option(hpccg_problem *p, int key, int64_t value) {
             if (value < 0 || value > 2) return fail(HPCCG_EINVAL, "halo peer: 0, 1 or 2");
             if (value && p->ctx->mode != MODE_SINGLE && !p->slabs[0].ptab) CHECK(enable_peer(p));
             p->opt_peer = (int)value;
+            return HPCCG_OK;
+        case HPCCG_OPT_SPMV_TRIPS:
+            if (value < 0 || value > 4096) return fail(HPCCG_EINVAL, "spmv trips: 0 (auto), 1 (off) .. 4096");
+            if (p->graph) cudaGraphExecDestroy(p->graph);
+            if (p->wgraph) cudaGraphExecDestroy(p->wgraph);
+            p->graph = p->wgraph = nullptr;
+            p->opt_spmv_trips = (int)value;
             return HPCCG_OK;
         case HPCCG_OPT_FUSE_PSPMV:
             if (value < -1 || value > 1) return fail(HPCCG_EINVAL, "fuse pspmv: -1 (auto), 0 or 1");

@@ -526,6 +526,7 @@ struct SpmvArgs {
                        // (same rows per block, same partials: identical bits)
     int nx;            // kDia (HPCCG_OPT_SPMV_FORMAT 1): row stride of the grid
     int dia;           // 1: spmv27x2_kernel<., ., false, true> (DIA-27, col[] not read)
+    int trips;         // spmv27x2_trips_kernel: 512-row trips per block (one partial per block)
 };
 
 // the row block this CTA handles (HPCCG_OPT_SERPENTINE)
@@ -825,6 +826,86 @@ __device__ __forceinline__ void spmv27x2_body(const SpmvArgs &a, int64_t row, in
     }
 }
 
+
+// Single slab, p.Ap partials for the finisher-free update (HPCCG_OPT_SPMV_TRIPS):
+// each block SpMVs `trips` consecutive 512-row trips (range 0 only) and writes
+// ONE partial, so a large slab (256^3: 32768 row blocks) leaves <= 4096
+// partials, which every update block sums itself -- no 1024-thread p.Ap
+// finisher kernel between the SpMV and the update.  Per row the same FMA chain
+// as spmv27x2_kernel (identical Ap bits); the partial tree differs (the sum
+// goes trip by trip per thread, then the block).
+template <bool kCheck>
+__global__ void __launch_bounds__(kBlock, 4) spmv27x2_trips_kernel(SpmvArgs a) {
+    const int64_t bid = spmv_bid(a);
+    const int64_t lim = a.r0 + a.len0;
+    const uint64_t pol = policy_evict_first();
+    double d = 0.0;
+    for (int t = 0; t < a.trips; ++t) {
+        const int64_t row = a.r0 + ((bid * a.trips + t) * kBlock + threadIdx.x) * 2;
+        if (row >= lim) {
+            if (t == 0) {
+                pdl_wait();
+                if (spmv_done<1, kCheck>(a)) return;
+            }
+            break;
+        }
+        if (row + 1 < lim) {
+            const double *v = a.val + row;
+            const int *c = a.col + row;
+            double s0 = 0.0, s1 = 0.0, x0 = 0.0, x1 = 0.0;
+            int c0 = 0, c1 = 0;
+#pragma unroll
+            for (int g = 0; g < kSlots / 3; ++g) {
+                double2 vv[3];
+                int2 cc[3];
+#pragma unroll
+                for (int u = 0; u < 3; ++u) {
+                    vv[u] = ld_stream2(v + (3 * g + u) * a.stride, pol);
+                    cc[u] = ld_stream2(c + (3 * g + u) * a.stride, pol);
+                }
+                if (t == 0 && g == 0) {
+                    pdl_wait();
+                    if (a.early_trigger) pdl_trigger();
+                    if (a.trace) trace_mark(a.trace, a.trace_max, ldg_o(&a.sc->k), 1, false);
+                    if (spmv_done<1, kCheck>(a)) return;  // uniform, before any store
+                }
+#pragma unroll
+                for (int u = 0; u < 3; ++u) {
+                    const double xa = __ldg(a.x + cc[u].x), xb = __ldg(a.x + cc[u].y);
+                    if (3 * g + u == kDiagSlot) {
+                        x0 = xa;
+                        x1 = xb;
+                        c0 = cc[u].x;
+                        c1 = cc[u].y;
+                    }
+                    s0 = fma(vv[u].x, xa, s0);
+                    s1 = fma(vv[u].y, xb, s1);
+                }
+            }
+            *reinterpret_cast<double2 *>(a.y + row) = make_double2(s0, s1);
+            const double p0 = c0 == row + a.plane ? x0 : __ldg(a.x + row + a.plane);
+            const double p1 = c1 == row + 1 + a.plane ? x1 : __ldg(a.x + row + 1 + a.plane);
+            d = fma(s1, p1, fma(s0, p0, d));
+        } else {  // odd tail: one row
+            if (t == 0) {
+                pdl_wait();
+                if (spmv_done<1, kCheck>(a)) return;
+            }
+            double s0 = 0.0;
+#pragma unroll
+            for (int k = 0; k < kSlots; ++k)
+                s0 = fma(ld_stream(a.val + k * a.stride + row, pol),
+                         __ldg(a.x + ld_stream(a.col + k * a.stride + row, pol)), s0);
+            a.y[row] = s0;
+            d = fma(s0, __ldg(a.x + row + a.plane), d);
+        }
+    }
+    pdl_trigger();
+    if (a.trace) trace_mark(a.trace, a.trace_max, ldg_o(&a.sc->k), 1, true);
+    __shared__ double shp[32];
+    d = block_reduce<false>(d, shp);
+    if (threadIdx.x == 0) a.parts_only[a.part_base + bid] = d;
+}
 
 template <int kDots, bool kCheck, bool kFused = false, bool kDia = false>
 __global__ void __launch_bounds__(kBlock, kDia ? kDiaMinB : 4) spmv27x2_kernel(SpmvArgs a) {

@@ -1123,3 +1123,24 @@ def test_fused_pspmv_spmv_bitwise_vs_oracle(ctx):
         ref = oracle.generate(*dims)
         o = oracle.cg(ref, 2, 0.0)
         np.testing.assert_array_equal(x1, o["x"])
+
+
+@pytest.mark.parametrize("dims,trips", [((64, 64, 64), 3), ((48, 16, 50), 0), ((31, 17, 10), 2)])
+def test_spmv_trips_option_parity(ctx, dims, trips):
+    """HPCCG_OPT_SPMV_TRIPS (opt-in): multi-trip SpMV blocks, one p.Ap partial
+    per block -- another fixed reduction tree, so the CG is held to the oracle
+    tolerance (niters +-1, 1e-10) and is run-to-run deterministic."""
+    with H.Problem(ctx, *dims) as p:
+        p.set_option(H.HPCCG_OPT_PERSISTENT, 0)
+        p.set_option(H.HPCCG_OPT_SPMV_TRIPS, trips)
+        ref = oracle.generate(*dims)
+        oref = oracle.cg(ref, 150, 1e-12)
+        outs = []
+        for _ in range(2):
+            p.set_vec(H.HPCCG_VEC_X, np.zeros(p.n))
+            r = p.solve(150, 1e-12)
+            outs.append((r["niters"], r["normr"], p.get_vec(H.HPCCG_VEC_X)))
+            check_cg(r, p.maxabsdiff(), oref, ref)
+        assert outs[0][:2] == outs[1][:2]
+        np.testing.assert_array_equal(outs[0][2], outs[1][2])
+        p.set_option(H.HPCCG_OPT_SPMV_TRIPS, 1)
