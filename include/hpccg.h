@@ -170,6 +170,12 @@ extern "C" {
                                takes another (fixed) tree.  Measured slower: 256^3 1066.7 (8
                                trips) vs 984.7 us/iteration, 512^3 8593 vs 8019 -- a block's
                                trips run back to back, so its loads drain between them */
+#define HPCCG_OPT_PAP_CLUSTER 27 /* p.Ap finisher of a slab whose SpMV leaves more than 4096
+                               partials (256^3: 32768): 0 one 1024-thread CTA, 1 one cluster of 8
+                               CTAs reading the partials in parallel (distributed shared memory
+                               for the 8 CTA sums).  Every mode of a problem uses the same one
+                               (identical bits across modes); the two differ in the last bits.
+                               Measured no faster (256^3 986.3 vs 986.0 us/iteration): default 0 */
 #define HPCCG_OPT_PS_LEAD 25 /* its production lead in chunks (0 default: plane/512 + 8) */
 #define HPCCG_OPT_PEER_TIMEOUT_MS 22 /* HALO_PEER waits: give up after this many milliseconds
                                (1 .. 3600000; default 30000 -- above any host-side skew

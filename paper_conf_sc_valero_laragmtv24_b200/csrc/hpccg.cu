@@ -174,6 +174,7 @@ struct hpccg_problem {
     int opt_defer_x = -1;              // finisher-free loop: x update deferred into the p update (-1 auto)
     int opt_fuse_ps = 0;               // p update + SpMV in one pipelined kernel (-1 auto, 0 off, 1 on)
     int opt_spmv_trips = 1;            // single-slab SpMV trips per block (0 auto, 1 off, T)
+    int opt_pap_cluster = 0;           // p.Ap finisher as one 8-CTA cluster (1) or one CTA (0)
     int opt_ps_lead = 0;               // its production lead in chunks (0: plane / 512 + 8)
     std::vector<void *> ipc_opened;    // peers' buffers mapped with cudaIpcOpenMemHandle
     int last_persist_mode = 3;
@@ -253,6 +254,33 @@ cudaError_t launch_k(bool pdl, void (*kernel)(KArgs...), dim3 grid, cudaStream_t
     cfg.attrs = pdl ? at : nullptr;
     cfg.numAttrs = pdl ? 1 : 0;
     return cudaLaunchKernelEx(&cfg, kernel, std::forward<Args>(args)...);
+}
+
+// the p.Ap finisher of a slab whose SpMV left more than kUpdSumMax partials:
+// one 1024-thread CTA, or (HPCCG_OPT_PAP_CLUSTER) a cluster of kPapCl CTAs
+int launch_pap_finish(hpccg_ctx *ctx, int cluster, const double *parts, unsigned np, CgScalars *sc, bool pdl) {
+    cudaLaunchConfig_t cfg{};
+    cfg.gridDim = dim3(cluster ? kPapCl : 1);
+    cfg.blockDim = dim3(1024);
+    cfg.stream = ctx->stream;
+    cudaLaunchAttribute at[2];
+    int na = 0;
+    if (pdl) {
+        at[na].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+        at[na++].val.programmaticStreamSerializationAllowed = 1;
+    }
+    if (cluster) {
+        at[na].id = cudaLaunchAttributeClusterDimension;
+        at[na].val.clusterDim.x = kPapCl;
+        at[na].val.clusterDim.y = 1;
+        at[na++].val.clusterDim.z = 1;
+    }
+    cfg.attrs = na ? at : nullptr;
+    cfg.numAttrs = na;
+    void (*fk)(const double *, unsigned, CgScalars *) = cluster ? cg_pap_finish_cl_kernel : cg_pap_finish_kernel;
+    const cudaError_t e = cudaLaunchKernelEx(&cfg, fk, parts, np, sc);
+    if (e != cudaSuccess) return fail(HPCCG_ECUDA, "p.Ap finisher launch: %s", cudaGetErrorString(e));
+    return check_launch(ctx);
 }
 
 template <class K>
@@ -569,7 +597,7 @@ int launch_update_u(hpccg_ctx *ctx, int waves, int unroll, int64_t cap, const Up
 }
 
 int launch_update(hpccg_ctx *ctx, int waves, int unroll, int64_t cap, const Slab &s, int single,
-                  bool check, unsigned long long cond, bool pdl, int rows) {
+                  bool check, unsigned long long cond, bool pdl, int rows, int pap_cluster) {
     UpdArgs a{};
     a.n = s.n;
     a.x = s.x;
@@ -588,19 +616,8 @@ int launch_update(hpccg_ctx *ctx, int waves, int unroll, int64_t cap, const Slab
         if (np <= kUpdSumMax) {  // every update block sums them
             a.pAp_parts = s.spmv_parts;
             a.n_parts = np;
-        } else {  // one finisher block, then the update reads sc->pAp
-            void (*fk)(const double *, unsigned, CgScalars *) = cg_pap_finish_kernel;
-            cudaLaunchConfig_t cfg{};
-            cfg.gridDim = dim3(1);
-            cfg.blockDim = dim3(1024);
-            cfg.stream = ctx->stream;
-            cudaLaunchAttribute at[1];
-            at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-            at[0].val.programmaticStreamSerializationAllowed = 1;
-            cfg.attrs = pdl ? at : nullptr;
-            cfg.numAttrs = pdl ? 1 : 0;
-            cudaLaunchKernelEx(&cfg, fk, (const double *)s.spmv_parts, np, s.sc);
-            CHECK(check_launch(ctx));
+        } else {  // the finisher writes sc->pAp, then the update reads it
+            CHECK(launch_pap_finish(ctx, pap_cluster, s.spmv_parts, np, s.sc, pdl));
         }
     }
     const bool vec = aligned16(a.x) && aligned16(a.r) && aligned16(a.p) && aligned16(a.Ap);
@@ -1028,9 +1045,7 @@ int enqueue_iteration_ff_u(hpccg_problem *p, bool timing, bool check, unsigned l
     if (pre) {
         if (np > kUpdSumMax)
             for (const Slab &s : p->slabs) {  // sc->pAp = the slab's sum, then post it
-                launch_kb(pdl, cg_pap_finish_kernel, dim3(1), dim3(1024), ctx->stream,
-                          (const double *)s.spmv_parts, np, s.sc);
-                CHECK(check_launch(ctx));
+                CHECK(launch_pap_finish(ctx, p->opt_pap_cluster, s.spmv_parts, np, s.sc, pdl));
             }
         for (const Slab &s : p->slabs)
             CHECK(post(s, np <= kUpdSumMax ? s.spmv_parts : nullptr, np, 1));
@@ -1056,19 +1071,8 @@ int enqueue_iteration_ff_u(hpccg_problem *p, bool timing, bool check, unsigned l
             a.pAp_parts = s.spmv_parts;
             a.n_parts = np;
         } else if (pre) {  // finished and posted below, ahead of every update
-        } else {  // one finisher block writes the slab's p.Ap into sc->pAp
-            void (*fk)(const double *, unsigned, CgScalars *) = cg_pap_finish_kernel;
-            cudaLaunchConfig_t cfg{};
-            cfg.gridDim = dim3(1);
-            cfg.blockDim = dim3(1024);
-            cfg.stream = ctx->stream;
-            cudaLaunchAttribute at[1];
-            at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-            at[0].val.programmaticStreamSerializationAllowed = 1;
-            cfg.attrs = pdl ? at : nullptr;
-            cfg.numAttrs = pdl ? 1 : 0;
-            CU(cudaLaunchKernelEx(&cfg, fk, (const double *)s.spmv_parts, np, s.sc));
-            CHECK(check_launch(ctx));
+        } else {  // the finisher writes the slab's p.Ap into sc->pAp
+            CHECK(launch_pap_finish(ctx, p->opt_pap_cluster, s.spmv_parts, np, s.sc, pdl));
         }
         launch_k(pdl, upd, dim3(ug), ctx->stream, a);
         CHECK(check_launch(ctx));
@@ -1107,7 +1111,7 @@ int enqueue_iteration(hpccg_problem *p, bool timing, bool check, unsigned long l
         // while-graph condition
         for (size_t i = 0; i < p->slabs.size(); ++i)
             CHECK(launch_update(ctx, p->opt_vec_waves, p->opt_unroll, p->red_cap, p->slabs[i],
-                                single, check, i == 0 ? cond : 0ull, pdl, p->opt_rows));
+                                single, check, i == 0 ? cond : 0ull, pdl, p->opt_rows, p->opt_pap_cluster));
     }
     CHECK(allreduce_cg(p, true, timing));
     return HPCCG_OK;
@@ -2467,6 +2471,13 @@ int hpccg_set_option(hpccg_problem *p, int key, int64_t value) {
             if (value < 0 || value > 2) return fail(HPCCG_EINVAL, "halo peer: 0, 1 or 2");
             if (value && p->ctx->mode != MODE_SINGLE && !p->slabs[0].ptab) CHECK(enable_peer(p));
             p->opt_peer = (int)value;
+            return HPCCG_OK;
+        case HPCCG_OPT_PAP_CLUSTER:
+            if (value != 0 && value != 1) return fail(HPCCG_EINVAL, "pap cluster: 0 or 1");
+            if (p->graph) cudaGraphExecDestroy(p->graph);
+            if (p->wgraph) cudaGraphExecDestroy(p->wgraph);
+            p->graph = p->wgraph = nullptr;
+            p->opt_pap_cluster = (int)value;
             return HPCCG_OK;
         case HPCCG_OPT_SPMV_TRIPS:
             if (value < 0 || value > 4096) return fail(HPCCG_EINVAL, "spmv trips: 0 (auto), 1 (off) .. 4096");

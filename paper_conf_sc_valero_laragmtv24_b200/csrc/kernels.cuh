@@ -1047,6 +1047,52 @@ __device__ __forceinline__ void set_cond(unsigned long long h, int cont) {
 // update block to sum them (> kUpdSumMax): one 1024-thread block, fixed order.
 constexpr unsigned kUpdSumMax = 4096;
 
+// The same sum over kPapCl CTAs of one thread-block cluster: CTA c reduces the
+// c-th contiguous share of the partials (8 independent loads in flight per
+// thread), the leader adds the kPapCl CTA sums in rank order from distributed
+// shared memory.  32768 partials (256^3) are 256 KB: one SM's L2 bandwidth and
+// latency set the single-CTA finisher's ~5.3 us; eight SMs read them in
+// parallel.  Deterministic (fixed shares and order), another tree than
+// cg_pap_finish_kernel's.
+constexpr int kPapCl = 8;
+__global__ void __launch_bounds__(1024, 1) cg_pap_finish_cl_kernel(const double *parts, unsigned n_parts,
+                                                                CgScalars *sc) {
+    namespace cgx = cooperative_groups;
+    pdl_wait();
+    pdl_trigger();
+    __shared__ double sh[32];
+    __shared__ double s_res;
+    auto cl = cgx::this_cluster();
+    const unsigned rank = cl.block_rank();
+    const unsigned share = (n_parts + kPapCl - 1) / kPapCl;
+    const unsigned lo = rank * share, hi = min(n_parts, lo + share);
+    double acc[8] = {0.0, 0.0, 0.0, 0.0, 0.0, 0.0, 0.0, 0.0};
+    unsigned i = lo + threadIdx.x;
+    for (; i + 7u * 1024u < hi; i += 8u * 1024u) {
+        double v[8];
+#pragma unroll
+        for (int u = 0; u < 8; ++u) v[u] = ldg_o(parts + i + u * 1024u);
+#pragma unroll
+        for (int u = 0; u < 8; ++u) acc[u] += v[u];
+    }
+    for (; i < hi; i += 1024) acc[0] += ldg_o(parts + i);
+    double q = ((acc[0] + acc[1]) + (acc[2] + acc[3])) + ((acc[4] + acc[5]) + (acc[6] + acc[7]));
+    q = warp_sum(q);
+    if ((threadIdx.x & 31) == 0) sh[threadIdx.x >> 5] = q;
+    __syncthreads();
+    if (threadIdx.x < 32) {
+        q = warp_sum(sh[threadIdx.x]);
+        if (threadIdx.x == 0) s_res = q;
+    }
+    cl.sync();
+    if (rank == 0 && threadIdx.x == 0) {
+        double t = 0.0;
+        for (int c = 0; c < kPapCl; ++c) t += *cl.map_shared_rank(&s_res, c);
+        sc->pAp = t;
+    }
+    cl.sync();  // the leader has read every CTA's s_res before any CTA exits
+}
+
 __global__ void __launch_bounds__(1024, 1) cg_pap_finish_kernel(const double *parts, unsigned n_parts,
                                                              CgScalars *sc) {
     pdl_wait();

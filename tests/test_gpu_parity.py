@@ -1144,3 +1144,25 @@ def test_spmv_trips_option_parity(ctx, dims, trips):
         assert outs[0][:2] == outs[1][:2]
         np.testing.assert_array_equal(outs[0][2], outs[1][2])
         p.set_option(H.HPCCG_OPT_SPMV_TRIPS, 1)
+
+
+def test_pap_cluster_finisher(ctx):
+    """HPCCG_OPT_PAP_CLUSTER (opt-in): the p.Ap finisher as one 8-CTA cluster.
+    A slab with > 4096 SpMV row blocks (128x128x160: 5120) takes the finisher;
+    both finishers give a converged solve with SURVEY-consistent iterations, and
+    with the cluster finisher every launch mode gives the same bits."""
+    with H.Problem(ctx, 128, 128, 160) as p:
+        outs = {}
+        for cl in (0, 1):
+            p.set_option(H.HPCCG_OPT_PAP_CLUSTER, cl)
+            for mode in ("while", "timing"):
+                p.set_option(H.HPCCG_OPT_TIMING, 1 if mode == "timing" else 0)
+                p.set_vec(H.HPCCG_VEC_X, np.zeros(p.n))
+                r = p.solve(150, 1e-12)
+                outs[(cl, mode)] = (r["niters"], r["normr"], p.maxabsdiff())
+        p.set_option(H.HPCCG_OPT_TIMING, 0)
+        p.set_option(H.HPCCG_OPT_PAP_CLUSTER, 0)
+        assert outs[(1, "while")] == outs[(1, "timing")]
+        assert outs[(0, "while")] == outs[(0, "timing")]
+        assert abs(outs[(1, "while")][0] - outs[(0, "while")][0]) <= 1
+        assert outs[(1, "while")][2] < 1e-13 and outs[(1, "while")][1] <= 1e-12
