@@ -194,6 +194,7 @@ struct hpccg_problem {
     std::vector<TimedOp> timed;
     cudaEvent_t ev_t0 = nullptr, ev_t1 = nullptr;
     int *h_done = nullptr;  // pinned poll flags [2]
+    CgScalars *h_sc = nullptr;  // pinned copy of slab 0's scalars at the end of a solve
     cudaEvent_t ev_poll[2] = {nullptr, nullptr};
     hpccg_stats stats{};
 };
@@ -2788,6 +2789,9 @@ int hpccg_solve(hpccg_problem *p, int max_iter, double tol, int *niters, double 
         CHECK(enqueue_xfix(p));
     }
     CU(cudaEventRecord(p->ev_t1, ctx->stream));
+    // the loop state comes back in the same synchronisation as the solve
+    if (!p->h_sc) CU(cudaMallocHost((void **)&p->h_sc, sizeof(CgScalars)));
+    CU(cudaMemcpyAsync(p->h_sc, p->slabs[0].sc, sizeof(CgScalars), cudaMemcpyDeviceToHost, ctx->stream));
     CU(cudaStreamSynchronize(ctx->stream));
     CU(cudaGetLastError());
     l2win.release();
@@ -2802,8 +2806,7 @@ int hpccg_solve(hpccg_problem *p, int max_iter, double tol, int *niters, double 
             }
         }
 
-    CgScalars hs;
-    CU(cudaMemcpy(&hs, p->slabs[0].sc, sizeof hs, cudaMemcpyDeviceToHost));
+    const CgScalars hs = *p->h_sc;
     hpccg_stats st{};
     float ms = 0.f;
     CU(cudaEventElapsedTime(&ms, p->ev_t0, p->ev_t1));
@@ -2874,6 +2877,7 @@ void hpccg_free(hpccg_problem *p) {
     if (p->ev_poll[0]) cudaEventDestroy(p->ev_poll[0]);
     if (p->ev_poll[1]) cudaEventDestroy(p->ev_poll[1]);
     if (p->h_done) cudaFreeHost(p->h_done);
+    if (p->h_sc) cudaFreeHost(p->h_sc);
     delete p;
 }
 
