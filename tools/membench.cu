@@ -77,6 +77,31 @@ __global__ void __launch_bounds__(256) upd_kernel(double2 *__restrict__ x, doubl
     }
 }
 
+// p-update-like with the deferred x update: read r, p, x; write p, x (3R:2W)
+template <int kU>
+__global__ void __launch_bounds__(256) pupd_kernel(const double2 *__restrict__ r, double2 *__restrict__ p,
+                                                   double2 *__restrict__ x, int64_t n2, double be, double al) {
+    const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const int64_t nth = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t b = tid; b < n2; b += kU * nth) {
+        double2 ra[kU], pa[kU], xa[kU];
+#pragma unroll
+        for (int u = 0; u < kU; ++u) {
+            const int64_t i = b + u * nth;
+            if (i < n2) { ra[u] = r[i]; pa[u] = p[i]; xa[u] = x[i]; }
+        }
+#pragma unroll
+        for (int u = 0; u < kU; ++u) {
+            const int64_t i = b + u * nth;
+            if (i < n2) {
+                xa[u].x += al * pa[u].x; xa[u].y += al * pa[u].y;
+                p[i] = make_double2(ra[u].x + be * pa[u].x, ra[u].y + be * pa[u].y);
+                x[i] = xa[u];
+            }
+        }
+    }
+}
+
 template <class F>
 float timeit(F f, int reps) {
     cudaEvent_t e0, e1;
@@ -127,6 +152,26 @@ int main() {
     printf("{\"probe\": \"copy\", \"bytes\": %zu, \"ms\": %.4f, \"GBs\": %.1f}\n", 2 * big, ms, 2 * big / ms / 1e6);
     ms = timeit([&] { triad_kernel<<<grid, 256>>>(a, b, c, n2); }, 10);
     printf("{\"probe\": \"triad_2r1w\", \"bytes\": %zu, \"ms\": %.4f, \"GBs\": %.1f}\n", 3 * big, ms, 3 * big / ms / 1e6);
+    // the 256^3 CG vectors (n = 2^24 doubles = 128 MiB each): p update with the
+    // deferred x (3R:2W), one persistent wave x kU units vs a full grid
+    {
+        const int64_t m2 = ((int64_t)1 << 24) / 2;
+        double2 *r = a, *pp = b, *xx = c;
+        int o1, o4;
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o1, pupd_kernel<1>, 256, 0);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o4, pupd_kernel<4>, 256, 0);
+        const double bytes = 5.0 * 16 * m2;
+        for (int rep = 0; rep < 2; ++rep) {
+            ms = timeit([&] { pupd_kernel<1><<<(unsigned)((m2 + 255) / 256), 256>>>(r, pp, xx, m2, 0.5, 0.25); }, 10);
+            printf("{\"probe\": \"pupd_3r2w_fullgrid\", \"us\": %.2f, \"GBs\": %.1f}\n", ms * 1e3, bytes / ms / 1e6);
+            ms = timeit([&] { pupd_kernel<4><<<sms * o4, 256>>>(r, pp, xx, m2, 0.5, 0.25); }, 10);
+            printf("{\"probe\": \"pupd_3r2w_wave_u4\", \"us\": %.2f, \"GBs\": %.1f}\n", ms * 1e3, bytes / ms / 1e6);
+            ms = timeit([&] { pupd_kernel<1><<<sms * o1, 256>>>(r, pp, xx, m2, 0.5, 0.25); }, 10);
+            printf("{\"probe\": \"pupd_3r2w_wave_u1\", \"us\": %.2f, \"GBs\": %.1f}\n", ms * 1e3, bytes / ms / 1e6);
+            ms = timeit([&] { pupd_kernel<2><<<sms * o4 * 2, 256>>>(r, pp, xx, m2, 0.5, 0.25); }, 10);
+            printf("{\"probe\": \"pupd_3r2w_2waves_u2\", \"us\": %.2f, \"GBs\": %.1f}\n", ms * 1e3, bytes / ms / 1e6);
+        }
+    }
     // L2-resident re-reads: 16, 32, 64 MB
     for (size_t mb : {16, 32, 64, 96}) {
         const size_t bytes = mb << 20;
