@@ -94,9 +94,15 @@ def full(rep):
     return res
 
 
+# the x update is deferred into the p update when the CG vectors exceed L2
+# (HPCCG_OPT_DEFER_X auto: 256^3 and 512^3): x/r update 24n, p update 40n
+DEFER = {"hpccg256": True, "hpccg512s": True, "hpccg128": False, "hpccg20": False}
+
+
 def per_kernel(rows, n, nnz):
-    alg = {"spmv27x2_kernel": 12.0 * nnz + 16.0 * n, "cg_update1_kernel": 48.0 * n,
-           "cg_pupdate1_kernel": 24.0 * n}
+    d = DEFER.get(W, False)
+    alg = {"spmv27x2_kernel": 12.0 * nnz + 16.0 * n, "cg_update1_kernel": (24.0 if d else 48.0) * n,
+           "cg_pupdate1_kernel": (40.0 if d else 24.0) * n}
     out = {}
     for d in rows:
         name = next((k for k in alg if k in d["kernel"]), None)
