@@ -1166,3 +1166,27 @@ def test_pap_cluster_finisher(ctx):
         assert outs[(0, "while")] == outs[(0, "timing")]
         assert abs(outs[(1, "while")][0] - outs[(0, "while")][0]) <= 1
         assert outs[(1, "while")][2] < 1e-13 and outs[(1, "while")][1] <= 1e-12
+
+
+# ------------- the scaling configurations' GLOBAL problems on one GPU (loopback)
+
+@pytest.mark.parametrize("P,nz,expect", [(2, 256, 113), (4, 256, 114), (8, 256, 115), (8, 64, 115)])
+def test_scaling_configs_global_problem_loopback(P, nz, expect):
+    """configs[2] (256^3 per GPU, weak) at P = 2 / 4 / 8 and configs[3] (512^3
+    global, strong) at P = 8, each as P slabs of 256^2 x nz (512^2 x 64 for the
+    strong split) in ONE process, through the multi-GPU default exchange (the
+    halo push and the scalar allreduces fused into the CG kernels, HALO_PEER 2,
+    deferred x update): the global tol 1e-12 solve must take SURVEY's
+    independently computed iteration count (+-1) and reach max|x - 1| < 1e-13.
+    Up to 134M rows / 3.6G stored entries -- the exact P = 8 problems."""
+    nx = 512 if nz == 64 else 256
+    with H.Context(0, nranks=P, loopback=True) as c, H.Problem(c, nx, nx, nz) as p:
+        assert p.info["nrow_global"] == nx * nx * nz * P
+        nzg = nz * P
+        assert p.info["nnz_global"] == (3 * nx - 2) * (3 * nx - 2) * (3 * nzg - 2)
+        p.set_option(H.HPCCG_OPT_HALO_PEER, 2)
+        r = p.solve(150, 1e-12)
+        assert abs(r["niters"] - expect) <= 1, r
+        assert r["normr"] <= 1e-12
+        assert p.maxabsdiff() < 1e-13
+        assert p.stats()["x_deferred"] == 1
