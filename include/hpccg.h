@@ -176,6 +176,17 @@ extern "C" {
                                for the 8 CTA sums).  Every mode of a problem uses the same one
                                (identical bits across modes); the two differ in the last bits.
                                Measured no faster (256^3 986.3 vs 986.0 us/iteration): default 0 */
+#define HPCCG_OPT_SPMV_SLICED 28 /* single slab, finisher-free loop: the CG SpMV reads a
+                               CHUNK-SLICED copy of the matrix (128 rows' val[27][128] +
+                               col[27][128] contiguous, built from the slot-major ELL at
+                               generate time; 324 B per row of extra HBM) with ONE TMA bulk copy
+                               per chunk into a two-stage shared-memory ring per persistent CTA
+                               (spmv_sliced_kernel); same Ap bits; one p.Ap partial per CTA, so
+                               no p.Ap finisher kernel.  0 (default) off; 1 on (allocates and
+                               fills the copy); -1 auto (on when the CG vectors exceed L2).
+                               Measured on two boxes: 256^3 971 / 977 vs 985 / 979
+                               us/iteration, 512^3 7880 / 8048 vs 8014 / 7968 -- a gain on one
+                               box, noise or a loss on the other, so not the default */
 #define HPCCG_OPT_PS_LEAD 25 /* its production lead in chunks (0 default: plane/512 + 8) */
 #define HPCCG_OPT_PEER_TIMEOUT_MS 22 /* HALO_PEER waits: give up after this many milliseconds
                                (1 .. 3600000; default 30000 -- above any host-side skew

@@ -129,6 +129,7 @@ struct Slab {
     int early_trigger = 1;      // HPCCG_OPT_PDL 1: SpMV triggers its successor early
     int nx = 0;                 // grid row stride (DIA-27 column formation)
     int dia = 0;                // HPCCG_OPT_SPMV_FORMAT 1: DIA-27 SpMV (col[] not read)
+    unsigned char *sl = nullptr;  // HPCCG_OPT_SPMV_SLICED: chunk-sliced copy of the ELL (324 B per row)
     // HPCCG_OPT_FUSE_PSPMV: ticket counter, error word, per-chunk flags
     unsigned char *ps_mem = nullptr;
     unsigned *ps_ticket = nullptr;
@@ -175,6 +176,7 @@ struct hpccg_problem {
     int opt_fuse_ps = 0;               // p update + SpMV in one pipelined kernel (-1 auto, 0 off, 1 on)
     int opt_spmv_trips = 1;            // single-slab SpMV trips per block (0 auto, 1 off, T)
     int opt_pap_cluster = 0;           // p.Ap finisher as one 8-CTA cluster (1) or one CTA (0)
+    int opt_sliced = 0;                // CG SpMV from the chunk-sliced copy via TMA (-1 auto, 0, 1)
     int opt_ps_lead = 0;               // its production lead in chunks (0: plane / 512 + 8)
     std::vector<void *> ipc_opened;    // peers' buffers mapped with cudaIpcOpenMemHandle
     int last_persist_mode = 3;
@@ -685,6 +687,54 @@ int serpentine(const hpccg_problem *p) {
 // CG SpMV of every slab with the p.Ap epilogue.  Multi-slab: the rows that
 // do not touch a halo plane (interior) run first, overlapped with the halo
 // exchange on the comm stream (NCCL), then the two boundary planes.
+// HPCCG_OPT_SPMV_SLICED: the single-slab CG SpMV (finisher-free loop) reads the
+// chunk-sliced copy through TMA (spmv_sliced_kernel); auto = when the CG
+// vectors exceed L2 (256^3 and up), where the copy's 324 B per row of extra HBM
+// is cheap next to 180 GB
+bool sliced_wanted(const hpccg_problem *p) {
+    if (p->ctx->mode != MODE_SINGLE || p->opt_sliced == 0) return false;
+    return p->opt_sliced == 1 || p->slabs[0].arena_bytes > ((size_t)126 << 20);
+}
+
+bool sliced_on(const hpccg_problem *p) {
+    const Slab &s = p->slabs[0];
+    return sliced_wanted(p) && s.sl && !s.dia && ff_path(p);
+}
+
+int alloc_zero(void **ptr, size_t bytes);
+
+// allocate and fill the sliced copy (never during a graph capture: called at
+// generate / set_option time)
+int sliced_alloc(hpccg_problem *p) {
+    Slab &s = p->slabs[0];
+    if (s.sl || !sliced_wanted(p)) return HPCCG_OK;
+    const int64_t nch = cdiv(s.n, kSlR);
+    CHECK(alloc_zero((void **)&s.sl, (size_t)nch * kSlBytes));
+    ell_to_sliced_kernel<<<(unsigned)cdiv(nch * kSlR, kBlock), kBlock, 0, p->ctx->stream>>>(
+        s.n, s.plane, s.val, s.col, s.sl);
+    CHECK(check_launch(p->ctx));
+    CU(cudaStreamSynchronize(p->ctx->stream));
+    return HPCCG_OK;
+}
+
+int sliced_grid(hpccg_ctx *ctx) {
+    static bool attr = false;
+    if (!attr) {
+        cudaFuncSetAttribute(spmv_sliced_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             (int)(kSlStages * kSlBytes));
+        cudaFuncSetAttribute(spmv_sliced_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             (int)(kSlStages * kSlBytes));
+        attr = true;
+    }
+    int b = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, spmv_sliced_kernel<false>, kSlR,
+                                                      kSlStages * kSlBytes) != cudaSuccess || b < 1) {
+        cudaGetLastError();
+        b = 1;
+    }
+    return std::min(b, 2) * ctx->num_sms;
+}
+
 // HPCCG_OPT_SPMV_TRIPS: 512-row trips per block of the single-slab CG SpMV on
 // the finisher-free loop (spmv27x2_trips_kernel), so the update blocks can sum
 // the partials themselves (<= kUpdSumMax); 1: one trip (the finisher kernel
@@ -711,6 +761,25 @@ int cg_spmv_all(hpccg_problem *p, bool timing, bool check) {
         a.total_blocks = (unsigned)spmv_blocks(s.n, rows);
         a.parts_only = s.spmv_parts;  // the update kernel finishes p.Ap
         a.rev = ff_path(p) && (serpentine(p) & 2);
+        if (sliced_on(p)) {
+            a.r0 = 0;
+            a.len0 = s.n;
+            const unsigned g = (unsigned)sliced_grid(ctx);
+            cudaLaunchConfig_t cfg{};
+            cfg.gridDim = dim3(g);
+            cfg.blockDim = dim3(kSlR);
+            cfg.dynamicSmemBytes = kSlStages * kSlBytes;
+            cfg.stream = ctx->stream;
+            cudaLaunchAttribute at[1];
+            at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+            at[0].val.programmaticStreamSerializationAllowed = 1;
+            cfg.attrs = p->opt_pdl ? at : nullptr;
+            cfg.numAttrs = p->opt_pdl ? 1 : 0;
+            const unsigned char *sl = s.sl;
+            if (check) CU(cudaLaunchKernelEx(&cfg, spmv_sliced_kernel<true>, a, sl));
+            else CU(cudaLaunchKernelEx(&cfg, spmv_sliced_kernel<false>, a, sl));
+            return check_launch(ctx);
+        }
         const int trips = spmv_trips(p);
         if (trips > 1) {
             a.r0 = 0;
@@ -754,6 +823,7 @@ double **tab(hpccg_problem *p, int which) { return p->d_tab + (size_t)which * p-
 
 // SpMV partial count of a single slab's CG SpMV (the update sums them).
 unsigned single_spmv_parts(const hpccg_problem *p, const Slab &s) {
+    if (sliced_on(p)) return (unsigned)sliced_grid(p->ctx);
     const int trips = spmv_trips(p);
     if (trips > 1) return (unsigned)cdiv(spmv_blocks(s.n, 2), trips);
     return (unsigned)spmv_blocks(s.n, spmv_rows_per_thread(p->opt_rows, spmv_args(s, s.p, s.Ap), 0, 0));
@@ -1765,6 +1835,7 @@ void free_slab(Slab &s) {
     cudaFree(s.ptab);
     cudaFree(s.trace);
     cudaFree(s.ps_mem);
+    cudaFree(s.sl);
     s = Slab{};
 }
 
@@ -2348,6 +2419,10 @@ int hpccg_generate(hpccg_ctx *ctx, int nx, int ny, int nz, hpccg_problem **out) 
         cudaEventCreateWithFlags(&p->ev_poll[0], cudaEventDisableTiming) != cudaSuccess ||
         cudaEventCreateWithFlags(&p->ev_poll[1], cudaEventDisableTiming) != cudaSuccess)
         return bail(fail(HPCCG_ECUDA, "event create"));
+    if (ctx->mode == MODE_SINGLE) {  // the CG SpMV's chunk-sliced copy (auto: large problems)
+        const int rc = sliced_alloc(p);
+        if (rc) return bail(rc);
+    }
     *out = p;
     return HPCCG_OK;
 }
@@ -2473,6 +2548,13 @@ int hpccg_set_option(hpccg_problem *p, int key, int64_t value) {
             if (value && p->ctx->mode != MODE_SINGLE && !p->slabs[0].ptab) CHECK(enable_peer(p));
             p->opt_peer = (int)value;
             return HPCCG_OK;
+        case HPCCG_OPT_SPMV_SLICED:
+            if (value < -1 || value > 1) return fail(HPCCG_EINVAL, "spmv sliced: -1 (auto), 0 or 1");
+            if (p->graph) cudaGraphExecDestroy(p->graph);
+            if (p->wgraph) cudaGraphExecDestroy(p->wgraph);
+            p->graph = p->wgraph = nullptr;
+            p->opt_sliced = (int)value;
+            return sliced_alloc(p);
         case HPCCG_OPT_PAP_CLUSTER:
             if (value != 0 && value != 1) return fail(HPCCG_EINVAL, "pap cluster: 0 or 1");
             if (p->graph) cudaGraphExecDestroy(p->graph);

@@ -907,6 +907,131 @@ __global__ void __launch_bounds__(kBlock, 4) spmv27x2_trips_kernel(SpmvArgs a) {
     if (threadIdx.x == 0) a.parts_only[a.part_base + bid] = d;
 }
 
+// ---- a.3 + a.4 with the matrix stream fed by TMA (HPCCG_OPT_SPMV_SLICED):
+// the CG loop's SpMV reads a CHUNK-SLICED copy of the same ELL-27 matrix --
+// chunk c of kSlR rows stored contiguously as val[27][kSlR] doubles followed by
+// col[27][kSlR] ints (324 B per row, built once from the slot-major arrays by
+// ell_to_sliced_kernel) -- so a whole chunk is ONE cp.async.bulk copy (41.5 KB)
+// into a two-stage shared-memory ring per CTA (mbarrier completion).  Persistent
+// CTAs (two per SM) take chunks c = b, b + G, ... (reversed under serpentine);
+// one row per thread, its 27 column indices and values read from shared memory
+// and its 27 gathers of p in flight at once.  The same per-row FMA chain in
+// ascending slot order as every other SpMV (identical Ap bits); each thread
+// accumulates its p.Ap over its chunks in order and each CTA writes ONE partial,
+// so the update sums G <= 4096 partials itself -- no p.Ap finisher kernel.
+// Measured at 256^3 (tools/tmaspmv.cu): 792 vs 802 us per SpMV (7.15 TB/s on
+// 12 nnz + 16n B); a TMA copy per slot of the slot-major arrays instead (54 per
+// chunk) is issue-bound at 2.6-3.8 TB/s.  In the CG loop the gain depends on
+// the box (DESIGN 7.1): opt-in.
+constexpr int kSlR = 128;                  // rows per chunk = threads per CTA
+constexpr int kSlStages = 2;
+constexpr unsigned kSlBytes = kSlR * 324;  // one chunk: 27 x (8 + 4) B per row
+
+// one thread per row of the padded chunk grid; rows >= n are padding (0.0, the
+// halo'd index of row 0's own entry -- a finite value, multiplied by 0)
+__global__ void __launch_bounds__(kBlock) ell_to_sliced_kernel(int64_t n, int64_t plane, const double *val,
+                                                               const int *col, unsigned char *sl) {
+    const int64_t i = (int64_t)blockIdx.x * kBlock + threadIdx.x;
+    const int64_t nch = (n + kSlR - 1) / kSlR;
+    if (i >= nch * kSlR) return;
+    const int64_t c = i / kSlR, j = i % kSlR;
+    double *v = reinterpret_cast<double *>(sl + (size_t)c * kSlBytes);
+    int *cc = reinterpret_cast<int *>(sl + (size_t)c * kSlBytes + (size_t)kSlR * kSlots * 8);
+    for (int k = 0; k < kSlots; ++k) {
+        v[k * kSlR + j] = i < n ? val[(int64_t)k * n + i] : 0.0;
+        cc[k * kSlR + j] = i < n ? col[(int64_t)k * n + i] : (int)plane;
+    }
+}
+
+// one chunk into a stage; the matrix is read once per SpMV: evict-first in L2,
+// so it does not push out the planes of p the gathers reuse
+// (measured without the hint: 512^3 8496 vs 7880 us/iteration -- the stream
+// evicted the gathered planes of p)
+__device__ __forceinline__ void sl_issue(const unsigned char *src, unsigned char *dst, unsigned long long *bar) {
+    const unsigned mb = (unsigned)__cvta_generic_to_shared(bar);
+    const uint64_t pol = policy_evict_first();
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(mb), "r"(kSlBytes) : "memory");
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], %4;"
+                 ::"r"((unsigned)__cvta_generic_to_shared(dst)), "l"(src), "r"(kSlBytes), "r"(mb), "l"(pol) : "memory");
+}
+
+__device__ __forceinline__ void sl_wait(unsigned long long *bar, unsigned parity) {
+    const unsigned mb = (unsigned)__cvta_generic_to_shared(bar);
+    unsigned ok = 0;
+    while (!ok)
+        asm volatile("{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2; selp.u32 %0, 1, 0, p; }"
+                     : "=r"(ok) : "r"(mb), "r"(parity) : "memory");
+}
+
+template <bool kCheck>
+__global__ void __launch_bounds__(kSlR, 2) spmv_sliced_kernel(SpmvArgs a, const unsigned char *sl) {
+    extern __shared__ __align__(128) unsigned char ring[];
+    __shared__ __align__(8) unsigned long long full[kSlStages];
+    __shared__ double shp[32];
+    const int64_t n = a.len0, nch = (n + kSlR - 1) / kSlR;
+    const int64_t G = gridDim.x, b = blockIdx.x;
+    const int64_t mine = b < nch ? (nch - 1 - b) / G + 1 : 0;
+    auto chunk = [&](int64_t i) { const int64_t c = b + i * G; return a.rev ? nch - 1 - c : c; };
+    // the matrix does not depend on the predecessor: the first stages are in
+    // flight before the PDL wait
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < kSlStages; ++s)
+            asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"((unsigned)__cvta_generic_to_shared(&full[s])));
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+        for (int s = 0; s < kSlStages && s < mine; ++s)
+            sl_issue(sl + (size_t)chunk(s) * kSlBytes, ring + (size_t)s * kSlBytes, &full[s]);
+    }
+    __syncthreads();
+    pdl_wait();
+    if (a.early_trigger) pdl_trigger();
+    if (a.trace) trace_mark(a.trace, a.trace_max, ldg_o(&a.sc->k), 1, false);
+    if (spmv_done<1, kCheck>(a)) {  // uniform: let the copies in flight land before leaving
+        for (int s = 0; s < kSlStages && s < mine; ++s) sl_wait(&full[s], 0);
+        return;
+    }
+    double d = 0.0;
+    for (int64_t i = 0; i < mine; ++i) {
+        const int s = (int)(i % kSlStages);
+        sl_wait(&full[s], (unsigned)((i / kSlStages) & 1));
+        const unsigned char *st = ring + (size_t)s * kSlBytes;
+        const double *sv = reinterpret_cast<const double *>(st);
+        const int *sc = reinterpret_cast<const int *>(st + (size_t)kSlR * kSlots * 8);
+        const int j = threadIdx.x;
+        const int64_t row = chunk(i) * kSlR + j;
+        double xv[kSlots];
+        int cd = 0;
+#pragma unroll
+        for (int k = 0; k < kSlots; ++k) {  // all 27 gathers in flight
+            const int cc = sc[k * kSlR + j];
+            if (k == kDiagSlot) cd = cc;
+            xv[k] = __ldg(a.x + cc);
+        }
+        double s0 = 0.0;  // FMA chain in ascending column from +0.0 (A8)
+#pragma unroll
+        for (int k = 0; k < kSlots; ++k) s0 = fma(sv[k * kSlR + j], xv[k], s0);
+        __syncthreads();  // stage s consumed by every thread
+        if (threadIdx.x == 0 && i + kSlStages < mine)
+            sl_issue(sl + (size_t)chunk(i + kSlStages) * kSlBytes, ring + (size_t)s * kSlBytes, &full[s]);
+        if (row < n) {
+            a.y[row] = s0;
+            const double p0 = cd == row + a.plane ? xv[kDiagSlot] : __ldg(a.x + row + a.plane);
+            d = fma(s0, p0, d);
+        }
+    }
+    pdl_trigger();
+    if (a.trace) trace_mark(a.trace, a.trace_max, ldg_o(&a.sc->k), 1, true);
+    // CTA sum of kSlR / 32 warps (block_reduce assumes kBlock threads)
+    d = warp_sum(d);
+    if ((threadIdx.x & 31) == 0) shp[threadIdx.x >> 5] = d;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        double t = shp[0];
+#pragma unroll
+        for (int w = 1; w < kSlR / 32; ++w) t += shp[w];
+        a.parts_only[a.part_base + b] = t;
+    }
+}
+
 template <int kDots, bool kCheck, bool kFused = false, bool kDia = false>
 __global__ void __launch_bounds__(kBlock, kDia ? kDiaMinB : 4) spmv27x2_kernel(SpmvArgs a) {
     int64_t row, lim;

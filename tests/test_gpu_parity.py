@@ -1190,3 +1190,62 @@ def test_scaling_configs_global_problem_loopback(P, nz, expect):
         assert r["normr"] <= 1e-12
         assert p.maxabsdiff() < 1e-13
         assert p.stats()["x_deferred"] == 1
+
+
+# ------------- the CG SpMV from the chunk-sliced copy via TMA (SPMV_SLICED)
+
+@pytest.mark.parametrize("dims", [(20, 30, 12), (31, 17, 9), (64, 64, 64), (7, 5, 6)])
+def test_sliced_spmv_first_step_exact(ctx, dims):
+    """HPCCG_OPT_SPMV_SLICED forced on: one CG iteration from x0 = 0 gives x1 =
+    alpha_1 b with alpha_1 = b.b / b.Ab, both exact integers, so
+    x1 must equal the oracle's bit for bit whatever the p.Ap summation tree --
+    this pins every Ap row of the TMA-fed kernel (padding rows of the last
+    chunk included: n is not a multiple of 128 for three of the grids)."""
+    with H.Problem(ctx, *dims) as p:
+        p.set_option(H.HPCCG_OPT_PERSISTENT, 0)
+        p.set_option(H.HPCCG_OPT_SPMV_SLICED, 1)
+        p.set_vec(H.HPCCG_VEC_X, np.zeros(p.n))
+        p.solve(2, 0.0)
+        x1 = p.get_vec(H.HPCCG_VEC_X)
+        o = oracle.cg(oracle.generate(*dims), 2, 0.0)
+        np.testing.assert_array_equal(x1, o["x"])
+        p.set_option(H.HPCCG_OPT_SPMV_SLICED, 0)
+
+
+@pytest.mark.parametrize("dims,max_iter,tol", [((24, 20, 12), 150, 1e-12), ((64, 64, 64), 150, 1e-12),
+                                               ((33, 9, 3), 40, 0.0), ((128, 128, 130), 25, 0.0)])
+def test_sliced_spmv_cg_modes_and_oracle(ctx, dims, max_iter, tol):
+    """The sliced SpMV in every launch mode (while-graph, per-iteration graph,
+    plain timed launches): bit-identical solves for a given chunk order (its
+    per-CTA p.Ap partials are a fixed tree; the serpentine order reverses each
+    CTA's chunk sequence, so it is another fixed tree), within the north_star
+    tolerance of the oracle in both orders."""
+    with H.Problem(ctx, *dims) as p:
+        p.set_option(H.HPCCG_OPT_PERSISTENT, 0)
+        p.set_option(H.HPCCG_OPT_SPMV_SLICED, 1)
+        outs = []
+        for serp in (0, 3):
+            p.set_option(H.HPCCG_OPT_SERPENTINE, serp)
+            for wh, tm in ((1, 0), (0, 0), (0, 1)):
+                p.set_option(H.HPCCG_OPT_WHILE, wh)
+                p.set_option(H.HPCCG_OPT_TIMING, tm)
+                p.set_vec(H.HPCCG_VEC_X, np.zeros(p.n))
+                r = p.solve(max_iter, tol)
+                outs.append((r["niters"], r["normr"], p.get_vec(H.HPCCG_VEC_X)))
+        p.set_option(H.HPCCG_OPT_TIMING, 0)
+        p.set_option(H.HPCCG_OPT_WHILE, 1)
+        p.set_option(H.HPCCG_OPT_SERPENTINE, -1)
+        p.set_option(H.HPCCG_OPT_SPMV_SLICED, 0)
+        for g in (outs[:3], outs[3:]):  # per chunk order: every mode the same bits
+            for o in g[1:]:
+                assert o[:2] == g[0][:2]
+                np.testing.assert_array_equal(o[2], g[0][2])
+        if p.n <= 300_000:
+            ref = oracle.generate(*dims)
+            oref = oracle.cg(ref, max_iter, tol)
+            for o in (outs[0], outs[3]):
+                assert abs(o[0] - oref["niters"]) <= 1
+                assert np.max(np.abs(o[2] - oref["x"])) <= CG_ATOL
+        else:
+            for o in (outs[0], outs[3]):
+                assert o[0] == max_iter - 1 and np.all(np.isfinite(o[2]))

@@ -21,7 +21,8 @@ KEYS = {"graph": H.HPCCG_OPT_GRAPH, "timing": H.HPCCG_OPT_TIMING, "while": H.HPC
         "fmt": getattr(H, "HPCCG_OPT_SPMV_FORMAT", -1),
         "defer": getattr(H, "HPCCG_OPT_DEFER_X", -1),
         "fuse": getattr(H, "HPCCG_OPT_FUSE_PSPMV", -1), "lead": getattr(H, "HPCCG_OPT_PS_LEAD", -1),
-        "trips": getattr(H, "HPCCG_OPT_SPMV_TRIPS", -1), "papcl": getattr(H, "HPCCG_OPT_PAP_CLUSTER", -1)}
+        "trips": getattr(H, "HPCCG_OPT_SPMV_TRIPS", -1), "papcl": getattr(H, "HPCCG_OPT_PAP_CLUSTER", -1),
+        "sliced": getattr(H, "HPCCG_OPT_SPMV_SLICED", -1)}
 nx, ny, nz, iters = (int(v) for v in sys.argv[1:5])
 P = int(os.environ.get("PROBE_P", "1"))  # > 1: loopback slabs on one GPU
 if os.environ.get("PROBE_NCCL"):  # 1-rank NCCL communicator (the multi-GPU code path)
