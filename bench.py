@@ -386,7 +386,7 @@ def _stats_add(acc, prob, r):
     acc["pupdate_ms"] += st["pupdate_ms"]
     acc["niters"] += r["niters"]
     acc["graph_mode"] = st["graph_mode"]
-    acc["x_deferred"] = bool(st["x_deferred"])
+    acc["x_deferred"] = int(st["x_deferred"])  # deferral depth m (0 off; m >= 2: ring of m + 1 p buffers)
 
 
 class CgRunner:
@@ -550,8 +550,10 @@ def measure_workload(H, D, ctx, stream, world, rank, local, coll_dev, name, step
         t = prob.trace(k_tr).astype("float64")[5:]
         prob.set_option(H.HPCCG_OPT_TRACE, 0)
         if len(t):
-            dur = np.median((t[:, :, 1] - t[:, :, 0]) / 1e3, axis=0)   # us
-            period = float(np.median(np.diff(t[:, 0, 0])) / 1e3) if len(t) > 1 else None
+            # means over the traced iterations: with the ring-deferred x update
+            # every m-th p update also flushes x (a periodic pattern, not noise)
+            dur = np.mean((t[:, :, 1] - t[:, :, 0]) / 1e3, axis=0)   # us
+            period = float(np.mean(np.diff(t[:, 0, 0])) / 1e3) if len(t) > 1 else None
             tr = {"period_us": round(period, 2) if period else None,
                   "pupdate_us": round(float(dur[0]), 2), "spmv_us": round(float(dur[1]), 2),
                   "update_us": round(float(dur[2]), 2)}
@@ -648,6 +650,8 @@ def run_ours(args):
     opts = [(H.HPCCG_OPT_CG_VARIANT, 1 if sr else 0), (H.HPCCG_OPT_SPMV_FORMAT, 1 if dia else 0)]
     if args.no_defer_x:
         opts.append((H.HPCCG_OPT_DEFER_X, 0))
+    elif args.defer_x is not None:
+        opts.append((H.HPCCG_OPT_DEFER_X, args.defer_x))
     mode_want = 1 if args.halo == "peer" else 2
 
     def setup_multirank(prob):
@@ -685,7 +689,7 @@ def run_ours(args):
                             args.steps, args.warmup, events=True, trace=not sr, clocks=True,
                             opts=opts, setup=setup_multirank)
     n, nnz_local = main["_n"], main["_nnz_local"]
-    defer = bool(main.get("x_deferred"))
+    defer = int(main.get("x_deferred") or 0)
     ev, trace = main["_ev"], main["_trace"]
     # per-rank record of what actually ran (transport, exchange mode, NCCL view)
     cinfo = ctx.info()
@@ -763,10 +767,14 @@ def run_ours(args):
                                      "by a pure-read stream measured live here (our dot kernel, 2 x 4 GiB, best of 6)")
             # the fused vector kernels (north_star: >= 75 % of the 8 TB/s HBM peak on
             # "SpMV and fused waxpby/ddot"): x/r update + r.r 48n B, p update 24n B;
-            # with the deferred x update (default) r update + r.r 24n, x and p update 40n
+            # with the deferred x update (default) r update + r.r 24n, x and p update 40n;
+            # deferred over a ring of m + 1 p buffers (m >= 2): per m iterations the p
+            # update reads r, p m times, x once and m - 1 old p's, writes p m times and
+            # x once: (32 + 8/m) n per iteration on average
             vec = {}
-            u_bytes, p_bytes = ((72.0 * n, None) if sr else (24.0 * n, 40.0 * n) if defer
-                                else (48.0 * n, 24.0 * n))
+            u_bytes, p_bytes = ((72.0 * n, None) if sr else
+                                (24.0 * n, (32.0 + 8.0 / defer) * n) if defer >= 2 else
+                                (24.0 * n, 40.0 * n) if defer else (48.0 * n, 24.0 * n))
             u_us = ev["update_ms"] * 1e3 / max(ev["niters"], 1)
             p_us = ev["pupdate_ms"] * 1e3 / max(ev["niters"], 1)
             for nm_k, by, us_ev, us_tr in (("update", u_bytes, u_us, trace and trace["update_us"]),
@@ -815,8 +823,12 @@ def run_ours(args):
                                     "global_nnz", "tol", "max_iter", "solve_graph", "l2", "gen_ms")}
         cfg.update({"iters": main["niters_per_step"], "parallelism": f"zslab{world}",
                     "cg_variant": "single-reduction (Chronopoulos-Gear, f2)" if sr else "HPCCG",
-                    "x_update": ("deferred into the next p update (HPCCG_OPT_DEFER_X, auto: the CG vectors "
-                                 "exceed L2): 12 nnz + 80n B per iteration" if defer
+                    "x_update": (f"deferred over a ring of {defer + 1} p buffers (HPCCG_OPT_DEFER_X = {defer}, "
+                                 f"auto when the CG vectors exceed L2): x += alpha_j p_j applied every "
+                                 f"{defer} iterations, 12 nnz + {72 + 8 / defer:g}n B per iteration"
+                                 if defer >= 2 else
+                                 "deferred into the next p update (HPCCG_OPT_DEFER_X 1): 12 nnz + 80n B "
+                                 "per iteration" if defer
                                  else "in the x/r update: 12 nnz + 88n B per iteration"),
                     "spmv_format": ("DIA-27 (columns from stencil offsets) -- EFFECTIVE, a different "
                                     "method (SURVEY 8(d): OUT)") if dia
@@ -1197,6 +1209,9 @@ def main():
                          "EFFECTIVE numbers of a different method (SURVEY 8(d): OUT), never the headline")
     ap.add_argument("--no-defer-x", action="store_true",
                     help="HPCCG_OPT_DEFER_X 0: update x in the x/r update (88n instead of 80n B/iteration)")
+    ap.add_argument("--defer-x", type=int, default=None,
+                    help="HPCCG_OPT_DEFER_X: 1 = x deferred by one iteration, m = 2..8 over a ring of "
+                         "m + 1 p buffers (default: the library's auto)")
     ap.add_argument("--no-sub-configs", action="store_true",
                     help="skip the configs[1] / [0] / [3] sub-records of the CG line")
     ap.add_argument("--no-cpu-baseline", action="store_true")

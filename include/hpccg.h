@@ -146,9 +146,20 @@ extern "C" {
                                x/r update moves 24n instead of 48n B and the p update 40n
                                instead of 24n: 80n + 12 nnz B per iteration instead of 88n.
                                Bitwise the same results (the same FMA on the same operands);
-                               0: x updated in the x/r update; -1 (default): auto, 1 when the
-                               CG vectors exceed L2 (256^3: 989 vs 1005 us/iteration; at 128^3
-                               the vectors are L2-resident and 0 is 0.4 % faster) */
+                               0: x updated in the x/r update.  m = 2..8 (single slab only;
+                               z-slabs fall back to 1): deferred over a ring of m + 1 p buffers
+                               -- p_k is written to slot k % (m + 1) (slot 0 = the problem's p
+                               buffer, the SpMV gathers from the slot of iteration k) and every
+                               m-th p update applies x = fma(alpha_j, p_j, x) for the m
+                               directions since the last one, in ascending j; the pending ones
+                               run after the loop (cg_xfix_ring_kernel).  Per m iterations x
+                               is read and written once and m - 1 old p's re-read: 12 nnz +
+                               (72 + 8/m) n B per iteration, the writes drop from 2 to 1 + 1/m
+                               per row.  Bitwise the same results.  Device memory: m extra
+                               p-sized buffers (allocated when the option is set, or at
+                               generate time for auto).  -1 (default): auto -- 8 on a single
+                               slab whose CG vectors exceed L2, 1 on z-slabs there, 0 below
+                               (at 128^3 the vectors are L2-resident and 0 is 0.4 % faster) */
 #define HPCCG_OPT_FUSE_PSPMV 24 /* single slab, finisher-free loop: the p update and the
                                SpMV of an iteration as ONE pipelined kernel (cg_pspmv_kernel:
                                chunks of 512 rows taken in launch order; each block updates p
@@ -248,7 +259,8 @@ typedef struct hpccg_stats {
     int64_t graph_mode;     /* 5 shared-memory-resident cluster kernel, 4 one-cluster
                                persistent kernel, 3 cooperative-grid persistent kernel,
                                2 while-graph, 1 per-iteration graph, 0 plain */
-    int64_t x_deferred;     /* 1: the solve ran with the deferred x update (HPCCG_OPT_DEFER_X) */
+    int64_t x_deferred;     /* the deferral depth the solve ran with (HPCCG_OPT_DEFER_X): 0 none,
+                               1 by one iteration, m >= 2 over a ring of m + 1 p buffers */
     int64_t ps_fused;       /* 1: the solve ran the fused p update + SpMV (HPCCG_OPT_FUSE_PSPMV) */
 } hpccg_stats;
 

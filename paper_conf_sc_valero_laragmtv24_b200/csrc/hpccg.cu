@@ -135,6 +135,11 @@ struct Slab {
     unsigned *ps_ticket = nullptr;
     unsigned long long *ps_flags = nullptr;
     int *ps_err = nullptr;
+    // HPCCG_OPT_DEFER_X = m >= 2: ring slots 1..pring_slots of p (slot 0 = p),
+    // each laid out like p (halo base, ncol), pring_stride doubles apart
+    double *pring_alloc = nullptr, *pring = nullptr;
+    int64_t pring_stride = 0;
+    int pring_slots = 0;
 };
 
 struct TimedOp {
@@ -172,7 +177,8 @@ struct hpccg_problem {
     int opt_smem_threads = 0;          // on-chip solve CTA width: 0 auto, 256, 512
     int opt_peer = 0;                  // multi-slab: halo push + allreduce over peer memory
     int64_t opt_peer_timeout_ms = 30000;  // give up a peer-memory wait after this long
-    int opt_defer_x = -1;              // finisher-free loop: x update deferred into the p update (-1 auto)
+    int opt_defer_x = -1;              // finisher-free loop: x update deferred into the p update (-1 auto,
+                                       // 0 off, 1 every iteration, m >= 2 over a ring of m + 1 p buffers)
     int opt_fuse_ps = 0;               // p update + SpMV in one pipelined kernel (-1 auto, 0 off, 1 on)
     int opt_spmv_trips = 1;            // single-slab SpMV trips per block (0 auto, 1 off, T)
     int opt_pap_cluster = 0;           // p.Ap finisher as one 8-CTA cluster (1) or one CTA (0)
@@ -748,6 +754,8 @@ int spmv_trips(const hpccg_problem *p) {
     return blocks > kUpdSumMax ? (int)cdiv(blocks, kUpdSumMax) : 1;
 }
 
+int defer_m(const hpccg_problem *p);
+
 int cg_spmv_all(hpccg_problem *p, bool timing, bool check) {
     hpccg_ctx *ctx = p->ctx;
     const int minb = p->opt_minb;
@@ -761,6 +769,11 @@ int cg_spmv_all(hpccg_problem *p, bool timing, bool check) {
         a.total_blocks = (unsigned)spmv_blocks(s.n, rows);
         a.parts_only = s.spmv_parts;  // the update kernel finishes p.Ap
         a.rev = ff_path(p) && (serpentine(p) & 2);
+        if (const int m = defer_m(p); m >= 2) {  // p_k in ring slot k % (m + 1)
+            a.ring = s.pring;
+            a.ring_stride = s.pring_stride;
+            a.ring_n = m + 1;
+        }
         if (sliced_on(p)) {
             a.r0 = 0;
             a.len0 = s.n;
@@ -943,11 +956,64 @@ bool defer_x_on(const hpccg_problem *p) {
     return on && ff_path(p);
 }
 
+bool fuse_ps_on(hpccg_problem *p);
+bool sliced_on(const hpccg_problem *p);
+int spmv_trips(const hpccg_problem *p);
+
+// auto depth of the ring-deferred x update (CG vectors beyond L2, single slab):
+// tools/ringbench.cu -- the saving levels off from m = 6 (21.8 -> 21.9 -> 22.5 us
+// per iteration at m = 6 / 8 / 12 at 256^3)
+constexpr int kRingAutoM = kRingMaxM;
+
+// the deferral depth in effect: 0 off, 1 every iteration (cg_pupdate1_kernel),
+// m >= 2 over the ring (single slab on the plain finisher-free path only)
+int defer_m(const hpccg_problem *p) {
+    if (!defer_x_on(p)) return 0;
+    const int want = p->opt_defer_x < 0 ? kRingAutoM : p->opt_defer_x;
+    if (want < 2 || p->ctx->mode != MODE_SINGLE) return 1;
+    const Slab &s = p->slabs[0];
+    if (s.pring_slots < want || s.dia || fuse_ps_on(const_cast<hpccg_problem *>(p)) || sliced_on(p) ||
+        spmv_trips(p) > 1)
+        return 1;
+    return want;
+}
+
+// ring slots for depth m (never during a graph capture: generate / set_option)
+int ring_alloc(hpccg_problem *p, int m) {
+    if (p->ctx->mode != MODE_SINGLE || m < 2) return HPCCG_OK;
+    Slab &s = p->slabs[0];
+    if (s.pring_slots >= m) return HPCCG_OK;
+    cudaFree(s.pring_alloc);
+    s.pring_alloc = s.pring = nullptr;
+    s.pring_slots = 0;
+    const int64_t seg = cdiv(s.ncol + 2, 32) * 32;  // as the arena's p segment
+    CHECK(alloc_zero((void **)&s.pring_alloc, sizeof(double) * (size_t)(seg * m)));
+    s.pring = s.pring_alloc + (s.p - s.p_alloc);  // the same 16-B alignment shift as p
+    s.pring_stride = seg;
+    s.pring_slots = m;
+    return HPCCG_OK;
+}
+
+PRing ring_of(const Slab &s, int m, bool owned) {
+    PRing g{};
+    g.base = s.pring + (owned ? s.plane : 0);
+    g.stride = s.pring_stride;
+    g.m = m;
+    return g;
+}
+
 // end of a solve on the finisher-free loop with the deferred x update: the
-// last iteration's x += alpha p (cg_xfix_kernel), every slab
+// last iteration's x += alpha p (cg_xfix_kernel; ring: the pending ones,
+// cg_xfix_ring_kernel), every slab
 int enqueue_xfix(hpccg_problem *p) {
     if (!defer_x_on(p)) return HPCCG_OK;
     hpccg_ctx *ctx = p->ctx;
+    if (const int m = defer_m(p); m >= 2) {
+        const Slab &s = p->slabs[0];
+        launch_k(false, cg_xfix_ring_kernel, dim3(wave_grid(s.n / 2 + 1, wave(ctx, cg_xfix_ring_kernel))),
+                 ctx->stream, (int64_t)s.n, s.x, s.p + s.plane, ring_of(s, m, true), (const CgScalars *)s.sc);
+        return check_launch(ctx);
+    }
     for (const Slab &s : p->slabs) {
         launch_k(false, cg_xfix_kernel, dim3(wave_grid(s.n / 2 + 1, wave(ctx, cg_xfix_kernel))),
                  ctx->stream, (int64_t)s.n, s.x, (const double *)(s.p + s.plane), (const CgScalars *)s.sc);
@@ -1070,6 +1136,25 @@ int enqueue_iteration_ff_u(hpccg_problem *p, bool timing, bool check, unsigned l
         }
         PhaseTimer t(p, ctx->stream, PH_SPMV, timing);
         CHECK(launch_pspmv(p, s0, q));
+    } else if (const int m = zs ? 0 : defer_m(p); m >= 2) {  // ring-deferred x update
+        PhaseTimer t(p, ctx->stream, PH_PUPDATE, timing);
+        PringArgs a{};
+        a.n = s0.n;
+        a.r = s0.r;
+        a.p = s0.p + s0.plane;
+        a.ring = ring_of(s0, m, true);
+        a.x = s0.x;
+        a.rr_parts = s0.red.partials;
+        a.n_rr = (unsigned)ug;
+        a.sc = s0.sc;
+        a.q = q;
+        a.trace = s0.trace_on ? s0.trace : nullptr;
+        a.trace_max = s0.trace_max;
+        a.rev = serpentine(p) & 1;
+        auto rk = cg_pupdate_ring_kernel<kU>;
+        const int rg = vec_grid(ctx, rk, cdiv(s0.n, 2 * kU), p->opt_vec_waves, 0x7fffffff);
+        launch_k(pdl, rk, dim3(rg), ctx->stream, a);
+        CHECK(check_launch(ctx));
     } else {
         PhaseTimer t(p, ctx->stream, PH_PUPDATE, timing);
         if (pre)
@@ -1836,6 +1921,7 @@ void free_slab(Slab &s) {
     cudaFree(s.trace);
     cudaFree(s.ps_mem);
     cudaFree(s.sl);
+    cudaFree(s.pring_alloc);
     s = Slab{};
 }
 
@@ -2420,8 +2506,10 @@ int hpccg_generate(hpccg_ctx *ctx, int nx, int ny, int nz, hpccg_problem **out) 
         cudaEventCreateWithFlags(&p->ev_poll[1], cudaEventDisableTiming) != cudaSuccess)
         return bail(fail(HPCCG_ECUDA, "event create"));
     if (ctx->mode == MODE_SINGLE) {  // the CG SpMV's chunk-sliced copy (auto: large problems)
-        const int rc = sliced_alloc(p);
+        int rc = sliced_alloc(p);
         if (rc) return bail(rc);
+        // the ring of the deferred x update (auto: CG vectors beyond L2)
+        if (p->slabs[0].arena_bytes > ((size_t)126 << 20) && (rc = ring_alloc(p, kRingAutoM))) return bail(rc);
     }
     *out = p;
     return HPCCG_OK;
@@ -2587,12 +2675,15 @@ int hpccg_set_option(hpccg_problem *p, int key, int64_t value) {
             p->opt_ps_lead = (int)value;
             return HPCCG_OK;
         case HPCCG_OPT_DEFER_X:
-            if (value < -1 || value > 1) return fail(HPCCG_EINVAL, "defer x: -1 (auto), 0 or 1");
+            if (value < -1 || value > kRingMaxM)
+                return fail(HPCCG_EINVAL, "defer x: -1 (auto), 0, 1 or a ring depth 2 .. %d", kRingMaxM);
             if (p->opt_defer_x != (int)value) {  // graphs capture the choice
                 if (p->graph) cudaGraphExecDestroy(p->graph);
                 if (p->wgraph) cudaGraphExecDestroy(p->wgraph);
                 p->graph = p->wgraph = nullptr;
             }
+            CHECK(ring_alloc(p, value < 0 ? (p->slabs[0].arena_bytes > ((size_t)126 << 20) ? kRingAutoM : 0)
+                                          : (int)value));
             p->opt_defer_x = (int)value;
             return HPCCG_OK;
         case HPCCG_OPT_PEER_TIMEOUT_MS:
@@ -2910,7 +3001,7 @@ int hpccg_solve(hpccg_problem *p, int max_iter, double tol, int *niters, double 
     st.kernel_launches = ctx->launches - l0;
     st.l2_persist_bytes = (int64_t)l2win.kept;
     st.graph_mode = use_persist ? p->last_persist_mode : (use_while ? 2 : (use_graph ? 1 : 0));
-    st.x_deferred = !use_persist && defer_x_on(p);
+    st.x_deferred = use_persist ? 0 : defer_m(p);
     st.ps_fused = !use_persist && fuse_ps_on(p);
     p->stats = st;
     if (niters) *niters = hs.niters;

@@ -58,6 +58,12 @@ struct CgScalars {
     unsigned long long epoch;  // solves initialised so far (HALO_PEER = 2 tags)
     double alpha_x;   // deferred x update: alpha of the last x/r update (x += alpha_x p
                       // is applied by the next p update, or by cg_xfix_kernel at the end)
+    // deferred x update over a ring of p buffers (HPCCG_OPT_DEFER_X = m >= 2):
+    // alpha_k of every x/r update (slot k & 15), and the index of the last p
+    // update that ran, double-buffered by iteration parity (ring_k[q] written
+    // by p update k, q = k & 1; read by p update k + 1 before its PDL wait)
+    double alpha_h[16];
+    int ring_k[2];
 };
 
 // Scratch for the deterministic single-pass grid reduction.
@@ -495,6 +501,12 @@ __device__ __forceinline__ double2 fused_collect2_block(const PeerTab *t, int q,
 // interior / boundary split used to overlap the halo exchange).
 struct SpmvArgs {
     int64_t r0, len0, r1, len1;
+    // HPCCG_OPT_DEFER_X = m >= 2: p_k lives in ring slot k % ring_n (slot 0 =
+    // x, slot j > 0 = ring + (j - 1) ring_stride), k = sc->k read after the
+    // PDL wait; ring_n <= 1: x
+    const double *ring;
+    int64_t ring_stride;
+    int ring_n;
     int64_t nb0;            // blocks covering range 0
     int64_t r2, len2;       // a third range (HALO_PEER = 2: interior, plane 0, plane nz-1)
     int64_t nb01;           // blocks covering ranges 0 and 1
@@ -539,6 +551,13 @@ __device__ __forceinline__ int spmv_done(const SpmvArgs &a) {
     if (!kCheck || kDots == 0) return 0;
     if (kDots == 2) return !ldg_o(&a.sc->run_q[a.sr_q]);
     return ldg_o(&a.sc->done);
+}
+
+// the gathered vector of this SpMV (after pdl_wait: sc->k is the predecessor's)
+__device__ __forceinline__ const double *spmv_xg(const SpmvArgs &a) {
+    if (a.ring_n <= 1) return a.x;
+    const int j = ldg_o(&a.sc->k) % a.ring_n;
+    return j == 0 ? a.x : a.ring + (int64_t)(j - 1) * a.ring_stride;
 }
 
 // Block sums of two values in a fixed order; valid in thread 0.
@@ -604,6 +623,7 @@ __global__ void __launch_bounds__(kBlock, kMinB) spmv27_kernel(SpmvArgs a) {
         double sum = 0.0;  // FMA chain in ascending column from +0.0 (A8)
         double xd = 0.0;
         int cd = 0;
+        const double *xg = a.x;
         // three groups of 9 slots (one z-plane of the stencil each); all 18
         // loads of a group are issued before its gathers and FMAs, and the
         // compiler may hoist the next group's loads above them
@@ -622,10 +642,11 @@ __global__ void __launch_bounds__(kBlock, kMinB) spmv27_kernel(SpmvArgs a) {
                 if (kDot && a.trace) trace_mark(a.trace, a.trace_max, ldg_o(&a.sc->k), 1, false);
                 done = spmv_done<kDots, kCheck>(a);
                 if (done) return;  // uniform over the grid, before any store
+                xg = spmv_xg(a);
             }
 #pragma unroll
             for (int t = 0; t < 9; ++t) {
-                const double xv = __ldg(a.x + cc[t]);
+                const double xv = __ldg(xg + cc[t]);
                 if (9 * g + t == kDiagSlot) {
                     xd = xv;
                     cd = cc[t];
@@ -637,7 +658,7 @@ __global__ void __launch_bounds__(kBlock, kMinB) spmv27_kernel(SpmvArgs a) {
         // p_i: the diagonal slot's gathered value when that slot really is the
         // row's own column (always, for generated matrices); else reload it.
         if (kDots > 0) {
-            const double xi = cd == row + a.plane ? xd : __ldg(a.x + row + a.plane);
+            const double xi = cd == row + a.plane ? xd : __ldg(xg + row + a.plane);
             d = sum * xi;
             if (kDots == 2) dg = xi * xi;
         }
@@ -740,6 +761,7 @@ __device__ __forceinline__ void spmv27x2_body(const SpmvArgs &a, int64_t row, in
         const int *c = a.col + row;
         double s0 = 0.0, s1 = 0.0, x0 = 0.0, x1 = 0.0;
         int c0 = 0, c1 = 0;
+        const double *xg = a.x;
         // slots whose loads are issued together: 3 (ELL: 72 B per thread in
         // flight); DIA has no index stream, so it takes kDiaGroup slots
         constexpr int kG = kDia ? kDiaGroup : 3;
@@ -758,11 +780,12 @@ __device__ __forceinline__ void spmv27x2_body(const SpmvArgs &a, int64_t row, in
                 if (kDot && a.trace) trace_mark(a.trace, a.trace_max, ldg_o(&a.sc->k), 1, false);
                 done = spmv_done<kDots, kCheck>(a);
                 if (done) return;  // uniform over the grid, before any store
+                xg = spmv_xg(a);
             }
 #pragma unroll
             for (int t = 0; t < kG; ++t) {
                 if (kDia) cc[t] = spmv_cols<true>(a, c, kG * g + t, vv[t], row, pol);
-                const double xa = ld_gather<kCoh>(a.x + cc[t].x), xb = ld_gather<kCoh>(a.x + cc[t].y);
+                const double xa = ld_gather<kCoh>(xg + cc[t].x), xb = ld_gather<kCoh>(xg + cc[t].y);
                 if (kG * g + t == kDiagSlot) {
                     x0 = xa;
                     x1 = xb;
@@ -775,8 +798,8 @@ __device__ __forceinline__ void spmv27x2_body(const SpmvArgs &a, int64_t row, in
         }
         *reinterpret_cast<double2 *>(a.y + row) = make_double2(s0, s1);
         if (kDots > 0) {
-            const double p0 = c0 == row + a.plane ? x0 : ld_gather<kCoh>(a.x + row + a.plane);
-            const double p1 = c1 == row + 1 + a.plane ? x1 : ld_gather<kCoh>(a.x + row + 1 + a.plane);
+            const double p0 = c0 == row + a.plane ? x0 : ld_gather<kCoh>(xg + row + a.plane);
+            const double p1 = c1 == row + 1 + a.plane ? x1 : ld_gather<kCoh>(xg + row + 1 + a.plane);
             d = fma(s1, p1, s0 * p0);
             if (kDots == 2) dg = fma(p1, p1, p0 * p0);
         }
@@ -785,14 +808,15 @@ __device__ __forceinline__ void spmv27x2_body(const SpmvArgs &a, int64_t row, in
         pdl_wait();
         done = spmv_done<kDots, kCheck>(a);
         if (done) return;
+        const double *xg = spmv_xg(a);
         double s0 = 0.0;
 #pragma unroll
         for (int k = 0; k < kSlots; ++k)
             s0 = fma(ld_stream(a.val + k * a.stride + row, pol),
-                     ld_gather<kCoh>(a.x + ld_stream(a.col + k * a.stride + row, pol)), s0);
+                     ld_gather<kCoh>(xg + ld_stream(a.col + k * a.stride + row, pol)), s0);
         a.y[row] = s0;
         if (kDots > 0) {
-            const double xi = ld_gather<kCoh>(a.x + row + a.plane);
+            const double xi = ld_gather<kCoh>(xg + row + a.plane);
             d = s0 * xi;
             if (kDots == 2) dg = xi * xi;
         }
@@ -1628,6 +1652,234 @@ __global__ void __launch_bounds__(kBlock) cg_xfix_kernel(int64_t n, double *x, c
     if (tid == 0 && (n & 1)) x[n - 1] = fma(alpha, p[n - 1], x[n - 1]);
 }
 
+// ---- a.6 with the x update deferred over m iterations (HPCCG_OPT_DEFER_X =
+// m >= 2, single slab).  x_k = x_(k-1) + alpha_k p_k is applied m iterations
+// at a time: p_k of iteration k is written to ring slot k % (m + 1) (slot 0 is
+// the problem's p buffer, the SpMV gathers from the slot of sc->k), so the m
+// directions since the last flush stay in HBM, and the p update of iteration
+// K with (K - 1) % m == 0 reads them once more and applies
+//   x = fma(alpha_j, p_j, x),  j = K - m, ..., K - 1 (ascending)
+// -- the FMAs the per-iteration update does, on the same operands in the same
+// order, so x is bitwise identical.  Per m iterations the x stream costs one
+// read and one write (16n B) plus m - 1 re-reads of old p (8n B each) instead
+// of m reads and m writes: the reads stay 3 per iteration, the writes drop
+// from 2 to 1 + 1/m (measured, tools/ringbench.cu: 2R:1W ring + one flush per
+// m against 3R:2W in place).  cg_xfix_ring_kernel applies the pending ones
+// after the loop.
+constexpr int kRingMaxM = 8;
+
+struct PRing {
+    double *base;    // slot 1 (slot j >= 1 at base + (j - 1) stride; slot 0: the kernel's p)
+    int64_t stride;  // doubles between slots
+    int m;           // deferral depth: m + 1 slots
+};
+
+__device__ __forceinline__ double *ring_slot(double *p0, const PRing &g, int j) {
+    return j == 0 ? p0 : g.base + (int64_t)(j - 1) * g.stride;
+}
+
+struct PringArgs {
+    int64_t n;
+    const double *r;
+    double *p;  // slot 0 (owned part)
+    PRing ring; // owned-part bases
+    double *x;
+    const double *rr_parts;
+    unsigned n_rr;
+    CgScalars *sc;
+    int q;
+    TraceSlot *trace;
+    int trace_max;
+    int rev;
+};
+
+// the scalar part of p update K (after the PDL wait): beta, and block 0's
+// loop state; false: iteration K does not run (uniform exit)
+__device__ __forceinline__ bool ring_scalars(const PringArgs &a, int K, bool first, double *sh, double *beta) {
+    CgScalars *sc = a.sc;
+    if (!run_check(sc, a.q)) return false;
+    trace_mark(a.trace, a.trace_max, K, 0, false);
+    const double rtrans = first ? ldg_o(&sc->rr_cur) : sum_parts_fixed(a.rr_parts, a.n_rr, sh);
+    *beta = first ? 0.0 : rtrans / ldg_o(&sc->rr_prev);
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+        if (!first) sc->rr_cur = rtrans;
+        sc->normr = sqrt(rtrans);
+        sc->niters = K;
+        sc->ring_k[a.q] = K;
+    }
+    return true;
+}
+
+// flush iteration (K - 1 divisible by m): one double per thread per trip
+// (scalar: the m + 2 loads in flight per thread fit the normal path's
+// register budget); x, p_(K-1) and the m - 1 older directions are loaded
+// before the wait
+__device__ __forceinline__ void ring_flush(const PringArgs &a, int K, double *sh) {
+    const int m = a.ring.m, R = m + 1;
+    const int64_t tid = gtid(), nth = gnth(), n = a.n;
+    const double *src = ring_slot(a.p, a.ring, (K - 1) % R);
+    double *dst = ring_slot(a.p, a.ring, K % R);
+    const double *__restrict__ r = a.r;
+    double *x = a.x;
+    // the older directions' slots (K - m + t) % R, t < m - 1
+    __shared__ const double *sop[kRingMaxM - 1];
+    if (threadIdx.x < kRingMaxM - 1)
+        sop[threadIdx.x] =
+            (int)threadIdx.x < m - 1 ? ring_slot(a.p, a.ring, (K - m + (int)threadIdx.x) % R) : nullptr;
+    __syncthreads();
+    const int64_t step = nth;
+    const int64_t b0 = (a.rev && tid < n) ? tid + ((n - 1 - tid) / step) * step : tid;
+    double pa = 0.0, ra = 0.0, xa = 0.0, oa[kRingMaxM - 1];
+    auto ld_old = [&](int64_t i) {
+        xa = x[i];
+        pa = src[i];
+#pragma unroll
+        for (int t = 0; t < kRingMaxM - 1; ++t)
+            if (t < m - 1) oa[t] = sop[t][i];
+    };
+    if (b0 < n) ld_old(b0);
+    pdl_wait();
+    pdl_trigger();
+    if (b0 < n) ra = r[b0];
+    double beta;
+    if (!ring_scalars(a, K, false, sh, &beta)) return;
+    __shared__ double sal[kRingMaxM];
+    if (threadIdx.x < kRingMaxM)
+        sal[threadIdx.x] = (int)threadIdx.x < m ? ldg_o(&a.sc->alpha_h[(K - m + (int)threadIdx.x) & 15]) : 0.0;
+    __syncthreads();
+    const double am = sal[m - 1];
+    for (int64_t b = b0; b >= 0 && b < n;) {
+        // x += alpha_j p_j, j = K - m .. K - 1 in ascending order (p_(K-1) = pa)
+#pragma unroll
+        for (int t = 0; t < kRingMaxM - 1; ++t)
+            if (t < m - 1) xa = fma(sal[t], oa[t], xa);
+        x[b] = fma(am, pa, xa);
+        dst[b] = fma(beta, pa, ra);
+        b += a.rev ? -step : step;
+        if (b >= 0 && b < n) {
+            ra = r[b];
+            ld_old(b);
+        }
+    }
+    if (a.trace) {
+        __syncthreads();
+        trace_mark(a.trace, a.trace_max, K, 0, true);
+    }
+}
+
+// (__launch_bounds__(kBlock, 3): the flush path's loads must not push the
+// kernel past the 80 registers of cg_pupdate1_kernel<4>)
+template <int kU>
+__global__ void __launch_bounds__(kBlock, 3) cg_pupdate_ring_kernel(PringArgs a) {
+    __shared__ double sh[33];
+    // this iteration's index from the p update before it (ring_k[q ^ 1],
+    // written by p update K - 1, which completed before this grid's PDL
+    // predecessor began): the slots are known before the wait
+    const int K = ldp(&a.sc->ring_k[a.q ^ 1]) + 1;
+    const int m = a.ring.m, R = m + 1;
+    const bool first = (K == 1);
+    if (!first && (K - 1) % m == 0) {
+        ring_flush(a, K, sh);
+        return;
+    }
+    const int64_t tid = gtid(), nth = gnth(), nv = a.n >> 1;
+    // plain loads (no const __restrict__): the first ones precede the PDL wait
+    const double *srcd = ring_slot(a.p, a.ring, (K - 1) % R);
+    double *dstd = ring_slot(a.p, a.ring, K % R);
+    const double2 *src = reinterpret_cast<const double2 *>(srcd);
+    double2 *dst = reinterpret_cast<double2 *>(dstd);
+    const double2 *__restrict__ r2 = reinterpret_cast<const double2 *>(a.r);
+    const int64_t step = kU * nth;
+    const int64_t b0 = (a.rev && tid < nv) ? tid + ((nv - 1 - tid) / step) * step : tid;
+    double2 ra[kU], pa[kU];
+    auto load_p = [&](int64_t b) {
+#pragma unroll
+        for (int u = 0; u < kU; ++u) {
+            const int64_t i = b + u * nth;
+            if (i < nv) pa[u] = src[i];
+        }
+    };
+    auto load_r = [&](int64_t b) {
+#pragma unroll
+        for (int u = 0; u < kU; ++u) {
+            const int64_t i = b + u * nth;
+            if (i < nv) ra[u] = r2[i];
+        }
+    };
+    if (!first) load_p(b0);
+    pdl_wait();
+    pdl_trigger();
+    load_r(b0);
+    double beta;
+    if (!ring_scalars(a, K, first, sh, &beta)) return;
+    for (int64_t b = b0; b >= 0 && b < nv;) {
+#pragma unroll
+        for (int u = 0; u < kU; ++u) {
+            const int64_t i = b + u * nth;
+            if (i < nv) {
+                double2 v = ra[u];
+                if (!first) {
+                    v.x = fma(beta, pa[u].x, ra[u].x);
+                    v.y = fma(beta, pa[u].y, ra[u].y);
+                }
+                dst[i] = v;
+            }
+        }
+        b += a.rev ? -step : step;
+        if (b >= 0 && b < nv) {
+            load_r(b);
+            if (!first) load_p(b);
+        }
+    }
+    if (tid == 0 && (a.n & 1)) {
+        const int64_t i = a.n - 1;
+        dstd[i] = first ? a.r[i] : fma(beta, srcd[i], a.r[i]);
+    }
+    if (a.trace) {
+        __syncthreads();
+        trace_mark(a.trace, a.trace_max, K, 0, true);
+    }
+}
+
+// end of a solve with the ring-deferred x update: the directions since the
+// last flush, j = F + 1 .. N with F = m floor((N - 1) / m) and N = niters (p
+// update N flushed up to N - 1 only when m divides N - 1), in ascending order
+__global__ void __launch_bounds__(kBlock) cg_xfix_ring_kernel(int64_t n, double *x, double *p0, PRing g,
+                                                              const CgScalars *sc) {
+    pdl_wait();
+    const int N = ldg_o(&sc->niters);
+    if (N < 1) return;
+    const int m = g.m, R = m + 1, F = m * ((N - 1) / m), c = N - F;
+    const double *pj[kRingMaxM];
+    double al[kRingMaxM];
+#pragma unroll
+    for (int t = 0; t < kRingMaxM; ++t) {
+        pj[t] = t < c ? ring_slot(p0, g, (F + 1 + t) % R) : nullptr;
+        al[t] = t < c ? ldg_o(&sc->alpha_h[(F + 1 + t) & 15]) : 0.0;
+    }
+    const int64_t tid = gtid(), nth = gnth(), nv = n >> 1;
+    double2 *__restrict__ x2 = reinterpret_cast<double2 *>(x);
+    for (int64_t i = tid; i < nv; i += nth) {
+        double2 xv = x2[i];
+#pragma unroll
+        for (int t = 0; t < kRingMaxM; ++t) {
+            if (t < c) {
+                const double2 pv = reinterpret_cast<const double2 *>(pj[t])[i];
+                xv.x = fma(al[t], pv.x, xv.x);
+                xv.y = fma(al[t], pv.y, xv.y);
+            }
+        }
+        x2[i] = xv;
+    }
+    if (tid == 0 && (n & 1)) {
+        double xv = x[n - 1];
+#pragma unroll
+        for (int t = 0; t < kRingMaxM; ++t)
+            if (t < c) xv = fma(al[t], pj[t][n - 1], xv);
+        x[n - 1] = xv;
+    }
+}
+
 // ---- a.6 + a.3 + a.4 fused and pipelined (HPCCG_OPT_FUSE_PSPMV): the p
 // update of iteration k and the SpMV Ap = A p_k in ONE kernel, single slab.
 // Chunk c = rows [512c, 512c + 512) (one 256-thread block's SpMV rows, 2 per
@@ -1889,6 +2141,7 @@ __global__ void __launch_bounds__(kBlock) cg_update1_kernel(Upd1Args a) {
         sc->pAp = pAp;
         sc->rr_prev = rtrans;
         sc->alpha_x = alpha;
+        sc->alpha_h[k & 15] = alpha;
         sc->k = k + 1;
         sc->run_q[a.q] = run;
         sc->done = !run;
@@ -1968,6 +2221,8 @@ __global__ void cg_initstate_kernel(CgScalars *sc, int max_iter, double tol,
     sc->done = done;
     sc->run_q[0] = !done;  // finisher-free loop: iteration 1 (parity 1) runs
     sc->run_q[1] = 0;
+    sc->ring_k[0] = 0;  // ring-deferred x update: p update 1 (parity 1) reads ring_k[0]
+    sc->ring_k[1] = 0;
     sc->epoch = sc->epoch + 1;
     set_cond(cond, !done);
 }

@@ -1015,26 +1015,35 @@ def test_peer_mode_nccl_one_rank():
 
 @pytest.mark.parametrize("dims,max_iter,tol", [((20, 30, 10), 150, 1e-12), ((31, 17, 9), 40, 0.0),
                                                ((64, 64, 64), 150, 1e-12), ((33, 9, 3), 7, 0.0),
-                                               ((128, 128, 128), 21, 0.0)])
+                                               ((21, 13, 7), 150, 1e-12), ((128, 128, 128), 21, 0.0),
+                                               ((64, 48, 40), 10, 0.0), ((64, 48, 40), 18, 0.0)])
 def test_defer_x_bitwise_identical(ctx, dims, max_iter, tol):
     """HPCCG_OPT_DEFER_X (x += alpha p moved into the next p update, the last
     one into cg_xfix_kernel): the same FMA on the same operands, so x, niters
     and normr are bit for bit those of the undeferred loop, in every launch
     mode (while-graph, per-iteration graph, plain launches with events);
-    and within the north_star tolerance of the oracle."""
+    and within the north_star tolerance of the oracle.  Depths m >= 2 defer
+    over a ring of m + 1 p buffers (flush every m iterations, the pending
+    ones in cg_xfix_ring_kernel): iteration counts that end 0 .. m - 1
+    iterations after a flush, odd n (31x17x9, 21x13x7, 33x9x3), and both walk
+    directions (serpentine)."""
     with H.Problem(ctx, *dims) as p:
         p.set_option(H.HPCCG_OPT_PERSISTENT, 0)        # the graph / plain loops, not on-chip
         outs = []
-        for defer in (0, 1):
+        for defer, serp in ((0, 0), (1, 0), (2, 0), (3, 3), (5, 0), (8, 0), (8, 3)):
             p.set_option(H.HPCCG_OPT_DEFER_X, defer)
+            p.set_option(H.HPCCG_OPT_SERPENTINE, serp)
             for mode in ("while", "graph", "timing"):
                 p.set_option(H.HPCCG_OPT_WHILE, 1 if mode == "while" else 0)
                 p.set_option(H.HPCCG_OPT_TIMING, 1 if mode == "timing" else 0)
                 p.set_vec(H.HPCCG_VEC_X, np.zeros(p.n))
                 r = p.solve(max_iter, tol)
+                assert p.stats()["x_deferred"] == defer, (defer, mode)
                 outs.append((defer, mode, r["niters"], r["normr"], p.get_vec(H.HPCCG_VEC_X)))
         p.set_option(H.HPCCG_OPT_TIMING, 0)
         p.set_option(H.HPCCG_OPT_WHILE, 1)
+        p.set_option(H.HPCCG_OPT_SERPENTINE, -1)
+        p.set_option(H.HPCCG_OPT_DEFER_X, -1)
         for o in outs[1:]:
             assert o[2:4] == outs[0][2:4], (o[:4], outs[0][:4])
             np.testing.assert_array_equal(o[4], outs[0][4])
