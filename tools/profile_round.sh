@@ -17,5 +17,10 @@ for cc in all none; do
   timeout 900 ncu --set full --clock-control none --cache-control $cc --import-source on \
       -k regex:"spmv27x2_kernel|cg_update1_kernel|cg_pupdate1_kernel" -s 0 -c 9 \
       -o gpurun_out/prof_${W}_$tag -f $B --steps 1 --warmup 3 --iters 5 > gpurun_out/ncu_$tag.log 2>&1
+  # the ring-deferred p update (HPCCG_OPT_DEFER_X auto = 8 beyond L2): p updates 1..10
+  # of the first solve -- 1 (p = r), 2..8 (2R:1W), 9 (the flush: x and 8 directions)
+  timeout 900 ncu --set full --clock-control none --cache-control $cc --import-source on \
+      -k regex:"cg_pupdate_ring_kernel" -s 0 -c 10 \
+      -o gpurun_out/prof_${W}_ring_$tag -f $B --steps 1 --warmup 3 --iters 12 > gpurun_out/ncu_ring_$tag.log 2>&1
 done
 tail -n 2 gpurun_out/ncu_*.log

@@ -18,7 +18,7 @@ import sys
 
 tag = sys.argv[1] if len(sys.argv) > 1 else "r2"
 W = sys.argv[2] if len(sys.argv) > 2 else "hpccg256"
-G, P = "gpurun_out", "profiles"
+G, P = "gpurun_out", os.environ.get("PROFILES_OUT", "profiles")
 os.makedirs(P, exist_ok=True)
 DIMS = {"hpccg256": (256, 256, 256), "hpccg128": (128, 128, 128), "hpccg512s": (512, 512, 512),
         "hpccg20": (20, 30, 10)}
@@ -127,6 +127,28 @@ def per_kernel(rows, n, nnz):
     return out
 
 
+RING_M = {"hpccg256": 8, "hpccg512s": 8}
+
+
+def per_ring(rows, n):
+    """cg_pupdate_ring_kernel launches K = 1, 2, ... of the first solve:
+    algorithmic bytes 16n (K = 1: r -> p), 24n (r, p -> p), (m + 4) 8n at the
+    flush (K - 1 divisible by m: r, p, x and m - 1 old p's -> p, x)."""
+    m = RING_M.get(W, 0)
+    out = []
+    for K, d in enumerate((r for r in rows if "cg_pupdate_ring_kernel" in r["kernel"]), start=1):
+        flush = K > 1 and (K - 1) % m == 0
+        alg = (16.0 if K == 1 else (m + 4) * 8.0 if flush else 24.0) * n
+        dram = num(d["dram__bytes_read.sum"]) + num(d["dram__bytes_write.sum"])
+        t = num(d["gpu__time_duration.sum"])
+        out.append({"K": K, "flush": flush, "algorithmic_bytes": alg, "dram_read": num(d["dram__bytes_read.sum"]),
+                    "dram_write": num(d["dram__bytes_write.sum"]), "dram_over_algorithmic": round(dram / alg, 4),
+                    "duration_us": round(t * 1e6, 2), "algorithmic_GBs": round(alg / t / 1e9, 1),
+                    "l2_hit_pct": d.get("lts__t_sector_hit_rate.pct"),
+                    "registers": d.get("launch__registers_per_thread")})
+    return out
+
+
 nx, ny, nz = DIMS[W]
 n, nnz = nx * ny * nz, nnz_of(nx, ny, nz)
 summary = {"tag": tag, "workload": W, "n": n, "nnz": nnz, "launch_list": launch_list()}
@@ -134,6 +156,10 @@ for cache in ("cold", "warm"):
     rows = full(f"prof_{W}_{cache}.ncu-rep")
     summary[f"{cache}_raw"] = rows
     summary[cache] = per_kernel(rows, n, nnz)
+    rr = full(f"prof_{W}_ring_{cache}.ncu-rep")
+    if rr:
+        summary[f"{cache}_ring_raw"] = rr
+        summary[f"{cache}_ring"] = per_ring(rr, n)
 out = os.path.join(P, f"{tag}_ncu_{W}.json")
 json.dump(summary, open(out, "w"), indent=1)
 sp = summary.get("cold", {}).get("spmv27x2_kernel")
@@ -152,3 +178,5 @@ print(json.dumps(summary["launch_list"][:8], indent=1))
 for cache in ("cold", "warm"):
     for k, v in summary[cache].items():
         print(cache, k, v["dram_over_algorithmic"], [x["duration_us"] for x in v["launches"]])
+    for x in summary.get(f"{cache}_ring", []):
+        print(cache, "ring K=%d" % x["K"], x["flush"], x["dram_over_algorithmic"], x["duration_us"], x["algorithmic_GBs"])
