@@ -652,6 +652,8 @@ def run_ours(args):
         opts.append((H.HPCCG_OPT_DEFER_X, 0))
     elif args.defer_x is not None:
         opts.append((H.HPCCG_OPT_DEFER_X, args.defer_x))
+    if args.spmv_cluster is not None:
+        opts.append((H.HPCCG_OPT_SPMV_CLUSTER, args.spmv_cluster))
     mode_want = 1 if args.halo == "peer" else 2
 
     def setup_multirank(prob):
@@ -1209,6 +1211,9 @@ def main():
                          "EFFECTIVE numbers of a different method (SURVEY 8(d): OUT), never the headline")
     ap.add_argument("--no-defer-x", action="store_true",
                     help="HPCCG_OPT_DEFER_X 0: update x in the x/r update (88n instead of 80n B/iteration)")
+    ap.add_argument("--spmv-cluster", type=int, default=None, choices=[-1, 0, 1],
+                    help="HPCCG_OPT_SPMV_CLUSTER: the CG SpMV in 8-CTA clusters, one p.Ap partial "
+                         "per cluster (default: the library's)")
     ap.add_argument("--defer-x", type=int, default=None,
                     help="HPCCG_OPT_DEFER_X: 1 = x deferred by one iteration, m = 2..8 over a ring of "
                          "m + 1 p buffers (default: the library's auto)")

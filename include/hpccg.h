@@ -187,6 +187,15 @@ extern "C" {
                                for the 8 CTA sums).  Every mode of a problem uses the same one
                                (identical bits across modes); the two differ in the last bits.
                                Measured no faster (256^3 986.3 vs 986.0 us/iteration): default 0 */
+#define HPCCG_OPT_SPMV_CLUSTER 29 /* single slab, finisher-free loop, 2-rows/thread SpMV: launch
+                               the CG SpMV in clusters of 8 CTAs that fold their p.Ap partials
+                               into one through distributed shared memory (cluster-rank order),
+                               so a slab of up to 8 x 4096 x 512 rows leaves <= 4096 partials and
+                               the update blocks sum them without the p.Ap finisher kernel.
+                               A different (fixed) summation tree: results are deterministic
+                               and within the oracle tolerance, not bitwise the unclustered
+                               loop's.  0 (default) off, 1 on, -1 auto (on when the unclustered
+                               SpMV would leave more than 4096 partials) */
 #define HPCCG_OPT_SPMV_SLICED 28 /* single slab, finisher-free loop: the CG SpMV reads a
                                CHUNK-SLICED copy of the matrix (128 rows' val[27][128] +
                                col[27][128] contiguous, built from the slot-major ELL at

@@ -183,6 +183,7 @@ struct hpccg_problem {
     int opt_spmv_trips = 1;            // single-slab SpMV trips per block (0 auto, 1 off, T)
     int opt_pap_cluster = 0;           // p.Ap finisher as one 8-CTA cluster (1) or one CTA (0)
     int opt_sliced = 0;                // CG SpMV from the chunk-sliced copy via TMA (-1 auto, 0, 1)
+    int opt_spmv_cl = 0;               // CG SpMV in 8-CTA clusters, one p.Ap partial per cluster (-1 auto, 0, 1)
     int opt_ps_lead = 0;               // its production lead in chunks (0: plane / 512 + 8)
     std::vector<void *> ipc_opened;    // peers' buffers mapped with cudaIpcOpenMemHandle
     int last_persist_mode = 3;
@@ -755,6 +756,18 @@ int spmv_trips(const hpccg_problem *p) {
 }
 
 int defer_m(const hpccg_problem *p);
+bool fuse_ps_on(hpccg_problem *p);
+
+// HPCCG_OPT_SPMV_CLUSTER: the single-slab CG SpMV (finisher-free loop, 2 rows
+// per thread) in clusters of kSpmvCl CTAs, one p.Ap partial per cluster; auto:
+// when the per-CTA partials would exceed what the update blocks sum themselves
+bool spmv_cl_on(const hpccg_problem *p) {
+    if (p->ctx->mode != MODE_SINGLE || p->opt_spmv_cl == 0 || !ff_path(p)) return false;
+    const Slab &s = p->slabs[0];
+    if (s.dia || sliced_on(p) || spmv_trips(p) > 1 || fuse_ps_on(const_cast<hpccg_problem *>(p))) return false;
+    if (spmv_rows_per_thread(p->opt_rows, spmv_args(s, s.p, s.Ap), 0, 0) != 2) return false;
+    return p->opt_spmv_cl == 1 || spmv_blocks(s.n, 2) > (int64_t)kUpdSumMax;
+}
 
 int cg_spmv_all(hpccg_problem *p, bool timing, bool check) {
     hpccg_ctx *ctx = p->ctx;
@@ -791,6 +804,32 @@ int cg_spmv_all(hpccg_problem *p, bool timing, bool check) {
             const unsigned char *sl = s.sl;
             if (check) CU(cudaLaunchKernelEx(&cfg, spmv_sliced_kernel<true>, a, sl));
             else CU(cudaLaunchKernelEx(&cfg, spmv_sliced_kernel<false>, a, sl));
+            return check_launch(ctx);
+        }
+        if (spmv_cl_on(p)) {
+            a.r0 = 0;
+            a.len0 = s.n;
+            const int64_t nb = spmv_blocks(s.n, 2), g = cdiv(nb, kSpmvCl) * kSpmvCl;
+            a.nb0 = g;
+            a.total_blocks = (unsigned)g;
+            cudaLaunchConfig_t cfg{};
+            cfg.gridDim = dim3((unsigned)g);
+            cfg.blockDim = dim3(kBlock);
+            cfg.stream = ctx->stream;
+            cudaLaunchAttribute at[2];
+            int na = 0;
+            at[na].id = cudaLaunchAttributeClusterDimension;
+            at[na].val.clusterDim.x = kSpmvCl;
+            at[na].val.clusterDim.y = 1;
+            at[na++].val.clusterDim.z = 1;
+            if (p->opt_pdl) {
+                at[na].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+                at[na++].val.programmaticStreamSerializationAllowed = 1;
+            }
+            cfg.attrs = at;
+            cfg.numAttrs = na;
+            if (check) CU(cudaLaunchKernelEx(&cfg, spmv27x2_cl_kernel<true>, a));
+            else CU(cudaLaunchKernelEx(&cfg, spmv27x2_cl_kernel<false>, a));
             return check_launch(ctx);
         }
         const int trips = spmv_trips(p);
@@ -837,6 +876,7 @@ double **tab(hpccg_problem *p, int which) { return p->d_tab + (size_t)which * p-
 // SpMV partial count of a single slab's CG SpMV (the update sums them).
 unsigned single_spmv_parts(const hpccg_problem *p, const Slab &s) {
     if (sliced_on(p)) return (unsigned)sliced_grid(p->ctx);
+    if (spmv_cl_on(p)) return (unsigned)cdiv(spmv_blocks(s.n, 2), kSpmvCl);
     const int trips = spmv_trips(p);
     if (trips > 1) return (unsigned)cdiv(spmv_blocks(s.n, 2), trips);
     return (unsigned)spmv_blocks(s.n, spmv_rows_per_thread(p->opt_rows, spmv_args(s, s.p, s.Ap), 0, 0));
@@ -2643,6 +2683,13 @@ int hpccg_set_option(hpccg_problem *p, int key, int64_t value) {
             p->graph = p->wgraph = nullptr;
             p->opt_sliced = (int)value;
             return sliced_alloc(p);
+        case HPCCG_OPT_SPMV_CLUSTER:
+            if (value < -1 || value > 1) return fail(HPCCG_EINVAL, "spmv cluster: -1 (auto), 0 or 1");
+            if (p->graph) cudaGraphExecDestroy(p->graph);
+            if (p->wgraph) cudaGraphExecDestroy(p->wgraph);
+            p->graph = p->wgraph = nullptr;
+            p->opt_spmv_cl = (int)value;
+            return HPCCG_OK;
         case HPCCG_OPT_PAP_CLUSTER:
             if (value != 0 && value != 1) return fail(HPCCG_EINVAL, "pap cluster: 0 or 1");
             if (p->graph) cudaGraphExecDestroy(p->graph);

@@ -750,7 +750,14 @@ __device__ __forceinline__ int2 spmv_cols(const SpmvArgs &a, const int *c, int s
     return make_int2(v.x != 0.0 ? own + off : own, v.y != 0.0 ? own + 1 + off : own + 1);
 }
 
-template <int kDots, bool kCheck, bool kFused, bool kCoh, bool kDia = false>
+// HPCCG_OPT_SPMV_CLUSTER: the single-slab CG SpMV launched in clusters of
+// kSpmvCl CTAs; each cluster folds its CTAs' p.Ap partials (row-block order)
+// into ONE partial through distributed shared memory, so a 256^3 slab
+// leaves 4096 partials -- few enough for every update block to sum itself, no
+// 1024-thread finisher kernel between the SpMV and the update
+constexpr int kSpmvCl = 8;
+
+template <int kDots, bool kCheck, bool kFused, bool kCoh, bool kDia = false, bool kCl = false>
 __device__ __forceinline__ void spmv27x2_body(const SpmvArgs &a, int64_t row, int64_t lim, int64_t bid) {
     constexpr bool kDot = kDots == 1;
     double d = 0.0, dg = 0.0;  // kDots 1: p.Ap; kDots 2: delta (d) and gamma (dg)
@@ -835,6 +842,22 @@ __device__ __forceinline__ void spmv27x2_body(const SpmvArgs &a, int64_t row, in
         if (a.parts_only) {  // block partial only; the update kernel sums them
             __shared__ double shp[32];
             d = block_reduce<false>(d, shp);
+            if (kCl) {
+                __shared__ double clp[kSpmvCl];
+                namespace cgx = cooperative_groups;
+                cgx::cluster_group cl = cgx::this_cluster();
+                // slot by row block (not cluster rank): the same sum when the grid
+                // walks the rows backwards (serpentine)
+                if (threadIdx.x == 0) *cl.map_shared_rank(&clp[bid % kSpmvCl], 0) = d;
+                cl.sync();
+                if (cl.block_rank() == 0 && threadIdx.x == 0) {
+                    double t = clp[0];
+#pragma unroll
+                    for (int c = 1; c < kSpmvCl; ++c) t += clp[c];
+                    a.parts_only[a.part_base + bid / kSpmvCl] = t;
+                }
+                return;
+            }
             if (threadIdx.x == 0) a.parts_only[a.part_base + bid] = d;
             return;
         }
@@ -1092,6 +1115,15 @@ __global__ void __launch_bounds__(kBlock, kDia ? kDiaMinB : 4) spmv27x2_kernel(S
         return;
     }
     spmv27x2_body<kDots, kCheck, kFused, false, kDia>(a, row, lim, bid);
+}
+
+// the single-slab CG SpMV in clusters of kSpmvCl CTAs (grid a multiple of
+// kSpmvCl; the padding blocks have no rows and contribute 0)
+template <bool kCheck>
+__global__ void __launch_bounds__(kBlock, 4) spmv27x2_cl_kernel(SpmvArgs a) {
+    const int64_t bid = spmv_bid(a);
+    const int64_t row = a.r0 + (bid * kBlock + threadIdx.x) * 2, lim = a.r0 + a.len0;
+    spmv27x2_body<1, kCheck, false, false, false, true>(a, row, lim, bid);
 }
 
 // ------------------------------------------------ streaming vector kernels

@@ -1177,6 +1177,49 @@ def test_pap_cluster_finisher(ctx):
         assert outs[(1, "while")][2] < 1e-13 and outs[(1, "while")][1] <= 1e-12
 
 
+@pytest.mark.parametrize("dims,max_iter,tol", [((64, 64, 64), 150, 1e-12), ((31, 17, 10), 150, 1e-12),
+                                               ((48, 16, 50), 40, 0.0), ((128, 128, 160), 150, 1e-12)])
+def test_spmv_cluster_parity(ctx, dims, max_iter, tol):
+    """HPCCG_OPT_SPMV_CLUSTER forced on: the CG SpMV in 8-CTA clusters, one
+    p.Ap partial per cluster through distributed shared memory (grid padded
+    to a multiple of 8: 31x17x10 has 5 row blocks, 48x16x50 38).  Another
+    fixed reduction tree: within the oracle tolerance, bitwise the same in
+    every launch mode and run to run, with and without the ring-deferred x
+    update and serpentine order; the first CG step is exact (alpha_1 = b.b /
+    b.Ab in integers), so x_1 pins every Ap row and the cluster sum bitwise."""
+    with H.Problem(ctx, *dims) as p:
+        p.set_option(H.HPCCG_OPT_PERSISTENT, 0)
+        p.set_option(H.HPCCG_OPT_SPMV_CLUSTER, 1)
+        ref = oracle.generate(*dims)
+        p.set_vec(H.HPCCG_VEC_X, np.zeros(p.n))
+        p.solve(2, 0.0)
+        np.testing.assert_array_equal(p.get_vec(H.HPCCG_VEC_X), oracle.cg(ref, 2, 0.0)["x"])
+        oref = oracle.cg(ref, max_iter, tol) if p.n <= 300_000 else None
+        outs = []
+        for defer, serp in ((0, 0), (8, 3), (1, 0)):
+            p.set_option(H.HPCCG_OPT_DEFER_X, defer)
+            p.set_option(H.HPCCG_OPT_SERPENTINE, serp)
+            for mode in ("while", "graph", "timing"):
+                p.set_option(H.HPCCG_OPT_WHILE, 1 if mode == "while" else 0)
+                p.set_option(H.HPCCG_OPT_TIMING, 1 if mode == "timing" else 0)
+                p.set_vec(H.HPCCG_VEC_X, np.zeros(p.n))
+                r = p.solve(max_iter, tol)
+                outs.append((r["niters"], r["normr"], p.get_vec(H.HPCCG_VEC_X)))
+                if oref is not None:
+                    check_cg(r, p.maxabsdiff(), oref, ref)
+                else:
+                    assert r["normr"] <= 1e-12 and p.maxabsdiff() < 1e-13
+        for k in (H.HPCCG_OPT_TIMING, H.HPCCG_OPT_SPMV_CLUSTER):
+            p.set_option(k, 0)
+        for k in (H.HPCCG_OPT_WHILE,):
+            p.set_option(k, 1)
+        for k in (H.HPCCG_OPT_SERPENTINE, H.HPCCG_OPT_DEFER_X):
+            p.set_option(k, -1)
+        for o in outs[1:]:
+            assert o[:2] == outs[0][:2]
+            np.testing.assert_array_equal(o[2], outs[0][2])
+
+
 # ------------- the scaling configurations' GLOBAL problems on one GPU (loopback)
 
 @pytest.mark.parametrize("P,nz,expect", [(2, 256, 113), (4, 256, 114), (8, 256, 115), (8, 64, 115)])
