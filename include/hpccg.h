@@ -471,7 +471,9 @@ typedef struct hpccg_tri hpccg_tri;
  * frees with hpccg_tri_free.  EINVAL if n < 1. */
 HPCCG_API int hpccg_tri_generate(hpccg_ctx *ctx, int64_t n, hpccg_tri **out);
 
-/* Borrowed device pointer (n doubles) to X, B, R, P or a coefficient array. */
+/* Borrowed device pointer (n doubles) to X, B, R, P or a coefficient array
+ * (P: the buffer holding the last solve's final p -- a ring slot after a
+ * variant-2 solve). */
 HPCCG_API int hpccg_tri_vec(hpccg_tri *t, int which, double **dev_ptr);
 
 /* y = A x (Fig. 12 matvecmul): y_i = a0_i x_{i-1} + a1_i x_i + a2_i x_{i+1}
@@ -482,9 +484,15 @@ HPCCG_API int hpccg_tri_spmv(hpccg_tri *t, const double *x, double *y);
 /* Reset x = 0, r = p = b and run the CG.  variant 0: the iteration exactly as
  * Fig. 12 writes it -- copy r_old, matvec, 5 dots, 3 axpys (axpy(i, a, x, y):
  * x[i] += a*y[i]), 2 more copies -- with every scalar on the device; variant
- * 1: fused (matvec + p.s, x/r update + r.r, p update).  Both run as one graph
- * with a device-driven WHILE node.  *iters, *cond (last r.r), *ms (device
- * time of the whole solve): HOST out, nullable. */
+ * 1: fused (matvec + p.s, x/r update + r.r, p update: 112n B per iteration);
+ * variant 2: variant 1 with x += alpha_k p_k deferred over 8 iterations
+ * through a ring of 9 p buffers (p_k in slot (k - 1) % 9; x read and written
+ * once per 8 iterations, the pending directions applied after the loop: 97n
+ * B per iteration, 8 more p-sized device buffers allocated on first use) --
+ * the same FMAs on x in the same order, so bitwise variant 1's x, iterations,
+ * r.r and p.  All run as one graph with a device-driven WHILE node.  *iters,
+ * *cond (last r.r), *ms (device time of the whole solve): HOST out, nullable.
+ * EINVAL for another variant. */
 HPCCG_API int hpccg_tri_solve(hpccg_tri *t, int max_iter, double tol, int variant, int *iters,
                               double *cond, double *ms);
 

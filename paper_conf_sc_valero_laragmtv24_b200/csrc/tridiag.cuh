@@ -4,7 +4,10 @@
 // one CG iteration timed.  Two iteration structures:
 //   variant 0 -- Fig. 12 as written: 3 copies, 1 matvec, 5 dots, 3 axpys per
 //                iteration (12 kernels + 1 control kernel), scalars on device;
-//   variant 1 -- fused: matvec + p.s, x/r update + r.r, p update (3 kernels).
+//   variant 1 -- fused: matvec + p.s, x/r update + r.r, p update (3 kernels);
+//   variant 2 -- variant 1 with x deferred over kTriM iterations (a ring of
+//                kTriM + 1 p buffers, the same FMAs on x in the same order:
+//                bitwise variant 1's results) -- 97n instead of 112n B.
 // Included by hpccg.cu (one translation unit).
 #pragma once
 
@@ -22,7 +25,22 @@ struct TriScalars {
     double tol;
     int it;           // iterations done
     int max_iter;
+    double alpha_h[16];  // variant 2: alpha of iteration k in slot k & 15
 };
+
+// variant 2: p_k (iteration k's direction) lives in slot (k - 1) % (m + 1);
+// slot 0 is the problem's p buffer (the init writes p_1 = b there), slots
+// j >= 1 at base + (j - 1) stride.  m == 0: no ring (variants 0 / 1).
+constexpr int kTriM = 8;
+struct TriRing {
+    double *p0, *base;
+    int64_t stride;
+    int m;
+};
+
+__host__ __device__ __forceinline__ double *tri_slot(const TriRing &g, int j) {
+    return j == 0 ? g.p0 : g.base + (int64_t)(j - 1) * g.stride;
+}
 
 // a0[i] = 1 (i > 0), a1[i] = 4, a2[i] = 1 (i < n-1), zero outside; b = 0.5.
 __global__ void __launch_bounds__(kBlock) tri_gen_kernel(int64_t n, double *a0, double *a1, double *a2,
@@ -44,10 +62,13 @@ __global__ void __launch_bounds__(kBlock) tri_spmv_kernel(int64_t n, const doubl
                                                          const double *__restrict__ a2,
                                                          const double *__restrict__ x,
                                                          double *__restrict__ y, Reduction red,
-                                                         double *dot_out) {
+                                                         double *dot_out, TriRing g = TriRing{},
+                                                         const TriScalars *sc = nullptr) {
     const uint64_t pol = policy_evict_first();
     pdl_wait();
     pdl_trigger();
+    // variant 2: iteration it + 1 gathers p_(it+1) from slot it % (m + 1)
+    if (g.m >= 2) x = tri_slot(g, ldg_o(&sc->it) % (g.m + 1));
     double d = 0.0;
     const int64_t nth = gnth();
     for (int64_t b0 = gtid(); b0 < n; b0 += kTriU * nth) {
@@ -201,6 +222,9 @@ __global__ void __launch_bounds__(kBlock) tri_rr_kernel(int64_t n, const double 
 
 // variant 1: alpha = rr / p.s; r = fma(-alpha, s, r); x = fma(alpha, p, x);
 // r.r -> last block: beta = rr_new / rr, cond = rr_new, it++, loop control.
+// kDefer (variant 2): x is left to the p updates (alpha -> sc->alpha_h), so
+// this pass reads s, r and writes r only (24n instead of 48n B)
+template <bool kDefer = false>
 __global__ void __launch_bounds__(kBlock) tri_update_kernel(int64_t n, double *__restrict__ x,
                                                            double *__restrict__ r,
                                                            const double *__restrict__ p,
@@ -212,6 +236,7 @@ __global__ void __launch_bounds__(kBlock) tri_update_kernel(int64_t n, double *_
     const double rr = ldg_o(&sc->rr);
     const double alpha = rr / ldg_o(&sc->pAp);
     const double nalpha = alpha * (-1.0);
+    if (kDefer && blockIdx.x == 0 && threadIdx.x == 0) sc->alpha_h[(ldg_o(&sc->it) + 1) & 15] = alpha;
     double acc = 0.0;
     const int64_t nth = gnth();
     for (int64_t b0 = gtid(); b0 < n; b0 += kTriU * nth) {
@@ -222,8 +247,10 @@ __global__ void __launch_bounds__(kBlock) tri_update_kernel(int64_t n, double *_
             if (i < n) {
                 sv[u] = s[i];
                 rv[u] = r[i];
-                pv[u] = p[i];
-                xv[u] = x[i];
+                if (!kDefer) {
+                    pv[u] = p[i];
+                    xv[u] = x[i];
+                }
             }
         }
 #pragma unroll
@@ -232,7 +259,7 @@ __global__ void __launch_bounds__(kBlock) tri_update_kernel(int64_t n, double *_
             if (i < n) {
                 const double rn = fma(nalpha, sv[u], rv[u]);
                 r[i] = rn;
-                x[i] = fma(alpha, pv[u], xv[u]);
+                if (!kDefer) x[i] = fma(alpha, pv[u], xv[u]);
                 acc = fma(rn, rn, acc);
             }
         }
@@ -270,6 +297,93 @@ __global__ void __launch_bounds__(kBlock) tri_pupdate_kernel(int64_t n, const do
             const int64_t i = b0 + u * nth;
             if (i < n) p[i] = fma(beta, pv[u], rv[u]);
         }
+    }
+}
+
+// variant 2: p_(k+1) = r + beta p_k into slot k % (m + 1) (k = it, after the
+// update of iteration k); when m divides k also x = fma(alpha_j, p_j, x) for
+// j = k - m + 1 .. k ascending -- the x/r update's FMAs of variant 1, m
+// iterations at a time.  Flush iterations take one element per thread per
+// trip (m + 2 loads in flight).
+__global__ void __launch_bounds__(kBlock) tri_pupdate_ring_kernel(int64_t n, const double *__restrict__ r,
+                                                                 double *x, TriRing g,
+                                                                 const TriScalars *sc) {
+    pdl_wait();
+    pdl_trigger();
+    const double beta = ldg_o(&sc->slot[2]);
+    const int k = ldg_o(&sc->it), m = g.m, R = m + 1;
+    const double *src = tri_slot(g, (k - 1) % R);
+    double *dst = tri_slot(g, k % R);
+    const int64_t nth = gnth();
+    if (k < 1) return;  // (max_iter 0: the body never runs)
+    if (k % m != 0) {
+        for (int64_t b0 = gtid(); b0 < n; b0 += kTriU * nth) {
+            double pv[kTriU], rv[kTriU];
+#pragma unroll
+            for (int u = 0; u < kTriU; ++u) {
+                const int64_t i = b0 + u * nth;
+                if (i < n) {
+                    pv[u] = src[i];
+                    rv[u] = r[i];
+                }
+            }
+#pragma unroll
+            for (int u = 0; u < kTriU; ++u) {
+                const int64_t i = b0 + u * nth;
+                if (i < n) dst[i] = fma(beta, pv[u], rv[u]);
+            }
+        }
+        return;
+    }
+    __shared__ const double *sop[kTriM];
+    __shared__ double sal[kTriM];
+    if (threadIdx.x < kTriM) {
+        const int t = threadIdx.x, j = k - m + 1 + t;  // iterations k - m + 1 .. k
+        sop[t] = t < m ? tri_slot(g, (j - 1) % R) : nullptr;
+        sal[t] = t < m ? ldg_o(&sc->alpha_h[j & 15]) : 0.0;
+    }
+    __syncthreads();
+    const double am = sal[m - 1];
+    for (int64_t i = gtid(); i < n; i += nth) {
+        double ov[kTriM - 1];
+        const double rv = r[i], pk = src[i];  // p_k: the last direction (slot (k - 1) % R)
+        double xv = x[i];
+#pragma unroll
+        for (int t = 0; t < kTriM - 1; ++t)
+            if (t < m - 1) ov[t] = sop[t][i];
+#pragma unroll
+        for (int t = 0; t < kTriM - 1; ++t)
+            if (t < m - 1) xv = fma(sal[t], ov[t], xv);
+        x[i] = fma(am, pk, xv);
+        dst[i] = fma(beta, pk, rv);
+    }
+}
+
+// variant 2, after the loop: the directions since the last flush, j = F + 1
+// .. N with F = m floor(N / m), N = it
+__global__ void __launch_bounds__(kBlock) tri_xfix_kernel(int64_t n, double *x, TriRing g,
+                                                         const TriScalars *sc) {
+    pdl_wait();
+    const int N = ldg_o(&sc->it), m = g.m, R = m + 1, F = m * (N / m), c = N - F;
+    if (c == 0) return;
+    __shared__ const double *sop[kTriM];
+    __shared__ double sal[kTriM];
+    if (threadIdx.x < kTriM) {
+        const int t = threadIdx.x, j = F + 1 + t;
+        sop[t] = t < c ? tri_slot(g, (j - 1) % R) : nullptr;
+        sal[t] = t < c ? ldg_o(&sc->alpha_h[j & 15]) : 0.0;
+    }
+    __syncthreads();
+    for (int64_t i = gtid(); i < n; i += gnth()) {
+        double ov[kTriM];
+#pragma unroll
+        for (int t = 0; t < kTriM; ++t)
+            if (t < c) ov[t] = sop[t][i];
+        double xv = x[i];
+#pragma unroll
+        for (int t = 0; t < kTriM; ++t)
+            if (t < c) xv = fma(sal[t], ov[t], xv);
+        x[i] = xv;
     }
 }
 

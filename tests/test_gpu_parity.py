@@ -519,11 +519,12 @@ def test_tri_generate_and_spmv_bitwise(ctx, n):
         np.testing.assert_array_equal(y.cpu().numpy(), oracle.tri_spmv(ref, x))
 
 
-@pytest.mark.parametrize("variant", [0, 1])
+@pytest.mark.parametrize("variant", [0, 1, 2])
 @pytest.mark.parametrize("n,tol", [(1000, 1e-12), (100_003, 1e-20), (7, 1e-30), (3_000_000, 1e-24)])
 def test_tri_cg_vs_oracle(ctx, variant, n, tol):
-    """Fig. 12 as written (variant 0) and fused (variant 1) against the
-    oracle's Fig. 12: iterations +-1, x within 1e-10, final r.r <= tol."""
+    """Fig. 12 as written (variant 0), fused (variant 1) and fused with the
+    ring-deferred x update (variant 2) against the oracle's Fig. 12:
+    iterations +-1, x within 1e-10, final r.r <= tol."""
     with H.Tri(ctx, n) as t:
         ref = oracle.Tri(n)
         o = oracle.tri_cg(ref, 300, tol)
@@ -533,7 +534,7 @@ def test_tri_cg_vs_oracle(ctx, variant, n, tol):
         assert np.max(np.abs(t.get(H.HPCCG_TRI_X) - o["x"])) <= CG_ATOL
 
 
-@pytest.mark.parametrize("variant", [0, 1])
+@pytest.mark.parametrize("variant", [0, 1, 2])
 def test_tri_cg_first_step_and_fixed_count(ctx, variant):
     """max_iter 1: x1 = alpha/2 with alpha = n/(6n-2) correctly rounded (exact
     integer dots); tol 0 runs exactly max_iter iterations."""
@@ -546,6 +547,25 @@ def test_tri_cg_first_step_and_fixed_count(ctx, variant):
         np.testing.assert_array_equal(t.get(H.HPCCG_TRI_X), np.full(n, alpha / 2))
         g = t.solve(17, 0.0, variant)
         assert g["iters"] == 17
+
+
+@pytest.mark.parametrize("n", [7, 1000, 100_003, 1_000_001])
+def test_tri_ring_variant_bitwise(ctx, n):
+    """Variant 2 defers x += alpha_k p_k over 8 iterations through a ring of 9
+    p buffers (flush in the p update of every 8th iteration, the rest after
+    the loop): the same FMAs on x in the same order as variant 1, so x, the
+    iteration count, r.r and the final p are bit for bit variant 1's -- for
+    iteration counts ending 0..7 after a flush, and for tol-stopped solves."""
+    with H.Tri(ctx, n) as t:
+        for max_iter, tol in [(1, 0.0), (2, 0.0), (7, 0.0), (8, 0.0), (9, 0.0), (16, 0.0), (21, 0.0),
+                              (300, 1e-24)]:
+            out = []
+            for v in (1, 2):
+                g = t.solve(max_iter, tol, v)
+                out.append((g["iters"], g["cond"], t.get(H.HPCCG_TRI_X), t.get(H.HPCCG_TRI_P)))
+            assert out[0][:2] == out[1][:2], (max_iter, out[0][:2], out[1][:2])
+            np.testing.assert_array_equal(out[0][2], out[1][2])
+            np.testing.assert_array_equal(out[0][3], out[1][3])
 
 
 def test_tri_full_size_sampled(ctx):
@@ -570,7 +590,7 @@ def test_tri_full_size_sampled(ctx):
             exp.append(s)
         np.testing.assert_array_equal(y.cpu().numpy()[rows], np.array(exp))
         alpha = float(Fraction(n, 6 * n - 2))
-        for v in (0, 1):
+        for v in (0, 1, 2):
             g = t.solve(1, 0.0, v)
             xv = t.view(H.HPCCG_TRI_X)
             assert g["iters"] == 1 and float(xv[rows].max()) == float(xv[rows].min()) == alpha / 2
