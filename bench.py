@@ -654,6 +654,9 @@ def run_ours(args):
         opts.append((H.HPCCG_OPT_DEFER_X, args.defer_x))
     if args.spmv_cluster is not None:
         opts.append((H.HPCCG_OPT_SPMV_CLUSTER, args.spmv_cluster))
+    for kv in args.opt:  # experiments: any library option, e.g. --opt SMEM_HALO=0
+        k, v = kv.split("=")
+        opts.append((getattr(H, "HPCCG_OPT_" + k), int(v)))
     mode_want = 1 if args.halo == "peer" else 2
 
     def setup_multirank(prob):
@@ -1219,6 +1222,8 @@ def main():
                          "EFFECTIVE numbers of a different method (SURVEY 8(d): OUT), never the headline")
     ap.add_argument("--no-defer-x", action="store_true",
                     help="HPCCG_OPT_DEFER_X 0: update x in the x/r update (88n instead of 80n B/iteration)")
+    ap.add_argument("--opt", action="append", default=[], metavar="NAME=VALUE",
+                    help="set HPCCG_OPT_<NAME> on every CG problem (experiments; repeatable)")
     ap.add_argument("--spmv-cluster", type=int, default=None, choices=[-1, 0, 1],
                     help="HPCCG_OPT_SPMV_CLUSTER: the CG SpMV in 8-CTA clusters, one p.Ap partial "
                          "per cluster (default: the library's)")

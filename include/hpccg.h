@@ -187,6 +187,15 @@ extern "C" {
                                for the 8 CTA sums).  Every mode of a problem uses the same one
                                (identical bits across modes); the two differ in the last bits.
                                Measured no faster (256^3 986.3 vs 986.0 us/iteration): default 0 */
+#define HPCCG_OPT_SMEM_HALO 30 /* the on-chip (shared-memory cluster) solve: every CTA keeps the
+                               gathered vector (p; r for the single-reduction CG) with the
+                               stencil's reach (plane + nx + 1 rows) of halo on each side in its
+                               own shared memory, refreshed once per SpMV by coalesced reads of
+                               the owner CTAs' rows, so the 27 gathers of a row are local
+                               instead of distributed-shared-memory reads.  The same values in
+                               the same order: bitwise the unhalo'd solve.  -1 (default) auto /
+                               1: when the halo (16 (plane + nx + 1) B per CTA) fits next to the
+                               rows; 0 off */
 #define HPCCG_OPT_SPMV_CLUSTER 29 /* single slab, finisher-free loop, 2-rows/thread SpMV: launch
                                the CG SpMV in clusters of 8 CTAs that fold their p.Ap partials
                                into one through distributed shared memory (cluster-rank order),

@@ -183,6 +183,7 @@ struct hpccg_problem {
     int opt_spmv_trips = 1;            // single-slab SpMV trips per block (0 auto, 1 off, T)
     int opt_pap_cluster = 0;           // p.Ap finisher as one 8-CTA cluster (1) or one CTA (0)
     int opt_sliced = 0;                // CG SpMV from the chunk-sliced copy via TMA (-1 auto, 0, 1)
+    int opt_smem_halo = -1;            // on-chip solve: gathered vector halo'd in every CTA (-1 auto, 0, 1)
     int opt_spmv_cl = 0;               // CG SpMV in 8-CTA clusters, one p.Ap partial per cluster (-1 auto, 0, 1)
     int opt_ps_lead = 0;               // its production lead in chunks (0: plane / 512 + 8)
     std::vector<void *> ipc_opened;    // peers' buffers mapped with cudaIpcOpenMemHandle
@@ -1700,6 +1701,16 @@ int64_t smem_rows(const hpccg_problem *p) {
     return p->slabs[0].dia && R * smem_bytes_per_row(sr, true) <= ctx->smem_bytes ? R : 0;
 }
 
+// on-chip solve: halo rows per side of the gathered vector's local copy in
+// every CTA (the stencil's reach, plane + nx + 1), 0 when it does not fit
+// (the gathers then read the owner CTAs' shared memory)
+int64_t smem_halo(const hpccg_problem *p, int64_t R, int64_t bytes_per_row) {
+    if (p->opt_smem_halo == 0) return 0;
+    const Slab &s = p->slabs[0];
+    const int64_t H = s.plane + s.nx + 1;
+    return R * bytes_per_row + 2 * H * (int64_t)sizeof(double) <= p->ctx->smem_bytes ? H : 0;
+}
+
 // the on-chip solve keeps no column slice (DIA reading): format 1 and the ELL slice does not fit
 bool smem_dia(const hpccg_problem *p, int64_t R) {
     return p->slabs[0].dia && R * smem_bytes_per_row(p->opt_variant == 1, false) > p->ctx->smem_bytes;
@@ -1746,13 +1757,15 @@ int launch_persistent(hpccg_problem *p, int max_iter, double tol) {
             m.sc = s.sc;
             m.max_iter = max_iter;
             m.tol = tol;
+            const int64_t H = smem_halo(p, R, bytes_per_row);
+            m.H = (int)H;
             const int64_t g = cdiv(s.n, R);
             cudaLaunchConfig_t cfg{};
             // auto: 512 threads when a CTA holds more than 256 rows (one trip)
             const int nt = p->opt_smem_threads ? p->opt_smem_threads : (R > kBlock ? 512 : kBlock);
             cfg.gridDim = dim3((unsigned)g);
             cfg.blockDim = dim3(nt);
-            cfg.dynamicSmemBytes = (size_t)(R * bytes_per_row);
+            cfg.dynamicSmemBytes = (size_t)(R * bytes_per_row + 2 * H * (int64_t)sizeof(double));
             cfg.stream = ctx->stream;
             cudaLaunchAttribute at[1];
             at[0].id = cudaLaunchAttributeClusterDimension;
@@ -1761,25 +1774,20 @@ int launch_persistent(hpccg_problem *p, int max_iter, double tol) {
             at[0].val.clusterDim.z = 1;
             cfg.attrs = at;
             cfg.numAttrs = 1;
-            if (nt == 512) {
-                if (m.dia) {
-                    if (sr) CU(cudaLaunchKernelEx(&cfg, cg_smem_cluster_kernel<512, true, true>, m));
-                    else CU(cudaLaunchKernelEx(&cfg, cg_smem_cluster_kernel<512, false, true>, m));
-                } else if (sr) {
-                    CU(cudaLaunchKernelEx(&cfg, cg_smem_cluster_kernel<512, true>, m));
-                } else {
-                    CU(cudaLaunchKernelEx(&cfg, cg_smem_cluster_kernel<512, false>, m));
-                }
+            auto pick = [&](auto k512, auto k256) { return nt == 512 ? k512 : k256; };
+            void (*kern)(SmemArgs) = nullptr;
+            if (H > 0) {
+                if (m.dia) kern = sr ? pick(cg_smem_cluster_kernel<512, true, true, true>, cg_smem_cluster_kernel<kBlock, true, true, true>)
+                                     : pick(cg_smem_cluster_kernel<512, false, true, true>, cg_smem_cluster_kernel<kBlock, false, true, true>);
+                else kern = sr ? pick(cg_smem_cluster_kernel<512, true, false, true>, cg_smem_cluster_kernel<kBlock, true, false, true>)
+                               : pick(cg_smem_cluster_kernel<512, false, false, true>, cg_smem_cluster_kernel<kBlock, false, false, true>);
             } else {
-                if (m.dia) {
-                    if (sr) CU(cudaLaunchKernelEx(&cfg, cg_smem_cluster_kernel<kBlock, true, true>, m));
-                    else CU(cudaLaunchKernelEx(&cfg, cg_smem_cluster_kernel<kBlock, false, true>, m));
-                } else if (sr) {
-                    CU(cudaLaunchKernelEx(&cfg, cg_smem_cluster_kernel<kBlock, true>, m));
-                } else {
-                    CU(cudaLaunchKernelEx(&cfg, cg_smem_cluster_kernel<kBlock, false>, m));
-                }
+                if (m.dia) kern = sr ? pick(cg_smem_cluster_kernel<512, true, true>, cg_smem_cluster_kernel<kBlock, true, true>)
+                                     : pick(cg_smem_cluster_kernel<512, false, true>, cg_smem_cluster_kernel<kBlock, false, true>);
+                else kern = sr ? pick(cg_smem_cluster_kernel<512, true>, cg_smem_cluster_kernel<kBlock, true>)
+                               : pick(cg_smem_cluster_kernel<512, false>, cg_smem_cluster_kernel<kBlock, false>);
             }
+            CU(cudaLaunchKernelEx(&cfg, kern, m));
             p->last_persist_mode = 5;
             return check_launch(ctx);
         }
@@ -1986,7 +1994,15 @@ int ctx_common_init(hpccg_ctx *c, int device, void *stream) {
                               (const void *)cg_smem_cluster_kernel<kBlock, false, true>,
                               (const void *)cg_smem_cluster_kernel<kBlock, true, true>,
                               (const void *)cg_smem_cluster_kernel<512, false, true>,
-                              (const void *)cg_smem_cluster_kernel<512, true, true>})
+                              (const void *)cg_smem_cluster_kernel<512, true, true>,
+                              (const void *)cg_smem_cluster_kernel<kBlock, false, false, true>,
+                              (const void *)cg_smem_cluster_kernel<kBlock, true, false, true>,
+                              (const void *)cg_smem_cluster_kernel<512, false, false, true>,
+                              (const void *)cg_smem_cluster_kernel<512, true, false, true>,
+                              (const void *)cg_smem_cluster_kernel<kBlock, false, true, true>,
+                              (const void *)cg_smem_cluster_kernel<kBlock, true, true, true>,
+                              (const void *)cg_smem_cluster_kernel<512, false, true, true>,
+                              (const void *)cg_smem_cluster_kernel<512, true, true, true>})
             attr_ok = attr_ok &&
                       cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                            (int)c->smem_bytes) == cudaSuccess &&
@@ -2683,6 +2699,10 @@ int hpccg_set_option(hpccg_problem *p, int key, int64_t value) {
             p->graph = p->wgraph = nullptr;
             p->opt_sliced = (int)value;
             return sliced_alloc(p);
+        case HPCCG_OPT_SMEM_HALO:
+            if (value < -1 || value > 1) return fail(HPCCG_EINVAL, "smem halo: -1 (auto), 0 or 1");
+            p->opt_smem_halo = (int)value;
+            return HPCCG_OK;
         case HPCCG_OPT_SPMV_CLUSTER:
             if (value < -1 || value > 1) return fail(HPCCG_EINVAL, "spmv cluster: -1 (auto), 0 or 1");
             if (p->graph) cudaGraphExecDestroy(p->graph);

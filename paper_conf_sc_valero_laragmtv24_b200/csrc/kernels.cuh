@@ -2738,6 +2738,10 @@ struct SmemArgs {
     CgScalars *sc;
     int max_iter;
     double tol;
+    int H;      // > 0: the gathered vector is kept with H halo rows each side in every
+                // CTA's own shared memory (refreshed once per SpMV by coalesced reads of
+                // the owners' rows), so the 27 gathers of a row are local; 0: each
+                // gather reads the owner CTA's shared memory (DSMEM)
 };
 
 // Block sum of two values over NT threads in a fixed order (butterfly per
@@ -2810,7 +2814,8 @@ __device__ __forceinline__ double2 cluster_sum2(double *mine, double u, double v
 //   kSR = false: HPCCG's CG (A4, A11), 3 cluster barriers per iteration;
 //   kSR = true:  the single-reduction CG of f2 (oracle_cg_sr), 2 per iteration.
 // Per-row FMA chain as A8.
-template <int NT, bool kSR, bool kDia = false>
+// kHalo (HPCCG_OPT_SMEM_HALO): a.H > 0 halo rows, gathers from the local copy
+template <int NT, bool kSR, bool kDia = false, bool kHalo = false>
 __global__ void __launch_bounds__(NT, 1) cg_smem_cluster_kernel(SmemArgs a) {
     namespace cgx = cooperative_groups;
     auto cl = cgx::this_cluster();
@@ -2819,9 +2824,13 @@ __global__ void __launch_bounds__(NT, 1) cg_smem_cluster_kernel(SmemArgs a) {
     __shared__ double part_a[2], part_b[2];
     const int R = a.R;
     const unsigned me = cl.block_rank();
+    const int Hh = kHalo ? a.H : 0;             // halo rows of the gathered vector (0: DSMEM gathers)
     double *sval = smem;                        // [27][R]
     double *sb = sval + (size_t)kSlots * R;     // [R] each
-    double *sx = sb + R, *sr = sx + R, *sp = sr + R, *sq = sp + R;  // sq: Ap (HPCCG) / w (SR)
+    // the gathered vector (SR: r, HPCCG: p) gets Hh halo rows on each side
+    double *sx = sb + R, *sr = sx + R + (kSR ? Hh : 0);
+    double *sp = sr + R + (kSR ? Hh : Hh);      // (SR: after r's upper halo; HPCCG: after p's lower halo)
+    double *sq = sp + R + (kSR ? 0 : Hh);       // sq: Ap (HPCCG) / w (SR)
     double *ss = sq + R;                        // SR: s = A p recurrence
     int *scol = reinterpret_cast<int *>(ss + (kSR ? R : 0));  // [27][R]
     const int64_t row0 = (int64_t)me * R;
@@ -2859,14 +2868,35 @@ __global__ void __launch_bounds__(NT, 1) cg_smem_cluster_kernel(SmemArgs a) {
                                        ? own + (k / 9 - 1) * plane32 + ((k / 3) % 3 - 1) * a.nx + (k % 3 - 1)
                                        : own)
                                 : scol[k * R + i] - plane32;
-            const unsigned owner = (unsigned)c / (unsigned)R;
-            const int off = c - (int)owner * R;
-            pv[k] = *cl.map_shared_rank(g + off, owner);
+            if (kHalo) {  // local copy: own rows at g[0, R), halo at g[-Hh, 0) and g[R, R + Hh)
+                pv[k] = g[c - (int)row0];
+            } else {
+                const unsigned owner = (unsigned)c / (unsigned)R;
+                const int off = c - (int)owner * R;
+                pv[k] = *cl.map_shared_rank(g + off, owner);
+            }
         }
         double s = 0.0;
 #pragma unroll
         for (int k = 0; k < kSlots; ++k) s = fma(sval[k * R + i], pv[k], s);
         return s;
+    };
+    // after a cluster barrier that completed every CTA's rows of g: copy the
+    // rows [row0 - Hh, row0) and [row0 + R, row0 + R + Hh) from their owners
+    // (consecutive threads read consecutive rows of one owner), then make them
+    // visible to this CTA.  The owners write those rows again only after the
+    // next cluster barrier.
+    auto fill_halo = [&](double *g) {
+        if (!kHalo) return;
+        for (int j = threadIdx.x; j < 2 * Hh; j += NT) {
+            const int lo = j < Hh;
+            const int64_t gr = lo ? row0 - Hh + j : row0 + R + (j - Hh);
+            if (gr < 0 || gr >= a.n) continue;  // outside the matrix: never a column
+            const unsigned owner = (unsigned)(gr / R);
+            const int off = (int)(gr - (int64_t)owner * R);
+            g[lo ? j - Hh : R + (j - Hh)] = *cl.map_shared_rank(g + off, owner);
+        }
+        __syncthreads();
     };
     int niters = 0;
     double normr, rr_out, rr_prev_out;
@@ -2874,6 +2904,7 @@ __global__ void __launch_bounds__(NT, 1) cg_smem_cluster_kernel(SmemArgs a) {
         // ---- init (a.7): p = x; Ap = A p; r = b - Ap; rtrans = r.r
         for (int i = threadIdx.x; i < nr; i += NT) sp[i] = sx[i];
         cl.sync();
+        fill_halo(sp);
         double acc = 0.0;
         for (int i = threadIdx.x; i < nr; i += NT) {
             const double rv = fma(-1.0, spmv_row(sp, i), sb[i]);
@@ -2894,6 +2925,7 @@ __global__ void __launch_bounds__(NT, 1) cg_smem_cluster_kernel(SmemArgs a) {
             for (int i = threadIdx.x; i < nr; i += NT) sp[i] = (k == 1) ? sr[i] : fma(beta, sp[i], sr[i]);
             normr = sqrt(rtrans);
             cl.sync();
+            fill_halo(sp);
             double d = 0.0;
             for (int i = threadIdx.x; i < nr; i += NT) {
                 const double ap = spmv_row(sp, i);
@@ -2920,10 +2952,12 @@ __global__ void __launch_bounds__(NT, 1) cg_smem_cluster_kernel(SmemArgs a) {
         // ---- init: r = b - A x0 (x0 gathered from sr), w = A r, (gamma, delta)
         for (int i = threadIdx.x; i < nr; i += NT) sr[i] = sx[i];
         cl.sync();
+        fill_halo(sr);
         for (int i = threadIdx.x; i < nr; i += NT) sq[i] = fma(-1.0, spmv_row(sr, i), sb[i]);
         cl.sync();  // every CTA has finished gathering x0 from sr
         for (int i = threadIdx.x; i < nr; i += NT) sr[i] = sq[i];
         cl.sync();
+        fill_halo(sr);
         double g = 0.0, dl = 0.0;
         for (int i = threadIdx.x; i < nr; i += NT) {
             const double w = spmv_row(sr, i);
@@ -2954,6 +2988,7 @@ __global__ void __launch_bounds__(NT, 1) cg_smem_cluster_kernel(SmemArgs a) {
             // the next iteration would not run (A4, A11): skip its SpMV
             if (stop || !(k + 1 < a.max_iter && normr > a.tol)) break;
             cl.sync();
+            fill_halo(sr);
             g = 0.0;
             dl = 0.0;
             for (int i = threadIdx.x; i < nr; i += NT) {

@@ -41,6 +41,7 @@ HPCCG_OPT_SMEM_THREADS, HPCCG_OPT_HALO_PEER, HPCCG_OPT_SERPENTINE = 18, 19, 20
 HPCCG_OPT_SPMV_FORMAT, HPCCG_OPT_PEER_TIMEOUT_MS, HPCCG_OPT_DEFER_X = 21, 22, 23
 HPCCG_OPT_FUSE_PSPMV, HPCCG_OPT_PS_LEAD, HPCCG_OPT_SPMV_TRIPS = 24, 25, 26
 HPCCG_OPT_PAP_CLUSTER, HPCCG_OPT_SPMV_SLICED, HPCCG_OPT_SPMV_CLUSTER = 27, 28, 29
+HPCCG_OPT_SMEM_HALO = 30
 
 _lock = threading.Lock()
 _lib = None

@@ -377,6 +377,44 @@ def test_cg_persistent_grid_and_cluster_variants(ctx, crows, smem, mode):
         assert res["niters"] == 50
 
 
+@pytest.mark.parametrize("dims,max_iter,tol", [((20, 30, 10), 150, 1e-12), ((3, 3, 3), 150, 1e-12),
+                                               ((16, 16, 16), 150, 1e-12), ((33, 9, 3), 150, 1e-12),
+                                               ((20, 20, 20), 150, 1e-12), ((20, 30, 10), 40, 0.0),
+                                               ((7, 5, 6), 2, 0.0), ((1, 1, 1), 150, 1e-12),
+                                               ((40, 3, 50), 150, 1e-12), ((30, 33, 10), 150, 1e-12)])
+@pytest.mark.parametrize("variant", [0, 1])
+def test_smem_halo_bitwise(ctx, dims, max_iter, tol, variant):
+    """HPCCG_OPT_SMEM_HALO: the on-chip solve with the gathered vector (p, or r
+    for the single-reduction CG) copied with the stencil's reach of halo rows
+    into every CTA's own shared memory once per SpMV, the 27 gathers then
+    local -- the same values in the same order as the distributed-shared-
+    memory gathers, so niters, normr and x are bit for bit equal (256- and
+    512-thread CTAs, halos spanning several CTAs at 20x30x10; 30x33x10 is
+    on chip without room for the halo: the DSMEM fallback); and within the
+    oracle tolerance."""
+    with H.Problem(ctx, *dims) as p:
+        p.set_option(H.HPCCG_OPT_PERSISTENT, 2)
+        p.set_option(H.HPCCG_OPT_SMEM_SOLVE, 1)
+        p.set_option(H.HPCCG_OPT_CG_VARIANT, variant)
+        ref = oracle.generate(*dims)
+        oref = (oracle.cg_sr if variant else oracle.cg)(ref, max_iter, tol)
+        for threads in (0, 256):
+            p.set_option(H.HPCCG_OPT_SMEM_THREADS, threads)
+            outs = []
+            for halo in (0, 1):
+                p.set_option(H.HPCCG_OPT_SMEM_HALO, halo)
+                p.set_vec(H.HPCCG_VEC_X, np.zeros(p.n))
+                r = p.solve(max_iter, tol)
+                assert p.stats()["graph_mode"] == 5
+                outs.append((r["niters"], r["normr"], p.get_vec(H.HPCCG_VEC_X)))
+            assert outs[1][:2] == outs[0][:2]
+            np.testing.assert_array_equal(outs[1][2], outs[0][2])
+            assert abs(outs[1][0] - oref["niters"]) <= 1
+            assert np.max(np.abs(outs[1][2] - oref["x"])) <= CG_ATOL
+        for k, v in ((H.HPCCG_OPT_SMEM_HALO, -1), (H.HPCCG_OPT_SMEM_THREADS, 0), (H.HPCCG_OPT_CG_VARIANT, 0)):
+            p.set_option(k, v)
+
+
 def test_cg_persistent_auto_threshold(ctx):
     with H.Problem(ctx, 20, 30, 10) as p:       # 6000 rows fit on chip: persistent
         p.solve(150, 1e-12)
