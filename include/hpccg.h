@@ -152,14 +152,19 @@ extern "C" {
                                buffer, the SpMV gathers from the slot of iteration k) and every
                                m-th p update applies x = fma(alpha_j, p_j, x) for the m
                                directions since the last one, in ascending j; the pending ones
-                               run after the loop (cg_xfix_ring_kernel).  Per m iterations x
+                               run after the loop (cg_xfix_ring_kernel).  On z-slabs (HALO_PEER 2)
+                               the p update pushes p_k's boundary planes into slot k % (m + 1) of
+                               the neighbours' rings: a ring is exchanged only if it exists when the
+                               peer tables are built (auto: allocated at generate; explicit m on
+                               one-slab-per-process contexts: set it before HALO_PEER / the peer
+                               export), else z-slabs run m = 1.  Per m iterations x
                                is read and written once and m - 1 old p's re-read: 12 nnz +
                                (72 + 8/m) n B per iteration, the writes drop from 2 to 1 + 1/m
                                per row.  Bitwise the same results.  Device memory: m extra
-                               p-sized buffers (allocated when the option is set, or at
-                               generate time for auto).  -1 (default): auto -- 8 on a single
-                               slab whose CG vectors exceed L2, 1 on z-slabs there, 0 below
-                               (at 128^3 the vectors are L2-resident and 0 is 0.4 % faster) */
+                               p-sized buffers per slab (allocated when the option is set, or at
+                               generate time for auto).  -1 (default): auto -- 8 when the CG
+                               vectors exceed L2, 0 below (at 128^3 the vectors are L2-resident
+                               and 0 is 0.4 % faster) */
 #define HPCCG_OPT_FUSE_PSPMV 24 /* single slab, finisher-free loop: the p update and the
                                SpMV of an iteration as ONE pipelined kernel (cg_pspmv_kernel:
                                chunks of 512 rows taken in launch order; each block updates p

@@ -187,6 +187,7 @@ struct hpccg_problem {
     int opt_spmv_cl = 0;               // CG SpMV in 8-CTA clusters, one p.Ap partial per cluster (-1 auto, 0, 1)
     int opt_ps_lead = 0;               // its production lead in chunks (0: plane / 512 + 8)
     std::vector<void *> ipc_opened;    // peers' buffers mapped with cudaIpcOpenMemHandle
+    bool peer_ring = false;            // the peer tables address the neighbours' p rings
     int last_persist_mode = 3;
     // graph of one CG iteration (per-iteration replay) ...
     cudaGraphExec_t graph = nullptr;
@@ -534,6 +535,9 @@ int launch_spmv(hpccg_ctx *ctx, int minb, bool check, SpmvArgs a, int64_t r0, in
         if (a.dia) {
             if (check) launch_k(pdl, spmv27x2_kernel<kDots, true, false, true>, dim3((unsigned)blocks), st, a);
             else launch_k(pdl, spmv27x2_kernel<kDots, false, false, true>, dim3((unsigned)blocks), st, a);
+        } else if (kDots == 1 && a.ring_n > 1) {  // p in a ring slot (ring-deferred x update)
+            if (check) launch_k(pdl, spmv27x2_kernel<kDots, true, false, false, true>, dim3((unsigned)blocks), st, a);
+            else launch_k(pdl, spmv27x2_kernel<kDots, false, false, false, true>, dim3((unsigned)blocks), st, a);
         } else if (check) {
             launch_k(pdl, spmv27x2_kernel<kDots, true>, dim3((unsigned)blocks), st, a);
         } else {
@@ -829,8 +833,13 @@ int cg_spmv_all(hpccg_problem *p, bool timing, bool check) {
             }
             cfg.attrs = at;
             cfg.numAttrs = na;
-            if (check) CU(cudaLaunchKernelEx(&cfg, spmv27x2_cl_kernel<true>, a));
-            else CU(cudaLaunchKernelEx(&cfg, spmv27x2_cl_kernel<false>, a));
+            if (a.ring_n > 1) {
+                if (check) CU(cudaLaunchKernelEx(&cfg, spmv27x2_cl_kernel<true, true>, a));
+                else CU(cudaLaunchKernelEx(&cfg, spmv27x2_cl_kernel<false, true>, a));
+            } else {
+                if (check) CU(cudaLaunchKernelEx(&cfg, spmv27x2_cl_kernel<true, false>, a));
+                else CU(cudaLaunchKernelEx(&cfg, spmv27x2_cl_kernel<false, false>, a));
+            }
             return check_launch(ctx);
         }
         const int trips = spmv_trips(p);
@@ -924,8 +933,11 @@ bool fused_on(const hpccg_problem *p) {
 // Blocks of a grid-stride vector grid (g blocks, 16-B unit i handled by
 // thread i mod (g * kBlock)) that hold a unit of rows [0, plane) or
 // [n - plane, n): the blocks that push a boundary plane.
-unsigned push_blocks(int64_t n, int64_t plane, int g, bool has_lo, bool has_hi) {
-    const int64_t nth = (int64_t)g * kBlock, nv = n >> 1;
+// unit = 2: thread t holds the double2 units u == t (mod nth) (and thread 0
+// the odd last row); unit = 1: the rows i == t (mod nth) (the ring-deferred p
+// update's flush pass)
+unsigned push_blocks(int64_t n, int64_t plane, int g, bool has_lo, bool has_hi, int unit = 2) {
+    const int64_t nth = (int64_t)g * kBlock, nv = unit == 2 ? n >> 1 : n;
     std::vector<char> mark((size_t)g, 0);
     auto units = [&](int64_t u0, int64_t u1) {  // units [u0, u1)
         if (u1 <= u0) return;
@@ -940,9 +952,9 @@ unsigned push_blocks(int64_t n, int64_t plane, int g, bool has_lo, bool has_hi) 
             t = 0;
         }
     };
-    if (has_lo) units(0, std::min<int64_t>(cdiv(plane, 2), nv));  // units holding a row < plane
-    if (has_hi) units(std::max<int64_t>((n - plane) / 2, 0), nv); // ... a row >= n - plane
-    if ((n & 1) && (has_hi || (has_lo && n - 1 < plane))) mark[0] = 1;  // thread 0 does row n - 1
+    if (has_lo) units(0, std::min<int64_t>(cdiv(plane, unit), nv));  // units holding a row < plane
+    if (has_hi) units(std::max<int64_t>((n - plane) / unit, 0), nv); // ... a row >= n - plane
+    if (unit == 2 && (n & 1) && (has_hi || (has_lo && n - 1 < plane))) mark[0] = 1;  // thread 0: row n - 1
     return (unsigned)std::count(mark.begin(), mark.end(), 1);
 }
 
@@ -969,10 +981,22 @@ int launch_spmv_fused(hpccg_problem *p, const Slab &s, bool check, unsigned *npa
     *nparts = (unsigned)blocks;
     const bool pdl = p->opt_pdl != 0;
     a.sr_q = sr_q;
+    if (kDots == 1) {
+        if (const int m = defer_m(p); m >= 2) {  // p_k in ring slot k % (m + 1)
+            a.ring = s.pring;
+            a.ring_stride = s.pring_stride;
+            a.ring_n = m + 1;
+        }
+    }
     if (kDots == 2) a.trace = nullptr;
     if (a.dia) {
         if (check) launch_k(pdl, spmv27x2_kernel<kDots, true, true, true>, dim3((unsigned)blocks), p->ctx->stream, a);
         else launch_k(pdl, spmv27x2_kernel<kDots, false, true, true>, dim3((unsigned)blocks), p->ctx->stream, a);
+    } else if (kDots == 1 && a.ring_n > 1) {  // p in a ring slot (ring-deferred x update)
+        if (check)
+            launch_k(pdl, spmv27x2_kernel<kDots, true, true, false, true>, dim3((unsigned)blocks), p->ctx->stream, a);
+        else
+            launch_k(pdl, spmv27x2_kernel<kDots, false, true, false, true>, dim3((unsigned)blocks), p->ctx->stream, a);
     } else if (check) {
         launch_k(pdl, spmv27x2_kernel<kDots, true, true>, dim3((unsigned)blocks), p->ctx->stream, a);
     } else {
@@ -1011,27 +1035,29 @@ constexpr int kRingAutoM = kRingMaxM;
 int defer_m(const hpccg_problem *p) {
     if (!defer_x_on(p)) return 0;
     const int want = p->opt_defer_x < 0 ? kRingAutoM : p->opt_defer_x;
-    if (want < 2 || p->ctx->mode != MODE_SINGLE) return 1;
-    const Slab &s = p->slabs[0];
-    if (s.pring_slots < want || s.dia || fuse_ps_on(const_cast<hpccg_problem *>(p)) || sliced_on(p) ||
-        spmv_trips(p) > 1)
-        return 1;
+    if (want < 2) return 1;
+    for (const Slab &s : p->slabs)
+        if (s.pring_slots < want || s.dia) return 1;
+    if (p->ctx->mode != MODE_SINGLE)  // z-slabs: the peer tables must address the neighbours' rings
+        return p->peer_ring ? want : 1;
+    if (fuse_ps_on(const_cast<hpccg_problem *>(p)) || sliced_on(p) || spmv_trips(p) > 1) return 1;
     return want;
 }
 
 // ring slots for depth m (never during a graph capture: generate / set_option)
 int ring_alloc(hpccg_problem *p, int m) {
-    if (p->ctx->mode != MODE_SINGLE || m < 2) return HPCCG_OK;
-    Slab &s = p->slabs[0];
-    if (s.pring_slots >= m) return HPCCG_OK;
-    cudaFree(s.pring_alloc);
-    s.pring_alloc = s.pring = nullptr;
-    s.pring_slots = 0;
-    const int64_t seg = cdiv(s.ncol + 2, 32) * 32;  // as the arena's p segment
-    CHECK(alloc_zero((void **)&s.pring_alloc, sizeof(double) * (size_t)(seg * m)));
-    s.pring = s.pring_alloc + (s.p - s.p_alloc);  // the same 16-B alignment shift as p
-    s.pring_stride = seg;
-    s.pring_slots = m;
+    if (m < 2) return HPCCG_OK;
+    for (Slab &s : p->slabs) {
+        if (s.pring_slots >= m) continue;
+        cudaFree(s.pring_alloc);
+        s.pring_alloc = s.pring = nullptr;
+        s.pring_slots = 0;
+        const int64_t seg = cdiv(s.ncol + 2, 32) * 32;  // as the arena's p segment
+        CHECK(alloc_zero((void **)&s.pring_alloc, sizeof(double) * (size_t)(seg * m)));
+        s.pring = s.pring_alloc + (s.p - s.p_alloc);  // the same 16-B alignment shift as p
+        s.pring_stride = seg;
+        s.pring_slots = m;
+    }
     return HPCCG_OK;
 }
 
@@ -1050,10 +1076,12 @@ int enqueue_xfix(hpccg_problem *p) {
     if (!defer_x_on(p)) return HPCCG_OK;
     hpccg_ctx *ctx = p->ctx;
     if (const int m = defer_m(p); m >= 2) {
-        const Slab &s = p->slabs[0];
-        launch_k(false, cg_xfix_ring_kernel, dim3(wave_grid(s.n / 2 + 1, wave(ctx, cg_xfix_ring_kernel))),
-                 ctx->stream, (int64_t)s.n, s.x, s.p + s.plane, ring_of(s, m, true), (const CgScalars *)s.sc);
-        return check_launch(ctx);
+        for (const Slab &s : p->slabs) {
+            launch_k(false, cg_xfix_ring_kernel, dim3(wave_grid(s.n / 2 + 1, wave(ctx, cg_xfix_ring_kernel))),
+                     ctx->stream, (int64_t)s.n, s.x, s.p + s.plane, ring_of(s, m, true), (const CgScalars *)s.sc);
+            CHECK(check_launch(ctx));
+        }
+        return HPCCG_OK;
     }
     for (const Slab &s : p->slabs) {
         launch_k(false, cg_xfix_kernel, dim3(wave_grid(s.n / 2 + 1, wave(ctx, cg_xfix_kernel))),
@@ -1177,25 +1205,37 @@ int enqueue_iteration_ff_u(hpccg_problem *p, bool timing, bool check, unsigned l
         }
         PhaseTimer t(p, ctx->stream, PH_SPMV, timing);
         CHECK(launch_pspmv(p, s0, q));
-    } else if (const int m = zs ? 0 : defer_m(p); m >= 2) {  // ring-deferred x update
+    } else if (const int m = defer_m(p); m >= 2) {  // ring-deferred x update
         PhaseTimer t(p, ctx->stream, PH_PUPDATE, timing);
-        PringArgs a{};
-        a.n = s0.n;
-        a.r = s0.r;
-        a.p = s0.p + s0.plane;
-        a.ring = ring_of(s0, m, true);
-        a.x = s0.x;
-        a.rr_parts = s0.red.partials;
-        a.n_rr = (unsigned)ug;
-        a.sc = s0.sc;
-        a.q = q;
-        a.trace = s0.trace_on ? s0.trace : nullptr;
-        a.trace_max = s0.trace_max;
-        a.rev = serpentine(p) & 1;
-        auto rk = cg_pupdate_ring_kernel<kU>;
+        if (pre)
+            for (const Slab &s : p->slabs) CHECK(post(s, s.red.partials, (unsigned)ug, 0));
+        auto rk = zs ? cg_pupdate_ring_kernel<kU, true> : cg_pupdate_ring_kernel<kU, false>;
         const int rg = vec_grid(ctx, rk, cdiv(s0.n, 2 * kU), p->opt_vec_waves, 0x7fffffff);
-        launch_k(pdl, rk, dim3(rg), ctx->stream, a);
-        CHECK(check_launch(ctx));
+        for (const Slab &s : p->slabs) {
+            PringArgs a{};
+            a.n = s.n;
+            a.r = s.r;
+            a.p = s.p + s.plane;
+            a.ring = ring_of(s, m, true);
+            a.x = s.x;
+            a.rr_parts = s.red.partials;
+            a.n_rr = (unsigned)ug;
+            a.sc = s.sc;
+            a.q = q;
+            a.trace = s.trace_on ? s.trace : nullptr;
+            a.trace_max = s.trace_max;
+            a.rev = serpentine(p) & 1;
+            a.post = !pre;
+            if (zs) {
+                const bool lo = s.rank > 0, hi = s.rank < ctx->nranks - 1;
+                a.t = s.ptab;
+                a.plane = s.plane;
+                a.n_push = push_blocks(s.n, s.plane, rg, lo, hi, 2);
+                a.n_push1 = push_blocks(s.n, s.plane, rg, lo, hi, 1);
+            }
+            launch_k(pdl, rk, dim3(rg), ctx->stream, a);
+            CHECK(check_launch(ctx));
+        }
     } else {
         PhaseTimer t(p, ctx->stream, PH_PUPDATE, timing);
         if (pre)
@@ -2164,16 +2204,25 @@ int peer_export(hpccg_problem *p, unsigned char *blob) {
     CU(cudaIpcGetMemHandle(&h[0], s0.arena));
     CU(cudaIpcGetMemHandle(&h[1], s0.psync));
     memcpy(blob, h, sizeof h);
+    if (s0.pring_alloc) {  // the p ring of the deferred x update (slot count in the last 4 bytes)
+        cudaIpcMemHandle_t hr;
+        CU(cudaIpcGetMemHandle(&hr, s0.pring_alloc));
+        memcpy(blob + 2 * sizeof(cudaIpcMemHandle_t), &hr, sizeof hr);
+        const int slots = s0.pring_slots;
+        memcpy(blob + HPCCG_PEER_BLOB_BYTES - sizeof(int), &slots, sizeof slots);
+    }
     return HPCCG_OK;
 }
 
 // sync[q] / pvec[q]: rank q's PeerSync and local-with-halo vector base (may
 // be null for non-neighbours' vectors) -> device tables of the hosted slabs
+// rvec[q]: rank q's p ring (halo base of slot 1; null: none / not a neighbour)
 int peer_build_tables(hpccg_problem *p, const std::vector<PeerSync *> &sync,
-                      const std::vector<double *> &pvec) {
+                      const std::vector<double *> &pvec, const std::vector<double *> &rvec) {
     hpccg_ctx *ctx = p->ctx;
     const int P = ctx->nranks;
     const int64_t n = p->slabs[0].n, plane = p->slabs[0].plane;
+    bool ring = true;
     for (size_t i = 0; i < p->slabs.size(); ++i) {
         Slab &sl = p->slabs[i];
         const int r = ctx->mode == MODE_LOOPBACK ? (int)i : ctx->rank;
@@ -2185,10 +2234,14 @@ int peer_build_tables(hpccg_problem *p, const std::vector<PeerSync *> &sync,
         t.hi = r < P - 1 ? sync[r + 1] : nullptr;
         t.halo_to_lo = r > 0 ? pvec[r - 1] + plane + n : nullptr;
         t.halo_to_hi = r < P - 1 ? pvec[r + 1] : nullptr;
+        t.ring_to_lo = r > 0 && rvec[r - 1] ? rvec[r - 1] + plane + n : nullptr;
+        t.ring_to_hi = r < P - 1 ? rvec[r + 1] : nullptr;
+        ring = ring && sl.pring && (r == 0 || t.ring_to_lo) && (r == P - 1 || t.ring_to_hi);
         for (int q = 0; q < P; ++q) t.all[q] = sync[q];
         if (!sl.ptab) CHECK(alloc_zero((void **)&sl.ptab, sizeof(PeerTab)));
         CU(cudaMemcpy(sl.ptab, &t, sizeof t, cudaMemcpyHostToDevice));
     }
+    p->peer_ring = ring;
     return HPCCG_OK;
 }
 
@@ -2199,11 +2252,12 @@ int peer_attach(hpccg_problem *p, const unsigned char *blobs) {
     const int P = ctx->nranks, r = ctx->rank;
     const Slab &s0 = p->slabs[0];
     std::vector<PeerSync *> sync(P, nullptr);
-    std::vector<double *> pvec(P, nullptr);
+    std::vector<double *> pvec(P, nullptr), rvec(P, nullptr);
     for (int q = 0; q < P; ++q) {
         if (q == r) {
             sync[q] = s0.psync;
             pvec[q] = s0.p;
+            rvec[q] = s0.pring;
             continue;
         }
         cudaIpcMemHandle_t hq[2];
@@ -2217,9 +2271,20 @@ int peer_attach(hpccg_problem *p, const unsigned char *blobs) {
             CU(cudaIpcOpenMemHandle(&pa, hq[0], cudaIpcMemLazyEnablePeerAccess));
             p->ipc_opened.push_back(pa);
             pvec[q] = (double *)pa + (s0.p - s0.arena);
+            cudaIpcMemHandle_t hr, zero{};
+            int slots = 0;
+            memcpy(&hr, blobs + (size_t)HPCCG_PEER_BLOB_BYTES * q + 2 * sizeof(cudaIpcMemHandle_t), sizeof hr);
+            memcpy(&slots, blobs + (size_t)HPCCG_PEER_BLOB_BYTES * (q + 1) - sizeof(int), sizeof slots);
+            // the neighbour's ring, when both have one of the same depth (identical layouts)
+            if (s0.pring && slots == s0.pring_slots && memcmp(&hr, &zero, sizeof hr) != 0) {
+                void *pr = nullptr;
+                CU(cudaIpcOpenMemHandle(&pr, hr, cudaIpcMemLazyEnablePeerAccess));
+                p->ipc_opened.push_back(pr);
+                rvec[q] = (double *)pr + (s0.pring - s0.pring_alloc);
+            }
         }
     }
-    return peer_build_tables(p, sync, pvec);
+    return peer_build_tables(p, sync, pvec, rvec);
 }
 
 // HPCCG_OPT_HALO_PEER = 1 (collective): loopback and NCCL contexts build the
@@ -2230,12 +2295,13 @@ int enable_peer(hpccg_problem *p) {
     const int P = ctx->nranks;
     if (ctx->mode == MODE_LOOPBACK) {
         std::vector<PeerSync *> sync(P);
-        std::vector<double *> pvec(P);
+        std::vector<double *> pvec(P), rvec(P);
         for (int q = 0; q < P; ++q) {
             sync[q] = p->slabs[q].psync;
             pvec[q] = p->slabs[q].p;
+            rvec[q] = p->slabs[q].pring;
         }
-        return peer_build_tables(p, sync, pvec);
+        return peer_build_tables(p, sync, pvec, rvec);
     }
     if (ctx->mode == MODE_NCCL) {
 #ifdef HPCCG_WITH_NCCL
@@ -2564,8 +2630,12 @@ int hpccg_generate(hpccg_ctx *ctx, int nx, int ny, int nz, hpccg_problem **out) 
     if (ctx->mode == MODE_SINGLE) {  // the CG SpMV's chunk-sliced copy (auto: large problems)
         int rc = sliced_alloc(p);
         if (rc) return bail(rc);
-        // the ring of the deferred x update (auto: CG vectors beyond L2)
-        if (p->slabs[0].arena_bytes > ((size_t)126 << 20) && (rc = ring_alloc(p, kRingAutoM))) return bail(rc);
+    }
+    // the p rings of the deferred x update (auto: CG vectors beyond L2), before any
+    // peer exchange so the neighbours can address them
+    if (p->slabs[0].arena_bytes > ((size_t)126 << 20)) {
+        const int rc = ring_alloc(p, kRingAutoM);
+        if (rc) return bail(rc);
     }
     *out = p;
     return HPCCG_OK;
@@ -2752,6 +2822,9 @@ int hpccg_set_option(hpccg_problem *p, int key, int64_t value) {
             CHECK(ring_alloc(p, value < 0 ? (p->slabs[0].arena_bytes > ((size_t)126 << 20) ? kRingAutoM : 0)
                                           : (int)value));
             p->opt_defer_x = (int)value;
+            // loopback slabs: re-address the (new) rings in the peer tables; one slab per
+            // process exchanges them only at HALO_PEER setup (a collective)
+            if (p->ctx->mode == MODE_LOOPBACK && p->slabs[0].ptab) CHECK(enable_peer(p));
             return HPCCG_OK;
         case HPCCG_OPT_PEER_TIMEOUT_MS:
             if (value < 1 || value > 3600000) return fail(HPCCG_EINVAL, "peer timeout: 1 .. 3600000 ms");

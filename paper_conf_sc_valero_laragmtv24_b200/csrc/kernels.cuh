@@ -303,6 +303,9 @@ struct PeerTab {                       // device copy per slab; pointers may be 
     int rank, nranks;
     double *halo_to_lo;                // rank-1's upper halo plane (gets my first owned plane)
     double *halo_to_hi;                // rank+1's lower halo plane (gets my last owned plane)
+    // ring-deferred x update (HPCCG_OPT_DEFER_X >= 2): the same planes in slot 1
+    // of the neighbours' p rings (slot j >= 1: + (j - 1) ring_stride); null: no ring
+    double *ring_to_lo, *ring_to_hi;
     PeerSync *mine, *lo, *hi;
     PeerSync *all[kMaxPeers];          // every rank's PeerSync (allreduce posts)
 };
@@ -553,9 +556,13 @@ __device__ __forceinline__ int spmv_done(const SpmvArgs &a) {
     return ldg_o(&a.sc->done);
 }
 
-// the gathered vector of this SpMV (after pdl_wait: sc->k is the predecessor's)
+// the gathered vector of this SpMV (after pdl_wait: sc->k is the predecessor's).
+// kRing = false: a.x, no load -- the 2-rows/thread kernels instantiate the ring
+// separately (the extra live pointer made the fused z-slab kCheck variant spill
+// at 64 registers: 812.8 -> 853.0 us at 256^3)
+template <bool kRing = true>
 __device__ __forceinline__ const double *spmv_xg(const SpmvArgs &a) {
-    if (a.ring_n <= 1) return a.x;
+    if (!kRing || a.ring_n <= 1) return a.x;
     const int j = ldg_o(&a.sc->k) % a.ring_n;
     return j == 0 ? a.x : a.ring + (int64_t)(j - 1) * a.ring_stride;
 }
@@ -757,7 +764,7 @@ __device__ __forceinline__ int2 spmv_cols(const SpmvArgs &a, const int *c, int s
 // 1024-thread finisher kernel between the SpMV and the update
 constexpr int kSpmvCl = 8;
 
-template <int kDots, bool kCheck, bool kFused, bool kCoh, bool kDia = false, bool kCl = false>
+template <int kDots, bool kCheck, bool kFused, bool kCoh, bool kDia = false, bool kCl = false, bool kRing = false>
 __device__ __forceinline__ void spmv27x2_body(const SpmvArgs &a, int64_t row, int64_t lim, int64_t bid) {
     constexpr bool kDot = kDots == 1;
     double d = 0.0, dg = 0.0;  // kDots 1: p.Ap; kDots 2: delta (d) and gamma (dg)
@@ -768,7 +775,10 @@ __device__ __forceinline__ void spmv27x2_body(const SpmvArgs &a, int64_t row, in
         const int *c = a.col + row;
         double s0 = 0.0, s1 = 0.0, x0 = 0.0, x1 = 0.0;
         int c0 = 0, c1 = 0;
-        const double *xg = a.x;
+        // kRing: the slot of sc->k (set after the wait); else the parameter itself
+        // (no copy held in a register)
+        const double *xgr = nullptr;
+#define XG (kRing ? xgr : a.x)
         // slots whose loads are issued together: 3 (ELL: 72 B per thread in
         // flight); DIA has no index stream, so it takes kDiaGroup slots
         constexpr int kG = kDia ? kDiaGroup : 3;
@@ -787,12 +797,12 @@ __device__ __forceinline__ void spmv27x2_body(const SpmvArgs &a, int64_t row, in
                 if (kDot && a.trace) trace_mark(a.trace, a.trace_max, ldg_o(&a.sc->k), 1, false);
                 done = spmv_done<kDots, kCheck>(a);
                 if (done) return;  // uniform over the grid, before any store
-                xg = spmv_xg(a);
+                if (kRing) xgr = spmv_xg<true>(a);
             }
 #pragma unroll
             for (int t = 0; t < kG; ++t) {
                 if (kDia) cc[t] = spmv_cols<true>(a, c, kG * g + t, vv[t], row, pol);
-                const double xa = ld_gather<kCoh>(xg + cc[t].x), xb = ld_gather<kCoh>(xg + cc[t].y);
+                const double xa = ld_gather<kCoh>(XG + cc[t].x), xb = ld_gather<kCoh>(XG + cc[t].y);
                 if (kG * g + t == kDiagSlot) {
                     x0 = xa;
                     x1 = xb;
@@ -805,8 +815,9 @@ __device__ __forceinline__ void spmv27x2_body(const SpmvArgs &a, int64_t row, in
         }
         *reinterpret_cast<double2 *>(a.y + row) = make_double2(s0, s1);
         if (kDots > 0) {
-            const double p0 = c0 == row + a.plane ? x0 : ld_gather<kCoh>(xg + row + a.plane);
-            const double p1 = c1 == row + 1 + a.plane ? x1 : ld_gather<kCoh>(xg + row + 1 + a.plane);
+            const double p0 = c0 == row + a.plane ? x0 : ld_gather<kCoh>(XG + row + a.plane);
+            const double p1 = c1 == row + 1 + a.plane ? x1 : ld_gather<kCoh>(XG + row + 1 + a.plane);
+#undef XG
             d = fma(s1, p1, s0 * p0);
             if (kDots == 2) dg = fma(p1, p1, p0 * p0);
         }
@@ -815,7 +826,7 @@ __device__ __forceinline__ void spmv27x2_body(const SpmvArgs &a, int64_t row, in
         pdl_wait();
         done = spmv_done<kDots, kCheck>(a);
         if (done) return;
-        const double *xg = spmv_xg(a);
+        const double *xg = spmv_xg<kRing>(a);
         double s0 = 0.0;
 #pragma unroll
         for (int k = 0; k < kSlots; ++k)
@@ -1079,8 +1090,10 @@ __global__ void __launch_bounds__(kSlR, 2) spmv_sliced_kernel(SpmvArgs a, const 
     }
 }
 
-template <int kDots, bool kCheck, bool kFused = false, bool kDia = false>
-__global__ void __launch_bounds__(kBlock, kDia ? kDiaMinB : 4) spmv27x2_kernel(SpmvArgs a) {
+// (the fused z-slab kernel with the ring slot pointer: 3 blocks per SM -- at
+// 64 registers its kCheck variant spills, 849 vs 813 us at 256^3)
+template <int kDots, bool kCheck, bool kFused = false, bool kDia = false, bool kRing = false>
+__global__ void __launch_bounds__(kBlock, kDia ? kDiaMinB : (kFused && kRing ? 3 : 4)) spmv27x2_kernel(SpmvArgs a) {
     int64_t row, lim;
     const int64_t bid = spmv_bid(a);
     bool bnd = false;
@@ -1111,19 +1124,19 @@ __global__ void __launch_bounds__(kBlock, kDia ? kDiaMinB : 4) spmv27x2_kernel(S
         }
     }
     if (kFused && bnd) {
-        spmv27x2_body<kDots, kCheck, kFused, true, kDia>(a, row, lim, bid);
+        spmv27x2_body<kDots, kCheck, kFused, true, kDia, false, kRing>(a, row, lim, bid);
         return;
     }
-    spmv27x2_body<kDots, kCheck, kFused, false, kDia>(a, row, lim, bid);
+    spmv27x2_body<kDots, kCheck, kFused, false, kDia, false, kRing>(a, row, lim, bid);
 }
 
 // the single-slab CG SpMV in clusters of kSpmvCl CTAs (grid a multiple of
 // kSpmvCl; the padding blocks have no rows and contribute 0)
-template <bool kCheck>
+template <bool kCheck, bool kRing>
 __global__ void __launch_bounds__(kBlock, 4) spmv27x2_cl_kernel(SpmvArgs a) {
     const int64_t bid = spmv_bid(a);
     const int64_t row = a.r0 + (bid * kBlock + threadIdx.x) * 2, lim = a.r0 + a.len0;
-    spmv27x2_body<1, kCheck, false, false, false, true>(a, row, lim, bid);
+    spmv27x2_body<1, kCheck, false, false, false, true, kRing>(a, row, lim, bid);
 }
 
 // ------------------------------------------------ streaming vector kernels
@@ -1723,15 +1736,35 @@ struct PringArgs {
     TraceSlot *trace;
     int trace_max;
     int rev;
+    // HALO_PEER = 2 on z-slabs (kPeer): as Pupd1Args, the boundary planes of
+    // p_K pushed into slot K % (m + 1) of the neighbours' rings; n_push / n_push1:
+    // blocks holding a boundary row in the double2 / the flush (one element
+    // per thread) mapping
+    const PeerTab *t;
+    int64_t plane;
+    unsigned n_push, n_push1;
+    int post;
 };
+
+// the neighbour halo plane of ring slot j (slot 0: the problem's p buffer)
+__device__ __forceinline__ double *ring_peer_plane(double *slot0, double *slot1, int64_t stride, int j) {
+    if (!slot0) return nullptr;
+    return j == 0 ? slot0 : slot1 + (int64_t)(j - 1) * stride;
+}
 
 // the scalar part of p update K (after the PDL wait): beta, and block 0's
 // loop state; false: iteration K does not run (uniform exit)
+template <bool kPeer>
 __device__ __forceinline__ bool ring_scalars(const PringArgs &a, int K, bool first, double *sh, double *beta) {
     CgScalars *sc = a.sc;
     if (!run_check(sc, a.q)) return false;
     trace_mark(a.trace, a.trace_max, K, 0, false);
-    const double rtrans = first ? ldg_o(&sc->rr_cur) : sum_parts_fixed(a.rr_parts, a.n_rr, sh);
+    double rtrans = first ? ldg_o(&sc->rr_cur) : sum_parts_fixed(a.rr_parts, a.n_rr, sh);
+    if (kPeer && !first) {  // z-slabs: the slab's r.r -> every rank; the global sum back
+        const unsigned tag = ll_tag(ldg_o(&sc->epoch), 2ull * (unsigned)(K - 1));
+        if (a.post && blockIdx.x == 0 && threadIdx.x == 0) fused_post(a.t, 0, rtrans, tag);
+        rtrans = fused_collect_block(a.t, 0, tag, rtrans, &sh[32]);
+    }
     *beta = first ? 0.0 : rtrans / ldg_o(&sc->rr_prev);
     if (blockIdx.x == 0 && threadIdx.x == 0) {
         if (!first) sc->rr_cur = rtrans;
@@ -1746,6 +1779,7 @@ __device__ __forceinline__ bool ring_scalars(const PringArgs &a, int K, bool fir
 // (scalar: the m + 2 loads in flight per thread fit the normal path's
 // register budget); x, p_(K-1) and the m - 1 older directions are loaded
 // before the wait
+template <bool kPeer>
 __device__ __forceinline__ void ring_flush(const PringArgs &a, int K, double *sh) {
     const int m = a.ring.m, R = m + 1;
     const int64_t tid = gtid(), nth = gnth(), n = a.n;
@@ -1774,7 +1808,13 @@ __device__ __forceinline__ void ring_flush(const PringArgs &a, int K, double *sh
     pdl_trigger();
     if (b0 < n) ra = r[b0];
     double beta;
-    if (!ring_scalars(a, K, false, sh, &beta)) return;
+    if (!ring_scalars<kPeer>(a, K, false, sh, &beta)) return;
+    double *plo = nullptr, *phi = nullptr;
+    if (kPeer) {
+        plo = ring_peer_plane(a.t->halo_to_lo, a.t->ring_to_lo, a.ring.stride, K % R);
+        phi = ring_peer_plane(a.t->halo_to_hi, a.t->ring_to_hi, a.ring.stride, K % R);
+    }
+    int pushed = 0;
     __shared__ double sal[kRingMaxM];
     if (threadIdx.x < kRingMaxM)
         sal[threadIdx.x] = (int)threadIdx.x < m ? ldg_o(&a.sc->alpha_h[(K - m + (int)threadIdx.x) & 15]) : 0.0;
@@ -1786,7 +1826,18 @@ __device__ __forceinline__ void ring_flush(const PringArgs &a, int K, double *sh
         for (int t = 0; t < kRingMaxM - 1; ++t)
             if (t < m - 1) xa = fma(sal[t], oa[t], xa);
         x[b] = fma(am, pa, xa);
-        dst[b] = fma(beta, pa, ra);
+        const double v = fma(beta, pa, ra);
+        dst[b] = v;
+        if (kPeer) {
+            if (plo && b < a.plane) {
+                plo[b] = v;
+                pushed = 1;
+            }
+            if (phi && b >= n - a.plane) {
+                phi[b - (n - a.plane)] = v;
+                pushed = 1;
+            }
+        }
         b += a.rev ? -step : step;
         if (b >= 0 && b < n) {
             ra = r[b];
@@ -1797,11 +1848,12 @@ __device__ __forceinline__ void ring_flush(const PringArgs &a, int K, double *sh
         __syncthreads();
         trace_mark(a.trace, a.trace_max, K, 0, true);
     }
+    if (kPeer) fused_push_signal(a.t, pushed, a.n_push1, ftag(ldg_o(&a.sc->epoch), (unsigned long long)K));
 }
 
 // (__launch_bounds__(kBlock, 3): the flush path's loads must not push the
 // kernel past the 80 registers of cg_pupdate1_kernel<4>)
-template <int kU>
+template <int kU, bool kPeer = false>
 __global__ void __launch_bounds__(kBlock, 3) cg_pupdate_ring_kernel(PringArgs a) {
     __shared__ double sh[33];
     // this iteration's index from the p update before it (ring_k[q ^ 1],
@@ -1811,7 +1863,7 @@ __global__ void __launch_bounds__(kBlock, 3) cg_pupdate_ring_kernel(PringArgs a)
     const int m = a.ring.m, R = m + 1;
     const bool first = (K == 1);
     if (!first && (K - 1) % m == 0) {
-        ring_flush(a, K, sh);
+        ring_flush<kPeer>(a, K, sh);
         return;
     }
     const int64_t tid = gtid(), nth = gnth(), nv = a.n >> 1;
@@ -1843,7 +1895,24 @@ __global__ void __launch_bounds__(kBlock, 3) cg_pupdate_ring_kernel(PringArgs a)
     pdl_trigger();
     load_r(b0);
     double beta;
-    if (!ring_scalars(a, K, first, sh, &beta)) return;
+    if (!ring_scalars<kPeer>(a, K, first, sh, &beta)) return;
+    const int64_t n = a.n;
+    double *plo = nullptr, *phi = nullptr;
+    if (kPeer) {
+        plo = ring_peer_plane(a.t->halo_to_lo, a.t->ring_to_lo, a.ring.stride, K % R);
+        phi = ring_peer_plane(a.t->halo_to_hi, a.t->ring_to_hi, a.ring.stride, K % R);
+    }
+    int pushed = 0;
+    auto put = [&](int64_t i, double v) {  // row i of p_K -> a neighbour's halo (slot K % R)
+        if (plo && i < a.plane) {
+            plo[i] = v;
+            pushed = 1;
+        }
+        if (phi && i >= n - a.plane) {
+            phi[i - (n - a.plane)] = v;
+            pushed = 1;
+        }
+    };
     for (int64_t b = b0; b >= 0 && b < nv;) {
 #pragma unroll
         for (int u = 0; u < kU; ++u) {
@@ -1855,6 +1924,10 @@ __global__ void __launch_bounds__(kBlock, 3) cg_pupdate_ring_kernel(PringArgs a)
                     v.y = fma(beta, pa[u].y, ra[u].y);
                 }
                 dst[i] = v;
+                if (kPeer && (2 * i < a.plane || 2 * i + 1 >= n - a.plane)) {
+                    put(2 * i, v.x);
+                    put(2 * i + 1, v.y);
+                }
             }
         }
         b += a.rev ? -step : step;
@@ -1865,12 +1938,15 @@ __global__ void __launch_bounds__(kBlock, 3) cg_pupdate_ring_kernel(PringArgs a)
     }
     if (tid == 0 && (a.n & 1)) {
         const int64_t i = a.n - 1;
-        dstd[i] = first ? a.r[i] : fma(beta, srcd[i], a.r[i]);
+        const double v = first ? a.r[i] : fma(beta, srcd[i], a.r[i]);
+        dstd[i] = v;
+        if (kPeer) put(i, v);
     }
     if (a.trace) {
         __syncthreads();
         trace_mark(a.trace, a.trace_max, K, 0, true);
     }
+    if (kPeer) fused_push_signal(a.t, pushed, a.n_push, ftag(ldg_o(&a.sc->epoch), (unsigned long long)K));
 }
 
 // end of a solve with the ring-deferred x update: the directions since the

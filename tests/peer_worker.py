@@ -8,12 +8,14 @@ flags and allreduce slots -- that NCCL cannot (it refuses two ranks on one
 GPU)."""
 
 
-def run(rank, nranks, dims, variant, max_iter, tol, to_parent, from_parent, halo=1):
+def run(rank, nranks, dims, variant, max_iter, tol, to_parent, from_parent, halo=1, defer=None):
     try:
         import numpy as np
         from paper_conf_sc_valero_laragmtv24_b200 import hpccg as H
         with H.Context(0, rank=rank, nranks=nranks, peer=True) as c, H.Problem(c, *dims) as p:
             p.set_option(H.HPCCG_OPT_CG_VARIANT, variant)
+            if defer is not None:  # before the export: a ring is exchanged with the blob
+                p.set_option(H.HPCCG_OPT_DEFER_X, defer)
             to_parent.put(("blob", rank, p.peer_export()))
             blobs = from_parent.get(timeout=120)
             p.peer_attach(blobs)
@@ -26,7 +28,7 @@ def run(rank, nranks, dims, variant, max_iter, tol, to_parent, from_parent, halo
                 r = p.solve(max_iter, tol)
                 out.append({"niters": r["niters"], "normr": r["normr"], "err": p.maxabsdiff(),
                             "x": p.get_vec(H.HPCCG_VEC_X), "mode": p.stats()["graph_mode"],
-                            "nnz_global": p.info["nnz_global"]})
+                            "nnz_global": p.info["nnz_global"], "x_deferred": p.stats()["x_deferred"]})
             to_parent.put(("done", rank, out))
     except Exception as e:  # reported to the parent, which fails the test
         to_parent.put(("error", rank, repr(e)))

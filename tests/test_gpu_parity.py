@@ -1112,20 +1112,32 @@ def test_defer_x_bitwise_identical(ctx, dims, max_iter, tol):
             assert np.max(np.abs(outs[-1][4] - oref["x"])) <= CG_ATOL
 
 
-@pytest.mark.parametrize("P", [2, 3])
-def test_defer_x_fused_loopback_bitwise(P):
-    """The same on z-slabs with the exchange fused into the kernels (HALO_PEER 2)."""
-    dims = (16, 12, 6)
+@pytest.mark.parametrize("P,dims,max_iter,tol", [(2, (16, 12, 6), 150, 1e-12), (3, (16, 12, 6), 150, 1e-12),
+                                                 (4, (10, 6, 1), 30, 0.0), (3, (10, 7, 5), 21, 0.0)])
+def test_defer_x_fused_loopback_bitwise(P, dims, max_iter, tol):
+    """The same on z-slabs with the exchange fused into the kernels (HALO_PEER
+    2), including the ring depths: the p update pushes p_K's boundary planes
+    into slot K % (m + 1) of the neighbours' rings (nz = 1: every row is a
+    boundary row; odd planes), in every launch mode."""
     with H.Context(0, nranks=P, loopback=True) as c, H.Problem(c, *dims) as p:
         p.set_option(H.HPCCG_OPT_HALO_PEER, 2)
         res = []
-        for defer in (0, 1):
+        for defer in (0, 1, 2, 5, 8):
             p.set_option(H.HPCCG_OPT_DEFER_X, defer)
-            p.set_vec(H.HPCCG_VEC_X, np.zeros(P * p.n))
-            r = p.solve(150, 1e-12)
-            res.append((r["niters"], r["normr"], p.get_vec(H.HPCCG_VEC_X)))
-        assert res[0][:2] == res[1][:2]
-        np.testing.assert_array_equal(res[0][2], res[1][2])
+            for mode in ("while", "graph", "timing"):
+                p.set_option(H.HPCCG_OPT_WHILE, 1 if mode == "while" else 0)
+                p.set_option(H.HPCCG_OPT_TIMING, 1 if mode == "timing" else 0)
+                p.set_vec(H.HPCCG_VEC_X, np.zeros(P * p.n))
+                r = p.solve(max_iter, tol)
+                assert p.stats()["x_deferred"] == defer, (defer, mode)
+                res.append((r["niters"], r["normr"], p.get_vec(H.HPCCG_VEC_X)))
+        p.set_option(H.HPCCG_OPT_TIMING, 0)
+        p.set_option(H.HPCCG_OPT_WHILE, 1)
+        for o in res[1:]:
+            assert o[:2] == res[0][:2]
+            np.testing.assert_array_equal(o[2], res[0][2])
+        if (max_iter, tol) != (150, 1e-12):
+            return
         ref = oracle.generate(dims[0], dims[1], dims[2] * P)
         oref = oracle.cg(ref, 150, 1e-12)
         assert abs(res[1][0] - oref["niters"]) <= 1
@@ -1299,7 +1311,7 @@ def test_scaling_configs_global_problem_loopback(P, nz, expect):
         assert abs(r["niters"] - expect) <= 1, r
         assert r["normr"] <= 1e-12
         assert p.maxabsdiff() < 1e-13
-        assert p.stats()["x_deferred"] == 1
+        assert p.stats()["x_deferred"] == 8  # auto: x deferred over a ring of 9 p buffers per slab
 
 
 # ------------- the CG SpMV from the chunk-sliced copy via TMA (SPMV_SLICED)

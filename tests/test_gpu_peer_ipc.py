@@ -17,13 +17,13 @@ torch = pytest.importorskip("torch")
 from paper_conf_sc_valero_laragmtv24_b200 import hpccg as H  # noqa: E402
 
 
-def run_ranks(nranks, dims, variant, max_iter, tol, timeout=240, halo=1):  # noqa: PLR0913
+def run_ranks(nranks, dims, variant, max_iter, tol, timeout=240, halo=1, defer=None):  # noqa: PLR0913
     import peer_worker
     ctx = mp.get_context("spawn")
     to_parent = ctx.Queue()
     inbox = [ctx.Queue() for _ in range(nranks)]
     procs = [ctx.Process(target=peer_worker.run,
-                         args=(r, nranks, dims, variant, max_iter, tol, to_parent, inbox[r], halo))
+                         args=(r, nranks, dims, variant, max_iter, tol, to_parent, inbox[r], halo, defer))
              for r in range(nranks)]
     for pr in procs:
         pr.start()
@@ -105,6 +105,29 @@ def test_processes_fused_peer_kernels(P, dims, max_iter, tol):
         np.testing.assert_array_equal(x, xl)
         assert abs(outs[0]["niters"] - oref["niters"]) <= 1
         assert np.max(np.abs(x - oref["x"])) <= 1e-10
+
+
+@pytest.mark.parametrize("P,dims,max_iter,tol,m", [(2, (16, 12, 6), 150, 1e-12, 8), (3, (8, 8, 4), 12, 0.0, 3),
+                                                   (2, (10, 6, 1), 40, 0.0, 5)])
+def test_processes_ring_deferred_x(P, dims, max_iter, tol, m):
+    """HALO_PEER = 2 across processes with x deferred over m iterations: each
+    rank's p ring is exported with its IPC blob, the p update pushes p_K's
+    boundary planes into slot K % (m + 1) of the neighbours' rings and the
+    SpMV gathers that slot -- bit for bit the same loop with x deferred by one
+    iteration (loopback), in both graph modes."""
+    res = run_ranks(P, dims, 0, max_iter, tol, halo=2, defer=m)
+    with H.Context(0, nranks=P, loopback=True) as c, H.Problem(c, *dims) as p:
+        p.set_option(H.HPCCG_OPT_HALO_PEER, 2)
+        p.set_option(H.HPCCG_OPT_DEFER_X, 1)
+        rl = p.solve(max_iter, tol)
+        xl = p.get_vec(H.HPCCG_VEC_X)
+    for k in range(2):
+        outs = [res[r][k] for r in range(P)]
+        x = np.concatenate([o["x"] for o in outs])
+        for o in outs:
+            assert o["x_deferred"] == m
+            assert (o["niters"], o["normr"]) == (rl["niters"], rl["normr"])
+        np.testing.assert_array_equal(x, xl)
 
 
 def test_processes_fused_peer_single_reduction():

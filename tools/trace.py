@@ -12,7 +12,8 @@ KEYS = {"graph": H.HPCCG_OPT_GRAPH, "timing": H.HPCCG_OPT_TIMING, "while": H.HPC
         "pdl": H.HPCCG_OPT_PDL, "waves": H.HPCCG_OPT_VEC_WAVES, "unroll": H.HPCCG_OPT_VEC_UNROLL,
         "rows": H.HPCCG_OPT_SPMV_ROWS, "l2": H.HPCCG_OPT_L2_PERSIST,
         "wu": H.HPCCG_OPT_WHILE_UNROLL, "ff": H.HPCCG_OPT_FINISHER_FREE,
-        "peer": H.HPCCG_OPT_HALO_PEER, "serp": H.HPCCG_OPT_SERPENTINE}
+        "peer": H.HPCCG_OPT_HALO_PEER, "serp": H.HPCCG_OPT_SERPENTINE,
+        "defer": H.HPCCG_OPT_DEFER_X}
 if os.environ.get("PROBE_NCCL"):  # 1-rank NCCL communicator: the multi-GPU code path
     ctx = H.Context(0, rank=0, nranks=1, unique_id=H.hpccg_unique_id())
 else:
