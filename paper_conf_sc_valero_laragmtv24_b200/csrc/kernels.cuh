@@ -504,12 +504,6 @@ __device__ __forceinline__ double2 fused_collect2_block(const PeerTab *t, int q,
 // interior / boundary split used to overlap the halo exchange).
 struct SpmvArgs {
     int64_t r0, len0, r1, len1;
-    // HPCCG_OPT_DEFER_X = m >= 2: p_k lives in ring slot k % ring_n (slot 0 =
-    // x, slot j > 0 = ring + (j - 1) ring_stride), k = sc->k read after the
-    // PDL wait; ring_n <= 1: x
-    const double *ring;
-    int64_t ring_stride;
-    int ring_n;
     int64_t nb0;            // blocks covering range 0
     int64_t r2, len2;       // a third range (HALO_PEER = 2: interior, plane 0, plane nz-1)
     int64_t nb01;           // blocks covering ranges 0 and 1
@@ -542,6 +536,14 @@ struct SpmvArgs {
     int nx;            // kDia (HPCCG_OPT_SPMV_FORMAT 1): row stride of the grid
     int dia;           // 1: spmv27x2_kernel<., ., false, true> (DIA-27, col[] not read)
     int trips;         // spmv27x2_trips_kernel: 512-row trips per block (one partial per block)
+    // HPCCG_OPT_DEFER_X = m >= 2: p_k lives in ring slot k % ring_n (slot 0 =
+    // x, slot j > 0 = ring + (j - 1) ring_stride), k = sc->k read after the
+    // PDL wait; ring_n <= 1: x.  (Kept last: inserted after r0..len1 the field
+    // offsets made ptxas spill 8 B in spmv27x2_kernel<1, true>, 95.2 -> 97.8 us
+    // at 128^3)
+    const double *ring;
+    int64_t ring_stride;
+    int ring_n;
 };
 
 // the row block this CTA handles (HPCCG_OPT_SERPENTINE)
