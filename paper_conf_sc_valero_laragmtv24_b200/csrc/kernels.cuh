@@ -111,6 +111,29 @@ __device__ __forceinline__ int2 ld_stream2(const int *ptr, uint64_t pol) {
     return v;
 }
 
+// L2 retention hints on the CG loop's vector stores (HPCCG_STORE_HINTS): bit 0
+// p (ring p update), bit 1 Ap (CG SpMV), bit 2 r (x/r update) stored with an L2
+// evict_last policy, so the next kernel's reads of them hit L2.  Default 5 (p
+// and r): measured at 256^3 (profiles/r2_store_hints_ab.log, one box, two
+// runs) period 929.3 / 929.8 -> 923.4 / 923.1 us (p alone 924.8, p + Ap 927,
+// all three 926: Ap kept in L2 costs the next SpMV more than the update gains);
+// 128^3 (vectors L2-resident) unchanged
+#ifndef HPCCG_STORE_HINTS
+#define HPCCG_STORE_HINTS 5
+#endif
+template <int kBit>
+__device__ __forceinline__ void st_hint(double2 *p, double2 v) {
+    if (HPCCG_STORE_HINTS & kBit) {
+        uint64_t pol;
+        asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
+        asm volatile("st.global.L2::cache_hint.v2.f64 [%0], {%1, %2}, %3;" ::"l"(p), "d"(v.x), "d"(v.y), "l"(pol)
+                     : "memory");
+    } else {
+        *p = v;
+    }
+}
+__device__ __forceinline__ void st_p(double2 *p, double2 v) { st_hint<1>(p, v); }
+
 // Loads of data the PREDECESSOR grid wrote (device scalars, reduction
 // partials), after pdl_wait().  ldg_o: the read-only path (one L2 request per
 // SM serves every warp; plain loads cost 1.6 % at 128^3).  The compiler may
@@ -815,7 +838,8 @@ __device__ __forceinline__ void spmv27x2_body(const SpmvArgs &a, int64_t row, in
                 s1 = fma(vv[t].y, xb, s1);
             }
         }
-        *reinterpret_cast<double2 *>(a.y + row) = make_double2(s0, s1);
+        if (kDots == 1) st_hint<2>(reinterpret_cast<double2 *>(a.y + row), make_double2(s0, s1));
+        else *reinterpret_cast<double2 *>(a.y + row) = make_double2(s0, s1);
         if (kDots > 0) {
             const double p0 = c0 == row + a.plane ? x0 : ld_gather<kCoh>(XG + row + a.plane);
             const double p1 = c1 == row + 1 + a.plane ? x1 : ld_gather<kCoh>(XG + row + 1 + a.plane);
@@ -1855,6 +1879,7 @@ __device__ __forceinline__ void ring_flush(const PringArgs &a, int K, double *sh
 
 // (__launch_bounds__(kBlock, 3): the flush path's loads must not push the
 // kernel past the 80 registers of cg_pupdate1_kernel<4>)
+
 template <int kU, bool kPeer = false>
 __global__ void __launch_bounds__(kBlock, 3) cg_pupdate_ring_kernel(PringArgs a) {
     __shared__ double sh[33];
@@ -1925,7 +1950,7 @@ __global__ void __launch_bounds__(kBlock, 3) cg_pupdate_ring_kernel(PringArgs a)
                     v.x = fma(beta, pa[u].x, ra[u].x);
                     v.y = fma(beta, pa[u].y, ra[u].y);
                 }
-                dst[i] = v;
+                st_p(dst + i, v);
                 if (kPeer && (2 * i < a.plane || 2 * i + 1 >= n - a.plane)) {
                     put(2 * i, v.x);
                     put(2 * i + 1, v.y);
@@ -2270,7 +2295,7 @@ __global__ void __launch_bounds__(kBlock) cg_update1_kernel(Upd1Args a) {
                 }
                 ra[u].x = fma(-alpha, qa[u].x, ra[u].x);
                 ra[u].y = fma(-alpha, qa[u].y, ra[u].y);
-                r2[i] = ra[u];
+                st_hint<4>(r2 + i, ra[u]);
                 acc = fma(ra[u].x, ra[u].x, acc);
                 acc2 = fma(ra[u].y, ra[u].y, acc2);
             }
