@@ -133,6 +133,19 @@ __device__ __forceinline__ void st_hint(double2 *p, double2 v) {
     }
 }
 __device__ __forceinline__ void st_p(double2 *p, double2 v) { st_hint<1>(p, v); }
+// loads with an L2 evict_first policy when bit kBit of HPCCG_STORE_HINTS is set
+// (bit 3: the ring p update's r and p_(K-1); bit 4: the x/r update's Ap)
+template <int kBit>
+__device__ __forceinline__ double2 ld_hint(const double2 *p) {
+    if (HPCCG_STORE_HINTS & kBit) {
+        uint64_t pol;
+        asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+        double2 v;
+        asm volatile("ld.global.L2::cache_hint.v2.f64 {%0, %1}, [%2], %3;" : "=d"(v.x), "=d"(v.y) : "l"(p), "l"(pol));
+        return v;
+    }
+    return *p;
+}
 
 // Loads of data the PREDECESSOR grid wrote (device scalars, reduction
 // partials), after pdl_wait().  ldg_o: the read-only path (one L2 request per
@@ -1907,14 +1920,14 @@ __global__ void __launch_bounds__(kBlock, 3) cg_pupdate_ring_kernel(PringArgs a)
 #pragma unroll
         for (int u = 0; u < kU; ++u) {
             const int64_t i = b + u * nth;
-            if (i < nv) pa[u] = src[i];
+            if (i < nv) pa[u] = ld_hint<8>(src + i);
         }
     };
     auto load_r = [&](int64_t b) {
 #pragma unroll
         for (int u = 0; u < kU; ++u) {
             const int64_t i = b + u * nth;
-            if (i < nv) ra[u] = r2[i];
+            if (i < nv) ra[u] = ld_hint<8>(r2 + i);
         }
     };
     if (!first) load_p(b0);
@@ -2241,7 +2254,7 @@ __global__ void __launch_bounds__(kBlock) cg_update1_kernel(Upd1Args a) {
 #pragma unroll
         for (int u = 0; u < kU; ++u) {
             const int64_t i = b + u * nth;
-            if (i < nv) qa[u] = q2[i];
+            if (i < nv) qa[u] = ld_hint<16>(q2 + i);
         }
     };
     auto load = [&](int64_t b) {
