@@ -133,17 +133,6 @@ __device__ __forceinline__ void st_hint(double2 *p, double2 v) {
     }
 }
 __device__ __forceinline__ void st_p(double2 *p, double2 v) { st_hint<1>(p, v); }
-// scalar form (the tridiagonal CG's kernels)
-template <int kBit>
-__device__ __forceinline__ void st_hint1(double *p, double v) {
-    if (HPCCG_STORE_HINTS & kBit) {
-        uint64_t pol;
-        asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
-        asm volatile("st.global.L2::cache_hint.f64 [%0], %1, %2;" ::"l"(p), "d"(v), "l"(pol) : "memory");
-    } else {
-        *p = v;
-    }
-}
 // loads with an L2 evict_first policy when bit kBit of HPCCG_STORE_HINTS is set
 // (bit 3: the ring p update's r and p_(K-1); bit 4: the x/r update's Ap)
 template <int kBit>

@@ -258,8 +258,7 @@ __global__ void __launch_bounds__(kBlock) tri_update_kernel(int64_t n, double *_
             const int64_t i = b0 + u * nth;
             if (i < n) {
                 const double rn = fma(nalpha, sv[u], rv[u]);
-                if (kDefer) st_hint1<4>(r + i, rn);  // variant 2: r is read by the p update right after
-                else r[i] = rn;
+                r[i] = rn;
                 if (!kDefer) x[i] = fma(alpha, pv[u], xv[u]);
                 acc = fma(rn, rn, acc);
             }
@@ -331,7 +330,7 @@ __global__ void __launch_bounds__(kBlock) tri_pupdate_ring_kernel(int64_t n, con
 #pragma unroll
             for (int u = 0; u < kTriU; ++u) {
                 const int64_t i = b0 + u * nth;
-                if (i < n) st_hint1<1>(dst + i, fma(beta, pv[u], rv[u]));  // gathered by the next matvec
+                if (i < n) dst[i] = fma(beta, pv[u], rv[u]);
             }
         }
         return;
