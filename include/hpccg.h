@@ -162,7 +162,9 @@ extern "C" {
                                (72 + 8/m) n B per iteration, the writes drop from 2 to 1 + 1/m
                                per row.  Bitwise the same results.  Device memory: m extra
                                p-sized buffers per slab (allocated when the option is set, or at
-                               generate time for auto).  -1 (default): auto -- 8 when the CG
+                               generate time for auto).  The single-reduction CG (CG_VARIANT 1)
+                               defers x over its own (not gathered) p vector the same way, any
+                               context.  -1 (default): auto -- 8 when the CG
                                vectors exceed L2, 0 below (at 128^3 the vectors are L2-resident
                                and 0 is 0.4 % faster) */
 #define HPCCG_OPT_FUSE_PSPMV 24 /* single slab, finisher-free loop: the p update and the

@@ -1069,16 +1069,39 @@ PRing ring_of(const Slab &s, int m, bool owned) {
     return g;
 }
 
+// f2 (single-reduction CG): x deferred over a ring of its p vector (s.r, not
+// gathered, so no SpMV or halo change) -- HPCCG_OPT_DEFER_X as for HPCCG's loop
+// (auto 8 beyond L2; 0 / 1: every iteration); the 2-rows/thread update only
+int sr_ring_m(const hpccg_problem *p) {
+    if (p->opt_variant != 1 || p->opt_defer_x == 0 || p->opt_defer_x == 1) return 0;
+    if (p->opt_defer_x < 0 && p->slabs[0].arena_bytes <= ((size_t)126 << 20)) return 0;
+    const int m = p->opt_defer_x < 0 ? kRingAutoM : p->opt_defer_x;
+    for (const Slab &s : p->slabs)
+        if (s.pring_slots < m || !aligned16(s.x) || !aligned16(s.p + s.plane) || !aligned16(s.r) ||
+            !aligned16(s.sv) || !aligned16(s.Ap))
+            return 0;
+    return m;
+}
+
 // end of a solve on the finisher-free loop with the deferred x update: the
 // last iteration's x += alpha p (cg_xfix_kernel; ring: the pending ones,
 // cg_xfix_ring_kernel), every slab
 int enqueue_xfix(hpccg_problem *p) {
-    if (!defer_x_on(p)) return HPCCG_OK;
     hpccg_ctx *ctx = p->ctx;
+    if (const int m = sr_ring_m(p); m >= 2) {  // f2: update k flushes up to k itself
+        for (const Slab &s : p->slabs) {
+            PRing g = ring_of(s, m, true);
+            launch_k(false, cg_xfix_ring_kernel, dim3(wave_grid(s.n / 2 + 1, wave(ctx, cg_xfix_ring_kernel))),
+                     ctx->stream, (int64_t)s.n, s.x, s.r, g, (const CgScalars *)s.sc, 0);
+            CHECK(check_launch(ctx));
+        }
+        return HPCCG_OK;
+    }
+    if (!defer_x_on(p)) return HPCCG_OK;
     if (const int m = defer_m(p); m >= 2) {
         for (const Slab &s : p->slabs) {
             launch_k(false, cg_xfix_ring_kernel, dim3(wave_grid(s.n / 2 + 1, wave(ctx, cg_xfix_ring_kernel))),
-                     ctx->stream, (int64_t)s.n, s.x, s.p + s.plane, ring_of(s, m, true), (const CgScalars *)s.sc);
+                     ctx->stream, (int64_t)s.n, s.x, s.p + s.plane, ring_of(s, m, true), (const CgScalars *)s.sc, 1);
             CHECK(check_launch(ctx));
         }
         return HPCCG_OK;
@@ -1501,6 +1524,7 @@ int launch_sr_update(hpccg_problem *p, const Slab &s, int q, unsigned long long 
     a.sc = s.sc;
     a.q = q;
     a.cond = cond;
+    if (const int m = sr_ring_m(p); m >= 2) a.ring = ring_of(s, m, true);
     if (ctx->mode == MODE_SINGLE) {
         const unsigned np = single_spmv_parts(p, s);
         if (np <= kUpdSumMax) {
@@ -1562,6 +1586,10 @@ int enqueue_iteration_sr_fused_u(hpccg_problem *p, bool timing, bool check, unsi
             if (cache.first != key)
                 cache = {key, push_blocks(s.n, s.plane, g, s.rank > 0, s.rank < ctx->nranks - 1)};
             a.n_push = cache.second;
+            if (const int m = sr_ring_m(p); m >= 2) {
+                a.ring = ring_of(s, m, true);
+                a.n_push1 = push_blocks(s.n, s.plane, g, s.rank > 0, s.rank < ctx->nranks - 1, 1);
+            }
             launch_k(pdl, upd, dim3(g), ctx->stream, a);
             CHECK(check_launch(ctx));
         }
@@ -1952,7 +1980,7 @@ int build_while_graph(hpccg_problem *p, int max_iter, double tol) {
     if (e != cudaSuccess) return bail(fail(HPCCG_ECUDA, "end capture (body): %s", cudaGetErrorString(e)));
     p->wgraph_init_kernels = l1 - l0;
     p->wgraph_body_kernels = (ctx->launches - l1) / U;
-    if (defer_x_on(p)) {  // after the WHILE node: the last iteration's deferred x update
+    if (defer_x_on(p) || sr_ring_m(p) >= 2) {  // after the WHILE node: the deferred x update's pending ones
         const int64_t l2 = ctx->launches;
         if (cudaStreamBeginCaptureToGraph(ctx->stream, g, &wnode, nullptr, 1,
                                           cudaStreamCaptureModeThreadLocal) != cudaSuccess)
@@ -3141,7 +3169,7 @@ int hpccg_solve(hpccg_problem *p, int max_iter, double tol, int *niters, double 
     st.kernel_launches = ctx->launches - l0;
     st.l2_persist_bytes = (int64_t)l2win.kept;
     st.graph_mode = use_persist ? p->last_persist_mode : (use_while ? 2 : (use_graph ? 1 : 0));
-    st.x_deferred = use_persist ? 0 : defer_m(p);
+    st.x_deferred = use_persist ? 0 : (p->opt_variant == 1 ? sr_ring_m(p) : defer_m(p));
     st.ps_fused = !use_persist && fuse_ps_on(p);
     p->stats = st;
     if (niters) *niters = hs.niters;

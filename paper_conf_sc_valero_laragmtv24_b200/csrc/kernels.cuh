@@ -1992,12 +1992,15 @@ __global__ void __launch_bounds__(kBlock, 3) cg_pupdate_ring_kernel(PringArgs a)
 // end of a solve with the ring-deferred x update: the directions since the
 // last flush, j = F + 1 .. N with F = m floor((N - 1) / m) and N = niters (p
 // update N flushed up to N - 1 only when m divides N - 1), in ascending order
+// shift: 1 for HPCCG's loop (p update K flushes up to K - 1), 0 for f2's
+// (update k flushes up to k itself)
 __global__ void __launch_bounds__(kBlock) cg_xfix_ring_kernel(int64_t n, double *x, double *p0, PRing g,
-                                                              const CgScalars *sc) {
+                                                              const CgScalars *sc, int shift) {
     pdl_wait();
     const int N = ldg_o(&sc->niters);
     if (N < 1) return;
-    const int m = g.m, R = m + 1, F = m * ((N - 1) / m), c = N - F;
+    const int m = g.m, R = m + 1, F = m * ((N - shift) / m), c = N - F;
+    if (c <= 0) return;
     const double *pj[kRingMaxM];
     double al[kRingMaxM];
 #pragma unroll
@@ -2395,6 +2398,10 @@ __global__ void cg_initstate_kernel(CgScalars *sc, int max_iter, double tol,
 struct SrUpdArgs {
     int64_t n;
     double *x, *r, *p, *s;     // r: owned part of the gathered (halo) vector
+    // x deferred over ring.m >= 2 iterations (HPCCG_OPT_DEFER_X): p_k in slot
+    // k % (m + 1) (slot 0 = p), x += alpha_j p_j for the last m directions in
+    // the update with k % m == 0 (the same FMAs in the same order); m < 2: none
+    PRing ring;
     const double *w;
     const double *parts;       // non-null: (gamma, delta) = fixed-order sums of
     unsigned n_parts;          //   parts[0, n_parts) and parts[n_parts, 2 n_parts)
@@ -2407,6 +2414,7 @@ struct SrUpdArgs {
     const PeerTab *t;
     int64_t plane;
     unsigned n_push;
+    unsigned n_push1;  // pushing blocks of the ring flush pass (one element per thread per trip)
     int post;
 };
 
@@ -2524,8 +2532,10 @@ __global__ void __launch_bounds__(kBlock) cg_sr_update_kernel(SrUpdArgs a) {
             const int64_t i = gtid() + u * gnth();
             if (i < nv0) {
                 asm volatile("prefetch.global.L2 [%0];" ::"l"(a.r + 2 * i));
-                asm volatile("prefetch.global.L2 [%0];" ::"l"(a.x + 2 * i));
-                asm volatile("prefetch.global.L2 [%0];" ::"l"(a.p + 2 * i));
+                if (a.ring.m < 2) {  // (with the ring: p's slot is known only after the wait, x unused)
+                    asm volatile("prefetch.global.L2 [%0];" ::"l"(a.x + 2 * i));
+                    asm volatile("prefetch.global.L2 [%0];" ::"l"(a.p + 2 * i));
+                }
                 asm volatile("prefetch.global.L2 [%0];" ::"l"(a.s + 2 * i));
             }
         }
@@ -2563,7 +2573,14 @@ __global__ void __launch_bounds__(kBlock) cg_sr_update_kernel(SrUpdArgs a) {
         first ? delta : __dsub_rn(delta, __ddiv_rn(__dmul_rn(beta, gamma), ldg_o(&sc->sr_alpha[qp])));
     const bool stop = (gamma == 0.0) || (den == 0.0);  // A11
     const double alpha = stop ? 0.0 : __ddiv_rn(gamma, den);
+    // the ring-deferred x update: this iteration's p source / destination slots
+    const int rm = a.ring.m, rR = rm + 1;
+    const bool ring = kVec && rm >= 2;
+    double *psrc = ring ? ring_slot(a.p, a.ring, (k - 1) % rR) : a.p;
+    double *pdst = ring ? ring_slot(a.p, a.ring, k % rR) : a.p;
+    const bool flush = ring && (k % rm == 0);
     if (blockIdx.x == 0 && threadIdx.x == 0) {
+        sc->alpha_h[k & 15] = alpha;
         const double normr = sqrt(gamma);  // ||r_(k-1)||: the lagged check (A4)
         const int nrun = !stop && (k + 1 < ldg_o(&sc->max_iter)) && normr > ldg_o(&sc->tol);
         sc->sr_gamma[q] = gamma;
@@ -2588,11 +2605,44 @@ __global__ void __launch_bounds__(kBlock) cg_sr_update_kernel(SrUpdArgs a) {
             pushed = 1;
         }
     };
-    if (kVec) {
+    if (flush) {
+        // x += alpha_j p_j, j = k - m + 1 .. k (p_k computed here): one element
+        // per thread per trip, the m - 1 older directions from their slots
+        __shared__ const double *sop[kRingMaxM - 1];
+        __shared__ double sal[kRingMaxM];
+        if (threadIdx.x < kRingMaxM) {
+            const int t = threadIdx.x, j = k - rm + 1 + t;
+            if (t < kRingMaxM - 1) sop[t] = t < rm - 1 ? ring_slot(a.p, a.ring, j % rR) : nullptr;
+            sal[t] = t < rm ? ldg_o(&sc->alpha_h[j & 15]) : 0.0;
+        }
+        __syncthreads();
+        const double ak = alpha;
+        for (int64_t i = tid; i < a.n; i += nth) {
+            double ov[kRingMaxM - 1];
+            const double rv = a.r[i], wv = a.w[i], pv0 = psrc[i], sv0 = a.s[i];
+            double xv = a.x[i];
+#pragma unroll
+            for (int t = 0; t < kRingMaxM - 1; ++t)
+                if (t < rm - 1) ov[t] = sop[t][i];
+            const double pv = first ? rv : fma(beta, pv0, rv);
+            const double sv = first ? wv : fma(beta, sv0, wv);
+#pragma unroll
+            for (int t = 0; t < kRingMaxM - 1; ++t)
+                if (t < rm - 1) xv = fma(sal[t], ov[t], xv);
+            pdst[i] = pv;
+            a.s[i] = sv;
+            a.x[i] = fma(ak, pv, xv);
+            const double rn = fma(-alpha, sv, rv);
+            a.r[i] = rn;
+            if (kPeer) put(i, rn);
+        }
+        if (kPeer) fused_push_signal(a.t, pushed, a.n_push1, ftag(ldg_o(&sc->epoch), (unsigned long long)k));
+    } else if (kVec) {
         const int64_t nv = a.n >> 1;
         double2 *__restrict__ x2 = reinterpret_cast<double2 *>(a.x);
         double2 *__restrict__ r2 = reinterpret_cast<double2 *>(a.r);
-        double2 *__restrict__ p2 = reinterpret_cast<double2 *>(a.p);
+        const double2 *ps2 = reinterpret_cast<const double2 *>(psrc);  // (slot (k - 1) % R with the ring)
+        double2 *pd2 = reinterpret_cast<double2 *>(pdst);
         double2 *__restrict__ s2 = reinterpret_cast<double2 *>(a.s);
         const double2 *__restrict__ w2 = reinterpret_cast<const double2 *>(a.w);
         for (int64_t b = tid; b < nv; b += kU * nth) {
@@ -2604,10 +2654,10 @@ __global__ void __launch_bounds__(kBlock) cg_sr_update_kernel(SrUpdArgs a) {
                     ra[u] = r2[i];
                     wa[u] = w2[i];
                     if (!first) {
-                        pa[u] = p2[i];
+                        pa[u] = ps2[i];
                         sa[u] = s2[i];
                     }
-                    xa[u] = x2[i];
+                    if (!ring) xa[u] = x2[i];
                 }
             }
 #pragma unroll
@@ -2621,9 +2671,9 @@ __global__ void __launch_bounds__(kBlock) cg_sr_update_kernel(SrUpdArgs a) {
                         sv.x = fma(beta, sa[u].x, wa[u].x);
                         sv.y = fma(beta, sa[u].y, wa[u].y);
                     }
-                    p2[i] = pv;
+                    pd2[i] = pv;
                     s2[i] = sv;
-                    x2[i] = make_double2(fma(alpha, pv.x, xa[u].x), fma(alpha, pv.y, xa[u].y));
+                    if (!ring) x2[i] = make_double2(fma(alpha, pv.x, xa[u].x), fma(alpha, pv.y, xa[u].y));
                     const double2 rn = make_double2(fma(-alpha, sv.x, ra[u].x), fma(-alpha, sv.y, ra[u].y));
                     r2[i] = rn;
                     if (kPeer && (2 * i < a.plane || 2 * i + 1 >= a.n - a.plane)) {
@@ -2635,11 +2685,11 @@ __global__ void __launch_bounds__(kBlock) cg_sr_update_kernel(SrUpdArgs a) {
         }
         if (tid == 0 && (a.n & 1)) {
             const int64_t i = a.n - 1;
-            const double pv = first ? a.r[i] : fma(beta, a.p[i], a.r[i]);
+            const double pv = first ? a.r[i] : fma(beta, psrc[i], a.r[i]);
             const double sv = first ? a.w[i] : fma(beta, a.s[i], a.w[i]);
-            a.p[i] = pv;
+            pdst[i] = pv;
             a.s[i] = sv;
-            a.x[i] = fma(alpha, pv, a.x[i]);
+            if (!ring) a.x[i] = fma(alpha, pv, a.x[i]);
             a.r[i] = fma(-alpha, sv, a.r[i]);
             if (kPeer) put(i, a.r[i]);
         }

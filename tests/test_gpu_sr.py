@@ -202,3 +202,55 @@ def test_sr_full_128cubed(ctx, rows):
         r500 = p.solve(501, 0.0)
         assert r500["niters"] == 500
         assert p.maxabsdiff() < 1e-13 and 0 <= r500["normr"] < 1e-40
+
+
+@pytest.mark.parametrize("dims,max_iter,tol", [((20, 30, 10), 150, 1e-12), ((31, 17, 9), 40, 0.0),
+                                               ((64, 48, 40), 18, 0.0), ((64, 48, 40), 17, 0.0),
+                                               ((33, 9, 3), 7, 0.0), ((16, 16, 16), 150, 1e-12)])
+def test_sr_ring_deferred_x_bitwise(ctx, dims, max_iter, tol):
+    """f2 with x deferred over m iterations (HPCCG_OPT_DEFER_X = m): p_k goes
+    to ring slot k % (m + 1), the update with k % m == 0 also applies x =
+    fma(alpha_j, p_j, x) for the last m directions (p_k from registers), and
+    cg_xfix_ring_kernel the pending ones after the loop -- the FMAs of the
+    undeferred update in the same order, so niters, normr and x are bit for
+    bit equal, in every launch mode; iteration counts ending 0..m-1 after a
+    flush; odd n."""
+    with H.Problem(ctx, *dims) as p:
+        sr(p)
+        p.set_option(H.HPCCG_OPT_PERSISTENT, 0)
+        outs = []
+        for defer in (0, 2, 3, 8):
+            p.set_option(H.HPCCG_OPT_DEFER_X, defer)
+            for mode in ("while", "graph", "timing"):
+                p.set_option(H.HPCCG_OPT_WHILE, 1 if mode == "while" else 0)
+                p.set_option(H.HPCCG_OPT_TIMING, 1 if mode == "timing" else 0)
+                p.set_vec(H.HPCCG_VEC_X, np.zeros(p.n))
+                r = p.solve(max_iter, tol)
+                assert p.stats()["x_deferred"] == (defer if defer >= 2 else 0), (defer, mode)
+                outs.append((r["niters"], r["normr"], p.get_vec(H.HPCCG_VEC_X)))
+        for k, v in ((H.HPCCG_OPT_TIMING, 0), (H.HPCCG_OPT_WHILE, 1), (H.HPCCG_OPT_DEFER_X, -1),
+                     (H.HPCCG_OPT_CG_VARIANT, 0)):
+            p.set_option(k, v)
+        for o in outs[1:]:
+            assert o[:2] == outs[0][:2]
+            np.testing.assert_array_equal(o[2], outs[0][2])
+
+
+@pytest.mark.parametrize("P,dims", [(2, (16, 12, 6)), (3, (10, 6, 1))])
+def test_sr_ring_fused_loopback_bitwise(P, dims):
+    """The same on loopback z-slabs with f2's exchange fused into its kernels
+    (HALO_PEER 2; the flush pass pushes r's boundary planes with its own
+    pushing-block count; nz = 1: every row is a boundary row)."""
+    with H.Context(0, nranks=P, loopback=True) as c, H.Problem(c, *dims) as p:
+        sr(p)
+        p.set_option(H.HPCCG_OPT_HALO_PEER, 2)
+        outs = []
+        for defer in (0, 3, 8):
+            p.set_option(H.HPCCG_OPT_DEFER_X, defer)
+            p.set_vec(H.HPCCG_VEC_X, np.zeros(P * p.n))
+            r = p.solve(40, 0.0)
+            assert p.stats()["x_deferred"] == (defer if defer >= 2 else 0)
+            outs.append((r["niters"], r["normr"], p.get_vec(H.HPCCG_VEC_X)))
+        for o in outs[1:]:
+            assert o[:2] == outs[0][:2]
+            np.testing.assert_array_equal(o[2], outs[0][2])
