@@ -197,8 +197,9 @@ extern "C" {
 #define HPCCG_OPT_SMEM_HALO 30 /* the on-chip (shared-memory cluster) solve: every CTA keeps the
                                gathered vector (p; r for the single-reduction CG) with the
                                stencil's reach (plane + nx + 1 rows) of halo on each side in its
-                               own shared memory, refreshed once per SpMV by coalesced reads of
-                               the owner CTAs' rows, so the 27 gathers of a row are local
+                               own shared memory (every writer of an own row also stores it into
+                               the windows of the CTAs that hold it, published by the cluster
+                               barrier that follows), so the 27 gathers of a row are local
                                instead of distributed-shared-memory reads.  The same values in
                                the same order: bitwise the unhalo'd solve.  -1 (default) auto /
                                1: when the halo (16 (plane + nx + 1) B per CTA) fits next to the

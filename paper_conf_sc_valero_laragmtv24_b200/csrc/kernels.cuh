@@ -3047,30 +3047,29 @@ __global__ void __launch_bounds__(NT, 1) cg_smem_cluster_kernel(SmemArgs a) {
         for (int k = 0; k < kSlots; ++k) s = fma(sval[k * R + i], pv[k], s);
         return s;
     };
-    // after a cluster barrier that completed every CTA's rows of g: copy the
-    // rows [row0 - Hh, row0) and [row0 + R, row0 + R + Hh) from their owners
-    // (consecutive threads read consecutive rows of one owner), then make them
-    // visible to this CTA.  The owners write those rows again only after the
-    // next cluster barrier.
-    auto fill_halo = [&](double *g) {
+    // kHalo: a new value v of own row i of the gathered vector g is also stored
+    // into the halo copy of every other CTA whose window [c R - Hh, c R + R + Hh)
+    // holds that row (distributed shared memory stores, no round trip); the
+    // cluster barrier that follows makes them visible before any gather.  The
+    // receivers read those copies only between that barrier and the next one.
+    const int nct = (int)cl.num_blocks();
+    auto put = [&](double *g, int i, double v) {
+        g[i] = v;
         if (!kHalo) return;
-        for (int j = threadIdx.x; j < 2 * Hh; j += NT) {
-            const int lo = j < Hh;
-            const int64_t gr = lo ? row0 - Hh + j : row0 + R + (j - Hh);
-            if (gr < 0 || gr >= a.n) continue;  // outside the matrix: never a column
-            const unsigned owner = (unsigned)(gr / R);
-            const int off = (int)(gr - (int64_t)owner * R);
-            g[lo ? j - Hh : R + (j - Hh)] = *cl.map_shared_rank(g + off, owner);
+        const int64_t gr = row0 + i;
+        const int c_hi = min(nct - 1, (int)((gr + Hh) / R));
+        for (int c = max(0, (int)((gr - Hh - R) / R)); c <= c_hi; ++c) {
+            const int64_t off = gr - (int64_t)c * R;  // the row in CTA c's window
+            if (c == (int)me || off < -Hh || off >= R + Hh) continue;
+            *cl.map_shared_rank(g + off, (unsigned)c) = v;
         }
-        __syncthreads();
     };
     int niters = 0;
     double normr, rr_out, rr_prev_out;
     if (!kSR) {
         // ---- init (a.7): p = x; Ap = A p; r = b - Ap; rtrans = r.r
-        for (int i = threadIdx.x; i < nr; i += NT) sp[i] = sx[i];
+        for (int i = threadIdx.x; i < nr; i += NT) put(sp, i, sx[i]);
         cl.sync();
-        fill_halo(sp);
         double acc = 0.0;
         for (int i = threadIdx.x; i < nr; i += NT) {
             const double rv = fma(-1.0, spmv_row(sp, i), sb[i]);
@@ -3088,10 +3087,9 @@ __global__ void __launch_bounds__(NT, 1) cg_smem_cluster_kernel(SmemArgs a) {
                 beta = rtrans / old;
             }
             // every CTA has finished reading the previous p (cluster_sum2's barrier)
-            for (int i = threadIdx.x; i < nr; i += NT) sp[i] = (k == 1) ? sr[i] : fma(beta, sp[i], sr[i]);
+            for (int i = threadIdx.x; i < nr; i += NT) put(sp, i, (k == 1) ? sr[i] : fma(beta, sp[i], sr[i]));
             normr = sqrt(rtrans);
             cl.sync();
-            fill_halo(sp);
             double d = 0.0;
             for (int i = threadIdx.x; i < nr; i += NT) {
                 const double ap = spmv_row(sp, i);
@@ -3116,14 +3114,12 @@ __global__ void __launch_bounds__(NT, 1) cg_smem_cluster_kernel(SmemArgs a) {
         rr_prev_out = rtrans;
     } else {
         // ---- init: r = b - A x0 (x0 gathered from sr), w = A r, (gamma, delta)
-        for (int i = threadIdx.x; i < nr; i += NT) sr[i] = sx[i];
+        for (int i = threadIdx.x; i < nr; i += NT) put(sr, i, sx[i]);
         cl.sync();
-        fill_halo(sr);
         for (int i = threadIdx.x; i < nr; i += NT) sq[i] = fma(-1.0, spmv_row(sr, i), sb[i]);
         cl.sync();  // every CTA has finished gathering x0 from sr
-        for (int i = threadIdx.x; i < nr; i += NT) sr[i] = sq[i];
+        for (int i = threadIdx.x; i < nr; i += NT) put(sr, i, sq[i]);
         cl.sync();
-        fill_halo(sr);
         double g = 0.0, dl = 0.0;
         for (int i = threadIdx.x; i < nr; i += NT) {
             const double w = spmv_row(sr, i);
@@ -3148,13 +3144,12 @@ __global__ void __launch_bounds__(NT, 1) cg_smem_cluster_kernel(SmemArgs a) {
                 sp[i] = pv;
                 ss[i] = sv;
                 sx[i] = fma(alpha, pv, sx[i]);
-                sr[i] = fma(-alpha, sv, sr[i]);
+                put(sr, i, fma(-alpha, sv, sr[i]));
             }
             niters = k;
             // the next iteration would not run (A4, A11): skip its SpMV
             if (stop || !(k + 1 < a.max_iter && normr > a.tol)) break;
             cl.sync();
-            fill_halo(sr);
             g = 0.0;
             dl = 0.0;
             for (int i = threadIdx.x; i < nr; i += NT) {
