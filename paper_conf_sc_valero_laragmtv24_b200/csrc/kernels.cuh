@@ -1899,7 +1899,11 @@ __global__ void __launch_bounds__(kBlock, 3) cg_pupdate_ring_kernel(PringArgs a)
     // this iteration's index from the p update before it (ring_k[q ^ 1],
     // written by p update K - 1, which completed before this grid's PDL
     // predecessor began): the slots are known before the wait
-    const int K = ldp(&a.sc->ring_k[a.q ^ 1]) + 1;
+    // (ld.relaxed.gpu: a coherent read at GPU scope, never a stale L1 line -- it
+    // precedes the wait, so the PDL visibility guarantee does not cover it)
+    int kprev;
+    asm volatile("ld.relaxed.gpu.global.s32 %0, [%1];" : "=r"(kprev) : "l"(&a.sc->ring_k[a.q ^ 1]) : "memory");
+    const int K = kprev + 1;
     const int m = a.ring.m, R = m + 1;
     const bool first = (K == 1);
     if (!first && (K - 1) % m == 0) {
