@@ -1049,6 +1049,10 @@ int ring_alloc(hpccg_problem *p, int m) {
     if (m < 2) return HPCCG_OK;
     for (Slab &s : p->slabs) {
         if (s.pring_slots >= m) continue;
+        // the neighbours of a one-slab-per-process context mapped the old ring at the
+        // peer exchange: stop addressing rings (z-slabs run m = 1) rather than push
+        // into freed memory; loopback tables are rebuilt by the caller
+        if (s.ptab && one_slab_per_process(p->ctx)) p->peer_ring = false;
         cudaFree(s.pring_alloc);
         s.pring_alloc = s.pring = nullptr;
         s.pring_slots = 0;

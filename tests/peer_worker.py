@@ -8,7 +8,8 @@ flags and allreduce slots -- that NCCL cannot (it refuses two ranks on one
 GPU)."""
 
 
-def run(rank, nranks, dims, variant, max_iter, tol, to_parent, from_parent, halo=1, defer=None):
+def run(rank, nranks, dims, variant, max_iter, tol, to_parent, from_parent, halo=1, defer=None,
+        defer_after=None):
     try:
         import numpy as np
         from paper_conf_sc_valero_laragmtv24_b200 import hpccg as H
@@ -21,6 +22,8 @@ def run(rank, nranks, dims, variant, max_iter, tol, to_parent, from_parent, halo
             p.peer_attach(blobs)
             if halo != 1:  # 2: exchange + allreduces fused into the CG kernels
                 p.set_option(H.HPCCG_OPT_HALO_PEER, halo)
+            if defer_after is not None:  # a ring allocated after the exchange: not addressed
+                p.set_option(H.HPCCG_OPT_DEFER_X, defer_after)
             out = []
             for wh in (1, 0):
                 p.set_option(H.HPCCG_OPT_WHILE, wh)

@@ -17,13 +17,15 @@ torch = pytest.importorskip("torch")
 from paper_conf_sc_valero_laragmtv24_b200 import hpccg as H  # noqa: E402
 
 
-def run_ranks(nranks, dims, variant, max_iter, tol, timeout=240, halo=1, defer=None):  # noqa: PLR0913
+def run_ranks(nranks, dims, variant, max_iter, tol, timeout=240, halo=1, defer=None,  # noqa: PLR0913
+              defer_after=None):
     import peer_worker
     ctx = mp.get_context("spawn")
     to_parent = ctx.Queue()
     inbox = [ctx.Queue() for _ in range(nranks)]
     procs = [ctx.Process(target=peer_worker.run,
-                         args=(r, nranks, dims, variant, max_iter, tol, to_parent, inbox[r], halo, defer))
+                         args=(r, nranks, dims, variant, max_iter, tol, to_parent, inbox[r], halo, defer,
+                               defer_after))
              for r in range(nranks)]
     for pr in procs:
         pr.start()
@@ -128,6 +130,25 @@ def test_processes_ring_deferred_x(P, dims, max_iter, tol, m):
             assert o["x_deferred"] == m
             assert (o["niters"], o["normr"]) == (rl["niters"], rl["normr"])
         np.testing.assert_array_equal(x, xl)
+
+
+def test_processes_ring_requested_after_exchange_falls_back():
+    """A ring depth set only after the peer exchange (the neighbours mapped no
+    ring): the z-slab loop falls back to x deferred by one iteration (m = 1)
+    instead of pushing into unmapped rings -- same bits as loopback m = 1."""
+    P, dims = 2, (16, 12, 6)
+    res = run_ranks(P, dims, 0, 40, 0.0, halo=2, defer_after=5)
+    with H.Context(0, nranks=P, loopback=True) as c, H.Problem(c, *dims) as p:
+        p.set_option(H.HPCCG_OPT_HALO_PEER, 2)
+        p.set_option(H.HPCCG_OPT_DEFER_X, 1)
+        rl = p.solve(40, 0.0)
+        xl = p.get_vec(H.HPCCG_VEC_X)
+    for k in range(2):
+        outs = [res[r][k] for r in range(P)]
+        for o in outs:
+            assert o["x_deferred"] == 1
+            assert (o["niters"], o["normr"]) == (rl["niters"], rl["normr"])
+        np.testing.assert_array_equal(np.concatenate([o["x"] for o in outs]), xl)
 
 
 def test_processes_fused_peer_single_reduction():
