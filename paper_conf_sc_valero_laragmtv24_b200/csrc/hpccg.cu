@@ -2664,10 +2664,16 @@ int hpccg_generate(hpccg_ctx *ctx, int nx, int ny, int nz, hpccg_problem **out) 
         if (rc) return bail(rc);
     }
     // the p rings of the deferred x update (auto: CG vectors beyond L2), before any
-    // peer exchange so the neighbours can address them
-    if (p->slabs[0].arena_bytes > ((size_t)126 << 20)) {
-        const int rc = ring_alloc(p, kRingAutoM);
-        if (rc) return bail(rc);
+    // peer exchange so the neighbours can address them.  Best effort: a problem that
+    // fits without its ring still runs (x deferred by one iteration) when the m more
+    // p-sized buffers do not fit
+    if (p->slabs[0].arena_bytes > ((size_t)126 << 20) && ring_alloc(p, kRingAutoM) != HPCCG_OK) {
+        for (Slab &s : p->slabs) {
+            cudaFree(s.pring_alloc);
+            s.pring_alloc = s.pring = nullptr;
+            s.pring_slots = 0;
+        }
+        cudaGetLastError();
     }
     *out = p;
     return HPCCG_OK;
