@@ -1040,7 +1040,7 @@ int defer_m(const hpccg_problem *p) {
         if (s.pring_slots < want || s.dia) return 1;
     if (p->ctx->mode != MODE_SINGLE)  // z-slabs: the peer tables must address the neighbours' rings
         return p->peer_ring ? want : 1;
-    if (fuse_ps_on(const_cast<hpccg_problem *>(p)) || sliced_on(p) || spmv_trips(p) > 1) return 1;
+    if (fuse_ps_on(const_cast<hpccg_problem *>(p)) || spmv_trips(p) > 1) return 1;
     return want;
 }
 

@@ -1086,6 +1086,7 @@ __global__ void __launch_bounds__(kSlR, 2) spmv_sliced_kernel(SpmvArgs a, const 
         for (int s = 0; s < kSlStages && s < mine; ++s) sl_wait(&full[s], 0);
         return;
     }
+    const double *xg = spmv_xg<true>(a);  // p's ring slot (ring-deferred x update) or a.x
     double d = 0.0;
     for (int64_t i = 0; i < mine; ++i) {
         const int s = (int)(i % kSlStages);
@@ -1101,7 +1102,7 @@ __global__ void __launch_bounds__(kSlR, 2) spmv_sliced_kernel(SpmvArgs a, const 
         for (int k = 0; k < kSlots; ++k) {  // all 27 gathers in flight
             const int cc = sc[k * kSlR + j];
             if (k == kDiagSlot) cd = cc;
-            xv[k] = __ldg(a.x + cc);
+            xv[k] = __ldg(xg + cc);
         }
         double s0 = 0.0;  // FMA chain in ascending column from +0.0 (A8)
 #pragma unroll
@@ -1111,7 +1112,7 @@ __global__ void __launch_bounds__(kSlR, 2) spmv_sliced_kernel(SpmvArgs a, const 
             sl_issue(sl + (size_t)chunk(i + kSlStages) * kSlBytes, ring + (size_t)s * kSlBytes, &full[s]);
         if (row < n) {
             a.y[row] = s0;
-            const double p0 = cd == row + a.plane ? xv[kDiagSlot] : __ldg(a.x + row + a.plane);
+            const double p0 = cd == row + a.plane ? xv[kDiagSlot] : __ldg(xg + row + a.plane);
             d = fma(s0, p0, d);
         }
     }

@@ -1360,6 +1360,32 @@ def test_sliced_spmv_first_step_exact(ctx, dims):
         p.set_option(H.HPCCG_OPT_SPMV_SLICED, 0)
 
 
+@pytest.mark.parametrize("dims,max_iter,tol", [((24, 20, 12), 150, 1e-12), ((64, 48, 40), 19, 0.0)])
+def test_sliced_spmv_with_ring_bitwise(ctx, dims, max_iter, tol):
+    """The sliced SpMV gathers p from its ring slot when x is deferred over m
+    iterations: bit for bit the sliced loop with x deferred by one iteration,
+    in every launch mode."""
+    with H.Problem(ctx, *dims) as p:
+        p.set_option(H.HPCCG_OPT_PERSISTENT, 0)
+        p.set_option(H.HPCCG_OPT_SPMV_SLICED, 1)
+        outs = []
+        for defer in (1, 3, 8):
+            p.set_option(H.HPCCG_OPT_DEFER_X, defer)
+            for wh, tm in ((1, 0), (0, 0), (0, 1)):
+                p.set_option(H.HPCCG_OPT_WHILE, wh)
+                p.set_option(H.HPCCG_OPT_TIMING, tm)
+                p.set_vec(H.HPCCG_VEC_X, np.zeros(p.n))
+                r = p.solve(max_iter, tol)
+                assert p.stats()["x_deferred"] == defer
+                outs.append((r["niters"], r["normr"], p.get_vec(H.HPCCG_VEC_X)))
+        for k, v in ((H.HPCCG_OPT_TIMING, 0), (H.HPCCG_OPT_WHILE, 1), (H.HPCCG_OPT_DEFER_X, -1),
+                     (H.HPCCG_OPT_SPMV_SLICED, 0)):
+            p.set_option(k, v)
+        for o in outs[1:]:
+            assert o[:2] == outs[0][:2]
+            np.testing.assert_array_equal(o[2], outs[0][2])
+
+
 @pytest.mark.parametrize("dims,max_iter,tol", [((24, 20, 12), 150, 1e-12), ((64, 64, 64), 150, 1e-12),
                                                ((33, 9, 3), 40, 0.0), ((128, 128, 130), 25, 0.0)])
 def test_sliced_spmv_cg_modes_and_oracle(ctx, dims, max_iter, tol):
