@@ -157,7 +157,8 @@ extern "C" {
                                the neighbours' rings: a ring is exchanged only if it exists when the
                                peer tables are built (auto: allocated at generate; explicit m on
                                one-slab-per-process contexts: set it before HALO_PEER / the peer
-                               export), else z-slabs run m = 1.  Per m iterations x
+                               export), else z-slabs run m = 1; every rank must use the same value
+                               (the neighbours' slots are addressed by k % (m + 1)).  Per m iterations x
                                is read and written once and m - 1 old p's re-read: 12 nnz +
                                (72 + 8/m) n B per iteration, the writes drop from 2 to 1 + 1/m
                                per row.  Bitwise the same results.  Device memory: m extra
