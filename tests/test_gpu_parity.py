@@ -1100,7 +1100,9 @@ def test_peer_mode_nccl_one_rank():
 @pytest.mark.parametrize("dims,max_iter,tol", [((20, 30, 10), 150, 1e-12), ((31, 17, 9), 40, 0.0),
                                                ((64, 64, 64), 150, 1e-12), ((33, 9, 3), 7, 0.0),
                                                ((21, 13, 7), 150, 1e-12), ((128, 128, 128), 21, 0.0),
-                                               ((64, 48, 40), 10, 0.0), ((64, 48, 40), 18, 0.0)])
+                                               ((64, 48, 40), 10, 0.0), ((64, 48, 40), 18, 0.0),
+                                               ((16, 12, 10), 1, 0.0), ((16, 12, 10), 2, 0.0),
+                                               ((16, 12, 10), 3, 0.0)])
 def test_defer_x_bitwise_identical(ctx, dims, max_iter, tol):
     """HPCCG_OPT_DEFER_X (x += alpha p moved into the next p update, the last
     one into cg_xfix_kernel): the same FMA on the same operands, so x, niters
