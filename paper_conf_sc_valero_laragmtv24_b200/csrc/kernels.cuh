@@ -2968,9 +2968,9 @@ __device__ __forceinline__ double2 cluster_sum2(double *mine, double u, double v
         }
     }
     __syncthreads();
-    const double2 r = make_double2(sh[64], sh[65]);
-    __syncthreads();
-    return r;
+    // (no trailing barrier: sh[64..65] is written again only by warp 0 of the next
+    // call after that call's block barrier, which every reader has passed)
+    return make_double2(sh[64], sh[65]);
 }
 
 // ----------------------------------- on-chip solve (tiny single-GPU problems)
